@@ -1,0 +1,204 @@
+"""CPU oracle for the Proteus hot path -- TEST INFRASTRUCTURE ONLY.
+
+Only tests/, ``__graft_entry__.smoke()`` and bench.py's ``cpu_baseline`` /
+``--impl reference`` legs may import this package.  The product package
+(paper_conf_asplos_ahmadgfwsw24_b200) never imports it, and it shares no code
+with the CUDA path: the arithmetic lives in ``oracle.c`` (plain C, exhaustive
+enumeration, exact vertex-enumeration LP, event-driven simulator) and
+``lp_exact.py`` (the literal Eqs. 2-6 LP in exact rationals).
+
+Every function cites the passage of PAPER.md it follows; see oracle.c.
+"""
+
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_DIR = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_DIR, "oracle.c")
+_LIB = os.path.join(_DIR, "liboracle.so")
+_lib = None
+
+i32p = np.ctypeslib.ndpointer(dtype=np.int32, flags="C_CONTIGUOUS")
+i64p = np.ctypeslib.ndpointer(dtype=np.int64, flags="C_CONTIGUOUS")
+u32p = np.ctypeslib.ndpointer(dtype=np.uint32, flags="C_CONTIGUOUS")
+u64p = np.ctypeslib.ndpointer(dtype=np.uint64, flags="C_CONTIGUOUS")
+u8p = np.ctypeslib.ndpointer(dtype=np.uint8, flags="C_CONTIGUOUS")
+
+
+def build(force: bool = False) -> str:
+    """Compile oracle.c with gcc (building the checker is not using it)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-std=gnu11", "-pthread", "-shared", "-fPIC",
+                               "-o", _LIB + ".tmp", _SRC])
+        os.replace(_LIB + ".tmp", _LIB)
+    return _LIB
+
+
+class Problem(C.Structure):
+    _fields_ = [("T", C.c_int32), ("Q", C.c_int32), ("M", C.c_int32), ("D", C.c_int32),
+                ("V", C.c_void_p), ("acc", C.c_void_p), ("P", C.c_void_p),
+                ("dev_type", C.c_void_p), ("s", C.c_void_p)]
+
+
+class Result(C.Structure):
+    _fields_ = [("served", C.c_int64), ("accsum", C.c_int64), ("unmet", C.c_int64),
+                ("index", C.c_uint64), ("n_candidates", C.c_uint64),
+                ("eff", C.c_int32), ("pad", C.c_int32)]
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = C.CDLL(_LIB)
+        L.orc_capacity.argtypes = [C.c_int, C.c_int, C.c_int, i32p, i32p, i32p, i32p, i32p]
+        L.orc_family_lp.argtypes = [C.c_int, i64p, i64p, i32p, C.c_int64,
+                                    C.POINTER(C.c_int64), C.POINTER(C.c_int64)]
+        L.orc_score_placement.argtypes = [C.POINTER(Problem), i32p, C.POINTER(Result), i32p]
+        L.orc_enum_count.argtypes = [C.POINTER(Problem), C.c_int, C.POINTER(C.c_uint64)]
+        L.orc_solve_enum.argtypes = [C.POINTER(Problem), C.c_int, C.c_int, C.POINTER(Result), i32p, i32p]
+        L.orc_solve_factored.argtypes = [C.POINTER(Problem), C.c_int, C.c_int, C.POINTER(Result),
+                                         i32p, i32p, i32p]
+        L.orc_route_swrr.argtypes = [C.c_int64, u8p, C.c_int, C.c_int, i32p, i32p, i32p, i32p]
+        L.orc_replay_device.argtypes = [C.c_int64, u32p, i32p, C.c_int, C.c_int64, u32p]
+        L.orc_replay.argtypes = [C.c_int64, u32p, u8p, C.c_int, C.c_int, i32p, i32p, C.c_int, i32p,
+                                 C.c_int, i32p, i32p, i32p, i32p, i32p, C.c_int, i32p, C.c_int,
+                                 C.c_void_p, u64p, u64p, u64p]
+        _lib = L
+    return _lib
+
+
+def _i32(x):
+    return np.ascontiguousarray(np.asarray(x, dtype=np.int32))
+
+
+def family_of_variant(V) -> np.ndarray:
+    return np.repeat(np.arange(len(V), dtype=np.int32), np.asarray(V))
+
+
+def capacity(prof, slo_us):
+    """a1: P[t][m], b*[t][m], depth[t][m]."""
+    M = int(np.sum(prof.V))
+    slo_m = _i32(np.asarray(slo_us)[family_of_variant(prof.V)])
+    P = np.zeros((prof.T, M), np.int32)
+    bs = np.zeros_like(P)
+    dep = np.zeros_like(P)
+    lib().orc_capacity(prof.T, M, prof.bmax, _i32(prof.lat_us), slo_m, P, bs, dep)
+    return P, bs, dep
+
+
+class _Prob:
+    """Keeps the numpy buffers a Problem points at alive."""
+
+    def __init__(self, prof, device_type, slo_us, demand, P=None):
+        self.V = _i32(prof.V)
+        self.acc = _i32(prof.acc_micro)
+        self.P = _i32(capacity(prof, slo_us)[0] if P is None else P)
+        self.dev = _i32(device_type)
+        self.s = _i32(demand)
+        self.st = Problem(prof.T, len(self.V), int(self.V.sum()), len(self.dev),
+                          self.V.ctypes.data, self.acc.ctypes.data, self.P.ctypes.data,
+                          self.dev.ctypes.data, self.s.ctypes.data)
+
+
+def _res(r: Result, option=None, z=None, rc=0) -> dict:
+    if rc != 0:
+        raise RuntimeError(f"oracle returned {rc}")
+    out = dict(served=r.served, accsum=r.accsum, unmet=r.unmet, index=r.index,
+               n_candidates=r.n_candidates, eff=r.eff)
+    if option is not None:
+        out["option"] = option
+    if z is not None:
+        out["z"] = z
+    return out
+
+
+def family_lp(A, cap, mult, s):
+    """Per-family LP value (served, accsum) by vertex enumeration."""
+    sv, ac = C.c_int64(), C.c_int64()
+    rc = lib().orc_family_lp(len(A), np.ascontiguousarray(A, dtype=np.int64),
+                             np.ascontiguousarray(cap, dtype=np.int64), _i32(mult), int(s),
+                             C.byref(sv), C.byref(ac))
+    assert rc == 0
+    return sv.value, ac.value
+
+
+def score_placement(prof, device_type, slo_us, demand, option, P=None):
+    pr = _Prob(prof, device_type, slo_us, demand, P)
+    r = Result()
+    z = np.zeros(len(pr.dev), np.int32)
+    rc = lib().orc_score_placement(C.byref(pr.st), _i32(option), C.byref(r), z)
+    return _res(r, _i32(option), z, rc)
+
+
+def enum_count(prof, device_type, mode):
+    pr = _Prob(prof, device_type, np.ones(prof.Q, np.int32), np.zeros(prof.Q, np.int32),
+               P=np.zeros((prof.T, int(np.sum(prof.V))), np.int32))
+    n = C.c_uint64()
+    rc = lib().orc_enum_count(C.byref(pr.st), mode, C.byref(n))
+    if rc != 0:
+        raise OverflowError("candidate space exceeds 2^64")
+    return n.value
+
+
+def solve(prof, device_type, slo_us, demand, mode, threads=0, prune=1, P=None):
+    """Exhaustive optimum for one demand vector.  mode 0 flat mixed radix,
+    1 per-type multiset, 2 family-factored (reading C9 canonical forms)."""
+    pr = _Prob(prof, device_type, slo_us, demand, P)
+    r = Result()
+    D = len(pr.dev)
+    option = np.zeros(D, np.int32)
+    z = np.zeros(D, np.int32)
+    if mode in (0, 1):
+        rc = lib().orc_solve_enum(C.byref(pr.st), mode, threads, C.byref(r), option, z)
+        return _res(r, option, z, rc)
+    counts = np.zeros((prof.Q, 8, 16), np.int32)
+    rc = lib().orc_solve_factored(C.byref(pr.st), threads, prune, C.byref(r), option, z, counts)
+    out = _res(r, option, z, rc)
+    out["counts"] = counts[:, :prof.T, :]
+    return out
+
+
+def route_swrr(family, Q, dev_family, w_dev, w_sink):
+    """R8: literal SWRR; returns target device per query (D = sink)."""
+    family = np.ascontiguousarray(family, dtype=np.uint8)
+    tgt = np.zeros(len(family), np.int32)
+    D = len(dev_family)
+    rc = lib().orc_route_swrr(len(family), family, Q, D, _i32(dev_family), _i32(w_dev), _i32(w_sink), tgt)
+    assert rc == 0
+    return tgt
+
+
+def replay_device(arrival_us, Tproc, Bmax, L):
+    """§5 on one device.  Tproc[b] for b = 1..Bmax (Tproc[0] unused)."""
+    a = np.ascontiguousarray(arrival_us, dtype=np.uint32)
+    lat = np.zeros(len(a), np.uint32)
+    rc = lib().orc_replay_device(len(a), a, _i32(Tproc), int(Bmax), int(L), lat)
+    assert rc == 0
+    return lat
+
+
+def replay(prof, device_type, option, z, demand, slo_base, arrival_us, family, scenarios,
+           want_latency=True, threads=0):
+    """a11-a13: route + simulate.  Returns dict(latency [S][N] or None,
+    violations, on_time, acc_sum) per scenario."""
+    a = np.ascontiguousarray(arrival_us, dtype=np.uint32)
+    f = np.ascontiguousarray(family, dtype=np.uint8)
+    sc = _i32(scenarios).reshape(-1, 3)
+    S, N = sc.shape[0], len(a)
+    lat = np.zeros((S, N), np.uint32) if want_latency else None
+    viol = np.zeros(S, np.uint64)
+    ont = np.zeros(S, np.uint64)
+    accs = np.zeros(S, np.uint64)
+    rc = lib().orc_replay(N, a, f, prof.T, prof.Q, _i32(prof.V), _i32(prof.acc_micro), prof.bmax,
+                          _i32(prof.lat_us), len(device_type), _i32(option), _i32(z), _i32(device_type),
+                          _i32(demand), _i32(slo_base), S, sc, threads,
+                          lat.ctypes.data if lat is not None else None, viol, ont, accs)
+    if rc != 0:
+        raise RuntimeError(f"orc_replay returned {rc}")
+    return dict(latency=lat, violations=viol, on_time=ont, acc_sum=accs)
