@@ -1,0 +1,216 @@
+"""Proteus (ASPLOS '24) allocation search and adaptive-batching replay on B200.
+
+Thin Python binding of libproteus.so (include/proteus.h): argument marshalling
+only.  Arrays may be numpy arrays (host memory) or CUDA torch tensors (device
+memory, passed by pointer); the library detects which.
+
+    px = Proteus()                       # context on cuda:0, torch's current stream
+    px.load_profiles(prof)               # workloads.Profiles or equivalent arrays
+    sol = px.solve(device_type, slo_us, demand, mode=0)[0]
+    out = px.replay(arrival_us, family, sol.option, sol.z, device_type, demand, slo_us, scenarios)
+"""
+
+from __future__ import annotations
+
+import ctypes as C
+import dataclasses
+
+import numpy as np
+
+from . import _native as N
+from ._native import ProteusError  # noqa: F401
+
+__all__ = ["Proteus", "Solution", "ProteusError", "MODE_FLAT", "MODE_MULTISET", "MODE_FACTORED"]
+
+MODE_FLAT, MODE_MULTISET, MODE_FACTORED = 0, 1, 2
+UINT64_MAX = (1 << 64) - 1
+
+
+@dataclasses.dataclass
+class Solution:
+    score: int
+    index: int
+    served: int
+    unmet: int
+    accsum: int
+    eff_acc_micro: int
+    n_candidates: int
+    option: np.ndarray
+    z: np.ndarray
+
+
+def _is_torch(x):
+    return type(x).__module__.startswith("torch")
+
+
+def _arg(x, np_dtype, keep):
+    """Pointer to x's data: a torch tensor's data_ptr (host or device) or a
+    contiguous numpy copy's buffer.  `keep` holds references for the call."""
+    if x is None:
+        return None
+    if _is_torch(x):
+        import torch
+        want = {np.int32: torch.int32, np.uint32: torch.uint32, np.uint8: torch.uint8,
+                np.uint64: torch.uint64, np.int64: torch.int64}[np_dtype]
+        if x.dtype != want or not x.is_contiguous():
+            raise TypeError(f"tensor must be contiguous {want}, got {x.dtype}")
+        keep.append(x)
+        return x.data_ptr()
+    a = np.ascontiguousarray(x, dtype=np_dtype)
+    keep.append(a)
+    return a.ctypes.data
+
+
+class Proteus:
+    """One library context: one GPU, one CUDA stream (proteus.h)."""
+
+    def __init__(self, device: int = 0, stream=None):
+        self._lib = N.load()
+        if stream is None:
+            try:
+                import torch
+                if torch.cuda.is_available():
+                    stream = torch.cuda.current_stream(device).cuda_stream
+            except ImportError:
+                stream = None
+        h = C.c_void_p()
+        rc = self._lib.proteus_create(C.byref(h), device, C.c_void_p(stream) if stream else None)
+        if rc != 0:
+            raise ProteusError(rc, f"proteus_create(device={device}) failed (no CUDA device?)")
+        self._h = h
+        self.device = device
+        self.Q = None
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.proteus_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _check(self, rc):
+        if rc != 0:
+            msg = self._lib.proteus_last_error(self._h)
+            raise ProteusError(rc, msg.decode() if msg else "")
+
+    def set_stream(self, stream):
+        self._check(self._lib.proteus_set_stream(self._h, C.c_void_p(stream) if stream else None))
+
+    # ------------------------------------------------------------ profiles --
+    def load_profiles(self, prof=None, *, T=None, Q=None, V=None, acc_micro=None, bmax=None, lat_us=None):
+        if prof is not None:
+            T, Q, V, acc_micro, bmax, lat_us = prof.T, prof.Q, prof.V, prof.acc_micro, prof.bmax, prof.lat_us
+        keep = []
+        p = N.proteus_profiles(int(T), int(Q), _arg(V, np.int32, keep), _arg(acc_micro, np.int32, keep), int(bmax),
+                               _arg(lat_us, np.int32, keep))
+        self._check(self._lib.proteus_load_profiles(self._h, C.byref(p)))
+        self.Q = int(Q)
+
+    # --------------------------------------------------------------- solve --
+    def _solve_args(self, device_type, slo_us, demand, mode, shard_rank, shard_world, max_candidates, generic, keep):
+        dem = demand
+        if not _is_torch(dem):
+            dem = np.atleast_2d(np.asarray(demand, dtype=np.int32))
+            n_vec = dem.shape[0]
+        else:
+            n_vec = dem.shape[0] if dem.dim() == 2 else 1
+        D = len(device_type)
+        a = N.proteus_solve_args(D, _arg(device_type, np.int32, keep), int(mode), _arg(slo_us, np.int32, keep),
+                                 int(n_vec), _arg(dem, np.int32, keep), int(max_candidates), int(shard_rank),
+                                 int(shard_world), N.PROTEUS_SOLVE_GENERIC if generic else 0)
+        return a, n_vec, D
+
+    def solve(self, device_type, slo_us, demand, mode=MODE_FLAT, shard_rank=0, shard_world=1,
+              max_candidates=0, generic=False):
+        """Optimal allocation per demand vector (proteus_solve)."""
+        keep = []
+        a, n_vec, D = self._solve_args(device_type, slo_us, demand, mode, shard_rank, shard_world, max_candidates,
+                                       generic, keep)
+        opts = np.zeros((n_vec, D), np.int32)
+        zs = np.zeros((n_vec, D), np.int32)
+        sols = (N.proteus_solution * n_vec)()
+        for i in range(n_vec):
+            sols[i].option = opts[i].ctypes.data
+            sols[i].z_qps = zs[i].ctypes.data
+        self._check(self._lib.proteus_solve(self._h, C.byref(a), sols))
+        return [self._sol(sols[i], opts[i], zs[i]) for i in range(n_vec)]
+
+    def materialize(self, device_type, slo_us, demand, index, vec=0, mode=MODE_FLAT):
+        keep = []
+        a, n_vec, D = self._solve_args(device_type, slo_us, demand, mode, 0, 1, 0, False, keep)
+        opt = np.zeros(D, np.int32)
+        z = np.zeros(D, np.int32)
+        s = N.proteus_solution()
+        s.option = opt.ctypes.data
+        s.z_qps = z.ctypes.data
+        self._check(self._lib.proteus_materialize(self._h, C.byref(a), int(vec), int(index), C.byref(s)))
+        return self._sol(s, opt, z)
+
+    def candidate_count(self, device_type, mode=MODE_FLAT):
+        keep = []
+        a, _, _ = self._solve_args(device_type, np.zeros(self.Q, np.int32), np.zeros(self.Q, np.int32), mode, 0, 1,
+                                   0, False, keep)
+        n = C.c_uint64()
+        self._check(self._lib.proteus_candidate_count(self._h, C.byref(a), C.byref(n)))
+        return n.value
+
+    @staticmethod
+    def _sol(s, opt, z):
+        return Solution(s.score, s.index, s.served, s.unmet, s.accsum, s.eff_acc_micro, s.n_candidates,
+                        opt.copy(), z.copy())
+
+    # -------------------------------------------------------------- replay --
+    def replay(self, arrival_us, family, option, z, device_type, demand, slo_base_us, scenarios,
+               latency=True, aggregates_out=None):
+        """Adaptive-batching replay (proteus_replay).  latency: True -> host
+        numpy [S][N]; a CUDA uint32 tensor [S][N] -> written in place; None ->
+        not produced."""
+        keep = []
+        sc = np.ascontiguousarray(np.asarray(scenarios, dtype=np.int32).reshape(-1, 3))
+        S = sc.shape[0]
+        scs = (N.proteus_scenario * S)(*[N.proteus_scenario(*map(int, row)) for row in sc])
+        n = int(arrival_us.shape[0]) if hasattr(arrival_us, "shape") else len(arrival_us)
+        lat_np = None
+        if latency is True:
+            lat_np = np.empty((S, n), np.uint32)
+            lat_ptr = lat_np.ctypes.data
+        elif latency is None or latency is False:
+            lat_ptr = None
+        else:
+            lat_ptr = _arg(latency, np.uint32, keep)
+        if aggregates_out is not None:  # torch uint64 [3][S] on device
+            viol = _arg(aggregates_out[0], np.uint64, keep)
+            ont = _arg(aggregates_out[1], np.uint64, keep)
+            accs = _arg(aggregates_out[2], np.uint64, keep)
+            out = None
+        else:
+            out = np.zeros((3, S), np.uint64)
+            viol, ont, accs = out[0].ctypes.data, out[1].ctypes.data, out[2].ctypes.data
+        D = len(device_type)
+        rc = self._lib.proteus_replay(
+            self._h, _arg(arrival_us, np.uint32, keep), _arg(family, np.uint8, keep), n,
+            _arg(option, np.int32, keep), _arg(z, np.int32, keep), _arg(device_type, np.int32, keep), D,
+            _arg(demand, np.int32, keep), _arg(slo_base_us, np.int32, keep), scs, S, lat_ptr, viol, ont, accs)
+        self._check(rc)
+        res = {"latency": lat_np if latency is True else latency}
+        if out is not None:
+            res.update(violations=out[0], on_time=out[1], acc_sum=out[2])
+        return res
+
+    # ----------------------------------------------------- instrumentation --
+    def set_timing(self, on=True):
+        self._check(self._lib.proteus_set_timing(self._h, 1 if on else 0))
+
+    def kernel_times(self):
+        n = self._lib.proteus_kernel_times(self._h, None, None, 0)
+        names = (C.c_char_p * max(n, 1))()
+        ms = (C.c_float * max(n, 1))()
+        self._lib.proteus_kernel_times(self._h, names, ms, n)
+        return [(names[i].decode(), ms[i]) for i in range(n)]
+
+    def launch_count(self):
+        return int(self._lib.proteus_launch_count(self._h))

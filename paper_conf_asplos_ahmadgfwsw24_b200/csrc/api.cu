@@ -1,0 +1,461 @@
+// api.cu -- the C ABI (include/proteus.h) and the host runtime around the
+// kernels: context, grow-only device scratch, host/device pointer staging,
+// validation (overflow guards) and kernel timing.  All arithmetic of the method
+// runs in the kernels of prepare.cu, solve_enum.cu, solve_factored.cu and
+// replay.cu.
+#include <cstdarg>
+#include <cstring>
+
+#include "internal.cuh"
+
+// ---------------------------------------------------------------- utils ----
+int px_fail(proteus_ctx *ctx, int code, const char *fmt, ...) {
+  if (ctx) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    ctx->err = buf;
+  }
+  return code;
+}
+
+void *px_buf(proteus_ctx *ctx, int id, size_t bytes) {
+  DevBuf &b = ctx->bufs[id];
+  if (bytes == 0) bytes = 16;
+  if (b.n < bytes) {
+    if (b.p) {
+      cudaStreamSynchronize(ctx->stream);
+      cudaFree(b.p);
+      b.p = nullptr;
+      b.n = 0;
+    }
+    size_t n = bytes + bytes / 8;
+    if (cudaMalloc(&b.p, n) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    b.n = n;
+  }
+  return b.p;
+}
+
+bool px_is_device_ptr(const void *p) {
+  if (!p) return false;
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+void px_launch_begin(proteus_ctx *ctx, const char *name) {
+  ctx->launches++;
+  if (!ctx->timing) return;
+  cudaEvent_t a, b;
+  if (ctx->ev_pool.size() >= 2) {
+    a = ctx->ev_pool.back(); ctx->ev_pool.pop_back();
+    b = ctx->ev_pool.back(); ctx->ev_pool.pop_back();
+  } else {
+    cudaEventCreate(&a);
+    cudaEventCreate(&b);
+  }
+  cudaEventRecord(a, ctx->stream);
+  ctx->tnames.push_back(name);
+  ctx->tev.push_back(a);
+  ctx->tev.push_back(b);
+}
+
+int px_launch_end(proteus_ctx *ctx) {
+  cudaError_t e = cudaGetLastError();
+  if (ctx->timing) cudaEventRecord(ctx->tev.back(), ctx->stream);
+  if (e != cudaSuccess) return px_fail(ctx, PROTEUS_ECUDA, "kernel launch: %s", cudaGetErrorString(e));
+  return 0;
+}
+
+static void timing_reset(proteus_ctx *ctx) {
+  for (auto e : ctx->tev) ctx->ev_pool.push_back(e);
+  ctx->tev.clear();
+  ctx->tnames.clear();
+  ctx->tms.clear();
+}
+
+static int timing_collect(proteus_ctx *ctx) {
+  if (!ctx->timing) return 0;
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  ctx->tms.resize(ctx->tnames.size());
+  for (size_t i = 0; i < ctx->tnames.size(); i++) {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, ctx->tev[2 * i], ctx->tev[2 * i + 1]);
+    ctx->tms[i] = ms;
+  }
+  return 0;
+}
+
+// copy n elements of T from a host-or-device pointer into host memory
+template <class T>
+static int to_host(proteus_ctx *ctx, const T *p, size_t n, std::vector<T> &out) {
+  out.resize(n);
+  if (n == 0) return 0;
+  if (px_is_device_ptr(p)) {
+    PX_CUDA(ctx, cudaMemcpyAsync(out.data(), p, n * sizeof(T), cudaMemcpyDeviceToHost, ctx->stream));
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  } else {
+    memcpy(out.data(), p, n * sizeof(T));
+  }
+  return 0;
+}
+
+// device pointer for an input: the caller's if it is on the device, else a staged copy
+template <class T>
+static const T *to_device(proteus_ctx *ctx, const T *p, size_t n, int buf, int *rc) {
+  *rc = 0;
+  if (px_is_device_ptr(p)) return p;
+  T *d = (T *)px_buf(ctx, buf, n * sizeof(T));
+  if (!d) { *rc = px_fail(ctx, PROTEUS_ENOMEM, "device scratch (%zu bytes)", n * sizeof(T)); return nullptr; }
+  if (n) {
+    cudaError_t e = cudaMemcpyAsync(d, p, n * sizeof(T), cudaMemcpyHostToDevice, ctx->stream);
+    if (e != cudaSuccess) { *rc = px_fail(ctx, PROTEUS_ECUDA, "H2D: %s", cudaGetErrorString(e)); return nullptr; }
+  }
+  return d;
+}
+
+
+// --------------------------------------------------------------- ABI -----
+extern "C" {
+
+int proteus_abi_version(void) { return PROTEUS_ABI_VERSION; }
+
+int proteus_create(proteus_ctx **out, int cuda_device, void *cuda_stream) {
+  if (!out) return PROTEUS_EINVAL;
+  *out = nullptr;
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || cuda_device < 0 || cuda_device >= n) {
+    cudaGetLastError();
+    return PROTEUS_ECUDA;
+  }
+  if (cudaSetDevice(cuda_device) != cudaSuccess) return PROTEUS_ECUDA;
+  proteus_ctx *c = new proteus_ctx();
+  c->device = cuda_device;
+  c->stream = (cudaStream_t)cuda_stream;
+  *out = c;
+  return PROTEUS_OK;
+}
+
+void proteus_destroy(proteus_ctx *ctx) {
+  if (!ctx) return;
+  cudaSetDevice(ctx->device);
+  cudaStreamSynchronize(ctx->stream);
+  for (auto &b : ctx->bufs) if (b.p) cudaFree(b.p);
+  for (int32_t *p : {ctx->d_lat, ctx->d_acc, ctx->d_fam, ctx->d_off, ctx->d_V}) if (p) cudaFree(p);
+  for (auto e : ctx->tev) cudaEventDestroy(e);
+  for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+  delete ctx;
+}
+
+int proteus_set_stream(proteus_ctx *ctx, void *cuda_stream) {
+  if (!ctx) return PROTEUS_EINVAL;
+  ctx->stream = (cudaStream_t)cuda_stream;
+  return PROTEUS_OK;
+}
+
+const char *proteus_last_error(const proteus_ctx *ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+int proteus_set_timing(proteus_ctx *ctx, int enable) {
+  if (!ctx) return PROTEUS_EINVAL;
+  ctx->timing = enable != 0;
+  return PROTEUS_OK;
+}
+
+int proteus_kernel_times(const proteus_ctx *ctx, const char **names, float *ms, int cap) {
+  if (!ctx) return PROTEUS_EINVAL;
+  int n = (int)ctx->tms.size();
+  for (int i = 0; i < n && i < cap; i++) {
+    if (names) names[i] = ctx->tnames[i];
+    if (ms) ms[i] = ctx->tms[i];
+  }
+  return n;
+}
+
+uint64_t proteus_launch_count(const proteus_ctx *ctx) { return ctx ? ctx->launches : 0; }
+
+int proteus_load_profiles(proteus_ctx *ctx, const proteus_profiles *p) {
+  if (!ctx || !p || !p->V || !p->acc_micro || !p->lat_us) return px_fail(ctx, PROTEUS_EINVAL, "null argument");
+  ctx->err.clear();
+  if (p->T < 1 || p->T > PX_MAXT || p->Q < 1 || p->Q > PX_MAXQ || p->bmax < 1 || p->bmax > PX_MAXB)
+    return px_fail(ctx, PROTEUS_EINVAL, "T=%d Q=%d bmax=%d out of range", p->T, p->Q, p->bmax);
+  PX_CUDA(ctx, cudaSetDevice(ctx->device));
+  std::vector<int32_t> V, acc, lat;
+  int rc;
+  if ((rc = to_host(ctx, p->V, p->Q, V))) return rc;
+  int M = 0;
+  for (int q = 0; q < p->Q; q++) {
+    if (V[q] < 1 || V[q] > PX_MAXV) return px_fail(ctx, PROTEUS_EINVAL, "V[%d]=%d out of range", q, V[q]);
+    M += V[q];
+  }
+  if (M > PX_MAXM) return px_fail(ctx, PROTEUS_EINVAL, "sum V = %d > %d", M, PX_MAXM);
+  if ((rc = to_host(ctx, p->acc_micro, M, acc))) return rc;
+  for (int m = 0; m < M; m++)
+    if (acc[m] < 1 || acc[m] > 1000000) return px_fail(ctx, PROTEUS_ERANGE, "acc_micro[%d]=%d not in [1, 1e6]", m, acc[m]);
+  if ((rc = to_host(ctx, p->lat_us, (size_t)p->T * M * p->bmax, lat))) return rc;
+  for (int32_t x : lat)
+    if (x < 0) return px_fail(ctx, PROTEUS_EINVAL, "negative latency");
+  std::vector<int32_t> fam(M), off(p->Q);
+  for (int q = 0, m = 0; q < p->Q; q++) {
+    off[q] = m;
+    for (int v = 0; v < V[q]; v++) fam[m++] = q;
+  }
+  for (int32_t *ptr : {ctx->d_lat, ctx->d_acc, ctx->d_fam, ctx->d_off, ctx->d_V}) if (ptr) cudaFree(ptr);
+  ctx->d_lat = ctx->d_acc = ctx->d_fam = ctx->d_off = ctx->d_V = nullptr;
+  PX_CUDA(ctx, cudaMalloc(&ctx->d_lat, lat.size() * 4));
+  PX_CUDA(ctx, cudaMalloc(&ctx->d_acc, M * 4));
+  PX_CUDA(ctx, cudaMalloc(&ctx->d_fam, M * 4));
+  PX_CUDA(ctx, cudaMalloc(&ctx->d_off, p->Q * 4));
+  PX_CUDA(ctx, cudaMalloc(&ctx->d_V, p->Q * 4));
+  PX_CUDA(ctx, cudaMemcpyAsync(ctx->d_lat, lat.data(), lat.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(ctx->d_acc, acc.data(), M * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(ctx->d_fam, fam.data(), M * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(ctx->d_off, off.data(), p->Q * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(ctx->d_V, V.data(), p->Q * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  ctx->T = p->T; ctx->Q = p->Q; ctx->M = M; ctx->bmax = p->bmax;
+  ctx->V = V; ctx->acc = acc; ctx->lat = lat; ctx->fam = fam; ctx->off = off;
+  ctx->have_prof = true;
+  return PROTEUS_OK;
+}
+
+}  // extern "C"
+
+// -------------------------------------------------------------- solve -----
+struct SolveInputs {
+  std::vector<int32_t> dev_type, slo, demand;
+};
+
+static int validate_solve(proteus_ctx *ctx, const proteus_solve_args *a, SolveInputs &in) {
+  if (!ctx) return PROTEUS_EINVAL;
+  ctx->err.clear();
+  if (!a) return px_fail(ctx, PROTEUS_EINVAL, "null args");
+  if (!ctx->have_prof) return px_fail(ctx, PROTEUS_EINVAL, "no profiles loaded");
+  if (a->D < 1 || a->D > PX_MAXD) return px_fail(ctx, PROTEUS_EINVAL, "D=%d out of range [1, %d]", a->D, PX_MAXD);
+  if (a->mode < 0 || a->mode > 2) return px_fail(ctx, PROTEUS_EINVAL, "mode %d", a->mode);
+  if (a->n_vec < 1) return px_fail(ctx, PROTEUS_EINVAL, "n_vec=%d", a->n_vec);
+  if (!a->device_type || !a->slo_us || !a->demand_qps) return px_fail(ctx, PROTEUS_EINVAL, "null array");
+  if (a->shard_world < 0 || a->shard_rank < 0 || (a->shard_world > 0 && a->shard_rank >= a->shard_world))
+    return px_fail(ctx, PROTEUS_EINVAL, "shard %d/%d", a->shard_rank, a->shard_world);
+  int rc;
+  PX_CUDA(ctx, cudaSetDevice(ctx->device));
+  if ((rc = to_host(ctx, a->device_type, a->D, in.dev_type))) return rc;
+  if ((rc = to_host(ctx, a->slo_us, ctx->Q, in.slo))) return rc;
+  if ((rc = to_host(ctx, a->demand_qps, (size_t)a->n_vec * ctx->Q, in.demand))) return rc;
+  for (int d = 0; d < a->D; d++)
+    if (in.dev_type[d] < 0 || in.dev_type[d] >= ctx->T)
+      return px_fail(ctx, PROTEUS_EINVAL, "device_type[%d]=%d", d, in.dev_type[d]);
+  for (int q = 0; q < ctx->Q; q++)
+    if (in.slo[q] < 0) return px_fail(ctx, PROTEUS_EINVAL, "slo_us[%d] < 0", q);
+  for (int v = 0; v < a->n_vec; v++) {
+    int64_t sum = 0;
+    for (int q = 0; q < ctx->Q; q++) {
+      int32_t s = in.demand[(size_t)v * ctx->Q + q];
+      if (s < 0) return px_fail(ctx, PROTEUS_EINVAL, "negative demand");
+      sum += s;
+    }
+    if (sum >= (1 << 22)) return px_fail(ctx, PROTEUS_ERANGE, "sum of demand %lld >= 2^22", (long long)sum);
+  }
+  return 0;
+}
+
+// families supplied in accuracy order (non-increasing within each family)?
+static bool families_sorted(const proteus_ctx *ctx) {
+  for (int q = 0; q < ctx->Q; q++)
+    for (int v = 1; v < ctx->V[q]; v++)
+      if (ctx->acc[ctx->off[q] + v] > ctx->acc[ctx->off[q] + v - 1]) return false;
+  return true;
+}
+
+int px_flat_template_vm(int Q, int maxV);  // solve_enum.cu: VM of the specialised kernel, 0 if none
+
+static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_solution *out, bool mat_only,
+                        int32_t mat_vec, uint64_t mat_index) {
+  SolveInputs in;
+  int rc = validate_solve(ctx, a, in);
+  if (rc) return rc;
+  if (!out) return px_fail(ctx, PROTEUS_EINVAL, "null out");
+  if (mat_only && (a->mode == 2 || mat_vec < 0 || mat_vec >= a->n_vec))
+    return px_fail(ctx, PROTEUS_EINVAL, "materialize: mode %d vec %d", a->mode, mat_vec);
+  timing_reset(ctx);
+  int K = 1 + ctx->M;
+  int maxV = 0;
+  for (int q = 0; q < ctx->Q; q++) maxV = ctx->V[q] > maxV ? ctx->V[q] : maxV;
+  int VM = maxV;
+  bool use_flat = false;
+  if (a->mode == 0 && !(a->flags & PROTEUS_SOLVE_GENERIC) && a->D >= 3 && families_sorted(ctx)) {
+    int vm = px_flat_template_vm(ctx->Q, maxV);
+    if (vm) { VM = vm; use_flat = true; }
+  }
+  if (a->mode != 2) {
+    bool ovf = false;
+    uint64_t n = px_count_candidates(a->mode, a->D, in.dev_type.data(), ctx->T, K, &ovf);
+    if (ovf || n > (1ull << 63)) return px_fail(ctx, PROTEUS_ERANGE, "candidate space exceeds 2^63");
+    if (a->max_candidates && n > a->max_candidates)
+      return px_fail(ctx, PROTEUS_ERANGE, "candidate space %llu > max_candidates %llu", (unsigned long long)n,
+                     (unsigned long long)a->max_candidates);
+  }
+  const int32_t *d_dev = to_device(ctx, in.dev_type.data(), in.dev_type.size(), B_IN0, &rc);
+  if (rc) return rc;
+  const int32_t *d_slo = to_device(ctx, in.slo.data(), in.slo.size(), B_IN1, &rc);
+  if (rc) return rc;
+  const int32_t *d_dem = to_device(ctx, in.demand.data(), in.demand.size(), B_IN2, &rc);
+  if (rc) return rc;
+  Tables tab;
+  if ((rc = px_prepare_tables(ctx, a->D, d_dev, d_slo, VM, tab))) return rc;
+  // the launch parameters of the scoring kernels carry the capacity table
+  std::vector<int32_t> h_P((size_t)ctx->T * ctx->M), h_slot_code((size_t)ctx->Q * VM);
+  PX_CUDA(ctx, cudaMemcpyAsync(h_P.data(), tab.P, h_P.size() * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(h_slot_code.data(), tab.slot_code, h_slot_code.size() * 4, cudaMemcpyDeviceToHost,
+                               ctx->stream));
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  int nout = mat_only ? 1 : a->n_vec;
+  SolRec *d_sol = (SolRec *)px_buf(ctx, B_SOL, sizeof(SolRec) * nout);
+  if (!d_sol) return px_fail(ctx, PROTEUS_ENOMEM, "solution buffer");
+  if (a->mode == 2) {
+    rc = px_solve_factored(ctx, a, in.dev_type.data(), d_dev, d_dem, VM, tab, h_P, d_sol);
+  } else if (mat_only) {
+    rc = px_solve_enum(ctx, a, in.dev_type.data(), in.slo.data(), in.demand.data(), VM, tab, h_P, h_slot_code,
+                       d_sol, mat_vec, mat_vec + 1, true, mat_index, use_flat);
+  } else {
+    rc = px_solve_enum(ctx, a, in.dev_type.data(), in.slo.data(), in.demand.data(), VM, tab, h_P, h_slot_code,
+                       d_sol, 0, a->n_vec, false, 0, use_flat);
+  }
+  if (rc) return rc;
+  std::vector<SolRec> h(nout);
+  PX_CUDA(ctx, cudaMemcpyAsync(h.data(), d_sol, sizeof(SolRec) * nout, cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  if ((rc = timing_collect(ctx))) return rc;
+  for (int i = 0; i < nout; i++)
+    if (h[i].status != 0) return px_fail(ctx, PROTEUS_EINTERNAL, "internal check failed (vector %d, code %d)", i, h[i].status);
+  for (int i = 0; i < nout; i++) {
+    proteus_solution &o = out[i];
+    o.score = h[i].score;
+    o.index = h[i].index;
+    o.served = h[i].served;
+    o.unmet = h[i].unmet;
+    o.accsum = h[i].accsum;
+    o.eff_acc_micro = h[i].eff;
+    o.n_candidates = h[i].n_candidates;
+    if (o.option) {
+      if (px_is_device_ptr(o.option)) PX_CUDA(ctx, cudaMemcpy(o.option, h[i].option, a->D * 4, cudaMemcpyHostToDevice));
+      else memcpy(o.option, h[i].option, a->D * 4);
+    }
+    if (o.z_qps) {
+      if (px_is_device_ptr(o.z_qps)) PX_CUDA(ctx, cudaMemcpy(o.z_qps, h[i].z, a->D * 4, cudaMemcpyHostToDevice));
+      else memcpy(o.z_qps, h[i].z, a->D * 4);
+    }
+  }
+  return PROTEUS_OK;
+}
+
+extern "C" {
+
+int proteus_solve(proteus_ctx *ctx, const proteus_solve_args *args, proteus_solution *out) {
+  return solve_common(ctx, args, out, false, 0, 0);
+}
+
+int proteus_materialize(proteus_ctx *ctx, const proteus_solve_args *args, int32_t vec, uint64_t index,
+                        proteus_solution *out) {
+  return solve_common(ctx, args, out, true, vec, index);
+}
+
+int proteus_candidate_count(proteus_ctx *ctx, const proteus_solve_args *a, uint64_t *count) {
+  if (!ctx || !a || !count) return PROTEUS_EINVAL;
+  if (!ctx->have_prof) return px_fail(ctx, PROTEUS_EINVAL, "no profiles loaded");
+  if (a->mode != 0 && a->mode != 1) return px_fail(ctx, PROTEUS_EINVAL, "mode %d", a->mode);
+  std::vector<int32_t> dev;
+  int rc;
+  if ((rc = to_host(ctx, a->device_type, a->D, dev))) return rc;
+  bool ovf = false;
+  *count = px_count_candidates(a->mode, a->D, dev.data(), ctx->T, 1 + ctx->M, &ovf);
+  return ovf ? px_fail(ctx, PROTEUS_ERANGE, "candidate space exceeds 2^64") : PROTEUS_OK;
+}
+
+// ------------------------------------------------------------- replay -----
+int proteus_replay(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *family, int64_t N,
+                   const int32_t *option, const int32_t *z_qps, const int32_t *device_type, int32_t D,
+                   const int32_t *demand_qps, const int32_t *slo_base_us, const proteus_scenario *sc, int32_t S,
+                   uint32_t *latency_us, uint64_t *violations, uint64_t *on_time, uint64_t *acc_sum) {
+  if (!ctx) return PROTEUS_EINVAL;
+  ctx->err.clear();
+  if (!ctx->have_prof) return px_fail(ctx, PROTEUS_EINVAL, "no profiles loaded");
+  if (N < 0 || (N > 0 && (!arrival_us || !family))) return px_fail(ctx, PROTEUS_EINVAL, "trace");
+  if (N >= (1ll << 32)) return px_fail(ctx, PROTEUS_ERANGE, "N >= 2^32");
+  if (D < 1 || D > PX_MAXD || !option || !z_qps || !device_type || !demand_qps || !slo_base_us)
+    return px_fail(ctx, PROTEUS_EINVAL, "allocation arguments");
+  if (S < 1 || S > 4096 || !sc) return px_fail(ctx, PROTEUS_EINVAL, "S=%d", S);
+  PX_CUDA(ctx, cudaSetDevice(ctx->device));
+  timing_reset(ctx);
+  int rc;
+  std::vector<int32_t> opt, z, dev, dem, slo;
+  std::vector<proteus_scenario> scv;
+  if ((rc = to_host(ctx, option, D, opt)) || (rc = to_host(ctx, z_qps, D, z)) ||
+      (rc = to_host(ctx, device_type, D, dev)) || (rc = to_host(ctx, demand_qps, ctx->Q, dem)) ||
+      (rc = to_host(ctx, slo_base_us, ctx->Q, slo)) || (rc = to_host(ctx, sc, S, scv)))
+    return rc;
+  int64_t dsum = 0;
+  for (int q = 0; q < ctx->Q; q++) {
+    if (dem[q] < 0 || slo[q] < 0) return px_fail(ctx, PROTEUS_EINVAL, "negative demand/slo");
+    dsum += dem[q];
+  }
+  if (dsum >= (1 << 22)) return px_fail(ctx, PROTEUS_ERANGE, "sum of demand >= 2^22");
+  std::vector<int64_t> zsum(ctx->Q, 0);
+  for (int d = 0; d < D; d++) {
+    if (dev[d] < 0 || dev[d] >= ctx->T) return px_fail(ctx, PROTEUS_EINVAL, "device_type[%d]", d);
+    if (opt[d] < 0 || opt[d] > ctx->M) return px_fail(ctx, PROTEUS_EINVAL, "option[%d]=%d", d, opt[d]);
+    if (z[d] < 0 || (opt[d] == 0 && z[d] != 0)) return px_fail(ctx, PROTEUS_EINVAL, "z[%d]=%d", d, z[d]);
+    if (opt[d]) zsum[ctx->fam[opt[d] - 1]] += z[d];
+  }
+  for (int q = 0; q < ctx->Q; q++)
+    if (zsum[q] > dem[q]) return px_fail(ctx, PROTEUS_EINVAL, "sum z of family %d exceeds its demand", q);
+  for (int s = 0; s < S; s++)
+    if (scv[s].slo_mult_milli < 0 || scv[s].batch_cap < 0 || scv[s].routing < 0 || scv[s].routing > 1)
+      return px_fail(ctx, PROTEUS_EINVAL, "scenario %d", s);
+  const uint32_t *d_arr = to_device(ctx, arrival_us, (size_t)N, B_IN0, &rc);
+  if (rc) return rc;
+  const uint8_t *d_fam = to_device(ctx, family, (size_t)N, B_IN1, &rc);
+  if (rc) return rc;
+  uint32_t *d_lat = nullptr;
+  bool lat_dev = latency_us && px_is_device_ptr(latency_us);
+  if (latency_us) {
+    d_lat = lat_dev ? latency_us : (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S * N * 4);
+    if (!d_lat) return px_fail(ctx, PROTEUS_ENOMEM, "latency buffer");
+  }
+  uint64_t *d_agg = (uint64_t *)px_buf(ctx, B_R_AGG, (size_t)3 * S * 8 + 8);
+  if (!d_agg) return px_fail(ctx, PROTEUS_ENOMEM, "aggregate buffer");
+  rc = px_replay(ctx, d_arr, d_fam, N, opt.data(), z.data(), dev.data(), D, dem.data(), slo.data(), scv.data(), S,
+                 d_lat, d_agg);
+  if (rc) return rc;
+  std::vector<uint64_t> agg((size_t)3 * S + 1);
+  PX_CUDA(ctx, cudaMemcpyAsync(agg.data(), d_agg, ((size_t)3 * S + 1) * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  if (latency_us && !lat_dev)
+    PX_CUDA(ctx, cudaMemcpyAsync(latency_us, d_lat, (size_t)S * N * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  if ((rc = timing_collect(ctx))) return rc;
+  if (agg[3 * S] != 0) return px_fail(ctx, PROTEUS_ERANGE, "arrival timestamps not sorted");
+  for (int s = 0; s < S; s++) {
+    if (violations) {
+      if (px_is_device_ptr(violations)) PX_CUDA(ctx, cudaMemcpy(violations + s, &agg[s], 8, cudaMemcpyHostToDevice));
+      else violations[s] = agg[s];
+    }
+    if (on_time) {
+      if (px_is_device_ptr(on_time)) PX_CUDA(ctx, cudaMemcpy(on_time + s, &agg[S + s], 8, cudaMemcpyHostToDevice));
+      else on_time[s] = agg[S + s];
+    }
+    if (acc_sum) {
+      if (px_is_device_ptr(acc_sum)) PX_CUDA(ctx, cudaMemcpy(acc_sum + s, &agg[2 * S + s], 8, cudaMemcpyHostToDevice));
+      else acc_sum[s] = agg[2 * S + s];
+    }
+  }
+  return PROTEUS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,373 @@
+// replay.cu -- trace replay of an allocation under the adaptive batching
+// policy of §5: a11 routing pre-pass, a12 lane kernel, a13
+// per-scenario reductions.
+//
+// Routing (reading R8): per family q, the SWRR sequence over the members
+// (hosting devices ascending with weight z_d, then a drop sink with weight
+// s_q - sum z) has period W_q = sum of weights; query k of family q (k = its
+// ordinal among family-q queries) goes to pattern_q[k mod W_q].  The pre-pass
+// computes every query's family ordinal and target device with stable
+// per-tile counting (warp match + per-tile offsets), then scatters the
+// arrivals into per-device arrays (device-major, arrival order kept).
+//
+// Lane kernel: one thread per (scenario, device) walks the device's arrival
+// array with the §5 rule written as a window walk (readings R1-R5): at decision
+// time t = max(F, a[h]) with q queued (capped at Bmax), dispatch Bmax when
+// q >= Bmax; otherwise with W = a[h] + SLO - T(q+1) dispatch q once t >= W,
+// else move t to the next arrival if it comes by W (Case 2), else to W (Case 1).
+#include "internal.cuh"
+
+#define TILE 1024
+#define TILE_WARPS 8
+#define LANE_THREADS 128
+
+// -------------------------------------------------------------- checks ----
+__global__ void k_check_trace(const uint32_t *__restrict__ arr, const uint8_t *__restrict__ fam, int64_t N, int Q,
+                              uint32_t *flags) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    if (i > 0 && arr[i] < arr[i - 1]) atomicOr(flags, 1u);
+    if (fam[i] >= Q) atomicOr(flags, 2u);
+  }
+}
+
+// ------------------------------------------------------------- routing ----
+// One block.  Weights and the SWRR pattern of every family (R8).
+//   routing 0: member weight z_d for hosting devices with z_d > 0, sink weight
+//              s_q - sum z (unmet demand, reading R7)
+//   routing 1: weight 1 per hosting device that fits batch 1 (depth >= 1); no sink
+__global__ void k_route_prepare(int routing, int Q, int D, int M, int bmax, const int32_t *__restrict__ option,
+                                const int32_t *__restrict__ z, const int32_t *__restrict__ dev_type,
+                                const int32_t *__restrict__ demand, const int32_t *__restrict__ fam_of_m,
+                                const int32_t *__restrict__ lat, uint8_t *pattern, int32_t *pat_off,
+                                int32_t *pat_len) {
+  __shared__ int32_t W[PX_MAXQ];
+  const int q = threadIdx.x;
+  int32_t w[PX_MAXD + 1];
+  int32_t cur[PX_MAXD + 1];
+  if (q < Q) {
+    int64_t tot = 0, zsum = 0;
+    for (int d = 0; d < D; d++) {
+      w[d] = 0;
+      const int o = option[d];
+      if (o <= 0 || fam_of_m[o - 1] != q) continue;
+      if (routing == 0) {
+        w[d] = z[d];
+        zsum += z[d];
+      } else {
+        w[d] = lat[((size_t)dev_type[d] * M + (o - 1)) * bmax] > 0 ? 1 : 0;
+      }
+      tot += w[d];
+    }
+    w[D] = routing == 0 ? (int32_t)(demand[q] - zsum) : 0;
+    tot += w[D];
+    W[q] = (int32_t)tot;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int32_t acc = 0;
+    for (int k = 0; k < Q; k++) { pat_off[k] = acc; pat_len[k] = W[k]; acc += W[k]; }
+  }
+  __syncthreads();
+  if (q >= Q) return;
+  const int32_t Wq = W[q];
+  uint8_t *pat = pattern + pat_off[q];
+  for (int d = 0; d <= D; d++) cur[d] = 0;
+  for (int32_t k = 0; k < Wq; k++) {
+    int best = -1;
+    for (int d = 0; d <= D; d++) {
+      if (w[d] == 0) continue;
+      cur[d] += w[d];
+      if (best < 0 || cur[d] > cur[best]) best = d;
+    }
+    cur[best] -= Wq;
+    pat[k] = (uint8_t)best;
+  }
+}
+
+// per-tile key histogram: one warp per tile of TILE queries
+__global__ void k_tile_count(const uint8_t *__restrict__ keys, int64_t N, int nkeys, int32_t *hist) {
+  __shared__ int32_t cnt[TILE_WARPS][PX_MAXD + 2];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t tile = (int64_t)blockIdx.x * TILE_WARPS + w;
+  for (int k = lane; k < nkeys; k += 32) cnt[w][k] = 0;
+  __syncwarp();
+  const int64_t t0 = tile * TILE;
+  if (t0 < N) {
+    for (int c = 0; c < TILE; c += 32) {
+      const int64_t i = t0 + c + lane;
+      const bool valid = i < N;
+      const int key = valid ? keys[i] : 255;
+      const unsigned peers = __match_any_sync(0xffffffffu, key);
+      if (valid && lane == __ffs(peers) - 1) cnt[w][key] += __popc(peers);
+      __syncwarp();
+    }
+    for (int k = lane; k < nkeys; k += 32) hist[tile * nkeys + k] = cnt[w][k];
+  }
+}
+
+// exclusive scan over tiles, one block per key; totals[key]
+__global__ void k_tile_scan(const int32_t *__restrict__ hist, int64_t ntiles, int nkeys, int32_t *base,
+                            int64_t *totals) {
+  const int key = blockIdx.x;
+  __shared__ int64_t part[1024];
+  const int64_t per = (ntiles + blockDim.x - 1) / blockDim.x;
+  const int64_t lo = threadIdx.x * per, hi = lo + per < ntiles ? lo + per : ntiles;
+  int64_t s = 0;
+  for (int64_t t = lo; t < hi; t++) s += hist[t * nkeys + key];
+  part[threadIdx.x] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int64_t acc = 0;
+    for (int i = 0; i < (int)blockDim.x; i++) { int64_t v = part[i]; part[i] = acc; acc += v; }
+    totals[key] = acc;
+  }
+  __syncthreads();
+  int64_t acc = part[threadIdx.x];
+  for (int64_t t = lo; t < hi; t++) {
+    base[t * nkeys + key] = (int32_t)acc;
+    acc += hist[t * nkeys + key];
+  }
+}
+
+// family ordinal -> target device (pattern lookup); per-tile target histogram
+__global__ void k_route_target(const uint8_t *__restrict__ fam, int64_t N, int Q, const int32_t *__restrict__ famBase,
+                               const uint8_t *__restrict__ pattern, const int32_t *__restrict__ pat_off,
+                               const int32_t *__restrict__ pat_len, int D, uint8_t *target, int32_t *histDev) {
+  __shared__ int32_t run[TILE_WARPS][PX_MAXQ];
+  __shared__ int32_t cnt[TILE_WARPS][PX_MAXD + 2];
+  __shared__ int32_t sOff[PX_MAXQ], sLen[PX_MAXQ];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x < Q) { sOff[threadIdx.x] = pat_off[threadIdx.x]; sLen[threadIdx.x] = pat_len[threadIdx.x]; }
+  const int64_t tile = (int64_t)blockIdx.x * TILE_WARPS + w;
+  const int64_t t0 = tile * TILE;
+  if (t0 < N)
+    for (int k = lane; k < Q; k += 32) run[w][k] = famBase[tile * Q + k];
+  for (int k = lane; k <= D; k += 32) cnt[w][k] = 0;
+  __syncthreads();
+  if (t0 >= N) return;
+  for (int c = 0; c < TILE; c += 32) {
+    const int64_t i = t0 + c + lane;
+    const bool valid = i < N;
+    const int key = valid ? fam[i] : 255;
+    const unsigned peers = __match_any_sync(0xffffffffu, key);
+    const int rank = __popc(peers & ((1u << lane) - 1));
+    int ord = 0;
+    if (valid) ord = run[w][key] + rank;
+    __syncwarp();
+    if (valid && lane == __ffs(peers) - 1) run[w][key] += __popc(peers);
+    int tgt = D;
+    if (valid) {
+      const int len = sLen[key];
+      tgt = len > 0 ? pattern[sOff[key] + (ord % len)] : D;
+      target[i] = (uint8_t)tgt;
+    }
+    const unsigned tp = __match_any_sync(0xffffffffu, valid ? tgt : 255);
+    if (valid && lane == __ffs(tp) - 1) cnt[w][tgt] += __popc(tp);
+    __syncwarp();
+  }
+  for (int k = lane; k <= D; k += 32) histDev[tile * (D + 1) + k] = cnt[w][k];
+}
+
+__global__ void k_dev_offsets(const int64_t *__restrict__ totals, int n, int64_t *off) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    int64_t acc = 0;
+    for (int k = 0; k < n; k++) { off[k] = acc; acc += totals[k]; }
+    off[n] = acc;
+  }
+}
+
+// stable scatter into device-major arrays
+__global__ void k_scatter(const uint8_t *__restrict__ target, const uint32_t *__restrict__ arr, int64_t N, int D,
+                          const int32_t *__restrict__ devBase, const int64_t *__restrict__ devOff, uint32_t *devArr,
+                          uint32_t *devIdx) {
+  __shared__ int64_t run[TILE_WARPS][PX_MAXD + 2];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t tile = (int64_t)blockIdx.x * TILE_WARPS + w;
+  const int64_t t0 = tile * TILE;
+  if (t0 >= N) return;
+  for (int k = lane; k <= D; k += 32) run[w][k] = devOff[k] + devBase[tile * (D + 1) + k];
+  __syncwarp();
+  for (int c = 0; c < TILE; c += 32) {
+    const int64_t i = t0 + c + lane;
+    const bool valid = i < N;
+    const int key = valid ? target[i] : 255;
+    const unsigned peers = __match_any_sync(0xffffffffu, key);
+    const int rank = __popc(peers & ((1u << lane) - 1));
+    int64_t pos = 0;
+    if (valid) pos = run[w][key] + rank;
+    __syncwarp();
+    if (valid && lane == __ffs(peers) - 1) run[w][key] += __popc(peers);
+    __syncwarp();
+    if (valid) { devArr[pos] = arr[i]; devIdx[pos] = (uint32_t)i; }
+  }
+}
+
+// --------------------------------------------------------------- lanes ----
+struct LaneArgs {
+  int S, D, M, bmax;
+  int64_t N;
+  const int32_t *option, *dev_type, *fam_of_m, *acc, *lat, *slo_base;
+  const proteus_scenario *sc;
+  const int64_t *devOff[2];
+  const uint32_t *devArr[2], *devIdx[2];
+  uint32_t *lat_out;  // [S][N] or null
+  uint64_t *agg;      // [3][S]
+};
+
+__global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ LaneArgs a) {
+  const int lane_id = blockIdx.x * blockDim.x + threadIdx.x;
+  if (lane_id >= a.S * a.D) return;
+  const int s = lane_id / a.D, d = lane_id % a.D;
+  const int o = a.option[d];
+  if (o <= 0) return;
+  const proteus_scenario sc = a.sc[s];
+  const int rt = sc.routing;
+  const int64_t st = a.devOff[rt][d], n = a.devOff[rt][d + 1] - st;
+  if (n == 0) return;
+  const uint32_t *arr = a.devArr[rt] + st;
+  const uint32_t *idx = a.devIdx[rt] + st;
+  const int m = o - 1;
+  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + m) * a.bmax;  // T[b-1]
+  int depth = 0;
+  while (depth < a.bmax && T[depth] > 0) depth++;
+  const int Bmax = (sc.batch_cap > 0 && sc.batch_cap < depth) ? sc.batch_cap : depth;
+  const int64_t L = (int64_t)sc.slo_mult_milli * a.slo_base[a.fam_of_m[m]] / 1000;
+  const uint32_t A = (uint32_t)a.acc[m];
+  uint64_t viol = 0, ont = 0, accs = 0;
+  if (Bmax < 1) {  // cannot run even batch 1 (routing 1 never routes here; routing 0 has z = 0)
+    viol = (uint64_t)n;
+    if (a.lat_out)
+      for (int64_t j = 0; j < n; j++) a.lat_out[(size_t)s * a.N + idx[j]] = 0xFFFFFFFFu;
+  } else {
+    int64_t h = 0, F = 0;
+    while (h < n) {
+      const int64_t ah = arr[h];
+      int64_t t = F > ah ? F : ah;
+      int q = 1;
+      while (q < Bmax && h + q < n && (int64_t)arr[h + q] <= t) q++;
+      int b;
+      for (;;) {
+        if (q >= Bmax) { b = Bmax; break; }
+        const int64_t W = ah + L - T[q];  // T(q+1)
+        if (t >= W) { b = q; break; }
+        if (h + q < n && (int64_t)arr[h + q] <= W) {
+          t = arr[h + q];
+          while (q < Bmax && h + q < n && (int64_t)arr[h + q] <= t) q++;
+          continue;
+        }
+        t = W;
+        b = q;
+        break;
+      }
+      F = t + T[b - 1];
+      for (int j = 0; j < b; j++) {
+        const int64_t l = F - (int64_t)arr[h + j];
+        const uint32_t lv = l >= 0xFFFFFFFFll ? 0xFFFFFFFEu : (uint32_t)l;
+        if ((int64_t)lv > L) viol++;
+        else { ont++; accs += A; }
+        if (a.lat_out) a.lat_out[(size_t)s * a.N + idx[h + j]] = lv;
+      }
+      h += b;
+    }
+  }
+  atomicAdd((unsigned long long *)&a.agg[s], (unsigned long long)viol);
+  atomicAdd((unsigned long long *)&a.agg[a.S + s], (unsigned long long)ont);
+  atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], (unsigned long long)accs);
+}
+
+// dropped queries (the sink segment, device index D)
+__global__ void k_sink(const proteus_scenario *__restrict__ sc, int S, int D, int64_t N, const int64_t *devOff0,
+                       const uint32_t *devIdx0, const int64_t *devOff1, const uint32_t *devIdx1, uint32_t *lat_out,
+                       uint64_t *agg) {
+  for (int s = blockIdx.y; s < S; s += gridDim.y) {
+    const int rt = sc[s].routing;
+    const int64_t *off = rt ? devOff1 : devOff0;
+    const uint32_t *idx = rt ? devIdx1 : devIdx0;
+    const int64_t st = off[D], n = off[D + 1] - st;
+    if (blockIdx.x == 0 && threadIdx.x == 0 && n) atomicAdd((unsigned long long *)&agg[s], (unsigned long long)n);
+    if (lat_out)
+      for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
+        lat_out[(size_t)s * N + idx[st + j]] = 0xFFFFFFFFu;
+  }
+}
+
+// ---------------------------------------------------------------- host ----
+int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int64_t N, const int32_t *h_option,
+              const int32_t *h_z, const int32_t *h_dev_type, int D, const int32_t *h_demand, const int32_t *h_slo,
+              const proteus_scenario *h_sc, int S, uint32_t *d_lat_out, uint64_t *d_agg) {
+  const int Q = ctx->Q, M = ctx->M;
+  PX_CUDA(ctx, cudaMemsetAsync(d_agg, 0, ((size_t)3 * S + 1) * 8, ctx->stream));
+  // small inputs: option, z, dev_type, demand, slo, scenarios
+  const size_t small = (size_t)(4 * D + 2 * Q) * 4 + (size_t)S * sizeof(proteus_scenario) + 64;
+  char *sb = (char *)px_buf(ctx, B_R_MISC, small + 4096);
+  if (!sb) return px_fail(ctx, PROTEUS_ENOMEM, "replay scratch");
+  int32_t *d_opt = (int32_t *)sb, *d_z = d_opt + D, *d_dev = d_z + D, *d_dem = d_dev + D, *d_slo = d_dem + Q;
+  int32_t *d_pat_off = d_slo + Q, *d_pat_len = d_pat_off + PX_MAXQ;
+  uint32_t *d_flags = (uint32_t *)(d_pat_len + PX_MAXQ);
+  proteus_scenario *d_sc = (proteus_scenario *)(((uintptr_t)(d_flags + 4) + 15) & ~(uintptr_t)15);
+  PX_CUDA(ctx, cudaMemcpyAsync(d_opt, h_option, D * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_z, h_z, D * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_dev, h_dev_type, D * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_dem, h_demand, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_slo, h_slo, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_sc, h_sc, S * sizeof(proteus_scenario), cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemsetAsync(d_flags, 0, 4, ctx->stream));
+  if (N > 0) {
+    PX_LAUNCH(ctx, "replay_check", k_check_trace, 1184, 256, 0, d_arr, d_fam, N, Q, d_flags);
+    uint32_t flags = 0;
+    PX_CUDA(ctx, cudaMemcpyAsync(&flags, d_flags, 4, cudaMemcpyDeviceToHost, ctx->stream));
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+    if (flags & 1) return px_fail(ctx, PROTEUS_ERANGE, "arrival timestamps not sorted");
+    if (flags & 2) return px_fail(ctx, PROTEUS_EINVAL, "family id >= Q");
+  }
+  const int64_t ntiles = (N + TILE - 1) / TILE;
+  const unsigned tblocks = (unsigned)((ntiles + TILE_WARPS - 1) / TILE_WARPS);
+  int64_t dsum = 0;
+  for (int q = 0; q < Q; q++) dsum += h_demand[q];
+  const size_t pat_cap = (size_t)dsum + (size_t)Q * D + 16;
+  bool used[2] = {false, false};
+  for (int s = 0; s < S; s++) used[h_sc[s].routing] = true;
+  const int64_t *devOff[2] = {nullptr, nullptr};
+  const uint32_t *devArr[2] = {nullptr, nullptr}, *devIdx[2] = {nullptr, nullptr};
+  for (int rt = 0; rt < 2; rt++) {
+    if (!used[rt]) continue;
+    uint8_t *pat = (uint8_t *)px_buf(ctx, B_R_PAT, pat_cap);
+    int32_t *hist = (int32_t *)px_buf(ctx, B_R_HIST, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
+    int32_t *base = (int32_t *)px_buf(ctx, B_R_BASE, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
+    uint8_t *tgt = (uint8_t *)px_buf(ctx, B_R_TGT, (size_t)N + 16);
+    int64_t *off = (int64_t *)px_buf(ctx, rt ? B_R_OFF1 : B_R_OFF, (size_t)2 * (PX_MAXD + 2) * 8);
+    uint32_t *darr = (uint32_t *)px_buf(ctx, rt ? B_R_DEVARR1 : B_R_DEVARR, (size_t)N * 4 + 16);
+    uint32_t *didx = (uint32_t *)px_buf(ctx, rt ? B_R_DEVIDX1 : B_R_DEVIDX, (size_t)N * 4 + 16);
+    if (!pat || !hist || !base || !tgt || !off || !darr || !didx) return px_fail(ctx, PROTEUS_ENOMEM, "routing buffers");
+    int64_t *totals = off + (PX_MAXD + 2);
+    PX_LAUNCH(ctx, "route_prepare", k_route_prepare, 1, 32, 0, rt, Q, D, M, ctx->bmax, d_opt, d_z, d_dev, d_dem,
+              ctx->d_fam, ctx->d_lat, pat, d_pat_off, d_pat_len);
+    if (N > 0) {
+      PX_LAUNCH(ctx, "route_count", k_tile_count, tblocks, TILE_WARPS * 32, 0, d_fam, N, Q, hist);
+      PX_LAUNCH(ctx, "route_scan", k_tile_scan, Q, 1024, 0, hist, ntiles, Q, base, totals);
+      PX_LAUNCH(ctx, "route_target", k_route_target, tblocks, TILE_WARPS * 32, 0, d_fam, N, Q, base, pat, d_pat_off,
+                d_pat_len, D, tgt, hist);
+      PX_LAUNCH(ctx, "route_scan_dev", k_tile_scan, D + 1, 1024, 0, hist, ntiles, D + 1, base, totals);
+      PX_LAUNCH(ctx, "route_offsets", k_dev_offsets, 1, 32, 0, totals, D + 1, off);
+      PX_LAUNCH(ctx, "route_scatter", k_scatter, tblocks, TILE_WARPS * 32, 0, tgt, d_arr, N, D, base, off, darr, didx);
+    } else {
+      PX_CUDA(ctx, cudaMemsetAsync(off, 0, (size_t)(PX_MAXD + 2) * 8, ctx->stream));
+    }
+    devOff[rt] = off; devArr[rt] = darr; devIdx[rt] = didx;
+  }
+  if (N == 0) return 0;
+  LaneArgs la;
+  la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.N = N;
+  la.option = d_opt; la.dev_type = d_dev; la.fam_of_m = ctx->d_fam; la.acc = ctx->d_acc; la.lat = ctx->d_lat;
+  la.slo_base = d_slo; la.sc = d_sc;
+  for (int rt = 0; rt < 2; rt++) { la.devOff[rt] = devOff[rt]; la.devArr[rt] = devArr[rt]; la.devIdx[rt] = devIdx[rt]; }
+  la.lat_out = d_lat_out;
+  la.agg = d_agg;
+  const int nl = S * D;
+  PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
+  dim3 g(64, S < 65535 ? S : 65535);
+  PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, d_sc, S, D, N, devOff[0] ? devOff[0] : devOff[1],
+            devIdx[0] ? devIdx[0] : devIdx[1], devOff[1] ? devOff[1] : devOff[0], devIdx[1] ? devIdx[1] : devIdx[0],
+            d_lat_out, d_agg);
+  return 0;
+}

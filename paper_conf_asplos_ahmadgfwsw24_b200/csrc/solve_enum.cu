@@ -1,0 +1,495 @@
+// solve_enum.cu -- exhaustive allocation search, modes 0 (flat mixed radix) and
+// 1 (per-type multiset): a2 candidate decode, a3 capacity aggregation, a4
+// per-family water-fill, a5 score pack, a6 warp -> block -> grid argmax with
+// lowest-index tie-break, a9 winner materialisation.
+//
+// Two scoring kernels:
+//  * k_flat_pair<QM, VM>: mode 0 with families supplied in accuracy order and
+//    Q <= QM, V_q <= VM.  Every thread owns a contiguous range of "prefixes"
+//    (the options of devices 0..D-3); for each prefix it scores the K^2
+//    candidates formed by the last two devices.  Capacities live in registers
+//    (slots are compile-time indices), the per-device capacity of the last two
+//    devices and the accuracies are launch parameters (constant bank), so a
+//    candidate costs one 64-bit add + compare, or one joint water-fill when
+//    both of the last two devices host the same family.
+//  * k_enum_generic: any mode 0/1 instance within the ABI limits; decodes the
+//    start index once (mixed radix over groups, combinadic unrank inside a
+//    group) and walks successors, rescoring every candidate from scratch.
+#include <algorithm>
+
+#include "internal.cuh"
+
+#define FLAT_THREADS 256
+#define GEN_THREADS 128
+
+// ------------------------------------------------------------ reduce ----
+__device__ __forceinline__ void warp_best(uint64_t &s, uint64_t &i) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    uint64_t s2 = __shfl_xor_sync(0xffffffffu, s, o);
+    uint64_t i2 = __shfl_xor_sync(0xffffffffu, i, o);
+    if (px_better(s2, i2, s, i)) { s = s2; i = i2; }
+  }
+}
+
+// block-wide (score desc, index asc) maximum; result valid in thread 0
+__device__ __forceinline__ void block_best(uint64_t &s, uint64_t &i) {
+  __shared__ uint64_t ws[32], wi[32];
+  warp_best(s, i);
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+  if (lane == 0) { ws[w] = s; wi[w] = i; }
+  __syncthreads();
+  if (w == 0) {
+    s = lane < nw ? ws[lane] : 0;
+    i = lane < nw ? wi[lane] : ~0ull;
+    warp_best(s, i);
+  }
+}
+
+__global__ void k_best_final(const BestRec *__restrict__ in, int n, BestRec *out) {
+  uint64_t s = 0, i = ~0ull;
+  for (int k = threadIdx.x; k < n; k += blockDim.x)
+    if (px_better(in[k].score, in[k].index, s, i)) { s = in[k].score; i = in[k].index; }
+  block_best(s, i);
+  if (threadIdx.x == 0) { out->score = s; out->index = i; }
+}
+
+// ------------------------------------------------------ group layout ----
+// Candidates are tuples per group; a group's devices are interchangeable and
+// take a non-decreasing option tuple (mode 0: every device is a group of one).
+// Index = mixed radix over groups (group 0 most significant) of the tuple's
+// lexicographic rank (reading C9).
+struct EnumArgs {
+  int32_t D, K, Q, VM, npos, ngroups;
+  int32_t pos_dev[PX_MAXD];
+  int32_t pos_group[PX_MAXD];
+  int32_t group_start[PX_MAXD + 1];
+  uint64_t group_stride[PX_MAXD];
+  uint64_t lo, hi, per_thread;
+  int32_t s[PX_MAXQ];
+  int32_t V[PX_MAXQ];
+  const int32_t *Pdev, *code_slot, *slot_acc, *slot_code;
+  BestRec *out;
+};
+
+__device__ __forceinline__ uint64_t binom_dev(uint64_t n, uint64_t k) {
+  if (k > n) return 0;
+  if (k > n - k) k = n - k;
+  unsigned __int128 r = 1;
+  for (uint64_t i = 1; i <= k; i++) r = r * (n - k + i) / i;
+  return (uint64_t)r;
+}
+
+// rank r -> non-decreasing tuple of length len over [0, K), lexicographic
+__device__ void unrank_tuple(uint64_t r, int len, int K, int32_t *out) {
+  int v = 0;
+  for (int i = 0; i < len; i++) {
+    int rest = len - i - 1;
+    for (;; v++) {
+      // tuples of length `rest` over symbols [v, K)
+      uint64_t cnt = binom_dev((uint64_t)(K - v) + rest - 1, (uint64_t)rest);
+      if (r < cnt) break;
+      r -= cnt;
+    }
+    out[i] = v;
+  }
+}
+
+__device__ void decode_index(const EnumArgs &a, uint64_t idx, int32_t *opt /* [npos] */) {
+  for (int g = 0; g < a.ngroups; g++) {
+    uint64_t r = idx / a.group_stride[g];
+    idx -= r * a.group_stride[g];
+    int gs = a.group_start[g], len = a.group_start[g + 1] - gs;
+    unrank_tuple(r, len, a.K, opt + gs);
+  }
+}
+
+// -------------------------------------------------- generic scoring ----
+__global__ void __launch_bounds__(GEN_THREADS) k_enum_generic(const __grid_constant__ EnumArgs a) {
+  __shared__ int32_t sAcc[PX_MAXQ * PX_MAXV];
+  __shared__ int32_t sCS[PX_MAXM + 1];
+  for (int i = threadIdx.x; i < a.Q * a.VM; i += blockDim.x) sAcc[i] = a.slot_acc[i];
+  for (int i = threadIdx.x; i < a.K; i += blockDim.x) sCS[i] = a.code_slot[i];
+  __syncthreads();
+  const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  uint64_t c = a.lo + tid * a.per_thread;
+  const uint64_t cend = c + a.per_thread < a.hi ? c + a.per_thread : a.hi;
+  uint64_t best_s = 0, best_i = ~0ull;
+  if (c < cend) {
+    int32_t opt[PX_MAXD];
+    int32_t cap[PX_MAXQ * PX_MAXV];
+    for (int i = 0; i < a.Q * a.VM; i++) cap[i] = 0;
+    decode_index(a, c, opt);
+    for (int p = 0; p < a.npos; p++) {
+      int o = opt[p];
+      if (o) cap[sCS[o]] += __ldg(&a.Pdev[a.pos_dev[p] * a.K + o]);
+    }
+    for (;;) {
+      uint64_t score = 0;
+      for (int q = 0; q < a.Q; q++) {
+        int rem = a.s[q];
+        uint64_t acc = 0;
+        for (int j = 0; j < a.V[q]; j++) {
+          int t = min(rem, cap[q * a.VM + j]);
+          acc += (uint64_t)(uint32_t)sAcc[q * a.VM + j] * (uint32_t)t;
+          rem -= t;
+        }
+        score += px_pack((uint32_t)(a.s[q] - rem), acc);
+      }
+      if (px_better(score, c, best_s, best_i)) { best_s = score; best_i = c; }
+      if (++c >= cend) break;
+      // successor: rightmost group that can advance; its suffix is reset
+      int p = a.npos - 1;
+      for (;;) {
+        int g = a.pos_group[p], gs = a.group_start[g], ge = a.group_start[g + 1];
+        int i = ge - 1;
+        while (i >= gs && opt[i] == a.K - 1) i--;
+        if (i >= gs) {
+          int nv = opt[i] + 1;
+          for (int j = i; j < ge; j++) {
+            int o = opt[j], dv = a.pos_dev[j];
+            if (o) cap[sCS[o]] -= __ldg(&a.Pdev[dv * a.K + o]);
+            opt[j] = nv;
+            cap[sCS[nv]] += __ldg(&a.Pdev[dv * a.K + nv]);
+          }
+          break;
+        }
+        for (int j = gs; j < ge; j++) {
+          int o = opt[j];
+          if (o) cap[sCS[o]] -= __ldg(&a.Pdev[a.pos_dev[j] * a.K + o]);
+          opt[j] = 0;
+        }
+        p = gs - 1;  // carry into the previous group (exists: c < hi)
+      }
+    }
+  }
+  block_best(best_s, best_i);
+  if (threadIdx.x == 0) { a.out[blockIdx.x].score = best_s; a.out[blockIdx.x].index = best_i; }
+}
+
+// -------------------------------------------- specialised flat kernel ----
+template <int QM, int VM>
+struct FlatArgs {
+  int32_t D, K;
+  uint64_t p_lo, p_hi, per_thread;
+  int32_t A[QM * VM];   // accuracy per slot
+  int32_t PA[QM * VM];  // capacity of slot on device D-2
+  int32_t PB[QM * VM];  // capacity of slot on device D-1
+  int32_t code[QM * VM];
+  int32_t s[QM];
+  const int32_t *Pdev, *code_slot;
+  BestRec *out;
+};
+
+// water-fill of family q over slots q*VM..q*VM+VM-1, with capacity pa added
+// to slot ja and pb to slot jb (compile-time; -1 = none) -> packed score
+template <int QM, int VM>
+__device__ __forceinline__ uint64_t fill(const int (&caps)[QM * VM], const FlatArgs<QM, VM> &a, int q, int ja,
+                                         int pa, int jb, int pb) {
+  int rem = a.s[q];
+  uint64_t acc = 0;
+#pragma unroll
+  for (int j = 0; j < VM; j++) {
+    int c = caps[q * VM + j] + (j == ja ? pa : 0) + (j == jb ? pb : 0);
+    int t = min(rem, c);
+    acc += (uint64_t)(uint32_t)a.A[q * VM + j] * (uint32_t)t;
+    rem -= t;
+  }
+  return px_pack((uint32_t)(a.s[q] - rem), acc);
+}
+
+template <int QM, int VM>
+__global__ void __launch_bounds__(FLAT_THREADS) k_flat_pair(const __grid_constant__ FlatArgs<QM, VM> a) {
+  constexpr int S = QM * VM;
+  extern __shared__ int32_t smem[];
+  const int D = a.D, K = a.K;
+  int32_t *sP = smem;          // [D][K]
+  int32_t *sCS = smem + D * K; // [K]
+  for (int i = threadIdx.x; i < D * K; i += blockDim.x) sP[i] = a.Pdev[i];
+  for (int i = threadIdx.x; i < K; i += blockDim.x) sCS[i] = a.code_slot[i];
+  __syncthreads();
+  const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  uint64_t p = a.p_lo + tid * a.per_thread;
+  const uint64_t pend = p + a.per_thread < a.p_hi ? p + a.per_thread : a.p_hi;
+  const uint64_t KK = (uint64_t)K * K;
+  uint64_t best_s = 0, best_i = ~0ull;
+  if (p < pend) {
+    int dig[PX_MAXD];
+    {
+      uint64_t x = p;
+      for (int i = D - 3; i >= 0; i--) { dig[i] = (int)(x % K); x /= K; }
+    }
+    int capsB[S];
+    auto rebuild = [&]() {
+#pragma unroll
+      for (int s = 0; s < S; s++) capsB[s] = 0;
+      for (int i = 0; i < D - 3; i++) {
+        const int o = dig[i];
+        const int sl = sCS[o], pv = sP[i * K + o];
+#pragma unroll
+        for (int s = 0; s < S; s++) capsB[s] += (sl == s) ? pv : 0;
+      }
+    };
+    rebuild();
+    for (;;) {
+      const int o3 = dig[D - 3];
+      const int sl3 = sCS[o3], p3 = sP[(D - 3) * K + o3];
+      int caps[S];
+#pragma unroll
+      for (int s = 0; s < S; s++) caps[s] = capsB[s] + (sl3 == s ? p3 : 0);
+      uint64_t Fq[QM];
+      uint64_t base = 0;
+#pragma unroll
+      for (int q = 0; q < QM; q++) { Fq[q] = fill<QM, VM>(caps, a, q, -1, 0, -1, 0); base += Fq[q]; }
+      uint64_t Fa[S], Fb[S];
+#pragma unroll
+      for (int s = 0; s < S; s++) {
+        const int q = s / VM, j = s % VM;
+        Fa[s] = fill<QM, VM>(caps, a, q, j, a.PA[s], -1, 0) - Fq[q];
+        Fb[s] = fill<QM, VM>(caps, a, q, j, a.PB[s], -1, 0) - Fq[q];
+      }
+      // the K^2 candidates of this prefix, in increasing index order
+      uint64_t lb = best_s;
+      int lp = -1;
+      if (base > lb || best_i == ~0ull) { lb = base; lp = 0; }
+#pragma unroll
+      for (int sb = 0; sb < S; sb++)
+        if (a.code[sb]) {
+          const uint64_t c = base + Fb[sb];
+          if (c > lb) { lb = c; lp = a.code[sb]; }
+        }
+#pragma unroll
+      for (int sa = 0; sa < S; sa++) {
+        if (!a.code[sa]) continue;
+        const uint64_t ba = base + Fa[sa];
+        if (ba > lb) { lb = ba; lp = a.code[sa] * K; }
+#pragma unroll
+        for (int sb = 0; sb < S; sb++) {
+          if (!a.code[sb]) continue;
+          uint64_t c;
+          if (sa / VM == sb / VM) {
+            const int q = sa / VM;
+            c = base - Fq[q] + fill<QM, VM>(caps, a, q, sa % VM, a.PA[sa], sb % VM, a.PB[sb]);
+          } else {
+            c = ba + Fb[sb];
+          }
+          if (c > lb) { lb = c; lp = a.code[sa] * K + a.code[sb]; }
+        }
+      }
+      if (lp >= 0) { best_s = lb; best_i = p * KK + (uint64_t)lp; }
+      if (++p >= pend) break;
+      if (++dig[D - 3] == K) {
+        dig[D - 3] = 0;
+        for (int i = D - 4; i >= 0; i--) {
+          if (++dig[i] < K) break;
+          dig[i] = 0;
+        }
+        rebuild();
+      }
+    }
+  }
+  block_best(best_s, best_i);
+  if (threadIdx.x == 0) { a.out[blockIdx.x].score = best_s; a.out[blockIdx.x].index = best_i; }
+}
+
+// ------------------------------------------------------- materialise ----
+// a9: decode the winner, water-fill z in (accuracy desc, code asc, device asc)
+// order (reading C10), report served / unmet / accsum / eff; re-check the score.
+__global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const BestRec *best, uint64_t fixed_index,
+                                   int use_fixed, uint64_t n_candidates, SolRec *out) {
+  if (threadIdx.x != 0) return;
+  SolRec &r = *out;
+  uint64_t idx = use_fixed ? fixed_index : best->index;
+  if (idx == ~0ull) {  // empty shard: nothing scored
+    for (int d = 0; d < a.D; d++) { r.option[d] = 0; r.z[d] = 0; }
+    int64_t stot = 0;
+    for (int q = 0; q < a.Q; q++) stot += a.s[q];
+    r.score = 0; r.index = idx; r.served = 0; r.unmet = stot; r.accsum = 0; r.eff = 0;
+    r.n_candidates = n_candidates; r.status = 0;
+    return;
+  }
+  int32_t opt[PX_MAXD];
+  decode_index(a, idx, opt);
+  for (int d = 0; d < a.D; d++) { r.option[d] = 0; r.z[d] = 0; }
+  for (int p = 0; p < a.npos; p++) r.option[a.pos_dev[p]] = opt[p];
+  int64_t served = 0, accsum = 0, stot = 0;
+  uint64_t score = 0;
+  for (int q = 0; q < a.Q; q++) {
+    int rem = a.s[q];
+    uint64_t acc = 0;
+    stot += a.s[q];
+    for (int j = 0; j < a.V[q]; j++) {
+      const int code = a.slot_code[q * a.VM + j];
+      const int A = a.slot_acc[q * a.VM + j];
+      for (int d = 0; d < a.D; d++) {
+        if (r.option[d] != code) continue;
+        const int t = min(rem, a.Pdev[d * a.K + code]);
+        r.z[d] = t;
+        rem -= t;
+        acc += (uint64_t)A * (uint64_t)t;
+      }
+    }
+    served += a.s[q] - rem;
+    accsum += (int64_t)acc;
+    score += px_pack((uint32_t)(a.s[q] - rem), acc);
+  }
+  r.score = score;
+  r.index = idx;
+  r.served = served;
+  r.unmet = stot - served;
+  r.accsum = accsum;
+  r.eff = served > 0 ? (int32_t)(accsum / served) : 0;
+  r.n_candidates = n_candidates;
+  r.status = (!use_fixed && score != best->score) ? 1 : 0;
+}
+
+// ------------------------------------------------------------- host -----
+template <int QM, int VM>
+static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p_hi, const int32_t *dev_type,
+                       const int32_t *demand, const std::vector<int32_t> &h_P, const std::vector<int32_t> &h_slot_code,
+                       const Tables &tab, BestRec *d_blocks, int *nblocks_out) {
+  FlatArgs<QM, VM> a;
+  memset(&a, 0, sizeof a);
+  a.D = D; a.K = K;
+  const int M = ctx->M;
+  for (int s = 0; s < QM * VM; s++) {
+    const int q = s / VM;
+    const int code = q < ctx->Q ? h_slot_code[q * VM + s % VM] : 0;
+    a.code[s] = code;
+    a.A[s] = code ? ctx->acc[code - 1] : 0;
+    a.PA[s] = code ? h_P[dev_type[D - 2] * M + code - 1] : 0;
+    a.PB[s] = code ? h_P[dev_type[D - 1] * M + code - 1] : 0;
+  }
+  for (int q = 0; q < QM; q++) a.s[q] = q < ctx->Q ? demand[q] : 0;
+  a.Pdev = tab.Pdev;
+  a.code_slot = tab.code_slot;
+  a.out = d_blocks;
+  const size_t smem = (size_t)(D * K + K) * 4;
+  auto kern = k_flat_pair<QM, VM>;
+  if (smem > 48 * 1024) PX_CUDA(ctx, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int nsm = 0, occ = 0;
+  PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
+  PX_CUDA(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, FLAT_THREADS, smem));
+  if (occ < 1) occ = 1;
+  const uint64_t np = p_hi - p_lo;
+  uint64_t nb = (uint64_t)nsm * occ;
+  const uint64_t need = (np + FLAT_THREADS - 1) / FLAT_THREADS;
+  if (need < nb) nb = need ? need : 1;
+  a.p_lo = p_lo; a.p_hi = p_hi;
+  a.per_thread = (np + nb * FLAT_THREADS - 1) / (nb * FLAT_THREADS);
+  if (a.per_thread == 0) a.per_thread = 1;
+  PX_LAUNCH(ctx, "score_flat_pair", kern, (unsigned)nb, FLAT_THREADS, smem, a);
+  *nblocks_out = (int)nb;
+  return 0;
+}
+
+typedef int (*flat_fn)(proteus_ctx *, int, int, uint64_t, uint64_t, const int32_t *, const int32_t *,
+                       const std::vector<int32_t> &, const std::vector<int32_t> &, const Tables &, BestRec *, int *);
+
+struct FlatInst { int QM, VM; flat_fn fn; };
+static const FlatInst kFlat[] = {
+    {1, 2, launch_flat<1, 2>}, {1, 3, launch_flat<1, 3>}, {1, 4, launch_flat<1, 4>}, {1, 5, launch_flat<1, 5>},
+    {2, 2, launch_flat<2, 2>}, {2, 3, launch_flat<2, 3>}, {2, 4, launch_flat<2, 4>}, {2, 5, launch_flat<2, 5>},
+    {3, 2, launch_flat<3, 2>}, {3, 3, launch_flat<3, 3>}, {3, 4, launch_flat<3, 4>}, {3, 5, launch_flat<3, 5>},
+    {4, 2, launch_flat<4, 2>}, {4, 3, launch_flat<4, 3>}, {4, 4, launch_flat<4, 4>}, {4, 5, launch_flat<4, 5>},
+};
+
+static const FlatInst *pick_flat(int Q, int maxV) {
+  const FlatInst *best = nullptr;
+  for (const auto &f : kFlat)
+    if (f.QM >= Q && f.VM >= maxV && (!best || f.QM * f.VM < best->QM * best->VM)) best = &f;
+  return best;
+}
+
+int px_flat_template_vm(int Q, int maxV) {
+  const FlatInst *f = pick_flat(Q, maxV);
+  return f ? f->VM : 0;
+}
+
+static uint64_t mul_div(uint64_t a, uint64_t b, uint64_t c) {
+  return (uint64_t)((unsigned __int128)a * b / c);
+}
+
+int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_t *h_dev_type,
+                  const int32_t *h_slo, const int32_t *h_demand, int VM, const Tables &tab,
+                  const std::vector<int32_t> &h_P, const std::vector<int32_t> &h_slot_code,
+                  SolRec *d_sol, int32_t vec_lo, int32_t vec_hi, bool materialize_only, uint64_t mat_index,
+                  bool use_flat) {
+  (void)h_slo;
+  const int D = args->D, K = 1 + ctx->M, Q = ctx->Q, T = ctx->T;
+  const int mode = args->mode;
+  // group layout
+  EnumArgs ea;
+  memset(&ea, 0, sizeof ea);
+  ea.D = D; ea.K = K; ea.Q = Q; ea.VM = VM;
+  int np = 0, ng = 0;
+  if (mode == 0) {
+    for (int d = 0; d < D; d++) { ea.group_start[ng] = np; ea.pos_dev[np] = d; ea.pos_group[np] = ng; np++; ng++; }
+  } else {
+    for (int t = 0; t < T; t++) {
+      int start = np;
+      for (int d = 0; d < D; d++)
+        if (h_dev_type[d] == t) { ea.pos_dev[np] = d; ea.pos_group[np] = ng; np++; }
+      if (np > start) { ea.group_start[ng] = start; ng++; }
+    }
+  }
+  ea.group_start[ng] = np;
+  ea.npos = np; ea.ngroups = ng;
+  {
+    uint64_t stride = 1;
+    for (int g = ng - 1; g >= 0; g--) {
+      ea.group_stride[g] = stride;
+      int len = ea.group_start[g + 1] - ea.group_start[g];
+      unsigned __int128 c = 1;
+      for (int i = 1; i <= len; i++) c = c * (unsigned)(K - 1 + i) / (unsigned)i;
+      stride = (uint64_t)((unsigned __int128)stride * c);
+    }
+  }
+  for (int q = 0; q < Q; q++) ea.V[q] = ctx->V[q];
+  ea.Pdev = tab.Pdev; ea.code_slot = tab.code_slot; ea.slot_acc = tab.slot_acc; ea.slot_code = tab.slot_code;
+  bool ovf = false;
+  const uint64_t N = px_count_candidates(mode, D, h_dev_type, T, K, &ovf);
+  const int world = args->shard_world > 0 ? args->shard_world : 1, rank = args->shard_world > 0 ? args->shard_rank : 0;
+  const bool flat_ok = use_flat;
+  int nsm = 0;
+  PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
+  const size_t max_blocks = (size_t)nsm * 64;
+  BestRec *d_blocks = (BestRec *)px_buf(ctx, B_BEST, sizeof(BestRec) * (max_blocks + 1));
+  if (!d_blocks) return px_fail(ctx, PROTEUS_ENOMEM, "block results");
+  BestRec *d_best = d_blocks + max_blocks;
+  for (int v = vec_lo; v < vec_hi; v++) {
+    const int32_t *dem = h_demand + (size_t)v * Q;
+    for (int q = 0; q < Q; q++) ea.s[q] = dem[q];
+    SolRec *rec = d_sol + (materialize_only ? 0 : v - vec_lo);
+    uint64_t ncand = 0;
+    if (!materialize_only) {
+      int nb = 0;
+      if (flat_ok) {
+        const uint64_t NP = N / ((uint64_t)K * K);
+        const uint64_t plo = mul_div(NP, rank, world), phi = mul_div(NP, rank + 1, world);
+        ncand = (phi - plo) * (uint64_t)K * K;
+        const FlatInst *f = pick_flat(Q, *std::max_element(ctx->V.begin(), ctx->V.end()));
+        int rc = f->fn(ctx, D, K, plo, phi, h_dev_type, dem, h_P, h_slot_code, tab, d_blocks, &nb);
+        if (rc) return rc;
+      } else {
+        const uint64_t lo = mul_div(N, rank, world), hi = mul_div(N, rank + 1, world);
+        ncand = hi - lo;
+        int occ = 0;
+        PX_CUDA(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_enum_generic, GEN_THREADS, 0));
+        uint64_t nb64 = (uint64_t)nsm * (occ > 0 ? occ : 1);
+        const uint64_t need = (ncand + GEN_THREADS - 1) / GEN_THREADS;
+        if (need < nb64) nb64 = need ? need : 1;
+        ea.lo = lo; ea.hi = hi;
+        ea.per_thread = (ncand + nb64 * GEN_THREADS - 1) / (nb64 * GEN_THREADS);
+        if (!ea.per_thread) ea.per_thread = 1;
+        ea.out = d_blocks;
+        PX_LAUNCH(ctx, "score_generic", k_enum_generic, (unsigned)nb64, GEN_THREADS, 0, ea);
+        nb = (int)nb64;
+      }
+      PX_LAUNCH(ctx, "argmax_grid", k_best_final, 1, 1024, 0, d_blocks, nb, d_best);
+    }
+    PX_LAUNCH(ctx, "materialize", k_materialize_enum, 1, 32, 0, ea, d_best, mat_index, materialize_only ? 1 : 0,
+              ncand, rec);
+  }
+  return 0;
+}

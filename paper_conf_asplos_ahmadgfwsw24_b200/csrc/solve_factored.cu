@@ -1,0 +1,364 @@
+// solve_factored.cu -- mode 2, the family-factored exact search (a8) and the
+// batched per-second re-solve (a10).
+//
+// Eqs. 1, 3 and 5 make a device serve only the family of the
+// variant it hosts, so a placement's value is the sum over families of the
+// family's water-fill value, which depends only on the family's count vector
+// n[t][v] (devices of type t hosting variant v).  The search is therefore
+//   g_q(u) = max over count vectors of family q with usage u (u_t = sum_v n[t][v])
+//   G_q(b) = max_{u <= b} g_q(u) + G_{q+1}(b - u),  G_Q = 0,  optimum G_0(N),
+// and the canonical solution is the lexicographically smallest tensor n
+// (q-major, then t, then v) among optima (reading C9), reconstructed family
+// by family.  Variants with P = 0 on a type are never used by that solution
+// (reading C16) and are left out of the type's count vectors.
+//
+// Kernels:
+//  k_fact_lists  one thread per (family, type): the type's count vectors in
+//                lexicographic order (rank), their capacity vector in fill
+//                order, their usage, and a stable bucketing by usage.
+//  k_fact_g      one warp per (vector, family, usage u): the product of the
+//                per-type usage buckets, water-filled and reduced to the best
+//                (score desc, lexicographic rank asc).
+//  k_fact_dp     one block per vector: the budget DP over the usage lattice,
+//                reconstruction, materialisation (a9).
+#include <algorithm>
+
+#include "internal.cuh"
+
+#define FG_WARPS 8
+#define DP_THREADS 256
+
+struct FactLayout {
+  int32_t Q, T, VM, U;
+  int32_t Nt[PX_MAXT];
+  int32_t ustride[PX_MAXT];           // u key = sum_t u_t * ustride[t], type T-1 stride 1
+  int64_t list_off[PX_MAXQ][PX_MAXT]; // entry offset of list (q, t)
+  int32_t V[PX_MAXQ], off[PX_MAXQ];
+  // device arrays
+  int32_t *L;          // [Q][T] list lengths
+  int32_t *bstart;     // [Q][T][PX_MAXD + 2] bucket starts by usage
+  int32_t *bucket;     // [entries] ranks ordered by (usage, rank)
+  int32_t *ecap;       // [entries][VM] capacity vector in fill (slot) order
+  uint8_t *ecnt;       // [entries][16] counts in caller's variant order
+  int32_t *esum;       // [entries]
+};
+
+// ------------------------------------------------------------- lists ----
+__global__ void k_fact_lists(const __grid_constant__ FactLayout f, const int32_t *__restrict__ P,
+                             const int32_t *__restrict__ slot_of, int M) {
+  const int id = blockIdx.x * blockDim.x + threadIdx.x;
+  if (id >= f.Q * f.T) return;
+  const int q = id / f.T, t = id % f.T;
+  const int V = f.V[q], N = f.Nt[t];
+  const int64_t base = f.list_off[q][t];
+  int feas[PX_MAXV], capv[PX_MAXV], jof[PX_MAXV];
+  for (int v = 0; v < V; v++) {
+    const int m = f.off[q] + v;
+    capv[v] = P[t * M + m];
+    feas[v] = capv[v] > 0;
+    jof[v] = slot_of[m] - q * f.VM;
+  }
+  int n[PX_MAXV];
+  for (int v = 0; v < V; v++) n[v] = 0;
+  int cnt_by_sum[PX_MAXD + 2];
+  for (int u = 0; u <= N + 1; u++) cnt_by_sum[u] = 0;
+  int r = 0, sum = 0;
+  for (;;) {
+    // emit entry r
+    int32_t *cap = f.ecap + (base + r) * f.VM;
+    for (int j = 0; j < f.VM; j++) cap[j] = 0;
+    for (int v = 0; v < V; v++) {
+      cap[jof[v]] = n[v] * capv[v];
+      f.ecnt[(base + r) * 16 + v] = (uint8_t)n[v];
+    }
+    for (int v = V; v < 16; v++) f.ecnt[(base + r) * 16 + v] = 0;
+    f.esum[base + r] = sum;
+    cnt_by_sum[sum]++;
+    r++;
+    // lexicographic successor: rightmost feasible position that can grow,
+    // later positions reset to 0
+    int i = V - 1;
+    for (; i >= 0; i--) {
+      if (!feas[i]) continue;
+      int pre = 0;
+      for (int k = 0; k < i; k++) pre += n[k];
+      if (pre + n[i] + 1 <= N) break;
+    }
+    if (i < 0) break;
+    n[i]++;
+    for (int k = i + 1; k < V; k++) n[k] = 0;
+    sum = 0;
+    for (int k = 0; k < V; k++) sum += n[k];
+  }
+  f.L[id] = r;
+  int32_t *bs = f.bstart + (size_t)id * (PX_MAXD + 2);
+  int acc = 0;
+  for (int u = 0; u <= N; u++) { bs[u] = acc; acc += cnt_by_sum[u]; }
+  bs[N + 1] = acc;
+  for (int u = 0; u <= N; u++) cnt_by_sum[u] = bs[u];
+  for (int k = 0; k < r; k++) f.bucket[base + cnt_by_sum[f.esum[base + k]]++] = k;
+}
+
+// ----------------------------------------------------------------- g ----
+__device__ __forceinline__ void warp_best_f(uint64_t &s, uint64_t &i) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    uint64_t s2 = __shfl_xor_sync(0xffffffffu, s, o);
+    uint64_t i2 = __shfl_xor_sync(0xffffffffu, i, o);
+    if (px_better(s2, i2, s, i)) { s = s2; i = i2; }
+  }
+}
+
+__global__ void __launch_bounds__(FG_WARPS * 32) k_fact_g(const __grid_constant__ FactLayout f, int n_vec,
+                                                          const int32_t *__restrict__ demand,
+                                                          const int32_t *__restrict__ slot_acc, BestRec *g) {
+  const int lane = threadIdx.x & 31;
+  const int64_t item = (int64_t)blockIdx.x * FG_WARPS + (threadIdx.x >> 5);
+  const int64_t nitems = (int64_t)n_vec * f.Q * f.U;
+  if (item >= nitems) return;
+  const int ukey = (int)(item % f.U);
+  const int q = (int)((item / f.U) % f.Q);
+  const int vec = (int)(item / ((int64_t)f.U * f.Q));
+  const int T = f.T, VM = f.VM;
+  int bsz[PX_MAXT], bst[PX_MAXT];
+  int64_t lstride[PX_MAXT];
+  int64_t prod = 1;
+  {
+    int64_t ls = 1;
+    for (int t = T - 1; t >= 0; t--) {
+      const int ut = (ukey / f.ustride[t]) % (f.Nt[t] + 1);
+      const int32_t *bs = f.bstart + ((size_t)q * T + t) * (PX_MAXD + 2);
+      bst[t] = bs[ut];
+      bsz[t] = bs[ut + 1] - bs[ut];
+      prod *= bsz[t];
+      lstride[t] = ls;
+      ls *= f.L[q * T + t];
+    }
+  }
+  const int s = demand[(size_t)vec * f.Q + q];
+  uint64_t best_s = 0, best_i = ~0ull;
+  for (int64_t k = lane; k < prod; k += 32) {
+    int64_t x = k;
+    int cap[PX_MAXV];
+    for (int j = 0; j < VM; j++) cap[j] = 0;
+    uint64_t sub = 0;
+    for (int t = T - 1; t >= 0; t--) {
+      const int o = (int)(x % bsz[t]);
+      x /= bsz[t];
+      const int r = f.bucket[f.list_off[q][t] + bst[t] + o];
+      sub += (uint64_t)r * lstride[t];
+      const int32_t *ec = f.ecap + (f.list_off[q][t] + r) * VM;
+      for (int j = 0; j < VM; j++) cap[j] += ec[j];
+    }
+    int rem = s;
+    uint64_t acc = 0;
+    for (int j = 0; j < VM; j++) {
+      const int tk = min(rem, cap[j]);
+      acc += (uint64_t)(uint32_t)slot_acc[q * VM + j] * (uint32_t)tk;
+      rem -= tk;
+    }
+    const uint64_t sc = px_pack((uint32_t)(s - rem), acc);
+    if (px_better(sc, sub, best_s, best_i)) { best_s = sc; best_i = sub; }
+  }
+  warp_best_f(best_s, best_i);
+  if (lane == 0) {
+    BestRec &o = g[item];
+    o.score = best_s;
+    o.index = best_i;  // ~0 when no count vector has this usage
+  }
+}
+
+// ---------------------------------------------------------------- DP ----
+__device__ __forceinline__ void ukey_decode(const FactLayout &f, int key, int *u) {
+  for (int t = 0; t < f.T; t++) u[t] = (key / f.ustride[t]) % (f.Nt[t] + 1);
+}
+
+__global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ FactLayout f,
+                                                         const BestRec *__restrict__ g, uint64_t *Gbuf,
+                                                         const int32_t *__restrict__ demand,
+                                                         const int32_t *__restrict__ dev_type, int D,
+                                                         const int32_t *__restrict__ Pdev, int K,
+                                                         const int32_t *__restrict__ slot_code,
+                                                         const int32_t *__restrict__ slot_acc, SolRec *out) {
+  const int vec = blockIdx.x;
+  const int Q = f.Q, U = f.U, T = f.T;
+  const BestRec *gv = g + (size_t)vec * Q * U;
+  uint64_t *G = Gbuf + (size_t)vec * (Q + 1) * U;
+  for (int b = threadIdx.x; b < U; b += blockDim.x) G[(size_t)Q * U + b] = 0;
+  __syncthreads();
+  for (int q = Q - 1; q >= 0; q--) {
+    for (int b = threadIdx.x; b < U; b += blockDim.x) {
+      int bv[PX_MAXT], u[PX_MAXT];
+      ukey_decode(f, b, bv);
+      for (int t = 0; t < T; t++) u[t] = 0;
+      uint64_t best = 0;
+      bool have = false;
+      for (;;) {
+        int uk = 0, rk = 0;
+        for (int t = 0; t < T; t++) { uk += u[t] * f.ustride[t]; rk += (bv[t] - u[t]) * f.ustride[t]; }
+        const BestRec e = gv[(size_t)q * U + uk];
+        if (e.index != ~0ull) {
+          const uint64_t c = e.score + G[(size_t)(q + 1) * U + rk];
+          if (!have || c > best) { best = c; have = true; }
+        }
+        int t = T - 1;
+        for (; t >= 0; t--) {
+          if (++u[t] <= bv[t]) break;
+          u[t] = 0;
+        }
+        if (t < 0) break;
+      }
+      G[(size_t)q * U + b] = best;
+    }
+    __syncthreads();
+  }
+  // reconstruction (warp 0): lexicographically smallest count tensor
+  __shared__ uint64_t pick_sub[PX_MAXQ];
+  __shared__ int pick_u[PX_MAXQ];
+  if (threadIdx.x < 32) {
+    const int lane = threadIdx.x;
+    int bv[PX_MAXT];
+    for (int t = 0; t < T; t++) bv[t] = f.Nt[t];
+    for (int q = 0; q < Q; q++) {
+      int bkey = 0, box = 1;
+      for (int t = 0; t < T; t++) { bkey += bv[t] * f.ustride[t]; box *= bv[t] + 1; }
+      const uint64_t target = G[(size_t)q * U + bkey];
+      uint64_t bsub = ~0ull;
+      uint64_t bu = 0;
+      for (int i = lane; i < box; i += 32) {
+        int x = i, uk = 0, rk = 0;
+        for (int t = T - 1; t >= 0; t--) {
+          const int ut = x % (bv[t] + 1);
+          x /= bv[t] + 1;
+          uk += ut * f.ustride[t];
+          rk += (bv[t] - ut) * f.ustride[t];
+        }
+        const BestRec e = gv[(size_t)q * U + uk];
+        if (e.index == ~0ull) continue;
+        if (e.score + G[(size_t)(q + 1) * U + rk] == target && e.index < bsub) { bsub = e.index; bu = (uint64_t)uk; }
+      }
+      for (int o = 16; o; o >>= 1) {
+        const uint64_t s2 = __shfl_xor_sync(0xffffffffu, bsub, o), u2 = __shfl_xor_sync(0xffffffffu, bu, o);
+        if (s2 < bsub) { bsub = s2; bu = u2; }
+      }
+      if (lane == 0) { pick_sub[q] = bsub; pick_u[q] = (int)bu; }
+      int uu[PX_MAXT];
+      ukey_decode(f, (int)bu, uu);
+      for (int t = 0; t < T; t++) bv[t] -= uu[t];
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  // materialise (a9): family q's pick is the mixed-radix number of its
+  // per-type lexicographic ranks (type 0 most significant)
+  SolRec &r = out[vec];
+  int status = 0;
+  for (int q = 0; q < Q; q++)
+    if (pick_sub[q] == ~0ull) status = 2;
+  for (int d = 0; d < D; d++) { r.option[d] = 0; r.z[d] = 0; }
+  for (int t = 0; t < T && !status; t++) {
+    int d = 0;
+    for (int q = 0; q < Q; q++) {
+      uint64_t ls = 1;
+      for (int t2 = T - 1; t2 > t; t2--) ls *= (uint64_t)f.L[q * T + t2];
+      const int rk = (int)((pick_sub[q] / ls) % (uint64_t)f.L[q * T + t]);
+      const uint8_t *ec = f.ecnt + (f.list_off[q][t] + rk) * 16;
+      for (int v = 0; v < f.V[q]; v++)
+        for (int k = 0; k < ec[v]; k++) {
+          while (d < D && dev_type[d] != t) d++;
+          if (d >= D) { status = 3; break; }
+          r.option[d] = 1 + f.off[q] + v;
+          d++;
+        }
+    }
+  }
+  int64_t served = 0, accsum = 0, stot = 0;
+  uint64_t score = 0;
+  const int32_t *s = demand + (size_t)vec * Q;
+  for (int q = 0; q < Q; q++) {
+    int rem = s[q];
+    uint64_t acc = 0;
+    stot += s[q];
+    for (int j = 0; j < f.VM; j++) {
+      const int code = slot_code[q * f.VM + j];
+      if (!code) continue;
+      const int A = slot_acc[q * f.VM + j];
+      for (int d = 0; d < D; d++) {
+        if (r.option[d] != code) continue;
+        const int tk = min(rem, Pdev[d * K + code]);
+        r.z[d] = tk;
+        rem -= tk;
+        acc += (uint64_t)A * (uint64_t)tk;
+      }
+    }
+    served += s[q] - rem;
+    accsum += (int64_t)acc;
+    score += px_pack((uint32_t)(s[q] - rem), acc);
+  }
+  if (score != G[U - 1]) status = status ? status : 1;
+  uint64_t ncand = 0;
+  for (int q = 0; q < Q; q++) {
+    uint64_t p = 1;
+    for (int t = 0; t < T; t++) p *= (uint64_t)f.L[q * T + t];
+    ncand += p;
+  }
+  r.score = score;
+  r.index = ~0ull;
+  r.served = served;
+  r.unmet = stot - served;
+  r.accsum = accsum;
+  r.eff = served > 0 ? (int32_t)(accsum / served) : 0;
+  r.n_candidates = ncand;
+  r.status = status;
+}
+
+// -------------------------------------------------------------- host ----
+int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32_t *h_dev_type,
+                      const int32_t *d_dev, const int32_t *d_demand, int VM, const Tables &tab, const std::vector<int32_t> &h_P,
+                      SolRec *d_sol) {
+  (void)h_P;
+  const int Q = ctx->Q, T = ctx->T, D = a->D, K = 1 + ctx->M;
+  FactLayout f;
+  memset(&f, 0, sizeof f);
+  f.Q = Q; f.T = T; f.VM = VM;
+  for (int d = 0; d < D; d++) f.Nt[h_dev_type[d]]++;
+  int64_t U = 1;
+  for (int t = T - 1; t >= 0; t--) { f.ustride[t] = (int32_t)U; U *= f.Nt[t] + 1; }
+  if (U > (1 << 22)) return px_fail(ctx, PROTEUS_ERANGE, "usage lattice %lld too large", (long long)U);
+  f.U = (int32_t)U;
+  // list capacity: count vectors with sum <= N_t over V_q variants (before pruning)
+  int64_t total = 0;
+  for (int q = 0; q < Q; q++) {
+    f.V[q] = ctx->V[q];
+    f.off[q] = ctx->off[q];
+    for (int t = 0; t < T; t++) {
+      unsigned __int128 c = 1;
+      for (int i = 1; i <= ctx->V[q]; i++) c = c * (unsigned)(f.Nt[t] + i) / (unsigned)i;
+      if (c > (1u << 24)) return px_fail(ctx, PROTEUS_ERANGE, "count-vector list too large");
+      f.list_off[q][t] = total;
+      total += (int64_t)c;
+    }
+  }
+  if (total > (1ll << 26)) return px_fail(ctx, PROTEUS_ERANGE, "count-vector lists too large");
+  const size_t szL = (size_t)Q * T * 4, szB = (size_t)Q * T * (PX_MAXD + 2) * 4;
+  const size_t szE = (size_t)total * (4 + (size_t)VM * 4 + 16 + 4);
+  char *buf = (char *)px_buf(ctx, B_FACT0, szL + szB + szE + 64);
+  if (!buf) return px_fail(ctx, PROTEUS_ENOMEM, "factored tables");
+  f.L = (int32_t *)buf; buf += szL;
+  f.bstart = (int32_t *)buf; buf += szB;
+  f.bucket = (int32_t *)buf; buf += (size_t)total * 4;
+  f.ecap = (int32_t *)buf; buf += (size_t)total * VM * 4;
+  f.esum = (int32_t *)buf; buf += (size_t)total * 4;
+  f.ecnt = (uint8_t *)buf;
+  const int n_vec = a->n_vec;
+  BestRec *g = (BestRec *)px_buf(ctx, B_FACT1, sizeof(BestRec) * (size_t)n_vec * Q * U);
+  uint64_t *G = (uint64_t *)px_buf(ctx, B_FACT2, 8 * (size_t)n_vec * (Q + 1) * U);
+  if (!g || !G) return px_fail(ctx, PROTEUS_ENOMEM, "factored DP buffers");
+  PX_LAUNCH(ctx, "fact_lists", k_fact_lists, (Q * T + 63) / 64, 64, 0, f, tab.P, tab.slot_of, ctx->M);
+  const int64_t nitems = (int64_t)n_vec * Q * U;
+  PX_LAUNCH(ctx, "fact_g", k_fact_g, (unsigned)((nitems + FG_WARPS - 1) / FG_WARPS), FG_WARPS * 32, 0, f, n_vec,
+            d_demand, tab.slot_acc, g);
+  PX_LAUNCH(ctx, "fact_dp", k_fact_dp, n_vec, DP_THREADS, 0, f, g, G, d_demand, d_dev, D, tab.Pdev, K,
+            tab.slot_code, tab.slot_acc, d_sol);
+  return 0;
+}

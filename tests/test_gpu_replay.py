@@ -1,0 +1,105 @@
+"""GPU parity of proteus_replay against the oracle's event-driven simulator:
+every per-query latency bit-exact, and the per-scenario aggregates."""
+
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def px():
+    from paper_conf_asplos_ahmadgfwsw24_b200 import Proteus
+    return Proteus(0)
+
+
+def _alloc(oracle_mod, cfg, v=0):
+    prof, cl = cfg["prof"], cfg["cluster"]
+    return oracle_mod.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][v], 2)
+
+
+def _compare(px, oracle_mod, prof, cl, option, z, demand, arr, fam, sc):
+    px.load_profiles(prof)
+    g = px.replay(arr, fam, option, z, cl.device_type, demand, cl.slo_us, sc)
+    o = oracle_mod.replay(prof, cl.device_type, option, z, demand, cl.slo_us, arr, fam, sc)
+    for s in range(len(sc)):
+        if not np.array_equal(g["latency"][s], o["latency"][s]):
+            bad = np.nonzero(g["latency"][s] != o["latency"][s])[0]
+            raise AssertionError(f"scenario {sc[s]}: {len(bad)} latencies differ, first at {bad[0]}: "
+                                 f"gpu {g['latency'][s][bad[0]]} oracle {o['latency'][s][bad[0]]}")
+    for k in ("violations", "on_time", "acc_sum"):
+        assert np.array_equal(g[k], o[k]), k
+    return g
+
+
+@pytest.mark.parametrize("kind", ["poisson", "gamma", "uniform"])
+def test_replay_small_all_scenarios(px, oracle_mod, kind):
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    r = _alloc(oracle_mod, cfg, 0)
+    rate = float(cfg["demand"][0].sum())
+    arr, fam = W.query_trace(60_000, rate, cfg["weights"], 9, kind)
+    for routing in (0, 1):
+        _compare(px, oracle_mod, cfg["prof"], cfg["cluster"], r["option"], r["z"], cfg["demand"][0], arr, fam,
+                 W.scenarios_64(routing))
+
+
+def test_replay_overload_with_sink(px, oracle_mod):
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    r = _alloc(oracle_mod, cfg, 1)
+    assert r["unmet"] > 0
+    arr, fam = W.query_trace(80_000, float(cfg["demand"][1].sum()), cfg["weights"], 10, "gamma")
+    g = _compare(px, oracle_mod, cfg["prof"], cfg["cluster"], r["option"], r["z"], cfg["demand"][1], arr, fam,
+                 W.scenarios_64(0))
+    assert np.all(g["violations"] + g["on_time"] == len(arr))
+
+
+def test_replay_edge_cases(px, oracle_mod):
+    from paper_conf_asplos_ahmadgfwsw24_b200 import ProteusError, workloads as W
+    cfg = W.config("c3")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    r = _alloc(oracle_mod, cfg, 0)
+    sc = np.array([[1000, 0, 0], [2000, 1, 0], [1500, 4, 1]], np.int32)
+    # empty trace
+    px.load_profiles(prof)
+    g = px.replay(np.zeros(0, np.uint32), np.zeros(0, np.uint8), r["option"], r["z"], cl.device_type,
+                  cfg["demand"][0], cl.slo_us, sc)
+    assert g["latency"].shape == (3, 0) and g["violations"].sum() == 0
+    # one query; all simultaneous; ragged sizes around the 1024-query tiles
+    for n in (1, 31, 1023, 1025, 4097):
+        arr = np.sort(np.random.default_rng(n).integers(0, 2_000, size=n)).astype(np.uint32)
+        fam = np.random.default_rng(n + 1).integers(0, prof.Q, size=n).astype(np.uint8)
+        _compare(px, oracle_mod, prof, cl, r["option"], r["z"], cfg["demand"][0], arr, fam, sc)
+    arr = np.zeros(500, np.uint32)
+    fam = np.zeros(500, np.uint8)
+    _compare(px, oracle_mod, prof, cl, r["option"], r["z"], cfg["demand"][0], arr, fam, sc)
+    # all demand zero -> everything of a routed family goes to the sink
+    _compare(px, oracle_mod, prof, cl, r["option"], np.zeros_like(r["z"]), np.zeros(prof.Q, np.int32),
+             np.arange(100, dtype=np.uint32), np.zeros(100, np.uint8), sc)
+    # unsorted timestamps -> ERANGE
+    with pytest.raises(ProteusError) as e:
+        px.replay(np.array([5, 3], np.uint32), np.zeros(2, np.uint8), r["option"], r["z"], cl.device_type,
+                  cfg["demand"][0], cl.slo_us, sc)
+    assert e.value.code == -5
+
+
+def test_replay_c5_full_size(px, oracle_mod):
+    """Config 5 at full size: 10M Poisson queries x 64 scenarios on the c3
+    allocation, latencies written to HBM in the bench's launch configuration;
+    compared with the oracle on every query of every scenario."""
+    import torch
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c5")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    r = oracle_mod.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][0], 2)
+    arr, fam, sc = cfg["arrival_us"], cfg["family"], cfg["scenarios"]
+    px.load_profiles(prof)
+    lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
+    g = px.replay(torch.from_numpy(arr).cuda(), torch.from_numpy(fam).cuda(), r["option"], r["z"], cl.device_type,
+                  cfg["demand"][0], cl.slo_us, sc, latency=lat)
+    o = oracle_mod.replay(prof, cl.device_type, r["option"], r["z"], cfg["demand"][0], cl.slo_us, arr, fam, sc)
+    for k in ("violations", "on_time", "acc_sum"):
+        assert np.array_equal(g[k], o[k]), k
+    glat = lat.cpu().numpy()
+    assert np.array_equal(glat, o["latency"])

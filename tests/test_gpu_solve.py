@@ -1,0 +1,204 @@
+"""GPU parity of proteus_solve against the oracle (bit-exact: every quantity is
+an integer).  Compared per demand vector: packed score, served, unmet, accsum,
+effective accuracy, the canonical index (modes 0/1), the placement and z.
+Where several placements are optimal the canonical tie-break (reading C9)
+makes the answer unique; independently, the GPU's placement is re-scored by
+the oracle (catches decode bugs regardless of tie-breaking)."""
+
+import numpy as np
+import pytest
+
+from tests._util import golden, packed_score, profiles_from_capacity, random_instance
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def px():
+    from paper_conf_asplos_ahmadgfwsw24_b200 import Proteus
+    return Proteus(0)
+
+
+def check(px, oracle_mod, prof, dev, slo, demand, mode, generic=False, threads=0):
+    px.load_profiles(prof)
+    dem = np.atleast_2d(np.asarray(demand, np.int32))
+    sols = px.solve(dev, slo, dem, mode=mode, generic=generic)
+    for v, sol in enumerate(sols):
+        r = oracle_mod.solve(prof, dev, slo, dem[v], mode, threads=threads)
+        got = (sol.served, sol.unmet, sol.accsum, sol.eff_acc_micro)
+        assert got == (r["served"], r["unmet"], r["accsum"], r["eff"]), (mode, v, got, r)
+        assert sol.score == packed_score(r["served"], r["accsum"])
+        if mode in (0, 1):
+            assert sol.index == r["index"], (mode, sol.index, r["index"])
+            assert sol.n_candidates == r["n_candidates"]
+        assert sol.option.tolist() == r["option"].tolist(), (mode, sol.option, r["option"])
+        assert sol.z.tolist() == r["z"].tolist()
+        chk = oracle_mod.score_placement(prof, dev, slo, dem[v], sol.option)
+        assert (chk["served"], chk["accsum"]) == (sol.served, sol.accsum)
+        assert chk["z"].tolist() == sol.z.tolist()
+    return sols
+
+
+def test_golden_h1_g1(px, oracle_mod):
+    from paper_conf_asplos_ahmadgfwsw24_b200.workloads import Profiles
+    g = golden()
+    h = g["H1"]
+    prof = Profiles(T=1, Q=1, V=np.array(h["V"], np.int32), acc_micro=np.array(h["acc_micro"], np.int32), bmax=1,
+                    lat_us=np.array(h["lat_us"], np.int32))
+    px.load_profiles(prof)
+    for c in h["cases"]:
+        for generic in (False, True):
+            s = px.solve(h["device_type"], h["slo_us"], c["s"], mode=0, generic=generic)[0]
+            assert (s.index, s.served, s.accsum, s.eff_acc_micro) == (c["index"], c["served"], c["accsum"], c["eff"])
+            assert s.option.tolist() == c["option"] and s.z.tolist() == c["z"]
+    G = g["G1"]
+    prof = profiles_from_capacity(G["P"], G["acc_micro"], G["V"])
+    px.load_profiles(prof)
+    for c in G["cases"]:
+        for generic in (False, True):
+            s = px.solve(G["device_type"], G["slo_us"], c["s"], mode=0, generic=generic)[0]
+            assert (s.index, s.served, s.accsum, s.eff_acc_micro) == (c["index"], c["served"], c["accsum"], c["eff"])
+            assert s.option.tolist() == c["option"] and s.z.tolist() == c["z"]
+            if "score_hex" in c:
+                assert s.score == int(c["score_hex"], 16)
+        if "multiset_index" in c:
+            assert px.solve(G["device_type"], G["slo_us"], c["s"], mode=1)[0].index == c["multiset_index"]
+
+
+@pytest.mark.parametrize("total", [600, 1200, 0, 17])
+def test_c1_all_modes(px, oracle_mod, total):
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c1", total=total)
+    prof, cl = cfg["prof"], cfg["cluster"]
+    for mode, generic in ((0, False), (0, True), (1, False), (2, False)):
+        check(px, oracle_mod, prof, cl.device_type, cl.slo_us, cfg["demand"], mode, generic)
+
+
+def test_random_small_instances(px, oracle_mod):
+    """Random toys incl. tied accuracies, unsorted variant order, P = 0 holes,
+    zero demand, D from 1 to 6, 1-4 families."""
+    rng = np.random.default_rng(1234)
+    for trial in range(60):
+        T = int(rng.integers(1, 4))
+        Q = int(rng.integers(1, 5))
+        D = int(rng.integers(1, 7))
+        prof, dev, slo, P = random_instance(rng, T=T, Q=Q, Vmax=3, D=D, Pmax=40, tie_acc=trial % 3 == 0)
+        if trial % 4 == 1:  # unsorted accuracy order inside families
+            prof.acc_micro = prof.acc_micro[::-1].copy()
+            prof.V = prof.V[::-1].copy()
+        s = rng.integers(0, 80, size=(2, prof.Q)).astype(np.int32)
+        for mode, generic in ((0, False), (0, True), (1, False), (2, False)):
+            check(px, oracle_mod, prof, dev, slo, s, mode, generic, threads=2)
+
+
+def test_c2_flat_full(px, oracle_mod):
+    """Config 2 at full size (13^8 = 815 730 721 candidates), both demand
+    vectors, specialised kernel; oracle = exhaustive enumeration."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c2")
+    sols = check(px, oracle_mod, cfg["prof"], cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"], 0)
+    assert sols[0].n_candidates == 13**8
+    assert sols[1].unmet > 0
+
+
+def test_c2_generic_kernel_and_multiset(px, oracle_mod):
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c2")
+    args = (cfg["prof"], cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"])
+    a = check(px, oracle_mod, *args, 0, generic=True)
+    b = check(px, oracle_mod, *args, 1)
+    c = check(px, oracle_mod, *args, 2)
+    for x, y, z in zip(a, b, c):
+        assert x.score == y.score == z.score  # invariant (iii)
+
+
+def test_c2_sharded_identical(px, oracle_mod):
+    """Index-range shards (as on 1/2/4/8 GPUs) combined by the slot order give
+    the single-GPU result."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    from paper_conf_asplos_ahmadgfwsw24_b200.dist import pick_best, slot_vector
+    cfg = W.config("c2")
+    px.load_profiles(cfg["prof"])
+    dev, slo, dem = cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"][0]
+    full = px.solve(dev, slo, dem, mode=0)[0]
+    for world in (2, 3, 8):
+        slots = sum(slot_vector(r, world, s.score, s.index)
+                    for r in range(world) for s in [px.solve(dev, slo, dem, mode=0, shard_rank=r, shard_world=world)[0]])
+        s, i, _ = pick_best(slots)
+        assert (s, i) == (full.score, full.index)
+        m = px.materialize(dev, slo, dem, i)
+        assert m.option.tolist() == full.option.tolist() and m.z.tolist() == full.z.tolist()
+
+
+def test_c3_factored(px, oracle_mod):
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    sols = check(px, oracle_mod, cfg["prof"], cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"], 2)
+    assert sols[0].unmet == 0 and sols[1].unmet > 0
+
+
+def test_c3mini_multiset_vs_factored(px, oracle_mod):
+    """c3-mini: flat multiset over the 20-device cluster (1.146e9 candidates)
+    = factored optimum (invariant iii); both modes bit-exact vs the oracle."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3mini")
+    args = (cfg["prof"], cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"])
+    f = check(px, oracle_mod, *args, 2)
+    m = check(px, oracle_mod, *args, 1)
+    assert m[0].n_candidates == 286 * 2002 * 2002
+    for x, y in zip(f, m):
+        assert x.score == y.score
+
+
+def test_c4_batched_resolve_sample(px, oracle_mod):
+    """All 3600 per-second vectors in one call; a seeded sample of 12 checked
+    against the oracle one by one, plus every vector's reported value checked
+    by re-scoring its placement."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c4")
+    prof, cl, dem = cfg["prof"], cfg["cluster"], cfg["demand"]
+    px.load_profiles(prof)
+    sols = px.solve(cl.device_type, cl.slo_us, dem, mode=2)
+    assert len(sols) == 3600
+    rng = np.random.default_rng(404)
+    for v in sorted(rng.choice(3600, size=12, replace=False)):
+        r = oracle_mod.solve(prof, cl.device_type, cl.slo_us, dem[v], 2)
+        s = sols[v]
+        assert (s.served, s.accsum, s.unmet) == (r["served"], r["accsum"], r["unmet"])
+        assert s.option.tolist() == r["option"].tolist() and s.z.tolist() == r["z"].tolist()
+    for v in range(0, 3600, 7):
+        chk = oracle_mod.score_placement(prof, cl.device_type, cl.slo_us, dem[v], sols[v].option)
+        assert (chk["served"], chk["accsum"]) == (sols[v].served, sols[v].accsum)
+    assert any(s.unmet > 0 for s in sols) and any(s.unmet == 0 for s in sols)
+
+
+def test_errors(px):
+    from paper_conf_asplos_ahmadgfwsw24_b200 import ProteusError, workloads as W
+    from paper_conf_asplos_ahmadgfwsw24_b200._native import PROTEUS_EINVAL, PROTEUS_ERANGE
+    cfg = W.config("c2")
+    px.load_profiles(cfg["prof"])
+    dev, slo = cfg["cluster"].device_type, cfg["cluster"].slo_us
+    with pytest.raises(ProteusError) as e:
+        px.solve(dev, slo, cfg["demand"][0], mode=0, max_candidates=10**6)
+    assert e.value.code == PROTEUS_ERANGE
+    with pytest.raises(ProteusError) as e:
+        px.solve(dev, slo, np.full(4, 2**21, np.int32), mode=2)
+    assert e.value.code == PROTEUS_ERANGE
+    with pytest.raises(ProteusError) as e:
+        px.solve(np.full(8, 7, np.int32), slo, cfg["demand"][0], mode=2)
+    assert e.value.code == PROTEUS_EINVAL
+    assert px.candidate_count(dev, 0) == 13**8
+    assert px.candidate_count(dev, 1) == 91 * 455 * 455
+
+
+def test_device_pointer_inputs(px, oracle_mod):
+    """torch CUDA tensors as inputs (the in-HBM path the bench times)."""
+    import torch
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c1")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    host = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=0)[0]
+    t = lambda a: torch.as_tensor(np.asarray(a, np.int32)).cuda()
+    dev = px.solve(t(cl.device_type), t(cl.slo_us), t(cfg["demand"]), mode=0)[0]
+    assert (dev.score, dev.index, dev.option.tolist()) == (host.score, host.index, host.option.tolist())
