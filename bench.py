@@ -1,0 +1,405 @@
+#!/usr/bin/env python
+"""Benchmark of the Proteus hot path on B200 (contract: see DESIGN.md §6).
+
+Headline (the JSON line's metric/value): allocations scored per second on
+BASELINE.json configs[1] -- config c2, 4 families x 3 variants on 8
+heterogeneous devices (2 CPU-like, 3 GPU-A, 3 GPU-B), exhaustive flat
+mixed-radix search over 13^8 = 815 730 721 candidates, demand vector 0
+(rho ~ 0.5).  One step = one proteus_solve over the whole index space (on N
+GPUs: each rank its contiguous slice + one NCCL slot all-reduce + the winner's
+materialisation), inputs resident in HBM.  The same run also measures, as
+`extra`, the other two parts of BASELINE.json's metric: the per-second
+re-solve of the paper-scale cluster (c4, 3600 demand vectors, factored search)
+and the adaptive-batching replay (c5, 10M queries x 64 scenarios).
+
+--impl reference times the CPU oracle (oracle/, test infrastructure) on the
+same workload: the paper ships no code, so the oracle is the reference arm.
+"""
+
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+SM_COUNT = 148
+INT_LANES_PER_SM_CLK = 128   # 4 SMSPs x 1 warp-instruction/clk x 32 lanes
+SM_MAX_MHZ_FALLBACK = 1965.0
+WORKLOAD = ("c2: exhaustive flat mixed-radix allocation search, 4 families x 3 variants on 8 devices "
+            "(types cpu x2, gpu_a x3, gpu_b x3), 13^8 = 815730721 candidates, demand vector rho~0.5 (seed 202)")
+
+
+def env_int(name, default):
+    try:
+        return int(os.environ.get(name, default))
+    except ValueError:
+        return default
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f), "measured"
+    return {"hbm_gbs": 6650.0, "sm_max_mhz": SM_MAX_MHZ_FALLBACK}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 8:
+                self.rows.append(parts)
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[4 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# algorithmic int32 ops of the pair-incremental scoring
+def flat_pair_ops_per_candidate(Q, V, K):
+    S = Q * V
+    fill = 3 * V + 2
+    per_prefix = (S                       # add device D-3's capacity
+                  + Q * fill              # family values of the prefix
+                  + 2 * S * (fill + 2)    # deltas of the last two devices
+                  + Q * V * V * (fill + 4)  # joint fills when both host one family
+                  + K * K * 4)            # 64-bit add + compare per candidate
+    return per_prefix / (K * K)
+
+
+def oracle_cpu_baseline(cfg, vec=0):
+    import oracle
+    prof, cl = cfg["prof"], cfg["cluster"]
+    cores = len(os.sched_getaffinity(0))
+    t0 = time.perf_counter()
+    r = oracle.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][vec], 0, threads=cores)
+    dt = time.perf_counter() - t0
+    return r, dt, cores
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    import oracle
+    oracle.build()
+    cfg = W.config("c2")
+    for _ in range(args.warmup):
+        pass  # the oracle has no warm-up state; warm-up steps are skipped to bound the run time
+    times = []
+    r = None
+    for _ in range(args.steps):
+        r, dt, cores = oracle_cpu_baseline(cfg)
+        times.append(dt)
+    total = sum(times)
+    value = r["n_candidates"] * args.steps / total
+    line = {
+        "impl": "reference", "metric": "allocations scored/s", "value": value, "unit": "candidates/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / args.steps,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic",
+        "config": {"workload": WORKLOAD},
+        "cpu_baseline": {"value": value, "unit": "candidates/s", "cores": cores, "kind": "oracle",
+                         "sample": "full c2 search (815730721 candidates, vector 0) per step, exhaustive "
+                                   "enumeration + memoised vertex-enumeration LP per family"},
+        "e2e": {"value": value, "unit": "candidates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-extra", action="store_true", help="skip the c4/c5 measurements")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_asplos_ahmadgfwsw24_b200 import Proteus, workloads as W
+    from paper_conf_asplos_ahmadgfwsw24_b200.dist import allreduce_best
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    args.warmup = max(args.warmup, 3)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    px = Proteus(local)
+    stream = torch.cuda.current_stream(dev)
+    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)  # > 126 MB L2
+
+    # ------------------------------------------------------------ c2 --
+    cfg = W.config("c2")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    t_dev = torch.as_tensor(cl.device_type, dtype=torch.int32, device=dev)
+    t_slo = torch.as_tensor(cl.slo_us, dtype=torch.int32, device=dev)
+    t_dem = torch.as_tensor(cfg["demand"][:1], dtype=torch.int32, device=dev)
+
+    def step():
+        loc = px.solve(t_dev, t_slo, t_dem, mode=0, shard_rank=rank, shard_world=world)[0]
+        if world > 1:
+            s, i, _ = allreduce_best(loc.score, loc.index, None, dev)
+            return px.materialize(t_dev, t_slo, t_dem, i, mode=0), loc
+        return loc, loc
+
+    for _ in range(args.warmup):
+        step()
+    sol_ref = step()[0]
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    px.set_timing(True)
+    kern_ms = []
+    launches0 = px.launch_count()
+    wall = []
+    with ClockSampler(local) as clk:
+        for k in range(args.steps):
+            flush.zero_()
+            barrier()
+            t0 = time.perf_counter()
+            ev[k][0].record(stream)
+            sol, loc = step()
+            ev[k][1].record(stream)
+            barrier()
+            wall.append(time.perf_counter() - t0)
+            kern_ms += [ms for name, ms in px.kernel_times() if name == "score_flat_pair"]
+            assert sol.score == sol_ref.score and sol.index == sol_ref.index
+    launches = px.launch_count() - launches0
+    px.set_timing(False)
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    total_ms = max_over_ranks(sum(step_ms))
+    ms_per_step = total_ms / args.steps
+    n_cand = 13**8
+    value = n_cand / (ms_per_step / 1e3)
+    clocks = clk.summary()
+    # roofline of the dominant kernel (score_flat_pair)
+    peaks, peak_src = measured_peaks()
+    k_ms = statistics.mean(kern_ms) if kern_ms else float("nan")
+    cand_per_launch = loc.n_candidates
+    ops = flat_pair_ops_per_candidate(4, 3, 13) * cand_per_launch
+    sm_mhz = clocks["sm_mhz"] or peaks.get("sm_max_mhz", SM_MAX_MHZ_FALLBACK)
+    peak_ops = SM_COUNT * INT_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12
+    achieved = ops / (k_ms / 1e3) / 1e12
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            traffic = json.load(f).get("score_flat_pair")
+
+    # e2e: the same solve through the public API with HOST buffers
+    e2e_t = []
+    for _ in range(max(3, args.steps // 2)):
+        flush.zero_()
+        barrier()
+        t0 = time.perf_counter()
+        loc = px.solve(cl.device_type, cl.slo_us, cfg["demand"][:1], mode=0, shard_rank=rank, shard_world=world)[0]
+        if world > 1:
+            s, i, _ = allreduce_best(loc.score, loc.index, None, dev)
+            px.materialize(cl.device_type, cl.slo_us, cfg["demand"][:1], i, mode=0)
+        barrier()
+        e2e_t.append(time.perf_counter() - t0)
+    e2e_s = max_over_ranks(statistics.median(e2e_t))
+    h2d = cl.device_type.nbytes + cl.slo_us.nbytes + cfg["demand"][:1].nbytes
+    d2h = 2 * 4 * len(cl.device_type) + 64
+    time_to_opt_ms = max_over_ranks(statistics.median(wall)) * 1e3
+
+    line = {
+        "metric": "allocations scored/s", "value": value, "unit": "candidates/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "int32/int64 (exact integer)", "data": "synthetic",
+        "config": {"workload": WORKLOAD, "l2": "flushed (256 MB write) before every timed step",
+                   "parallelism": f"index-range shards x{world}, NCCL slot all-reduce" if world > 1 else "1 GPU"},
+        "roofline": {"kernel": "score_flat_pair", "bound": "alu", "achieved": achieved, "peak": peak_ops,
+                     "unit": "Tops/s (int32 lane-ops)", "frac": achieved / peak_ops, "traffic": traffic,
+                     "kernel_ms": k_ms, "ops_per_candidate": flat_pair_ops_per_candidate(4, 3, 13),
+                     "peak_basis": f"148 SMs x 128 int32 lane-ops/clk x {sm_mhz:.0f} MHz (median SM clock "
+                                   f"during the run; DESIGN.md §5)"},
+        "e2e": {"value": n_cand / e2e_s, "unit": "candidates/s", "h2d_bytes_per_step": int(h2d),
+                "d2h_bytes_per_step": int(d2h)},
+        "gpu_launches": int(sum_over_ranks(launches)),
+        "clocks": clocks,
+        "time_to_optimal_ms": time_to_opt_ms,
+        "result": {"score": sol.score, "index": sol.index, "served": sol.served, "unmet": sol.unmet,
+                   "eff_acc_micro": sol.eff_acc_micro},
+    }
+
+    # ---------------------------------------------------------- extra --
+    if not args.no_extra:
+        line["extra"] = extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, peaks, peak_src)
+
+    if rank == 0 and not args.no_cpu_baseline and world == 1:
+        r, dt, cores = oracle_cpu_baseline(cfg)
+        assert r["index"] == sol.index and r["served"] == sol.served and r["accsum"] == sol.accsum
+        line["cpu_baseline"] = {"value": r["n_candidates"] / dt, "unit": "candidates/s", "cores": cores,
+                                "kind": "oracle",
+                                "sample": "the full c2 search, vector 0 (815730721 candidates), exhaustive "
+                                          "enumeration + memoised vertex-enumeration LP; same answer as the GPU"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, peaks, peak_src):
+    import torch
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    from paper_conf_asplos_ahmadgfwsw24_b200.dist import shard_range
+    out = {}
+    stream = torch.cuda.current_stream(dev)
+    # c4: per-second re-solve of the paper-scale cluster, 3600 vectors (weak: vectors split by rank)
+    cfg = W.config("c4")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    lo, hi = shard_range(len(cfg["demand"]), rank, world)
+    t_dev = torch.as_tensor(cl.device_type, dtype=torch.int32, device=dev)
+    t_slo = torch.as_tensor(cl.slo_us, dtype=torch.int32, device=dev)
+    t_dem = torch.as_tensor(cfg["demand"][lo:hi], dtype=torch.int32, device=dev)
+    t_one = torch.as_tensor(cfg["demand"][:1], dtype=torch.int32, device=dev)
+    for _ in range(2):
+        px.solve(t_dev, t_slo, t_dem, mode=2)
+    ts = []
+    for _ in range(3):
+        flush.zero_()
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        sols = px.solve(t_dev, t_slo, t_dem, mode=2)
+        b.record(stream)
+        barrier()
+        ts.append(a.elapsed_time(b))
+    ms = max_over_ranks(statistics.median(ts))
+    one = []
+    for _ in range(5):
+        barrier()
+        t0 = time.perf_counter()
+        px.solve(t_dev, t_slo, t_one, mode=2)
+        one.append((time.perf_counter() - t0) * 1e3)
+    out["c4_resolve"] = {
+        "vectors": len(cfg["demand"]), "ms_all_vectors": ms, "ms_per_vector_batched": ms / max(1, hi - lo),
+        "single_vector_time_to_optimal_ms": statistics.median(one),
+        "subplacements_per_vector": sols[0].n_candidates if sols else 0,
+        "subplacements_per_s": (len(cfg["demand"]) * (sols[0].n_candidates if sols else 0)) / (ms / 1e3),
+        "scaling": "weak (vectors split by rank)"}
+    # c5: replay 10M queries x 64 scenarios (scenarios on every rank; N>1 = replicas)
+    cfg = W.config("c5")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    alloc = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=2)[0]
+    arr = torch.from_numpy(cfg["arrival_us"]).to(dev)
+    fam = torch.from_numpy(cfg["family"]).to(dev)
+    sc = cfg["scenarios"]
+    S, N = len(sc), len(cfg["arrival_us"])
+    lat = torch.empty((S, N), dtype=torch.uint32, device=dev)
+    for _ in range(2):
+        px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
+    px.set_timing(True)
+    ts, lane_ms = [], []
+    for _ in range(3):
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        res = px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
+        b.record(stream)
+        barrier()
+        ts.append(a.elapsed_time(b))
+        kt = px.kernel_times()
+        lane_ms.append(sum(ms for n, ms in kt if n == "replay_lanes"))
+        route_ms = sum(ms for n, ms in kt if n.startswith("route"))
+    px.set_timing(False)
+    ms = max_over_ranks(statistics.median(ts))
+    lane = statistics.median(lane_ms)
+    alg_bytes = N * S * 4 + N * 8   # latency writes + one read of the per-device arrays
+    hbm = peaks.get("hbm_gbs", 6650.0)
+    # e2e with host buffers: H2D of the trace, D2H of all latencies
+    arr_h, fam_h = cfg["arrival_us"], cfg["family"]
+    barrier()
+    t0 = time.perf_counter()
+    px.replay(arr_h, fam_h, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=True)
+    e2e = time.perf_counter() - t0
+    out["c5_replay"] = {
+        "queries": N, "scenarios": S, "ms": ms, "query_scenarios_per_s": N * S / (ms / 1e3),
+        "routing_ms": route_ms, "lane_kernel_ms": lane,
+        "roofline": {"kernel": "replay_lanes", "bound": "hbm", "achieved": alg_bytes / (lane / 1e3) / 1e9,
+                     "peak": hbm, "unit": "GB/s", "frac": alg_bytes / (lane / 1e3) / 1e9 / hbm,
+                     "peak_source": peak_src, "alg_bytes": alg_bytes},
+        "violations_first_scenarios": [int(x) for x in res["violations"][:4]],
+        "e2e": {"value": N * S / e2e, "unit": "query-scenarios/s", "h2d_bytes_per_step": int(N * 5),
+                "d2h_bytes_per_step": int(N * S * 4)},
+        "scaling": "replicas" if world > 1 else "1 GPU"}
+    return out
+
+
+if __name__ == "__main__":
+    main()

@@ -15,6 +15,9 @@
 // time t = max(F, a[h]) with q queued (capped at Bmax), dispatch Bmax when
 // q >= Bmax; otherwise with W = a[h] + SLO - T(q+1) dispatch q once t >= W,
 // else move t to the next arrival if it comes by W (Case 2), else to W (Case 1).
+#include <cstdlib>
+#include <cstring>
+
 #include "internal.cuh"
 
 #define TILE 1024
@@ -120,6 +123,7 @@ __global__ void k_tile_scan(const int32_t *__restrict__ hist, int64_t ntiles, in
     int64_t acc = 0;
     for (int i = 0; i < (int)blockDim.x; i++) { int64_t v = part[i]; part[i] = acc; acc += v; }
     totals[key] = acc;
+    base[ntiles * nkeys + key] = (int32_t)acc;  // row ntiles: totals
   }
   __syncthreads();
   int64_t acc = part[threadIdx.x];
@@ -291,25 +295,310 @@ __global__ void k_sink(const proteus_scenario *__restrict__ sc, int S, int D, in
   }
 }
 
+// ------------------------------------------------------ chunked lanes ----
+// Phase A (k_spec): the device arrays are cut at global windows of win_tiles
+// routing tiles; every (window, device, scenario) lane replays its piece
+// speculatively from an idle device (the true state at the start of the trace,
+// R13).  Every query of the window gets a latency and the window's output rows
+// are written by one CTA (full L2 sectors).  The lane's exit state (the first
+// batch head at or after the window end and the device free time) is kept.
+// Phase B (k_stitch): one warp per (scenario, device) carries the true state
+// across windows.  A window whose speculative start matches the true state is
+// correct as is; otherwise the true run is replayed until it meets the
+// speculative run in the same state (same next head, same free time) -- from
+// there the two are identical -- rewriting latencies and count deltas on the
+// way.  Backlogged stretches (>= Bmax queued at every completion) are jumped
+// 32 batches at a time: batch k of such a stretch is exactly the next Bmax
+// queries, finishing at F + (k+1) T(Bmax).
+struct SpecExit {
+  int64_t F;
+  int32_t ov;  // exit head - window end (the last batch's overhang)
+  int32_t pad;
+};
+
+struct ChunkArgs {
+  int S, D, M, bmax, nsc, win_tiles, nwin;
+  int64_t N, ntiles;
+  const int32_t *option, *dev_type, *fam_of_m, *acc, *lat, *slo_base, *sc_list;
+  const proteus_scenario *sc;
+  const int64_t *devOff;   // [D + 2]
+  const int32_t *devBase;  // [ntiles + 1][D + 1]
+  const uint32_t *devArr, *devIdx;
+  uint32_t *lat_out;       // [S][N]
+  uint64_t *agg;           // [3][S]
+  SpecExit *ex;            // [S][D][nwin]
+};
+
+struct LaneP {
+  int Bmax;
+  int64_t L;
+  uint32_t A;
+};
+
+__device__ __forceinline__ LaneP lane_params(const ChunkArgs &a, int s, int d, const int32_t *T) {
+  LaneP p;
+  const int m = a.option[d] - 1;
+  int depth = 0;
+  while (depth < a.bmax && T[depth] > 0) depth++;
+  const proteus_scenario sc = a.sc[s];
+  p.Bmax = (sc.batch_cap > 0 && sc.batch_cap < depth) ? sc.batch_cap : depth;
+  p.L = (int64_t)sc.slo_mult_milli * a.slo_base[a.fam_of_m[m]] / 1000;
+  p.A = (uint32_t)a.acc[m];
+  return p;
+}
+
+// one decision of the §5 rule from head h with the device free at F over
+// arr[0, n): returns the batch size, *t = dispatch time
+__device__ __forceinline__ int decide(const uint32_t *arr, int64_t n, int64_t h, int64_t F, int Bmax, int64_t L,
+                                      const int32_t *T, int64_t *t_out) {
+  const int64_t ah = arr[h];
+  int64_t t = F > ah ? F : ah;
+  int q = 1;
+  while (q < Bmax && h + q < n && (int64_t)arr[h + q] <= t) q++;
+  int b;
+  for (;;) {
+    if (q >= Bmax) { b = Bmax; break; }
+    const int64_t W = ah + L - T[q];  // Tmax_wait(q+1) = Texp(1) - Tprocess(q+1)
+    if (t >= W) { b = q; break; }
+    if (h + q < n && (int64_t)arr[h + q] <= W) {  // Case 2: the (q+1)-st query comes by W
+      t = arr[h + q];
+      while (q < Bmax && h + q < n && (int64_t)arr[h + q] <= t) q++;
+      continue;
+    }
+    t = W;  // Case 1: start at Tmax_wait(q+1)
+    b = q;
+    break;
+  }
+  *t_out = t;
+  return b;
+}
+
+__device__ __forceinline__ uint32_t sat_lat(int64_t l) { return l >= 0xFFFFFFFFll ? 0xFFFFFFFEu : (uint32_t)l; }
+
+__global__ void k_spec(const __grid_constant__ ChunkArgs a) {
+  extern __shared__ uint32_t sm[];
+  __shared__ int sOff[33], sStage[32];
+  __shared__ unsigned long long sCnt[32][3];
+  const int c = blockIdx.x, sg = blockIdx.y, dg = blockIdx.z;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  const int d = dg * 32 + w;
+  const int64_t tile0 = (int64_t)c * a.win_tiles;
+  const int64_t tile1 = tile0 + a.win_tiles < a.ntiles ? tile0 + a.win_tiles : a.ntiles;
+  int32_t *sT = (int32_t *)sm;                // [nw][bmax]
+  uint32_t *sA = sm + (size_t)nw * a.bmax;    // staged arrivals
+  const bool dvalid = d < a.D;
+  const int64_t n_d = dvalid ? a.devOff[d + 1] - a.devOff[d] : 0;
+  const int64_t st = dvalid ? a.devBase[tile0 * (a.D + 1) + d] : 0;
+  const int64_t en = dvalid ? a.devBase[tile1 * (a.D + 1) + d] : 0;
+  const int64_t len = en - st;
+  const bool host = dvalid && a.option[d] > 0;
+  int64_t look = n_d - en < a.bmax ? n_d - en : a.bmax;
+  const int stage = host ? (int)(len + look) : 0;
+  if (lane == 0) sStage[w] = stage;
+  if (threadIdx.x < 32) { sCnt[threadIdx.x][0] = 0; sCnt[threadIdx.x][1] = 0; sCnt[threadIdx.x][2] = 0; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int acc = 0;
+    for (int k = 0; k < nw; k++) { sOff[k] = acc; acc += sStage[k]; }
+    sOff[nw] = acc;
+  }
+  __syncthreads();
+  uint32_t *arr = sA + sOff[w];
+  if (host) {
+    const uint32_t *src = a.devArr + a.devOff[d] + st;
+    for (int i = lane; i < stage; i += 32) arr[i] = src[i];
+  }
+  const int32_t *T = sT + w * a.bmax;
+  if (host) {
+    const int32_t *row = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+    for (int i = lane; i < a.bmax; i += 32) sT[w * a.bmax + i] = row[i];
+  }
+  __syncthreads();
+  const int si = sg * 32 + lane;
+  if (host && len > 0 && si < a.nsc) {
+    const int s = a.sc_list[si];
+    const LaneP p = lane_params(a, s, d, T);
+    const uint32_t *ix = a.devIdx + a.devOff[d] + st;
+    uint32_t *out = a.lat_out + (size_t)s * a.N;
+    unsigned long long viol = 0, ont = 0, accs = 0;
+    int64_t h = 0, F = 0;
+    if (p.Bmax < 1) {
+      for (int64_t j = 0; j < len; j++) out[ix[j]] = 0xFFFFFFFFu;
+      viol = (unsigned long long)len;
+      h = len;
+    } else {
+      while (h < len) {
+        int64_t t;
+        const int b = decide(arr, stage, h, F, p.Bmax, p.L, T, &t);
+        F = t + T[b - 1];
+        const int64_t jend = h + b < len ? h + b : len;
+        for (int64_t j = h; j < jend; j++) {
+          const uint32_t l = sat_lat(F - (int64_t)arr[j]);
+          out[ix[j]] = l;
+          if ((int64_t)l > p.L) viol++;
+          else { ont++; accs += p.A; }
+        }
+        h += b;
+      }
+    }
+    SpecExit e;
+    e.F = F;
+    e.ov = (int32_t)(h - len);
+    e.pad = 0;
+    a.ex[((size_t)s * a.D + d) * a.nwin + c] = e;
+    atomicAdd(&sCnt[lane][0], viol);
+    atomicAdd(&sCnt[lane][1], ont);
+    atomicAdd(&sCnt[lane][2], accs);
+  }
+  __syncthreads();
+  if (threadIdx.x < 32 && sg * 32 + (int)threadIdx.x < a.nsc) {
+    const int s = a.sc_list[sg * 32 + threadIdx.x];
+    if (sCnt[threadIdx.x][0]) atomicAdd((unsigned long long *)&a.agg[s], sCnt[threadIdx.x][0]);
+    if (sCnt[threadIdx.x][1]) atomicAdd((unsigned long long *)&a.agg[a.S + s], sCnt[threadIdx.x][1]);
+    if (sCnt[threadIdx.x][2]) atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], sCnt[threadIdx.x][2]);
+  }
+}
+
+struct Delta {
+  long long viol, ont, accs;
+};
+
+// rewrite latencies of device-relative queries [lo, hi) of one batch finishing at F (warp-cooperative)
+__device__ __forceinline__ void rewrite_const(const uint32_t *arr, const uint32_t *ix, uint32_t *out, int64_t lo,
+                                              int64_t hi, int64_t F, const LaneP &p, Delta &dl, int lane) {
+  for (int64_t j = lo + lane; j < hi; j += 32) {
+    const uint32_t nl = sat_lat(F - (int64_t)arr[j]);
+    const uint32_t g = ix[j];
+    const uint32_t ol = out[g];
+    out[g] = nl;
+    const int nv = (int64_t)nl > p.L, ov = (int64_t)ol > p.L;
+    dl.viol += nv - ov;
+    dl.ont += (1 - nv) - (1 - ov);
+    dl.accs += ((long long)(1 - nv) - (long long)(1 - ov)) * (long long)p.A;
+  }
+}
+
+__global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ ChunkArgs a) {
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = (int64_t)blockIdx.x * 4 + (threadIdx.x >> 5);
+  if (gw >= (int64_t)a.nsc * a.D) return;
+  const int si = (int)(gw / a.D), d = (int)(gw % a.D);
+  const int s = a.sc_list[si];
+  if (a.option[d] <= 0 || a.nwin < 2) return;
+  const int64_t n_d = a.devOff[d + 1] - a.devOff[d];
+  if (n_d == 0) return;
+  const uint32_t *arr = a.devArr + a.devOff[d], *ix = a.devIdx + a.devOff[d];
+  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  const LaneP p = lane_params(a, s, d, T);
+  if (p.Bmax < 1) return;
+  uint32_t *out = a.lat_out + (size_t)s * a.N;
+  const SpecExit *ex = a.ex + ((size_t)s * a.D + d) * a.nwin;
+  auto win_start = [&](int c) -> int64_t {
+    const int64_t t = (int64_t)c * a.win_tiles < a.ntiles ? (int64_t)c * a.win_tiles : a.ntiles;
+    return a.devBase[t * (a.D + 1) + d];
+  };
+  Delta dl = {0, 0, 0};
+  int64_t h = win_start(1) + ex[0].ov, F = ex[0].F;
+  const int64_t TB = T[p.Bmax - 1];
+  for (int c = 1; c < a.nwin; c++) {
+    const int64_t st = win_start(c), en = win_start(c + 1);
+    if (en == st) continue;
+    if (h > st) rewrite_const(arr, ix, out, st, h < en ? h : en, F, p, dl, lane);  // overhang of the last batch
+    if (h >= en) continue;
+    if (h == st && F <= (int64_t)arr[st]) {  // the speculative start was the true state
+      h = en + ex[c].ov;
+      F = ex[c].F;
+      continue;
+    }
+    while (h < en) {
+      // backlogged stretch: >= Bmax queued at completion -> full batches back to back
+      if (F > (int64_t)arr[h] && h + p.Bmax - 1 < n_d && (int64_t)arr[h + p.Bmax - 1] <= F) {
+        const int64_t kmax = (en - h + p.Bmax - 1) / p.Bmax;
+        const int64_t idx = h + (int64_t)(lane + 1) * p.Bmax - 1;
+        const bool ok = lane < kmax && idx < n_d && (int64_t)arr[idx] <= F + (int64_t)lane * TB;
+        const unsigned bal = __ballot_sync(0xffffffffu, ok);
+        const int r = bal == 0xffffffffu ? 32 : __ffs(~bal) - 1;
+        const int64_t nq = (int64_t)r * p.Bmax;
+        for (int64_t i = lane; i < nq; i += 32) {
+          const int64_t k = i / p.Bmax, j = h + i;
+          const uint32_t nl = sat_lat(F + (k + 1) * TB - (int64_t)arr[j]);
+          const uint32_t g = ix[j];
+          const uint32_t ol = out[g];
+          out[g] = nl;
+          const int nv = (int64_t)nl > p.L, ov = (int64_t)ol > p.L;
+          dl.viol += nv - ov;
+          dl.ont += ov - nv;
+          dl.accs += ((long long)ov - (long long)nv) * (long long)p.A;
+        }
+        h += nq;
+        F += (int64_t)r * TB;
+        continue;
+      }
+      int64_t t;
+      const int b = decide(arr, n_d, h, F, p.Bmax, p.L, T, &t);
+      const int64_t Fn = t + T[b - 1];
+      const int64_t j2 = h + b;
+      bool conv;
+      if (j2 < en) {
+        const int64_t f1 = (int64_t)arr[j2 - 1] + out[ix[j2 - 1]], f2 = (int64_t)arr[j2] + out[ix[j2]];
+        conv = f1 == Fn && f2 != Fn;
+      } else {
+        conv = j2 == en + ex[c].ov && Fn == ex[c].F;
+      }
+      __syncwarp();
+      rewrite_const(arr, ix, out, h, j2 < en ? j2 : en, Fn, p, dl, lane);
+      h = j2;
+      F = Fn;
+      if (conv && h < en) {
+        h = en + ex[c].ov;
+        F = ex[c].F;
+        break;
+      }
+    }
+  }
+  for (int o = 16; o; o >>= 1) {
+    dl.viol += __shfl_xor_sync(0xffffffffu, dl.viol, o);
+    dl.ont += __shfl_xor_sync(0xffffffffu, dl.ont, o);
+    dl.accs += __shfl_xor_sync(0xffffffffu, dl.accs, o);
+  }
+  if (lane == 0) {
+    if (dl.viol) atomicAdd((unsigned long long *)&a.agg[s], (unsigned long long)dl.viol);
+    if (dl.ont) atomicAdd((unsigned long long *)&a.agg[a.S + s], (unsigned long long)dl.ont);
+    if (dl.accs) atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], (unsigned long long)dl.accs);
+  }
+}
+
 // ---------------------------------------------------------------- host ----
+static int env_int(const char *name, int dflt) {
+  const char *v = getenv(name);
+  return v && *v ? atoi(v) : dflt;
+}
+
 int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int64_t N, const int32_t *h_option,
               const int32_t *h_z, const int32_t *h_dev_type, int D, const int32_t *h_demand, const int32_t *h_slo,
               const proteus_scenario *h_sc, int S, uint32_t *d_lat_out, uint64_t *d_agg) {
   const int Q = ctx->Q, M = ctx->M;
   PX_CUDA(ctx, cudaMemsetAsync(d_agg, 0, ((size_t)3 * S + 1) * 8, ctx->stream));
-  // small inputs: option, z, dev_type, demand, slo, scenarios
-  const size_t small = (size_t)(4 * D + 2 * Q) * 4 + (size_t)S * sizeof(proteus_scenario) + 64;
+  // small inputs: option, z, dev_type, demand, slo, scenarios, scenario lists
+  const size_t small = (size_t)(4 * D + 2 * Q + 2 * PX_MAXQ + 8 + 2 * S) * 4 + (size_t)S * sizeof(proteus_scenario);
   char *sb = (char *)px_buf(ctx, B_R_MISC, small + 4096);
   if (!sb) return px_fail(ctx, PROTEUS_ENOMEM, "replay scratch");
   int32_t *d_opt = (int32_t *)sb, *d_z = d_opt + D, *d_dev = d_z + D, *d_dem = d_dev + D, *d_slo = d_dem + Q;
   int32_t *d_pat_off = d_slo + Q, *d_pat_len = d_pat_off + PX_MAXQ;
   uint32_t *d_flags = (uint32_t *)(d_pat_len + PX_MAXQ);
-  proteus_scenario *d_sc = (proteus_scenario *)(((uintptr_t)(d_flags + 4) + 15) & ~(uintptr_t)15);
+  int32_t *d_scl = (int32_t *)(d_flags + 8);  // [2][S] scenario lists per routing mode
+  proteus_scenario *d_sc = (proteus_scenario *)(((uintptr_t)(d_scl + 2 * S) + 15) & ~(uintptr_t)15);
+  std::vector<int32_t> scl[2];
+  for (int s = 0; s < S; s++) scl[h_sc[s].routing].push_back(s);
+  std::vector<int32_t> scl_all(2 * S, 0);
+  for (int rt = 0; rt < 2; rt++)
+    for (size_t k = 0; k < scl[rt].size(); k++) scl_all[rt * S + k] = scl[rt][k];
   PX_CUDA(ctx, cudaMemcpyAsync(d_opt, h_option, D * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_z, h_z, D * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_dev, h_dev_type, D * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_dem, h_demand, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_slo, h_slo, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_scl, scl_all.data(), 2 * S * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_sc, h_sc, S * sizeof(proteus_scenario), cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemsetAsync(d_flags, 0, 4, ctx->stream));
   if (N > 0) {
@@ -325,46 +614,81 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   int64_t dsum = 0;
   for (int q = 0; q < Q; q++) dsum += h_demand[q];
   const size_t pat_cap = (size_t)dsum + (size_t)Q * D + 16;
-  bool used[2] = {false, false};
-  for (int s = 0; s < S; s++) used[h_sc[s].routing] = true;
   const int64_t *devOff[2] = {nullptr, nullptr};
+  const int32_t *devBase[2] = {nullptr, nullptr};
   const uint32_t *devArr[2] = {nullptr, nullptr}, *devIdx[2] = {nullptr, nullptr};
   for (int rt = 0; rt < 2; rt++) {
-    if (!used[rt]) continue;
+    if (scl[rt].empty()) continue;
     uint8_t *pat = (uint8_t *)px_buf(ctx, B_R_PAT, pat_cap);
     int32_t *hist = (int32_t *)px_buf(ctx, B_R_HIST, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
-    int32_t *base = (int32_t *)px_buf(ctx, B_R_BASE, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
+    int32_t *fbase = (int32_t *)px_buf(ctx, B_R_BASE, (size_t)(ntiles + 1) * (PX_MAXQ + 2) * 4);
+    int32_t *dbase = (int32_t *)px_buf(ctx, rt ? B_R_DBASE1 : B_R_DBASE0, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
     uint8_t *tgt = (uint8_t *)px_buf(ctx, B_R_TGT, (size_t)N + 16);
     int64_t *off = (int64_t *)px_buf(ctx, rt ? B_R_OFF1 : B_R_OFF, (size_t)2 * (PX_MAXD + 2) * 8);
     uint32_t *darr = (uint32_t *)px_buf(ctx, rt ? B_R_DEVARR1 : B_R_DEVARR, (size_t)N * 4 + 16);
     uint32_t *didx = (uint32_t *)px_buf(ctx, rt ? B_R_DEVIDX1 : B_R_DEVIDX, (size_t)N * 4 + 16);
-    if (!pat || !hist || !base || !tgt || !off || !darr || !didx) return px_fail(ctx, PROTEUS_ENOMEM, "routing buffers");
+    if (!pat || !hist || !fbase || !dbase || !tgt || !off || !darr || !didx)
+      return px_fail(ctx, PROTEUS_ENOMEM, "routing buffers");
     int64_t *totals = off + (PX_MAXD + 2);
     PX_LAUNCH(ctx, "route_prepare", k_route_prepare, 1, 32, 0, rt, Q, D, M, ctx->bmax, d_opt, d_z, d_dev, d_dem,
               ctx->d_fam, ctx->d_lat, pat, d_pat_off, d_pat_len);
     if (N > 0) {
       PX_LAUNCH(ctx, "route_count", k_tile_count, tblocks, TILE_WARPS * 32, 0, d_fam, N, Q, hist);
-      PX_LAUNCH(ctx, "route_scan", k_tile_scan, Q, 1024, 0, hist, ntiles, Q, base, totals);
-      PX_LAUNCH(ctx, "route_target", k_route_target, tblocks, TILE_WARPS * 32, 0, d_fam, N, Q, base, pat, d_pat_off,
+      PX_LAUNCH(ctx, "route_scan", k_tile_scan, Q, 1024, 0, hist, ntiles, Q, fbase, totals);
+      PX_LAUNCH(ctx, "route_target", k_route_target, tblocks, TILE_WARPS * 32, 0, d_fam, N, Q, fbase, pat, d_pat_off,
                 d_pat_len, D, tgt, hist);
-      PX_LAUNCH(ctx, "route_scan_dev", k_tile_scan, D + 1, 1024, 0, hist, ntiles, D + 1, base, totals);
+      PX_LAUNCH(ctx, "route_scan_dev", k_tile_scan, D + 1, 1024, 0, hist, ntiles, D + 1, dbase, totals);
       PX_LAUNCH(ctx, "route_offsets", k_dev_offsets, 1, 32, 0, totals, D + 1, off);
-      PX_LAUNCH(ctx, "route_scatter", k_scatter, tblocks, TILE_WARPS * 32, 0, tgt, d_arr, N, D, base, off, darr, didx);
+      PX_LAUNCH(ctx, "route_scatter", k_scatter, tblocks, TILE_WARPS * 32, 0, tgt, d_arr, N, D, dbase, off, darr,
+                didx);
     } else {
       PX_CUDA(ctx, cudaMemsetAsync(off, 0, (size_t)(PX_MAXD + 2) * 8, ctx->stream));
     }
-    devOff[rt] = off; devArr[rt] = darr; devIdx[rt] = didx;
+    devOff[rt] = off; devArr[rt] = darr; devIdx[rt] = didx; devBase[rt] = dbase;
   }
   if (N == 0) return 0;
-  LaneArgs la;
-  la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.N = N;
-  la.option = d_opt; la.dev_type = d_dev; la.fam_of_m = ctx->d_fam; la.acc = ctx->d_acc; la.lat = ctx->d_lat;
-  la.slo_base = d_slo; la.sc = d_sc;
-  for (int rt = 0; rt < 2; rt++) { la.devOff[rt] = devOff[rt]; la.devArr[rt] = devArr[rt]; la.devIdx[rt] = devIdx[rt]; }
-  la.lat_out = d_lat_out;
-  la.agg = d_agg;
-  const int nl = S * D;
-  PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
+  // latencies are needed by the stitch even when the caller does not want them
+  uint32_t *lat = d_lat_out;
+  if (!lat) {
+    lat = (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S * N * 4);
+    if (!lat) return px_fail(ctx, PROTEUS_ENOMEM, "latency scratch");
+  }
+  const int win_tiles = env_int("PROTEUS_REPLAY_WIN_TILES", 4);
+  const int nwin = (int)((ntiles + win_tiles - 1) / win_tiles);
+  const int ndg = (D + 31) / 32;
+  const int dpb = D < 32 ? D : 32;
+  const size_t smem = ((size_t)dpb * ctx->bmax + (size_t)win_tiles * TILE + (size_t)dpb * ctx->bmax) * 4;
+  const bool simple = env_int("PROTEUS_REPLAY_SIMPLE", 0) != 0 || smem > 200 * 1024;
+  if (simple) {
+    LaneArgs la;
+    la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.N = N;
+    la.option = d_opt; la.dev_type = d_dev; la.fam_of_m = ctx->d_fam; la.acc = ctx->d_acc; la.lat = ctx->d_lat;
+    la.slo_base = d_slo; la.sc = d_sc;
+    for (int rt = 0; rt < 2; rt++) { la.devOff[rt] = devOff[rt]; la.devArr[rt] = devArr[rt]; la.devIdx[rt] = devIdx[rt]; }
+    la.lat_out = d_lat_out;
+    la.agg = d_agg;
+    const int nl = S * D;
+    PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
+  } else {
+    SpecExit *ex = (SpecExit *)px_buf(ctx, B_R_LANE, sizeof(SpecExit) * (size_t)S * D * nwin);
+    if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
+    if (smem > 48 * 1024) PX_CUDA(ctx, cudaFuncSetAttribute(k_spec, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    for (int rt = 0; rt < 2; rt++) {
+      if (scl[rt].empty()) continue;
+      ChunkArgs ca;
+      memset(&ca, 0, sizeof ca);
+      ca.S = S; ca.D = D; ca.M = M; ca.bmax = ctx->bmax; ca.nsc = (int)scl[rt].size();
+      ca.win_tiles = win_tiles; ca.nwin = nwin; ca.N = N; ca.ntiles = ntiles;
+      ca.option = d_opt; ca.dev_type = d_dev; ca.fam_of_m = ctx->d_fam; ca.acc = ctx->d_acc; ca.lat = ctx->d_lat;
+      ca.slo_base = d_slo; ca.sc_list = d_scl + rt * S; ca.sc = d_sc;
+      ca.devOff = devOff[rt]; ca.devBase = devBase[rt]; ca.devArr = devArr[rt]; ca.devIdx = devIdx[rt];
+      ca.lat_out = lat; ca.agg = d_agg; ca.ex = ex;
+      dim3 grid(nwin, (ca.nsc + 31) / 32, ndg);
+      PX_LAUNCH(ctx, "replay_spec", k_spec, grid, dpb * 32, smem, ca);
+      const int64_t warps = (int64_t)ca.nsc * D;
+      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 0, ca);
+    }
+  }
   dim3 g(64, S < 65535 ? S : 65535);
   PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, d_sc, S, D, N, devOff[0] ? devOff[0] : devOff[1],
             devIdx[0] ? devIdx[0] : devIdx[1], devOff[1] ? devOff[1] : devOff[0], devIdx[1] ? devIdx[1] : devIdx[0],

@@ -239,7 +239,8 @@ def config(name: str, **kw) -> dict:
         fams = C3_FAMILIES if name == "c3" else C3MINI_FAMILIES
         prof = make_profiles(303, ("cpu", "gpu_a", "gpu_b"), fams,
                              n_variants=None if name == "c3" else 3, bmax=64)
-        cl = Cluster(cluster_types(kw.get("counts", (10, 5, 5))), slo_from_cpu_rule(prof))
+        cl = Cluster(cluster_types(kw.get("counts", (10, 5, 5) if name == "c3" else C3MINI_COUNTS)),
+                     slo_from_cpu_rule(prof))
         w = zipf_weights(prof.Q, 303)
         totals = kw.get("totals", C3_TOTALS if name == "c3" else C3MINI_TOTALS)
         dem = np.stack([split_demand(t, w) for t in totals])
@@ -267,6 +268,7 @@ def config(name: str, **kw) -> dict:
 C1_TOTAL = 600
 C2_TOTALS = (3000, 7000)
 C3_TOTALS = (3000, 12000)
-C3MINI_TOTALS = (12000, 60000)
+C3MINI_TOTALS = (8000, 30000)
+C3MINI_COUNTS = (6, 3, 3)   # 12 devices: multiset space 5005 * 220^2 = 2.42e8
 C4_LAM_MID = 2500.0
 C5_RATE = 3000

@@ -1,0 +1,45 @@
+"""One invocation of a hot-path workload, for ncu captures (never timed).
+
+    python scripts/profile_target.py c2      # flat search over 13^8 candidates
+    python scripts/profile_target.py c4      # factored re-solve, 3600 vectors
+    python scripts/profile_target.py c5      # replay 10M queries x 64 scenarios
+"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_asplos_ahmadgfwsw24_b200 import Proteus, workloads as W  # noqa: E402
+
+
+def main(what):
+    px = Proteus(0)
+    if what == "c2":
+        cfg = W.config("c2")
+        px.load_profiles(cfg["prof"])
+        s = px.solve(cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"][:1], mode=0)[0]
+        print("c2", s.index, s.served, s.accsum)
+    elif what == "c4":
+        cfg = W.config("c4")
+        px.load_profiles(cfg["prof"])
+        sols = px.solve(cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"], mode=2)
+        print("c4", len(sols), sum(s.unmet for s in sols))
+    elif what == "c5":
+        cfg = W.config("c5")
+        prof, cl = cfg["prof"], cfg["cluster"]
+        px.load_profiles(prof)
+        a = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=2)[0]
+        arr = torch.from_numpy(cfg["arrival_us"]).cuda()
+        fam = torch.from_numpy(cfg["family"]).cuda()
+        sc = cfg["scenarios"]
+        lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
+        r = px.replay(arr, fam, a.option, a.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
+        print("c5", r["violations"][:8])
+    torch.cuda.synchronize()
+
+
+if __name__ == "__main__":
+    main(sys.argv[1])

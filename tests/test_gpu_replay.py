@@ -32,8 +32,19 @@ def _compare(px, oracle_mod, prof, cl, option, z, demand, arr, fam, sc):
     return g
 
 
+PATHS = {"chunked": {}, "small_windows": {"PROTEUS_REPLAY_WIN_TILES": "1"},
+         "simple": {"PROTEUS_REPLAY_SIMPLE": "1"}}
+
+
+@pytest.mark.parametrize("path", sorted(PATHS))
 @pytest.mark.parametrize("kind", ["poisson", "gamma", "uniform"])
-def test_replay_small_all_scenarios(px, oracle_mod, kind):
+def test_replay_small_all_scenarios(px, oracle_mod, kind, path, monkeypatch):
+    """60k queries x 64 scenarios x both routings; `small_windows` cuts the
+    device arrays every 1024 global queries so the stitch (backlogged jumps,
+    re-walks, convergence) runs at every window; `simple` is one thread per
+    (device, scenario) lane."""
+    for k, v in PATHS[path].items():
+        monkeypatch.setenv(k, v)
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
     cfg = W.config("c3")
     r = _alloc(oracle_mod, cfg, 0)
@@ -44,7 +55,10 @@ def test_replay_small_all_scenarios(px, oracle_mod, kind):
                  W.scenarios_64(routing))
 
 
-def test_replay_overload_with_sink(px, oracle_mod):
+@pytest.mark.parametrize("path", sorted(PATHS))
+def test_replay_overload_with_sink(px, oracle_mod, path, monkeypatch):
+    for k, v in PATHS[path].items():
+        monkeypatch.setenv(k, v)
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
     cfg = W.config("c3")
     r = _alloc(oracle_mod, cfg, 1)

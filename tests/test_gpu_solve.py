@@ -138,16 +138,34 @@ def test_c3_factored(px, oracle_mod):
 
 
 def test_c3mini_multiset_vs_factored(px, oracle_mod):
-    """c3-mini: flat multiset over the 20-device cluster (1.146e9 candidates)
-    = factored optimum (invariant iii); both modes bit-exact vs the oracle."""
+    """c3-mini: flat multiset over a 12-device cluster of the three types
+    (5005 * 220^2 = 2.42e8 candidates) = factored optimum (invariant iii);
+    both modes bit-exact vs the oracle."""
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
     cfg = W.config("c3mini")
     args = (cfg["prof"], cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"])
     f = check(px, oracle_mod, *args, 2)
     m = check(px, oracle_mod, *args, 1)
-    assert m[0].n_candidates == 286 * 2002 * 2002
+    assert m[0].n_candidates == 5005 * 220 * 220
     for x, y in zip(f, m):
         assert x.score == y.score
+
+
+def test_c3mini_20_devices_multiset_full_size(px, oracle_mod):
+    """The same families on the full 20-device cluster: 92378 * 2002^2 =
+    3.7e11 multisets on the GPU (too many for the oracle); property at full
+    size: the multiset optimum equals the factored optimum, which the oracle
+    computes exactly, and the returned placement re-scores to that value."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3mini", counts=(10, 5, 5), totals=(12000,))
+    prof, cl, dem = cfg["prof"], cfg["cluster"], cfg["demand"]
+    px.load_profiles(prof)
+    m = px.solve(cl.device_type, cl.slo_us, dem, mode=1)[0]
+    assert m.n_candidates == 92378 * 2002 * 2002
+    r = oracle_mod.solve(prof, cl.device_type, cl.slo_us, dem[0], 2)
+    assert (m.served, m.accsum) == (r["served"], r["accsum"])
+    chk = oracle_mod.score_placement(prof, cl.device_type, cl.slo_us, dem[0], m.option)
+    assert (chk["served"], chk["accsum"]) == (m.served, m.accsum)
 
 
 def test_c4_batched_resolve_sample(px, oracle_mod):
