@@ -375,8 +375,9 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
         barrier()
         ts.append(a.elapsed_time(b))
         kt = px.kernel_times()
-        lane_ms.append(sum(ms for n, ms in kt if n == "replay_lanes"))
+        lane_ms.append(sum(ms for n, ms in kt if n in ("replay_spec", "replay_stitch", "replay_lanes")))
         route_ms = sum(ms for n, ms in kt if n.startswith("route"))
+        split = {n: ms for n, ms in kt if n in ("replay_spec", "replay_stitch", "replay_lanes")}
     px.set_timing(False)
     ms = max_over_ranks(statistics.median(ts))
     lane = statistics.median(lane_ms)
@@ -390,8 +391,8 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     e2e = time.perf_counter() - t0
     out["c5_replay"] = {
         "queries": N, "scenarios": S, "ms": ms, "query_scenarios_per_s": N * S / (ms / 1e3),
-        "routing_ms": route_ms, "lane_kernel_ms": lane,
-        "roofline": {"kernel": "replay_lanes", "bound": "hbm", "achieved": alg_bytes / (lane / 1e3) / 1e9,
+        "routing_ms": route_ms, "lane_kernels_ms": lane, "lane_kernel_split_ms": split,
+        "roofline": {"kernel": "replay_spec + replay_stitch", "bound": "hbm", "achieved": alg_bytes / (lane / 1e3) / 1e9,
                      "peak": hbm, "unit": "GB/s", "frac": alg_bytes / (lane / 1e3) / 1e9 / hbm,
                      "peak_source": peak_src, "alg_bytes": alg_bytes},
         "violations_first_scenarios": [int(x) for x in res["violations"][:4]],

@@ -10,17 +10,27 @@
 // per-tile counting (warp match + per-tile offsets), then scatters the
 // arrivals into per-device arrays (device-major, arrival order kept).
 //
-// Lane kernel: one thread per (scenario, device) walks the device's arrival
-// array with the §5 rule written as a window walk (readings R1-R5): at decision
-// time t = max(F, a[h]) with q queued (capped at Bmax), dispatch Bmax when
-// q >= Bmax; otherwise with W = a[h] + SLO - T(q+1) dispatch q once t >= W,
-// else move t to the next arrival if it comes by W (Case 2), else to W (Case 1).
+// Lanes: the §5 rule per (device, scenario) written as a window walk
+// (readings R1-R5): at decision time t = max(F, a[h]) with q queued (capped at
+// Bmax), dispatch Bmax when q >= Bmax; otherwise with W = a[h] + SLO - T(q+1)
+// dispatch q once t >= W, else move t to the next arrival if it comes by W
+// (Case 2), else to W (Case 1).  Three executions of that rule:
+//   k_spec   (phase A) every (global window, device, scenario) piece replayed
+//            from an idle device into a shared-memory tile of the window's
+//            output rows, flushed with coalesced stores; exit states kept;
+//   k_stitch (phase B) one warp per (device, scenario) carries the true state
+//            across windows and replays only where the speculative start was
+//            wrong, until the two runs meet (see below);
+//   k_lanes  one thread per (device, scenario) walking everything (fallback,
+//            and the reference formulation in the tests).
+// a13: k_count reduces the final latency rows to per-scenario violations,
+// on-time counts and accuracy sums.
 #include <cstdlib>
 #include <cstring>
 
 #include "internal.cuh"
 
-#define TILE 1024
+#define TILE 512
 #define TILE_WARPS 8
 #define LANE_THREADS 128
 
@@ -207,165 +217,64 @@ __global__ void k_scatter(const uint8_t *__restrict__ target, const uint32_t *__
 }
 
 // --------------------------------------------------------------- lanes ----
-struct LaneArgs {
-  int S, D, M, bmax;
-  int64_t N;
-  const int32_t *option, *dev_type, *fam_of_m, *acc, *lat, *slo_base;
-  const proteus_scenario *sc;
-  const int64_t *devOff[2];
-  const uint32_t *devArr[2], *devIdx[2];
-  uint32_t *lat_out;  // [S][N] or null
-  uint64_t *agg;      // [3][S]
-};
-
-__global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ LaneArgs a) {
-  const int lane_id = blockIdx.x * blockDim.x + threadIdx.x;
-  if (lane_id >= a.S * a.D) return;
-  const int s = lane_id / a.D, d = lane_id % a.D;
-  const int o = a.option[d];
-  if (o <= 0) return;
-  const proteus_scenario sc = a.sc[s];
-  const int rt = sc.routing;
-  const int64_t st = a.devOff[rt][d], n = a.devOff[rt][d + 1] - st;
-  if (n == 0) return;
-  const uint32_t *arr = a.devArr[rt] + st;
-  const uint32_t *idx = a.devIdx[rt] + st;
-  const int m = o - 1;
-  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + m) * a.bmax;  // T[b-1]
-  int depth = 0;
-  while (depth < a.bmax && T[depth] > 0) depth++;
-  const int Bmax = (sc.batch_cap > 0 && sc.batch_cap < depth) ? sc.batch_cap : depth;
-  const int64_t L = (int64_t)sc.slo_mult_milli * a.slo_base[a.fam_of_m[m]] / 1000;
-  const uint32_t A = (uint32_t)a.acc[m];
-  uint64_t viol = 0, ont = 0, accs = 0;
-  if (Bmax < 1) {  // cannot run even batch 1 (routing 1 never routes here; routing 0 has z = 0)
-    viol = (uint64_t)n;
-    if (a.lat_out)
-      for (int64_t j = 0; j < n; j++) a.lat_out[(size_t)s * a.N + idx[j]] = 0xFFFFFFFFu;
-  } else {
-    int64_t h = 0, F = 0;
-    while (h < n) {
-      const int64_t ah = arr[h];
-      int64_t t = F > ah ? F : ah;
-      int q = 1;
-      while (q < Bmax && h + q < n && (int64_t)arr[h + q] <= t) q++;
-      int b;
-      for (;;) {
-        if (q >= Bmax) { b = Bmax; break; }
-        const int64_t W = ah + L - T[q];  // T(q+1)
-        if (t >= W) { b = q; break; }
-        if (h + q < n && (int64_t)arr[h + q] <= W) {
-          t = arr[h + q];
-          while (q < Bmax && h + q < n && (int64_t)arr[h + q] <= t) q++;
-          continue;
-        }
-        t = W;
-        b = q;
-        break;
-      }
-      F = t + T[b - 1];
-      for (int j = 0; j < b; j++) {
-        const int64_t l = F - (int64_t)arr[h + j];
-        const uint32_t lv = l >= 0xFFFFFFFFll ? 0xFFFFFFFEu : (uint32_t)l;
-        if ((int64_t)lv > L) viol++;
-        else { ont++; accs += A; }
-        if (a.lat_out) a.lat_out[(size_t)s * a.N + idx[h + j]] = lv;
-      }
-      h += b;
-    }
-  }
-  atomicAdd((unsigned long long *)&a.agg[s], (unsigned long long)viol);
-  atomicAdd((unsigned long long *)&a.agg[a.S + s], (unsigned long long)ont);
-  atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], (unsigned long long)accs);
-}
-
-// dropped queries (the sink segment, device index D)
-__global__ void k_sink(const proteus_scenario *__restrict__ sc, int S, int D, int64_t N, const int64_t *devOff0,
-                       const uint32_t *devIdx0, const int64_t *devOff1, const uint32_t *devIdx1, uint32_t *lat_out,
-                       uint64_t *agg) {
-  for (int s = blockIdx.y; s < S; s += gridDim.y) {
-    const int rt = sc[s].routing;
-    const int64_t *off = rt ? devOff1 : devOff0;
-    const uint32_t *idx = rt ? devIdx1 : devIdx0;
-    const int64_t st = off[D], n = off[D + 1] - st;
-    if (blockIdx.x == 0 && threadIdx.x == 0 && n) atomicAdd((unsigned long long *)&agg[s], (unsigned long long)n);
-    if (lat_out)
-      for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
-        lat_out[(size_t)s * N + idx[st + j]] = 0xFFFFFFFFu;
-  }
-}
-
-// ------------------------------------------------------ chunked lanes ----
-// Phase A (k_spec): the device arrays are cut at global windows of win_tiles
-// routing tiles; every (window, device, scenario) lane replays its piece
-// speculatively from an idle device (the true state at the start of the trace,
-// R13).  Every query of the window gets a latency and the window's output rows
-// are written by one CTA (full L2 sectors).  The lane's exit state (the first
-// batch head at or after the window end and the device free time) is kept.
-// Phase B (k_stitch): one warp per (scenario, device) carries the true state
-// across windows.  A window whose speculative start matches the true state is
-// correct as is; otherwise the true run is replayed until it meets the
-// speculative run in the same state (same next head, same free time) -- from
-// there the two are identical -- rewriting latencies and count deltas on the
-// way.  Backlogged stretches (>= Bmax queued at every completion) are jumped
-// 32 batches at a time: batch k of such a stretch is exactly the next Bmax
-// queries, finishing at F + (k+1) T(Bmax).
 struct SpecExit {
   int64_t F;
-  int32_t ov;  // exit head - window end (the last batch's overhang)
+  int32_t ov;  // exit head - window end (overhang of the last batch into the next window)
   int32_t pad;
 };
 
-struct ChunkArgs {
-  int S, D, M, bmax, nsc, win_tiles, nwin;
+struct LaneArgs {
+  int S, D, M, bmax, Q;
   int64_t N, ntiles;
-  const int32_t *option, *dev_type, *fam_of_m, *acc, *lat, *slo_base, *sc_list;
+  const int32_t *option, *dev_type, *fam_of_m, *acc, *lat, *slo_base;
   const proteus_scenario *sc;
+  // one routing mode
+  int nsc, win_tiles, nwin, use_tile;
+  const int32_t *sc_list;
   const int64_t *devOff;   // [D + 2]
   const int32_t *devBase;  // [ntiles + 1][D + 1]
   const uint32_t *devArr, *devIdx;
   uint32_t *lat_out;       // [S][N]
-  uint64_t *agg;           // [3][S]
   SpecExit *ex;            // [S][D][nwin]
 };
 
 struct LaneP {
   int Bmax;
   int64_t L;
-  uint32_t A;
 };
 
-__device__ __forceinline__ LaneP lane_params(const ChunkArgs &a, int s, int d, const int32_t *T) {
-  LaneP p;
-  const int m = a.option[d] - 1;
+__device__ __forceinline__ LaneP lane_params(const LaneArgs &a, int s, int d, const int32_t *T) {
   int depth = 0;
   while (depth < a.bmax && T[depth] > 0) depth++;
   const proteus_scenario sc = a.sc[s];
-  p.Bmax = (sc.batch_cap > 0 && sc.batch_cap < depth) ? sc.batch_cap : depth;
-  p.L = (int64_t)sc.slo_mult_milli * a.slo_base[a.fam_of_m[m]] / 1000;
-  p.A = (uint32_t)a.acc[m];
+  LaneP p;
+  p.Bmax = (sc.batch_cap > 0 && sc.batch_cap < depth) ? sc.batch_cap : depth;  // R4
+  p.L = (int64_t)sc.slo_mult_milli * a.slo_base[a.fam_of_m[a.option[d] - 1]] / 1000;  // R12
   return p;
 }
 
-// one decision of the §5 rule from head h with the device free at F over
-// arr[0, n): returns the batch size, *t = dispatch time
-__device__ __forceinline__ int decide(const uint32_t *arr, int64_t n, int64_t h, int64_t F, int Bmax, int64_t L,
+__device__ __forceinline__ uint32_t sat_lat(int64_t l) { return l >= 0xFFFFFFFFll ? 0xFFFFFFFEu : (uint32_t)l; }
+
+// One decision of the §5 rule from head h (device free at F) over arr[0, n):
+// returns the batch size b, *t_out = dispatch time.  T[b-1] = T(b).
+template <class Arr>
+__device__ __forceinline__ int decide(const Arr &arr, int64_t n, int64_t h, int64_t F, int Bmax, int64_t L,
                                       const int32_t *T, int64_t *t_out) {
-  const int64_t ah = arr[h];
-  int64_t t = F > ah ? F : ah;
+  const int64_t ah = arr(h);
+  int64_t t = F > ah ? F : ah;                                       // R5
   int q = 1;
-  while (q < Bmax && h + q < n && (int64_t)arr[h + q] <= t) q++;
+  while (q < Bmax && h + q < n && (int64_t)arr(h + q) <= t) q++;      // R3
   int b;
   for (;;) {
-    if (q >= Bmax) { b = Bmax; break; }
+    if (q >= Bmax) { b = Bmax; break; }                               // R4
     const int64_t W = ah + L - T[q];  // Tmax_wait(q+1) = Texp(1) - Tprocess(q+1)
-    if (t >= W) { b = q; break; }
-    if (h + q < n && (int64_t)arr[h + q] <= W) {  // Case 2: the (q+1)-st query comes by W
-      t = arr[h + q];
-      while (q < Bmax && h + q < n && (int64_t)arr[h + q] <= t) q++;
+    if (t >= W) { b = q; break; }                                     // R1
+    if (h + q < n && (int64_t)arr(h + q) <= W) {                      // Case 2 (R2)
+      t = arr(h + q);
+      while (q < Bmax && h + q < n && (int64_t)arr(h + q) <= t) q++;
       continue;
     }
-    t = W;  // Case 1: start at Tmax_wait(q+1)
+    t = W;                                                            // Case 1
     b = q;
     break;
   }
@@ -373,29 +282,69 @@ __device__ __forceinline__ int decide(const uint32_t *arr, int64_t n, int64_t h,
   return b;
 }
 
-__device__ __forceinline__ uint32_t sat_lat(int64_t l) { return l >= 0xFFFFFFFFll ? 0xFFFFFFFEu : (uint32_t)l; }
+struct PtrArr {
+  const uint32_t *p;
+  __device__ __forceinline__ uint32_t operator()(int64_t j) const { return p[j]; }
+};
 
-__global__ void k_spec(const __grid_constant__ ChunkArgs a) {
+// ---- fallback: one thread per (device, scenario) walks the whole array
+__global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ LaneArgs a) {
+  const int lane_id = blockIdx.x * blockDim.x + threadIdx.x;
+  if (lane_id >= a.nsc * a.D) return;
+  const int s = a.sc_list[lane_id / a.D], d = lane_id % a.D;
+  if (a.option[d] <= 0) return;
+  const int64_t st = a.devOff[d], n = a.devOff[d + 1] - st;
+  if (n == 0) return;
+  const uint32_t *idx = a.devIdx + st;
+  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  const LaneP p = lane_params(a, s, d, T);
+  uint32_t *out = a.lat_out + (size_t)s * a.N;
+  if (p.Bmax < 1) {  // cannot run even batch 1: never routed to (z = 0 / depth 0), kept for safety
+    for (int64_t j = 0; j < n; j++) out[idx[j]] = 0xFFFFFFFFu;
+    return;
+  }
+  PtrArr arr{a.devArr + st};
+  int64_t h = 0, F = 0;  // R13
+  while (h < n) {
+    int64_t t;
+    const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
+    F = t + T[b - 1];
+    for (int j = 0; j < b; j++) out[idx[h + j]] = sat_lat(F - (int64_t)arr(h + j));
+    h += b;
+  }
+}
+
+// ---- phase A: speculative windows
+// grid (nwin, scenario groups of 32, device groups of 32); warp = device,
+// lane = scenario.  With use_tile (one device group) the window's output rows
+// of the block's 32 scenarios are assembled in shared memory (initialised to
+// "dropped" so sink queries need no extra pass) and flushed with coalesced
+// stores.
+__global__ void k_spec(const __grid_constant__ LaneArgs a) {
   extern __shared__ uint32_t sm[];
   __shared__ int sOff[33], sStage[32];
-  __shared__ unsigned long long sCnt[32][3];
   const int c = blockIdx.x, sg = blockIdx.y, dg = blockIdx.z;
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
   const int d = dg * 32 + w;
+  const int win = a.win_tiles * TILE;
+  const int64_t i0 = (int64_t)c * win;
+  const int wlen = (int)(a.N - i0 < win ? a.N - i0 : win);
+  uint32_t *tile = sm;                                          // [32][win] if use_tile
+  int32_t *sT = (int32_t *)(sm + (a.use_tile ? 32 * win : 0));  // [nw][bmax]
+  uint32_t *sA = (uint32_t *)(sT + nw * a.bmax);                // staged arrivals
   const int64_t tile0 = (int64_t)c * a.win_tiles;
   const int64_t tile1 = tile0 + a.win_tiles < a.ntiles ? tile0 + a.win_tiles : a.ntiles;
-  int32_t *sT = (int32_t *)sm;                // [nw][bmax]
-  uint32_t *sA = sm + (size_t)nw * a.bmax;    // staged arrivals
   const bool dvalid = d < a.D;
   const int64_t n_d = dvalid ? a.devOff[d + 1] - a.devOff[d] : 0;
   const int64_t st = dvalid ? a.devBase[tile0 * (a.D + 1) + d] : 0;
   const int64_t en = dvalid ? a.devBase[tile1 * (a.D + 1) + d] : 0;
   const int64_t len = en - st;
-  const bool host = dvalid && a.option[d] > 0;
-  int64_t look = n_d - en < a.bmax ? n_d - en : a.bmax;
+  const bool host = dvalid && a.option[d] > 0 && len > 0;
+  const int64_t look = n_d - en < a.bmax ? n_d - en : a.bmax;
   const int stage = host ? (int)(len + look) : 0;
   if (lane == 0) sStage[w] = stage;
-  if (threadIdx.x < 32) { sCnt[threadIdx.x][0] = 0; sCnt[threadIdx.x][1] = 0; sCnt[threadIdx.x][2] = 0; }
+  if (a.use_tile)
+    for (int k = threadIdx.x; k < 32 * win; k += blockDim.x) tile[k] = 0xFFFFFFFFu;
   __syncthreads();
   if (threadIdx.x == 0) {
     int acc = 0;
@@ -404,40 +353,34 @@ __global__ void k_spec(const __grid_constant__ ChunkArgs a) {
   }
   __syncthreads();
   uint32_t *arr = sA + sOff[w];
-  if (host) {
-    const uint32_t *src = a.devArr + a.devOff[d] + st;
-    for (int i = lane; i < stage; i += 32) arr[i] = src[i];
-  }
   const int32_t *T = sT + w * a.bmax;
   if (host) {
+    const uint32_t *src = a.devArr + a.devOff[d] + st;
+    for (int k = lane; k < stage; k += 32) arr[k] = src[k];
     const int32_t *row = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
-    for (int i = lane; i < a.bmax; i += 32) sT[w * a.bmax + i] = row[i];
+    for (int k = lane; k < a.bmax; k += 32) sT[w * a.bmax + k] = row[k];
   }
   __syncthreads();
   const int si = sg * 32 + lane;
-  if (host && len > 0 && si < a.nsc) {
+  if (host && si < a.nsc) {
     const int s = a.sc_list[si];
     const LaneP p = lane_params(a, s, d, T);
     const uint32_t *ix = a.devIdx + a.devOff[d] + st;
-    uint32_t *out = a.lat_out + (size_t)s * a.N;
-    unsigned long long viol = 0, ont = 0, accs = 0;
+    uint32_t *out = a.use_tile ? tile + (size_t)lane * win : a.lat_out + (size_t)s * a.N;
+    const int64_t obase = a.use_tile ? i0 : 0;
     int64_t h = 0, F = 0;
     if (p.Bmax < 1) {
-      for (int64_t j = 0; j < len; j++) out[ix[j]] = 0xFFFFFFFFu;
-      viol = (unsigned long long)len;
+      if (!a.use_tile)
+        for (int64_t j = 0; j < len; j++) out[ix[j] - obase] = 0xFFFFFFFFu;
       h = len;
     } else {
+      PtrArr A{arr};
       while (h < len) {
         int64_t t;
-        const int b = decide(arr, stage, h, F, p.Bmax, p.L, T, &t);
+        const int b = decide(A, stage, h, F, p.Bmax, p.L, T, &t);
         F = t + T[b - 1];
         const int64_t jend = h + b < len ? h + b : len;
-        for (int64_t j = h; j < jend; j++) {
-          const uint32_t l = sat_lat(F - (int64_t)arr[j]);
-          out[ix[j]] = l;
-          if ((int64_t)l > p.L) viol++;
-          else { ont++; accs += p.A; }
-        }
+        for (int64_t j = h; j < jend; j++) out[ix[j] - obase] = sat_lat(F - (int64_t)arr[j]);
         h += b;
       }
     }
@@ -446,125 +389,182 @@ __global__ void k_spec(const __grid_constant__ ChunkArgs a) {
     e.ov = (int32_t)(h - len);
     e.pad = 0;
     a.ex[((size_t)s * a.D + d) * a.nwin + c] = e;
-    atomicAdd(&sCnt[lane][0], viol);
-    atomicAdd(&sCnt[lane][1], ont);
-    atomicAdd(&sCnt[lane][2], accs);
   }
+  if (!a.use_tile) return;
   __syncthreads();
-  if (threadIdx.x < 32 && sg * 32 + (int)threadIdx.x < a.nsc) {
-    const int s = a.sc_list[sg * 32 + threadIdx.x];
-    if (sCnt[threadIdx.x][0]) atomicAdd((unsigned long long *)&a.agg[s], sCnt[threadIdx.x][0]);
-    if (sCnt[threadIdx.x][1]) atomicAdd((unsigned long long *)&a.agg[a.S + s], sCnt[threadIdx.x][1]);
-    if (sCnt[threadIdx.x][2]) atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], sCnt[threadIdx.x][2]);
+  for (int r = 0; r < 32; r++) {
+    if (sg * 32 + r >= a.nsc) break;
+    uint32_t *row = a.lat_out + (size_t)a.sc_list[sg * 32 + r] * a.N + i0;
+    const uint32_t *tr = tile + (size_t)r * win;
+    for (int k = threadIdx.x; k < wlen; k += blockDim.x) row[k] = tr[k];
   }
 }
 
-struct Delta {
-  long long viol, ont, accs;
+// ---- phase B: exact stitch, one warp per (device, scenario)
+// The true state (h, F) is carried from window to window.  A window whose
+// speculative start (its first query, device idle) equals the true state is
+// already right.  Otherwise the true run is replayed batch by batch until it
+// meets the speculative run: after a batch [h, j2) finishing at Fn, if the
+// speculative run also has a batch ending at j2 - 1 with finish Fn (its
+// latency + arrival) and a new batch at j2, both runs are in the same state
+// (j2, Fn) and agree from there on.  Only batches that the device waited for
+// (t > F) are tested: a batch dispatched the moment the previous one finished
+// can only meet a run that had already met.  Backlogged stretches (Bmax
+// queued when the device frees) are full batches back to back -- batch k
+// finishes at F + (k+1) T(Bmax) -- and are taken 32 batches per step with a
+// ballot.  The device array streams through a shared-memory buffer.
+#define SBUF 2048
+#define SAHEAD 1024
+
+struct BufArr {
+  const uint32_t *buf, *g;
+  int64_t base;
+  __device__ __forceinline__ uint32_t operator()(int64_t j) const {
+    const int64_t o = j - base;
+    return (o >= 0 && o < SBUF) ? buf[o] : __ldg(g + j);
+  }
 };
 
-// rewrite latencies of device-relative queries [lo, hi) of one batch finishing at F (warp-cooperative)
-__device__ __forceinline__ void rewrite_const(const uint32_t *arr, const uint32_t *ix, uint32_t *out, int64_t lo,
-                                              int64_t hi, int64_t F, const LaneP &p, Delta &dl, int lane) {
-  for (int64_t j = lo + lane; j < hi; j += 32) {
-    const uint32_t nl = sat_lat(F - (int64_t)arr[j]);
-    const uint32_t g = ix[j];
-    const uint32_t ol = out[g];
-    out[g] = nl;
-    const int nv = (int64_t)nl > p.L, ov = (int64_t)ol > p.L;
-    dl.viol += nv - ov;
-    dl.ont += (1 - nv) - (1 - ov);
-    dl.accs += ((long long)(1 - nv) - (long long)(1 - ov)) * (long long)p.A;
-  }
-}
-
-__global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ ChunkArgs a) {
-  const int lane = threadIdx.x & 31;
-  const int64_t gw = (int64_t)blockIdx.x * 4 + (threadIdx.x >> 5);
-  if (gw >= (int64_t)a.nsc * a.D) return;
-  const int si = (int)(gw / a.D), d = (int)(gw % a.D);
-  const int s = a.sc_list[si];
-  if (a.option[d] <= 0 || a.nwin < 2) return;
-  const int64_t n_d = a.devOff[d + 1] - a.devOff[d];
-  if (n_d == 0) return;
-  const uint32_t *arr = a.devArr + a.devOff[d], *ix = a.devIdx + a.devOff[d];
+__global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs a) {
+  __shared__ uint32_t sbuf[4][SBUF];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int64_t gw = (int64_t)blockIdx.x * 4 + w;
+  if (gw >= (int64_t)a.nsc * a.D || a.nwin < 2) return;
+  const int s = a.sc_list[gw / a.D], d = (int)(gw % a.D);
+  if (a.option[d] <= 0) return;
+  const int64_t n = a.devOff[d + 1] - a.devOff[d];
+  if (n == 0) return;
+  const uint32_t *garr = a.devArr + a.devOff[d], *ix = a.devIdx + a.devOff[d];
   const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
   const LaneP p = lane_params(a, s, d, T);
   if (p.Bmax < 1) return;
   uint32_t *out = a.lat_out + (size_t)s * a.N;
   const SpecExit *ex = a.ex + ((size_t)s * a.D + d) * a.nwin;
+  BufArr A{sbuf[w], garr, -(int64_t)SBUF};
+  auto ensure = [&](int64_t h) {
+    if (h >= A.base && h + SAHEAD <= A.base + SBUF) return;
+    __syncwarp();
+    A.base = h & ~(int64_t)31;
+    for (int k = lane; k < SBUF; k += 32) sbuf[w][k] = A.base + k < n ? garr[A.base + k] : 0xFFFFFFFFu;
+    __syncwarp();
+  };
   auto win_start = [&](int c) -> int64_t {
     const int64_t t = (int64_t)c * a.win_tiles < a.ntiles ? (int64_t)c * a.win_tiles : a.ntiles;
     return a.devBase[t * (a.D + 1) + d];
   };
-  Delta dl = {0, 0, 0};
-  int64_t h = win_start(1) + ex[0].ov, F = ex[0].F;
+  auto write_batch = [&](int64_t lo, int64_t hi, int64_t Fb) {
+    for (int64_t j = lo + lane; j < hi; j += 32) out[ix[j]] = sat_lat(Fb - (int64_t)A(j));
+  };
   const int64_t TB = T[p.Bmax - 1];
+  int64_t h = win_start(1) + ex[0].ov, F = ex[0].F;
   for (int c = 1; c < a.nwin; c++) {
     const int64_t st = win_start(c), en = win_start(c + 1);
     if (en == st) continue;
-    if (h > st) rewrite_const(arr, ix, out, st, h < en ? h : en, F, p, dl, lane);  // overhang of the last batch
+    if (h > st) {  // queries of this window in the last batch of the previous one
+      ensure(st);
+      write_batch(st, h < en ? h : en, F);
+    }
     if (h >= en) continue;
-    if (h == st && F <= (int64_t)arr[st]) {  // the speculative start was the true state
+    ensure(h);
+    if (h == st && F <= (int64_t)A(st)) {  // speculative start = true state
       h = en + ex[c].ov;
       F = ex[c].F;
       continue;
     }
     while (h < en) {
-      // backlogged stretch: >= Bmax queued at completion -> full batches back to back
-      if (F > (int64_t)arr[h] && h + p.Bmax - 1 < n_d && (int64_t)arr[h + p.Bmax - 1] <= F) {
-        const int64_t kmax = (en - h + p.Bmax - 1) / p.Bmax;
+      ensure(h);
+      if (F > (int64_t)A(h) && h + p.Bmax - 1 < n && (int64_t)A(h + p.Bmax - 1) <= F) {
+        // backlog: full batches back to back
+        int64_t kmax = (en - h + p.Bmax - 1) / p.Bmax;
+        const int64_t room = (A.base + SBUF - h) / p.Bmax;
+        if (kmax > room) kmax = room;
+        if (kmax > 32) kmax = 32;
         const int64_t idx = h + (int64_t)(lane + 1) * p.Bmax - 1;
-        const bool ok = lane < kmax && idx < n_d && (int64_t)arr[idx] <= F + (int64_t)lane * TB;
+        const bool ok = lane < kmax && idx < n && (int64_t)A(idx) <= F + (int64_t)lane * TB;
         const unsigned bal = __ballot_sync(0xffffffffu, ok);
         const int r = bal == 0xffffffffu ? 32 : __ffs(~bal) - 1;
         const int64_t nq = (int64_t)r * p.Bmax;
         for (int64_t i = lane; i < nq; i += 32) {
           const int64_t k = i / p.Bmax, j = h + i;
-          const uint32_t nl = sat_lat(F + (k + 1) * TB - (int64_t)arr[j]);
-          const uint32_t g = ix[j];
-          const uint32_t ol = out[g];
-          out[g] = nl;
-          const int nv = (int64_t)nl > p.L, ov = (int64_t)ol > p.L;
-          dl.viol += nv - ov;
-          dl.ont += ov - nv;
-          dl.accs += ((long long)ov - (long long)nv) * (long long)p.A;
+          out[ix[j]] = sat_lat(F + (k + 1) * TB - (int64_t)A(j));
         }
         h += nq;
         F += (int64_t)r * TB;
         continue;
       }
       int64_t t;
-      const int b = decide(arr, n_d, h, F, p.Bmax, p.L, T, &t);
+      const int b = decide(A, n, h, F, p.Bmax, p.L, T, &t);
       const int64_t Fn = t + T[b - 1];
       const int64_t j2 = h + b;
-      bool conv;
-      if (j2 < en) {
-        const int64_t f1 = (int64_t)arr[j2 - 1] + out[ix[j2 - 1]], f2 = (int64_t)arr[j2] + out[ix[j2]];
+      bool conv = false;
+      if (t > F && j2 < en) {
+        const int64_t f1 = (int64_t)A(j2 - 1) + out[ix[j2 - 1]];
+        const int64_t f2 = (int64_t)A(j2) + out[ix[j2]];
         conv = f1 == Fn && f2 != Fn;
-      } else {
-        conv = j2 == en + ex[c].ov && Fn == ex[c].F;
       }
       __syncwarp();
-      rewrite_const(arr, ix, out, h, j2 < en ? j2 : en, Fn, p, dl, lane);
+      write_batch(h, j2 < en ? j2 : en, Fn);
       h = j2;
       F = Fn;
-      if (conv && h < en) {
+      if (conv) {
         h = en + ex[c].ov;
         F = ex[c].F;
         break;
       }
     }
   }
-  for (int o = 16; o; o >>= 1) {
-    dl.viol += __shfl_xor_sync(0xffffffffu, dl.viol, o);
-    dl.ont += __shfl_xor_sync(0xffffffffu, dl.ont, o);
-    dl.accs += __shfl_xor_sync(0xffffffffu, dl.accs, o);
+}
+
+// dropped queries (the sink segment, device index D): latency UINT32_MAX (R7)
+__global__ void k_sink(int64_t N, int D, const int32_t *__restrict__ sc_list, int nsc, const int64_t *devOff,
+                       const uint32_t *devIdx, uint32_t *lat_out) {
+  for (int k = blockIdx.y; k < nsc; k += gridDim.y) {
+    const int64_t st = devOff[D], n = devOff[D + 1] - st;
+    uint32_t *row = lat_out + (size_t)sc_list[k] * N;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
+      row[devIdx[st + j]] = 0xFFFFFFFFu;
   }
-  if (lane == 0) {
-    if (dl.viol) atomicAdd((unsigned long long *)&a.agg[s], (unsigned long long)dl.viol);
-    if (dl.ont) atomicAdd((unsigned long long *)&a.agg[a.S + s], (unsigned long long)dl.ont);
-    if (dl.accs) atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], (unsigned long long)dl.accs);
+}
+
+// ------------------------------------------------------------- counts ----
+// a13: per scenario, violations (latency > SLO of the query's family, R6;
+// dropped included), on-time count and the serving variant's accuracy summed
+// over on-time queries (R9).
+__global__ void k_count(int64_t N, int S, int D, int Q, const proteus_scenario *__restrict__ sc,
+                        const int32_t *__restrict__ slo_base, const int32_t *__restrict__ option,
+                        const int32_t *__restrict__ acc, const uint8_t *__restrict__ fam,
+                        const uint8_t *__restrict__ tgt0, const uint8_t *__restrict__ tgt1,
+                        const uint32_t *__restrict__ lat, uint64_t *agg) {
+  __shared__ int64_t sL[PX_MAXQ];
+  __shared__ uint32_t sA[PX_MAXD + 1];
+  __shared__ unsigned long long red[3][32];
+  const int s = blockIdx.y;
+  const proteus_scenario scn = sc[s];
+  if (threadIdx.x < Q) sL[threadIdx.x] = (int64_t)scn.slo_mult_milli * slo_base[threadIdx.x] / 1000;
+  if (threadIdx.x <= D) sA[threadIdx.x] = threadIdx.x < D && option[threadIdx.x] > 0 ? acc[option[threadIdx.x] - 1] : 0;
+  __syncthreads();
+  const uint8_t *tgt = scn.routing ? tgt1 : tgt0;
+  const uint32_t *row = lat + (size_t)s * N;
+  unsigned long long viol = 0, ont = 0, accs = 0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t l = row[i];
+    if ((int64_t)l > sL[fam[i]]) viol++;
+    else { ont++; accs += sA[tgt[i]]; }
+  }
+  for (int o = 16; o; o >>= 1) {
+    viol += __shfl_xor_sync(0xffffffffu, viol, o);
+    ont += __shfl_xor_sync(0xffffffffu, ont, o);
+    accs += __shfl_xor_sync(0xffffffffu, accs, o);
+  }
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) { red[0][w] = viol; red[1][w] = ont; red[2][w] = accs; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, o2 = 0, a2 = 0;
+    for (int k = 0; k < (int)(blockDim.x >> 5); k++) { v += red[0][k]; o2 += red[1][k]; a2 += red[2][k]; }
+    if (v) atomicAdd((unsigned long long *)&agg[s], v);
+    if (o2) atomicAdd((unsigned long long *)&agg[S + s], o2);
+    if (a2) atomicAdd((unsigned long long *)&agg[2 * S + s], a2);
   }
 }
 
@@ -579,7 +579,6 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
               const proteus_scenario *h_sc, int S, uint32_t *d_lat_out, uint64_t *d_agg) {
   const int Q = ctx->Q, M = ctx->M;
   PX_CUDA(ctx, cudaMemsetAsync(d_agg, 0, ((size_t)3 * S + 1) * 8, ctx->stream));
-  // small inputs: option, z, dev_type, demand, slo, scenarios, scenario lists
   const size_t small = (size_t)(4 * D + 2 * Q + 2 * PX_MAXQ + 8 + 2 * S) * 4 + (size_t)S * sizeof(proteus_scenario);
   char *sb = (char *)px_buf(ctx, B_R_MISC, small + 4096);
   if (!sb) return px_fail(ctx, PROTEUS_ENOMEM, "replay scratch");
@@ -617,13 +616,14 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   const int64_t *devOff[2] = {nullptr, nullptr};
   const int32_t *devBase[2] = {nullptr, nullptr};
   const uint32_t *devArr[2] = {nullptr, nullptr}, *devIdx[2] = {nullptr, nullptr};
+  const uint8_t *tgts[2] = {nullptr, nullptr};
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
     uint8_t *pat = (uint8_t *)px_buf(ctx, B_R_PAT, pat_cap);
     int32_t *hist = (int32_t *)px_buf(ctx, B_R_HIST, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
     int32_t *fbase = (int32_t *)px_buf(ctx, B_R_BASE, (size_t)(ntiles + 1) * (PX_MAXQ + 2) * 4);
     int32_t *dbase = (int32_t *)px_buf(ctx, rt ? B_R_DBASE1 : B_R_DBASE0, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
-    uint8_t *tgt = (uint8_t *)px_buf(ctx, B_R_TGT, (size_t)N + 16);
+    uint8_t *tgt = (uint8_t *)px_buf(ctx, rt ? B_R_TGT1 : B_R_TGT, (size_t)N + 16);
     int64_t *off = (int64_t *)px_buf(ctx, rt ? B_R_OFF1 : B_R_OFF, (size_t)2 * (PX_MAXD + 2) * 8);
     uint32_t *darr = (uint32_t *)px_buf(ctx, rt ? B_R_DEVARR1 : B_R_DEVARR, (size_t)N * 4 + 16);
     uint32_t *didx = (uint32_t *)px_buf(ctx, rt ? B_R_DEVIDX1 : B_R_DEVIDX, (size_t)N * 4 + 16);
@@ -644,54 +644,66 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     } else {
       PX_CUDA(ctx, cudaMemsetAsync(off, 0, (size_t)(PX_MAXD + 2) * 8, ctx->stream));
     }
-    devOff[rt] = off; devArr[rt] = darr; devIdx[rt] = didx; devBase[rt] = dbase;
+    devOff[rt] = off; devArr[rt] = darr; devIdx[rt] = didx; devBase[rt] = dbase; tgts[rt] = tgt;
   }
   if (N == 0) return 0;
-  // latencies are needed by the stitch even when the caller does not want them
+  // the stitch reads speculative latencies, so rows exist even when the caller wants none
   uint32_t *lat = d_lat_out;
   if (!lat) {
     lat = (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S * N * 4);
     if (!lat) return px_fail(ctx, PROTEUS_ENOMEM, "latency scratch");
   }
-  const int win_tiles = env_int("PROTEUS_REPLAY_WIN_TILES", 4);
+  const int win_tiles = env_int("PROTEUS_REPLAY_WIN_TILES", 2);
   const int nwin = (int)((ntiles + win_tiles - 1) / win_tiles);
-  const int ndg = (D + 31) / 32;
+  const int win = win_tiles * TILE;
   const int dpb = D < 32 ? D : 32;
-  const size_t smem = ((size_t)dpb * ctx->bmax + (size_t)win_tiles * TILE + (size_t)dpb * ctx->bmax) * 4;
+  const int ndg = (D + 31) / 32;
+  int use_tile = ndg == 1 && !env_int("PROTEUS_REPLAY_NO_TILE", 0);
+  auto spec_smem = [&](int tile) {
+    return ((size_t)(tile ? 32 * win : 0) + (size_t)dpb * ctx->bmax + (size_t)win + (size_t)dpb * ctx->bmax) * 4;
+  };
+  if (use_tile && spec_smem(1) > 200 * 1024) use_tile = 0;
+  const size_t smem = spec_smem(use_tile);
   const bool simple = env_int("PROTEUS_REPLAY_SIMPLE", 0) != 0 || smem > 200 * 1024;
-  if (simple) {
+  SpecExit *ex = nullptr;
+  if (!simple) {
+    ex = (SpecExit *)px_buf(ctx, B_R_LANE, sizeof(SpecExit) * (size_t)S * D * nwin);
+    if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
+    if (smem > 48 * 1024)
+      PX_CUDA(ctx, cudaFuncSetAttribute(k_spec, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  }
+  for (int rt = 0; rt < 2; rt++) {
+    if (scl[rt].empty()) continue;
     LaneArgs la;
-    la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.N = N;
+    memset(&la, 0, sizeof la);
+    la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.Q = Q; la.N = N; la.ntiles = ntiles;
     la.option = d_opt; la.dev_type = d_dev; la.fam_of_m = ctx->d_fam; la.acc = ctx->d_acc; la.lat = ctx->d_lat;
     la.slo_base = d_slo; la.sc = d_sc;
-    for (int rt = 0; rt < 2; rt++) { la.devOff[rt] = devOff[rt]; la.devArr[rt] = devArr[rt]; la.devIdx[rt] = devIdx[rt]; }
-    la.lat_out = d_lat_out;
-    la.agg = d_agg;
-    const int nl = S * D;
-    PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
-  } else {
-    SpecExit *ex = (SpecExit *)px_buf(ctx, B_R_LANE, sizeof(SpecExit) * (size_t)S * D * nwin);
-    if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
-    if (smem > 48 * 1024) PX_CUDA(ctx, cudaFuncSetAttribute(k_spec, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    for (int rt = 0; rt < 2; rt++) {
-      if (scl[rt].empty()) continue;
-      ChunkArgs ca;
-      memset(&ca, 0, sizeof ca);
-      ca.S = S; ca.D = D; ca.M = M; ca.bmax = ctx->bmax; ca.nsc = (int)scl[rt].size();
-      ca.win_tiles = win_tiles; ca.nwin = nwin; ca.N = N; ca.ntiles = ntiles;
-      ca.option = d_opt; ca.dev_type = d_dev; ca.fam_of_m = ctx->d_fam; ca.acc = ctx->d_acc; ca.lat = ctx->d_lat;
-      ca.slo_base = d_slo; ca.sc_list = d_scl + rt * S; ca.sc = d_sc;
-      ca.devOff = devOff[rt]; ca.devBase = devBase[rt]; ca.devArr = devArr[rt]; ca.devIdx = devIdx[rt];
-      ca.lat_out = lat; ca.agg = d_agg; ca.ex = ex;
-      dim3 grid(nwin, (ca.nsc + 31) / 32, ndg);
-      PX_LAUNCH(ctx, "replay_spec", k_spec, grid, dpb * 32, smem, ca);
-      const int64_t warps = (int64_t)ca.nsc * D;
-      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 0, ca);
+    la.nsc = (int)scl[rt].size(); la.win_tiles = win_tiles; la.nwin = nwin; la.use_tile = simple ? 0 : use_tile;
+    la.sc_list = d_scl + rt * S;
+    la.devOff = devOff[rt]; la.devBase = devBase[rt]; la.devArr = devArr[rt]; la.devIdx = devIdx[rt];
+    la.lat_out = lat; la.ex = ex;
+    if (simple) {
+      const int nl = la.nsc * D;
+      PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
+    } else {
+      dim3 grid(nwin, (la.nsc + 31) / 32, ndg);
+      PX_LAUNCH(ctx, "replay_spec", k_spec, grid, dpb * 32, smem, la);
+      const int64_t warps = (int64_t)la.nsc * D;
+      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 0, la);
+    }
+    if (simple || !la.use_tile) {
+      dim3 g(64, la.nsc < 65535 ? la.nsc : 65535);
+      PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, N, D, d_scl + rt * S, la.nsc, devOff[rt], devIdx[rt], lat);
     }
   }
-  dim3 g(64, S < 65535 ? S : 65535);
-  PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, d_sc, S, D, N, devOff[0] ? devOff[0] : devOff[1],
-            devIdx[0] ? devIdx[0] : devIdx[1], devOff[1] ? devOff[1] : devOff[0], devIdx[1] ? devIdx[1] : devIdx[0],
-            d_lat_out, d_agg);
+  int nsm = 0;
+  PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
+  int bx = (int)((N + 255) / 256);
+  const int cap_bx = (nsm * 8 + S - 1) / S;
+  if (bx > cap_bx) bx = cap_bx > 0 ? cap_bx : 1;
+  dim3 cg(bx, S);
+  PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, S, D, Q, d_sc, d_slo, d_opt, ctx->d_acc, d_fam,
+            tgts[0] ? tgts[0] : tgts[1], tgts[1] ? tgts[1] : tgts[0], lat, d_agg);
   return 0;
 }

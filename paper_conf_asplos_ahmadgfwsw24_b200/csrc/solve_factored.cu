@@ -26,7 +26,7 @@
 #include "internal.cuh"
 
 #define FG_WARPS 8
-#define DP_THREADS 256
+#define DP_THREADS 512
 
 struct FactLayout {
   int32_t Q, T, VM, U;
@@ -180,41 +180,58 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
                                                          const int32_t *__restrict__ Pdev, int K,
                                                          const int32_t *__restrict__ slot_code,
                                                          const int32_t *__restrict__ slot_acc, SolRec *out) {
+  // Budget DP with the current stage in shared memory: G_q(b) = max over
+  // u <= b of g_q(u) + G_{q+1}(b - u).  One warp per budget b; lanes split the
+  // box {u <= b}.  Every stage is also written to global memory for the
+  // reconstruction.  A score of ~0 marks "no count vector with this usage"
+  // (a real score has accsum < 10^6 * served < 2^42 - 1, so it is never ~0).
+  extern __shared__ uint64_t dsm[];
   const int vec = blockIdx.x;
   const int Q = f.Q, U = f.U, T = f.T;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
   const BestRec *gv = g + (size_t)vec * Q * U;
   uint64_t *G = Gbuf + (size_t)vec * (Q + 1) * U;
-  for (int b = threadIdx.x; b < U; b += blockDim.x) G[(size_t)Q * U + b] = 0;
-  __syncthreads();
+  uint64_t *Gn = dsm, *gq = dsm + U;
+  const uint64_t NONE = ~0ull;
+  for (int b = threadIdx.x; b < U; b += blockDim.x) { Gn[b] = 0; G[(size_t)Q * U + b] = 0; }
   for (int q = Q - 1; q >= 0; q--) {
-    for (int b = threadIdx.x; b < U; b += blockDim.x) {
-      int bv[PX_MAXT], u[PX_MAXT];
-      ukey_decode(f, b, bv);
-      for (int t = 0; t < T; t++) u[t] = 0;
+    for (int u = threadIdx.x; u < U; u += blockDim.x) {
+      const BestRec e = gv[(size_t)q * U + u];
+      gq[u] = e.index == ~0ull ? NONE : e.score;
+    }
+    __syncthreads();
+    uint64_t *Gq = G + (size_t)q * U;
+    for (int b = w; b < U; b += nw) {
+      int bv[PX_MAXT], box = 1;
+      for (int t = 0; t < T; t++) { bv[t] = (b / f.ustride[t]) % (f.Nt[t] + 1); box *= bv[t] + 1; }
       uint64_t best = 0;
       bool have = false;
-      for (;;) {
-        int uk = 0, rk = 0;
-        for (int t = 0; t < T; t++) { uk += u[t] * f.ustride[t]; rk += (bv[t] - u[t]) * f.ustride[t]; }
-        const BestRec e = gv[(size_t)q * U + uk];
-        if (e.index != ~0ull) {
-          const uint64_t c = e.score + G[(size_t)(q + 1) * U + rk];
-          if (!have || c > best) { best = c; have = true; }
+      for (int i = lane; i < box; i += 32) {
+        int x = i, uk = 0, rk = 0;
+        for (int t = T - 1; t >= 0; t--) {
+          const int ut = x % (bv[t] + 1);
+          x /= bv[t] + 1;
+          uk += ut * f.ustride[t];
+          rk += (bv[t] - ut) * f.ustride[t];
         }
-        int t = T - 1;
-        for (; t >= 0; t--) {
-          if (++u[t] <= bv[t]) break;
-          u[t] = 0;
-        }
-        if (t < 0) break;
+        const uint64_t gs = gq[uk];
+        if (gs == NONE) continue;
+        const uint64_t c = gs + Gn[rk];
+        if (!have || c > best) { best = c; have = true; }
       }
-      G[(size_t)q * U + b] = best;
+      for (int o = 16; o; o >>= 1) {
+        const uint64_t b2 = __shfl_xor_sync(0xffffffffu, best, o);
+        const int h2 = __shfl_xor_sync(0xffffffffu, (int)have, o);
+        if (h2 && (!have || b2 > best)) { best = b2; have = true; }
+      }
+      if (lane == 0) Gq[b] = best;  // u = 0 is always valid: have == true
     }
+    __syncthreads();
+    for (int b = threadIdx.x; b < U; b += blockDim.x) Gn[b] = Gq[b];
     __syncthreads();
   }
   // reconstruction (warp 0): lexicographically smallest count tensor
   __shared__ uint64_t pick_sub[PX_MAXQ];
-  __shared__ int pick_u[PX_MAXQ];
   if (threadIdx.x < 32) {
     const int lane = threadIdx.x;
     int bv[PX_MAXT];
@@ -241,7 +258,7 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
         const uint64_t s2 = __shfl_xor_sync(0xffffffffu, bsub, o), u2 = __shfl_xor_sync(0xffffffffu, bu, o);
         if (s2 < bsub) { bsub = s2; bu = u2; }
       }
-      if (lane == 0) { pick_sub[q] = bsub; pick_u[q] = (int)bu; }
+      if (lane == 0) pick_sub[q] = bsub;
       int uu[PX_MAXT];
       ukey_decode(f, (int)bu, uu);
       for (int t = 0; t < T; t++) bv[t] -= uu[t];
@@ -358,7 +375,11 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
   const int64_t nitems = (int64_t)n_vec * Q * U;
   PX_LAUNCH(ctx, "fact_g", k_fact_g, (unsigned)((nitems + FG_WARPS - 1) / FG_WARPS), FG_WARPS * 32, 0, f, n_vec,
             d_demand, tab.slot_acc, g);
-  PX_LAUNCH(ctx, "fact_dp", k_fact_dp, n_vec, DP_THREADS, 0, f, g, G, d_demand, d_dev, D, tab.Pdev, K,
+  const size_t dsmem = (size_t)2 * U * 8;
+  if (dsmem > 200 * 1024) return px_fail(ctx, PROTEUS_ERANGE, "usage lattice %lld too large for the DP", (long long)U);
+  if (dsmem > 48 * 1024)
+    PX_CUDA(ctx, cudaFuncSetAttribute(k_fact_dp, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem));
+  PX_LAUNCH(ctx, "fact_dp", k_fact_dp, n_vec, DP_THREADS, dsmem, f, g, G, d_demand, d_dev, D, tab.Pdev, K,
             tab.slot_code, tab.slot_acc, d_sol);
   return 0;
 }

@@ -32,7 +32,7 @@ def _compare(px, oracle_mod, prof, cl, option, z, demand, arr, fam, sc):
     return g
 
 
-PATHS = {"chunked": {}, "small_windows": {"PROTEUS_REPLAY_WIN_TILES": "1"},
+PATHS = {"chunked": {}, "small_windows": {"PROTEUS_REPLAY_WIN_TILES": "1"}, "no_tile": {"PROTEUS_REPLAY_NO_TILE": "1"},
          "simple": {"PROTEUS_REPLAY_SIMPLE": "1"}}
 
 
