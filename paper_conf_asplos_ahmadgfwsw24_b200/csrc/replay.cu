@@ -316,10 +316,11 @@ __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ 
 
 // ---- phase A: speculative windows
 // grid (nwin, scenario groups of 32, device groups of 32); warp = device,
-// lane = scenario.  With use_tile (one device group) the window's output rows
-// of the block's 32 scenarios are assembled in shared memory (initialised to
-// "dropped" so sink queries need no extra pass) and flushed with coalesced
-// stores.
+// lane = scenario.  A window's arrivals and query indices of every device are
+// staged in shared memory.  With use_tile (one device group) the window's
+// output rows of the block's 32 scenarios are assembled in shared memory
+// (initialised to "dropped" so sink queries need no extra pass) and flushed
+// with coalesced stores.
 __global__ void k_spec(const __grid_constant__ LaneArgs a) {
   extern __shared__ uint32_t sm[];
   __shared__ int sOff[33], sStage[32];
@@ -329,9 +330,11 @@ __global__ void k_spec(const __grid_constant__ LaneArgs a) {
   const int win = a.win_tiles * TILE;
   const int64_t i0 = (int64_t)c * win;
   const int wlen = (int)(a.N - i0 < win ? a.N - i0 : win);
+  const int stage_cap = win + nw * a.bmax;
   uint32_t *tile = sm;                                          // [32][win] if use_tile
   int32_t *sT = (int32_t *)(sm + (a.use_tile ? 32 * win : 0));  // [nw][bmax]
-  uint32_t *sA = (uint32_t *)(sT + nw * a.bmax);                // staged arrivals
+  uint32_t *sA = (uint32_t *)(sT + nw * a.bmax);                // staged arrivals [stage_cap]
+  uint32_t *sI = sA + stage_cap;                                // staged query indices [stage_cap]
   const int64_t tile0 = (int64_t)c * a.win_tiles;
   const int64_t tile1 = tile0 + a.win_tiles < a.ntiles ? tile0 + a.win_tiles : a.ntiles;
   const bool dvalid = d < a.D;
@@ -353,10 +356,14 @@ __global__ void k_spec(const __grid_constant__ LaneArgs a) {
   }
   __syncthreads();
   uint32_t *arr = sA + sOff[w];
+  uint32_t *ixs = sI + sOff[w];
   const int32_t *T = sT + w * a.bmax;
   if (host) {
-    const uint32_t *src = a.devArr + a.devOff[d] + st;
-    for (int k = lane; k < stage; k += 32) arr[k] = src[k];
+    const uint32_t *src = a.devArr + a.devOff[d] + st, *isrc = a.devIdx + a.devOff[d] + st;
+    for (int k = lane; k < stage; k += 32) {
+      arr[k] = src[k];
+      ixs[k] = k < len ? isrc[k] : 0;
+    }
     const int32_t *row = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
     for (int k = lane; k < a.bmax; k += 32) sT[w * a.bmax + k] = row[k];
   }
@@ -365,13 +372,12 @@ __global__ void k_spec(const __grid_constant__ LaneArgs a) {
   if (host && si < a.nsc) {
     const int s = a.sc_list[si];
     const LaneP p = lane_params(a, s, d, T);
-    const uint32_t *ix = a.devIdx + a.devOff[d] + st;
     uint32_t *out = a.use_tile ? tile + (size_t)lane * win : a.lat_out + (size_t)s * a.N;
-    const int64_t obase = a.use_tile ? i0 : 0;
+    const uint32_t obase = a.use_tile ? (uint32_t)i0 : 0u;
     int64_t h = 0, F = 0;
     if (p.Bmax < 1) {
       if (!a.use_tile)
-        for (int64_t j = 0; j < len; j++) out[ix[j] - obase] = 0xFFFFFFFFu;
+        for (int64_t j = 0; j < len; j++) out[ixs[j] - obase] = 0xFFFFFFFFu;
       h = len;
     } else {
       PtrArr A{arr};
@@ -380,7 +386,7 @@ __global__ void k_spec(const __grid_constant__ LaneArgs a) {
         const int b = decide(A, stage, h, F, p.Bmax, p.L, T, &t);
         F = t + T[b - 1];
         const int64_t jend = h + b < len ? h + b : len;
-        for (int64_t j = h; j < jend; j++) out[ix[j] - obase] = sat_lat(F - (int64_t)arr[j]);
+        for (int64_t j = h; j < jend; j++) out[ixs[j] - obase] = sat_lat(F - (int64_t)arr[j]);
         h += b;
       }
     }
@@ -412,9 +418,11 @@ __global__ void k_spec(const __grid_constant__ LaneArgs a) {
 // can only meet a run that had already met.  Backlogged stretches (Bmax
 // queued when the device frees) are full batches back to back -- batch k
 // finishes at F + (k+1) T(Bmax) -- and are taken 32 batches per step with a
-// ballot.  The device array streams through a shared-memory buffer.
+// ballot.  The device's arrivals and query indices stream through a
+// shared-memory ring; window bounds and exit states are fetched 32 windows
+// at a time.
 #define SBUF 2048
-#define SAHEAD 1024
+#define SAHEAD 1088
 
 struct BufArr {
   const uint32_t *buf, *g;
@@ -425,8 +433,49 @@ struct BufArr {
   }
 };
 
+// number of j in [h + q, h + min(Bmax, n - h)) with arr(j) <= t, added to q
+// (arrivals are sorted, so the ballot is a prefix)
+template <class Arr>
+__device__ __forceinline__ int count_le(const Arr &A, int64_t n, int64_t h, int q, int Bmax, int64_t t, int lane) {
+  for (;;) {
+    const int64_t j = h + q + lane;
+    const bool le = q + lane < Bmax && j < n && (int64_t)A(j) <= t;
+    const int c = __popc(__ballot_sync(0xffffffffu, le));
+    q += c;
+    if (c < 32) return q;
+  }
+}
+
+// decide() with the counting done 32 arrivals at a time by the warp
+template <class Arr>
+__device__ __forceinline__ int decide_warp(const Arr &A, int64_t n, int64_t h, int64_t F, int Bmax, int64_t L,
+                                           const int32_t *T, int lane, int64_t *t_out) {
+  const int64_t ah = A(h);
+  int64_t t = F > ah ? F : ah;
+  int q = count_le(A, n, h, 1, Bmax, t, lane);
+  int b;
+  for (;;) {
+    if (q >= Bmax) { b = Bmax; break; }
+    const int64_t W = ah + L - T[q];
+    if (t >= W) { b = q; break; }
+    if (h + q < n) {
+      const int64_t nx = A(h + q);
+      if (nx <= W) {
+        t = nx;
+        q = count_le(A, n, h, q, Bmax, t, lane);
+        continue;
+      }
+    }
+    t = W;
+    b = q;
+    break;
+  }
+  *t_out = t;
+  return b;
+}
+
 __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs a) {
-  __shared__ uint32_t sbuf[4][SBUF];
+  extern __shared__ uint32_t ssm[];  // [4 warps][2][SBUF]
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t gw = (int64_t)blockIdx.x * 4 + w;
   if (gw >= (int64_t)a.nsc * a.D || a.nwin < 2) return;
@@ -434,82 +483,105 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   if (a.option[d] <= 0) return;
   const int64_t n = a.devOff[d + 1] - a.devOff[d];
   if (n == 0) return;
-  const uint32_t *garr = a.devArr + a.devOff[d], *ix = a.devIdx + a.devOff[d];
+  uint32_t *bufA = ssm + (size_t)w * 2 * SBUF, *bufI = bufA + SBUF;
+  const uint32_t *garr = a.devArr + a.devOff[d], *gix = a.devIdx + a.devOff[d];
   const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
   const LaneP p = lane_params(a, s, d, T);
   if (p.Bmax < 1) return;
   uint32_t *out = a.lat_out + (size_t)s * a.N;
   const SpecExit *ex = a.ex + ((size_t)s * a.D + d) * a.nwin;
-  BufArr A{sbuf[w], garr, -(int64_t)SBUF};
+  BufArr A{bufA, garr, -(int64_t)(4 * SBUF)};
   auto ensure = [&](int64_t h) {
     if (h >= A.base && h + SAHEAD <= A.base + SBUF) return;
     __syncwarp();
     A.base = h & ~(int64_t)31;
-    for (int k = lane; k < SBUF; k += 32) sbuf[w][k] = A.base + k < n ? garr[A.base + k] : 0xFFFFFFFFu;
+    for (int k = lane; k < SBUF; k += 32) {
+      const int64_t j = A.base + k;
+      bufA[k] = j < n ? garr[j] : 0xFFFFFFFFu;
+      bufI[k] = j < n ? gix[j] : 0u;
+    }
     __syncwarp();
   };
-  auto win_start = [&](int c) -> int64_t {
-    const int64_t t = (int64_t)c * a.win_tiles < a.ntiles ? (int64_t)c * a.win_tiles : a.ntiles;
-    return a.devBase[t * (a.D + 1) + d];
+  auto IX = [&](int64_t j) -> uint32_t {
+    const int64_t o = j - A.base;
+    return (o >= 0 && o < SBUF) ? bufI[o] : __ldg(gix + j);
   };
   auto write_batch = [&](int64_t lo, int64_t hi, int64_t Fb) {
-    for (int64_t j = lo + lane; j < hi; j += 32) out[ix[j]] = sat_lat(Fb - (int64_t)A(j));
+    for (int64_t j = lo + lane; j < hi; j += 32) out[IX(j)] = sat_lat(Fb - (int64_t)A(j));
   };
   const int64_t TB = T[p.Bmax - 1];
-  int64_t h = win_start(1) + ex[0].ov, F = ex[0].F;
-  for (int c = 1; c < a.nwin; c++) {
-    const int64_t st = win_start(c), en = win_start(c + 1);
-    if (en == st) continue;
-    if (h > st) {  // queries of this window in the last batch of the previous one
-      ensure(st);
-      write_batch(st, h < en ? h : en, F);
+  const int64_t nwin = a.nwin;
+  auto tile_of = [&](int64_t c) { return c * a.win_tiles < a.ntiles ? c * a.win_tiles : a.ntiles; };
+  int64_t h = a.devBase[tile_of(1) * (a.D + 1) + d] + ex[0].ov, F = ex[0].F;
+  for (int64_t c0 = 1; c0 < nwin; c0 += 32) {
+    // lane k prefetches window c0 + k: its start, end and speculative exit
+    const int64_t ck = c0 + lane;
+    int64_t pst = 0, pen = 0, pF = 0;
+    int pov = 0;
+    if (ck < nwin) {
+      pst = a.devBase[tile_of(ck) * (a.D + 1) + d];
+      pen = a.devBase[tile_of(ck + 1) * (a.D + 1) + d];
+      const SpecExit e = ex[ck];
+      pF = e.F;
+      pov = e.ov;
     }
-    if (h >= en) continue;
-    ensure(h);
-    if (h == st && F <= (int64_t)A(st)) {  // speculative start = true state
-      h = en + ex[c].ov;
-      F = ex[c].F;
-      continue;
-    }
-    while (h < en) {
+    const int cnt = nwin - c0 < 32 ? (int)(nwin - c0) : 32;
+    for (int k = 0; k < cnt; k++) {
+      const int64_t st = __shfl_sync(0xffffffffu, pst, k), en = __shfl_sync(0xffffffffu, pen, k);
+      const int64_t eF = __shfl_sync(0xffffffffu, pF, k);
+      const int eov = __shfl_sync(0xffffffffu, pov, k);
+      if (en == st) continue;
+      if (h > st) {  // queries of this window in the last batch of the previous one
+        ensure(st);
+        write_batch(st, h < en ? h : en, F);
+      }
+      if (h >= en) continue;
       ensure(h);
-      if (F > (int64_t)A(h) && h + p.Bmax - 1 < n && (int64_t)A(h + p.Bmax - 1) <= F) {
-        // backlog: full batches back to back
-        int64_t kmax = (en - h + p.Bmax - 1) / p.Bmax;
-        const int64_t room = (A.base + SBUF - h) / p.Bmax;
-        if (kmax > room) kmax = room;
-        if (kmax > 32) kmax = 32;
-        const int64_t idx = h + (int64_t)(lane + 1) * p.Bmax - 1;
-        const bool ok = lane < kmax && idx < n && (int64_t)A(idx) <= F + (int64_t)lane * TB;
-        const unsigned bal = __ballot_sync(0xffffffffu, ok);
-        const int r = bal == 0xffffffffu ? 32 : __ffs(~bal) - 1;
-        const int64_t nq = (int64_t)r * p.Bmax;
-        for (int64_t i = lane; i < nq; i += 32) {
-          const int64_t k = i / p.Bmax, j = h + i;
-          out[ix[j]] = sat_lat(F + (k + 1) * TB - (int64_t)A(j));
-        }
-        h += nq;
-        F += (int64_t)r * TB;
+      if (h == st && F <= (int64_t)A(st)) {  // speculative start = true state
+        h = en + eov;
+        F = eF;
         continue;
       }
-      int64_t t;
-      const int b = decide(A, n, h, F, p.Bmax, p.L, T, &t);
-      const int64_t Fn = t + T[b - 1];
-      const int64_t j2 = h + b;
-      bool conv = false;
-      if (t > F && j2 < en) {
-        const int64_t f1 = (int64_t)A(j2 - 1) + out[ix[j2 - 1]];
-        const int64_t f2 = (int64_t)A(j2) + out[ix[j2]];
-        conv = f1 == Fn && f2 != Fn;
-      }
-      __syncwarp();
-      write_batch(h, j2 < en ? j2 : en, Fn);
-      h = j2;
-      F = Fn;
-      if (conv) {
-        h = en + ex[c].ov;
-        F = ex[c].F;
-        break;
+      while (h < en) {
+        ensure(h);
+        if (F > (int64_t)A(h) && h + p.Bmax - 1 < n && (int64_t)A(h + p.Bmax - 1) <= F) {
+          // backlog: full batches back to back
+          int64_t kmax = (en - h + p.Bmax - 1) / p.Bmax;
+          const int64_t room = (A.base + SBUF - h) / p.Bmax;
+          if (kmax > room) kmax = room;
+          if (kmax > 32) kmax = 32;
+          const int64_t idx = h + (int64_t)(lane + 1) * p.Bmax - 1;
+          const bool ok = lane < kmax && idx < n && (int64_t)A(idx) <= F + (int64_t)lane * TB;
+          const unsigned bal = __ballot_sync(0xffffffffu, ok);
+          const int r = bal == 0xffffffffu ? 32 : __ffs(~bal) - 1;
+          const int64_t nq = (int64_t)r * p.Bmax;
+          for (int64_t i = lane; i < nq; i += 32) {
+            const int64_t kk = i / p.Bmax, j = h + i;
+            out[IX(j)] = sat_lat(F + (kk + 1) * TB - (int64_t)A(j));
+          }
+          h += nq;
+          F += (int64_t)r * TB;
+          continue;
+        }
+        int64_t t;
+        const int b = decide_warp(A, n, h, F, p.Bmax, p.L, T, lane, &t);
+        const int64_t Fn = t + T[b - 1];
+        const int64_t j2 = h + b;
+        bool conv = false;
+        if (t > F && j2 < en) {
+          const int64_t f1 = (int64_t)A(j2 - 1) + out[IX(j2 - 1)];
+          const int64_t f2 = (int64_t)A(j2) + out[IX(j2)];
+          conv = f1 == Fn && f2 != Fn;
+        }
+        __syncwarp();
+        write_batch(h, j2 < en ? j2 : en, Fn);
+        h = j2;
+        F = Fn;
+        if (conv) {
+          h = en + eov;
+          F = eF;
+          break;
+        }
       }
     }
   }
@@ -660,7 +732,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   const int ndg = (D + 31) / 32;
   int use_tile = ndg == 1 && !env_int("PROTEUS_REPLAY_NO_TILE", 0);
   auto spec_smem = [&](int tile) {
-    return ((size_t)(tile ? 32 * win : 0) + (size_t)dpb * ctx->bmax + (size_t)win + (size_t)dpb * ctx->bmax) * 4;
+    return ((size_t)(tile ? 32 * win : 0) + (size_t)dpb * ctx->bmax + 2 * ((size_t)win + (size_t)dpb * ctx->bmax)) * 4;
   };
   if (use_tile && spec_smem(1) > 200 * 1024) use_tile = 0;
   const size_t smem = spec_smem(use_tile);
@@ -671,6 +743,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
     if (smem > 48 * 1024)
       PX_CUDA(ctx, cudaFuncSetAttribute(k_spec, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    PX_CUDA(ctx, cudaFuncSetAttribute(k_stitch, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * 2 * SBUF * 4));
   }
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
@@ -690,7 +763,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       dim3 grid(nwin, (la.nsc + 31) / 32, ndg);
       PX_LAUNCH(ctx, "replay_spec", k_spec, grid, dpb * 32, smem, la);
       const int64_t warps = (int64_t)la.nsc * D;
-      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 0, la);
+      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 4 * 2 * SBUF * 4, la);
     }
     if (simple || !la.use_tile) {
       dim3 g(64, la.nsc < 65535 ? la.nsc : 65535);

@@ -199,7 +199,7 @@ __device__ __forceinline__ uint64_t fill(const int (&caps)[QM * VM], const FlatA
 }
 
 template <int QM, int VM>
-__global__ void __launch_bounds__(FLAT_THREADS) k_flat_pair(const __grid_constant__ FlatArgs<QM, VM> a) {
+__global__ void __launch_bounds__(FLAT_THREADS, 2) k_flat_pair(const __grid_constant__ FlatArgs<QM, VM> a) {
   constexpr int S = QM * VM;
   extern __shared__ int32_t smem[];
   const int D = a.D, K = a.K;
@@ -219,16 +219,22 @@ __global__ void __launch_bounds__(FLAT_THREADS) k_flat_pair(const __grid_constan
       uint64_t x = p;
       for (int i = D - 3; i >= 0; i--) { dig[i] = (int)(x % K); x /= K; }
     }
-    int capsB[S];
+    // capacities of devices 0..D-4 per slot: rebuilt only when a digit above
+    // D-3 changes, kept in shared memory ([slot][thread], conflict-free) to
+    // leave the registers to the candidate loop
+    __shared__ int sCapsB[S][FLAT_THREADS];
     auto rebuild = [&]() {
+      int cb[S];
 #pragma unroll
-      for (int s = 0; s < S; s++) capsB[s] = 0;
+      for (int s = 0; s < S; s++) cb[s] = 0;
       for (int i = 0; i < D - 3; i++) {
         const int o = dig[i];
         const int sl = sCS[o], pv = sP[i * K + o];
 #pragma unroll
-        for (int s = 0; s < S; s++) capsB[s] += (sl == s) ? pv : 0;
+        for (int s = 0; s < S; s++) cb[s] += (sl == s) ? pv : 0;
       }
+#pragma unroll
+      for (int s = 0; s < S; s++) sCapsB[s][threadIdx.x] = cb[s];
     };
     rebuild();
     for (;;) {
@@ -236,47 +242,50 @@ __global__ void __launch_bounds__(FLAT_THREADS) k_flat_pair(const __grid_constan
       const int sl3 = sCS[o3], p3 = sP[(D - 3) * K + o3];
       int caps[S];
 #pragma unroll
-      for (int s = 0; s < S; s++) caps[s] = capsB[s] + (sl3 == s ? p3 : 0);
+      for (int s = 0; s < S; s++) caps[s] = sCapsB[s][threadIdx.x] + (sl3 == s ? p3 : 0);
       uint64_t Fq[QM];
       uint64_t base = 0;
 #pragma unroll
       for (int q = 0; q < QM; q++) { Fq[q] = fill<QM, VM>(caps, a, q, -1, 0, -1, 0); base += Fq[q]; }
-      uint64_t Fa[S], Fb[S];
+      uint64_t Fb[S];
 #pragma unroll
-      for (int s = 0; s < S; s++) {
-        const int q = s / VM, j = s % VM;
-        Fa[s] = fill<QM, VM>(caps, a, q, j, a.PA[s], -1, 0) - Fq[q];
-        Fb[s] = fill<QM, VM>(caps, a, q, j, a.PB[s], -1, 0) - Fq[q];
+      for (int s = 0; s < S; s++) Fb[s] = fill<QM, VM>(caps, a, s / VM, s % VM, a.PB[s], -1, 0) - Fq[s / VM];
+      // The K^2 candidates of this prefix in increasing index order, spread
+      // over 4 independent running maxima (candidate (sa, sb) -> accumulator
+      // (sb + 1) & 3) so the compare chains overlap; each accumulator sees its
+      // candidates in index order and keeps the first maximum, and the merge
+      // below prefers the lower index on equal scores.  Pad slots (code 0,
+      // capacity 0) score exactly like the idle option with the same index,
+      // so they can never change the result.
+      uint64_t lb[4] = {best_s, best_s, best_s, best_s};
+      int lp[4] = {-1, -1, -1, -1};
+      if (base > lb[0] || best_i == ~0ull) { lb[0] = base; lp[0] = 0; }
+#pragma unroll
+      for (int sb = 0; sb < S; sb++) {
+        const uint64_t c = base + Fb[sb];
+        if (c > lb[(sb + 1) & 3]) { lb[(sb + 1) & 3] = c; lp[(sb + 1) & 3] = a.code[sb]; }
       }
-      // the K^2 candidates of this prefix, in increasing index order
-      uint64_t lb = best_s;
-      int lp = -1;
-      if (base > lb || best_i == ~0ull) { lb = base; lp = 0; }
-#pragma unroll
-      for (int sb = 0; sb < S; sb++)
-        if (a.code[sb]) {
-          const uint64_t c = base + Fb[sb];
-          if (c > lb) { lb = c; lp = a.code[sb]; }
-        }
 #pragma unroll
       for (int sa = 0; sa < S; sa++) {
-        if (!a.code[sa]) continue;
-        const uint64_t ba = base + Fa[sa];
-        if (ba > lb) { lb = ba; lp = a.code[sa] * K; }
+        const int qa = sa / VM;
+        const uint64_t ba = base + fill<QM, VM>(caps, a, qa, sa % VM, a.PA[sa], -1, 0) - Fq[qa];
+        if (ba > lb[0]) { lb[0] = ba; lp[0] = a.code[sa] * K; }
 #pragma unroll
         for (int sb = 0; sb < S; sb++) {
-          if (!a.code[sb]) continue;
           uint64_t c;
-          if (sa / VM == sb / VM) {
-            const int q = sa / VM;
-            c = base - Fq[q] + fill<QM, VM>(caps, a, q, sa % VM, a.PA[sa], sb % VM, a.PB[sb]);
-          } else {
+          if (qa == sb / VM)
+            c = base - Fq[qa] + fill<QM, VM>(caps, a, qa, sa % VM, a.PA[sa], sb % VM, a.PB[sb]);
+          else
             c = ba + Fb[sb];
-          }
-          if (c > lb) { lb = c; lp = a.code[sa] * K + a.code[sb]; }
+          if (c > lb[(sb + 1) & 3]) { lb[(sb + 1) & 3] = c; lp[(sb + 1) & 3] = a.code[sa] * K + a.code[sb]; }
         }
       }
-      if (lp >= 0) { best_s = lb; best_i = p * KK + (uint64_t)lp; }
+      uint64_t mb = lb[0];
+      int mp = lp[0];
+#pragma unroll
+      for (int k = 1; k < 4; k++)
+        if (lp[k] >= 0 && (lb[k] > mb || (lb[k] == mb && (mp < 0 || lp[k] < mp)))) { mb = lb[k]; mp = lp[k]; }
+      if (mp >= 0) { best_s = mb; best_i = p * KK + (uint64_t)mp; }
       if (++p >= pend) break;
       if (++dig[D - 3] == K) {
         dig[D - 3] = 0;

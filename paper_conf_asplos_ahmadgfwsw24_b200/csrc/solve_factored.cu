@@ -168,6 +168,96 @@ __global__ void __launch_bounds__(FG_WARPS * 32) k_fact_g(const __grid_constant_
   }
 }
 
+// Batched variant for many demand vectors: the count vectors of a (family,
+// usage) cell and their capacity vectors do not depend on the demand, only
+// the water-fill does.  One warp per (family, usage, 32 vectors): the warp
+// walks the cell's candidates once in lexicographic-rank order (uniform
+// control flow, broadcast loads; type T-1 fastest, so ranks ascend), every
+// lane water-fills for its own vector and keeps its first maximum.
+template <int VMT>
+__global__ void __launch_bounds__(128) k_fact_gv(const __grid_constant__ FactLayout f, int n_vec,
+                                                 const int32_t *__restrict__ demand,
+                                                 const int32_t *__restrict__ slot_acc, BestRec *g) {
+  const int lane = threadIdx.x & 31;
+  const int item = blockIdx.x * 4 + (threadIdx.x >> 5);
+  if (item >= f.Q * f.U) return;
+  const int q = item / f.U, ukey = item % f.U;
+  const int vec = blockIdx.y * 32 + lane;
+  const bool active = vec < n_vec;
+  const int s = active ? demand[(size_t)vec * f.Q + q] : 0;
+  const int T = f.T, VM = f.VM;
+  int bsz[PX_MAXT], bst[PX_MAXT], o[PX_MAXT];
+  int64_t lstride[PX_MAXT];
+  bool empty = false;
+  {
+    int64_t ls = 1;
+    for (int t = T - 1; t >= 0; t--) {
+      const int ut = (ukey / f.ustride[t]) % (f.Nt[t] + 1);
+      const int32_t *bs = f.bstart + ((size_t)q * T + t) * (PX_MAXD + 2);
+      bst[t] = bs[ut];
+      bsz[t] = bs[ut + 1] - bs[ut];
+      empty |= bsz[t] == 0;
+      lstride[t] = ls;
+      ls *= f.L[q * T + t];
+      o[t] = 0;
+    }
+  }
+  uint64_t best_s = 0, best_i = ~0ull;
+  if (!empty) {
+    int A[VMT];
+#pragma unroll
+    for (int j = 0; j < VMT; j++) A[j] = j < VM ? slot_acc[q * VM + j] : 0;
+    const int tl = T - 1;
+    const int32_t *binner = f.bucket + f.list_off[q][tl] + bst[tl];
+    const int32_t *einner = f.ecap + f.list_off[q][tl] * VM;
+    int pcap[VMT];
+    uint64_t psub = 0;
+    auto outer = [&]() {  // capacity and rank contribution of types 0..T-2
+#pragma unroll
+      for (int j = 0; j < VMT; j++) pcap[j] = 0;
+      psub = 0;
+      for (int t = 0; t < tl; t++) {
+        const int r = f.bucket[f.list_off[q][t] + bst[t] + o[t]];
+        psub += (uint64_t)r * lstride[t];
+        const int32_t *ec = f.ecap + (f.list_off[q][t] + r) * VM;
+#pragma unroll
+        for (int j = 0; j < VMT; j++) pcap[j] += j < VM ? ec[j] : 0;
+      }
+    };
+    outer();
+    for (;;) {
+      for (int k = 0; k < bsz[tl]; k++) {
+        const int r = binner[k];
+        const int32_t *ec = einner + (size_t)r * VM;
+        const uint64_t sub = psub + (uint64_t)r * lstride[tl];
+        int rem = s;
+        uint64_t acc = 0;
+#pragma unroll
+        for (int j = 0; j < VMT; j++) {
+          const int c = pcap[j] + (j < VM ? ec[j] : 0);
+          const int tk = min(rem, c);
+          acc += (uint64_t)(uint32_t)A[j] * (uint32_t)tk;
+          rem -= tk;
+        }
+        const uint64_t sc = px_pack((uint32_t)(s - rem), acc);
+        if (sc > best_s || best_i == ~0ull) { best_s = sc; best_i = sub; }
+      }
+      int t = tl - 1;
+      for (; t >= 0; t--) {
+        if (++o[t] < bsz[t]) break;
+        o[t] = 0;
+      }
+      if (t < 0) break;
+      outer();
+    }
+  }
+  if (active) {
+    BestRec &out = g[((size_t)vec * f.Q + q) * f.U + ukey];
+    out.score = best_s;
+    out.index = best_i;  // ~0 when no count vector has this usage
+  }
+}
+
 // ---------------------------------------------------------------- DP ----
 __device__ __forceinline__ void ukey_decode(const FactLayout &f, int key, int *u) {
   for (int t = 0; t < f.T; t++) u[t] = (key / f.ustride[t]) % (f.Nt[t] + 1);
@@ -373,8 +463,14 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
   if (!g || !G) return px_fail(ctx, PROTEUS_ENOMEM, "factored DP buffers");
   PX_LAUNCH(ctx, "fact_lists", k_fact_lists, (Q * T + 63) / 64, 64, 0, f, tab.P, tab.slot_of, ctx->M);
   const int64_t nitems = (int64_t)n_vec * Q * U;
-  PX_LAUNCH(ctx, "fact_g", k_fact_g, (unsigned)((nitems + FG_WARPS - 1) / FG_WARPS), FG_WARPS * 32, 0, f, n_vec,
-            d_demand, tab.slot_acc, g);
+  if (n_vec >= 8 && VM <= 8) {
+    dim3 grid((unsigned)((Q * U + 3) / 4), (unsigned)((n_vec + 31) / 32));
+    if (VM <= 4) PX_LAUNCH(ctx, "fact_g", k_fact_gv<4>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
+    else PX_LAUNCH(ctx, "fact_g", k_fact_gv<8>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
+  } else {
+    PX_LAUNCH(ctx, "fact_g", k_fact_g, (unsigned)((nitems + FG_WARPS - 1) / FG_WARPS), FG_WARPS * 32, 0, f, n_vec,
+              d_demand, tab.slot_acc, g);
+  }
   const size_t dsmem = (size_t)2 * U * 8;
   if (dsmem > 200 * 1024) return px_fail(ctx, PROTEUS_ERANGE, "usage lattice %lld too large for the DP", (long long)U);
   if (dsmem > 48 * 1024)
