@@ -331,8 +331,9 @@ __global__ void k_spec(const __grid_constant__ LaneArgs a) {
   const int64_t i0 = (int64_t)c * win;
   const int wlen = (int)(a.N - i0 < win ? a.N - i0 : win);
   const int stage_cap = win + nw * a.bmax;
-  uint32_t *tile = sm;                                          // [32][win] if use_tile
-  int32_t *sT = (int32_t *)(sm + (a.use_tile ? 32 * win : 0));  // [nw][bmax]
+  const int tstride = win + 1;                                   // padded rows: no bank conflicts
+  uint32_t *tile = sm;                                          // [32][tstride] if use_tile
+  int32_t *sT = (int32_t *)(sm + (a.use_tile ? 32 * tstride : 0));  // [nw][bmax]
   uint32_t *sA = (uint32_t *)(sT + nw * a.bmax);                // staged arrivals [stage_cap]
   uint32_t *sI = sA + stage_cap;                                // staged query indices [stage_cap]
   const int64_t tile0 = (int64_t)c * a.win_tiles;
@@ -347,7 +348,7 @@ __global__ void k_spec(const __grid_constant__ LaneArgs a) {
   const int stage = host ? (int)(len + look) : 0;
   if (lane == 0) sStage[w] = stage;
   if (a.use_tile)
-    for (int k = threadIdx.x; k < 32 * win; k += blockDim.x) tile[k] = 0xFFFFFFFFu;
+    for (int k = threadIdx.x; k < 32 * tstride; k += blockDim.x) tile[k] = 0xFFFFFFFFu;
   __syncthreads();
   if (threadIdx.x == 0) {
     int acc = 0;
@@ -372,7 +373,7 @@ __global__ void k_spec(const __grid_constant__ LaneArgs a) {
   if (host && si < a.nsc) {
     const int s = a.sc_list[si];
     const LaneP p = lane_params(a, s, d, T);
-    uint32_t *out = a.use_tile ? tile + (size_t)lane * win : a.lat_out + (size_t)s * a.N;
+    uint32_t *out = a.use_tile ? tile + (size_t)lane * tstride : a.lat_out + (size_t)s * a.N;
     const uint32_t obase = a.use_tile ? (uint32_t)i0 : 0u;
     int64_t h = 0, F = 0;
     if (p.Bmax < 1) {
@@ -401,7 +402,7 @@ __global__ void k_spec(const __grid_constant__ LaneArgs a) {
   for (int r = 0; r < 32; r++) {
     if (sg * 32 + r >= a.nsc) break;
     uint32_t *row = a.lat_out + (size_t)a.sc_list[sg * 32 + r] * a.N + i0;
-    const uint32_t *tr = tile + (size_t)r * win;
+    const uint32_t *tr = tile + (size_t)r * tstride;
     for (int k = threadIdx.x; k < wlen; k += blockDim.x) row[k] = tr[k];
   }
 }
@@ -474,8 +475,44 @@ __device__ __forceinline__ int decide_warp(const Arr &A, int64_t n, int64_t h, i
   return b;
 }
 
+// The same decision with the serial Case-2 loop replaced by one ballot over
+// up to 32 queue states: state k holds k + 1 queries at tau_k = max(t0,
+// a[h + k]); it is "complete" when the next arrival comes strictly later (or
+// the queue is at Bmax), and the batch leaves at the first complete state that
+// must dispatch now (k + 1 = Bmax, or tau_k >= Tmax_wait(k + 2)) or whose
+// timer Tmax_wait(k + 2) fires before the next arrival.  Ts[b - 1] = T(b).
+template <class Arr>
+__device__ __forceinline__ int decide_par(const Arr &A, int64_t n, int64_t h, int64_t F, int Bmax, int64_t L,
+                                          const int32_t *Ts, int lane, int64_t *t_out) {
+  const int64_t ah = A(h);
+  const int64_t t0 = F > ah ? F : ah;
+  const int q0 = count_le(A, n, h, 1, Bmax, t0, lane);
+  for (int kb = q0 - 1;; kb += 32) {
+    const int k = kb + lane;
+    const bool valid = k + 1 <= Bmax && h + k < n;
+    bool stop = false, now = false;
+    int64_t tau = 0, W = 0;
+    if (valid) {
+      const int64_t ak = A(h + k);
+      tau = ak > t0 ? ak : t0;
+      const bool capped = k + 1 == Bmax;
+      const int64_t nxt = h + k + 1 < n ? (int64_t)A(h + k + 1) : INT64_MAX;
+      W = capped ? 0 : ah + L - Ts[k + 1];
+      now = capped || tau >= W;
+      stop = (capped || nxt > tau) && (now || nxt > W);
+    }
+    const unsigned bal = __ballot_sync(0xffffffffu, stop);
+    if (bal) {
+      const int src = __ffs(bal) - 1;
+      const int64_t ts = __shfl_sync(0xffffffffu, now ? tau : W, src);
+      *t_out = ts;
+      return kb + src + 1;
+    }
+  }
+}
+
 __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs a) {
-  extern __shared__ uint32_t ssm[];  // [4 warps][2][SBUF]
+  extern __shared__ uint32_t ssm[];  // [4 warps][2][SBUF], then [4 warps][bmax] latencies T
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t gw = (int64_t)blockIdx.x * 4 + w;
   if (gw >= (int64_t)a.nsc * a.D || a.nwin < 2) return;
@@ -485,7 +522,10 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   if (n == 0) return;
   uint32_t *bufA = ssm + (size_t)w * 2 * SBUF, *bufI = bufA + SBUF;
   const uint32_t *garr = a.devArr + a.devOff[d], *gix = a.devIdx + a.devOff[d];
-  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  int32_t *T = (int32_t *)(ssm + 4 * 2 * SBUF) + w * a.bmax;
+  for (int k = lane; k < a.bmax; k += 32) T[k] = Tg[k];
+  __syncwarp();
   const LaneP p = lane_params(a, s, d, T);
   if (p.Bmax < 1) return;
   uint32_t *out = a.lat_out + (size_t)s * a.N;
@@ -542,6 +582,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         F = eF;
         continue;
       }
+      int checks = 4;  // meeting tests per window (each costs a global round trip)
       while (h < en) {
         ensure(h);
         if (F > (int64_t)A(h) && h + p.Bmax - 1 < n && (int64_t)A(h + p.Bmax - 1) <= F) {
@@ -564,11 +605,12 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
           continue;
         }
         int64_t t;
-        const int b = decide_warp(A, n, h, F, p.Bmax, p.L, T, lane, &t);
+        const int b = decide_par(A, n, h, F, p.Bmax, p.L, T, lane, &t);
         const int64_t Fn = t + T[b - 1];
         const int64_t j2 = h + b;
         bool conv = false;
-        if (t > F && j2 < en) {
+        if (t > F && j2 < en && checks > 0) {
+          checks--;
           const int64_t f1 = (int64_t)A(j2 - 1) + out[IX(j2 - 1)];
           const int64_t f2 = (int64_t)A(j2) + out[IX(j2)];
           conv = f1 == Fn && f2 != Fn;
@@ -732,7 +774,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   const int ndg = (D + 31) / 32;
   int use_tile = ndg == 1 && !env_int("PROTEUS_REPLAY_NO_TILE", 0);
   auto spec_smem = [&](int tile) {
-    return ((size_t)(tile ? 32 * win : 0) + (size_t)dpb * ctx->bmax + 2 * ((size_t)win + (size_t)dpb * ctx->bmax)) * 4;
+    return ((size_t)(tile ? 32 * (win + 1) : 0) + (size_t)dpb * ctx->bmax + 2 * ((size_t)win + (size_t)dpb * ctx->bmax)) * 4;
   };
   if (use_tile && spec_smem(1) > 200 * 1024) use_tile = 0;
   const size_t smem = spec_smem(use_tile);
@@ -743,7 +785,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
     if (smem > 48 * 1024)
       PX_CUDA(ctx, cudaFuncSetAttribute(k_spec, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    PX_CUDA(ctx, cudaFuncSetAttribute(k_stitch, cudaFuncAttributeMaxDynamicSharedMemorySize, 4 * 2 * SBUF * 4));
+    PX_CUDA(ctx, cudaFuncSetAttribute(k_stitch, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      4 * 2 * SBUF * 4 + 4 * ctx->bmax * 4));
   }
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
@@ -763,7 +806,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       dim3 grid(nwin, (la.nsc + 31) / 32, ndg);
       PX_LAUNCH(ctx, "replay_spec", k_spec, grid, dpb * 32, smem, la);
       const int64_t warps = (int64_t)la.nsc * D;
-      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 4 * 2 * SBUF * 4, la);
+      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 4 * 2 * SBUF * 4 + 4 * ctx->bmax * 4,
+                la);
     }
     if (simple || !la.use_tile) {
       dim3 g(64, la.nsc < 65535 ? la.nsc : 65535);
