@@ -190,10 +190,10 @@ __global__ void k_dev_offsets(const int64_t *__restrict__ totals, int n, int64_t
   }
 }
 
-// stable scatter into device-major arrays
+// stable scatter into device-major arrays; inv[i] = device-major position of query i
 __global__ void k_scatter(const uint8_t *__restrict__ target, const uint32_t *__restrict__ arr, int64_t N, int D,
                           const int32_t *__restrict__ devBase, const int64_t *__restrict__ devOff, uint32_t *devArr,
-                          uint32_t *devIdx) {
+                          uint32_t *inv) {
   __shared__ int64_t run[TILE_WARPS][PX_MAXD + 2];
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t tile = (int64_t)blockIdx.x * TILE_WARPS + w;
@@ -212,46 +212,61 @@ __global__ void k_scatter(const uint8_t *__restrict__ target, const uint32_t *__
     __syncwarp();
     if (valid && lane == __ffs(peers) - 1) run[w][key] += __popc(peers);
     __syncwarp();
-    if (valid) { devArr[pos] = arr[i]; devIdx[pos] = (uint32_t)i; }
+    if (valid) { devArr[pos] = arr[i]; inv[i] = (uint32_t)pos; }
   }
 }
 
 // --------------------------------------------------------------- lanes ----
+// Latencies are produced in device-major order (latd[s][p], p = position in
+// the per-device arrays), which every lane writes sequentially; k_unpermute
+// turns them into per-query order at the end.
 struct SpecExit {
   int64_t F;
-  int32_t ov;  // exit head - window end (overhang of the last batch into the next window)
+  int32_t ov;  // exit head - chunk end (overhang of the last batch into the next chunk)
   int32_t pad;
 };
 
-struct LaneArgs {
-  int S, D, M, bmax, Q;
-  int64_t N, ntiles;
-  const int32_t *option, *dev_type, *fam_of_m, *acc, *lat, *slo_base;
-  const proteus_scenario *sc;
-  // one routing mode
-  int nsc, win_tiles, nwin, use_tile;
-  const int32_t *sc_list;
-  const int64_t *devOff;   // [D + 2]
-  const int32_t *devBase;  // [ntiles + 1][D + 1]
-  const uint32_t *devArr, *devIdx;
-  uint32_t *lat_out;       // [S][N]
-  SpecExit *ex;            // [S][D][nwin]
+struct LaneParam {  // per (scenario, device)
+  int32_t Bmax;     // min(cap, depth) (R4); 0 for idle devices
+  uint32_t A;       // accuracy of the hosted variant
+  int64_t L;        // scenario SLO of the hosted family (R12)
 };
 
-struct LaneP {
-  int Bmax;
-  int64_t L;
-};
-
-__device__ __forceinline__ LaneP lane_params(const LaneArgs &a, int s, int d, const int32_t *T) {
-  int depth = 0;
-  while (depth < a.bmax && T[depth] > 0) depth++;
-  const proteus_scenario sc = a.sc[s];
-  LaneP p;
-  p.Bmax = (sc.batch_cap > 0 && sc.batch_cap < depth) ? sc.batch_cap : depth;  // R4
-  p.L = (int64_t)sc.slo_mult_milli * a.slo_base[a.fam_of_m[a.option[d] - 1]] / 1000;  // R12
-  return p;
+__global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__restrict__ option,
+                              const int32_t *__restrict__ dev_type, const int32_t *__restrict__ fam_of_m,
+                              const int32_t *__restrict__ acc, const int32_t *__restrict__ lat,
+                              const int32_t *__restrict__ slo_base, const proteus_scenario *__restrict__ sc,
+                              LaneParam *lp) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= S * D) return;
+  const int s = i / D, d = i % D;
+  LaneParam p = {0, 0, 0};
+  const int o = option[d];
+  if (o > 0) {
+    const int32_t *T = lat + ((size_t)dev_type[d] * M + (o - 1)) * bmax;
+    int depth = 0;
+    while (depth < bmax && T[depth] > 0) depth++;
+    const int cap = sc[s].batch_cap;
+    p.Bmax = (cap > 0 && cap < depth) ? cap : depth;
+    p.A = (uint32_t)acc[o - 1];
+    p.L = (int64_t)sc[s].slo_mult_milli * slo_base[fam_of_m[o - 1]] / 1000;
+  }
+  lp[i] = p;
 }
+
+struct LaneArgs {
+  int S, D, M, bmax, nsc, CH;
+  int64_t N, NCH;
+  const int32_t *option, *dev_type, *lat, *sc_list;
+  const LaneParam *lp;
+  const int64_t *devOff;  // [D + 2]; segment D = the sink
+  const int64_t *choff;   // [D + 1] chunk offsets
+  const int32_t *goff;    // [D + 1] phase-A warp-group offsets
+  const uint32_t *devArr;
+  uint32_t *latd;         // [S][N] device-major
+  SpecExit *ex;           // [S][NCH]
+  uint64_t *agg;          // [3][S]
+};
 
 __device__ __forceinline__ uint32_t sat_lat(int64_t l) { return l >= 0xFFFFFFFFll ? 0xFFFFFFFEu : (uint32_t)l; }
 
@@ -282,146 +297,133 @@ __device__ __forceinline__ int decide(const Arr &arr, int64_t n, int64_t h, int6
   return b;
 }
 
-struct PtrArr {
+struct GArr {
   const uint32_t *p;
-  __device__ __forceinline__ uint32_t operator()(int64_t j) const { return p[j]; }
+  __device__ __forceinline__ uint32_t operator()(int64_t j) const { return __ldg(p + j); }
 };
+
+__device__ __forceinline__ void count_lat(uint32_t l, const LaneParam &p, unsigned long long &viol,
+                                          unsigned long long &ont, unsigned long long &accs) {
+  if ((int64_t)l > p.L) viol++;
+  else { ont++; accs += p.A; }
+}
+
+__device__ __forceinline__ void warp_add_counts(unsigned long long v, unsigned long long o, unsigned long long ac,
+                                                uint64_t *agg, int S, int s, int lane) {
+  for (int k = 16; k; k >>= 1) {
+    v += __shfl_xor_sync(0xffffffffu, v, k);
+    o += __shfl_xor_sync(0xffffffffu, o, k);
+    ac += __shfl_xor_sync(0xffffffffu, ac, k);
+  }
+  if (lane == 0) {
+    if (v) atomicAdd((unsigned long long *)&agg[s], v);
+    if (o) atomicAdd((unsigned long long *)&agg[S + s], o);
+    if (ac) atomicAdd((unsigned long long *)&agg[2 * S + s], ac);
+  }
+}
 
 // ---- fallback: one thread per (device, scenario) walks the whole array
 __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ LaneArgs a) {
   const int lane_id = blockIdx.x * blockDim.x + threadIdx.x;
   if (lane_id >= a.nsc * a.D) return;
   const int s = a.sc_list[lane_id / a.D], d = lane_id % a.D;
-  if (a.option[d] <= 0) return;
+  const LaneParam p = a.lp[s * a.D + d];
   const int64_t st = a.devOff[d], n = a.devOff[d + 1] - st;
   if (n == 0) return;
-  const uint32_t *idx = a.devIdx + st;
-  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
-  const LaneP p = lane_params(a, s, d, T);
-  uint32_t *out = a.lat_out + (size_t)s * a.N;
-  if (p.Bmax < 1) {  // cannot run even batch 1: never routed to (z = 0 / depth 0), kept for safety
-    for (int64_t j = 0; j < n; j++) out[idx[j]] = 0xFFFFFFFFu;
-    return;
+  uint32_t *out = a.latd + (size_t)s * a.N + st;
+  unsigned long long viol = 0, ont = 0, accs = 0;
+  if (p.Bmax < 1) {  // never routed to (z = 0 / depth 0); kept for safety
+    for (int64_t j = 0; j < n; j++) out[j] = 0xFFFFFFFFu;
+    viol = n;
+  } else {
+    const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+    GArr arr{a.devArr + st};
+    int64_t h = 0, F = 0;  // R13
+    while (h < n) {
+      int64_t t;
+      const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
+      F = t + T[b - 1];
+      for (int j = 0; j < b; j++) {
+        const uint32_t l = sat_lat(F - (int64_t)arr(h + j));
+        out[h + j] = l;
+        count_lat(l, p, viol, ont, accs);
+      }
+      h += b;
+    }
   }
-  PtrArr arr{a.devArr + st};
-  int64_t h = 0, F = 0;  // R13
-  while (h < n) {
-    int64_t t;
-    const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
-    F = t + T[b - 1];
-    for (int j = 0; j < b; j++) out[idx[h + j]] = sat_lat(F - (int64_t)arr(h + j));
-    h += b;
-  }
+  atomicAdd((unsigned long long *)&a.agg[s], viol);
+  atomicAdd((unsigned long long *)&a.agg[a.S + s], ont);
+  atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], accs);
 }
 
-// ---- phase A: speculative windows
-// grid (nwin, scenario groups of 32, device groups of 32); warp = device,
-// lane = scenario.  A window's arrivals and query indices of every device are
-// staged in shared memory.  With use_tile (one device group) the window's
-// output rows of the block's 32 scenarios are assembled in shared memory
-// (initialised to "dropped" so sink queries need no extra pass) and flushed
-// with coalesced stores.
-__global__ void k_spec(const __grid_constant__ LaneArgs a) {
-  extern __shared__ uint32_t sm[];
-  __shared__ int sOff[33], sStage[32];
-  const int c = blockIdx.x, sg = blockIdx.y, dg = blockIdx.z;
-  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
-  const int d = dg * 32 + w;
-  const int win = a.win_tiles * TILE;
-  const int64_t i0 = (int64_t)c * win;
-  const int wlen = (int)(a.N - i0 < win ? a.N - i0 : win);
-  const int stage_cap = win + nw * a.bmax;
-  const int tstride = win + 1;                                   // padded rows: no bank conflicts
-  uint32_t *tile = sm;                                          // [32][tstride] if use_tile
-  int32_t *sT = (int32_t *)(sm + (a.use_tile ? 32 * tstride : 0));  // [nw][bmax]
-  uint32_t *sA = (uint32_t *)(sT + nw * a.bmax);                // staged arrivals [stage_cap]
-  uint32_t *sI = sA + stage_cap;                                // staged query indices [stage_cap]
-  const int64_t tile0 = (int64_t)c * a.win_tiles;
-  const int64_t tile1 = tile0 + a.win_tiles < a.ntiles ? tile0 + a.win_tiles : a.ntiles;
-  const bool dvalid = d < a.D;
-  const int64_t n_d = dvalid ? a.devOff[d + 1] - a.devOff[d] : 0;
-  const int64_t st = dvalid ? a.devBase[tile0 * (a.D + 1) + d] : 0;
-  const int64_t en = dvalid ? a.devBase[tile1 * (a.D + 1) + d] : 0;
-  const int64_t len = en - st;
-  const bool host = dvalid && a.option[d] > 0 && len > 0;
-  const int64_t look = n_d - en < a.bmax ? n_d - en : a.bmax;
-  const int stage = host ? (int)(len + look) : 0;
-  if (lane == 0) sStage[w] = stage;
-  if (a.use_tile)
-    for (int k = threadIdx.x; k < 32 * tstride; k += blockDim.x) tile[k] = 0xFFFFFFFFu;
+// ---- phase A: speculative chunks
+// Each device array is cut into chunks of CH queries.  One warp per (device,
+// scenario, 32 consecutive chunks); lane = chunk, replayed from an idle
+// device (the true state at the start of the trace, R13).  All lanes follow
+// the same rule parameters, so the warp stays close to converged.
+__global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a) {
+  __shared__ int32_t sG[PX_MAXD + 1];
+  for (int k = threadIdx.x; k <= a.D; k += blockDim.x) sG[k] = a.goff[k];
   __syncthreads();
-  if (threadIdx.x == 0) {
-    int acc = 0;
-    for (int k = 0; k < nw; k++) { sOff[k] = acc; acc += sStage[k]; }
-    sOff[nw] = acc;
-  }
-  __syncthreads();
-  uint32_t *arr = sA + sOff[w];
-  uint32_t *ixs = sI + sOff[w];
-  const int32_t *T = sT + w * a.bmax;
-  if (host) {
-    const uint32_t *src = a.devArr + a.devOff[d] + st, *isrc = a.devIdx + a.devOff[d] + st;
-    for (int k = lane; k < stage; k += 32) {
-      arr[k] = src[k];
-      ixs[k] = k < len ? isrc[k] : 0;
-    }
-    const int32_t *row = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
-    for (int k = lane; k < a.bmax; k += 32) sT[w * a.bmax + k] = row[k];
-  }
-  __syncthreads();
-  const int si = sg * 32 + lane;
-  if (host && si < a.nsc) {
-    const int s = a.sc_list[si];
-    const LaneP p = lane_params(a, s, d, T);
-    uint32_t *out = a.use_tile ? tile + (size_t)lane * tstride : a.lat_out + (size_t)s * a.N;
-    const uint32_t obase = a.use_tile ? (uint32_t)i0 : 0u;
-    int64_t h = 0, F = 0;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int g = blockIdx.x * 4 + w;
+  if (g >= sG[a.D]) return;
+  int d = 0;
+  while (g >= sG[d + 1]) d++;
+  const int s = a.sc_list[blockIdx.y];
+  const LaneParam p = a.lp[s * a.D + d];
+  const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+  const int64_t nch = a.choff[d + 1] - a.choff[d];
+  const int64_t c = (int64_t)(g - sG[d]) * 32 + lane;
+  unsigned long long viol = 0, ont = 0, accs = 0;
+  if (c < nch) {
+    const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
+    uint32_t *out = a.latd + (size_t)s * a.N + off;
+    int64_t h = st, F = 0;
     if (p.Bmax < 1) {
-      if (!a.use_tile)
-        for (int64_t j = 0; j < len; j++) out[ixs[j] - obase] = 0xFFFFFFFFu;
-      h = len;
+      for (int64_t j = st; j < en; j++) out[j] = 0xFFFFFFFFu;
+      viol = en - st;
+      h = en;
     } else {
-      PtrArr A{arr};
-      while (h < len) {
+      const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+      GArr arr{a.devArr + off};
+      while (h < en) {
         int64_t t;
-        const int b = decide(A, stage, h, F, p.Bmax, p.L, T, &t);
+        const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
         F = t + T[b - 1];
-        const int64_t jend = h + b < len ? h + b : len;
-        for (int64_t j = h; j < jend; j++) out[ixs[j] - obase] = sat_lat(F - (int64_t)arr[j]);
+        const int64_t jend = h + b < en ? h + b : en;
+        for (int64_t j = h; j < jend; j++) {
+          const uint32_t l = sat_lat(F - (int64_t)arr(j));
+          out[j] = l;
+          count_lat(l, p, viol, ont, accs);
+        }
         h += b;
       }
     }
     SpecExit e;
     e.F = F;
-    e.ov = (int32_t)(h - len);
+    e.ov = (int32_t)(h - en);
     e.pad = 0;
-    a.ex[((size_t)s * a.D + d) * a.nwin + c] = e;
+    a.ex[(size_t)s * a.NCH + a.choff[d] + c] = e;
   }
-  if (!a.use_tile) return;
-  __syncthreads();
-  for (int r = 0; r < 32; r++) {
-    if (sg * 32 + r >= a.nsc) break;
-    uint32_t *row = a.lat_out + (size_t)a.sc_list[sg * 32 + r] * a.N + i0;
-    const uint32_t *tr = tile + (size_t)r * tstride;
-    for (int k = threadIdx.x; k < wlen; k += blockDim.x) row[k] = tr[k];
-  }
+  warp_add_counts(viol, ont, accs, a.agg, a.S, s, lane);
 }
 
 // ---- phase B: exact stitch, one warp per (device, scenario)
-// The true state (h, F) is carried from window to window.  A window whose
+// The true state (h, F) is carried from chunk to chunk.  A chunk whose
 // speculative start (its first query, device idle) equals the true state is
 // already right.  Otherwise the true run is replayed batch by batch until it
 // meets the speculative run: after a batch [h, j2) finishing at Fn, if the
 // speculative run also has a batch ending at j2 - 1 with finish Fn (its
 // latency + arrival) and a new batch at j2, both runs are in the same state
 // (j2, Fn) and agree from there on.  Only batches that the device waited for
-// (t > F) are tested: a batch dispatched the moment the previous one finished
-// can only meet a run that had already met.  Backlogged stretches (Bmax
-// queued when the device frees) are full batches back to back -- batch k
-// finishes at F + (k+1) T(Bmax) -- and are taken 32 batches per step with a
-// ballot.  The device's arrivals and query indices stream through a
-// shared-memory ring; window bounds and exit states are fetched 32 windows
-// at a time.
+// (t > F) are tested -- a batch dispatched the moment the previous one
+// finished can only meet a run that had already met -- and at most a few per
+// chunk.  Backlogged stretches (Bmax queued when the device frees) are full
+// batches back to back -- batch k finishes at F + (k+1) T(Bmax) -- and are
+// taken 32 batches per step with a ballot.  Rewritten latencies adjust the
+// counts by their difference from the speculative ones.  Arrivals stream
+// through a shared-memory ring; exit states are fetched 32 chunks at a time.
 #define SBUF 2048
 #define SAHEAD 1088
 
@@ -447,40 +449,12 @@ __device__ __forceinline__ int count_le(const Arr &A, int64_t n, int64_t h, int 
   }
 }
 
-// decide() with the counting done 32 arrivals at a time by the warp
-template <class Arr>
-__device__ __forceinline__ int decide_warp(const Arr &A, int64_t n, int64_t h, int64_t F, int Bmax, int64_t L,
-                                           const int32_t *T, int lane, int64_t *t_out) {
-  const int64_t ah = A(h);
-  int64_t t = F > ah ? F : ah;
-  int q = count_le(A, n, h, 1, Bmax, t, lane);
-  int b;
-  for (;;) {
-    if (q >= Bmax) { b = Bmax; break; }
-    const int64_t W = ah + L - T[q];
-    if (t >= W) { b = q; break; }
-    if (h + q < n) {
-      const int64_t nx = A(h + q);
-      if (nx <= W) {
-        t = nx;
-        q = count_le(A, n, h, q, Bmax, t, lane);
-        continue;
-      }
-    }
-    t = W;
-    b = q;
-    break;
-  }
-  *t_out = t;
-  return b;
-}
-
-// The same decision with the serial Case-2 loop replaced by one ballot over
-// up to 32 queue states: state k holds k + 1 queries at tau_k = max(t0,
-// a[h + k]); it is "complete" when the next arrival comes strictly later (or
-// the queue is at Bmax), and the batch leaves at the first complete state that
-// must dispatch now (k + 1 = Bmax, or tau_k >= Tmax_wait(k + 2)) or whose
-// timer Tmax_wait(k + 2) fires before the next arrival.  Ts[b - 1] = T(b).
+// decide() with the serial Case-2 loop replaced by one ballot over up to 32
+// queue states: state k holds k + 1 queries at tau_k = max(t0, a[h + k]); it
+// is "complete" when the next arrival comes strictly later (or the queue is
+// at Bmax), and the batch leaves at the first complete state that must
+// dispatch now (k + 1 = Bmax, or tau_k >= Tmax_wait(k + 2)) or whose timer
+// Tmax_wait(k + 2) fires before the next arrival.  Ts[b - 1] = T(b).
 template <class Arr>
 __device__ __forceinline__ int decide_par(const Arr &A, int64_t n, int64_t h, int64_t F, int Bmax, int64_t L,
                                           const int32_t *Ts, int lane, int64_t *t_out) {
@@ -504,32 +478,30 @@ __device__ __forceinline__ int decide_par(const Arr &A, int64_t n, int64_t h, in
     const unsigned bal = __ballot_sync(0xffffffffu, stop);
     if (bal) {
       const int src = __ffs(bal) - 1;
-      const int64_t ts = __shfl_sync(0xffffffffu, now ? tau : W, src);
-      *t_out = ts;
+      *t_out = __shfl_sync(0xffffffffu, now ? tau : W, src);
       return kb + src + 1;
     }
   }
 }
 
 __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs a) {
-  extern __shared__ uint32_t ssm[];  // [4 warps][2][SBUF], then [4 warps][bmax] latencies T
+  extern __shared__ uint32_t ssm[];  // [4 warps][SBUF] arrivals, then [4 warps][bmax] T
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t gw = (int64_t)blockIdx.x * 4 + w;
-  if (gw >= (int64_t)a.nsc * a.D || a.nwin < 2) return;
+  if (gw >= (int64_t)a.nsc * a.D) return;
   const int s = a.sc_list[gw / a.D], d = (int)(gw % a.D);
-  if (a.option[d] <= 0) return;
-  const int64_t n = a.devOff[d + 1] - a.devOff[d];
-  if (n == 0) return;
-  uint32_t *bufA = ssm + (size_t)w * 2 * SBUF, *bufI = bufA + SBUF;
-  const uint32_t *garr = a.devArr + a.devOff[d], *gix = a.devIdx + a.devOff[d];
+  const LaneParam p = a.lp[s * a.D + d];
+  const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+  const int64_t nch = a.choff[d + 1] - a.choff[d];
+  if (p.Bmax < 1 || nch < 2) return;
+  uint32_t *bufA = ssm + (size_t)w * SBUF;
+  int32_t *T = (int32_t *)(ssm + 4 * SBUF) + w * a.bmax;
   const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
-  int32_t *T = (int32_t *)(ssm + 4 * 2 * SBUF) + w * a.bmax;
   for (int k = lane; k < a.bmax; k += 32) T[k] = Tg[k];
   __syncwarp();
-  const LaneP p = lane_params(a, s, d, T);
-  if (p.Bmax < 1) return;
-  uint32_t *out = a.lat_out + (size_t)s * a.N;
-  const SpecExit *ex = a.ex + ((size_t)s * a.D + d) * a.nwin;
+  const uint32_t *garr = a.devArr + off;
+  uint32_t *out = a.latd + (size_t)s * a.N + off;
+  const SpecExit *ex = a.ex + (size_t)s * a.NCH + a.choff[d];
   BufArr A{bufA, garr, -(int64_t)(4 * SBUF)};
   auto ensure = [&](int64_t h) {
     if (h >= A.base && h + SAHEAD <= A.base + SBUF) return;
@@ -538,42 +510,39 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
     for (int k = lane; k < SBUF; k += 32) {
       const int64_t j = A.base + k;
       bufA[k] = j < n ? garr[j] : 0xFFFFFFFFu;
-      bufI[k] = j < n ? gix[j] : 0u;
     }
     __syncwarp();
   };
-  auto IX = [&](int64_t j) -> uint32_t {
-    const int64_t o = j - A.base;
-    return (o >= 0 && o < SBUF) ? bufI[o] : __ldg(gix + j);
-  };
-  auto write_batch = [&](int64_t lo, int64_t hi, int64_t Fb) {
-    for (int64_t j = lo + lane; j < hi; j += 32) out[IX(j)] = sat_lat(Fb - (int64_t)A(j));
+  long long dv = 0, dont = 0, dacc = 0;
+  auto put = [&](int64_t j, int64_t Fb) {
+    const uint32_t nl = sat_lat(Fb - (int64_t)A(j));
+    const uint32_t ol = out[j];
+    out[j] = nl;
+    const int nv = (int64_t)nl > p.L, ov = (int64_t)ol > p.L;
+    dv += nv - ov;
+    dont += ov - nv;
+    dacc += ((long long)ov - (long long)nv) * (long long)p.A;
   };
   const int64_t TB = T[p.Bmax - 1];
-  const int64_t nwin = a.nwin;
-  auto tile_of = [&](int64_t c) { return c * a.win_tiles < a.ntiles ? c * a.win_tiles : a.ntiles; };
-  int64_t h = a.devBase[tile_of(1) * (a.D + 1) + d] + ex[0].ov, F = ex[0].F;
-  for (int64_t c0 = 1; c0 < nwin; c0 += 32) {
-    // lane k prefetches window c0 + k: its start, end and speculative exit
-    const int64_t ck = c0 + lane;
-    int64_t pst = 0, pen = 0, pF = 0;
+  const int64_t CH = a.CH;
+  int64_t h = (CH < n ? CH : n) + ex[0].ov, F = ex[0].F;
+  for (int64_t c0 = 1; c0 < nch; c0 += 32) {
+    int64_t pF = 0;
     int pov = 0;
-    if (ck < nwin) {
-      pst = a.devBase[tile_of(ck) * (a.D + 1) + d];
-      pen = a.devBase[tile_of(ck + 1) * (a.D + 1) + d];
-      const SpecExit e = ex[ck];
+    if (c0 + lane < nch) {
+      const SpecExit e = ex[c0 + lane];
       pF = e.F;
       pov = e.ov;
     }
-    const int cnt = nwin - c0 < 32 ? (int)(nwin - c0) : 32;
+    const int cnt = nch - c0 < 32 ? (int)(nch - c0) : 32;
     for (int k = 0; k < cnt; k++) {
-      const int64_t st = __shfl_sync(0xffffffffu, pst, k), en = __shfl_sync(0xffffffffu, pen, k);
+      const int64_t st = (c0 + k) * CH, en = st + CH < n ? st + CH : n;
       const int64_t eF = __shfl_sync(0xffffffffu, pF, k);
       const int eov = __shfl_sync(0xffffffffu, pov, k);
-      if (en == st) continue;
-      if (h > st) {  // queries of this window in the last batch of the previous one
+      if (h > st) {  // queries of this chunk in the last batch of the previous one
         ensure(st);
-        write_batch(st, h < en ? h : en, F);
+        const int64_t hi = h < en ? h : en;
+        for (int64_t j = st + lane; j < hi; j += 32) put(j, F);
       }
       if (h >= en) continue;
       ensure(h);
@@ -582,7 +551,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         F = eF;
         continue;
       }
-      int checks = 4;  // meeting tests per window (each costs a global round trip)
+      int checks = 2;
       while (h < en) {
         ensure(h);
         if (F > (int64_t)A(h) && h + p.Bmax - 1 < n && (int64_t)A(h + p.Bmax - 1) <= F) {
@@ -596,10 +565,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
           const unsigned bal = __ballot_sync(0xffffffffu, ok);
           const int r = bal == 0xffffffffu ? 32 : __ffs(~bal) - 1;
           const int64_t nq = (int64_t)r * p.Bmax;
-          for (int64_t i = lane; i < nq; i += 32) {
-            const int64_t kk = i / p.Bmax, j = h + i;
-            out[IX(j)] = sat_lat(F + (kk + 1) * TB - (int64_t)A(j));
-          }
+          for (int64_t i = lane; i < nq; i += 32) put(h + i, F + (i / p.Bmax + 1) * TB);
           h += nq;
           F += (int64_t)r * TB;
           continue;
@@ -611,12 +577,11 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         bool conv = false;
         if (t > F && j2 < en && checks > 0) {
           checks--;
-          const int64_t f1 = (int64_t)A(j2 - 1) + out[IX(j2 - 1)];
-          const int64_t f2 = (int64_t)A(j2) + out[IX(j2)];
-          conv = f1 == Fn && f2 != Fn;
+          conv = (int64_t)A(j2 - 1) + out[j2 - 1] == Fn && (int64_t)A(j2) + out[j2] != Fn;
         }
         __syncwarp();
-        write_batch(h, j2 < en ? j2 : en, Fn);
+        const int64_t hi = j2 < en ? j2 : en;
+        for (int64_t j = h + lane; j < hi; j += 32) put(j, Fn);
         h = j2;
         F = Fn;
         if (conv) {
@@ -627,58 +592,35 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
       }
     }
   }
+  warp_add_counts((unsigned long long)dv, (unsigned long long)dont, (unsigned long long)dacc, a.agg, a.S, s, lane);
 }
 
-// dropped queries (the sink segment, device index D): latency UINT32_MAX (R7)
-__global__ void k_sink(int64_t N, int D, const int32_t *__restrict__ sc_list, int nsc, const int64_t *devOff,
-                       const uint32_t *devIdx, uint32_t *lat_out) {
+// dropped queries (the sink segment, device index D): latency UINT32_MAX (R7), violations
+__global__ void k_sink(int64_t N, int S, int D, const int32_t *__restrict__ sc_list, int nsc, const int64_t *devOff,
+                       uint32_t *latd, uint64_t *agg) {
   for (int k = blockIdx.y; k < nsc; k += gridDim.y) {
     const int64_t st = devOff[D], n = devOff[D + 1] - st;
-    uint32_t *row = lat_out + (size_t)sc_list[k] * N;
+    const int s = sc_list[k];
+    uint32_t *row = latd + (size_t)s * N + st;
     for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
-      row[devIdx[st + j]] = 0xFFFFFFFFu;
+      row[j] = 0xFFFFFFFFu;
+    if (blockIdx.x == 0 && threadIdx.x == 0 && n) atomicAdd((unsigned long long *)&agg[s], (unsigned long long)n);
   }
 }
 
-// ------------------------------------------------------------- counts ----
-// a13: per scenario, violations (latency > SLO of the query's family, R6;
-// dropped included), on-time count and the serving variant's accuracy summed
-// over on-time queries (R9).
-__global__ void k_count(int64_t N, int S, int D, int Q, const proteus_scenario *__restrict__ sc,
-                        const int32_t *__restrict__ slo_base, const int32_t *__restrict__ option,
-                        const int32_t *__restrict__ acc, const uint8_t *__restrict__ fam,
-                        const uint8_t *__restrict__ tgt0, const uint8_t *__restrict__ tgt1,
-                        const uint32_t *__restrict__ lat, uint64_t *agg) {
-  __shared__ int64_t sL[PX_MAXQ];
-  __shared__ uint32_t sA[PX_MAXD + 1];
-  __shared__ unsigned long long red[3][32];
-  const int s = blockIdx.y;
-  const proteus_scenario scn = sc[s];
-  if (threadIdx.x < Q) sL[threadIdx.x] = (int64_t)scn.slo_mult_milli * slo_base[threadIdx.x] / 1000;
-  if (threadIdx.x <= D) sA[threadIdx.x] = threadIdx.x < D && option[threadIdx.x] > 0 ? acc[option[threadIdx.x] - 1] : 0;
+// per-query order: out[s][i] = latd[s][inv(i)] (coalesced stores, gathered loads
+// that walk ~D sequential streams)
+__global__ void k_unpermute(int64_t N, int S, const proteus_scenario *__restrict__ sc, const uint32_t *__restrict__ inv0,
+                            const uint32_t *__restrict__ inv1, const uint32_t *__restrict__ latd, uint32_t *out) {
+  __shared__ int8_t rt[4096];
+  for (int k = threadIdx.x; k < S; k += blockDim.x) rt[k] = (int8_t)sc[k].routing;
   __syncthreads();
-  const uint8_t *tgt = scn.routing ? tgt1 : tgt0;
-  const uint32_t *row = lat + (size_t)s * N;
-  unsigned long long viol = 0, ont = 0, accs = 0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t l = row[i];
-    if ((int64_t)l > sL[fam[i]]) viol++;
-    else { ont++; accs += sA[tgt[i]]; }
-  }
-  for (int o = 16; o; o >>= 1) {
-    viol += __shfl_xor_sync(0xffffffffu, viol, o);
-    ont += __shfl_xor_sync(0xffffffffu, ont, o);
-    accs += __shfl_xor_sync(0xffffffffu, accs, o);
-  }
-  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (lane == 0) { red[0][w] = viol; red[1][w] = ont; red[2][w] = accs; }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    unsigned long long v = 0, o2 = 0, a2 = 0;
-    for (int k = 0; k < (int)(blockDim.x >> 5); k++) { v += red[0][k]; o2 += red[1][k]; a2 += red[2][k]; }
-    if (v) atomicAdd((unsigned long long *)&agg[s], v);
-    if (o2) atomicAdd((unsigned long long *)&agg[S + s], o2);
-    if (a2) atomicAdd((unsigned long long *)&agg[2 * S + s], a2);
+    const uint32_t p0 = inv0 ? inv0[i] : 0, p1 = inv1 ? inv1[i] : 0;
+    for (int s = 0; s < S; s++) {
+      const size_t r = (size_t)s * N;
+      out[r + i] = latd[r + (rt[s] ? p1 : p0)];
+    }
   }
 }
 
@@ -693,14 +635,19 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
               const proteus_scenario *h_sc, int S, uint32_t *d_lat_out, uint64_t *d_agg) {
   const int Q = ctx->Q, M = ctx->M;
   PX_CUDA(ctx, cudaMemsetAsync(d_agg, 0, ((size_t)3 * S + 1) * 8, ctx->stream));
-  const size_t small = (size_t)(4 * D + 2 * Q + 2 * PX_MAXQ + 8 + 2 * S) * 4 + (size_t)S * sizeof(proteus_scenario);
+  const size_t small = (size_t)(4 * D + 2 * Q + 2 * PX_MAXQ + 8 + 2 * S + 4 * (PX_MAXD + 2)) * 4 +
+                       (size_t)S * sizeof(proteus_scenario) + (size_t)S * D * sizeof(LaneParam) +
+                       (size_t)2 * (PX_MAXD + 2) * 8;
   char *sb = (char *)px_buf(ctx, B_R_MISC, small + 4096);
   if (!sb) return px_fail(ctx, PROTEUS_ENOMEM, "replay scratch");
   int32_t *d_opt = (int32_t *)sb, *d_z = d_opt + D, *d_dev = d_z + D, *d_dem = d_dev + D, *d_slo = d_dem + Q;
   int32_t *d_pat_off = d_slo + Q, *d_pat_len = d_pat_off + PX_MAXQ;
   uint32_t *d_flags = (uint32_t *)(d_pat_len + PX_MAXQ);
-  int32_t *d_scl = (int32_t *)(d_flags + 8);  // [2][S] scenario lists per routing mode
-  proteus_scenario *d_sc = (proteus_scenario *)(((uintptr_t)(d_scl + 2 * S) + 15) & ~(uintptr_t)15);
+  int32_t *d_scl = (int32_t *)(d_flags + 8);              // [2][S] scenario lists per routing mode
+  int32_t *d_goff = d_scl + 2 * S;                        // [2][PX_MAXD + 2]
+  int64_t *d_choff = (int64_t *)(((uintptr_t)(d_goff + 2 * (PX_MAXD + 2)) + 15) & ~(uintptr_t)15);  // [2][PX_MAXD + 2]
+  proteus_scenario *d_sc = (proteus_scenario *)(d_choff + 2 * (PX_MAXD + 2));
+  LaneParam *d_lp = (LaneParam *)(((uintptr_t)(d_sc + S) + 15) & ~(uintptr_t)15);
   std::vector<int32_t> scl[2];
   for (int s = 0; s < S; s++) scl[h_sc[s].routing].push_back(s);
   std::vector<int32_t> scl_all(2 * S, 0);
@@ -722,26 +669,26 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     if (flags & 1) return px_fail(ctx, PROTEUS_ERANGE, "arrival timestamps not sorted");
     if (flags & 2) return px_fail(ctx, PROTEUS_EINVAL, "family id >= Q");
   }
+  PX_LAUNCH(ctx, "replay_params", k_lane_params, (S * D + 127) / 128, 128, 0, S, D, M, ctx->bmax, d_opt, d_dev,
+            ctx->d_fam, ctx->d_acc, ctx->d_lat, d_slo, d_sc, d_lp);
   const int64_t ntiles = (N + TILE - 1) / TILE;
   const unsigned tblocks = (unsigned)((ntiles + TILE_WARPS - 1) / TILE_WARPS);
   int64_t dsum = 0;
   for (int q = 0; q < Q; q++) dsum += h_demand[q];
   const size_t pat_cap = (size_t)dsum + (size_t)Q * D + 16;
-  const int64_t *devOff[2] = {nullptr, nullptr};
-  const int32_t *devBase[2] = {nullptr, nullptr};
-  const uint32_t *devArr[2] = {nullptr, nullptr}, *devIdx[2] = {nullptr, nullptr};
-  const uint8_t *tgts[2] = {nullptr, nullptr};
+  int64_t *devOff[2] = {nullptr, nullptr};
+  const uint32_t *devArr[2] = {nullptr, nullptr}, *inv[2] = {nullptr, nullptr};
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
     uint8_t *pat = (uint8_t *)px_buf(ctx, B_R_PAT, pat_cap);
     int32_t *hist = (int32_t *)px_buf(ctx, B_R_HIST, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
     int32_t *fbase = (int32_t *)px_buf(ctx, B_R_BASE, (size_t)(ntiles + 1) * (PX_MAXQ + 2) * 4);
-    int32_t *dbase = (int32_t *)px_buf(ctx, rt ? B_R_DBASE1 : B_R_DBASE0, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
-    uint8_t *tgt = (uint8_t *)px_buf(ctx, rt ? B_R_TGT1 : B_R_TGT, (size_t)N + 16);
+    int32_t *dbase = (int32_t *)px_buf(ctx, B_R_DBASE0, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
+    uint8_t *tgt = (uint8_t *)px_buf(ctx, B_R_TGT, (size_t)N + 16);
     int64_t *off = (int64_t *)px_buf(ctx, rt ? B_R_OFF1 : B_R_OFF, (size_t)2 * (PX_MAXD + 2) * 8);
     uint32_t *darr = (uint32_t *)px_buf(ctx, rt ? B_R_DEVARR1 : B_R_DEVARR, (size_t)N * 4 + 16);
-    uint32_t *didx = (uint32_t *)px_buf(ctx, rt ? B_R_DEVIDX1 : B_R_DEVIDX, (size_t)N * 4 + 16);
-    if (!pat || !hist || !fbase || !dbase || !tgt || !off || !darr || !didx)
+    uint32_t *dinv = (uint32_t *)px_buf(ctx, rt ? B_R_DEVIDX1 : B_R_DEVIDX, (size_t)N * 4 + 16);
+    if (!pat || !hist || !fbase || !dbase || !tgt || !off || !darr || !dinv)
       return px_fail(ctx, PROTEUS_ENOMEM, "routing buffers");
     int64_t *totals = off + (PX_MAXD + 2);
     PX_LAUNCH(ctx, "route_prepare", k_route_prepare, 1, 32, 0, rt, Q, D, M, ctx->bmax, d_opt, d_z, d_dev, d_dem,
@@ -754,73 +701,75 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       PX_LAUNCH(ctx, "route_scan_dev", k_tile_scan, D + 1, 1024, 0, hist, ntiles, D + 1, dbase, totals);
       PX_LAUNCH(ctx, "route_offsets", k_dev_offsets, 1, 32, 0, totals, D + 1, off);
       PX_LAUNCH(ctx, "route_scatter", k_scatter, tblocks, TILE_WARPS * 32, 0, tgt, d_arr, N, D, dbase, off, darr,
-                didx);
+                dinv);
     } else {
       PX_CUDA(ctx, cudaMemsetAsync(off, 0, (size_t)(PX_MAXD + 2) * 8, ctx->stream));
     }
-    devOff[rt] = off; devArr[rt] = darr; devIdx[rt] = didx; devBase[rt] = dbase; tgts[rt] = tgt;
+    devOff[rt] = off; devArr[rt] = darr; inv[rt] = dinv;
   }
   if (N == 0) return 0;
-  // the stitch reads speculative latencies, so rows exist even when the caller wants none
-  uint32_t *lat = d_lat_out;
-  if (!lat) {
-    lat = (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S * N * 4);
-    if (!lat) return px_fail(ctx, PROTEUS_ENOMEM, "latency scratch");
+  // chunk layout per routing mode (sizes only): the host reads the per-device counts
+  const int CH = env_int("PROTEUS_REPLAY_CHUNK", 256);
+  const bool simple = env_int("PROTEUS_REPLAY_SIMPLE", 0) != 0;
+  int64_t h_off[2][PX_MAXD + 2];
+  for (int rt = 0; rt < 2; rt++)
+    if (devOff[rt])
+      PX_CUDA(ctx, cudaMemcpyAsync(h_off[rt], devOff[rt], (D + 2) * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  int64_t NCH[2] = {0, 0};
+  int32_t ngroups[2] = {0, 0};
+  std::vector<int64_t> choff(2 * (PX_MAXD + 2), 0);
+  std::vector<int32_t> goff(2 * (PX_MAXD + 2), 0);
+  for (int rt = 0; rt < 2; rt++) {
+    if (!devOff[rt]) continue;
+    for (int d = 0; d < D; d++) {
+      const int64_t nch = (h_off[rt][d + 1] - h_off[rt][d] + CH - 1) / CH;
+      choff[rt * (PX_MAXD + 2) + d + 1] = choff[rt * (PX_MAXD + 2) + d] + nch;
+      goff[rt * (PX_MAXD + 2) + d + 1] = goff[rt * (PX_MAXD + 2) + d] + (int32_t)((nch + 31) / 32);
+    }
+    NCH[rt] = choff[rt * (PX_MAXD + 2) + D];
+    ngroups[rt] = goff[rt * (PX_MAXD + 2) + D];
   }
-  const int win_tiles = env_int("PROTEUS_REPLAY_WIN_TILES", 2);
-  const int nwin = (int)((ntiles + win_tiles - 1) / win_tiles);
-  const int win = win_tiles * TILE;
-  const int dpb = D < 32 ? D : 32;
-  const int ndg = (D + 31) / 32;
-  int use_tile = ndg == 1 && !env_int("PROTEUS_REPLAY_NO_TILE", 0);
-  auto spec_smem = [&](int tile) {
-    return ((size_t)(tile ? 32 * (win + 1) : 0) + (size_t)dpb * ctx->bmax + 2 * ((size_t)win + (size_t)dpb * ctx->bmax)) * 4;
-  };
-  if (use_tile && spec_smem(1) > 200 * 1024) use_tile = 0;
-  const size_t smem = spec_smem(use_tile);
-  const bool simple = env_int("PROTEUS_REPLAY_SIMPLE", 0) != 0 || smem > 200 * 1024;
+  PX_CUDA(ctx, cudaMemcpyAsync(d_choff, choff.data(), choff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_goff, goff.data(), goff.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S * N * 4);
+  if (!latd) return px_fail(ctx, PROTEUS_ENOMEM, "latency scratch");
   SpecExit *ex = nullptr;
   if (!simple) {
-    ex = (SpecExit *)px_buf(ctx, B_R_LANE, sizeof(SpecExit) * (size_t)S * D * nwin);
+    const int64_t nmax = NCH[0] > NCH[1] ? NCH[0] : NCH[1];
+    ex = (SpecExit *)px_buf(ctx, B_R_LANE, sizeof(SpecExit) * (size_t)S * (nmax + 1));
     if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
-    if (smem > 48 * 1024)
-      PX_CUDA(ctx, cudaFuncSetAttribute(k_spec, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     PX_CUDA(ctx, cudaFuncSetAttribute(k_stitch, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      4 * 2 * SBUF * 4 + 4 * ctx->bmax * 4));
+                                      4 * SBUF * 4 + 4 * ctx->bmax * 4));
   }
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
     LaneArgs la;
     memset(&la, 0, sizeof la);
-    la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.Q = Q; la.N = N; la.ntiles = ntiles;
-    la.option = d_opt; la.dev_type = d_dev; la.fam_of_m = ctx->d_fam; la.acc = ctx->d_acc; la.lat = ctx->d_lat;
-    la.slo_base = d_slo; la.sc = d_sc;
-    la.nsc = (int)scl[rt].size(); la.win_tiles = win_tiles; la.nwin = nwin; la.use_tile = simple ? 0 : use_tile;
-    la.sc_list = d_scl + rt * S;
-    la.devOff = devOff[rt]; la.devBase = devBase[rt]; la.devArr = devArr[rt]; la.devIdx = devIdx[rt];
-    la.lat_out = lat; la.ex = ex;
+    la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.nsc = (int)scl[rt].size(); la.CH = CH;
+    la.N = N; la.NCH = NCH[0] > NCH[1] ? NCH[0] : NCH[1];  // one row stride for both routing modes
+    la.option = d_opt; la.dev_type = d_dev; la.lat = ctx->d_lat; la.sc_list = d_scl + rt * S; la.lp = d_lp;
+    la.devOff = devOff[rt]; la.choff = d_choff + rt * (PX_MAXD + 2); la.goff = d_goff + rt * (PX_MAXD + 2);
+    la.devArr = devArr[rt]; la.latd = latd; la.ex = ex; la.agg = d_agg;
     if (simple) {
       const int nl = la.nsc * D;
       PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
     } else {
-      dim3 grid(nwin, (la.nsc + 31) / 32, ndg);
-      PX_LAUNCH(ctx, "replay_spec", k_spec, grid, dpb * 32, smem, la);
+      dim3 grid((unsigned)((ngroups[rt] + 3) / 4), (unsigned)la.nsc);
+      PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la);
       const int64_t warps = (int64_t)la.nsc * D;
-      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 4 * 2 * SBUF * 4 + 4 * ctx->bmax * 4,
+      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 4 * SBUF * 4 + 4 * ctx->bmax * 4,
                 la);
     }
-    if (simple || !la.use_tile) {
-      dim3 g(64, la.nsc < 65535 ? la.nsc : 65535);
-      PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, N, D, d_scl + rt * S, la.nsc, devOff[rt], devIdx[rt], lat);
-    }
+    dim3 g(32, la.nsc < 65535 ? la.nsc : 65535);
+    PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, N, S, D, d_scl + rt * S, la.nsc, devOff[rt], latd, d_agg);
   }
-  int nsm = 0;
-  PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
-  int bx = (int)((N + 255) / 256);
-  const int cap_bx = (nsm * 8 + S - 1) / S;
-  if (bx > cap_bx) bx = cap_bx > 0 ? cap_bx : 1;
-  dim3 cg(bx, S);
-  PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, S, D, Q, d_sc, d_slo, d_opt, ctx->d_acc, d_fam,
-            tgts[0] ? tgts[0] : tgts[1], tgts[1] ? tgts[1] : tgts[0], lat, d_agg);
+  if (d_lat_out) {
+    int nsm = 0;
+    PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
+    int64_t nb = (N + 255) / 256;
+    if (nb > (int64_t)nsm * 8) nb = (int64_t)nsm * 8;
+    PX_LAUNCH(ctx, "replay_unpermute", k_unpermute, (unsigned)nb, 256, 0, N, S, d_sc, inv[0], inv[1], latd, d_lat_out);
+  }
   return 0;
 }

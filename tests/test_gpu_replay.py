@@ -32,17 +32,17 @@ def _compare(px, oracle_mod, prof, cl, option, z, demand, arr, fam, sc):
     return g
 
 
-PATHS = {"chunked": {}, "small_windows": {"PROTEUS_REPLAY_WIN_TILES": "1"}, "no_tile": {"PROTEUS_REPLAY_NO_TILE": "1"},
+PATHS = {"chunked": {}, "small_chunks": {"PROTEUS_REPLAY_CHUNK": "16"}, "odd_chunks": {"PROTEUS_REPLAY_CHUNK": "37"},
          "simple": {"PROTEUS_REPLAY_SIMPLE": "1"}}
 
 
 @pytest.mark.parametrize("path", sorted(PATHS))
 @pytest.mark.parametrize("kind", ["poisson", "gamma", "uniform"])
 def test_replay_small_all_scenarios(px, oracle_mod, kind, path, monkeypatch):
-    """60k queries x 64 scenarios x both routings; `small_windows` cuts the
-    device arrays every 1024 global queries so the stitch (backlogged jumps,
-    re-walks, convergence) runs at every window; `simple` is one thread per
-    (device, scenario) lane."""
+    """60k queries x 64 scenarios x both routings; `small_chunks` /
+    `odd_chunks` cut the device arrays every 16 / 37 queries so the stitch
+    (backlogged jumps, re-walks, meeting tests) runs at every chunk; `simple`
+    is one thread per (device, scenario) lane."""
     for k, v in PATHS[path].items():
         monkeypatch.setenv(k, v)
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
