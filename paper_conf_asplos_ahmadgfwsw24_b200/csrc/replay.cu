@@ -331,29 +331,20 @@ __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ 
   const int64_t st = a.devOff[d], n = a.devOff[d + 1] - st;
   if (n == 0) return;
   uint32_t *out = a.latd + (size_t)s * a.N + st;
-  unsigned long long viol = 0, ont = 0, accs = 0;
   if (p.Bmax < 1) {  // never routed to (z = 0 / depth 0); kept for safety
     for (int64_t j = 0; j < n; j++) out[j] = 0xFFFFFFFFu;
-    viol = n;
-  } else {
-    const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
-    GArr arr{a.devArr + st};
-    int64_t h = 0, F = 0;  // R13
-    while (h < n) {
-      int64_t t;
-      const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
-      F = t + T[b - 1];
-      for (int j = 0; j < b; j++) {
-        const uint32_t l = sat_lat(F - (int64_t)arr(h + j));
-        out[h + j] = l;
-        count_lat(l, p, viol, ont, accs);
-      }
-      h += b;
-    }
+    return;
   }
-  atomicAdd((unsigned long long *)&a.agg[s], viol);
-  atomicAdd((unsigned long long *)&a.agg[a.S + s], ont);
-  atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], accs);
+  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  GArr arr{a.devArr + st};
+  int64_t h = 0, F = 0;  // R13
+  while (h < n) {
+    int64_t t;
+    const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
+    F = t + T[b - 1];
+    for (int j = 0; j < b; j++) out[h + j] = sat_lat(F - (int64_t)arr(h + j));
+    h += b;
+  }
 }
 
 // ---- phase A: speculative chunks
@@ -375,14 +366,12 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
   const int64_t c = (int64_t)(g - sG[d]) * 32 + lane;
-  unsigned long long viol = 0, ont = 0, accs = 0;
   if (c < nch) {
     const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
     uint32_t *out = a.latd + (size_t)s * a.N + off;
     int64_t h = st, F = 0;
     if (p.Bmax < 1) {
       for (int64_t j = st; j < en; j++) out[j] = 0xFFFFFFFFu;
-      viol = en - st;
       h = en;
     } else {
       const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
@@ -392,11 +381,7 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
         const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
         F = t + T[b - 1];
         const int64_t jend = h + b < en ? h + b : en;
-        for (int64_t j = h; j < jend; j++) {
-          const uint32_t l = sat_lat(F - (int64_t)arr(j));
-          out[j] = l;
-          count_lat(l, p, viol, ont, accs);
-        }
+        for (int64_t j = h; j < jend; j++) out[j] = sat_lat(F - (int64_t)arr(j));
         h += b;
       }
     }
@@ -406,7 +391,6 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
     e.pad = 0;
     a.ex[(size_t)s * a.NCH + a.choff[d] + c] = e;
   }
-  warp_add_counts(viol, ont, accs, a.agg, a.S, s, lane);
 }
 
 // ---- phase B: exact stitch, one warp per (device, scenario)
@@ -426,6 +410,7 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
 // through a shared-memory ring; exit states are fetched 32 chunks at a time.
 #define SBUF 2048
 #define SAHEAD 1088
+#define SPECCAP 1024
 
 struct BufArr {
   const uint32_t *buf, *g;
@@ -485,7 +470,7 @@ __device__ __forceinline__ int decide_par(const Arr &A, int64_t n, int64_t h, in
 }
 
 __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs a) {
-  extern __shared__ uint32_t ssm[];  // [4 warps][SBUF] arrivals, then [4 warps][bmax] T
+  extern __shared__ uint32_t ssm[];  // [4][SBUF] arrivals, then per warp: bmax T + SPECCAP spec latencies
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t gw = (int64_t)blockIdx.x * 4 + w;
   if (gw >= (int64_t)a.nsc * a.D) return;
@@ -495,7 +480,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   const int64_t nch = a.choff[d + 1] - a.choff[d];
   if (p.Bmax < 1 || nch < 2) return;
   uint32_t *bufA = ssm + (size_t)w * SBUF;
-  int32_t *T = (int32_t *)(ssm + 4 * SBUF) + w * a.bmax;
+  int32_t *T = (int32_t *)(ssm + 4 * SBUF) + w * (a.bmax + SPECCAP);
   const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
   for (int k = lane; k < a.bmax; k += 32) T[k] = Tg[k];
   __syncwarp();
@@ -513,15 +498,14 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
     }
     __syncwarp();
   };
-  long long dv = 0, dont = 0, dacc = 0;
-  auto put = [&](int64_t j, int64_t Fb) {
-    const uint32_t nl = sat_lat(Fb - (int64_t)A(j));
-    const uint32_t ol = out[j];
-    out[j] = nl;
-    const int nv = (int64_t)nl > p.L, ov = (int64_t)ol > p.L;
-    dv += nv - ov;
-    dont += ov - nv;
-    dacc += ((long long)ov - (long long)nv) * (long long)p.A;
+  auto put = [&](int64_t j, int64_t Fb) { out[j] = sat_lat(Fb - (int64_t)A(j)); };
+  // speculative finish time of position j of the current chunk (cached before rewriting)
+  uint32_t *specL = (uint32_t *)(T + a.bmax);
+  int64_t spec_base = -1;
+  auto spec_F = [&](int64_t j) -> int64_t {
+    const int64_t o = j - spec_base;
+    const uint32_t l = (o >= 0 && o < SPECCAP) ? specL[o] : out[j];
+    return (int64_t)A(j) + l;
   };
   const int64_t TB = T[p.Bmax - 1];
   const int64_t CH = a.CH;
@@ -552,6 +536,13 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         continue;
       }
       int checks = 2;
+      {  // cache the speculative latencies of this chunk before overwriting any of them
+        __syncwarp();
+        spec_base = h;
+        const int64_t m = en - h < SPECCAP ? en - h : SPECCAP;
+        for (int64_t i = lane; i < m; i += 32) specL[i] = out[h + i];
+        __syncwarp();
+      }
       while (h < en) {
         ensure(h);
         if (F > (int64_t)A(h) && h + p.Bmax - 1 < n && (int64_t)A(h + p.Bmax - 1) <= F) {
@@ -577,7 +568,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         bool conv = false;
         if (t > F && j2 < en && checks > 0) {
           checks--;
-          conv = (int64_t)A(j2 - 1) + out[j2 - 1] == Fn && (int64_t)A(j2) + out[j2] != Fn;
+          conv = spec_F(j2 - 1) == Fn && spec_F(j2) != Fn;
         }
         __syncwarp();
         const int64_t hi = j2 < en ? j2 : en;
@@ -592,10 +583,9 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
       }
     }
   }
-  warp_add_counts((unsigned long long)dv, (unsigned long long)dont, (unsigned long long)dacc, a.agg, a.S, s, lane);
 }
 
-// dropped queries (the sink segment, device index D): latency UINT32_MAX (R7), violations
+// dropped queries (the sink segment, device index D): latency UINT32_MAX (R7)
 __global__ void k_sink(int64_t N, int S, int D, const int32_t *__restrict__ sc_list, int nsc, const int64_t *devOff,
                        uint32_t *latd, uint64_t *agg) {
   for (int k = blockIdx.y; k < nsc; k += gridDim.y) {
@@ -604,7 +594,54 @@ __global__ void k_sink(int64_t N, int S, int D, const int32_t *__restrict__ sc_l
     uint32_t *row = latd + (size_t)s * N + st;
     for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
       row[j] = 0xFFFFFFFFu;
-    if (blockIdx.x == 0 && threadIdx.x == 0 && n) atomicAdd((unsigned long long *)&agg[s], (unsigned long long)n);
+  }
+}
+
+// a13: per scenario, violations (latency > the SLO of the device's family, R6;
+// dropped queries included), on-time count and the serving variant's accuracy
+// summed over on-time queries (R9), over the device-major rows.
+__global__ void k_count(int64_t N, int S, int D, const int32_t *__restrict__ sc_list, const int64_t *__restrict__ devOff,
+                        const LaneParam *__restrict__ lp, const uint32_t *__restrict__ latd, uint64_t *agg) {
+  __shared__ int64_t sOff[PX_MAXD + 2], sL[PX_MAXD + 1];
+  __shared__ uint32_t sA[PX_MAXD + 1];
+  __shared__ unsigned long long red[3][32];
+  const int s = sc_list[blockIdx.y];
+  for (int k = threadIdx.x; k <= D + 1; k += blockDim.x) sOff[k] = devOff[k];
+  for (int k = threadIdx.x; k <= D; k += blockDim.x) {
+    sL[k] = k < D ? lp[s * D + k].L : -1;  // the sink: every latency is a violation
+    sA[k] = k < D ? lp[s * D + k].A : 0;
+  }
+  __syncthreads();
+  const uint32_t *row = latd + (size_t)s * N;
+  unsigned long long viol = 0, ont = 0, accs = 0;
+  const int64_t per = (N + gridDim.x - 1) / gridDim.x;
+  const int64_t lo = (int64_t)blockIdx.x * per, hi = lo + per < N ? lo + per : N;
+  int d = 0;
+  for (int64_t p0 = lo; p0 < hi; p0 += blockDim.x) {
+    while (d < D && sOff[d + 1] <= p0) d++;  // segment of this step's first position (uniform)
+    const int64_t p = p0 + threadIdx.x;
+    if (p < hi) {
+      int dd = d;
+      while (dd < D && sOff[dd + 1] <= p) dd++;
+      const uint32_t l = row[p];
+      if ((int64_t)l > sL[dd]) viol++;
+      else { ont++; accs += sA[dd]; }
+    }
+  }
+  for (int o = 16; o; o >>= 1) {
+    viol += __shfl_xor_sync(0xffffffffu, viol, o);
+    ont += __shfl_xor_sync(0xffffffffu, ont, o);
+    accs += __shfl_xor_sync(0xffffffffu, accs, o);
+  }
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) { red[0][w] = viol; red[1][w] = ont; red[2][w] = accs; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, o2 = 0, a2 = 0;
+    for (int k = 0; k < (int)(blockDim.x >> 5); k++) { v += red[0][k]; o2 += red[1][k]; a2 += red[2][k]; }
+    if (v) atomicAdd((unsigned long long *)&agg[s], v);
+    if (o2) atomicAdd((unsigned long long *)&agg[S + s], o2);
+    if (a2) atomicAdd((unsigned long long *)&agg[2 * S + s], a2);
   }
 }
 
@@ -732,7 +769,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   }
   PX_CUDA(ctx, cudaMemcpyAsync(d_choff, choff.data(), choff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_goff, goff.data(), goff.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
-  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S * N * 4);
+  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * N * 4);  // B_R_LAT stages host outputs
   if (!latd) return px_fail(ctx, PROTEUS_ENOMEM, "latency scratch");
   SpecExit *ex = nullptr;
   if (!simple) {
@@ -740,7 +777,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     ex = (SpecExit *)px_buf(ctx, B_R_LANE, sizeof(SpecExit) * (size_t)S * (nmax + 1));
     if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
     PX_CUDA(ctx, cudaFuncSetAttribute(k_stitch, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      4 * SBUF * 4 + 4 * ctx->bmax * 4));
+                                      4 * SBUF * 4 + 4 * (ctx->bmax + SPECCAP) * 4));
   }
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
@@ -758,11 +795,18 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       dim3 grid((unsigned)((ngroups[rt] + 3) / 4), (unsigned)la.nsc);
       PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la);
       const int64_t warps = (int64_t)la.nsc * D;
-      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, 4 * SBUF * 4 + 4 * ctx->bmax * 4,
-                la);
+      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128,
+                4 * SBUF * 4 + 4 * (ctx->bmax + SPECCAP) * 4, la);
     }
     dim3 g(32, la.nsc < 65535 ? la.nsc : 65535);
     PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, N, S, D, d_scl + rt * S, la.nsc, devOff[rt], latd, d_agg);
+    int nsm = 0;
+    PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
+    int64_t cbx = (N + 4095) / 4096;
+    const int64_t cap_bx = ((int64_t)nsm * 16 + la.nsc - 1) / la.nsc;
+    if (cbx > cap_bx) cbx = cap_bx > 0 ? cap_bx : 1;
+    dim3 cg((unsigned)cbx, (unsigned)la.nsc);
+    PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, S, D, d_scl + rt * S, devOff[rt], d_lp, latd, d_agg);
   }
   if (d_lat_out) {
     int nsm = 0;
