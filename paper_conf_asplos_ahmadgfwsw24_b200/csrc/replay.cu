@@ -792,8 +792,10 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       const int nl = la.nsc * D;
       PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
     } else {
-      dim3 grid((unsigned)((ngroups[rt] + 3) / 4), (unsigned)la.nsc);
-      PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la);
+      if (ngroups[rt] > 0) {
+        dim3 grid((unsigned)((ngroups[rt] + 3) / 4), (unsigned)la.nsc);
+        PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la);
+      }
       const int64_t warps = (int64_t)la.nsc * D;
       PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128,
                 4 * SBUF * 4 + 4 * (ctx->bmax + SPECCAP) * 4, la);
