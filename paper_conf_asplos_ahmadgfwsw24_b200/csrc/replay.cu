@@ -544,25 +544,52 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         __syncwarp();
       }
       while (h < en) {
-        ensure(h);
-        if (F > (int64_t)A(h) && h + p.Bmax - 1 < n && (int64_t)A(h + p.Bmax - 1) <= F) {
+        ensure(h);  // from here on [h, h + SAHEAD) is in the ring: plain shared loads
+        const uint32_t *ab = bufA - A.base;
+        const int64_t ah = ab[h];
+        if (F > ah && h + p.Bmax - 1 < n && (int64_t)ab[h + p.Bmax - 1] <= F) {
           // backlog: full batches back to back
           int64_t kmax = (en - h + p.Bmax - 1) / p.Bmax;
           const int64_t room = (A.base + SBUF - h) / p.Bmax;
           if (kmax > room) kmax = room;
           if (kmax > 32) kmax = 32;
           const int64_t idx = h + (int64_t)(lane + 1) * p.Bmax - 1;
-          const bool ok = lane < kmax && idx < n && (int64_t)A(idx) <= F + (int64_t)lane * TB;
+          const bool ok = lane < kmax && idx < n && (int64_t)ab[idx] <= F + (int64_t)lane * TB;
           const unsigned bal = __ballot_sync(0xffffffffu, ok);
           const int r = bal == 0xffffffffu ? 32 : __ffs(~bal) - 1;
           const int64_t nq = (int64_t)r * p.Bmax;
-          for (int64_t i = lane; i < nq; i += 32) put(h + i, F + (i / p.Bmax + 1) * TB);
+          for (int64_t i = lane; i < nq; i += 32)
+            out[h + i] = sat_lat(F + (i / p.Bmax + 1) * TB - (int64_t)ab[h + i]);
           h += nq;
           F += (int64_t)r * TB;
           continue;
         }
+        // one decision (see decide_par): queue states k = 0.. in rounds of 32;
+        // states inside the initial queue are incomplete and never stop
+        const int64_t t0 = F > ah ? F : ah;
+        int b;
         int64_t t;
-        const int b = decide_par(A, n, h, F, p.Bmax, p.L, T, lane, &t);
+        for (int kb = 0;; kb += 32) {
+          const int k = kb + lane;
+          bool stop = false, now = false;
+          int64_t tau = 0, W = 0;
+          if (k < p.Bmax && h + k < n) {
+            const int64_t ak = ab[h + k];
+            tau = ak > t0 ? ak : t0;
+            const bool capped = k + 1 == p.Bmax;
+            const int64_t nxt = h + k + 1 < n ? (int64_t)ab[h + k + 1] : INT64_MAX;
+            W = capped ? 0 : ah + p.L - T[k + 1];
+            now = capped || tau >= W;
+            stop = (capped || nxt > tau) && (now || nxt > W);
+          }
+          const unsigned bal = __ballot_sync(0xffffffffu, stop);
+          if (bal) {
+            const int src = __ffs(bal) - 1;
+            t = __shfl_sync(0xffffffffu, now ? tau : W, src);
+            b = kb + src + 1;
+            break;
+          }
+        }
         const int64_t Fn = t + T[b - 1];
         const int64_t j2 = h + b;
         bool conv = false;
@@ -572,7 +599,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         }
         __syncwarp();
         const int64_t hi = j2 < en ? j2 : en;
-        for (int64_t j = h + lane; j < hi; j += 32) put(j, Fn);
+        for (int64_t jj = h + lane; jj < hi; jj += 32) out[jj] = sat_lat(Fn - (int64_t)ab[jj]);
         h = j2;
         F = Fn;
         if (conv) {
