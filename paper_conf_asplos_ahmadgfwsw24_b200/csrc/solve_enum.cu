@@ -250,42 +250,60 @@ __global__ void __launch_bounds__(FLAT_THREADS, 2) k_flat_pair(const __grid_cons
       uint64_t Fb[S];
 #pragma unroll
       for (int s = 0; s < S; s++) Fb[s] = fill<QM, VM>(caps, a, s / VM, s % VM, a.PB[s], -1, 0) - Fq[s / VM];
-      // The K^2 candidates of this prefix in increasing index order, spread
-      // over 4 independent running maxima (candidate (sa, sb) -> accumulator
-      // (sb + 1) & 3) so the compare chains overlap; each accumulator sees its
-      // candidates in index order and keeps the first maximum, and the merge
-      // below prefers the lower index on equal scores.  Pad slots (code 0,
-      // capacity 0) score exactly like the idle option with the same index,
-      // so they can never change the result.
-      uint64_t lb[4] = {best_s, best_s, best_s, best_s};
-      int lp[4] = {-1, -1, -1, -1};
-      if (base > lb[0] || best_i == ~0ull) { lb[0] = base; lp[0] = 0; }
+      // The K^2 candidates of this prefix, one row per option of device D-2
+      // (idle first).  Fast path per row: every candidate is scored and
+      // compared with the running best lb -- a candidate of another family
+      // than the row's as Fb[sb] > lb - ba (its score is ba + Fb[sb], Fb >= 0),
+      // a same-family candidate through its joint water-fill -- and the
+      // compares are only OR-ed into flags.  A flagged row (it holds a better
+      // candidate) is re-scanned in index order with strict >, so the first
+      // (lowest-index) maximum is kept.  If lb < ba the row's first candidate
+      // (sa, idle) = ba already flags the row, so the unsigned threshold never
+      // matters when it wraps.  Pad slots (code 0, capacity 0) score exactly
+      // like the idle option with the same index and never change the result.
+      uint64_t lb = best_s;
+      int lp = -1;
+      if (best_i == ~0ull) { lb = base; lp = 0; }  // the thread's first candidate
+      {
+        const uint64_t thr = lb - base;
+        bool f0 = base > lb, f1 = false, f2 = false, f3 = false;
 #pragma unroll
-      for (int sb = 0; sb < S; sb++) {
-        const uint64_t c = base + Fb[sb];
-        if (c > lb[(sb + 1) & 3]) { lb[(sb + 1) & 3] = c; lp[(sb + 1) & 3] = a.code[sb]; }
+        for (int sb = 0; sb < S; sb++) {
+          const bool g = Fb[sb] > thr;
+          if ((sb & 3) == 0) f0 |= g; else if ((sb & 3) == 1) f1 |= g; else if ((sb & 3) == 2) f2 |= g; else f3 |= g;
+        }
+        if (f0 | f1 | f2 | f3) {
+          if (base > lb) { lb = base; lp = 0; }
+#pragma unroll
+          for (int sb = 0; sb < S; sb++)
+            if (base + Fb[sb] > lb) { lb = base + Fb[sb]; lp = a.code[sb]; }
+        }
       }
 #pragma unroll
       for (int sa = 0; sa < S; sa++) {
         const int qa = sa / VM;
         const uint64_t ba = base + fill<QM, VM>(caps, a, qa, sa % VM, a.PA[sa], -1, 0) - Fq[qa];
-        if (ba > lb[0]) { lb[0] = ba; lp[0] = a.code[sa] * K; }
+        uint64_t jv[VM];  // same-family candidates (joint fills)
+#pragma unroll
+        for (int jb = 0; jb < VM; jb++)
+          jv[jb] = base - Fq[qa] + fill<QM, VM>(caps, a, qa, sa % VM, a.PA[sa], jb, a.PB[qa * VM + jb]);
+        const uint64_t thr = lb - ba;
+        bool f0 = ba > lb, f1 = false, f2 = false, f3 = false;
 #pragma unroll
         for (int sb = 0; sb < S; sb++) {
-          uint64_t c;
-          if (qa == sb / VM)
-            c = base - Fq[qa] + fill<QM, VM>(caps, a, qa, sa % VM, a.PA[sa], sb % VM, a.PB[sb]);
-          else
-            c = ba + Fb[sb];
-          if (c > lb[(sb + 1) & 3]) { lb[(sb + 1) & 3] = c; lp[(sb + 1) & 3] = a.code[sa] * K + a.code[sb]; }
+          const bool g = (qa == sb / VM) ? jv[sb % VM] > lb : Fb[sb] > thr;
+          if ((sb & 3) == 0) f0 |= g; else if ((sb & 3) == 1) f1 |= g; else if ((sb & 3) == 2) f2 |= g; else f3 |= g;
+        }
+        if (f0 | f1 | f2 | f3) {
+          if (ba > lb) { lb = ba; lp = a.code[sa] * K; }
+#pragma unroll
+          for (int sb = 0; sb < S; sb++) {
+            const uint64_t c = (qa == sb / VM) ? jv[sb % VM] : ba + Fb[sb];
+            if (c > lb) { lb = c; lp = a.code[sa] * K + a.code[sb]; }
+          }
         }
       }
-      uint64_t mb = lb[0];
-      int mp = lp[0];
-#pragma unroll
-      for (int k = 1; k < 4; k++)
-        if (lp[k] >= 0 && (lb[k] > mb || (lb[k] == mb && (mp < 0 || lp[k] < mp)))) { mb = lb[k]; mp = lp[k]; }
-      if (mp >= 0) { best_s = mb; best_i = p * KK + (uint64_t)mp; }
+      if (lp >= 0) { best_s = lb; best_i = p * KK + (uint64_t)lp; }
       if (++p >= pend) break;
       if (++dig[D - 3] == K) {
         dig[D - 3] = 0;
