@@ -223,6 +223,8 @@ int proteus_load_profiles(proteus_ctx *ctx, const proteus_profiles *p) {
   ctx->T = p->T; ctx->Q = p->Q; ctx->M = M; ctx->bmax = p->bmax;
   ctx->V = V; ctx->acc = acc; ctx->lat = lat; ctx->fam = fam; ctx->off = off;
   ctx->have_prof = true;
+  ctx->prof_gen++;
+  ctx->tab_valid = false;
   return PROTEUS_OK;
 }
 
@@ -231,8 +233,12 @@ int proteus_load_profiles(proteus_ctx *ctx, const proteus_profiles *p) {
 // -------------------------------------------------------------- solve -----
 struct SolveInputs {
   std::vector<int32_t> dev_type, slo, demand;
+  const int32_t *d_dev = nullptr, *d_slo = nullptr, *d_dem = nullptr;
 };
 
+// Host copies of the small solve inputs (validation, launch parameters) and
+// device pointers for the kernels: a device input is used in place and read
+// back with a single synchronisation; a host input is staged to the device.
 static int validate_solve(proteus_ctx *ctx, const proteus_solve_args *a, SolveInputs &in) {
   if (!ctx) return PROTEUS_EINVAL;
   ctx->err.clear();
@@ -244,11 +250,24 @@ static int validate_solve(proteus_ctx *ctx, const proteus_solve_args *a, SolveIn
   if (!a->device_type || !a->slo_us || !a->demand_qps) return px_fail(ctx, PROTEUS_EINVAL, "null array");
   if (a->shard_world < 0 || a->shard_rank < 0 || (a->shard_world > 0 && a->shard_rank >= a->shard_world))
     return px_fail(ctx, PROTEUS_EINVAL, "shard %d/%d", a->shard_rank, a->shard_world);
-  int rc;
   PX_CUDA(ctx, cudaSetDevice(ctx->device));
-  if ((rc = to_host(ctx, a->device_type, a->D, in.dev_type))) return rc;
-  if ((rc = to_host(ctx, a->slo_us, ctx->Q, in.slo))) return rc;
-  if ((rc = to_host(ctx, a->demand_qps, (size_t)a->n_vec * ctx->Q, in.demand))) return rc;
+  const int32_t *src[3] = {a->device_type, a->slo_us, a->demand_qps};
+  std::vector<int32_t> *dst[3] = {&in.dev_type, &in.slo, &in.demand};
+  const size_t cnt[3] = {(size_t)a->D, (size_t)ctx->Q, (size_t)a->n_vec * ctx->Q};
+  const int32_t **dptr[3] = {&in.d_dev, &in.d_slo, &in.d_dem};
+  bool dev[3], any_dev = false;
+  for (int k = 0; k < 3; k++) {
+    dst[k]->resize(cnt[k]);
+    dev[k] = px_is_device_ptr(src[k]);
+    if (dev[k]) {
+      PX_CUDA(ctx, cudaMemcpyAsync(dst[k]->data(), src[k], cnt[k] * 4, cudaMemcpyDeviceToHost, ctx->stream));
+      *dptr[k] = src[k];
+      any_dev = true;
+    } else {
+      memcpy(dst[k]->data(), src[k], cnt[k] * 4);
+    }
+  }
+  if (any_dev) PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
   for (int d = 0; d < a->D; d++)
     if (in.dev_type[d] < 0 || in.dev_type[d] >= ctx->T)
       return px_fail(ctx, PROTEUS_EINVAL, "device_type[%d]=%d", d, in.dev_type[d]);
@@ -262,6 +281,14 @@ static int validate_solve(proteus_ctx *ctx, const proteus_solve_args *a, SolveIn
       sum += s;
     }
     if (sum >= (1 << 22)) return px_fail(ctx, PROTEUS_ERANGE, "sum of demand %lld >= 2^22", (long long)sum);
+  }
+  const int bufid[3] = {B_IN0, B_IN1, B_IN2};
+  for (int k = 0; k < 3; k++) {
+    if (dev[k]) continue;
+    int32_t *d = (int32_t *)px_buf(ctx, bufid[k], cnt[k] * 4);
+    if (!d) return px_fail(ctx, PROTEUS_ENOMEM, "input staging");
+    PX_CUDA(ctx, cudaMemcpyAsync(d, dst[k]->data(), cnt[k] * 4, cudaMemcpyHostToDevice, ctx->stream));
+    *dptr[k] = d;
   }
   return 0;
 }
@@ -302,20 +329,32 @@ static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_s
       return px_fail(ctx, PROTEUS_ERANGE, "candidate space %llu > max_candidates %llu", (unsigned long long)n,
                      (unsigned long long)a->max_candidates);
   }
-  const int32_t *d_dev = to_device(ctx, in.dev_type.data(), in.dev_type.size(), B_IN0, &rc);
-  if (rc) return rc;
-  const int32_t *d_slo = to_device(ctx, in.slo.data(), in.slo.size(), B_IN1, &rc);
-  if (rc) return rc;
-  const int32_t *d_dem = to_device(ctx, in.demand.data(), in.demand.size(), B_IN2, &rc);
-  if (rc) return rc;
-  Tables tab;
-  if ((rc = px_prepare_tables(ctx, a->D, d_dev, d_slo, VM, tab))) return rc;
-  // the launch parameters of the scoring kernels carry the capacity table
-  std::vector<int32_t> h_P((size_t)ctx->T * ctx->M), h_slot_code((size_t)ctx->Q * VM);
-  PX_CUDA(ctx, cudaMemcpyAsync(h_P.data(), tab.P, h_P.size() * 4, cudaMemcpyDeviceToHost, ctx->stream));
-  PX_CUDA(ctx, cudaMemcpyAsync(h_slot_code.data(), tab.slot_code, h_slot_code.size() * 4, cudaMemcpyDeviceToHost,
-                               ctx->stream));
-  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  const int32_t *d_dev = in.d_dev, *d_dem = in.d_dem;
+  // Per-call tables (capacity a1, slot order, per-device capacity) depend only
+  // on the profiles, the inventory and the SLOs: reused while those repeat.
+  std::vector<int32_t> key;
+  key.reserve(4 + in.dev_type.size() + in.slo.size());
+  key.push_back((int32_t)ctx->prof_gen);
+  key.push_back(a->D);
+  key.push_back(VM);
+  key.insert(key.end(), in.dev_type.begin(), in.dev_type.end());
+  key.insert(key.end(), in.slo.begin(), in.slo.end());
+  if (!ctx->tab_valid || key != ctx->tab_key) {
+    ctx->tab_valid = false;
+    if ((rc = px_prepare_tables(ctx, a->D, d_dev, in.d_slo, VM, ctx->tab))) return rc;
+    // the launch parameters of the scoring kernels carry the capacity table
+    ctx->tab_P.resize((size_t)ctx->T * ctx->M);
+    ctx->tab_slot_code.resize((size_t)ctx->Q * VM);
+    PX_CUDA(ctx, cudaMemcpyAsync(ctx->tab_P.data(), ctx->tab.P, ctx->tab_P.size() * 4, cudaMemcpyDeviceToHost,
+                                 ctx->stream));
+    PX_CUDA(ctx, cudaMemcpyAsync(ctx->tab_slot_code.data(), ctx->tab.slot_code, ctx->tab_slot_code.size() * 4,
+                                 cudaMemcpyDeviceToHost, ctx->stream));
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+    ctx->tab_key = key;
+    ctx->tab_valid = true;
+  }
+  const Tables &tab = ctx->tab;
+  const std::vector<int32_t> &h_P = ctx->tab_P, &h_slot_code = ctx->tab_slot_code;
   int nout = mat_only ? 1 : a->n_vec;
   SolRec *d_sol = (SolRec *)px_buf(ctx, B_SOL, sizeof(SolRec) * nout);
   if (!d_sol) return px_fail(ctx, PROTEUS_ENOMEM, "solution buffer");

@@ -89,6 +89,11 @@ struct proteus_ctx {
   std::vector<cudaEvent_t> tev;  // pairs
   std::vector<float> tms;
   std::vector<cudaEvent_t> ev_pool;
+  // cached per-call solve tables (see solve_common)
+  uint32_t prof_gen = 0;
+  bool tab_valid = false;
+  std::vector<int32_t> tab_key, tab_P, tab_slot_code;
+  Tables tab;
 };
 
 // scratch buffer ids

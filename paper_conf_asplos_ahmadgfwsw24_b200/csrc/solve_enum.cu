@@ -322,10 +322,18 @@ __global__ void __launch_bounds__(FLAT_THREADS, 2) k_flat_pair(const __grid_cons
 // ------------------------------------------------------- materialise ----
 // a9: decode the winner, water-fill z in (accuracy desc, code asc, device asc)
 // order (reading C10), report served / unmet / accsum / eff; re-check the score.
-__global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const BestRec *best, uint64_t fixed_index,
-                                   int use_fixed, uint64_t n_candidates, SolRec *out) {
+// a6 (grid level) is folded in: the block first reduces the per-block winners.
+__global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const BestRec *__restrict__ blocks, int nb,
+                                   uint64_t fixed_index, int use_fixed, uint64_t n_candidates, SolRec *out) {
+  uint64_t bs = 0, bi = ~0ull;
+  if (!use_fixed)
+    for (int k = threadIdx.x; k < nb; k += blockDim.x)
+      if (px_better(blocks[k].score, blocks[k].index, bs, bi)) { bs = blocks[k].score; bi = blocks[k].index; }
+  block_best(bs, bi);
   if (threadIdx.x != 0) return;
   SolRec &r = *out;
+  const BestRec best_rec = {bs, bi};
+  const BestRec *best = &best_rec;
   uint64_t idx = use_fixed ? fixed_index : best->index;
   if (idx == ~0ull) {  // empty shard: nothing scored
     for (int d = 0; d < a.D; d++) { r.option[d] = 0; r.z[d] = 0; }
@@ -483,12 +491,12 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
   const size_t max_blocks = (size_t)nsm * 64;
   BestRec *d_blocks = (BestRec *)px_buf(ctx, B_BEST, sizeof(BestRec) * (max_blocks + 1));
   if (!d_blocks) return px_fail(ctx, PROTEUS_ENOMEM, "block results");
-  BestRec *d_best = d_blocks + max_blocks;
   for (int v = vec_lo; v < vec_hi; v++) {
     const int32_t *dem = h_demand + (size_t)v * Q;
     for (int q = 0; q < Q; q++) ea.s[q] = dem[q];
     SolRec *rec = d_sol + (materialize_only ? 0 : v - vec_lo);
     uint64_t ncand = 0;
+    int nb_used = 0;
     if (!materialize_only) {
       int nb = 0;
       if (flat_ok) {
@@ -513,10 +521,10 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
         PX_LAUNCH(ctx, "score_generic", k_enum_generic, (unsigned)nb64, GEN_THREADS, 0, ea);
         nb = (int)nb64;
       }
-      PX_LAUNCH(ctx, "argmax_grid", k_best_final, 1, 1024, 0, d_blocks, nb, d_best);
+      nb_used = nb;
     }
-    PX_LAUNCH(ctx, "materialize", k_materialize_enum, 1, 32, 0, ea, d_best, mat_index, materialize_only ? 1 : 0,
-              ncand, rec);
+    PX_LAUNCH(ctx, "argmax_materialize", k_materialize_enum, 1, 1024, 0, ea, d_blocks, nb_used, mat_index,
+              materialize_only ? 1 : 0, ncand, rec);
   }
   return 0;
 }
