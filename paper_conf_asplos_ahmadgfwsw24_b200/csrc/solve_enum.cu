@@ -343,10 +343,10 @@ __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const Bes
     r.n_candidates = n_candidates; r.status = 0;
     return;
   }
-  int32_t opt[PX_MAXD];
+  int32_t opt[PX_MAXD], o[PX_MAXD], z[PX_MAXD];  // thread-local: no global read-after-write
   decode_index(a, idx, opt);
-  for (int d = 0; d < a.D; d++) { r.option[d] = 0; r.z[d] = 0; }
-  for (int p = 0; p < a.npos; p++) r.option[a.pos_dev[p]] = opt[p];
+  for (int d = 0; d < a.D; d++) { o[d] = 0; z[d] = 0; }
+  for (int p = 0; p < a.npos; p++) o[a.pos_dev[p]] = opt[p];
   int64_t served = 0, accsum = 0, stot = 0;
   uint64_t score = 0;
   for (int q = 0; q < a.Q; q++) {
@@ -354,12 +354,12 @@ __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const Bes
     uint64_t acc = 0;
     stot += a.s[q];
     for (int j = 0; j < a.V[q]; j++) {
-      const int code = a.slot_code[q * a.VM + j];
-      const int A = a.slot_acc[q * a.VM + j];
+      const int code = __ldg(&a.slot_code[q * a.VM + j]);
+      const int A = __ldg(&a.slot_acc[q * a.VM + j]);
       for (int d = 0; d < a.D; d++) {
-        if (r.option[d] != code) continue;
-        const int t = min(rem, a.Pdev[d * a.K + code]);
-        r.z[d] = t;
+        if (o[d] != code) continue;
+        const int t = min(rem, __ldg(&a.Pdev[d * a.K + code]));
+        z[d] = t;
         rem -= t;
         acc += (uint64_t)A * (uint64_t)t;
       }
@@ -368,6 +368,7 @@ __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const Bes
     accsum += (int64_t)acc;
     score += px_pack((uint32_t)(a.s[q] - rem), acc);
   }
+  for (int d = 0; d < a.D; d++) { r.option[d] = o[d]; r.z[d] = z[d]; }
   r.score = score;
   r.index = idx;
   r.served = served;

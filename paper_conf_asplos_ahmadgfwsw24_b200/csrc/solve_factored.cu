@@ -292,22 +292,27 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
     __syncthreads();
     uint64_t *Gq = G + (size_t)q * U;
     for (int b = w; b < U; b += nw) {
-      int bv[PX_MAXT], box = 1;
-      for (int t = 0; t < T; t++) { bv[t] = (b / f.ustride[t]) % (f.Nt[t] + 1); box *= bv[t] + 1; }
+      // lanes split the usages of types 1..T-1; each lane walks type 0's range
+      int bv[PX_MAXT], inner = 1;
+      for (int t = 0; t < T; t++) bv[t] = (b / f.ustride[t]) % (f.Nt[t] + 1);
+      for (int t = 1; t < T; t++) inner *= bv[t] + 1;
+      const int s0 = f.ustride[0];
       uint64_t best = 0;
       bool have = false;
-      for (int i = lane; i < box; i += 32) {
-        int x = i, uk = 0, rk = 0;
-        for (int t = T - 1; t >= 0; t--) {
+      for (int i = lane; i < inner; i += 32) {
+        int x = i, uk = 0, rk = bv[0] * s0;
+        for (int t = T - 1; t >= 1; t--) {
           const int ut = x % (bv[t] + 1);
           x /= bv[t] + 1;
           uk += ut * f.ustride[t];
           rk += (bv[t] - ut) * f.ustride[t];
         }
-        const uint64_t gs = gq[uk];
-        if (gs == NONE) continue;
-        const uint64_t c = gs + Gn[rk];
-        if (!have || c > best) { best = c; have = true; }
+        for (int u0 = 0; u0 <= bv[0]; u0++, uk += s0, rk -= s0) {
+          const uint64_t gs = gq[uk];
+          if (gs == NONE) continue;
+          const uint64_t c = gs + Gn[rk];
+          if (!have || c > best) { best = c; have = true; }
+        }
       }
       for (int o = 16; o; o >>= 1) {
         const uint64_t b2 = __shfl_xor_sync(0xffffffffu, best, o);
@@ -362,7 +367,8 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
   int status = 0;
   for (int q = 0; q < Q; q++)
     if (pick_sub[q] == ~0ull) status = 2;
-  for (int d = 0; d < D; d++) { r.option[d] = 0; r.z[d] = 0; }
+  int32_t lopt[PX_MAXD], lz[PX_MAXD];  // thread-local: no global read-after-write
+  for (int d = 0; d < D; d++) { lopt[d] = 0; lz[d] = 0; }
   for (int t = 0; t < T && !status; t++) {
     int d = 0;
     for (int q = 0; q < Q; q++) {
@@ -374,7 +380,7 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
         for (int k = 0; k < ec[v]; k++) {
           while (d < D && dev_type[d] != t) d++;
           if (d >= D) { status = 3; break; }
-          r.option[d] = 1 + f.off[q] + v;
+          lopt[d] = 1 + f.off[q] + v;
           d++;
         }
     }
@@ -391,9 +397,9 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
       if (!code) continue;
       const int A = slot_acc[q * f.VM + j];
       for (int d = 0; d < D; d++) {
-        if (r.option[d] != code) continue;
+        if (lopt[d] != code) continue;
         const int tk = min(rem, Pdev[d * K + code]);
-        r.z[d] = tk;
+        lz[d] = tk;
         rem -= tk;
         acc += (uint64_t)A * (uint64_t)tk;
       }
@@ -402,6 +408,7 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
     accsum += (int64_t)acc;
     score += px_pack((uint32_t)(s[q] - rem), acc);
   }
+  for (int d = 0; d < D; d++) { r.option[d] = lopt[d]; r.z[d] = lz[d]; }
   if (score != G[U - 1]) status = status ? status : 1;
   uint64_t ncand = 0;
   for (int q = 0; q < Q; q++) {
@@ -465,7 +472,10 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
   const int64_t nitems = (int64_t)n_vec * Q * U;
   if (n_vec >= 8 && VM <= 8) {
     dim3 grid((unsigned)((Q * U + 3) / 4), (unsigned)((n_vec + 31) / 32));
-    if (VM <= 4) PX_LAUNCH(ctx, "fact_g", k_fact_gv<4>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
+    if (VM <= 3) PX_LAUNCH(ctx, "fact_g", k_fact_gv<3>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
+    else if (VM == 4) PX_LAUNCH(ctx, "fact_g", k_fact_gv<4>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
+    else if (VM == 5) PX_LAUNCH(ctx, "fact_g", k_fact_gv<5>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
+    else if (VM == 6) PX_LAUNCH(ctx, "fact_g", k_fact_gv<6>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
     else PX_LAUNCH(ctx, "fact_g", k_fact_gv<8>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
   } else {
     PX_LAUNCH(ctx, "fact_g", k_fact_g, (unsigned)((nitems + FG_WARPS - 1) / FG_WARPS), FG_WARPS * 32, 0, f, n_vec,
