@@ -97,15 +97,21 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.sm)}
 
 
-# algorithmic int32 ops of the pair-incremental scoring
+# algorithmic int32 lane-ops per candidate of the pair-incremental scoring in
+# k_flat_pair: per prefix (options of devices 0..D-3) the K^2
+# candidates of the last two devices.  fill = one family water-fill of V
+# variants (min, multiply-add, subtract per variant; pack 2).
 def flat_pair_ops_per_candidate(Q, V, K):
     S = Q * V
     fill = 3 * V + 2
-    per_prefix = (S                       # add device D-3's capacity
+    per_prefix = (S                       # add device D-3's capacity to its slot
                   + Q * fill              # family values of the prefix
-                  + 2 * S * (fill + 2)    # deltas of the last two devices
-                  + Q * V * V * (fill + 4)  # joint fills when both host one family
-                  + K * K * 4)            # 64-bit add + compare per candidate
+                  + S * (fill + 2)        # deltas Fb of every option of device D-1
+                  + 2 + 2 + 2 * S         # idle row: threshold, (idle, idle), (idle, sb) compares
+                  + S * ((fill + 4)       # row sa: delta of device D-2's option, ba
+                         + 2 + 2          #   threshold, (sa, idle) compare
+                         + 2 * (S - V)    #   other-family candidates: one 64-bit compare each
+                         + V * (fill + 6)))  # same-family candidates: joint fill, combine, compare
     return per_prefix / (K * K)
 
 

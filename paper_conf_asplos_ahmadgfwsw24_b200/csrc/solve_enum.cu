@@ -414,6 +414,11 @@ static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p
   a.p_lo = p_lo; a.p_hi = p_hi;
   a.per_thread = (np + nb * FLAT_THREADS - 1) / (nb * FLAT_THREADS);
   if (a.per_thread == 0) a.per_thread = 1;
+  // a multiple of K: every thread's prefix counter then carries (and rebuilds
+  // the capacities of devices 0..D-4) in the same iteration -- no divergence
+  if (a.per_thread > (uint64_t)K) a.per_thread = (a.per_thread + K - 1) / K * K;
+  nb = (np + a.per_thread * FLAT_THREADS - 1) / (a.per_thread * FLAT_THREADS);
+  if (nb == 0) nb = 1;
   PX_LAUNCH(ctx, "score_flat_pair", kern, (unsigned)nb, FLAT_THREADS, smem, a);
   *nblocks_out = (int)nb;
   return 0;
