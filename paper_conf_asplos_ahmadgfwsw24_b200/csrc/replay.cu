@@ -356,12 +356,14 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   __shared__ int32_t sG[PX_MAXD + 1];
   for (int k = threadIdx.x; k <= a.D; k += blockDim.x) sG[k] = a.goff[k];
   __syncthreads();
+  // blockIdx.x = scenario (fastest): consecutive blocks replay the same chunks
+  // for different scenarios, so the device arrays are read from L2
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int g = blockIdx.x * 4 + w;
+  const int g = blockIdx.y * 4 + w;
   if (g >= sG[a.D]) return;
   int d = 0;
   while (g >= sG[d + 1]) d++;
-  const int s = a.sc_list[blockIdx.y];
+  const int s = a.sc_list[blockIdx.x];
   const LaneParam p = a.lp[s * a.D + d];
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
@@ -644,14 +646,21 @@ __global__ void k_count(int64_t N, int S, int D, const int32_t *__restrict__ sc_
   const int64_t per = (N + gridDim.x - 1) / gridDim.x;
   const int64_t lo = (int64_t)blockIdx.x * per, hi = lo + per < N ? lo + per : N;
   int d = 0;
-  for (int64_t p0 = lo; p0 < hi; p0 += blockDim.x) {
+  for (int64_t p0 = lo; p0 < hi; p0 += 4 * blockDim.x) {
     while (d < D && sOff[d + 1] <= p0) d++;  // segment of this step's first position (uniform)
-    const int64_t p = p0 + threadIdx.x;
-    if (p < hi) {
+    uint32_t l[4];
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const int64_t p = p0 + threadIdx.x + (int64_t)k * blockDim.x;
+      l[k] = p < hi ? row[p] : 0;
+    }
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      const int64_t p = p0 + threadIdx.x + (int64_t)k * blockDim.x;
+      if (p >= hi) continue;
       int dd = d;
       while (dd < D && sOff[dd + 1] <= p) dd++;
-      const uint32_t l = row[p];
-      if ((int64_t)l > sL[dd]) viol++;
+      if ((int64_t)l[k] > sL[dd]) viol++;
       else { ont++; accs += sA[dd]; }
     }
   }
@@ -674,17 +683,34 @@ __global__ void k_count(int64_t N, int S, int D, const int32_t *__restrict__ sc_
 
 // per-query order: out[s][i] = latd[s][inv(i)] (coalesced stores, gathered loads
 // that walk ~D sequential streams)
-__global__ void k_unpermute(int64_t N, int S, const proteus_scenario *__restrict__ sc, const uint32_t *__restrict__ inv0,
-                            const uint32_t *__restrict__ inv1, const uint32_t *__restrict__ latd, uint32_t *out) {
+#define UNP_PER 16
+__global__ void __launch_bounds__(256) k_unpermute(int64_t N, int S, const proteus_scenario *__restrict__ sc,
+                                                   const uint32_t *__restrict__ inv0, const uint32_t *__restrict__ inv1,
+                                                   const uint32_t *__restrict__ latd, uint32_t *out) {
+  // one block per chunk of 256 * UNP_PER queries, all scenario rows: every
+  // 32-byte sector of a device stream read for a row is used by this block,
+  // and the positions stay in registers across the rows
   __shared__ int8_t rt[4096];
   for (int k = threadIdx.x; k < S; k += blockDim.x) rt[k] = (int8_t)sc[k].routing;
   __syncthreads();
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
-    const uint32_t p0 = inv0 ? inv0[i] : 0, p1 = inv1 ? inv1[i] : 0;
-    for (int s = 0; s < S; s++) {
-      const size_t r = (size_t)s * N;
-      out[r + i] = latd[r + (rt[s] ? p1 : p0)];
-    }
+  const int64_t i0 = (int64_t)blockIdx.x * (256 * UNP_PER) + threadIdx.x;
+  uint32_t p0[UNP_PER], p1[UNP_PER];
+#pragma unroll
+  for (int k = 0; k < UNP_PER; k++) {
+    const int64_t i = i0 + 256 * k;
+    p0[k] = (inv0 && i < N) ? inv0[i] : 0;
+    p1[k] = (inv1 && i < N) ? inv1[i] : 0;
+  }
+  for (int s = 0; s < S; s++) {
+    const size_t r = (size_t)s * N;
+    const bool m1 = rt[s] != 0;
+    uint32_t v[UNP_PER];
+#pragma unroll
+    for (int k = 0; k < UNP_PER; k++)
+      if (i0 + 256 * k < N) v[k] = latd[r + (m1 ? p1[k] : p0[k])];
+#pragma unroll
+    for (int k = 0; k < UNP_PER; k++)
+      if (i0 + 256 * k < N) out[r + i0 + 256 * k] = v[k];
   }
 }
 
@@ -820,7 +846,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
     } else {
       if (ngroups[rt] > 0) {
-        dim3 grid((unsigned)((ngroups[rt] + 3) / 4), (unsigned)la.nsc);
+        if ((ngroups[rt] + 3) / 4 > 65535) return px_fail(ctx, PROTEUS_ERANGE, "too many replay chunks");
+        dim3 grid((unsigned)la.nsc, (unsigned)((ngroups[rt] + 3) / 4));
         PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la);
       }
       const int64_t warps = (int64_t)la.nsc * D;
@@ -832,7 +859,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     int nsm = 0;
     PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
     int64_t cbx = (N + 4095) / 4096;
-    const int64_t cap_bx = ((int64_t)nsm * 16 + la.nsc - 1) / la.nsc;
+    const int64_t cap_bx = ((int64_t)nsm * 64 + la.nsc - 1) / la.nsc;
     if (cbx > cap_bx) cbx = cap_bx > 0 ? cap_bx : 1;
     dim3 cg((unsigned)cbx, (unsigned)la.nsc);
     PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, S, D, d_scl + rt * S, devOff[rt], d_lp, latd, d_agg);
@@ -840,8 +867,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   if (d_lat_out) {
     int nsm = 0;
     PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
-    int64_t nb = (N + 255) / 256;
-    if (nb > (int64_t)nsm * 8) nb = (int64_t)nsm * 8;
+    const int64_t nb = (N + 256 * UNP_PER - 1) / (256 * UNP_PER);
     PX_LAUNCH(ctx, "replay_unpermute", k_unpermute, (unsigned)nb, 256, 0, N, S, d_sc, inv[0], inv[1], latd, d_lat_out);
   }
   return 0;

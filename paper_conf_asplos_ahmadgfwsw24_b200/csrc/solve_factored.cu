@@ -291,35 +291,35 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
     }
     __syncthreads();
     uint64_t *Gq = G + (size_t)q * U;
-    for (int b = w; b < U; b += nw) {
-      // lanes split the usages of types 1..T-1; each lane walks type 0's range
-      int bv[PX_MAXT], inner = 1;
-      for (int t = 0; t < T; t++) bv[t] = (b / f.ustride[t]) % (f.Nt[t] + 1);
-      for (int t = 1; t < T; t++) inner *= bv[t] + 1;
-      const int s0 = f.ustride[0];
-      uint64_t best = 0;
-      bool have = false;
-      for (int i = lane; i < inner; i += 32) {
-        int x = i, uk = 0, rk = bv[0] * s0;
-        for (int t = T - 1; t >= 1; t--) {
-          const int ut = x % (bv[t] + 1);
-          x /= bv[t] + 1;
-          uk += ut * f.ustride[t];
-          rk += (bv[t] - ut) * f.ustride[t];
-        }
-        for (int u0 = 0; u0 <= bv[0]; u0++, uk += s0, rk -= s0) {
+    // one thread per budget b; budgets b and U-1-b (complementary boxes) go to
+    // the same thread to balance the work; the box {u <= b} is walked with an
+    // odometer (u key up, remainder key down) -- no division per element
+    for (int i = threadIdx.x; 2 * i < U; i += blockDim.x) {
+      for (int half = 0; half < 2; half++) {
+        const int b = half ? U - 1 - i : i;
+        if (half && b == i) break;
+        int bv[PX_MAXT], u[PX_MAXT];
+        for (int t = 0; t < T; t++) { bv[t] = (b / f.ustride[t]) % (f.Nt[t] + 1); u[t] = 0; }
+        int uk = 0, rk = b;
+        uint64_t best = 0;
+        bool have = false;
+        for (;;) {
           const uint64_t gs = gq[uk];
-          if (gs == NONE) continue;
-          const uint64_t c = gs + Gn[rk];
-          if (!have || c > best) { best = c; have = true; }
+          if (gs != NONE) {
+            const uint64_t c = gs + Gn[rk];
+            if (!have || c > best) { best = c; have = true; }
+          }
+          int t = T - 1;
+          for (; t >= 0; t--) {
+            if (u[t] < bv[t]) { u[t]++; uk += f.ustride[t]; rk -= f.ustride[t]; break; }
+            uk -= u[t] * f.ustride[t];
+            rk += u[t] * f.ustride[t];
+            u[t] = 0;
+          }
+          if (t < 0) break;
         }
+        Gq[b] = best;  // u = 0 is always valid: have == true
       }
-      for (int o = 16; o; o >>= 1) {
-        const uint64_t b2 = __shfl_xor_sync(0xffffffffu, best, o);
-        const int h2 = __shfl_xor_sync(0xffffffffu, (int)have, o);
-        if (h2 && (!have || b2 > best)) { best = b2; have = true; }
-      }
-      if (lane == 0) Gq[b] = best;  // u = 0 is always valid: have == true
     }
     __syncthreads();
     for (int b = threadIdx.x; b < U; b += blockDim.x) Gn[b] = Gq[b];
