@@ -94,6 +94,11 @@ struct proteus_ctx {
   bool tab_valid = false;
   std::vector<int32_t> tab_key, tab_P, tab_slot_code;
   Tables tab;
+  // cached DP key pairs of the factored search (solve_factored.cu)
+  void *dp_pairs = nullptr;
+  int64_t dp_pairs_n = 0;
+  int32_t dp_pairs_U = -1;
+  std::vector<int32_t> dp_pairs_key;
 };
 
 // scratch buffer ids

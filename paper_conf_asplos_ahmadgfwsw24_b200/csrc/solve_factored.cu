@@ -41,6 +41,8 @@ struct FactLayout {
   int32_t *ecap;       // [entries][VM] capacity vector in fill (slot) order
   uint8_t *ecnt;       // [entries][16] counts in caller's variant order
   int32_t *esum;       // [entries]
+  const int2 *pairs;   // DP: for each budget b, the keys (u, b - u) of every u <= b
+  const int32_t *pstart;  // [U + 1] offsets into pairs
 };
 
 // ------------------------------------------------------------- lists ----
@@ -291,35 +293,24 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
     }
     __syncthreads();
     uint64_t *Gq = G + (size_t)q * U;
-    // one thread per budget b; budgets b and U-1-b (complementary boxes) go to
-    // the same thread to balance the work; the box {u <= b} is walked with an
-    // odometer (u key up, remainder key down) -- no division per element
-    for (int i = threadIdx.x; 2 * i < U; i += blockDim.x) {
-      for (int half = 0; half < 2; half++) {
-        const int b = half ? U - 1 - i : i;
-        if (half && b == i) break;
-        int bv[PX_MAXT], u[PX_MAXT];
-        for (int t = 0; t < T; t++) { bv[t] = (b / f.ustride[t]) % (f.Nt[t] + 1); u[t] = 0; }
-        int uk = 0, rk = b;
-        uint64_t best = 0;
-        bool have = false;
-        for (;;) {
-          const uint64_t gs = gq[uk];
-          if (gs != NONE) {
-            const uint64_t c = gs + Gn[rk];
-            if (!have || c > best) { best = c; have = true; }
-          }
-          int t = T - 1;
-          for (; t >= 0; t--) {
-            if (u[t] < bv[t]) { u[t]++; uk += f.ustride[t]; rk -= f.ustride[t]; break; }
-            uk -= u[t] * f.ustride[t];
-            rk += u[t] * f.ustride[t];
-            u[t] = 0;
-          }
-          if (t < 0) break;
-        }
-        Gq[b] = best;  // u = 0 is always valid: have == true
+    for (int b = w; b < U; b += nw) {
+      // lanes stride over the precomputed (u, b - u) key pairs of budget b
+      uint64_t best = 0;
+      bool have = false;
+      const int pe = f.pstart[b + 1];
+      for (int k = f.pstart[b] + lane; k < pe; k += 32) {
+        const int2 pr = __ldg(&f.pairs[k]);
+        const uint64_t gs = gq[pr.x];
+        if (gs == NONE) continue;
+        const uint64_t c = gs + Gn[pr.y];
+        if (!have || c > best) { best = c; have = true; }
       }
+      for (int o = 16; o; o >>= 1) {
+        const uint64_t b2 = __shfl_xor_sync(0xffffffffu, best, o);
+        const int h2 = __shfl_xor_sync(0xffffffffu, (int)have, o);
+        if (h2 && (!have || b2 > best)) { best = b2; have = true; }
+      }
+      if (lane == 0) Gq[b] = best;  // u = 0 is always valid: have == true
     }
     __syncthreads();
     for (int b = threadIdx.x; b < U; b += blockDim.x) Gn[b] = Gq[b];
@@ -464,6 +455,39 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
   f.ecap = (int32_t *)buf; buf += (size_t)total * VM * 4;
   f.esum = (int32_t *)buf; buf += (size_t)total * 4;
   f.ecnt = (uint8_t *)buf;
+  // the DP's (u, b - u) key pairs of every budget b (lattice indexing only)
+  if (ctx->dp_pairs_U != U || ctx->dp_pairs_key != std::vector<int32_t>(f.Nt, f.Nt + T)) {
+    std::vector<int32_t> pst(U + 1);
+    std::vector<int2> pr;
+    for (int b = 0; b < U; b++) {
+      pst[b] = (int32_t)pr.size();
+      int bv[PX_MAXT], box = 1;
+      for (int t = 0; t < T; t++) { bv[t] = (b / f.ustride[t]) % (f.Nt[t] + 1); box *= bv[t] + 1; }
+      for (int x0 = 0; x0 < box; x0++) {
+        int x = x0, uk = 0, rk = 0;
+        for (int t = T - 1; t >= 0; t--) {
+          const int ut = x % (bv[t] + 1);
+          x /= bv[t] + 1;
+          uk += ut * f.ustride[t];
+          rk += (bv[t] - ut) * f.ustride[t];
+        }
+        pr.push_back(make_int2(uk, rk));
+      }
+      if (pr.size() > (1u << 26)) return px_fail(ctx, PROTEUS_ERANGE, "usage lattice too large for the DP");
+    }
+    pst[U] = (int32_t)pr.size();
+    char *pb = (char *)px_buf(ctx, B_FACT3, pr.size() * sizeof(int2) + pst.size() * 4 + 64);
+    if (!pb) return px_fail(ctx, PROTEUS_ENOMEM, "DP pairs");
+    PX_CUDA(ctx, cudaMemcpyAsync(pb, pr.data(), pr.size() * sizeof(int2), cudaMemcpyHostToDevice, ctx->stream));
+    PX_CUDA(ctx, cudaMemcpyAsync(pb + pr.size() * sizeof(int2), pst.data(), pst.size() * 4, cudaMemcpyHostToDevice,
+                                 ctx->stream));
+    ctx->dp_pairs = pb;
+    ctx->dp_pairs_n = (int64_t)pr.size();
+    ctx->dp_pairs_U = U;
+    ctx->dp_pairs_key.assign(f.Nt, f.Nt + T);
+  }
+  f.pairs = (const int2 *)ctx->dp_pairs;
+  f.pstart = (const int32_t *)((const char *)ctx->dp_pairs + ctx->dp_pairs_n * sizeof(int2));
   const int n_vec = a->n_vec;
   BestRec *g = (BestRec *)px_buf(ctx, B_FACT1, sizeof(BestRec) * (size_t)n_vec * Q * U);
   uint64_t *G = (uint64_t *)px_buf(ctx, B_FACT2, 8 * (size_t)n_vec * (Q + 1) * U);
