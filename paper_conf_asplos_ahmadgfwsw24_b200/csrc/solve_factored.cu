@@ -173,24 +173,27 @@ __global__ void __launch_bounds__(FG_WARPS * 32) k_fact_g(const __grid_constant_
 // Batched variant for many demand vectors: the count vectors of a (family,
 // usage) cell and their capacity vectors do not depend on the demand, only
 // the water-fill does.  One warp per (family, usage, 32 vectors): the warp
-// walks the cell's candidates once in lexicographic-rank order (uniform
-// control flow, broadcast loads; type T-1 fastest, so ranks ascend), every
-// lane water-fills for its own vector and keeps its first maximum.
+// materialises the cell's candidates 64 at a time in shared memory (capacity
+// vector in fill order + lexicographic rank; lanes decode 2 each, type T-1
+// fastest so ranks ascend), then every lane water-fills each of them for its
+// own vector (broadcast loads) and keeps its first maximum.
+#define GV_TILE 64
 template <int VMT>
 __global__ void __launch_bounds__(128) k_fact_gv(const __grid_constant__ FactLayout f, int n_vec,
                                                  const int32_t *__restrict__ demand,
                                                  const int32_t *__restrict__ slot_acc, BestRec *g) {
-  const int lane = threadIdx.x & 31;
-  const int item = blockIdx.x * 4 + (threadIdx.x >> 5);
+  __shared__ int32_t tcap[4][GV_TILE][VMT];
+  __shared__ uint64_t tsub[4][GV_TILE];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int item = blockIdx.x * 4 + w;
   if (item >= f.Q * f.U) return;
   const int q = item / f.U, ukey = item % f.U;
   const int vec = blockIdx.y * 32 + lane;
   const bool active = vec < n_vec;
   const int s = active ? demand[(size_t)vec * f.Q + q] : 0;
   const int T = f.T, VM = f.VM;
-  int bsz[PX_MAXT], bst[PX_MAXT], o[PX_MAXT];
-  int64_t lstride[PX_MAXT];
-  bool empty = false;
+  int bsz[PX_MAXT], bst[PX_MAXT];
+  int64_t lstride[PX_MAXT], prod = 1;
   {
     int64_t ls = 1;
     for (int t = T - 1; t >= 0; t--) {
@@ -198,60 +201,52 @@ __global__ void __launch_bounds__(128) k_fact_gv(const __grid_constant__ FactLay
       const int32_t *bs = f.bstart + ((size_t)q * T + t) * (PX_MAXD + 2);
       bst[t] = bs[ut];
       bsz[t] = bs[ut + 1] - bs[ut];
-      empty |= bsz[t] == 0;
+      prod *= bsz[t];
       lstride[t] = ls;
       ls *= f.L[q * T + t];
-      o[t] = 0;
     }
   }
+  int A[VMT];
+#pragma unroll
+  for (int j = 0; j < VMT; j++) A[j] = j < VM ? slot_acc[q * VM + j] : 0;
   uint64_t best_s = 0, best_i = ~0ull;
-  if (!empty) {
-    int A[VMT];
+  for (int64_t k0 = 0; k0 < prod; k0 += GV_TILE) {
+    for (int r = lane; r < GV_TILE; r += 32) {
+      const int64_t k = k0 + r;
+      if (k >= prod) break;
+      int64_t x = k;
+      int cap[VMT];
 #pragma unroll
-    for (int j = 0; j < VMT; j++) A[j] = j < VM ? slot_acc[q * VM + j] : 0;
-    const int tl = T - 1;
-    const int32_t *binner = f.bucket + f.list_off[q][tl] + bst[tl];
-    const int32_t *einner = f.ecap + f.list_off[q][tl] * VM;
-    int pcap[VMT];
-    uint64_t psub = 0;
-    auto outer = [&]() {  // capacity and rank contribution of types 0..T-2
+      for (int j = 0; j < VMT; j++) cap[j] = 0;
+      uint64_t sub = 0;
+      for (int t = T - 1; t >= 0; t--) {
+        const int o = (int)(x % bsz[t]);
+        x /= bsz[t];
+        const int rk = f.bucket[f.list_off[q][t] + bst[t] + o];
+        sub += (uint64_t)rk * lstride[t];
+        const int32_t *ec = f.ecap + (f.list_off[q][t] + rk) * VM;
 #pragma unroll
-      for (int j = 0; j < VMT; j++) pcap[j] = 0;
-      psub = 0;
-      for (int t = 0; t < tl; t++) {
-        const int r = f.bucket[f.list_off[q][t] + bst[t] + o[t]];
-        psub += (uint64_t)r * lstride[t];
-        const int32_t *ec = f.ecap + (f.list_off[q][t] + r) * VM;
-#pragma unroll
-        for (int j = 0; j < VMT; j++) pcap[j] += j < VM ? ec[j] : 0;
+        for (int j = 0; j < VMT; j++) cap[j] += j < VM ? ec[j] : 0;
       }
-    };
-    outer();
-    for (;;) {
-      for (int k = 0; k < bsz[tl]; k++) {
-        const int r = binner[k];
-        const int32_t *ec = einner + (size_t)r * VM;
-        const uint64_t sub = psub + (uint64_t)r * lstride[tl];
-        int rem = s;
-        uint64_t acc = 0;
 #pragma unroll
-        for (int j = 0; j < VMT; j++) {
-          const int c = pcap[j] + (j < VM ? ec[j] : 0);
-          const int tk = min(rem, c);
-          acc += (uint64_t)(uint32_t)A[j] * (uint32_t)tk;
-          rem -= tk;
-        }
-        const uint64_t sc = px_pack((uint32_t)(s - rem), acc);
-        if (sc > best_s || best_i == ~0ull) { best_s = sc; best_i = sub; }
-      }
-      int t = tl - 1;
-      for (; t >= 0; t--) {
-        if (++o[t] < bsz[t]) break;
-        o[t] = 0;
-      }
-      if (t < 0) break;
-      outer();
+      for (int j = 0; j < VMT; j++) tcap[w][r][j] = cap[j];
+      tsub[w][r] = sub;
     }
+    __syncwarp();
+    const int nt = prod - k0 < GV_TILE ? (int)(prod - k0) : GV_TILE;
+    for (int r = 0; r < nt; r++) {
+      int rem = s;
+      uint64_t acc = 0;
+#pragma unroll
+      for (int j = 0; j < VMT; j++) {
+        const int tk = min(rem, tcap[w][r][j]);
+        acc += (uint64_t)(uint32_t)A[j] * (uint32_t)tk;
+        rem -= tk;
+      }
+      const uint64_t sc = px_pack((uint32_t)(s - rem), acc);
+      if (sc > best_s || best_i == ~0ull) { best_s = sc; best_i = tsub[w][r]; }
+    }
+    __syncwarp();
   }
   if (active) {
     BestRec &out = g[((size_t)vec * f.Q + q) * f.U + ukey];
