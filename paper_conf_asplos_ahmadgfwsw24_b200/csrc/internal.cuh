@@ -99,6 +99,9 @@ struct proteus_ctx {
   int64_t dp_pairs_n = 0;
   int32_t dp_pairs_U = -1;
   std::vector<int32_t> dp_pairs_key;
+  // cached count-vector lists of the factored search
+  void *fact_lists_buf = nullptr;
+  std::vector<int32_t> fact_lists_key;
 };
 
 // scratch buffer ids

@@ -444,6 +444,9 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
   const size_t szE = (size_t)total * (4 + (size_t)VM * 4 + 16 + 4);
   char *buf = (char *)px_buf(ctx, B_FACT0, szL + szB + szE + 64);
   if (!buf) return px_fail(ctx, PROTEUS_ENOMEM, "factored tables");
+  // the count-vector lists depend only on the (cached) capacity tables and the
+  // inventory: rebuilt only when those change
+  const bool lists_ok = ctx->tab_valid && ctx->fact_lists_buf == (void *)buf && ctx->fact_lists_key == ctx->tab_key;
   f.L = (int32_t *)buf; buf += szL;
   f.bstart = (int32_t *)buf; buf += szB;
   f.bucket = (int32_t *)buf; buf += (size_t)total * 4;
@@ -487,7 +490,11 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
   BestRec *g = (BestRec *)px_buf(ctx, B_FACT1, sizeof(BestRec) * (size_t)n_vec * Q * U);
   uint64_t *G = (uint64_t *)px_buf(ctx, B_FACT2, 8 * (size_t)n_vec * (Q + 1) * U);
   if (!g || !G) return px_fail(ctx, PROTEUS_ENOMEM, "factored DP buffers");
-  PX_LAUNCH(ctx, "fact_lists", k_fact_lists, (Q * T + 63) / 64, 64, 0, f, tab.P, tab.slot_of, ctx->M);
+  if (!lists_ok) {
+    PX_LAUNCH(ctx, "fact_lists", k_fact_lists, (Q * T + 63) / 64, 64, 0, f, tab.P, tab.slot_of, ctx->M);
+    ctx->fact_lists_buf = (void *)f.L;
+    ctx->fact_lists_key = ctx->tab_key;
+  }
   const int64_t nitems = (int64_t)n_vec * Q * U;
   if (n_vec >= 8 && VM <= 8) {
     dim3 grid((unsigned)((Q * U + 3) / 4), (unsigned)((n_vec + 31) / 32));

@@ -1,0 +1,35 @@
+"""Small invocations of every kernel, for compute-sanitizer (tests/test_gpu_sanitizer.py)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np  # noqa: E402
+
+from paper_conf_asplos_ahmadgfwsw24_b200 import Proteus, workloads as W  # noqa: E402
+
+
+def main():
+    px = Proteus(0)
+    cfg = W.config("c1")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    for mode in (0, 1, 2):
+        px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=mode)
+    px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=0, generic=True)
+    px.solve(cl.device_type, cl.slo_us, np.repeat(cfg["demand"], 9, axis=0), mode=2)  # batched kernel
+    cfg = W.config("c3", totals=(3000,))
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    sol = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=2)[0]
+    arr, fam = W.query_trace(6000, 3000.0, cfg["weights"], 3, "gamma")
+    sc = np.array([[1000, 1, 0], [2000, 4, 0], [3500, 0, 0], [1500, 0, 1]], np.int32)
+    os.environ["PROTEUS_REPLAY_CHUNK"] = "16"
+    px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
+    os.environ["PROTEUS_REPLAY_SIMPLE"] = "1"
+    px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
+    print("sanitize target done")
+
+
+if __name__ == "__main__":
+    main()
