@@ -266,6 +266,12 @@ struct LaneArgs {
   uint32_t *latd;         // [S][N] device-major
   SpecExit *ex;           // [S][NCH]
   uint64_t *agg;          // [3][S]
+  int maxchk;             // convergence checks per chunk (free decisions only)
+  int rmax;               // phase runs: lanes with 2 <= Bmax <= rmax speculate Bmax runs per chunk
+  uint32_t *vlat;         // latencies of the phase runs r >= 1 (lane base voff[lane] + (r - 1) n)
+  SpecExit *vex;          // their exit states (lane base voff[S D + lane] + (r - 1) nch)
+  const int64_t *voff;    // [2][S * D]
+  long long debug;        // > 0: k_stitch prints lanes slower than this many cycles (diagnostic)
 };
 
 __device__ __forceinline__ uint32_t sat_lat(int64_t l) { return l >= 0xFFFFFFFFll ? 0xFFFFFFFEu : (uint32_t)l; }
@@ -347,6 +353,11 @@ __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ 
   }
 }
 
+// number of speculative runs per chunk of a lane (see k_spec)
+__host__ __device__ __forceinline__ int n_phase_runs(int Bmax, int rmax) {
+  return (Bmax >= 2 && Bmax <= rmax) ? Bmax : 1;
+}
+
 // ---- phase A: speculative chunks
 // Each device array is cut into chunks of CH queries.  One warp per (device,
 // scenario, 32 consecutive chunks); lane = chunk, replayed from an idle
@@ -368,10 +379,13 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
   const int64_t c = (int64_t)(g - sG[d]) * 32 + lane;
+  const int r = blockIdx.z;  // phase run r: first batch starts at st + r
+  if (r > 0 && r >= n_phase_runs(p.Bmax, a.rmax)) return;
   if (c < nch) {
     const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
-    uint32_t *out = a.latd + (size_t)s * a.N + off;
-    int64_t h = st, F = 0;
+    const int64_t lane_id = (int64_t)s * a.D + d;
+    uint32_t *out = r == 0 ? a.latd + (size_t)s * a.N + off : a.vlat + a.voff[lane_id] + (int64_t)(r - 1) * n;
+    int64_t h = st + r, F = 0;
     if (p.Bmax < 1) {
       for (int64_t j = st; j < en; j++) out[j] = 0xFFFFFFFFu;
       h = en;
@@ -391,7 +405,8 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
     e.F = F;
     e.ov = (int32_t)(h - en);
     e.pad = 0;
-    a.ex[(size_t)s * a.NCH + a.choff[d] + c] = e;
+    if (r == 0) a.ex[(size_t)s * a.NCH + a.choff[d] + c] = e;
+    else a.vex[a.voff[(int64_t)a.S * a.D + lane_id] + (int64_t)(r - 1) * nch + c] = e;
   }
 }
 
@@ -413,6 +428,7 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
 #define SBUF 2048
 #define SAHEAD 1088
 #define SPECCAP 1024
+#define LEAN_C (1 << 30)
 
 struct BufArr {
   const uint32_t *buf, *g;
@@ -488,6 +504,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   __syncwarp();
   const uint32_t *garr = a.devArr + off;
   uint32_t *out = a.latd + (size_t)s * a.N + off;
+  const uint32_t *src = out;  // the speculative run the current chunk is matched against
   const SpecExit *ex = a.ex + (size_t)s * a.NCH + a.choff[d];
   BufArr A{bufA, garr, -(int64_t)(4 * SBUF)};
   auto ensure = [&](int64_t h) {
@@ -506,12 +523,28 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   int64_t spec_base = -1;
   auto spec_F = [&](int64_t j) -> int64_t {
     const int64_t o = j - spec_base;
-    const uint32_t l = (o >= 0 && o < SPECCAP) ? specL[o] : out[j];
+    const uint32_t l = (o >= 0 && o < SPECCAP) ? specL[o] : src[j];
     return (int64_t)A(j) + l;
   };
   const int64_t TB = T[p.Bmax - 1];
+  // the 32-bit decision needs L < C / 2 and every T(b) < C (so W_k < C and
+  // t + T(b) < 2^31); per-lane W_k = L - T(k + 2) and T(k + 1) for the
+  // first two ballot rounds stay in registers
+  int32_t tmax = 0;
+  for (int k = lane; k < p.Bmax; k += 32) tmax = T[k] > tmax ? T[k] : tmax;
+  tmax = __reduce_max_sync(0xffffffffu, tmax);
+  const bool lean = p.L < LEAN_C / 2 && tmax < LEAN_C;
+  const int32_t W0 = lane + 1 < p.Bmax ? (int32_t)p.L - T[lane + 1] : 0;
+  const int32_t W1 = lane + 33 < p.Bmax ? (int32_t)p.L - T[lane + 33] : 0;
+  const int32_t T0 = lane < p.Bmax ? T[lane] : 0;
+  const int32_t T1 = lane + 32 < p.Bmax ? T[lane + 32] : 0;
   const int64_t CH = a.CH;
+  const int R = n_phase_runs(p.Bmax, a.rmax);
+  const int64_t lane_id = (int64_t)s * a.D + d;
+  const uint32_t *vl = R > 1 ? a.vlat + a.voff[lane_id] : nullptr;
+  const SpecExit *vx = R > 1 ? a.vex + a.voff[(int64_t)a.S * a.D + lane_id] : nullptr;
   int64_t h = (CH < n ? CH : n) + ex[0].ov, F = ex[0].F;
+  long long dbg_t0 = clock64(), dbg_dec = 0, dbg_jump = 0, dbg_match = 0, dbg_chk = 0;
   for (int64_t c0 = 1; c0 < nch; c0 += 32) {
     int64_t pF = 0;
     int pov = 0;
@@ -532,17 +565,33 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
       }
       if (h >= en) continue;
       ensure(h);
-      if (h == st && F <= (int64_t)A(st)) {  // speculative start = true state
-        h = en + eov;
-        F = eF;
+      // match against the run whose first batch starts where the true one
+      // does: phase r = h - st (run 0 = the chunk's own start)
+      const int ovr = (int)(h - st);
+      const bool var = ovr > 0 && ovr < R;
+      int64_t xF = eF;
+      int xov = eov;
+      src = out;
+      if (var) {
+        src = vl + (int64_t)(ovr - 1) * n;
+        const SpecExit ve = vx[(int64_t)(ovr - 1) * nch + c0 + k];
+        xF = ve.F;
+        xov = ve.ov;
+      }
+      if ((ovr == 0 || var) && F <= (int64_t)A(h)) {  // speculative start = true state
+        if (var)
+          for (int64_t j = h + lane; j < en; j += 32) out[j] = src[j];
+        h = en + xov;
+        F = xF;
+        dbg_match++;
         continue;
       }
-      int checks = 2;
+      int checks = a.maxchk;
       {  // cache the speculative latencies of this chunk before overwriting any of them
         __syncwarp();
         spec_base = h;
         const int64_t m = en - h < SPECCAP ? en - h : SPECCAP;
-        for (int64_t i = lane; i < m; i += 32) specL[i] = out[h + i];
+        for (int64_t i = lane; i < m; i += 32) specL[i] = src[h + i];
         __syncwarp();
       }
       while (h < en) {
@@ -564,39 +613,99 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
             out[h + i] = sat_lat(F + (i / p.Bmax + 1) * TB - (int64_t)ab[h + i]);
           h += nq;
           F += (int64_t)r * TB;
+          dbg_jump++;
           continue;
         }
+        dbg_dec++;
         // one decision (see decide_par): queue states k = 0.. in rounds of 32;
         // states inside the initial queue are incomplete and never stop
-        const int64_t t0 = F > ah ? F : ah;
         int b;
-        int64_t t;
-        for (int kb = 0;; kb += 32) {
-          const int k = kb + lane;
-          bool stop = false, now = false;
-          int64_t tau = 0, W = 0;
-          if (k < p.Bmax && h + k < n) {
-            const int64_t ak = ab[h + k];
-            tau = ak > t0 ? ak : t0;
-            const bool capped = k + 1 == p.Bmax;
-            const int64_t nxt = h + k + 1 < n ? (int64_t)ab[h + k + 1] : INT64_MAX;
-            W = capped ? 0 : ah + p.L - T[k + 1];
-            now = capped || tau >= W;
-            stop = (capped || nxt > tau) && (now || nxt > W);
+        int64_t Fn;
+        bool isfree;
+        const int64_t fr = F - ah;
+        if (lean && fr < LEAN_C) {
+          // 32-bit form relative to a_h: d_k = min(a_{h+k} - a_h, C), t0 = max(F - a_h, 0),
+          // W_k = L - T(k + 2).  Exact: C > max W_k and t0 < C, and the first
+          // state whose next arrival clamps (d >= C) is preceded by a state
+          // that stops (its next arrival exceeds both tau and W), so no clamped
+          // value ever reaches the chosen state.
+          const int32_t t0 = fr > 0 ? (int32_t)fr : 0;
+          const int64_t rem = n - h;
+          const int lim = rem < p.Bmax ? (int)rem : p.Bmax;
+          const uint32_t uah = (uint32_t)ah;
+          for (int kb = 0;; kb += 32) {
+            const int k = kb + lane;
+            int32_t Wk, Tk;
+            if (kb == 0) {
+              Wk = W0;
+              Tk = T0;
+            } else if (kb == 32) {
+              Wk = W1;
+              Tk = T1;
+            } else {
+              Wk = k + 1 < p.Bmax ? (int32_t)p.L - T[k + 1] : 0;
+              Tk = k < p.Bmax ? T[k] : 0;
+            }
+            bool stop = false, fre = false;
+            int32_t cand = 0;
+            if (k < lim) {
+              const uint32_t du = ab[h + k] - uah;
+              const int32_t dk = du < (uint32_t)LEAN_C ? (int32_t)du : LEAN_C;
+              const int32_t tau = dk > t0 ? dk : t0;
+              const bool capped = k + 1 == p.Bmax;
+              int32_t nx = LEAN_C;
+              if (k + 1 < lim) {
+                const uint32_t dn = ab[h + k + 1] - uah;
+                nx = dn < (uint32_t)LEAN_C ? (int32_t)dn : LEAN_C;
+              }
+              const bool now = capped || tau >= Wk;
+              stop = (capped || nx > tau) && (now || nx > Wk);
+              const int32_t tr = now ? tau : Wk;
+              fre = tr > t0;
+              cand = tr + Tk;
+            }
+            const unsigned bal = __ballot_sync(0xffffffffu, stop);
+            const unsigned fb = __ballot_sync(0xffffffffu, fre);
+            if (bal) {
+              const int sl = __ffs(bal) - 1;
+              Fn = ah + __shfl_sync(0xffffffffu, cand, sl);
+              b = kb + sl + 1;
+              isfree = fr < 0 || ((fb >> sl) & 1u);
+              break;
+            }
           }
-          const unsigned bal = __ballot_sync(0xffffffffu, stop);
-          if (bal) {
-            const int src = __ffs(bal) - 1;
-            t = __shfl_sync(0xffffffffu, now ? tau : W, src);
-            b = kb + src + 1;
-            break;
+        } else {
+          const int64_t t0 = F > ah ? F : ah;
+          int64_t t;
+          for (int kb = 0;; kb += 32) {
+            const int k = kb + lane;
+            bool stop = false, now = false;
+            int64_t tau = 0, W = 0;
+            if (k < p.Bmax && h + k < n) {
+              const int64_t ak = ab[h + k];
+              tau = ak > t0 ? ak : t0;
+              const bool capped = k + 1 == p.Bmax;
+              const int64_t nxt = h + k + 1 < n ? (int64_t)ab[h + k + 1] : INT64_MAX;
+              W = capped ? 0 : ah + p.L - T[k + 1];
+              now = capped || tau >= W;
+              stop = (capped || nxt > tau) && (now || nxt > W);
+            }
+            const unsigned bal = __ballot_sync(0xffffffffu, stop);
+            if (bal) {
+              const int sl = __ffs(bal) - 1;
+              t = __shfl_sync(0xffffffffu, now ? tau : W, sl);
+              b = kb + sl + 1;
+              break;
+            }
           }
+          Fn = t + T[b - 1];
+          isfree = t > F;
         }
-        const int64_t Fn = t + T[b - 1];
         const int64_t j2 = h + b;
         bool conv = false;
-        if (t > F && j2 < en && checks > 0) {
+        if (isfree && j2 < en && checks > 0) {
           checks--;
+          dbg_chk++;
           conv = spec_F(j2 - 1) == Fn && spec_F(j2) != Fn;
         }
         __syncwarp();
@@ -605,12 +714,19 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         h = j2;
         F = Fn;
         if (conv) {
-          h = en + eov;
-          F = eF;
+          if (var)  // the rest of the chunk is the phase run's
+            for (int64_t jj = j2 + lane; jj < en; jj += 32) out[jj] = specL[jj - spec_base];
+          h = en + xov;
+          F = xF;
           break;
         }
       }
     }
+  }
+  if (a.debug && lane == 0) {
+    const long long cyc = clock64() - dbg_t0;
+    if (cyc > a.debug) printf("stitch s=%d d=%d n=%lld Bmax=%d L=%lld nch=%lld cycles=%lld dec=%lld jump=%lld match=%lld chk=%lld\n", s, d,
+                              (long long)n, p.Bmax, (long long)p.L, (long long)nch, cyc, dbg_dec, dbg_jump, dbg_match, dbg_chk);
   }
 }
 
@@ -825,7 +941,44 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * N * 4);  // B_R_LAT stages host outputs
   if (!latd) return px_fail(ctx, PROTEUS_ENOMEM, "latency scratch");
   SpecExit *ex = nullptr;
+  // phase runs (k_spec): lanes with 2 <= Bmax <= rmax also speculate each
+  // chunk from its (r + 1)-th query, r < Bmax, so the true run (which enters
+  // a chunk up to Bmax - 1 queries late) always has a run that starts with it
+  const int rmax = simple ? 1 : env_int("PROTEUS_REPLAY_PHASES", 8);
+  uint32_t *vlat = nullptr;
+  SpecExit *vex = nullptr;
+  int64_t *d_voff = nullptr;
+  int rz = 1;
   if (!simple) {
+    std::vector<int64_t> voff(2 * (size_t)S * D, 0);
+    int64_t vtot = 0, vxtot = 0;
+    for (int s = 0; s < S; s++) {
+      const int rt = h_sc[s].routing;
+      for (int d = 0; d < D; d++) {
+        int Bmax = 0;
+        if (h_option[d] > 0) {
+          const int32_t *Tr = ctx->lat.data() + ((size_t)h_dev_type[d] * M + (h_option[d] - 1)) * ctx->bmax;
+          int depth = 0;
+          while (depth < ctx->bmax && Tr[depth] > 0) depth++;
+          const int cap = h_sc[s].batch_cap;
+          Bmax = (cap > 0 && cap < depth) ? cap : depth;  // as k_lane_params
+        }
+        const int R = n_phase_runs(Bmax, rmax);
+        const int64_t nd = h_off[rt][d + 1] - h_off[rt][d], nchd = (nd + CH - 1) / CH;
+        voff[(size_t)s * D + d] = vtot;
+        voff[(size_t)S * D + (size_t)s * D + d] = vxtot;
+        vtot += (int64_t)(R - 1) * nd;
+        vxtot += (int64_t)(R - 1) * nchd;
+        if (R > rz && nchd > 1) rz = R;
+      }
+    }
+    if (rz > 1) {
+      vlat = (uint32_t *)px_buf(ctx, B_R_VLAT, (size_t)vtot * 4 + 16);
+      vex = (SpecExit *)px_buf(ctx, B_R_VEX, sizeof(SpecExit) * (size_t)(vxtot + 1));
+      d_voff = (int64_t *)px_buf(ctx, B_R_VOFF, voff.size() * 8);
+      if (!vlat || !vex || !d_voff) return px_fail(ctx, PROTEUS_ENOMEM, "phase-run buffers");
+      PX_CUDA(ctx, cudaMemcpyAsync(d_voff, voff.data(), voff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
+    }
     const int64_t nmax = NCH[0] > NCH[1] ? NCH[0] : NCH[1];
     ex = (SpecExit *)px_buf(ctx, B_R_LANE, sizeof(SpecExit) * (size_t)S * (nmax + 1));
     if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
@@ -841,13 +994,17 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     la.option = d_opt; la.dev_type = d_dev; la.lat = ctx->d_lat; la.sc_list = d_scl + rt * S; la.lp = d_lp;
     la.devOff = devOff[rt]; la.choff = d_choff + rt * (PX_MAXD + 2); la.goff = d_goff + rt * (PX_MAXD + 2);
     la.devArr = devArr[rt]; la.latd = latd; la.ex = ex; la.agg = d_agg;
+    la.debug = env_int("PROTEUS_REPLAY_DEBUG", 0);
+    la.maxchk = env_int("PROTEUS_REPLAY_CHECKS", 1 << 30);
+    la.rmax = rz > 1 ? rmax : 1;
+    la.vlat = vlat; la.vex = vex; la.voff = d_voff;
     if (simple) {
       const int nl = la.nsc * D;
       PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
     } else {
       if (ngroups[rt] > 0) {
         if ((ngroups[rt] + 3) / 4 > 65535) return px_fail(ctx, PROTEUS_ERANGE, "too many replay chunks");
-        dim3 grid((unsigned)la.nsc, (unsigned)((ngroups[rt] + 3) / 4));
+        dim3 grid((unsigned)la.nsc, (unsigned)((ngroups[rt] + 3) / 4), (unsigned)rz);
         PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la);
       }
       const int64_t warps = (int64_t)la.nsc * D;
