@@ -223,7 +223,7 @@ __global__ void k_scatter(const uint8_t *__restrict__ target, const uint32_t *__
 struct SpecExit {
   int64_t F;
   int32_t ov;  // exit head - chunk end (overhang of the last batch into the next chunk)
-  int32_t pad;
+  int32_t mer;  // phase runs: offset from the chunk start where the run met run 0 (else the chunk length)
 };
 
 struct LaneParam {  // per (scenario, device)
@@ -355,7 +355,7 @@ __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ 
 
 // number of speculative runs per chunk of a lane (see k_spec)
 __host__ __device__ __forceinline__ int n_phase_runs(int Bmax, int rmax) {
-  return (Bmax >= 2 && Bmax <= rmax) ? Bmax : 1;
+  return Bmax < 2 ? 1 : Bmax < rmax ? Bmax : rmax;
 }
 
 // ---- phase A: speculative chunks
@@ -363,7 +363,10 @@ __host__ __device__ __forceinline__ int n_phase_runs(int Bmax, int rmax) {
 // scenario, 32 consecutive chunks); lane = chunk, replayed from an idle
 // device (the true state at the start of the trace, R13).  All lanes follow
 // the same rule parameters, so the warp stays close to converged.
-__global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a) {
+// Launched twice: run 0 (rbase 0, gridDim.z 1), then the phase runs r >= 1
+// (rbase 1), which stop as soon as they meet run 0 (same batch end, same
+// finish) and take run 0's exit; `mer` records where.
+__global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a, int rbase) {
   __shared__ int32_t sG[PX_MAXD + 1];
   for (int k = threadIdx.x; k <= a.D; k += blockDim.x) sG[k] = a.goff[k];
   __syncthreads();
@@ -379,32 +382,50 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
   const int64_t c = (int64_t)(g - sG[d]) * 32 + lane;
-  const int r = blockIdx.z;  // phase run r: first batch starts at st + r
+  const int r = blockIdx.z + rbase;  // phase run r: first batch starts at st + r
   if (r > 0 && r >= n_phase_runs(p.Bmax, a.rmax)) return;
   if (c < nch) {
     const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
     const int64_t lane_id = (int64_t)s * a.D + d;
     uint32_t *out = r == 0 ? a.latd + (size_t)s * a.N + off : a.vlat + a.voff[lane_id] + (int64_t)(r - 1) * n;
     int64_t h = st + r, F = 0;
+    SpecExit e;
+    e.mer = (int32_t)(en - st);
+    bool met = false;
     if (p.Bmax < 1) {
       for (int64_t j = st; j < en; j++) out[j] = 0xFFFFFFFFu;
       h = en;
     } else {
       const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
       GArr arr{a.devArr + off};
+      const uint32_t *run0 = a.latd + (size_t)s * a.N + off;
       while (h < en) {
         int64_t t;
         const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
-        F = t + T[b - 1];
+        const int64_t Fn = t + T[b - 1];
         const int64_t jend = h + b < en ? h + b : en;
-        for (int64_t j = h; j < jend; j++) out[j] = sat_lat(F - (int64_t)arr(j));
-        h += b;
+        for (int64_t j = h; j < jend; j++) out[j] = sat_lat(Fn - (int64_t)arr(j));
+        const int64_t j2 = h + b;
+        // met run 0: it also ends a batch at j2 - 1 finishing at Fn (the next
+        // batch always finishes later); tested after batches the device waited for
+        if (r > 0 && t > F && j2 < en && (int64_t)arr(j2 - 1) + run0[j2 - 1] == Fn &&
+            (int64_t)arr(j2) + run0[j2] != Fn) {
+          met = true;
+          e.mer = (int32_t)(j2 - st);
+          break;
+        }
+        F = Fn;
+        h = j2;
       }
     }
-    SpecExit e;
-    e.F = F;
-    e.ov = (int32_t)(h - en);
-    e.pad = 0;
+    if (met) {
+      const SpecExit e0 = a.ex[(size_t)s * a.NCH + a.choff[d] + c];
+      e.F = e0.F;
+      e.ov = e0.ov;
+    } else {
+      e.F = F;
+      e.ov = (int32_t)(h - en);
+    }
     if (r == 0) a.ex[(size_t)s * a.NCH + a.choff[d] + c] = e;
     else a.vex[a.voff[(int64_t)a.S * a.D + lane_id] + (int64_t)(r - 1) * nch + c] = e;
   }
@@ -425,19 +446,30 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
 // taken 32 batches per step with a ballot.  Rewritten latencies adjust the
 // counts by their difference from the speculative ones.  Arrivals stream
 // through a shared-memory ring; exit states are fetched 32 chunks at a time.
-#define SBUF 2048
-#define SAHEAD 1088
-#define SPECCAP 1024
+#define SPECCAP 1024                 // chunk length limit of the stitch
+#define RSEG 1024                    // ring segment (queries), one bulk copy
+#define RING (4 * RSEG)              // per-warp arrival ring
+#define SPB (SPECCAP + 8)            // speculative-latency buffer (+ alignment lead)
 #define LEAN_C (1 << 30)
+#define SUMAX 4
 
-struct BufArr {
-  const uint32_t *buf, *g;
-  int64_t base;
-  __device__ __forceinline__ uint32_t operator()(int64_t j) const {
-    const int64_t o = j - base;
-    return (o >= 0 && o < SBUF) ? buf[o] : __ldg(g + j);
-  }
-};
+// TMA bulk copies (cp.async.bulk, global -> shared, completion on an mbarrier)
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t *bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+  // the generic-proxy reads of dst are done (caller's __syncwarp): order them before the async write
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+  asm volatile("{\n\t.reg .pred P1;\n\tWAIT_%=:\n\t"
+               "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+               "@!P1 bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
+}
 
 // number of j in [h + q, h + min(Bmax, n - h)) with arr(j) <= t, added to q
 // (arrivals are sorted, so the ballot is a prefix)
@@ -487,8 +519,13 @@ __device__ __forceinline__ int decide_par(const Arr &A, int64_t n, int64_t h, in
   }
 }
 
+__host__ __device__ __forceinline__ size_t stitch_wstride(int bmax) { return ((size_t)RING + 2 * SPB + 12 + bmax + 3) & ~(size_t)3; }
+static size_t stitch_smem(int bmax) { return 4 * stitch_wstride(bmax) * 4; }
+
 __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs a) {
-  extern __shared__ uint32_t ssm[];  // [4][SBUF] arrivals, then per warp: bmax T + SPECCAP spec latencies
+  // shared memory per warp: arrival ring [RING], spec latencies [2][SPB],
+  // mbarriers [4 ring + 2 spec], T [bmax]
+  extern __shared__ __align__(16) uint32_t ssm[];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t gw = (int64_t)blockIdx.x * 4 + w;
   if (gw >= (int64_t)a.nsc * a.D) return;
@@ -497,34 +534,72 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
   if (p.Bmax < 1 || nch < 2) return;
-  uint32_t *bufA = ssm + (size_t)w * SBUF;
-  int32_t *T = (int32_t *)(ssm + 4 * SBUF) + w * (a.bmax + SPECCAP);
+  uint32_t *wsm = ssm + (size_t)w * stitch_wstride(a.bmax);
+  uint32_t *ring = wsm;
+  uint32_t *specbuf = wsm + RING;
+  uint64_t *bars = (uint64_t *)(wsm + RING + 2 * SPB);  // [0..3] ring slots, [4..5] spec buffers
+  int32_t *T = (int32_t *)(wsm + RING + 2 * SPB + 12);
   const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
   for (int k = lane; k < a.bmax; k += 32) T[k] = Tg[k];
+  if (lane < 6) mbar_init(bars + lane);
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncwarp();
-  const uint32_t *garr = a.devArr + off;
   uint32_t *out = a.latd + (size_t)s * a.N + off;
   const uint32_t *src = out;  // the speculative run the current chunk is matched against
+  int64_t mr = 0;             // ... whose own latencies cover [h, mr), run 0's from mr on
   const SpecExit *ex = a.ex + (size_t)s * a.NCH + a.choff[d];
-  BufArr A{bufA, garr, -(int64_t)(4 * SBUF)};
-  auto ensure = [&](int64_t h) {
-    if (h >= A.base && h + SAHEAD <= A.base + SBUF) return;
-    __syncwarp();
-    A.base = h & ~(int64_t)31;
-    for (int k = lane; k < SBUF; k += 32) {
-      const int64_t j = A.base + k;
-      bufA[k] = j < n ? garr[j] : 0xFFFFFFFFu;
-    }
-    __syncwarp();
+  const int64_t CH = a.CH;
+  int64_t h = (CH < n ? CH : n) + ex[0].ov, F = ex[0].F;
+  // Arrivals stream through a 4-segment ring by TMA bulk copies of whole
+  // 1024-query segments of the routed array (segment g >> 10 of the absolute
+  // index g = off + j sits in slot (g >> 10) & 3, so ring[g & (RING - 1)] is
+  // query g).  Segments up to the one 2 past h's are in flight; a slot is
+  // refilled only after its previous segment has been waited for and lies
+  // 2 segments behind h (the stitch reads back at most Bmax - 1 <= 1023).
+  const int64_t sg0 = (off + CH) >> 10;  // first segment ever read (chunk 1 starts at CH)
+  int64_t sg_iss = sg0, sg_wait = sg0;
+  auto seg_wait_one = [&]() {
+    mbar_wait(bars + (sg_wait & 3), (uint32_t)(((sg_wait - sg0) >> 2) & 1));
+    sg_wait++;
   };
-  auto put = [&](int64_t j, int64_t Fb) { out[j] = sat_lat(Fb - (int64_t)A(j)); };
-  // speculative finish time of position j of the current chunk (cached before rewriting)
-  uint32_t *specL = (uint32_t *)(T + a.bmax);
+  auto seg_issue = [&](int64_t hcur) {
+    const int64_t lim = ((off + hcur) >> 10) + 3;
+    while (sg_iss < lim) {
+      while (sg_wait <= sg_iss - 4) seg_wait_one();
+      __syncwarp();
+      if (lane == 0) bulk_load(ring + (sg_iss & 3) * RSEG, a.devArr + sg_iss * RSEG, RSEG * 4, bars + (sg_iss & 3));
+      sg_iss++;
+    }
+  };
+  // make queries [.., jend) of the device readable (jend <= the segment 3 past h's)
+  auto need = [&](int64_t hcur, int64_t jend) {
+    seg_issue(hcur);
+    const int64_t gend = off + jend;
+    while (sg_wait * RSEG < gend) seg_wait_one();
+  };
+  auto AR = [&](int64_t j) -> int64_t { return ring[(off + j) & (RING - 1)]; };
+  auto put = [&](int64_t j, int64_t Fb) { out[j] = sat_lat(Fb - AR(j)); };
+  // Speculative latencies of chunk c (run 0) are bulk-copied into buffer
+  // (c - 1) & 1 while chunk c - 1 is stitched.
+  uint32_t *specL = specbuf;
   int64_t spec_base = -1;
+  auto spec_issue = [&](int64_t c) {
+    if (c >= nch) return;
+    const int bi = (int)((c - 1) & 1);
+    if (c >= 3) mbar_wait(bars + 4 + bi, (uint32_t)(((c - 3) >> 1) & 1));  // previous use consumed
+    __syncwarp();
+    if (lane == 0) {
+      const int64_t st = c * CH, en = st + CH < n ? st + CH : n;
+      const uintptr_t g = (uintptr_t)(out + st), g0 = g & ~(uintptr_t)15;
+      const uint32_t bytes = (uint32_t)(((g - g0) + (uintptr_t)(en - st) * 4 + 15) & ~(uintptr_t)15);
+      bulk_load(specbuf + bi * SPB, (const void *)g0, bytes, bars + 4 + bi);
+    }
+  };
+  spec_issue(1);
   auto spec_F = [&](int64_t j) -> int64_t {
     const int64_t o = j - spec_base;
-    const uint32_t l = (o >= 0 && o < SPECCAP) ? specL[o] : src[j];
-    return (int64_t)A(j) + l;
+    const uint32_t l = (o >= 0 && o < SPB) ? specL[o] : (j < mr ? src : out)[j];
+    return AR(j) + l;
   };
   const int64_t TB = T[p.Bmax - 1];
   // the 32-bit decision needs L < C / 2 and every T(b) < C (so W_k < C and
@@ -538,12 +613,17 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   const int32_t W1 = lane + 33 < p.Bmax ? (int32_t)p.L - T[lane + 33] : 0;
   const int32_t T0 = lane < p.Bmax ? T[lane] : 0;
   const int32_t T1 = lane + 32 < p.Bmax ? T[lane + 32] : 0;
-  const int64_t CH = a.CH;
   const int R = n_phase_runs(p.Bmax, a.rmax);
   const int64_t lane_id = (int64_t)s * a.D + d;
   const uint32_t *vl = R > 1 ? a.vlat + a.voff[lane_id] : nullptr;
   const SpecExit *vx = R > 1 ? a.vex + a.voff[(int64_t)a.S * a.D + lane_id] : nullptr;
-  int64_t h = (CH < n ? CH : n) + ex[0].ov, F = ex[0].F;
+  const int SU = p.Bmax >= 16 ? 1 : p.Bmax >= 8 ? 2 : SUMAX;  // batches per lane in a full-batch stretch
+  // SW: a full batch needs its last arrival <= max(F_i, a[h_i] + SW) (see the stretch)
+  int32_t tbig = 0;
+  for (int k = lane; k + 1 < p.Bmax; k += 32) tbig = T[k] > tbig ? T[k] : tbig;
+  tbig = __reduce_max_sync(0xffffffffu, tbig);
+  const int64_t SW = tbig <= TB ? (p.L - TB > 0 ? p.L - TB : 0) : INT64_MIN / 4;
+  bool lastfull = true;
   long long dbg_t0 = clock64(), dbg_dec = 0, dbg_jump = 0, dbg_match = 0, dbg_chk = 0;
   for (int64_t c0 = 1; c0 < nch; c0 += 32) {
     int64_t pF = 0;
@@ -558,63 +638,144 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
       const int64_t st = (c0 + k) * CH, en = st + CH < n ? st + CH : n;
       const int64_t eF = __shfl_sync(0xffffffffu, pF, k);
       const int eov = __shfl_sync(0xffffffffu, pov, k);
+      const int64_t c = c0 + k;
+      spec_issue(c + 1);
+      need(h, (h < en ? h : en) + p.Bmax + 1);
       if (h > st) {  // queries of this chunk in the last batch of the previous one
-        ensure(st);
         const int64_t hi = h < en ? h : en;
         for (int64_t j = st + lane; j < hi; j += 32) put(j, F);
       }
       if (h >= en) continue;
-      ensure(h);
       // match against the run whose first batch starts where the true one
       // does: phase r = h - st (run 0 = the chunk's own start)
       const int ovr = (int)(h - st);
       const bool var = ovr > 0 && ovr < R;
       int64_t xF = eF;
       int xov = eov;
+      mr = st;
       src = out;
       if (var) {
         src = vl + (int64_t)(ovr - 1) * n;
-        const SpecExit ve = vx[(int64_t)(ovr - 1) * nch + c0 + k];
+        const SpecExit ve = vx[(int64_t)(ovr - 1) * nch + c];
         xF = ve.F;
         xov = ve.ov;
+        mr = st + ve.mer;
       }
-      if ((ovr == 0 || var) && F <= (int64_t)A(h)) {  // speculative start = true state
-        if (var)
-          for (int64_t j = h + lane; j < en; j += 32) out[j] = src[j];
+      if ((ovr == 0 || var) && F <= AR(h)) {  // speculative start = true state
+        for (int64_t j = h + lane; j < mr; j += 32) out[j] = src[j];
         h = en + xov;
         F = xF;
         dbg_match++;
         continue;
       }
       int checks = a.maxchk;
-      {  // cache the speculative latencies of this chunk before overwriting any of them
-        __syncwarp();
+      // the speculative latencies of [h, en) are cached at the first meeting
+      // test of the chunk: the true run has only rewritten positions < h
+      spec_base = -1;
+      auto spec_cache = [&]() {
+        if (spec_base >= 0) return;
+        const int bi = (int)((c - 1) & 1);
+        specL = specbuf + bi * SPB;
+        mbar_wait(bars + 4 + bi, (uint32_t)(((c - 1) >> 1) & 1));  // run 0's, prefetched
+        if (!var) {
+          spec_base = st - (int64_t)(((uintptr_t)(out + st) & 15) >> 2);
+          return;
+        }
+        __syncwarp();  // a phase run's: plain loads over the prefetched copy
         spec_base = h;
-        const int64_t m = en - h < SPECCAP ? en - h : SPECCAP;
-        for (int64_t i = lane; i < m; i += 32) specL[i] = src[h + i];
+        const int64_t m = en - h;
+        for (int64_t i = lane; i < m; i += 32) specL[i] = (h + i < mr ? src : out)[h + i];
         __syncwarp();
-      }
+      };
       while (h < en) {
-        ensure(h);  // from here on [h, h + SAHEAD) is in the ring: plain shared loads
-        const uint32_t *ab = bufA - A.base;
-        const int64_t ah = ab[h];
-        if (F > ah && h + p.Bmax - 1 < n && (int64_t)ab[h + p.Bmax - 1] <= F) {
-          // backlog: full batches back to back
-          int64_t kmax = (en - h + p.Bmax - 1) / p.Bmax;
-          const int64_t room = (A.base + SBUF - h) / p.Bmax;
+        need(h, h + p.Bmax + 1);
+        const int64_t ah = AR(h);
+        if ((lastfull || F > ah) && h + p.Bmax - 1 < n &&
+            AR(h + p.Bmax - 1) <= (F > ah + SW ? F : ah + SW)) {
+          // full-batch stretch: while every batch is full (Bmax queries), batch i
+          // dispatches when the device is free and its last query has arrived,
+          // F_{i+1} = max(F_i, A_i) + T(Bmax), A_i = a[h_i + Bmax - 1], so
+          // F_i = i T(Bmax) + max(F_0, max_{j<i} (A_j - j T(Bmax))): a max-plus
+          // scan.  Batch i is full if A_i <= max(F_i, a[h_i] + SW): every queue
+          // state k < Bmax - 1 then has its next arrival <= max(tau_k, W_k)
+          // because W_k = a[h_i] + L - T(k+2) >= a[h_i] + L - T(Bmax) when
+          // T(Bmax) is the largest of T(1..Bmax) (else SW = -inf: A_i <= F_i,
+          // the queue already holds Bmax queries).  Rounds of 32 SU batches,
+          // lane l taking [l SU, l SU + SU) of the round.
+          int64_t kmax = (en - h + p.Bmax - 1) / p.Bmax;  // batches starting in this chunk
+          const int64_t room = ((((off + h) >> 10) + 3) * RSEG - (off + h)) / p.Bmax;
+          const int64_t avail = (n - h) / p.Bmax;
           if (kmax > room) kmax = room;
-          if (kmax > 32) kmax = 32;
-          const int64_t idx = h + (int64_t)(lane + 1) * p.Bmax - 1;
-          const bool ok = lane < kmax && idx < n && (int64_t)ab[idx] <= F + (int64_t)lane * TB;
-          const unsigned bal = __ballot_sync(0xffffffffu, ok);
-          const int r = bal == 0xffffffffu ? 32 : __ffs(~bal) - 1;
-          const int64_t nq = (int64_t)r * p.Bmax;
-          for (int64_t i = lane; i < nq; i += 32)
-            out[h + i] = sat_lat(F + (i / p.Bmax + 1) * TB - (int64_t)ab[h + i]);
-          h += nq;
-          F += (int64_t)r * TB;
-          dbg_jump++;
-          continue;
+          if (kmax > avail) kmax = avail;
+          need(h, h + kmax * p.Bmax);
+          int64_t Mc = F;  // max(F_0, G_j for the batches taken so far)
+          int64_t done = 0;
+          while (done < kmax) {
+            const int64_t ib = done + lane * SU;
+            int64_t G[SUMAX];
+            int64_t gl = INT64_MIN;
+#pragma unroll
+            for (int u = 0; u < SUMAX; u++) {
+              G[u] = INT64_MIN;
+              if (u < SU && ib + u < kmax) {
+                G[u] = AR(h + (ib + u + 1) * p.Bmax - 1) - (ib + u) * TB;
+                gl = G[u] > gl ? G[u] : gl;
+              }
+            }
+            int64_t inc = gl;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+              const int64_t v = __shfl_up_sync(0xffffffffu, inc, o);
+              if (lane >= o && v > inc) inc = v;
+            }
+            int64_t exc = __shfl_up_sync(0xffffffffu, inc, 1);
+            if (lane == 0) exc = INT64_MIN;
+            int64_t M = Mc > exc ? Mc : exc;
+            int fl = SU;
+#pragma unroll
+            for (int u = 0; u < SUMAX; u++) {
+              if (u < SU && fl == SU) {
+                const int64_t i = ib + u;
+                if (i >= kmax) {
+                  fl = u;
+                } else {
+                  const int64_t Fi = i * TB + M;
+                  const int64_t lim = AR(h + i * p.Bmax) + SW;
+                  if (G[u] + i * TB > (Fi > lim ? Fi : lim)) fl = u;
+                  else M = G[u] > M ? G[u] : M;
+                }
+              }
+            }
+            const unsigned bal = __ballot_sync(0xffffffffu, fl < SU);
+            const int fs = bal ? __ffs(bal) - 1 : 31;
+            const int64_t r = bal ? (int64_t)fs * SU + __shfl_sync(0xffffffffu, fl, fs) : 32 * SU;
+            // latencies of the accepted batches; lane l writes its own
+            M = Mc > exc ? Mc : exc;
+#pragma unroll
+            for (int u = 0; u < SUMAX; u++) {
+              const int64_t i = ib + u;
+              if (u < SU && i < done + r) {
+                M = G[u] > M ? G[u] : M;
+                const int64_t Fe = (i + 1) * TB + M;
+                const int64_t hi = h + i * p.Bmax;
+                for (int q = 0; q < p.Bmax; q++) out[hi + q] = sat_lat(Fe - AR(hi + q));
+              }
+            }
+            if (r > 0) {
+              Mc = __shfl_sync(0xffffffffu, M, (int)((r - 1) / SU));
+              done += r;
+            }
+            if (r < 32 * SU) break;
+          }
+          if (done > 0) {
+            F = done * TB + Mc;
+            h += done * p.Bmax;
+            lastfull = true;
+            dbg_jump++;
+            // no meeting test here: the latency cache is filled lazily and
+            // position h - 1 was just rewritten; the next decision tests
+            continue;
+          }
         }
         dbg_dec++;
         // one decision (see decide_par): queue states k = 0.. in rounds of 32;
@@ -649,13 +810,13 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
             bool stop = false, fre = false;
             int32_t cand = 0;
             if (k < lim) {
-              const uint32_t du = ab[h + k] - uah;
+              const uint32_t du = (uint32_t)AR(h + k) - uah;
               const int32_t dk = du < (uint32_t)LEAN_C ? (int32_t)du : LEAN_C;
               const int32_t tau = dk > t0 ? dk : t0;
               const bool capped = k + 1 == p.Bmax;
               int32_t nx = LEAN_C;
               if (k + 1 < lim) {
-                const uint32_t dn = ab[h + k + 1] - uah;
+                const uint32_t dn = (uint32_t)AR(h + k + 1) - uah;
                 nx = dn < (uint32_t)LEAN_C ? (int32_t)dn : LEAN_C;
               }
               const bool now = capped || tau >= Wk;
@@ -682,10 +843,10 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
             bool stop = false, now = false;
             int64_t tau = 0, W = 0;
             if (k < p.Bmax && h + k < n) {
-              const int64_t ak = ab[h + k];
+              const int64_t ak = AR(h + k);
               tau = ak > t0 ? ak : t0;
               const bool capped = k + 1 == p.Bmax;
-              const int64_t nxt = h + k + 1 < n ? (int64_t)ab[h + k + 1] : INT64_MAX;
+              const int64_t nxt = h + k + 1 < n ? AR(h + k + 1) : INT64_MAX;
               W = capped ? 0 : ah + p.L - T[k + 1];
               now = capped || tau >= W;
               stop = (capped || nxt > tau) && (now || nxt > W);
@@ -706,16 +867,18 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         if (isfree && j2 < en && checks > 0) {
           checks--;
           dbg_chk++;
+          spec_cache();
           conv = spec_F(j2 - 1) == Fn && spec_F(j2) != Fn;
         }
         __syncwarp();
         const int64_t hi = j2 < en ? j2 : en;
-        for (int64_t jj = h + lane; jj < hi; jj += 32) out[jj] = sat_lat(Fn - (int64_t)ab[jj]);
+        for (int64_t jj = h + lane; jj < hi; jj += 32) out[jj] = sat_lat(Fn - AR(jj));
         h = j2;
         F = Fn;
+        lastfull = b == p.Bmax;
         if (conv) {
-          if (var)  // the rest of the chunk is the phase run's
-            for (int64_t jj = j2 + lane; jj < en; jj += 32) out[jj] = specL[jj - spec_base];
+          // the rest of the chunk is the phase run's (run 0's from mr on)
+          for (int64_t jj = j2 + lane; jj < mr; jj += 32) out[jj] = specL[jj - spec_base];
           h = en + xov;
           F = xF;
           break;
@@ -892,7 +1055,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     int32_t *dbase = (int32_t *)px_buf(ctx, B_R_DBASE0, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
     uint8_t *tgt = (uint8_t *)px_buf(ctx, B_R_TGT, (size_t)N + 16);
     int64_t *off = (int64_t *)px_buf(ctx, rt ? B_R_OFF1 : B_R_OFF, (size_t)2 * (PX_MAXD + 2) * 8);
-    uint32_t *darr = (uint32_t *)px_buf(ctx, rt ? B_R_DEVARR1 : B_R_DEVARR, (size_t)N * 4 + 16);
+    // + whole trailing ring segment: k_stitch bulk-copies 4 KB segments
+    uint32_t *darr = (uint32_t *)px_buf(ctx, rt ? B_R_DEVARR1 : B_R_DEVARR, ((size_t)N + 2 * RSEG) * 4);
     uint32_t *dinv = (uint32_t *)px_buf(ctx, rt ? B_R_DEVIDX1 : B_R_DEVIDX, (size_t)N * 4 + 16);
     if (!pat || !hist || !fbase || !dbase || !tgt || !off || !darr || !dinv)
       return px_fail(ctx, PROTEUS_ENOMEM, "routing buffers");
@@ -915,7 +1079,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   }
   if (N == 0) return 0;
   // chunk layout per routing mode (sizes only): the host reads the per-device counts
-  const int CH = env_int("PROTEUS_REPLAY_CHUNK", 256);
+  int CH = env_int("PROTEUS_REPLAY_CHUNK", 1024);
+  CH = CH < 1 ? 1 : CH > SPECCAP ? SPECCAP : CH;  // the stitch caches one chunk
   const bool simple = env_int("PROTEUS_REPLAY_SIMPLE", 0) != 0;
   int64_t h_off[2][PX_MAXD + 2];
   for (int rt = 0; rt < 2; rt++)
@@ -938,13 +1103,13 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   }
   PX_CUDA(ctx, cudaMemcpyAsync(d_choff, choff.data(), choff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_goff, goff.data(), goff.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
-  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * N * 4);  // B_R_LAT stages host outputs
+  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * N * 4 + 64);  // B_R_LAT stages host outputs
   if (!latd) return px_fail(ctx, PROTEUS_ENOMEM, "latency scratch");
   SpecExit *ex = nullptr;
   // phase runs (k_spec): lanes with 2 <= Bmax <= rmax also speculate each
   // chunk from its (r + 1)-th query, r < Bmax, so the true run (which enters
   // a chunk up to Bmax - 1 queries late) always has a run that starts with it
-  const int rmax = simple ? 1 : env_int("PROTEUS_REPLAY_PHASES", 8);
+  const int rmax = simple ? 1 : env_int("PROTEUS_REPLAY_PHASES", 1);
   uint32_t *vlat = nullptr;
   SpecExit *vex = nullptr;
   int64_t *d_voff = nullptr;
@@ -983,7 +1148,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     ex = (SpecExit *)px_buf(ctx, B_R_LANE, sizeof(SpecExit) * (size_t)S * (nmax + 1));
     if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
     PX_CUDA(ctx, cudaFuncSetAttribute(k_stitch, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      4 * SBUF * 4 + 4 * (ctx->bmax + SPECCAP) * 4));
+                                      (int)stitch_smem(ctx->bmax)));
   }
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
@@ -1004,12 +1169,16 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     } else {
       if (ngroups[rt] > 0) {
         if ((ngroups[rt] + 3) / 4 > 65535) return px_fail(ctx, PROTEUS_ERANGE, "too many replay chunks");
-        dim3 grid((unsigned)la.nsc, (unsigned)((ngroups[rt] + 3) / 4), (unsigned)rz);
-        PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la);
+        dim3 grid((unsigned)la.nsc, (unsigned)((ngroups[rt] + 3) / 4));
+        PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la, 0);
+        if (rz > 1) {
+          dim3 gv(grid.x, grid.y, (unsigned)(rz - 1));
+          PX_LAUNCH(ctx, "replay_spec_phase", k_spec, gv, 128, 0, la, 1);
+        }
       }
       const int64_t warps = (int64_t)la.nsc * D;
       PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128,
-                4 * SBUF * 4 + 4 * (ctx->bmax + SPECCAP) * 4, la);
+                stitch_smem(ctx->bmax), la);
     }
     dim3 g(32, la.nsc < 65535 ? la.nsc : 65535);
     PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, N, S, D, d_scl + rt * S, la.nsc, devOff[rt], latd, d_agg);

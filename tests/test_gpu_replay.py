@@ -33,7 +33,7 @@ def _compare(px, oracle_mod, prof, cl, option, z, demand, arr, fam, sc):
 
 
 PATHS = {"chunked": {}, "small_chunks": {"PROTEUS_REPLAY_CHUNK": "16"}, "odd_chunks": {"PROTEUS_REPLAY_CHUNK": "37"},
-         "no_phase_runs": {"PROTEUS_REPLAY_PHASES": "1", "PROTEUS_REPLAY_CHUNK": "37"},
+         "phase_runs": {"PROTEUS_REPLAY_PHASES": "8", "PROTEUS_REPLAY_CHUNK": "37"},
          "all_phase_runs": {"PROTEUS_REPLAY_PHASES": "64", "PROTEUS_REPLAY_CHUNK": "100"},
          "simple": {"PROTEUS_REPLAY_SIMPLE": "1"}}
 
