@@ -8,7 +8,7 @@ import ctypes as C
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libproteus.so")
+LIB_PATH = os.environ.get("PROTEUS_LIB") or os.path.join(_PKG, "libproteus.so")  # override: diagnostics builds
 
 PROTEUS_OK = 0
 PROTEUS_EINVAL = -1

@@ -17,8 +17,10 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-OBJ = os.path.join(PKG, "_build")
-LIB = os.path.join(PKG, "libproteus.so")
+# PROTEUS_BUILD_DEFS="-DPX_STITCH_DEBUG" builds a diagnostics library libproteus_dbg.so
+DEFS = os.environ.get("PROTEUS_BUILD_DEFS", "").split()
+OBJ = os.path.join(PKG, "_build_dbg" if DEFS else "_build")
+LIB = os.path.join(PKG, "libproteus_dbg.so" if DEFS else "libproteus.so")
 INCLUDE = os.path.join(ROOT, "include")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -42,7 +44,7 @@ def _compile(src: str, verbose: bool) -> str:
     obj = os.path.join(OBJ, os.path.basename(src) + ".o")
     if os.path.exists(obj) and os.path.getmtime(obj) >= max(os.path.getmtime(src), _newest_header()):
         return obj
-    cmd = [_nvcc(), *ARCH, *NVCC_FLAGS, "-c", src, "-o", obj + ".tmp"]
+    cmd = [_nvcc(), *ARCH, *NVCC_FLAGS, *DEFS, "-c", src, "-o", obj + ".tmp"]
     if verbose:
         cmd += ["-Xptxas", "-v"]
     r = subprocess.run(cmd, capture_output=True, text=True)

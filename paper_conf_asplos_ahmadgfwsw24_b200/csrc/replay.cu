@@ -452,6 +452,11 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
 #define SPB (SPECCAP + 8)            // speculative-latency buffer (+ alignment lead)
 #define LEAN_C (1 << 30)
 #define SUMAX 4
+#ifdef PX_STITCH_DEBUG  // per-lane counters printed by k_stitch (PROTEUS_REPLAY_DEBUG=cycles)
+#define PX_DBG(x) x
+#else
+#define PX_DBG(x)
+#endif
 
 // TMA bulk copies (cp.async.bulk, global -> shared, completion on an mbarrier)
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -571,13 +576,18 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
       sg_iss++;
     }
   };
-  // make queries [.., jend) of the device readable (jend <= the segment 3 past h's)
+  // make queries [.., jend) of the device readable (jend <= the segment 3 past h's);
+  // h_safe: below it a decision at h needs no ring work (issue or wait)
+  int64_t h_safe = 0;
   auto need = [&](int64_t hcur, int64_t jend) {
     seg_issue(hcur);
     const int64_t gend = off + jend;
     while (sg_wait * RSEG < gend) seg_wait_one();
+    const int64_t s1 = (sg_iss - 2) * RSEG - off, s2 = sg_wait * RSEG - off - p.Bmax;
+    h_safe = s1 < s2 ? s1 : s2;
   };
-  auto AR = [&](int64_t j) -> int64_t { return ring[(off + j) & (RING - 1)]; };
+  const uint32_t ro = (uint32_t)(off & (RING - 1));
+  auto AR = [&](int64_t j) -> int64_t { return ring[(ro + (uint32_t)j) & (RING - 1)]; };
   auto put = [&](int64_t j, int64_t Fb) { out[j] = sat_lat(Fb - AR(j)); };
   // Speculative latencies of chunk c (run 0) are bulk-copied into buffer
   // (c - 1) & 1 while chunk c - 1 is stitched.
@@ -596,11 +606,8 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
     }
   };
   spec_issue(1);
-  auto spec_F = [&](int64_t j) -> int64_t {
-    const int64_t o = j - spec_base;
-    const uint32_t l = (o >= 0 && o < SPB) ? specL[o] : (j < mr ? src : out)[j];
-    return AR(j) + l;
-  };
+  // j in [h, en): always inside the cached window [spec_base, en)
+  auto spec_F = [&](int64_t j) -> int64_t { return AR(j) + specL[(int32_t)(j - spec_base)]; };
   const int64_t TB = T[p.Bmax - 1];
   // the 32-bit decision needs L < C / 2 and every T(b) < C (so W_k < C and
   // t + T(b) < 2^31); per-lane W_k = L - T(k + 2) and T(k + 1) for the
@@ -625,6 +632,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   const int64_t SW = tbig <= TB ? (p.L - TB > 0 ? p.L - TB : 0) : INT64_MIN / 4;
   bool lastfull = true;
   long long dbg_t0 = clock64(), dbg_dec = 0, dbg_jump = 0, dbg_match = 0, dbg_chk = 0;
+  long long dbg_sec[5] = {0, 0, 0, 0, 0}, dbg_tk = 0;
   for (int64_t c0 = 1; c0 < nch; c0 += 32) {
     int64_t pF = 0;
     int pov = 0;
@@ -665,7 +673,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         for (int64_t j = h + lane; j < mr; j += 32) out[j] = src[j];
         h = en + xov;
         F = xF;
-        dbg_match++;
+        PX_DBG(dbg_match++);
         continue;
       }
       int checks = a.maxchk;
@@ -687,9 +695,12 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         for (int64_t i = lane; i < m; i += 32) specL[i] = (h + i < mr ? src : out)[h + i];
         __syncwarp();
       };
+      bool spec_ready = false;  // latency cache of this chunk loaded (at its first meeting test)
       while (h < en) {
-        need(h, h + p.Bmax + 1);
+        PX_DBG(if (dbg_tk) dbg_sec[3] += clock64() - dbg_tk; dbg_tk = clock64());
+        if (h >= h_safe) need(h, h + p.Bmax + 1);
         const int64_t ah = AR(h);
+        PX_DBG(__syncwarp(); dbg_sec[4] += clock64() - dbg_tk; dbg_tk = clock64());
         if ((lastfull || F > ah) && h + p.Bmax - 1 < n &&
             AR(h + p.Bmax - 1) <= (F > ah + SW ? F : ah + SW)) {
           // full-batch stretch: while every batch is full (Bmax queries), batch i
@@ -771,70 +782,118 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
             F = done * TB + Mc;
             h += done * p.Bmax;
             lastfull = true;
-            dbg_jump++;
+            PX_DBG(dbg_jump++);
             // no meeting test here: the latency cache is filled lazily and
             // position h - 1 was just rewritten; the next decision tests
             continue;
           }
         }
-        dbg_dec++;
+        PX_DBG(dbg_dec++; dbg_tk = clock64());
         // one decision (see decide_par): queue states k = 0.. in rounds of 32;
         // states inside the initial queue are incomplete and never stop
         int b;
         int64_t Fn;
-        bool isfree;
         const int64_t fr = F - ah;
         if (lean && fr < LEAN_C) {
           // 32-bit form relative to a_h: d_k = min(a_{h+k} - a_h, C), t0 = max(F - a_h, 0),
           // W_k = L - T(k + 2).  Exact: C > max W_k and t0 < C, and the first
           // state whose next arrival clamps (d >= C) is preceded by a state
           // that stops (its next arrival exceeds both tau and W), so no clamped
-          // value ever reaches the chosen state.
+          // value ever reaches the chosen state.  Lane k holds state k; it
+          // then writes query h + k's latency from its own d_k, and tests
+          // whether the speculative run's batch holding h + k finishes at Fn:
+          // the runs meet at j2 = h + b when lane b - 1 says yes and lane b no.
           const int32_t t0 = fr > 0 ? (int32_t)fr : 0;
           const int64_t rem = n - h;
           const int lim = rem < p.Bmax ? (int)rem : p.Bmax;
           const uint32_t uah = (uint32_t)ah;
-          for (int kb = 0;; kb += 32) {
-            const int k = kb + lane;
-            int32_t Wk, Tk;
-            if (kb == 0) {
-              Wk = W0;
-              Tk = T0;
-            } else if (kb == 32) {
-              Wk = W1;
-              Tk = T1;
+          const int k = lane;
+          const uint32_t du = (uint32_t)AR(h + k) - uah;
+          const uint32_t dn = (uint32_t)AR(h + k + 1) - uah;
+          const bool test = spec_ready && checks > 0;
+          const uint32_t sp = test && h + k < en ? specL[(int32_t)(h + k - spec_base)] : 0u;
+          const int32_t dk = du < (uint32_t)LEAN_C ? (int32_t)du : LEAN_C;
+          const int32_t tau = dk > t0 ? dk : t0;
+          const bool capped = k + 1 == p.Bmax;
+          const int32_t nx = k + 1 < lim ? (dn < (uint32_t)LEAN_C ? (int32_t)dn : LEAN_C) : LEAN_C;
+          const bool now = capped || tau >= W0;
+          const int32_t tr = now ? tau : W0;
+          const bool stop = k < lim && (capped || nx > tau) && (now || nx > W0);
+          const unsigned bal = __ballot_sync(0xffffffffu, stop);
+          const unsigned fb = __ballot_sync(0xffffffffu, tr > t0);
+          if (bal == 0) goto long_queue;  // no stop among the first 32 states (Bmax > 32)
+          const int sl = __ffs(bal) - 1;
+          const int32_t c = __shfl_sync(0xffffffffu, tr + T0, sl);  // Fn - a_h
+          Fn = ah + c;
+          b = sl + 1;
+          const bool isfree = fr < 0 || ((fb >> sl) & 1u);  // dispatched after the device freed (t > F)
+          const int64_t j2 = h + b;
+          bool conv = false;
+          if (isfree && j2 < en && checks > 0) {
+            checks--;
+            PX_DBG(dbg_chk++);
+            if (test && b < 32) {
+              const unsigned eb = __ballot_sync(0xffffffffu, (uint64_t)sp + du == (uint64_t)(uint32_t)c);
+              conv = ((eb >> (b - 1)) & 1u) && !((eb >> b) & 1u);
             } else {
-              Wk = k + 1 < p.Bmax ? (int32_t)p.L - T[k + 1] : 0;
-              Tk = k < p.Bmax ? T[k] : 0;
-            }
-            bool stop = false, fre = false;
-            int32_t cand = 0;
-            if (k < lim) {
-              const uint32_t du = (uint32_t)AR(h + k) - uah;
-              const int32_t dk = du < (uint32_t)LEAN_C ? (int32_t)du : LEAN_C;
-              const int32_t tau = dk > t0 ? dk : t0;
-              const bool capped = k + 1 == p.Bmax;
-              int32_t nx = LEAN_C;
-              if (k + 1 < lim) {
-                const uint32_t dn = (uint32_t)AR(h + k + 1) - uah;
-                nx = dn < (uint32_t)LEAN_C ? (int32_t)dn : LEAN_C;
-              }
-              const bool now = capped || tau >= Wk;
-              stop = (capped || nx > tau) && (now || nx > Wk);
-              const int32_t tr = now ? tau : Wk;
-              fre = tr > t0;
-              cand = tr + Tk;
-            }
-            const unsigned bal = __ballot_sync(0xffffffffu, stop);
-            const unsigned fb = __ballot_sync(0xffffffffu, fre);
-            if (bal) {
-              const int sl = __ffs(bal) - 1;
-              Fn = ah + __shfl_sync(0xffffffffu, cand, sl);
-              b = kb + sl + 1;
-              isfree = fr < 0 || ((fb >> sl) & 1u);
-              break;
+              spec_cache();
+              spec_ready = true;
+              conv = spec_F(j2 - 1) == Fn && spec_F(j2) != Fn;
             }
           }
+          // latency of query h + k (< 2^31); after the test: a phase run's cache reads out[] at its first fill
+          if (k < b && h + k < en) out[h + k] = (uint32_t)(c - dk);
+          PX_DBG(__syncwarp(); dbg_sec[0] += clock64() - dbg_tk; dbg_tk = clock64());
+          h = j2;
+          F = Fn;
+          lastfull = b == p.Bmax;
+          if (conv) {
+            // the rest of the chunk is the speculative run's (phase runs: their own latencies up to mr)
+            for (int64_t jj = h + lane; jj < mr; jj += 32) out[jj] = specL[jj - spec_base];
+            h = en + xov;
+            F = xF;
+            break;
+          }
+          continue;
+        }
+      long_queue:
+        bool isfree;
+        if (lean && fr < LEAN_C) {
+          const int32_t t0 = fr > 0 ? (int32_t)fr : 0;
+          const int64_t rem = n - h;
+          const int lim = rem < p.Bmax ? (int)rem : p.Bmax;
+          const uint32_t uah = (uint32_t)ah;
+          auto state = [&](int k, int32_t Wk, int32_t Tk, int32_t &cand, bool &fre) -> bool {
+            if (k >= lim) return false;
+            const uint32_t du = (uint32_t)AR(h + k) - uah;
+            const int32_t dk = du < (uint32_t)LEAN_C ? (int32_t)du : LEAN_C;
+            const int32_t tau = dk > t0 ? dk : t0;
+            const bool capped = k + 1 == p.Bmax;
+            const uint32_t dn = (uint32_t)AR(h + k + 1) - uah;
+            const int32_t nx = k + 1 < lim ? (dn < (uint32_t)LEAN_C ? (int32_t)dn : LEAN_C) : LEAN_C;
+            const bool now = capped || tau >= Wk;
+            const int32_t tr = now ? tau : Wk;
+            fre = tr > t0;
+            cand = tr + Tk;
+            return (capped || nx > tau) && (now || nx > Wk);
+          };
+          int32_t cand = 0;
+          bool fre = false;
+          unsigned bal = __ballot_sync(0xffffffffu, state(lane, W0, T0, cand, fre));
+          unsigned fb = __ballot_sync(0xffffffffu, fre);
+          int kb = 0;
+          while (!bal) {  // queues longer than 32 (Bmax > 32)
+            kb += 32;
+            const int k = kb + lane;
+            const int32_t Wk = kb == 32 ? W1 : (k + 1 < p.Bmax ? (int32_t)p.L - T[k + 1] : 0);
+            const int32_t Tk = kb == 32 ? T1 : (k < p.Bmax ? T[k] : 0);
+            bal = __ballot_sync(0xffffffffu, state(k, Wk, Tk, cand, fre));
+            fb = __ballot_sync(0xffffffffu, fre);
+          }
+          const int sl = __ffs(bal) - 1;
+          Fn = ah + __shfl_sync(0xffffffffu, cand, sl);
+          b = kb + sl + 1;
+          isfree = fr < 0 || ((fb >> sl) & 1u);  // dispatched after the device freed (t > F)
         } else {
           const int64_t t0 = F > ah ? F : ah;
           int64_t t;
@@ -862,23 +921,26 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
           Fn = t + T[b - 1];
           isfree = t > F;
         }
+        PX_DBG(__syncwarp(); dbg_sec[0] += clock64() - dbg_tk; dbg_tk = clock64());
         const int64_t j2 = h + b;
         bool conv = false;
         if (isfree && j2 < en && checks > 0) {
           checks--;
-          dbg_chk++;
+          PX_DBG(dbg_chk++);
           spec_cache();
+          spec_ready = true;
           conv = spec_F(j2 - 1) == Fn && spec_F(j2) != Fn;
         }
-        __syncwarp();
+        PX_DBG(__syncwarp(); dbg_sec[1] += clock64() - dbg_tk; dbg_tk = clock64());
         const int64_t hi = j2 < en ? j2 : en;
         for (int64_t jj = h + lane; jj < hi; jj += 32) out[jj] = sat_lat(Fn - AR(jj));
+        PX_DBG(__syncwarp(); dbg_sec[2] += clock64() - dbg_tk; dbg_tk = clock64());
         h = j2;
         F = Fn;
         lastfull = b == p.Bmax;
         if (conv) {
-          // the rest of the chunk is the phase run's (run 0's from mr on)
-          for (int64_t jj = j2 + lane; jj < mr; jj += 32) out[jj] = specL[jj - spec_base];
+          // the rest of the chunk is the speculative run's (phase runs: their own latencies up to mr)
+          for (int64_t jj = h + lane; jj < mr; jj += 32) out[jj] = specL[jj - spec_base];
           h = en + xov;
           F = xF;
           break;
@@ -888,8 +950,10 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   }
   if (a.debug && lane == 0) {
     const long long cyc = clock64() - dbg_t0;
-    if (cyc > a.debug) printf("stitch s=%d d=%d n=%lld Bmax=%d L=%lld nch=%lld cycles=%lld dec=%lld jump=%lld match=%lld chk=%lld\n", s, d,
-                              (long long)n, p.Bmax, (long long)p.L, (long long)nch, cyc, dbg_dec, dbg_jump, dbg_match, dbg_chk);
+    if (cyc > a.debug) printf("stitch s=%d d=%d n=%lld Bmax=%d L=%lld nch=%lld cycles=%lld dec=%lld jump=%lld match=%lld chk=%lld "
+                              "sdec=%lld schk=%lld swr=%lld sloop=%lld sring=%lld\n", s, d,
+                              (long long)n, p.Bmax, (long long)p.L, (long long)nch, cyc, dbg_dec, dbg_jump, dbg_match, dbg_chk,
+                              dbg_sec[0], dbg_sec[1], dbg_sec[2], dbg_sec[3], dbg_sec[4]);
   }
 }
 

@@ -14,9 +14,9 @@ sc = cfg["scenarios"]
 lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
 px.set_timing(True)
 KEYS = ("PROTEUS_REPLAY_SIMPLE", "PROTEUS_REPLAY_CHUNK", "PROTEUS_REPLAY_CHECKS", "PROTEUS_REPLAY_PHASES", "PROTEUS_REPLAY_DEBUG")
-variants = [{}, {"PROTEUS_REPLAY_PHASES": "1"}, {"PROTEUS_REPLAY_PHASES": "4"}, {"PROTEUS_REPLAY_PHASES": "16"}]
+variants = [{}, {"PROTEUS_REPLAY_PHASES": "4"}]
 variants += [{"PROTEUS_REPLAY_CHUNK": str(c)} for c in (256, 512)]
-variants += [{"PROTEUS_REPLAY_CHUNK": str(c), "PROTEUS_REPLAY_PHASES": "1"} for c in (256, 512)]
+
 variants += [eval(v) for v in sys.argv[1:]]
 ref = None
 for env in variants:
