@@ -524,7 +524,9 @@ __device__ __forceinline__ int decide_par(const Arr &A, int64_t n, int64_t h, in
   }
 }
 
-__host__ __device__ __forceinline__ size_t stitch_wstride(int bmax) { return ((size_t)RING + 2 * SPB + 12 + bmax + 3) & ~(size_t)3; }
+__host__ __device__ __forceinline__ size_t stitch_wstride(int bmax) {
+  return ((size_t)RING + 2 * SPB + 12 + 64 * SUMAX + bmax + 3) & ~(size_t)3;
+}
 static size_t stitch_smem(int bmax) { return 4 * stitch_wstride(bmax) * 4; }
 
 __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs a) {
@@ -543,7 +545,8 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   uint32_t *ring = wsm;
   uint32_t *specbuf = wsm + RING;
   uint64_t *bars = (uint64_t *)(wsm + RING + 2 * SPB);  // [0..3] ring slots, [4..5] spec buffers
-  int32_t *T = (int32_t *)(wsm + RING + 2 * SPB + 12);
+  int64_t *FeS = (int64_t *)(wsm + RING + 2 * SPB + 12);  // [32 SUMAX] stretch batch finishes
+  int32_t *T = (int32_t *)(wsm + RING + 2 * SPB + 12 + 64 * SUMAX);
   const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
   for (int k = lane; k < a.bmax; k += 32) T[k] = Tg[k];
   if (lane < 6) mbar_init(bars + lane);
@@ -625,6 +628,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   const uint32_t *vl = R > 1 ? a.vlat + a.voff[lane_id] : nullptr;
   const SpecExit *vx = R > 1 ? a.vex + a.voff[(int64_t)a.S * a.D + lane_id] : nullptr;
   const int SU = p.Bmax >= 16 ? 1 : p.Bmax >= 8 ? 2 : SUMAX;  // batches per lane in a full-batch stretch
+  const uint32_t bmagic = (uint32_t)((1ull << 32) / (uint64_t)p.Bmax + 1);  // q / Bmax = umulhi(q, bmagic), q < 2^16
   // SW: a full batch needs its last arrival <= max(F_i, a[h_i] + SW) (see the stretch)
   int32_t tbig = 0;
   for (int k = lane; k + 1 < p.Bmax; k += 32) tbig = T[k] > tbig ? T[k] : tbig;
@@ -701,8 +705,13 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         if (h >= h_safe) need(h, h + p.Bmax + 1);
         const int64_t ah = AR(h);
         PX_DBG(__syncwarp(); dbg_sec[4] += clock64() - dbg_tk; dbg_tk = clock64());
-        if ((lastfull || F > ah) && h + p.Bmax - 1 < n &&
-            AR(h + p.Bmax - 1) <= (F > ah + SW ? F : ah + SW)) {
+        bool stretch = false;
+        if ((lastfull || F > ah) && h + 2 * p.Bmax - 1 < n) {  // are the next two batches full?
+          const int64_t A0 = AR(h + p.Bmax - 1), A1 = AR(h + 2 * p.Bmax - 1), a1 = AR(h + p.Bmax);
+          const int64_t F1 = (F > A0 ? F : A0) + TB;
+          stretch = A0 <= (F > ah + SW ? F : ah + SW) && A1 <= (F1 > a1 + SW ? F1 : a1 + SW);
+        }
+        if (stretch) {
           // full-batch stretch: while every batch is full (Bmax queries), batch i
           // dispatches when the device is free and its last query has arrived,
           // F_{i+1} = max(F_i, A_i) + T(Bmax), A_i = a[h_i + Bmax - 1], so
@@ -713,9 +722,13 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
           // T(Bmax) is the largest of T(1..Bmax) (else SW = -inf: A_i <= F_i,
           // the queue already holds Bmax queries).  Rounds of 32 SU batches,
           // lane l taking [l SU, l SU + SU) of the round.
-          int64_t kmax = (en - h + p.Bmax - 1) / p.Bmax;  // batches starting in this chunk
-          const int64_t room = ((((off + h) >> 10) + 3) * RSEG - (off + h)) / p.Bmax;
-          const int64_t avail = (n - h) / p.Bmax;
+          auto divB = [&](int64_t x) -> int64_t {  // x / Bmax for 0 <= x (capped at 2^15)
+            const uint32_t u = (uint32_t)(x < 32768 ? x : 32768);
+            return p.Bmax == 1 ? u : __umulhi(u, bmagic);
+          };
+          int64_t kmax = divB(en - h + p.Bmax - 1);  // batches starting in this chunk
+          const int64_t room = divB((((off + h) >> 10) + 3) * RSEG - (off + h));
+          const int64_t avail = divB(n - h);
           if (kmax > room) kmax = room;
           if (kmax > avail) kmax = avail;
           need(h, h + kmax * p.Bmax);
@@ -760,18 +773,23 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
             const unsigned bal = __ballot_sync(0xffffffffu, fl < SU);
             const int fs = bal ? __ffs(bal) - 1 : 31;
             const int64_t r = bal ? (int64_t)fs * SU + __shfl_sync(0xffffffffu, fl, fs) : 32 * SU;
-            // latencies of the accepted batches; lane l writes its own
+            // latencies of the accepted batches: finishes through shared
+            // memory, then the round's queries in coalesced lane strides
             M = Mc > exc ? Mc : exc;
 #pragma unroll
             for (int u = 0; u < SUMAX; u++) {
               const int64_t i = ib + u;
               if (u < SU && i < done + r) {
                 M = G[u] > M ? G[u] : M;
-                const int64_t Fe = (i + 1) * TB + M;
-                const int64_t hi = h + i * p.Bmax;
-                for (int q = 0; q < p.Bmax; q++) out[hi + q] = sat_lat(Fe - AR(hi + q));
+                FeS[lane * SU + u] = (i + 1) * TB + M;
               }
             }
+            __syncwarp();
+            const int64_t hb = h + done * p.Bmax;
+            const uint32_t np = (uint32_t)(r * p.Bmax);
+            for (uint32_t q = lane; q < np; q += 32)
+              out[hb + q] = sat_lat(FeS[p.Bmax == 1 ? q : __umulhi(q, bmagic)] - AR(hb + q));
+            __syncwarp();
             if (r > 0) {
               Mc = __shfl_sync(0xffffffffu, M, (int)((r - 1) / SU));
               done += r;
@@ -807,42 +825,69 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
           const int64_t rem = n - h;
           const int lim = rem < p.Bmax ? (int)rem : p.Bmax;
           const uint32_t uah = (uint32_t)ah;
-          const int k = lane;
-          const uint32_t du = (uint32_t)AR(h + k) - uah;
-          const uint32_t dn = (uint32_t)AR(h + k + 1) - uah;
           const bool test = spec_ready && checks > 0;
-          const uint32_t sp = test && h + k < en ? specL[(int32_t)(h + k - spec_base)] : 0u;
-          const int32_t dk = du < (uint32_t)LEAN_C ? (int32_t)du : LEAN_C;
-          const int32_t tau = dk > t0 ? dk : t0;
-          const bool capped = k + 1 == p.Bmax;
-          const int32_t nx = k + 1 < lim ? (dn < (uint32_t)LEAN_C ? (int32_t)dn : LEAN_C) : LEAN_C;
-          const bool now = capped || tau >= W0;
-          const int32_t tr = now ? tau : W0;
-          const bool stop = k < lim && (capped || nx > tau) && (now || nx > W0);
-          const unsigned bal = __ballot_sync(0xffffffffu, stop);
-          const unsigned fb = __ballot_sync(0xffffffffu, tr > t0);
-          if (bal == 0) goto long_queue;  // no stop among the first 32 states (Bmax > 32)
-          const int sl = __ffs(bal) - 1;
-          const int32_t c = __shfl_sync(0xffffffffu, tr + T0, sl);  // Fn - a_h
+          // lane holds states k = lane and (Bmax > 32) k = lane + 32
+          struct St {
+            uint32_t du, sp;
+            int32_t dk, cand;
+            bool stop, fre;
+          };
+          auto st = [&](int k, int32_t Wk, int32_t Tk) {
+            St r;
+            r.du = (uint32_t)AR(h + k) - uah;
+            const uint32_t dn = (uint32_t)AR(h + k + 1) - uah;
+            r.sp = test && h + k < en ? specL[(int32_t)(h + k - spec_base)] : 0u;
+            r.dk = r.du < (uint32_t)LEAN_C ? (int32_t)r.du : LEAN_C;
+            const int32_t tau = r.dk > t0 ? r.dk : t0;
+            const bool capped = k + 1 == p.Bmax;
+            const int32_t nx = k + 1 < lim ? (dn < (uint32_t)LEAN_C ? (int32_t)dn : LEAN_C) : LEAN_C;
+            const bool now = capped || tau >= Wk;
+            const int32_t tr = now ? tau : Wk;
+            r.stop = k < lim && (capped || nx > tau) && (now || nx > Wk);
+            r.fre = tr > t0;
+            r.cand = tr + Tk;
+            return r;
+          };
+          const St s0 = st(lane, W0, T0);
+          const unsigned bal0 = __ballot_sync(0xffffffffu, s0.stop);
+          const unsigned fb0 = __ballot_sync(0xffffffffu, s0.fre);
+          int32_t c;
+          unsigned fbs, bals;
+          St s1{};
+          if (bal0) {
+            bals = bal0;
+            fbs = fb0;
+            b = 0;
+          } else {  // no stop among the first 32 states (Bmax > 32)
+            if (p.Bmax > 64) goto long_queue;
+            s1 = st(lane + 32, W1, T1);
+            bals = __ballot_sync(0xffffffffu, s1.stop);
+            fbs = __ballot_sync(0xffffffffu, s1.fre);
+            b = 32;
+          }
+          const int sl = __ffs(bals) - 1;
+          c = __shfl_sync(0xffffffffu, b ? s1.cand : s0.cand, sl);  // Fn - a_h
           Fn = ah + c;
-          b = sl + 1;
-          const bool isfree = fr < 0 || ((fb >> sl) & 1u);  // dispatched after the device freed (t > F)
+          b += sl + 1;
+          const bool isfree = fr < 0 || ((fbs >> sl) & 1u);  // dispatched after the device freed (t > F)
           const int64_t j2 = h + b;
           bool conv = false;
           if (isfree && j2 < en && checks > 0) {
             checks--;
             PX_DBG(dbg_chk++);
             if (test && b < 32) {
-              const unsigned eb = __ballot_sync(0xffffffffu, (uint64_t)sp + du == (uint64_t)(uint32_t)c);
-              conv = ((eb >> (b - 1)) & 1u) && !((eb >> b) & 1u);
+              // bit k: the speculative batch holding h + k finishes at Fn
+              const unsigned e = __ballot_sync(0xffffffffu, (uint64_t)s0.sp + s0.du == (uint64_t)(uint32_t)c);
+              conv = ((e >> (b - 1)) & 1u) && !((e >> b) & 1u);
             } else {
               spec_cache();
               spec_ready = true;
               conv = spec_F(j2 - 1) == Fn && spec_F(j2) != Fn;
             }
           }
-          // latency of query h + k (< 2^31); after the test: a phase run's cache reads out[] at its first fill
-          if (k < b && h + k < en) out[h + k] = (uint32_t)(c - dk);
+          // latencies of queries h + k (< 2^31); after the test: a phase run's cache reads out[] at its first fill
+          if (lane < b && h + lane < en) out[h + lane] = (uint32_t)(c - s0.dk);
+          if (lane + 32 < b && h + lane + 32 < en) out[h + lane + 32] = (uint32_t)(c - s1.dk);
           PX_DBG(__syncwarp(); dbg_sec[0] += clock64() - dbg_tk; dbg_tk = clock64());
           h = j2;
           F = Fn;
