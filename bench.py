@@ -328,19 +328,43 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     t_slo = torch.as_tensor(cl.slo_us, dtype=torch.int32, device=dev)
     t_dem = torch.as_tensor(cfg["demand"][lo:hi], dtype=torch.int32, device=dev)
     t_one = torch.as_tensor(cfg["demand"][:1], dtype=torch.int32, device=dev)
+    nv, D = hi - lo, len(cl.device_type)
+    dout = {"score": torch.empty(nv, dtype=torch.uint64, device=dev),
+            "served": torch.empty(nv, dtype=torch.int64, device=dev),
+            "unmet": torch.empty(nv, dtype=torch.int64, device=dev),
+            "accsum": torch.empty(nv, dtype=torch.int64, device=dev),
+            "option": torch.empty((nv, D), dtype=torch.int32, device=dev),
+            "z_qps": torch.empty((nv, D), dtype=torch.int32, device=dev)}
     for _ in range(2):
-        px.solve(t_dev, t_slo, t_dem, mode=2)
-    ts = []
-    for _ in range(3):
+        px.solve_batch(t_dev, t_slo, t_dem, mode=2, out=dout)
+    ts, kts = [], []
+    px.set_timing(True)
+    for _ in range(5):
         flush.zero_()
         barrier()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
-        sols = px.solve(t_dev, t_slo, t_dem, mode=2)
+        _, ncand = px.solve_batch(t_dev, t_slo, t_dem, mode=2, out=dout)
         b.record(stream)
         barrier()
         ts.append(a.elapsed_time(b))
+        kts.append(px.kernel_times())
+    px.set_timing(False)
     ms = max_over_ranks(statistics.median(ts))
+    ksplit = {}
+    for kt in kts:
+        for n_, v in kt:
+            ksplit.setdefault(n_, []).append(v)
+    ksplit = {k: statistics.median(v) for k, v in ksplit.items()}
+    # e2e: host demand in, host solutions out (the call a user makes)
+    e2e_t = []
+    for _ in range(3):
+        barrier()
+        t0 = time.perf_counter()
+        px.solve_batch(cl.device_type, cl.slo_us, cfg["demand"][lo:hi], mode=2)
+        barrier()
+        e2e_t.append(time.perf_counter() - t0)
+    e2e_ms = max_over_ranks(statistics.median(e2e_t)) * 1e3
     one = []
     for _ in range(5):
         barrier()
@@ -349,9 +373,11 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
         one.append((time.perf_counter() - t0) * 1e3)
     out["c4_resolve"] = {
         "vectors": len(cfg["demand"]), "ms_all_vectors": ms, "ms_per_vector_batched": ms / max(1, hi - lo),
+        "kernel_ms": ksplit,
+        "e2e_ms_host_buffers": e2e_ms,
         "single_vector_time_to_optimal_ms": statistics.median(one),
-        "subplacements_per_vector": sols[0].n_candidates if sols else 0,
-        "subplacements_per_s": (len(cfg["demand"]) * (sols[0].n_candidates if sols else 0)) / (ms / 1e3),
+        "subplacements_per_vector": ncand,
+        "subplacements_per_s": (len(cfg["demand"]) * ncand) / (ms / 1e3),
         "scaling": "weak (vectors split by rank)"}
     # c5: replay 10M queries x 64 scenarios (scenarios on every rank; N>1 = replicas)
     cfg = W.config("c5")

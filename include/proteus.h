@@ -167,6 +167,29 @@ typedef struct {
 
 int proteus_solve(proteus_ctx *ctx, const proteus_solve_args *args, proteus_solution *out /* [n_vec] */);
 
+/* Batched form of proteus_solve for many demand vectors (the per-second
+ * re-solve): the same search, outputs as arrays.
+ * Every pointer may be NULL (not produced), host memory or device memory,
+ * independently; device outputs are written by a kernel on the context's
+ * stream without a host round trip of the solutions.
+ *   score, index            [n_vec] as proteus_solution
+ *   served, unmet, accsum   [n_vec]
+ *   eff_acc_micro           [n_vec]
+ *   option, z_qps           [n_vec][D] row-major
+ * n_candidates (out) is the per-vector count of proteus_solve.  Host outputs
+ * are written only on success; device outputs are written before the final
+ * internal check, so a PROTEUS_EINTERNAL return may leave them written. */
+typedef struct {
+  uint64_t *score, *index;
+  int64_t *served, *unmet, *accsum;
+  int32_t *eff_acc_micro;
+  int32_t *option;
+  int32_t *z_qps;
+  uint64_t n_candidates;  /* out: count vectors / placements scored per vector */
+} proteus_batch;
+
+int proteus_solve_batch(proteus_ctx *ctx, const proteus_solve_args *args, proteus_batch *out);
+
 /* Modes 0/1: the full solution (placement, z, value) of canonical index
  * `index` for demand vector `vec` -- used after combining shard results. */
 int proteus_materialize(proteus_ctx *ctx, const proteus_solve_args *args, int32_t vec, uint64_t index,

@@ -139,6 +139,25 @@ class Proteus:
         self._check(self._lib.proteus_solve(self._h, C.byref(a), sols))
         return [self._sol(sols[i], opts[i], zs[i]) for i in range(n_vec)]
 
+    def solve_batch(self, device_type, slo_us, demand, mode=MODE_FACTORED, out=None, fields=None):
+        """Many demand vectors at once (proteus_solve_batch).  out: dict of
+        preallocated arrays (numpy or CUDA torch) keyed by field name, written
+        in place; else host numpy arrays are returned for `fields` (default
+        all).  Returns (dict of arrays, n_candidates per vector)."""
+        keep = []
+        a, n_vec, D = self._solve_args(device_type, slo_us, demand, mode, 0, 1, 0, False, keep)
+        shapes = {"score": ((n_vec,), np.uint64), "index": ((n_vec,), np.uint64), "served": ((n_vec,), np.int64),
+                  "unmet": ((n_vec,), np.int64), "accsum": ((n_vec,), np.int64),
+                  "eff_acc_micro": ((n_vec,), np.int32), "option": ((n_vec, D), np.int32),
+                  "z_qps": ((n_vec, D), np.int32)}
+        if out is None:
+            out = {k: np.empty(*shapes[k]) for k in (fields or shapes)}
+        b = N.proteus_batch()
+        for k, x in out.items():
+            setattr(b, k, _arg(x, shapes[k][1], keep))
+        self._check(self._lib.proteus_solve_batch(self._h, C.byref(a), C.byref(b)))
+        return out, int(b.n_candidates)
+
     def materialize(self, device_type, slo_us, demand, index, vec=0, mode=MODE_FLAT):
         keep = []
         a, n_vec, D = self._solve_args(device_type, slo_us, demand, mode, 0, 1, 0, False, keep)

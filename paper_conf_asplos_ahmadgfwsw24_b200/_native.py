@@ -20,7 +20,7 @@ PROTEUS_SOLVE_GENERIC = 1
 
 EXPORTED = (
     "proteus_abi_version", "proteus_create", "proteus_destroy", "proteus_set_stream", "proteus_last_error",
-    "proteus_load_profiles", "proteus_solve", "proteus_materialize", "proteus_candidate_count",
+    "proteus_load_profiles", "proteus_solve", "proteus_solve_batch", "proteus_materialize", "proteus_candidate_count",
     "proteus_replay", "proteus_set_timing", "proteus_kernel_times", "proteus_launch_count",
 )
 
@@ -40,6 +40,12 @@ class proteus_solution(C.Structure):
     _fields_ = [("score", C.c_uint64), ("index", C.c_uint64), ("served", C.c_int64), ("unmet", C.c_int64),
                 ("accsum", C.c_int64), ("eff_acc_micro", C.c_int32), ("reserved", C.c_int32),
                 ("n_candidates", C.c_uint64), ("option", C.c_void_p), ("z_qps", C.c_void_p)]
+
+
+class proteus_batch(C.Structure):
+    _fields_ = [("score", C.c_void_p), ("index", C.c_void_p), ("served", C.c_void_p), ("unmet", C.c_void_p),
+                ("accsum", C.c_void_p), ("eff_acc_micro", C.c_void_p), ("option", C.c_void_p),
+                ("z_qps", C.c_void_p), ("n_candidates", C.c_uint64)]
 
 
 class proteus_scenario(C.Structure):
@@ -74,6 +80,7 @@ def load(path: str = LIB_PATH):
     L.proteus_last_error.restype = C.c_char_p
     L.proteus_load_profiles.argtypes = [vp, C.POINTER(proteus_profiles)]
     L.proteus_solve.argtypes = [vp, C.POINTER(proteus_solve_args), C.POINTER(proteus_solution)]
+    L.proteus_solve_batch.argtypes = [vp, C.POINTER(proteus_solve_args), C.POINTER(proteus_batch)]
     L.proteus_materialize.argtypes = [vp, C.POINTER(proteus_solve_args), i32, u64, C.POINTER(proteus_solution)]
     L.proteus_candidate_count.argtypes = [vp, C.POINTER(proteus_solve_args), C.POINTER(u64)]
     L.proteus_replay.argtypes = [vp, vp, vp, i64, vp, vp, vp, i32, vp, vp, C.POINTER(proteus_scenario), i32,

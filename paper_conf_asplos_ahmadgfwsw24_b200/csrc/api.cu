@@ -4,6 +4,7 @@
 // runs in the kernels of prepare.cu, solve_enum.cu, solve_factored.cu and
 // replay.cu.
 #include <cstdarg>
+#include <cstddef>
 #include <cstring>
 
 #include "internal.cuh"
@@ -293,6 +294,79 @@ static int validate_solve(proteus_ctx *ctx, const proteus_solve_args *a, SolveIn
   return 0;
 }
 
+// Batched outputs (proteus_solve_batch): the solution records unpacked into
+// the caller's device arrays (layout only), and the OR of their status words.
+struct BatchPtrs {
+  uint64_t *score, *index;
+  int64_t *served, *unmet, *accsum;
+  int32_t *eff, *option, *z;
+};
+
+__global__ void k_sol_unpack(const SolRec *__restrict__ sol, int n, int D, BatchPtrs o, int32_t *status) {
+  const int i = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+  if (i >= n) return;
+  const SolRec &r = sol[i];
+  if (lane == 0) {
+    if (o.score) o.score[i] = r.score;
+    if (o.index) o.index[i] = r.index;
+    if (o.served) o.served[i] = r.served;
+    if (o.unmet) o.unmet[i] = r.unmet;
+    if (o.accsum) o.accsum[i] = r.accsum;
+    if (o.eff) o.eff[i] = r.eff;
+    if (r.status) atomicOr(status, 1 << (r.status & 15));
+  }
+  for (int d = lane; d < D; d += 32) {
+    if (o.option) o.option[(size_t)i * D + d] = r.option[d];
+    if (o.z) o.z[(size_t)i * D + d] = r.z[d];
+  }
+}
+
+static int batch_out(proteus_ctx *ctx, const proteus_solve_args *a, const SolRec *d_sol, int n, proteus_batch *o) {
+  void *ptrs[8] = {o->score, o->index, o->served, o->unmet, o->accsum, o->eff_acc_micro, o->option, o->z_qps};
+  bool dev[8], any_host = false;
+  for (int k = 0; k < 8; k++) {
+    dev[k] = px_is_device_ptr(ptrs[k]);
+    any_host |= ptrs[k] && !dev[k];
+  }
+  int32_t *d_status = (int32_t *)px_buf(ctx, B_IN3, 16);
+  if (!d_status) return px_fail(ctx, PROTEUS_ENOMEM, "status word");
+  PX_CUDA(ctx, cudaMemsetAsync(d_status, 0, 4, ctx->stream));
+  BatchPtrs bp = {(uint64_t *)(dev[0] ? ptrs[0] : nullptr), (uint64_t *)(dev[1] ? ptrs[1] : nullptr),
+                  (int64_t *)(dev[2] ? ptrs[2] : nullptr),  (int64_t *)(dev[3] ? ptrs[3] : nullptr),
+                  (int64_t *)(dev[4] ? ptrs[4] : nullptr),  (int32_t *)(dev[5] ? ptrs[5] : nullptr),
+                  (int32_t *)(dev[6] ? ptrs[6] : nullptr),  (int32_t *)(dev[7] ? ptrs[7] : nullptr)};
+  PX_LAUNCH(ctx, "sol_unpack", k_sol_unpack, (n + 7) / 8, 256, 0, d_sol, n, a->D, bp, d_status);
+  int32_t status = 0;
+  std::vector<SolRec> h;
+  if (any_host) {
+    h.resize(n);
+    PX_CUDA(ctx, cudaMemcpyAsync(h.data(), d_sol, sizeof(SolRec) * n, cudaMemcpyDeviceToHost, ctx->stream));
+  }
+  uint64_t n_cand = 0;
+  PX_CUDA(ctx, cudaMemcpyAsync(&status, d_status, 4, cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(&n_cand, (const char *)d_sol + offsetof(SolRec, n_candidates), 8,
+                               cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  int rc = timing_collect(ctx);
+  if (rc) return rc;
+  if (status) return px_fail(ctx, PROTEUS_EINTERNAL, "internal check failed (status bits 0x%x)", status);
+  o->n_candidates = n_cand;
+  if (!any_host) return PROTEUS_OK;
+  const int D = a->D;
+  for (int i = 0; i < n; i++) {
+    const SolRec &r = h[i];
+    if (o->score && !dev[0]) o->score[i] = r.score;
+    if (o->index && !dev[1]) o->index[i] = r.index;
+    if (o->served && !dev[2]) o->served[i] = r.served;
+    if (o->unmet && !dev[3]) o->unmet[i] = r.unmet;
+    if (o->accsum && !dev[4]) o->accsum[i] = r.accsum;
+    if (o->eff_acc_micro && !dev[5]) o->eff_acc_micro[i] = r.eff;
+    if (o->option && !dev[6]) memcpy(o->option + (size_t)i * D, r.option, D * 4);
+    if (o->z_qps && !dev[7]) memcpy(o->z_qps + (size_t)i * D, r.z, D * 4);
+  }
+  return PROTEUS_OK;
+}
+
 // families supplied in accuracy order (non-increasing within each family)?
 static bool families_sorted(const proteus_ctx *ctx) {
   for (int q = 0; q < ctx->Q; q++)
@@ -304,11 +378,11 @@ static bool families_sorted(const proteus_ctx *ctx) {
 int px_flat_template_vm(int Q, int maxV);  // solve_enum.cu: VM of the specialised kernel, 0 if none
 
 static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_solution *out, bool mat_only,
-                        int32_t mat_vec, uint64_t mat_index) {
+                        int32_t mat_vec, uint64_t mat_index, proteus_batch *bout = nullptr) {
   SolveInputs in;
   int rc = validate_solve(ctx, a, in);
   if (rc) return rc;
-  if (!out) return px_fail(ctx, PROTEUS_EINVAL, "null out");
+  if (!out && !bout) return px_fail(ctx, PROTEUS_EINVAL, "null out");
   if (mat_only && (a->mode == 2 || mat_vec < 0 || mat_vec >= a->n_vec))
     return px_fail(ctx, PROTEUS_EINVAL, "materialize: mode %d vec %d", a->mode, mat_vec);
   timing_reset(ctx);
@@ -368,6 +442,7 @@ static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_s
                        d_sol, 0, a->n_vec, false, 0, use_flat);
   }
   if (rc) return rc;
+  if (bout) return batch_out(ctx, a, d_sol, nout, bout);
   std::vector<SolRec> h(nout);
   PX_CUDA(ctx, cudaMemcpyAsync(h.data(), d_sol, sizeof(SolRec) * nout, cudaMemcpyDeviceToHost, ctx->stream));
   PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
@@ -399,6 +474,11 @@ extern "C" {
 
 int proteus_solve(proteus_ctx *ctx, const proteus_solve_args *args, proteus_solution *out) {
   return solve_common(ctx, args, out, false, 0, 0);
+}
+
+int proteus_solve_batch(proteus_ctx *ctx, const proteus_solve_args *args, proteus_batch *out) {
+  if (!out) return px_fail(ctx, PROTEUS_EINVAL, "null out");
+  return solve_common(ctx, args, nullptr, false, 0, 0, out);
 }
 
 int proteus_materialize(proteus_ctx *ctx, const proteus_solve_args *args, int32_t vec, uint64_t index,

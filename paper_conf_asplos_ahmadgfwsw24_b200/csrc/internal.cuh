@@ -81,7 +81,7 @@ struct proteus_ctx {
   int T = 0, Q = 0, M = 0, bmax = 0;
   std::vector<int32_t> V, acc, lat, fam, off;
   int32_t *d_lat = nullptr, *d_acc = nullptr, *d_fam = nullptr, *d_off = nullptr, *d_V = nullptr;
-  DevBuf bufs[32];
+  DevBuf bufs[48];
   // instrumentation
   bool timing = false;
   uint64_t launches = 0;
@@ -94,11 +94,14 @@ struct proteus_ctx {
   bool tab_valid = false;
   std::vector<int32_t> tab_key, tab_P, tab_slot_code;
   Tables tab;
-  // cached DP key pairs of the factored search (solve_factored.cu)
-  void *dp_pairs = nullptr;
-  int64_t dp_pairs_n = 0;
-  int32_t dp_pairs_U = -1;
-  std::vector<int32_t> dp_pairs_key;
+  // cached DP budget orders of the factored search (solve_factored.cu)
+  void *dp_order = nullptr;
+  int32_t dp_order_U = -1;
+  std::vector<int32_t> dp_order_key;
+  int64_t dp_items_stride = 0;
+  void *gv_order = nullptr;  // cells of the batched g kernel by decreasing size
+  std::vector<int32_t> gv_order_key;
+  std::vector<int32_t> dp_items_n;
   // cached count-vector lists of the factored search
   void *fact_lists_buf = nullptr;
   std::vector<int32_t> fact_lists_key;
@@ -108,9 +111,9 @@ struct proteus_ctx {
 enum {
   B_TABLES = 0, B_BEST, B_SOL, B_IN0, B_IN1, B_IN2, B_IN3, B_FACT0, B_FACT1, B_FACT2, B_FACT3,
   B_R_PAT, B_R_TGT, B_R_HIST, B_R_BASE, B_R_DEVARR, B_R_DEVIDX, B_R_OFF, B_R_LAT, B_R_AGG, B_R_TGT1,
-  B_R_DEVARR1, B_R_DEVIDX1, B_R_OFF1, B_R_MISC, B_R_LANE, B_R_DBASE0, B_R_DBASE1, B_R_LATD, B_R_VLAT, B_R_VEX, B_R_VOFF, B_NBUF
+  B_R_DEVARR1, B_R_DEVIDX1, B_R_OFF1, B_R_MISC, B_R_LANE, B_R_DBASE0, B_R_DBASE1, B_R_LATD, B_R_VLAT, B_R_VEX, B_R_VOFF, B_FACT4, B_NBUF
 };
-static_assert(B_NBUF <= 32, "proteus_ctx::bufs is too small");
+static_assert(B_NBUF <= 48, "proteus_ctx::bufs is too small");
 
 // errors
 int px_fail(proteus_ctx *ctx, int code, const char *fmt, ...);

@@ -582,11 +582,12 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   // make queries [.., jend) of the device readable (jend <= the segment 3 past h's);
   // h_safe: below it a decision at h needs no ring work (issue or wait)
   int64_t h_safe = 0;
+  const int64_t look = p.Bmax <= 512 ? 2 * p.Bmax : p.Bmax;  // read-ahead of a decision (+ stretch test)
   auto need = [&](int64_t hcur, int64_t jend) {
     seg_issue(hcur);
     const int64_t gend = off + jend;
     while (sg_wait * RSEG < gend) seg_wait_one();
-    const int64_t s1 = (sg_iss - 2) * RSEG - off, s2 = sg_wait * RSEG - off - p.Bmax;
+    const int64_t s1 = (sg_iss - 2) * RSEG - off, s2 = sg_wait * RSEG - off - look;
     h_safe = s1 < s2 ? s1 : s2;
   };
   const uint32_t ro = (uint32_t)(off & (RING - 1));
@@ -702,11 +703,11 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
       bool spec_ready = false;  // latency cache of this chunk loaded (at its first meeting test)
       while (h < en) {
         PX_DBG(if (dbg_tk) dbg_sec[3] += clock64() - dbg_tk; dbg_tk = clock64());
-        if (h >= h_safe) need(h, h + p.Bmax + 1);
+        if (h >= h_safe) need(h, h + look + 1);  // decision + the stretch test's two batches
         const int64_t ah = AR(h);
         PX_DBG(__syncwarp(); dbg_sec[4] += clock64() - dbg_tk; dbg_tk = clock64());
         bool stretch = false;
-        if ((lastfull || F > ah) && h + 2 * p.Bmax - 1 < n) {  // are the next two batches full?
+        if ((lastfull || F > ah) && p.Bmax <= 512 && h + 2 * p.Bmax - 1 < n) {  // are the next two batches full?
           const int64_t A0 = AR(h + p.Bmax - 1), A1 = AR(h + 2 * p.Bmax - 1), a1 = AR(h + p.Bmax);
           const int64_t F1 = (F > A0 ? F : A0) + TB;
           stretch = A0 <= (F > ah + SW ? F : ah + SW) && A1 <= (F1 > a1 + SW ? F1 : a1 + SW);
@@ -834,8 +835,9 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
           };
           auto st = [&](int k, int32_t Wk, int32_t Tk) {
             St r;
-            r.du = (uint32_t)AR(h + k) - uah;
-            const uint32_t dn = (uint32_t)AR(h + k + 1) - uah;
+            // only queries the ring holds for this decision are read (k <= lim: the meeting test's lane b)
+            r.du = k <= lim && h + k < n ? (uint32_t)AR(h + k) - uah : 0u;
+            const uint32_t dn = k + 1 < lim ? (uint32_t)AR(h + k + 1) - uah : 0u;
             r.sp = test && h + k < en ? specL[(int32_t)(h + k - spec_base)] : 0u;
             r.dk = r.du < (uint32_t)LEAN_C ? (int32_t)r.du : LEAN_C;
             const int32_t tau = r.dk > t0 ? r.dk : t0;
@@ -914,7 +916,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
             const int32_t dk = du < (uint32_t)LEAN_C ? (int32_t)du : LEAN_C;
             const int32_t tau = dk > t0 ? dk : t0;
             const bool capped = k + 1 == p.Bmax;
-            const uint32_t dn = (uint32_t)AR(h + k + 1) - uah;
+            const uint32_t dn = k + 1 < lim ? (uint32_t)AR(h + k + 1) - uah : 0u;
             const int32_t nx = k + 1 < lim ? (dn < (uint32_t)LEAN_C ? (int32_t)dn : LEAN_C) : LEAN_C;
             const bool now = capped || tau >= Wk;
             const int32_t tr = now ? tau : Wk;

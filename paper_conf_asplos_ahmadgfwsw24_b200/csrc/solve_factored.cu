@@ -41,8 +41,11 @@ struct FactLayout {
   int32_t *ecap;       // [entries][VM] capacity vector in fill (slot) order
   uint8_t *ecnt;       // [entries][16] counts in caller's variant order
   int32_t *esum;       // [entries]
-  const int2 *pairs;   // DP: for each budget b, the keys (u, b - u) of every u <= b
-  const int32_t *pstart;  // [U + 1] offsets into pairs
+  uint32_t fmask[PX_MAXQ];  // bit t: family q has a variant with P > 0 on type t (else u_t = 0)
+  int32_t morder[PX_MAXQ];  // family q's DP work list: row of items
+  int32_t nitems[PX_MAXQ];  // its length
+  int64_t istride;          // row stride of items
+  const int2 *items;        // [rows][istride] DP work items (lattice indexing only, see k_fact_dp)
 };
 
 // ------------------------------------------------------------- lists ----
@@ -172,86 +175,143 @@ __global__ void __launch_bounds__(FG_WARPS * 32) k_fact_g(const __grid_constant_
 
 // Batched variant for many demand vectors: the count vectors of a (family,
 // usage) cell and their capacity vectors do not depend on the demand, only
-// the water-fill does.  One warp per (family, usage, 32 vectors): the warp
-// materialises the cell's candidates 64 at a time in shared memory (capacity
-// vector in fill order + lexicographic rank; lanes decode 2 each, type T-1
-// fastest so ranks ascend), then every lane water-fills each of them for its
-// own vector (broadcast loads) and keeps its first maximum.
+// the water-fill does.  One warp per (family, usage, 64 vectors), two vectors
+// per lane.  The warp materialises the cell's candidates GV_TILE at a time in
+// shared memory as cumulative capacities C_j = cap_0 + ... + cap_{j-1} in
+// fill order (lanes decode 2 each, type T-1 fastest so ranks ascend), then
+// every lane water-fills each of them for its own vectors.  The fill is
+// written in summation-by-parts form: with m_j = min(s, C_j) the fill takes
+// m_{j+1} - m_j from slot j, so
+//   served = m_VM,   accsum = sum_{j=1..VM} m_j (A_{j-1} - A_j)   (A_VM = 0)
+// -- the same integers as the sequential fill (take = min(rem, cap)), two
+// instructions per slot and no serial dependence between slots.  Each lane
+// keeps the first maximum in candidate order (= lowest lexicographic rank)
+// as a candidate ordinal and decodes its rank once at the end.
 #define GV_TILE 64
+__device__ __forceinline__ uint64_t madw(uint32_t a, uint32_t b, uint64_t c) {
+  uint64_t r;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(a), "r"(b), "l"(c));
+  return r;
+}
+
 template <int VMT>
 __global__ void __launch_bounds__(128) k_fact_gv(const __grid_constant__ FactLayout f, int n_vec,
                                                  const int32_t *__restrict__ demand,
-                                                 const int32_t *__restrict__ slot_acc, BestRec *g) {
-  __shared__ int32_t tcap[4][GV_TILE][VMT];
-  __shared__ uint64_t tsub[4][GV_TILE];
+                                                 const int32_t *__restrict__ slot_acc,
+                                                 const int32_t *__restrict__ cell_order, BestRec *g) {
+  constexpr int CS = (VMT + 3) & ~3;  // cumulative-capacity row stride (int4 loads)
+  __shared__ __align__(16) int32_t tc[4][GV_TILE][CS];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int item = blockIdx.x * 4 + w;
   if (item >= f.Q * f.U) return;
-  const int q = item / f.U, ukey = item % f.U;
-  const int vec = blockIdx.y * 32 + lane;
-  const bool active = vec < n_vec;
-  const int s = active ? demand[(size_t)vec * f.Q + q] : 0;
+  // cells by decreasing candidate count: the warps of a block get similar
+  // work and the largest cells start first
+  const int cell = cell_order[item];
+  const int q = cell / f.U, ukey = cell % f.U;
+  const int vec0 = blockIdx.y * 64 + lane, vec1 = vec0 + 32;
+  const uint32_t s0 = vec0 < n_vec ? (uint32_t)demand[(size_t)vec0 * f.Q + q] : 0u;
+  const uint32_t s1 = vec1 < n_vec ? (uint32_t)demand[(size_t)vec1 * f.Q + q] : 0u;
   const int T = f.T, VM = f.VM;
+  // per type: start and size of the cell's usage bucket (register-resident:
+  // compile-time type indices, guarded by t < T)
   int bsz[PX_MAXT], bst[PX_MAXT];
-  int64_t lstride[PX_MAXT], prod = 1;
-  {
-    int64_t ls = 1;
-    for (int t = T - 1; t >= 0; t--) {
+  int64_t prod = 1;
+#pragma unroll
+  for (int t = 0; t < PX_MAXT; t++) {
+    bsz[t] = 1;
+    bst[t] = 0;
+    if (t < T) {
       const int ut = (ukey / f.ustride[t]) % (f.Nt[t] + 1);
       const int32_t *bs = f.bstart + ((size_t)q * T + t) * (PX_MAXD + 2);
       bst[t] = bs[ut];
       bsz[t] = bs[ut + 1] - bs[ut];
       prod *= bsz[t];
-      lstride[t] = ls;
-      ls *= f.L[q * T + t];
     }
   }
-  int A[VMT];
+  uint32_t dA[VMT];  // A_{j-1} - A_j for j = 1..VMT (fill order: non-increasing; pads 0)
 #pragma unroll
-  for (int j = 0; j < VMT; j++) A[j] = j < VM ? slot_acc[q * VM + j] : 0;
-  uint64_t best_s = 0, best_i = ~0ull;
+  for (int j = 0; j < VMT; j++) {
+    const uint32_t a0 = j < VM ? (uint32_t)slot_acc[q * VM + j] : 0u;
+    const uint32_t a1 = j + 1 < VM ? (uint32_t)slot_acc[q * VM + j + 1] : 0u;
+    dA[j] = a0 - a1;
+  }
+  uint32_t b0lo = 0, b0hi = 0, b1lo = 0, b1hi = 0;  // packed best scores (first candidate always taken)
+  int32_t k0best = 0, k1best = 0;
   for (int64_t k0 = 0; k0 < prod; k0 += GV_TILE) {
     for (int r = lane; r < GV_TILE; r += 32) {
       const int64_t k = k0 + r;
       if (k >= prod) break;
-      int64_t x = k;
+      uint32_t x = (uint32_t)k;  // < 2^31 (host check)
       int cap[VMT];
 #pragma unroll
       for (int j = 0; j < VMT; j++) cap[j] = 0;
-      uint64_t sub = 0;
-      for (int t = T - 1; t >= 0; t--) {
-        const int o = (int)(x % bsz[t]);
-        x /= bsz[t];
-        const int rk = f.bucket[f.list_off[q][t] + bst[t] + o];
-        sub += (uint64_t)rk * lstride[t];
-        const int32_t *ec = f.ecap + (f.list_off[q][t] + rk) * VM;
 #pragma unroll
-        for (int j = 0; j < VMT; j++) cap[j] += j < VM ? ec[j] : 0;
+      for (int t = PX_MAXT - 1; t >= 0; t--) {
+        if (t < T) {
+          const uint32_t o = x % (uint32_t)bsz[t];
+          x /= (uint32_t)bsz[t];
+          const int rk = f.bucket[f.list_off[q][t] + bst[t] + o];
+          const int32_t *ec = f.ecap + (f.list_off[q][t] + rk) * VM;
+#pragma unroll
+          for (int j = 0; j < VMT; j++) cap[j] += j < VM ? ec[j] : 0;
+        }
       }
+      int acc = 0;
 #pragma unroll
-      for (int j = 0; j < VMT; j++) tcap[w][r][j] = cap[j];
-      tsub[w][r] = sub;
+      for (int j = 0; j < VMT; j++) {
+        acc += cap[j];
+        tc[w][r][j] = acc;
+      }
     }
     __syncwarp();
     const int nt = prod - k0 < GV_TILE ? (int)(prod - k0) : GV_TILE;
+#pragma unroll 2
     for (int r = 0; r < nt; r++) {
-      int rem = s;
-      uint64_t acc = 0;
+      int32_t C[CS];
+#pragma unroll
+      for (int j = 0; j < CS; j += 4) *(int4 *)&C[j] = *(const int4 *)&tc[w][r][j];
+      uint64_t a0 = 0, a1 = 0;
+      uint32_t m0 = 0, m1 = 0;
 #pragma unroll
       for (int j = 0; j < VMT; j++) {
-        const int tk = min(rem, tcap[w][r][j]);
-        acc += (uint64_t)(uint32_t)A[j] * (uint32_t)tk;
-        rem -= tk;
+        m0 = min(s0, (uint32_t)C[j]);
+        m1 = min(s1, (uint32_t)C[j]);
+        a0 = madw(m0, dA[j], a0);
+        a1 = madw(m1, dA[j], a1);
       }
-      const uint64_t sc = px_pack((uint32_t)(s - rem), acc);
-      if (sc > best_s || best_i == ~0ull) { best_s = sc; best_i = tsub[w][r]; }
+      // packed score (served << 42) + accsum as (hi, lo) words; served = m_VM
+      const uint32_t h0 = (uint32_t)(a0 >> 32) + (m0 << (PX_ACC_BITS - 32)), l0 = (uint32_t)a0;
+      const uint32_t h1 = (uint32_t)(a1 >> 32) + (m1 << (PX_ACC_BITS - 32)), l1 = (uint32_t)a1;
+      const int32_t kk = (int32_t)(k0 + r);
+      if (h0 > b0hi || (h0 == b0hi && l0 > b0lo)) { b0hi = h0; b0lo = l0; k0best = kk; }
+      if (h1 > b1hi || (h1 == b1hi && l1 > b1lo)) { b1hi = h1; b1lo = l1; k1best = kk; }
     }
     __syncwarp();
   }
-  if (active) {
-    BestRec &out = g[((size_t)vec * f.Q + q) * f.U + ukey];
-    out.score = best_s;
-    out.index = best_i;  // ~0 when no count vector has this usage
+  // rank (lexicographic sub-index) of the chosen candidates
+  auto sub_of = [&](uint32_t k) -> uint64_t {
+    uint64_t sub = 0, ls = 1;
+#pragma unroll
+    for (int t = PX_MAXT - 1; t >= 0; t--) {
+      if (t < T) {
+        const uint32_t o = k % (uint32_t)bsz[t];
+        k /= (uint32_t)bsz[t];
+        sub += (uint64_t)f.bucket[f.list_off[q][t] + bst[t] + o] * ls;
+        ls *= (uint64_t)f.L[q * T + t];
+      }
+    }
+    return sub;
+  };
+  const bool none = prod == 0;  // no count vector has this usage
+  if (vec0 < n_vec) {
+    BestRec &out = g[((size_t)vec0 * f.Q + q) * f.U + ukey];
+    out.score = ((uint64_t)b0hi << 32) | b0lo;
+    out.index = none ? ~0ull : sub_of(k0best);
+  }
+  if (vec1 < n_vec) {
+    BestRec &out = g[((size_t)vec1 * f.Q + q) * f.U + ukey];
+    out.score = ((uint64_t)b1hi << 32) | b1lo;
+    out.index = none ? ~0ull : sub_of(k1best);
   }
 }
 
@@ -267,49 +327,55 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
                                                          const int32_t *__restrict__ Pdev, int K,
                                                          const int32_t *__restrict__ slot_code,
                                                          const int32_t *__restrict__ slot_acc, SolRec *out) {
-  // Budget DP with the current stage in shared memory: G_q(b) = max over
-  // u <= b of g_q(u) + G_{q+1}(b - u).  One warp per budget b; lanes split the
-  // box {u <= b}.  Every stage is also written to global memory for the
-  // reconstruction.  A score of ~0 marks "no count vector with this usage"
-  // (a real score has accsum < 10^6 * served < 2^42 - 1, so it is never ~0).
+  // Budget DP with the stages in shared memory: G_q(b) = max over u <= b of
+  // g_q(u) + G_{q+1}(b - u).  The boxes {u <= b} -- restricted to u_t = 0 on
+  // the types where family q has no feasible variant, the only usages it can
+  // have -- are cut into work items (b, outer digits of u), each a run of the
+  // innermost type's digit (contiguous keys); items are listed round-robin
+  // over budgets, so the threads of a warp update different budgets with a
+  // shared-memory atomicMax, and every thread gets a similar share.  The key
+  // of b - u is key(b) - key(u) (keys are linear).  Every stage is also
+  // written to global memory for the reconstruction.  A score of ~0 marks "no
+  // count vector with this usage" (a real score has accsum < 10^6 * served <
+  // 2^42 - 1, so it is never ~0).
   extern __shared__ uint64_t dsm[];
   const int vec = blockIdx.x;
   const int Q = f.Q, U = f.U, T = f.T;
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
   const BestRec *gv = g + (size_t)vec * Q * U;
   uint64_t *G = Gbuf + (size_t)vec * (Q + 1) * U;
-  uint64_t *Gn = dsm, *gq = dsm + U;
+  uint64_t *Gn = dsm, *gq = dsm + U, *Gc = dsm + 2 * U;
   const uint64_t NONE = ~0ull;
-  for (int b = threadIdx.x; b < U; b += blockDim.x) { Gn[b] = 0; G[(size_t)Q * U + b] = 0; }
+  for (int b = threadIdx.x; b < U; b += blockDim.x) { Gn[b] = 0; Gc[b] = 0; G[(size_t)Q * U + b] = 0; }
   for (int q = Q - 1; q >= 0; q--) {
     for (int u = threadIdx.x; u < U; u += blockDim.x) {
       const BestRec e = gv[(size_t)q * U + u];
       gq[u] = e.index == ~0ull ? NONE : e.score;
     }
     __syncthreads();
-    uint64_t *Gq = G + (size_t)q * U;
-    for (int b = w; b < U; b += nw) {
-      // lanes stride over the precomputed (u, b - u) key pairs of budget b
-      uint64_t best = 0;
-      bool have = false;
-      const int pe = f.pstart[b + 1];
-      for (int k = f.pstart[b] + lane; k < pe; k += 32) {
-        const int2 pr = __ldg(&f.pairs[k]);
-        const uint64_t gs = gq[pr.x];
+    const int2 *it = f.items + (size_t)f.morder[q] * f.istride;
+    const int n_it = f.nitems[q];
+    const bool inner = T >= 1 && ((f.fmask[q] >> (T - 1)) & 1u);
+    const int Nin = f.Nt[T - 1] + 1;
+    for (int i = threadIdx.x; i < n_it; i += blockDim.x) {
+      const int2 w = it[i];  // (budget key b, key of the usage's outer digits)
+      const int b = w.x, up = w.y;
+      const int lim_in = inner ? b % Nin : 0;  // innermost type: stride 1
+      uint64_t best = 0;  // partial maxima are >= 0; u = 0 is always a usage
+      for (int x = 0; x <= lim_in; x++) {
+        const uint64_t gs = gq[up + x];
         if (gs == NONE) continue;
-        const uint64_t c = gs + Gn[pr.y];
-        if (!have || c > best) { best = c; have = true; }
+        const uint64_t c = gs + Gn[b - up - x];
+        best = c > best ? c : best;
       }
-      for (int o = 16; o; o >>= 1) {
-        const uint64_t b2 = __shfl_xor_sync(0xffffffffu, best, o);
-        const int h2 = __shfl_xor_sync(0xffffffffu, (int)have, o);
-        if (h2 && (!have || b2 > best)) { best = b2; have = true; }
-      }
-      if (lane == 0) Gq[b] = best;  // u = 0 is always valid: have == true
+      atomicMax((unsigned long long *)&Gc[b], (unsigned long long)best);
     }
     __syncthreads();
-    for (int b = threadIdx.x; b < U; b += blockDim.x) Gn[b] = Gq[b];
+    for (int b = threadIdx.x; b < U; b += blockDim.x) {
+      G[(size_t)q * U + b] = Gc[b];
+      Gn[b] = 0;  // becomes the next stage's accumulator
+    }
     __syncthreads();
+    uint64_t *tmp = Gn; Gn = Gc; Gc = tmp;
   }
   // reconstruction (warp 0): lexicographically smallest count tensor
   __shared__ uint64_t pick_sub[PX_MAXQ];
@@ -318,19 +384,23 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
     int bv[PX_MAXT];
     for (int t = 0; t < T; t++) bv[t] = f.Nt[t];
     for (int q = 0; q < Q; q++) {
-      int bkey = 0, box = 1;
-      for (int t = 0; t < T; t++) { bkey += bv[t] * f.ustride[t]; box *= bv[t] + 1; }
+      int bkey = 0, box = 1, lim[PX_MAXT];
+      for (int t = 0; t < T; t++) {
+        bkey += bv[t] * f.ustride[t];
+        lim[t] = (f.fmask[q] >> t) & 1u ? bv[t] : 0;
+        box *= lim[t] + 1;
+      }
       const uint64_t target = G[(size_t)q * U + bkey];
       uint64_t bsub = ~0ull;
       uint64_t bu = 0;
       for (int i = lane; i < box; i += 32) {
         int x = i, uk = 0, rk = 0;
         for (int t = T - 1; t >= 0; t--) {
-          const int ut = x % (bv[t] + 1);
-          x /= bv[t] + 1;
+          const int ut = x % (lim[t] + 1);
+          x /= lim[t] + 1;
           uk += ut * f.ustride[t];
-          rk += (bv[t] - ut) * f.ustride[t];
         }
+        rk = bkey - uk;
         const BestRec e = gv[(size_t)q * U + uk];
         if (e.index == ~0ull) continue;
         if (e.score + G[(size_t)(q + 1) * U + rk] == target && e.index < bsub) { bsub = e.index; bu = (uint64_t)uk; }
@@ -416,7 +486,6 @@ __global__ void __launch_bounds__(DP_THREADS) k_fact_dp(const __grid_constant__ 
 int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32_t *h_dev_type,
                       const int32_t *d_dev, const int32_t *d_demand, int VM, const Tables &tab, const std::vector<int32_t> &h_P,
                       SolRec *d_sol) {
-  (void)h_P;
   const int Q = ctx->Q, T = ctx->T, D = a->D, K = 1 + ctx->M;
   FactLayout f;
   memset(&f, 0, sizeof f);
@@ -428,7 +497,9 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
   f.U = (int32_t)U;
   // list capacity: count vectors with sum <= N_t over V_q variants (before pruning)
   int64_t total = 0;
+  unsigned __int128 maxprod = 0;  // bound on the candidates of one (family, usage) cell
   for (int q = 0; q < Q; q++) {
+    unsigned __int128 prod = 1;
     f.V[q] = ctx->V[q];
     f.off[q] = ctx->off[q];
     for (int t = 0; t < T; t++) {
@@ -437,7 +508,9 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
       if (c > (1u << 24)) return px_fail(ctx, PROTEUS_ERANGE, "count-vector list too large");
       f.list_off[q][t] = total;
       total += (int64_t)c;
+      prod *= c;
     }
+    if (prod > maxprod) maxprod = prod;
   }
   if (total > (1ll << 26)) return px_fail(ctx, PROTEUS_ERANGE, "count-vector lists too large");
   const size_t szL = (size_t)Q * T * 4, szB = (size_t)Q * T * (PX_MAXD + 2) * 4;
@@ -453,39 +526,66 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
   f.ecap = (int32_t *)buf; buf += (size_t)total * VM * 4;
   f.esum = (int32_t *)buf; buf += (size_t)total * 4;
   f.ecnt = (uint8_t *)buf;
-  // the DP's (u, b - u) key pairs of every budget b (lattice indexing only)
-  if (ctx->dp_pairs_U != U || ctx->dp_pairs_key != std::vector<int32_t>(f.Nt, f.Nt + T)) {
-    std::vector<int32_t> pst(U + 1);
-    std::vector<int2> pr;
-    for (int b = 0; b < U; b++) {
-      pst[b] = (int32_t)pr.size();
-      int bv[PX_MAXT], box = 1;
-      for (int t = 0; t < T; t++) { bv[t] = (b / f.ustride[t]) % (f.Nt[t] + 1); box *= bv[t] + 1; }
-      for (int x0 = 0; x0 < box; x0++) {
-        int x = x0, uk = 0, rk = 0;
-        for (int t = T - 1; t >= 0; t--) {
-          const int ut = x % (bv[t] + 1);
-          x /= bv[t] + 1;
-          uk += ut * f.ustride[t];
-          rk += (bv[t] - ut) * f.ustride[t];
-        }
-        pr.push_back(make_int2(uk, rk));
-      }
-      if (pr.size() > (1u << 26)) return px_fail(ctx, PROTEUS_ERANGE, "usage lattice too large for the DP");
-    }
-    pst[U] = (int32_t)pr.size();
-    char *pb = (char *)px_buf(ctx, B_FACT3, pr.size() * sizeof(int2) + pst.size() * 4 + 64);
-    if (!pb) return px_fail(ctx, PROTEUS_ENOMEM, "DP pairs");
-    PX_CUDA(ctx, cudaMemcpyAsync(pb, pr.data(), pr.size() * sizeof(int2), cudaMemcpyHostToDevice, ctx->stream));
-    PX_CUDA(ctx, cudaMemcpyAsync(pb + pr.size() * sizeof(int2), pst.data(), pst.size() * 4, cudaMemcpyHostToDevice,
-                                 ctx->stream));
-    ctx->dp_pairs = pb;
-    ctx->dp_pairs_n = (int64_t)pr.size();
-    ctx->dp_pairs_U = U;
-    ctx->dp_pairs_key.assign(f.Nt, f.Nt + T);
+  // DP work items (lattice indexing only), per distinct feasibility mask:
+  // (budget b, key of the outer digits u_0..u_{T-2} <= b on the mask's
+  // types), round r holding the r-th outer combination of every budget
+  std::vector<uint32_t> masks;
+  for (int q = 0; q < Q; q++) {
+    uint32_t m = 0;
+    for (int t = 0; t < T; t++)
+      for (int v = 0; v < ctx->V[q]; v++)
+        if (h_P[(size_t)t * ctx->M + ctx->off[q] + v] > 0) m |= 1u << t;
+    f.fmask[q] = m;
+    int row = -1;
+    for (size_t k = 0; k < masks.size(); k++) if (masks[k] == m) row = (int)k;
+    if (row < 0) { row = (int)masks.size(); masks.push_back(m); }
+    f.morder[q] = row;
   }
-  f.pairs = (const int2 *)ctx->dp_pairs;
-  f.pstart = (const int32_t *)((const char *)ctx->dp_pairs + ctx->dp_pairs_n * sizeof(int2));
+  std::vector<int32_t> okey(f.Nt, f.Nt + T);
+  okey.insert(okey.end(), masks.begin(), masks.end());
+  if (ctx->dp_order_U != U || ctx->dp_order_key != okey) {
+    std::vector<std::vector<int2>> rows(masks.size());
+    for (size_t k = 0; k < masks.size(); k++) {
+      std::vector<std::vector<int32_t>> combos(U);
+      size_t maxc = 0;
+      for (int b = 0; b < U; b++) {
+        int lim[PX_MAXT], dig[PX_MAXT] = {0};
+        for (int t = 0; t < T; t++) lim[t] = (masks[k] >> t) & 1u ? (b / f.ustride[t]) % (f.Nt[t] + 1) : 0;
+        for (;;) {
+          int key = 0;
+          for (int t = 0; t + 1 < T; t++) key += dig[t] * f.ustride[t];
+          combos[b].push_back(key);
+          int t = T - 2;
+          for (; t >= 0; t--) {
+            if (dig[t] < lim[t]) { dig[t]++; break; }
+            dig[t] = 0;
+          }
+          if (t < 0) break;
+        }
+        maxc = std::max(maxc, combos[b].size());
+      }
+      for (size_t r = 0; r < maxc; r++)
+        for (int b = 0; b < U; b++)
+          if (r < combos[b].size()) rows[k].push_back(make_int2(b, combos[b][r]));
+      if (rows[k].size() > (1u << 26)) return px_fail(ctx, PROTEUS_ERANGE, "usage lattice too large for the DP");
+    }
+    size_t stride = 0;
+    for (auto &r : rows) stride = std::max(stride, r.size());
+    std::vector<int2> flat(rows.size() * stride, make_int2(0, 0));
+    for (size_t k = 0; k < rows.size(); k++) std::copy(rows[k].begin(), rows[k].end(), flat.begin() + k * stride);
+    char *pb = (char *)px_buf(ctx, B_FACT3, flat.size() * sizeof(int2) + 64);
+    if (!pb) return px_fail(ctx, PROTEUS_ENOMEM, "DP work items");
+    PX_CUDA(ctx, cudaMemcpyAsync(pb, flat.data(), flat.size() * sizeof(int2), cudaMemcpyHostToDevice, ctx->stream));
+    ctx->dp_order = pb;
+    ctx->dp_order_U = U;
+    ctx->dp_order_key = okey;
+    ctx->dp_items_stride = (int64_t)stride;
+    ctx->dp_items_n.clear();
+    for (auto &r : rows) ctx->dp_items_n.push_back((int32_t)r.size());
+  }
+  f.items = (const int2 *)ctx->dp_order;
+  f.istride = ctx->dp_items_stride;
+  for (int q = 0; q < Q; q++) f.nitems[q] = ctx->dp_items_n[f.morder[q]];
   const int n_vec = a->n_vec;
   BestRec *g = (BestRec *)px_buf(ctx, B_FACT1, sizeof(BestRec) * (size_t)n_vec * Q * U);
   uint64_t *G = (uint64_t *)px_buf(ctx, B_FACT2, 8 * (size_t)n_vec * (Q + 1) * U);
@@ -496,18 +596,58 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
     ctx->fact_lists_key = ctx->tab_key;
   }
   const int64_t nitems = (int64_t)n_vec * Q * U;
-  if (n_vec >= 8 && VM <= 8) {
-    dim3 grid((unsigned)((Q * U + 3) / 4), (unsigned)((n_vec + 31) / 32));
-    if (VM <= 3) PX_LAUNCH(ctx, "fact_g", k_fact_gv<3>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
-    else if (VM == 4) PX_LAUNCH(ctx, "fact_g", k_fact_gv<4>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
-    else if (VM == 5) PX_LAUNCH(ctx, "fact_g", k_fact_gv<5>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
-    else if (VM == 6) PX_LAUNCH(ctx, "fact_g", k_fact_gv<6>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
-    else PX_LAUNCH(ctx, "fact_g", k_fact_gv<8>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, g);
+  // cell order of the batched g kernel: count vectors of family q with usage
+  // u_t on type t = C(u_t + f - 1, f - 1) over the f feasible variants
+  std::vector<int32_t> gkey(okey);
+  gkey.insert(gkey.end(), ctx->V.begin(), ctx->V.end());
+  for (int q = 0; q < Q; q++)
+    for (int t = 0; t < T; t++) {
+      int fq = 0;
+      for (int v = 0; v < ctx->V[q]; v++) fq += h_P[(size_t)t * ctx->M + ctx->off[q] + v] > 0;
+      gkey.push_back(fq);
+    }
+  if (ctx->gv_order_key != gkey) {
+    std::vector<double> sz((size_t)Q * U);
+    for (int q = 0; q < Q; q++) {
+      int fq[PX_MAXT];
+      for (int t = 0; t < T; t++) {
+        fq[t] = 0;
+        for (int v = 0; v < ctx->V[q]; v++) fq[t] += h_P[(size_t)t * ctx->M + ctx->off[q] + v] > 0;
+      }
+      for (int u = 0; u < U; u++) {
+        double x = 1;
+        for (int t = 0; t < T; t++) {
+          const int ut = (u / f.ustride[t]) % (f.Nt[t] + 1);
+          if (fq[t] == 0) { x *= ut == 0; continue; }
+          double c = 1;  // C(ut + fq - 1, fq - 1)
+          for (int i = 1; i < fq[t]; i++) c = c * (ut + i) / i;
+          x *= c;
+        }
+        sz[(size_t)q * U + u] = x;
+      }
+    }
+    std::vector<int32_t> ord((size_t)Q * U);
+    for (size_t i = 0; i < ord.size(); i++) ord[i] = (int32_t)i;
+    std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return sz[a] > sz[b]; });
+    char *ob = (char *)px_buf(ctx, B_FACT4, ord.size() * 4 + 64);
+    if (!ob) return px_fail(ctx, PROTEUS_ENOMEM, "cell order");
+    PX_CUDA(ctx, cudaMemcpyAsync(ob, ord.data(), ord.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+    ctx->gv_order = ob;
+    ctx->gv_order_key = gkey;
+  }
+  const int32_t *cell_order = (const int32_t *)ctx->gv_order;
+  if (n_vec >= 8 && VM <= 8 && maxprod < ((unsigned __int128)1 << 31)) {  // candidate ordinals in int32
+    dim3 grid((unsigned)((Q * U + 3) / 4), (unsigned)((n_vec + 63) / 64));
+    if (VM <= 3) PX_LAUNCH(ctx, "fact_g", k_fact_gv<3>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
+    else if (VM == 4) PX_LAUNCH(ctx, "fact_g", k_fact_gv<4>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
+    else if (VM == 5) PX_LAUNCH(ctx, "fact_g", k_fact_gv<5>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
+    else if (VM == 6) PX_LAUNCH(ctx, "fact_g", k_fact_gv<6>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
+    else PX_LAUNCH(ctx, "fact_g", k_fact_gv<8>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
   } else {
     PX_LAUNCH(ctx, "fact_g", k_fact_g, (unsigned)((nitems + FG_WARPS - 1) / FG_WARPS), FG_WARPS * 32, 0, f, n_vec,
               d_demand, tab.slot_acc, g);
   }
-  const size_t dsmem = (size_t)2 * U * 8;
+  const size_t dsmem = (size_t)3 * U * 8;
   if (dsmem > 200 * 1024) return px_fail(ctx, PROTEUS_ERANGE, "usage lattice %lld too large for the DP", (long long)U);
   if (dsmem > 48 * 1024)
     PX_CUDA(ctx, cudaFuncSetAttribute(k_fact_dp, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsmem));

@@ -220,3 +220,37 @@ def test_device_pointer_inputs(px, oracle_mod):
     t = lambda a: torch.as_tensor(np.asarray(a, np.int32)).cuda()
     dev = px.solve(t(cl.device_type), t(cl.slo_us), t(cfg["demand"]), mode=0)[0]
     assert (dev.score, dev.index, dev.option.tolist()) == (host.score, host.index, host.option.tolist())
+
+
+def test_c4_solve_batch_outputs(px, oracle_mod):
+    """proteus_solve_batch: array outputs on the host and on the device equal
+    the per-vector proteus_solve results; a seeded sample is checked against
+    the oracle directly."""
+    import torch
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c4")
+    prof, cl, dem = cfg["prof"], cfg["cluster"], cfg["demand"][:700]
+    px.load_profiles(prof)
+    sols = px.solve(cl.device_type, cl.slo_us, dem, mode=2)
+    host, ncand = px.solve_batch(cl.device_type, cl.slo_us, dem, mode=2)
+    assert ncand == sols[0].n_candidates
+    D, n = len(cl.device_type), len(dem)
+    dev_out = {"score": torch.empty(n, dtype=torch.uint64, device="cuda"),
+               "served": torch.empty(n, dtype=torch.int64, device="cuda"),
+               "accsum": torch.empty(n, dtype=torch.int64, device="cuda"),
+               "option": torch.empty((n, D), dtype=torch.int32, device="cuda"),
+               "z_qps": torch.empty((n, D), dtype=torch.int32, device="cuda")}
+    t_dem = torch.as_tensor(dem, dtype=torch.int32, device="cuda")
+    px.solve_batch(cl.device_type, cl.slo_us, t_dem, mode=2, out=dev_out)
+    d = {k: v.cpu().numpy() for k, v in dev_out.items()}
+    for v, s in enumerate(sols):
+        assert (host["score"][v], host["served"][v], host["unmet"][v], host["accsum"][v], host["eff_acc_micro"][v]) \
+            == (s.score, s.served, s.unmet, s.accsum, s.eff_acc_micro)
+        assert host["option"][v].tolist() == s.option.tolist() and host["z_qps"][v].tolist() == s.z.tolist()
+        assert (int(d["score"][v]), d["served"][v], d["accsum"][v]) == (s.score, s.served, s.accsum)
+        assert d["option"][v].tolist() == s.option.tolist() and d["z_qps"][v].tolist() == s.z.tolist()
+    rng = np.random.default_rng(405)
+    for v in sorted(rng.choice(n, size=6, replace=False)):
+        r = oracle_mod.solve(prof, cl.device_type, cl.slo_us, dem[v], 2)
+        assert (host["served"][v], host["accsum"][v]) == (r["served"], r["accsum"])
+        assert host["option"][v].tolist() == r["option"].tolist()
