@@ -188,13 +188,16 @@ __global__ void __launch_bounds__(FG_WARPS * 32) k_fact_g(const __grid_constant_
 // keeps the first maximum in candidate order (= lowest lexicographic rank)
 // as a candidate ordinal and decodes its rank once at the end.
 #define GV_TILE 64
+#ifndef GV_NV
+#define GV_NV 4  // demand vectors per lane
+#endif
 __device__ __forceinline__ uint64_t madw(uint32_t a, uint32_t b, uint64_t c) {
   uint64_t r;
   asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(a), "r"(b), "l"(c));
   return r;
 }
 
-template <int VMT>
+template <int VMT, int NV>
 __global__ void __launch_bounds__(128) k_fact_gv(const __grid_constant__ FactLayout f, int n_vec,
                                                  const int32_t *__restrict__ demand,
                                                  const int32_t *__restrict__ slot_acc,
@@ -208,9 +211,12 @@ __global__ void __launch_bounds__(128) k_fact_gv(const __grid_constant__ FactLay
   // work and the largest cells start first
   const int cell = cell_order[item];
   const int q = cell / f.U, ukey = cell % f.U;
-  const int vec0 = blockIdx.y * 64 + lane, vec1 = vec0 + 32;
-  const uint32_t s0 = vec0 < n_vec ? (uint32_t)demand[(size_t)vec0 * f.Q + q] : 0u;
-  const uint32_t s1 = vec1 < n_vec ? (uint32_t)demand[(size_t)vec1 * f.Q + q] : 0u;
+  uint32_t sv[NV];  // demands of this lane's vectors blockIdx.y * 32 NV + lane + 32 i
+#pragma unroll
+  for (int i = 0; i < NV; i++) {
+    const int vec = blockIdx.y * 32 * NV + lane + 32 * i;
+    sv[i] = vec < n_vec ? (uint32_t)demand[(size_t)vec * f.Q + q] : 0u;
+  }
   const int T = f.T, VM = f.VM;
   // per type: start and size of the cell's usage bucket (register-resident:
   // compile-time type indices, guarded by t < T)
@@ -235,8 +241,10 @@ __global__ void __launch_bounds__(128) k_fact_gv(const __grid_constant__ FactLay
     const uint32_t a1 = j + 1 < VM ? (uint32_t)slot_acc[q * VM + j + 1] : 0u;
     dA[j] = a0 - a1;
   }
-  uint32_t b0lo = 0, b0hi = 0, b1lo = 0, b1hi = 0;  // packed best scores (first candidate always taken)
-  int32_t k0best = 0, k1best = 0;
+  uint32_t blo[NV], bhi[NV];  // packed best scores (first candidate always taken)
+  int32_t kbest[NV];
+#pragma unroll
+  for (int i = 0; i < NV; i++) { blo[i] = 0; bhi[i] = 0; kbest[i] = 0; }
   for (int64_t k0 = 0; k0 < prod; k0 += GV_TILE) {
     for (int r = lane; r < GV_TILE; r += 32) {
       const int64_t k = k0 + r;
@@ -270,21 +278,20 @@ __global__ void __launch_bounds__(128) k_fact_gv(const __grid_constant__ FactLay
       int32_t C[CS];
 #pragma unroll
       for (int j = 0; j < CS; j += 4) *(int4 *)&C[j] = *(const int4 *)&tc[w][r][j];
-      uint64_t a0 = 0, a1 = 0;
-      uint32_t m0 = 0, m1 = 0;
-#pragma unroll
-      for (int j = 0; j < VMT; j++) {
-        m0 = min(s0, (uint32_t)C[j]);
-        m1 = min(s1, (uint32_t)C[j]);
-        a0 = madw(m0, dA[j], a0);
-        a1 = madw(m1, dA[j], a1);
-      }
-      // packed score (served << 42) + accsum as (hi, lo) words; served = m_VM
-      const uint32_t h0 = (uint32_t)(a0 >> 32) + (m0 << (PX_ACC_BITS - 32)), l0 = (uint32_t)a0;
-      const uint32_t h1 = (uint32_t)(a1 >> 32) + (m1 << (PX_ACC_BITS - 32)), l1 = (uint32_t)a1;
       const int32_t kk = (int32_t)(k0 + r);
-      if (h0 > b0hi || (h0 == b0hi && l0 > b0lo)) { b0hi = h0; b0lo = l0; k0best = kk; }
-      if (h1 > b1hi || (h1 == b1hi && l1 > b1lo)) { b1hi = h1; b1lo = l1; k1best = kk; }
+#pragma unroll
+      for (int i = 0; i < NV; i++) {
+        uint64_t a = 0;
+        uint32_t m = 0;
+#pragma unroll
+        for (int j = 0; j < VMT; j++) {
+          m = min(sv[i], (uint32_t)C[j]);
+          a = madw(m, dA[j], a);
+        }
+        // packed score (served << 42) + accsum as (hi, lo) words; served = m_VM
+        const uint32_t h = (uint32_t)(a >> 32) + (m << (PX_ACC_BITS - 32)), l = (uint32_t)a;
+        if (h > bhi[i] || (h == bhi[i] && l > blo[i])) { bhi[i] = h; blo[i] = l; kbest[i] = kk; }
+      }
     }
     __syncwarp();
   }
@@ -303,15 +310,14 @@ __global__ void __launch_bounds__(128) k_fact_gv(const __grid_constant__ FactLay
     return sub;
   };
   const bool none = prod == 0;  // no count vector has this usage
-  if (vec0 < n_vec) {
-    BestRec &out = g[((size_t)vec0 * f.Q + q) * f.U + ukey];
-    out.score = ((uint64_t)b0hi << 32) | b0lo;
-    out.index = none ? ~0ull : sub_of(k0best);
-  }
-  if (vec1 < n_vec) {
-    BestRec &out = g[((size_t)vec1 * f.Q + q) * f.U + ukey];
-    out.score = ((uint64_t)b1hi << 32) | b1lo;
-    out.index = none ? ~0ull : sub_of(k1best);
+#pragma unroll
+  for (int i = 0; i < NV; i++) {
+    const int vec = blockIdx.y * 32 * NV + lane + 32 * i;
+    if (vec < n_vec) {
+      BestRec &out = g[((size_t)vec * f.Q + q) * f.U + ukey];
+      out.score = ((uint64_t)bhi[i] << 32) | blo[i];
+      out.index = none ? ~0ull : sub_of(kbest[i]);
+    }
   }
 }
 
@@ -637,12 +643,10 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
   }
   const int32_t *cell_order = (const int32_t *)ctx->gv_order;
   if (n_vec >= 8 && VM <= 8 && maxprod < ((unsigned __int128)1 << 31)) {  // candidate ordinals in int32
-    dim3 grid((unsigned)((Q * U + 3) / 4), (unsigned)((n_vec + 63) / 64));
-    if (VM <= 3) PX_LAUNCH(ctx, "fact_g", k_fact_gv<3>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
-    else if (VM == 4) PX_LAUNCH(ctx, "fact_g", k_fact_gv<4>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
-    else if (VM == 5) PX_LAUNCH(ctx, "fact_g", k_fact_gv<5>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
-    else if (VM == 6) PX_LAUNCH(ctx, "fact_g", k_fact_gv<6>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
-    else PX_LAUNCH(ctx, "fact_g", k_fact_gv<8>, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
+    dim3 grid((unsigned)((Q * U + 3) / 4), (unsigned)((n_vec + 32 * GV_NV - 1) / (32 * GV_NV)));
+    auto kern = VM <= 3 ? k_fact_gv<3, GV_NV> : VM == 4 ? k_fact_gv<4, GV_NV> : VM == 5 ? k_fact_gv<5, GV_NV>
+              : VM == 6 ? k_fact_gv<6, GV_NV> : k_fact_gv<8, GV_NV>;
+    PX_LAUNCH(ctx, "fact_g", kern, grid, 128, 0, f, n_vec, d_demand, tab.slot_acc, cell_order, g);
   } else {
     PX_LAUNCH(ctx, "fact_g", k_fact_g, (unsigned)((nitems + FG_WARPS - 1) / FG_WARPS), FG_WARPS * 32, 0, f, n_vec,
               d_demand, tab.slot_acc, g);
