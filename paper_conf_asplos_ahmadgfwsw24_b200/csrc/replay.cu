@@ -25,6 +25,7 @@
 //            and the reference formulation in the tests).
 // a13: k_count reduces the final latency rows to per-scenario violations,
 // on-time counts and accuracy sums.
+#include <climits>
 #include <cstdlib>
 #include <cstring>
 
@@ -44,56 +45,77 @@ __global__ void k_check_trace(const uint32_t *__restrict__ arr, const uint8_t *_
 }
 
 // ------------------------------------------------------------- routing ----
-// One block.  Weights and the SWRR pattern of every family (R8).
+// Weights and the SWRR pattern of every family (R8); one warp per family.
 //   routing 0: member weight z_d for hosting devices with z_d > 0, sink weight
 //              s_q - sum z (unmet demand, reading R7)
 //   routing 1: weight 1 per hosting device that fits batch 1 (depth >= 1); no sink
+// Each step adds every member's weight to its current value, picks the
+// largest current value (lowest member index on ties, the sink last) and
+// subtracts the period W_q from it: lanes hold members d = lane, lane + 32,
+// lane + 64 and the pick is a warp maximum of (current, -index).
+__device__ __forceinline__ int32_t route_weight(int routing, int q, int d, int D, int M, int bmax,
+                                                const int32_t *option, const int32_t *z, const int32_t *dev_type,
+                                                const int32_t *demand, const int32_t *fam_of_m, const int32_t *lat) {
+  if (d < D) {
+    const int o = option[d];
+    if (o <= 0 || fam_of_m[o - 1] != q) return 0;
+    if (routing == 0) return z[d];
+    return lat[((size_t)dev_type[d] * M + (o - 1)) * bmax] > 0 ? 1 : 0;
+  }
+  if (routing != 0) return 0;  // the sink: unmet demand
+  int64_t zs = 0;
+  for (int k = 0; k < D; k++) {
+    const int o = option[k];
+    if (o > 0 && fam_of_m[o - 1] == q) zs += z[k];
+  }
+  return (int32_t)(demand[q] - zs);
+}
+
 __global__ void k_route_prepare(int routing, int Q, int D, int M, int bmax, const int32_t *__restrict__ option,
                                 const int32_t *__restrict__ z, const int32_t *__restrict__ dev_type,
                                 const int32_t *__restrict__ demand, const int32_t *__restrict__ fam_of_m,
                                 const int32_t *__restrict__ lat, uint8_t *pattern, int32_t *pat_off,
                                 int32_t *pat_len) {
   __shared__ int32_t W[PX_MAXQ];
-  const int q = threadIdx.x;
-  int32_t w[PX_MAXD + 1];
-  int32_t cur[PX_MAXD + 1];
-  if (q < Q) {
-    int64_t tot = 0, zsum = 0;
-    for (int d = 0; d < D; d++) {
-      w[d] = 0;
-      const int o = option[d];
-      if (o <= 0 || fam_of_m[o - 1] != q) continue;
-      if (routing == 0) {
-        w[d] = z[d];
-        zsum += z[d];
-      } else {
-        w[d] = lat[((size_t)dev_type[d] * M + (o - 1)) * bmax] > 0 ? 1 : 0;
-      }
-      tot += w[d];
-    }
-    w[D] = routing == 0 ? (int32_t)(demand[q] - zsum) : 0;
-    tot += w[D];
-    W[q] = (int32_t)tot;
+  const int q = blockIdx.x, lane = threadIdx.x;
+  // periods of every family (for this family's pattern offset)
+  for (int k = lane; k < Q; k += 32) {
+    int64_t tot = 0;
+    for (int d = 0; d <= D; d++) tot += route_weight(routing, k, d, D, M, bmax, option, z, dev_type, demand, fam_of_m, lat);
+    W[k] = (int32_t)tot;
   }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    int32_t acc = 0;
-    for (int k = 0; k < Q; k++) { pat_off[k] = acc; pat_len[k] = W[k]; acc += W[k]; }
-  }
-  __syncthreads();
-  if (q >= Q) return;
+  __syncwarp();
+  int32_t off = 0;
+  for (int k = 0; k < q; k++) off += W[k];
   const int32_t Wq = W[q];
-  uint8_t *pat = pattern + pat_off[q];
-  for (int d = 0; d <= D; d++) cur[d] = 0;
+  if (lane == 0) { pat_off[q] = off; pat_len[q] = Wq; }
+  int32_t w[3], cur[3];
+#pragma unroll
+  for (int i = 0; i < 3; i++) {
+    const int d = lane + 32 * i;
+    w[i] = d <= D ? route_weight(routing, q, d, D, M, bmax, option, z, dev_type, demand, fam_of_m, lat) : 0;
+    cur[i] = 0;
+  }
+  uint8_t *pat = pattern + off;
   for (int32_t k = 0; k < Wq; k++) {
-    int best = -1;
-    for (int d = 0; d <= D; d++) {
-      if (w[d] == 0) continue;
-      cur[d] += w[d];
-      if (best < 0 || cur[d] > cur[best]) best = d;
+    long long key = LLONG_MIN;
+#pragma unroll
+    for (int i = 0; i < 3; i++) {
+      if (w[i] == 0) continue;
+      cur[i] += w[i];
+      const long long kk = ((long long)cur[i] << 32) | (0xFFFFFFFFu - (uint32_t)(lane + 32 * i));
+      key = kk > key ? kk : key;
     }
-    cur[best] -= Wq;
-    pat[k] = (uint8_t)best;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      const long long v = __shfl_xor_sync(0xffffffffu, key, o);
+      key = v > key ? v : key;
+    }
+    const int best = (int)(0xFFFFFFFFu - (uint32_t)(key & 0xFFFFFFFFll));
+#pragma unroll
+    for (int i = 0; i < 3; i++)
+      if (best == lane + 32 * i) cur[i] -= Wq;
+    if (lane == 0) pat[k] = (uint8_t)best;
   }
 }
 
@@ -220,10 +242,15 @@ __global__ void k_scatter(const uint8_t *__restrict__ target, const uint32_t *__
 // Latencies are produced in device-major order (latd[s][p], p = position in
 // the per-device arrays), which every lane writes sequentially; k_unpermute
 // turns them into per-query order at the end.
-struct SpecExit {
-  int64_t F;
-  int32_t ov;  // exit head - chunk end (overhang of the last batch into the next chunk)
-  int32_t mer;  // phase runs: offset from the chunk start where the run met run 0 (else the chunk length)
+// Per (scenario, chunk): the run whose latencies a chunk's rows hold -- it
+// entered the chunk at head st + edh with the device free at eF and left it
+// at head en + xov with the device free at xF.  k_spec writes runs entered
+// idle at the chunk start; k_fix and k_stitch replace them.
+struct ChunkSt {
+  int64_t xF;
+  int64_t eF;
+  int32_t xov;
+  int32_t edh;
 };
 
 struct LaneParam {  // per (scenario, device)
@@ -257,6 +284,7 @@ __global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__re
 struct LaneArgs {
   int S, D, M, bmax, nsc, CH;
   int64_t N, NCH;
+  int64_t NS;             // row stride of latd (N rounded up to 32: 16-byte aligned rows for bulk copies)
   const int32_t *option, *dev_type, *lat, *sc_list;
   const LaneParam *lp;
   const int64_t *devOff;  // [D + 2]; segment D = the sink
@@ -264,13 +292,15 @@ struct LaneArgs {
   const int32_t *goff;    // [D + 1] phase-A warp-group offsets
   const uint32_t *devArr;
   uint32_t *latd;         // [S][N] device-major
-  SpecExit *ex;           // [S][NCH]
+  ChunkSt *cs;            // [S][NCH] chunk runs (written by k_spec / k_fix, read by k_stitch)
+  const ChunkSt *csp;     // k_fix: the previous round's
   uint64_t *agg;          // [3][S]
   int maxchk;             // convergence checks per chunk (free decisions only)
-  int rmax;               // phase runs: lanes with 2 <= Bmax <= rmax speculate Bmax runs per chunk
-  uint32_t *vlat;         // latencies of the phase runs r >= 1 (lane base voff[lane] + (r - 1) n)
-  SpecExit *vex;          // their exit states (lane base voff[S D + lane] + (r - 1) nch)
-  const int64_t *voff;    // [2][S * D]
+  int scan1;              // Bmax = 1 lanes are produced by k_scan1_* (the chunk kernels skip them)
+  const int64_t *lstart;  // [S * D][2] (head, F) where k_stitch starts a lane the full-batch scan took (head -1: not taken)
+  unsigned *lstat;        // [S * D][2] speculative decisions that were full batches sent when the device
+                          // freed (backlog), and all speculative decisions; k_fix leaves backlogged lanes
+                          // (a quarter or more) to the stitch's max-plus stretches
   long long debug;        // > 0: k_stitch prints lanes slower than this many cycles (diagnostic)
 };
 
@@ -336,7 +366,7 @@ __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ 
   const LaneParam p = a.lp[s * a.D + d];
   const int64_t st = a.devOff[d], n = a.devOff[d + 1] - st;
   if (n == 0) return;
-  uint32_t *out = a.latd + (size_t)s * a.N + st;
+  uint32_t *out = a.latd + (size_t)s * a.NS + st;
   if (p.Bmax < 1) {  // never routed to (z = 0 / depth 0); kept for safety
     for (int64_t j = 0; j < n; j++) out[j] = 0xFFFFFFFFu;
     return;
@@ -353,20 +383,13 @@ __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ 
   }
 }
 
-// number of speculative runs per chunk of a lane (see k_spec)
-__host__ __device__ __forceinline__ int n_phase_runs(int Bmax, int rmax) {
-  return Bmax < 2 ? 1 : Bmax < rmax ? Bmax : rmax;
-}
-
 // ---- phase A: speculative chunks
 // Each device array is cut into chunks of CH queries.  One warp per (device,
 // scenario, 32 consecutive chunks); lane = chunk, replayed from an idle
-// device (the true state at the start of the trace, R13).  All lanes follow
-// the same rule parameters, so the warp stays close to converged.
-// Launched twice: run 0 (rbase 0, gridDim.z 1), then the phase runs r >= 1
-// (rbase 1), which stop as soon as they meet run 0 (same batch end, same
-// finish) and take run 0's exit; `mer` records where.
-__global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a, int rbase) {
+// device at the chunk's first query (the true state at the start of the
+// trace, R13).  All lanes follow the same rule parameters, so the warp stays
+// close to converged.
+__global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a) {
   __shared__ int32_t sG[PX_MAXD + 1];
   for (int k = threadIdx.x; k <= a.D; k += blockDim.x) sG[k] = a.goff[k];
   __syncthreads();
@@ -382,53 +405,38 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
   const int64_t c = (int64_t)(g - sG[d]) * 32 + lane;
-  const int r = blockIdx.z + rbase;  // phase run r: first batch starts at st + r
-  if (r > 0 && r >= n_phase_runs(p.Bmax, a.rmax)) return;
-  if (c < nch) {
-    const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
-    const int64_t lane_id = (int64_t)s * a.D + d;
-    uint32_t *out = r == 0 ? a.latd + (size_t)s * a.N + off : a.vlat + a.voff[lane_id] + (int64_t)(r - 1) * n;
-    int64_t h = st + r, F = 0;
-    SpecExit e;
-    e.mer = (int32_t)(en - st);
-    bool met = false;
-    if (p.Bmax < 1) {
-      for (int64_t j = st; j < en; j++) out[j] = 0xFFFFFFFFu;
-      h = en;
-    } else {
-      const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
-      GArr arr{a.devArr + off};
-      const uint32_t *run0 = a.latd + (size_t)s * a.N + off;
-      while (h < en) {
-        int64_t t;
-        const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
-        const int64_t Fn = t + T[b - 1];
-        const int64_t jend = h + b < en ? h + b : en;
-        for (int64_t j = h; j < jend; j++) out[j] = sat_lat(Fn - (int64_t)arr(j));
-        const int64_t j2 = h + b;
-        // met run 0: it also ends a batch at j2 - 1 finishing at Fn (the next
-        // batch always finishes later); tested after batches the device waited for
-        if (r > 0 && t > F && j2 < en && (int64_t)arr(j2 - 1) + run0[j2 - 1] == Fn &&
-            (int64_t)arr(j2) + run0[j2] != Fn) {
-          met = true;
-          e.mer = (int32_t)(j2 - st);
-          break;
-        }
-        F = Fn;
-        h = j2;
-      }
+  if (c >= nch || (a.scan1 && p.Bmax == 1)) return;
+  const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
+  uint32_t *out = a.latd + (size_t)s * a.NS + off;
+  int64_t h = st, F = 0;
+  if (p.Bmax < 1) {
+    for (int64_t j = st; j < en; j++) out[j] = 0xFFFFFFFFu;
+    h = en;
+  } else {
+    const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+    GArr arr{a.devArr + off};
+    unsigned nfull = 0, ndec = 0;
+    while (h < en) {
+      int64_t t;
+      const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
+      nfull += b == p.Bmax && t == F;
+      ndec++;
+      const int64_t Fn = t + T[b - 1];
+      const int64_t jend = h + b < en ? h + b : en;
+      for (int64_t j = h; j < jend; j++) out[j] = sat_lat(Fn - (int64_t)arr(j));
+      F = Fn;
+      h += b;
     }
-    if (met) {
-      const SpecExit e0 = a.ex[(size_t)s * a.NCH + a.choff[d] + c];
-      e.F = e0.F;
-      e.ov = e0.ov;
-    } else {
-      e.F = F;
-      e.ov = (int32_t)(h - en);
-    }
-    if (r == 0) a.ex[(size_t)s * a.NCH + a.choff[d] + c] = e;
-    else a.vex[a.voff[(int64_t)a.S * a.D + lane_id] + (int64_t)(r - 1) * nch + c] = e;
+    unsigned *ls = a.lstat + 2 * ((size_t)s * a.D + d);
+    if (nfull) atomicAdd(ls, nfull);
+    atomicAdd(ls + 1, ndec);
   }
+  ChunkSt e;
+  e.xF = F;
+  e.xov = (int32_t)(h - en);
+  e.eF = 0;
+  e.edh = 0;
+  a.cs[(size_t)s * a.NCH + a.choff[d] + c] = e;
 }
 
 // ---- phase B: exact stitch, one warp per (device, scenario)
@@ -446,10 +454,8 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
 // taken 32 batches per step with a ballot.  Rewritten latencies adjust the
 // counts by their difference from the speculative ones.  Arrivals stream
 // through a shared-memory ring; exit states are fetched 32 chunks at a time.
-#define SPECCAP 1024                 // chunk length limit of the stitch
 #define RSEG 1024                    // ring segment (queries), one bulk copy
 #define RING (4 * RSEG)              // per-warp arrival ring
-#define SPB (SPECCAP + 8)            // speculative-latency buffer (+ alignment lead)
 #define LEAN_C (1 << 30)
 #define SUMAX 4
 #ifdef PX_STITCH_DEBUG  // per-lane counters printed by k_stitch (PROTEUS_REPLAY_DEBUG=cycles)
@@ -469,6 +475,16 @@ __device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t b
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+// two bulk copies completing on one mbarrier (one arrival, both byte counts)
+__device__ __forceinline__ void bulk_load2(void *dst0, const void *src0, void *dst1, const void *src1, uint32_t bytes,
+                                           uint64_t *bar) {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(2 * bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(smem_u32(dst0)), "l"(src0), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(smem_u32(dst1)), "l"(src1), "r"(bytes), "r"(smem_u32(bar)) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
   asm volatile("{\n\t.reg .pred P1;\n\tWAIT_%=:\n\t"
@@ -525,13 +541,14 @@ __device__ __forceinline__ int decide_par(const Arr &A, int64_t n, int64_t h, in
 }
 
 __host__ __device__ __forceinline__ size_t stitch_wstride(int bmax) {
-  return ((size_t)RING + 2 * SPB + 12 + 64 * SUMAX + bmax + 3) & ~(size_t)3;
+  return ((size_t)2 * RING + 8 + 64 * SUMAX + bmax + 3) & ~(size_t)3;
 }
 static size_t stitch_smem(int bmax) { return 4 * stitch_wstride(bmax) * 4; }
 
 __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs a) {
-  // shared memory per warp: arrival ring [RING], spec latencies [2][SPB],
-  // mbarriers [4 ring + 2 spec], T [bmax]
+  // shared memory per warp: arrival ring [RING], stored-latency ring [RING]
+  // (the chunk runs' rows, same segments), mbarriers [4 ring slots], stretch
+  // finishes [32 SUMAX], T [bmax]
   extern __shared__ __align__(16) uint32_t ssm[];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int64_t gw = (int64_t)blockIdx.x * 4 + w;
@@ -540,31 +557,37 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   const LaneParam p = a.lp[s * a.D + d];
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
-  if (p.Bmax < 1 || nch < 2) return;
+  if (p.Bmax < 1 || nch < 2 || (a.scan1 && p.Bmax == 1)) return;
   uint32_t *wsm = ssm + (size_t)w * stitch_wstride(a.bmax);
   uint32_t *ring = wsm;
-  uint32_t *specbuf = wsm + RING;
-  uint64_t *bars = (uint64_t *)(wsm + RING + 2 * SPB);  // [0..3] ring slots, [4..5] spec buffers
-  int64_t *FeS = (int64_t *)(wsm + RING + 2 * SPB + 12);  // [32 SUMAX] stretch batch finishes
-  int32_t *T = (int32_t *)(wsm + RING + 2 * SPB + 12 + 64 * SUMAX);
+  uint32_t *lring = wsm + RING;
+  uint64_t *bars = (uint64_t *)(wsm + 2 * RING);  // ring slots
+  int64_t *FeS = (int64_t *)(wsm + 2 * RING + 8);  // [32 SUMAX] stretch batch finishes
+  int32_t *T = (int32_t *)(wsm + 2 * RING + 8 + 64 * SUMAX);
   const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
   for (int k = lane; k < a.bmax; k += 32) T[k] = Tg[k];
-  if (lane < 6) mbar_init(bars + lane);
+  if (lane < 4) mbar_init(bars + lane);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   __syncwarp();
-  uint32_t *out = a.latd + (size_t)s * a.N + off;
-  const uint32_t *src = out;  // the speculative run the current chunk is matched against
-  int64_t mr = 0;             // ... whose own latencies cover [h, mr), run 0's from mr on
-  const SpecExit *ex = a.ex + (size_t)s * a.NCH + a.choff[d];
+  uint32_t *out = a.latd + (size_t)s * a.NS + off;
+  const ChunkSt *cst = a.cs + (size_t)s * a.NCH + a.choff[d];
   const int64_t CH = a.CH;
-  int64_t h = (CH < n ? CH : n) + ex[0].ov, F = ex[0].F;
+  int64_t h = (CH < n ? CH : n) + cst[0].xov, F = cst[0].xF;
+  int64_t cstart = 1;  // first chunk to stitch; a lane the full-batch scan took starts where it stopped
+  bool fresh = false;  // ... with the positions below h of that chunk already written
+  if (a.lstart && a.lstart[2 * ((size_t)s * a.D + d)] >= 0) {
+    h = a.lstart[2 * ((size_t)s * a.D + d)];
+    F = a.lstart[2 * ((size_t)s * a.D + d) + 1];
+    cstart = h / CH;
+    fresh = true;
+  }
   // Arrivals stream through a 4-segment ring by TMA bulk copies of whole
   // 1024-query segments of the routed array (segment g >> 10 of the absolute
   // index g = off + j sits in slot (g >> 10) & 3, so ring[g & (RING - 1)] is
   // query g).  Segments up to the one 2 past h's are in flight; a slot is
   // refilled only after its previous segment has been waited for and lies
   // 2 segments behind h (the stitch reads back at most Bmax - 1 <= 1023).
-  const int64_t sg0 = (off + CH) >> 10;  // first segment ever read (chunk 1 starts at CH)
+  const int64_t sg0 = (off + (fresh ? h : CH)) >> 10;  // first segment ever read (chunk 1 starts at CH)
   int64_t sg_iss = sg0, sg_wait = sg0;
   auto seg_wait_one = [&]() {
     mbar_wait(bars + (sg_wait & 3), (uint32_t)(((sg_wait - sg0) >> 2) & 1));
@@ -575,7 +598,11 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
     while (sg_iss < lim) {
       while (sg_wait <= sg_iss - 4) seg_wait_one();
       __syncwarp();
-      if (lane == 0) bulk_load(ring + (sg_iss & 3) * RSEG, a.devArr + sg_iss * RSEG, RSEG * 4, bars + (sg_iss & 3));
+      // arrivals and the stored latencies of the same positions (the row holds
+      // the chunk runs' values at every position >= h: rewritten ones lie below)
+      if (lane == 0)
+        bulk_load2(ring + (sg_iss & 3) * RSEG, a.devArr + sg_iss * RSEG, lring + (sg_iss & 3) * RSEG,
+                   a.latd + (size_t)s * a.NS + sg_iss * RSEG, RSEG * 4, bars + (sg_iss & 3));
       sg_iss++;
     }
   };
@@ -592,26 +619,11 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   };
   const uint32_t ro = (uint32_t)(off & (RING - 1));
   auto AR = [&](int64_t j) -> int64_t { return ring[(ro + (uint32_t)j) & (RING - 1)]; };
+  auto LR = [&](int64_t j) -> uint32_t { return lring[(ro + (uint32_t)j) & (RING - 1)]; };
   auto put = [&](int64_t j, int64_t Fb) { out[j] = sat_lat(Fb - AR(j)); };
-  // Speculative latencies of chunk c (run 0) are bulk-copied into buffer
-  // (c - 1) & 1 while chunk c - 1 is stitched.
-  uint32_t *specL = specbuf;
-  int64_t spec_base = -1;
-  auto spec_issue = [&](int64_t c) {
-    if (c >= nch) return;
-    const int bi = (int)((c - 1) & 1);
-    if (c >= 3) mbar_wait(bars + 4 + bi, (uint32_t)(((c - 3) >> 1) & 1));  // previous use consumed
-    __syncwarp();
-    if (lane == 0) {
-      const int64_t st = c * CH, en = st + CH < n ? st + CH : n;
-      const uintptr_t g = (uintptr_t)(out + st), g0 = g & ~(uintptr_t)15;
-      const uint32_t bytes = (uint32_t)(((g - g0) + (uintptr_t)(en - st) * 4 + 15) & ~(uintptr_t)15);
-      bulk_load(specbuf + bi * SPB, (const void *)g0, bytes, bars + 4 + bi);
-    }
-  };
-  spec_issue(1);
-  // j in [h, en): always inside the cached window [spec_base, en)
-  auto spec_F = [&](int64_t j) -> int64_t { return AR(j) + specL[(int32_t)(j - spec_base)]; };
+  // the stored run's finish time of the batch holding query j (its latency
+  // row is rewritten only below the current head)
+  auto spec_F = [&](int64_t j) -> int64_t { return AR(j) + LR(j); };
   const int64_t TB = T[p.Bmax - 1];
   // the 32-bit decision needs L < C / 2 and every T(b) < C (so W_k < C and
   // t + T(b) < 2^31); per-lane W_k = L - T(k + 2) and T(k + 1) for the
@@ -624,10 +636,6 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   const int32_t W1 = lane + 33 < p.Bmax ? (int32_t)p.L - T[lane + 33] : 0;
   const int32_t T0 = lane < p.Bmax ? T[lane] : 0;
   const int32_t T1 = lane + 32 < p.Bmax ? T[lane + 32] : 0;
-  const int R = n_phase_runs(p.Bmax, a.rmax);
-  const int64_t lane_id = (int64_t)s * a.D + d;
-  const uint32_t *vl = R > 1 ? a.vlat + a.voff[lane_id] : nullptr;
-  const SpecExit *vx = R > 1 ? a.vex + a.voff[(int64_t)a.S * a.D + lane_id] : nullptr;
   const int SU = p.Bmax >= 16 ? 1 : p.Bmax >= 8 ? 2 : SUMAX;  // batches per lane in a full-batch stretch
   const uint32_t bmagic = (uint32_t)((1ull << 32) / (uint64_t)p.Bmax + 1);  // q / Bmax = umulhi(q, bmagic), q < 2^16
   // SW: a full batch needs its last arrival <= max(F_i, a[h_i] + SW) (see the stretch)
@@ -638,69 +646,34 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   bool lastfull = true;
   long long dbg_t0 = clock64(), dbg_dec = 0, dbg_jump = 0, dbg_match = 0, dbg_chk = 0;
   long long dbg_sec[5] = {0, 0, 0, 0, 0}, dbg_tk = 0;
-  for (int64_t c0 = 1; c0 < nch; c0 += 32) {
-    int64_t pF = 0;
-    int pov = 0;
-    if (c0 + lane < nch) {
-      const SpecExit e = ex[c0 + lane];
-      pF = e.F;
-      pov = e.ov;
-    }
+  for (int64_t c0 = cstart; c0 < nch; c0 += 32) {
+    ChunkSt cr = {0, 0, 0, 0};
+    if (c0 + lane < nch) cr = cst[c0 + lane];
     const int cnt = nch - c0 < 32 ? (int)(nch - c0) : 32;
     for (int k = 0; k < cnt; k++) {
-      const int64_t st = (c0 + k) * CH, en = st + CH < n ? st + CH : n;
-      const int64_t eF = __shfl_sync(0xffffffffu, pF, k);
-      const int eov = __shfl_sync(0xffffffffu, pov, k);
       const int64_t c = c0 + k;
-      spec_issue(c + 1);
+      const int64_t st = c * CH, en = st + CH < n ? st + CH : n;
+      const int64_t xF = __shfl_sync(0xffffffffu, cr.xF, k);
+      const int xov = __shfl_sync(0xffffffffu, cr.xov, k);
+      const int64_t eF = __shfl_sync(0xffffffffu, cr.eF, k);
+      const int edh = __shfl_sync(0xffffffffu, cr.edh, k);
       need(h, (h < en ? h : en) + p.Bmax + 1);
-      if (h > st) {  // queries of this chunk in the last batch of the previous one
+      if (h > st && !(fresh && c == cstart)) {  // queries of this chunk in the last batch of the previous one
         const int64_t hi = h < en ? h : en;
         for (int64_t j = st + lane; j < hi; j += 32) put(j, F);
       }
       if (h >= en) continue;
-      // match against the run whose first batch starts where the true one
-      // does: phase r = h - st (run 0 = the chunk's own start)
-      const int ovr = (int)(h - st);
-      const bool var = ovr > 0 && ovr < R;
-      int64_t xF = eF;
-      int xov = eov;
-      mr = st;
-      src = out;
-      if (var) {
-        src = vl + (int64_t)(ovr - 1) * n;
-        const SpecExit ve = vx[(int64_t)(ovr - 1) * nch + c];
-        xF = ve.F;
-        xov = ve.ov;
-        mr = st + ve.mer;
-      }
-      if ((ovr == 0 || var) && F <= AR(h)) {  // speculative start = true state
-        for (int64_t j = h + lane; j < mr; j += 32) out[j] = src[j];
+      // the stored run of the chunk entered at (st + edh, eF): the true run
+      // takes the same decisions from the same head when its device is free
+      // at the same time, or when both are free by the head's arrival
+      if (h - st == edh && (F == eF || (F <= AR(h) && eF <= AR(h)))) {
         h = en + xov;
         F = xF;
         PX_DBG(dbg_match++);
         continue;
       }
       int checks = a.maxchk;
-      // the speculative latencies of [h, en) are cached at the first meeting
-      // test of the chunk: the true run has only rewritten positions < h
-      spec_base = -1;
-      auto spec_cache = [&]() {
-        if (spec_base >= 0) return;
-        const int bi = (int)((c - 1) & 1);
-        specL = specbuf + bi * SPB;
-        mbar_wait(bars + 4 + bi, (uint32_t)(((c - 1) >> 1) & 1));  // run 0's, prefetched
-        if (!var) {
-          spec_base = st - (int64_t)(((uintptr_t)(out + st) & 15) >> 2);
-          return;
-        }
-        __syncwarp();  // a phase run's: plain loads over the prefetched copy
-        spec_base = h;
-        const int64_t m = en - h;
-        for (int64_t i = lane; i < m; i += 32) specL[i] = (h + i < mr ? src : out)[h + i];
-        __syncwarp();
-      };
-      bool spec_ready = false;  // latency cache of this chunk loaded (at its first meeting test)
+      const bool spec_ready = true;  // stored latencies stream through lring (positions >= h)
       while (h < en) {
         PX_DBG(if (dbg_tk) dbg_sec[3] += clock64() - dbg_tk; dbg_tk = clock64());
         if (h >= h_safe) need(h, h + look + 1);  // decision + the stretch test's two batches
@@ -838,7 +811,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
             // only queries the ring holds for this decision are read (k <= lim: the meeting test's lane b)
             r.du = k <= lim && h + k < n ? (uint32_t)AR(h + k) - uah : 0u;
             const uint32_t dn = k + 1 < lim ? (uint32_t)AR(h + k + 1) - uah : 0u;
-            r.sp = test && h + k < en ? specL[(int32_t)(h + k - spec_base)] : 0u;
+            r.sp = test && h + k < en ? LR(h + k) : 0u;
             r.dk = r.du < (uint32_t)LEAN_C ? (int32_t)r.du : LEAN_C;
             const int32_t tau = r.dk > t0 ? r.dk : t0;
             const bool capped = k + 1 == p.Bmax;
@@ -882,8 +855,6 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
               const unsigned e = __ballot_sync(0xffffffffu, (uint64_t)s0.sp + s0.du == (uint64_t)(uint32_t)c);
               conv = ((e >> (b - 1)) & 1u) && !((e >> b) & 1u);
             } else {
-              spec_cache();
-              spec_ready = true;
               conv = spec_F(j2 - 1) == Fn && spec_F(j2) != Fn;
             }
           }
@@ -895,8 +866,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
           F = Fn;
           lastfull = b == p.Bmax;
           if (conv) {
-            // the rest of the chunk is the speculative run's (phase runs: their own latencies up to mr)
-            for (int64_t jj = h + lane; jj < mr; jj += 32) out[jj] = specL[jj - spec_base];
+            // the rest of the chunk is the stored run's
             h = en + xov;
             F = xF;
             break;
@@ -974,8 +944,6 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         if (isfree && j2 < en && checks > 0) {
           checks--;
           PX_DBG(dbg_chk++);
-          spec_cache();
-          spec_ready = true;
           conv = spec_F(j2 - 1) == Fn && spec_F(j2) != Fn;
         }
         PX_DBG(__syncwarp(); dbg_sec[1] += clock64() - dbg_tk; dbg_tk = clock64());
@@ -986,8 +954,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         F = Fn;
         lastfull = b == p.Bmax;
         if (conv) {
-          // the rest of the chunk is the speculative run's (phase runs: their own latencies up to mr)
-          for (int64_t jj = h + lane; jj < mr; jj += 32) out[jj] = specL[jj - spec_base];
+          // the rest of the chunk is the stored run's
           h = en + xov;
           F = xF;
           break;
@@ -997,20 +964,441 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   }
   if (a.debug && lane == 0) {
     const long long cyc = clock64() - dbg_t0;
-    if (cyc > a.debug) printf("stitch s=%d d=%d n=%lld Bmax=%d L=%lld nch=%lld cycles=%lld dec=%lld jump=%lld match=%lld chk=%lld "
+    if (cyc > a.debug) printf("stitch s=%d d=%d n=%lld Bmax=%d L=%lld nch=%lld start=%lld full=%u dec_spec=%u cycles=%lld dec=%lld jump=%lld match=%lld chk=%lld "
                               "sdec=%lld schk=%lld swr=%lld sloop=%lld sring=%lld\n", s, d,
-                              (long long)n, p.Bmax, (long long)p.L, (long long)nch, cyc, dbg_dec, dbg_jump, dbg_match, dbg_chk,
+                              (long long)n, p.Bmax, (long long)p.L, (long long)nch, (long long)(fresh ? cstart * CH : -1),
+                              a.lstat[2 * ((size_t)s * a.D + d)], a.lstat[2 * ((size_t)s * a.D + d) + 1], cyc, dbg_dec, dbg_jump, dbg_match, dbg_chk,
                               dbg_sec[0], dbg_sec[1], dbg_sec[2], dbg_sec[3], dbg_sec[4]);
   }
 }
 
+// ---- phase B, parallel form: fix-up rounds, one warp per (chunk, scenario)
+// Round k re-walks every chunk c >= 1 whose entry state -- the exit of chunk
+// c - 1 in round k - 1 -- differs from the entry of the run its rows hold,
+// from that entry until the new run meets the stored one (same head and the
+// same finish time after a batch the device waited for: from there on the
+// two runs take the same decisions) or the chunk ends.  Entries that differ
+// only in a device-free time that is <= the head's arrival give the same
+// decisions and need only the overhang rewritten.  Chunk c's exit changes
+// only if it did not meet; *changed counts those, and a round with no
+// change leaves every chunk exact (chunk 0 starts at the true initial state,
+// R13, and by induction each chunk entry is the true one).  Reads of the
+// stored row happen before the round rewrites them (positions >= the head).
+__global__ void __launch_bounds__(128) k_fix(const __grid_constant__ LaneArgs a, unsigned *changed) {
+  __shared__ int64_t sC[PX_MAXD + 1];
+  for (int k = threadIdx.x; k <= a.D; k += blockDim.x) sC[k] = a.choff[k];
+  __syncthreads();
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t g = (int64_t)blockIdx.y * 4 + w;  // chunk index over all devices of the routing mode
+  if (g >= sC[a.D]) return;
+  int d = 0;
+  while (g >= sC[d + 1]) d++;
+  const int s = a.sc_list[blockIdx.x];
+  const int64_t c = g - sC[d];
+  const size_t row = (size_t)s * a.NCH + sC[d];
+  const ChunkSt old = a.csp[row + c];
+  const LaneParam p = a.lp[s * a.D + d];
+  if (a.scan1 && p.Bmax == 1) return;  // produced by k_scan1_*
+  const unsigned *ls = a.lstat + 2 * ((size_t)s * a.D + d);
+  if (c == 0 || p.Bmax < 1 || 4ull * ls[0] >= ls[1]) {
+    // chunk 0 is exact from the start; unrouted devices have no runs;
+    // backlogged lanes are left to the stitch (changed[1] says one exists)
+    if (c == 1 && p.Bmax >= 1 && 4ull * ls[0] >= ls[1] && lane == 0) atomicOr(changed + 1, 1u);
+    if (lane == 0) a.cs[row + c] = old;
+    return;
+  }
+  const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+  const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
+  const ChunkSt prev = a.csp[row + c - 1];
+  int64_t h = st + prev.xov, F = prev.xF;
+  const uint32_t *A = a.devArr + off;
+  uint32_t *out = a.latd + (size_t)s * a.NS + off;
+  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  ChunkSt nw = old;
+  nw.edh = (int32_t)(h - st);
+  nw.eF = F;
+  const int64_t ah0 = h < n ? (int64_t)__ldg(A + h) : INT64_MAX;
+  const bool same_head = h - st == old.edh;
+  if (same_head && (F == old.eF || (F <= ah0 && old.eF <= ah0))) {
+    if (F != old.eF) {  // same decisions; the overhang belongs to the new finish time
+      const int64_t hi = h < en ? h : en;
+      for (int64_t j = st + lane; j < hi; j += 32) out[j] = sat_lat(F - (int64_t)__ldg(A + j));
+    }
+    if (lane == 0) a.cs[row + c] = nw;
+    return;
+  }
+  {
+    const int64_t hi = h < en ? h : en;  // queries of this chunk in the last batch of the previous one
+    for (int64_t j = st + lane; j < hi; j += 32) out[j] = sat_lat(F - (int64_t)__ldg(A + j));
+  }
+  bool met = false;
+  while (h < en) {
+    // decision (R1-R5) as a ballot over queue states k = 0, 1, ... (decide_par),
+    // with the stored run's finish times of the same positions for the
+    // meeting test, all read before this batch's latencies are written
+    const int64_t ah = __ldg(A + h);
+    const int64_t t0 = F > ah ? F : ah;
+    int q0 = 1;
+    for (;;) {  // queries queued at t0 (arrivals are sorted: a prefix)
+      const int64_t j = h + q0 + lane;
+      const bool le = q0 + lane < p.Bmax && j < n && (int64_t)__ldg(A + j) <= t0;
+      const int cnt = __popc(__ballot_sync(0xffffffffu, le));
+      q0 += cnt;
+      if (cnt < 32) break;
+    }
+    int b = 0;
+    int64_t t = 0;
+    for (int kb = q0 - 1;; kb += 32) {
+      const int k = kb + lane;
+      bool stop = false, now = false;
+      int64_t tau = 0, W = 0;
+      if (k + 1 <= p.Bmax && h + k < n) {
+        const int64_t ak = __ldg(A + h + k);
+        tau = ak > t0 ? ak : t0;
+        const bool capped = k + 1 == p.Bmax;
+        const int64_t nxt = h + k + 1 < n ? (int64_t)__ldg(A + h + k + 1) : INT64_MAX;
+        W = capped ? 0 : ah + p.L - T[k + 1];
+        now = capped || tau >= W;
+        stop = (capped || nxt > tau) && (now || nxt > W);
+      }
+      const unsigned bal = __ballot_sync(0xffffffffu, stop);
+      if (bal) {
+        const int sl = __ffs(bal) - 1;
+        t = __shfl_sync(0xffffffffu, now ? tau : W, sl);
+        b = kb + sl + 1;
+        break;
+      }
+    }
+    const int64_t Fn = t + T[b - 1];
+    const int64_t j2 = h + b;
+    if (t > F && j2 < en) {  // met: the stored run also ends a batch at j2 - 1 finishing at Fn
+      const int64_t f1 = (int64_t)__ldg(A + j2 - 1) + out[j2 - 1];
+      const int64_t f2 = (int64_t)__ldg(A + j2) + out[j2];
+      met = f1 == Fn && f2 != Fn;
+    }
+    __syncwarp();
+    const int64_t hi = j2 < en ? j2 : en;
+    for (int64_t j = h + lane; j < hi; j += 32) out[j] = sat_lat(Fn - (int64_t)__ldg(A + j));
+    h = j2;
+    F = Fn;
+    if (met) break;
+  }
+  if (!met) {
+    nw.xF = F;
+    nw.xov = (int32_t)(h - en);
+    if (lane == 0 && (nw.xF != old.xF || nw.xov != old.xov)) atomicAdd(changed, 1u);
+  }
+  if (lane == 0) a.cs[row + c] = nw;
+}
+
+// ---- lanes with Bmax = 1 (no batching, "w/o AB"): every
+// decision dispatches the head at t = max(F, a_h) (R4: a queue of one is
+// full), so F_i = max(F_{i-1}, a_i) + T(1) with F_{-1} = 0 (R13).  With
+// G_i = F_i - (i + 1) T(1) this is G_i = max(G_{i-1}, a_i - i T(1)), G_{-1} = 0:
+// a prefix maximum, computed exactly in parallel (block maxima, per-device
+// prefix over blocks, then per-warp scans).  The SLO does not enter the rule,
+// so every Bmax = 1 scenario of a device gets the same latency row.
+#define SCAN_BLK 4096
+struct Scan1Args {
+  int D, nsc;
+  int64_t N, NS;
+  int64_t boff[PX_MAXD + 1];  // block offsets per device (SCAN_BLK queries per block)
+  const int64_t *devOff;
+  const uint32_t *devArr;
+  const int32_t *T1;          // [D] T(1) of the device's variant (0: device has no Bmax = 1 lane)
+  const int32_t *sc_list;
+  const LaneParam *lp;
+  uint32_t *latd;
+  int64_t *bmx, *bpre;        // [blocks] block maxima, exclusive prefix maxima
+};
+
+__device__ __forceinline__ int scan1_dev(const Scan1Args &a, int64_t b) {
+  int d = 0;
+  while (b >= a.boff[d + 1]) d++;
+  return d;
+}
+
+__global__ void __launch_bounds__(256) k_scan1_reduce(const __grid_constant__ Scan1Args a) {
+  const int64_t b = blockIdx.x;
+  const int d = scan1_dev(a, b);
+  const int64_t T1 = a.T1[d];
+  int64_t m = INT64_MIN;
+  if (T1 > 0) {
+    const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+    const int64_t i0 = (b - a.boff[d]) * SCAN_BLK;
+    for (int64_t i = i0 + threadIdx.x; i < i0 + SCAN_BLK && i < n; i += blockDim.x) {
+      const int64_t x = (int64_t)__ldg(a.devArr + off + i) - i * T1;
+      m = x > m ? x : m;
+    }
+  }
+  __shared__ int64_t red[8];
+  for (int o = 16; o; o >>= 1) {
+    const int64_t v = __shfl_xor_sync(0xffffffffu, m, o);
+    m = v > m ? v : m;
+  }
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = m;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int k = 1; k < 8; k++) m = red[k] > m ? red[k] : m;
+    a.bmx[b] = m;
+  }
+}
+
+// one warp per device: exclusive prefix maximum over its blocks, seeded with G_{-1} = 0
+__global__ void k_scan1_prefix(const __grid_constant__ Scan1Args a) {
+  const int d = blockIdx.x, lane = threadIdx.x;
+  int64_t carry = 0;
+  for (int64_t b0 = a.boff[d]; b0 < a.boff[d + 1]; b0 += 32) {
+    const int64_t b = b0 + lane;
+    int64_t v = b < a.boff[d + 1] ? a.bmx[b] : INT64_MIN;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t u = __shfl_up_sync(0xffffffffu, v, o);
+      if (lane >= o && u > v) v = u;
+    }
+    int64_t ex = __shfl_up_sync(0xffffffffu, v, 1);
+    if (lane == 0) ex = INT64_MIN;
+    if (b < a.boff[d + 1]) a.bpre[b] = ex > carry ? ex : carry;
+    const int64_t tot = __shfl_sync(0xffffffffu, v, 31);
+    carry = tot > carry ? tot : carry;
+  }
+}
+
+__global__ void __launch_bounds__(256) k_scan1_apply(const __grid_constant__ Scan1Args a) {
+  __shared__ int64_t wmax[8];
+  __shared__ int32_t rows[4096];
+  __shared__ int nrows;
+  const int64_t b = blockIdx.x;
+  const int d = scan1_dev(a, b);
+  const int64_t T1 = a.T1[d];
+  if (T1 <= 0) return;
+  if (threadIdx.x == 0) {
+    int k = 0;
+    for (int i = 0; i < a.nsc && k < 4096; i++) {
+      const int s = a.sc_list[i];
+      if (a.lp[s * a.D + d].Bmax == 1) rows[k++] = s;
+    }
+    nrows = k;
+  }
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+  const int64_t i0 = (b - a.boff[d]) * SCAN_BLK + (int64_t)w * (SCAN_BLK / 8);
+  const int64_t i1 = i0 + SCAN_BLK / 8 < n ? i0 + SCAN_BLK / 8 : n;
+  int64_t m = INT64_MIN;  // this warp's segment maximum
+  for (int64_t i = i0 + lane; i < i1; i += 32) {
+    const int64_t x = (int64_t)__ldg(a.devArr + off + i) - i * T1;
+    m = x > m ? x : m;
+  }
+  for (int o = 16; o; o >>= 1) {
+    const int64_t v = __shfl_xor_sync(0xffffffffu, m, o);
+    m = v > m ? v : m;
+  }
+  if (lane == 0) wmax[w] = m;
+  __syncthreads();
+  int64_t carry = a.bpre[b];
+  for (int k = 0; k < w; k++) carry = wmax[k] > carry ? wmax[k] : carry;
+  const int nr = nrows;
+  for (int64_t c0 = i0; c0 < i1; c0 += 32) {
+    const int64_t i = c0 + lane;
+    const int64_t ai = i < i1 ? (int64_t)__ldg(a.devArr + off + i) : 0;
+    int64_t v = i < i1 ? ai - i * T1 : INT64_MIN;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t u = __shfl_up_sync(0xffffffffu, v, o);
+      if (lane >= o && u > v) v = u;
+    }
+    const int64_t G = v > carry ? v : carry;
+    carry = __shfl_sync(0xffffffffu, G, 31);
+    if (i < i1) {
+      const uint32_t l = sat_lat(G + (i + 1) * T1 - ai);
+      for (int r = 0; r < nr; r++) a.latd[(size_t)rows[r] * a.NS + off + i] = l;
+    }
+  }
+}
+
+// ---- backlogged lanes (Bmax = B >= 2): while the device is backlogged
+// every batch is full, batch k = queries [kB, kB + B) from the trace start,
+// dispatched when the device frees and its last query A_k has arrived:
+// F_k = max(F_{k-1}, A_k) + T(B), F_{-1} = 0 -- the same prefix maximum as
+// above, G_k = max(G_{k-1}, A_k - k T(B)).  Batch k is full under the rule
+// (R1-R4) if A_k <= max(F_{k-1}, a_{kB} + SW), SW = L - T(B) when T(B) is the
+// largest of T(1..B) (else SW = -inf: the queue must hold B when the device
+// frees) -- the stretch condition of k_stitch.  The scan is exact up to the
+// first batch k* that fails it; k_stitch continues from (k* B, F_{k*-1}).
+// Lanes are taken when a quarter or more of their speculative decisions were
+// full batches sent the moment the device freed (k_spec's statistics).
+#define BSCAN_BLK 1024  // batches per block
+struct BScanArgs {
+  int D, nl;
+  int64_t NS;
+  const int64_t *loff;       // [nl + 1] block offsets per lane
+  const int32_t *lid;        // [nl] lane = s * D + d
+  const int64_t *devOff;
+  const uint32_t *devArr;
+  const int32_t *lat, *option, *dev_type;
+  int M, bmax;
+  const LaneParam *lp;
+  const unsigned *lstat;
+  uint32_t *latd;
+  int64_t *bmx, *bpre;       // [blocks]
+  unsigned long long *vio;   // [nl] first batch that fails the fullness test (init ~0)
+  int64_t *lstart;           // [S * D][2] stitch start (head, F); head -1 = lane not scanned
+};
+
+struct BScanLane {
+  int64_t off, n, nb, TB, SW;  // nb = full batches of the lane
+  int B, lane, blk;            // blk = block index within the lane
+  bool on;
+};
+
+__device__ __forceinline__ int bscan_find(const BScanArgs &a, int64_t b) {  // lane l: loff[l] <= b < loff[l + 1]
+  int lo = 0, hi = a.nl;
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (__ldg(a.loff + mid) <= b) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ BScanLane bscan_lane(const BScanArgs &a, int64_t b) {
+  BScanLane r;
+  const int l = bscan_find(a, b);
+  r.lane = a.lid[l];
+  r.blk = (int)(b - a.loff[l]);
+  const int d = r.lane % a.D;
+  const LaneParam p = a.lp[r.lane];
+  const unsigned *ls = a.lstat + 2 * (size_t)r.lane;
+  r.B = p.Bmax;
+  r.on = p.Bmax >= 2 && ls[1] > 0 && 4ull * ls[0] >= ls[1];
+  if (!r.on) return r;
+  r.off = a.devOff[d];
+  r.n = a.devOff[d + 1] - r.off;
+  r.nb = r.n / (r.B > 0 ? r.B : 1);
+  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  r.TB = r.B > 0 ? T[r.B - 1] : 0;
+  int32_t tbig = 0;
+  for (int k = 0; k + 1 < r.B; k++) tbig = T[k] > tbig ? T[k] : tbig;
+  r.SW = tbig <= r.TB ? (p.L - r.TB > 0 ? p.L - r.TB : 0) : INT64_MIN / 4;
+  return r;
+}
+
+__global__ void __launch_bounds__(256) k_bscan_reduce(const __grid_constant__ BScanArgs a) {
+  const BScanLane L = bscan_lane(a, blockIdx.x);
+  int64_t m = INT64_MIN;
+  if (L.on) {
+    const int64_t k0 = (int64_t)L.blk * BSCAN_BLK;
+    for (int64_t k = k0 + threadIdx.x; k < k0 + BSCAN_BLK && k < L.nb; k += blockDim.x) {
+      const int64_t x = (int64_t)__ldg(a.devArr + L.off + k * L.B + L.B - 1) - k * L.TB;
+      m = x > m ? x : m;
+    }
+  }
+  __shared__ int64_t red[8];
+  for (int o = 16; o; o >>= 1) {
+    const int64_t v = __shfl_xor_sync(0xffffffffu, m, o);
+    m = v > m ? v : m;
+  }
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = m;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int k = 1; k < 8; k++) m = red[k] > m ? red[k] : m;
+    a.bmx[blockIdx.x] = m;
+  }
+}
+
+__global__ void k_bscan_prefix(const __grid_constant__ BScanArgs a) {
+  const int l = blockIdx.x, lane = threadIdx.x;
+  int64_t carry = 0;  // G_{-1} = 0
+  for (int64_t b0 = a.loff[l]; b0 < a.loff[l + 1]; b0 += 32) {
+    const int64_t b = b0 + lane;
+    int64_t v = b < a.loff[l + 1] ? a.bmx[b] : INT64_MIN;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t u = __shfl_up_sync(0xffffffffu, v, o);
+      if (lane >= o && u > v) v = u;
+    }
+    int64_t ex = __shfl_up_sync(0xffffffffu, v, 1);
+    if (lane == 0) ex = INT64_MIN;
+    if (b < a.loff[l + 1]) a.bpre[b] = ex > carry ? ex : carry;
+    const int64_t tot = __shfl_sync(0xffffffffu, v, 31);
+    carry = tot > carry ? tot : carry;
+  }
+}
+
+// F_k of the block's batches into Fs (block-wide scan: per-warp segments of
+// BSCAN_BLK / 8 batches); returns false if the lane is not scanned
+__device__ __forceinline__ bool bscan_block_F(const BScanArgs &a, const BScanLane &L, int64_t *Fs, int64_t *wmax) {
+  if (!L.on) return false;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t k0 = (int64_t)L.blk * BSCAN_BLK + (int64_t)w * (BSCAN_BLK / 8);
+  const int64_t k1 = k0 + BSCAN_BLK / 8 < L.nb ? k0 + BSCAN_BLK / 8 : L.nb;
+  int64_t m = INT64_MIN;
+  for (int64_t k = k0 + lane; k < k1; k += 32) {
+    const int64_t x = (int64_t)__ldg(a.devArr + L.off + k * L.B + L.B - 1) - k * L.TB;
+    m = x > m ? x : m;
+  }
+  for (int o = 16; o; o >>= 1) {
+    const int64_t v = __shfl_xor_sync(0xffffffffu, m, o);
+    m = v > m ? v : m;
+  }
+  if (lane == 0) wmax[w] = m;
+  __syncthreads();
+  int64_t carry = a.bpre[blockIdx.x];
+  for (int k = 0; k < w; k++) carry = wmax[k] > carry ? wmax[k] : carry;
+  for (int64_t c0 = k0; c0 < k1; c0 += 32) {
+    const int64_t k = c0 + lane;
+    int64_t v = k < k1 ? (int64_t)__ldg(a.devArr + L.off + k * L.B + L.B - 1) - k * L.TB : INT64_MIN;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t u = __shfl_up_sync(0xffffffffu, v, o);
+      if (lane >= o && u > v) v = u;
+    }
+    const int64_t G = v > carry ? v : carry;
+    carry = __shfl_sync(0xffffffffu, G, 31);
+    if (k < k1) Fs[k - (int64_t)L.blk * BSCAN_BLK] = G + (k + 1) * L.TB;
+  }
+  __syncthreads();
+  return true;
+}
+
+__global__ void __launch_bounds__(256) k_bscan_verify(const __grid_constant__ BScanArgs a) {
+  __shared__ int64_t Fs[BSCAN_BLK], wmax[8];
+  const BScanLane L = bscan_lane(a, blockIdx.x);
+  if (!bscan_block_F(a, L, Fs, wmax)) return;
+  const int64_t kb = (int64_t)L.blk * BSCAN_BLK;
+  const int l = bscan_find(a, blockIdx.x);
+  for (int i = threadIdx.x; i < BSCAN_BLK && kb + i < L.nb; i += blockDim.x) {
+    const int64_t k = kb + i;
+    // F_{k-1} (F_{-1} = 0; at a block start G_{k-1} is the block's exclusive prefix)
+    const int64_t Fp = i > 0 ? Fs[i - 1] : k == 0 ? 0 : a.bpre[blockIdx.x] + k * L.TB;
+    const int64_t Ak = __ldg(a.devArr + L.off + k * L.B + L.B - 1);
+    const int64_t ah = __ldg(a.devArr + L.off + k * L.B);
+    const int64_t lim = Fp > ah + L.SW ? Fp : ah + L.SW;
+    if (Ak > lim) atomicMin(a.vio + l, (unsigned long long)k);
+  }
+}
+
+__global__ void __launch_bounds__(256) k_bscan_apply(const __grid_constant__ BScanArgs a) {
+  __shared__ int64_t Fs[BSCAN_BLK], wmax[8];
+  const BScanLane L = bscan_lane(a, blockIdx.x);
+  if (!bscan_block_F(a, L, Fs, wmax)) return;
+  const int l = bscan_find(a, blockIdx.x);
+  const unsigned long long v = a.vio[l];
+  const int64_t kstar = v < (unsigned long long)L.nb ? (int64_t)v : L.nb;  // batches taken
+  const int64_t kb = (int64_t)L.blk * BSCAN_BLK;
+  const int64_t ke = kb + BSCAN_BLK < kstar ? kb + BSCAN_BLK : kstar;
+  uint32_t *out = a.latd + (size_t)(L.lane / a.D) * a.NS + L.off;
+  for (int64_t j = kb * L.B + threadIdx.x; j < ke * L.B; j += blockDim.x)
+    out[j] = sat_lat(Fs[j / L.B - kb] - (int64_t)__ldg(a.devArr + L.off + j));
+  // the stitch starts at batch k* with the device free at F_{k*-1}
+  if (threadIdx.x == 0 && ((kstar == 0 && L.blk == 0) || (kstar > kb && kstar <= kb + BSCAN_BLK))) {
+    a.lstart[2 * (size_t)L.lane] = kstar * L.B;
+    a.lstart[2 * (size_t)L.lane + 1] = kstar == 0 ? 0 : Fs[kstar - 1 - kb];
+  }
+}
+
 // dropped queries (the sink segment, device index D): latency UINT32_MAX (R7)
-__global__ void k_sink(int64_t N, int S, int D, const int32_t *__restrict__ sc_list, int nsc, const int64_t *devOff,
+__global__ void k_sink(int64_t NS, int S, int D, const int32_t *__restrict__ sc_list, int nsc, const int64_t *devOff,
                        uint32_t *latd, uint64_t *agg) {
   for (int k = blockIdx.y; k < nsc; k += gridDim.y) {
     const int64_t st = devOff[D], n = devOff[D + 1] - st;
     const int s = sc_list[k];
-    uint32_t *row = latd + (size_t)s * N + st;
+    uint32_t *row = latd + (size_t)s * NS + st;
     for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n; j += (int64_t)gridDim.x * blockDim.x)
       row[j] = 0xFFFFFFFFu;
   }
@@ -1018,53 +1406,58 @@ __global__ void k_sink(int64_t N, int S, int D, const int32_t *__restrict__ sc_l
 
 // a13: per scenario, violations (latency > the SLO of the device's family, R6;
 // dropped queries included), on-time count and the serving variant's accuracy
-// summed over on-time queries (R9), over the device-major rows.
-__global__ void k_count(int64_t N, int S, int D, const int32_t *__restrict__ sc_list, const int64_t *__restrict__ devOff,
-                        const LaneParam *__restrict__ lp, const uint32_t *__restrict__ latd, uint64_t *agg) {
-  __shared__ int64_t sOff[PX_MAXD + 2], sL[PX_MAXD + 1];
-  __shared__ uint32_t sA[PX_MAXD + 1];
-  __shared__ unsigned long long red[3][32];
+// summed over on-time queries (R9), over the device-major rows.  A block takes
+// CNT_PER positions of one row and walks the device segments inside them:
+// per segment only the on-time count is accumulated (16-byte loads, one
+// compare per latency), then violations = length - on-time and the accuracy
+// sum = on-time x A.  The sink segment is all violations (nothing to read).
+#define CNT_PER 16384
+__global__ void __launch_bounds__(256) k_count(int64_t N, int64_t NS, int S, int D, const int32_t *__restrict__ sc_list,
+                                               const int64_t *__restrict__ devOff, const LaneParam *__restrict__ lp,
+                                               const uint32_t *__restrict__ latd, uint64_t *agg) {
+  __shared__ unsigned long long red[3][8];
   const int s = sc_list[blockIdx.y];
-  for (int k = threadIdx.x; k <= D + 1; k += blockDim.x) sOff[k] = devOff[k];
-  for (int k = threadIdx.x; k <= D; k += blockDim.x) {
-    sL[k] = k < D ? lp[s * D + k].L : -1;  // the sink: every latency is a violation
-    sA[k] = k < D ? lp[s * D + k].A : 0;
-  }
-  __syncthreads();
-  const uint32_t *row = latd + (size_t)s * N;
-  unsigned long long viol = 0, ont = 0, accs = 0;
-  const int64_t per = (N + gridDim.x - 1) / gridDim.x;
-  const int64_t lo = (int64_t)blockIdx.x * per, hi = lo + per < N ? lo + per : N;
-  int d = 0;
-  for (int64_t p0 = lo; p0 < hi; p0 += 4 * blockDim.x) {
-    while (d < D && sOff[d + 1] <= p0) d++;  // segment of this step's first position (uniform)
-    uint32_t l[4];
-#pragma unroll
-    for (int k = 0; k < 4; k++) {
-      const int64_t p = p0 + threadIdx.x + (int64_t)k * blockDim.x;
-      l[k] = p < hi ? row[p] : 0;
+  const uint32_t *row = latd + (size_t)s * NS;
+  const int64_t lo = (int64_t)blockIdx.x * CNT_PER, hi = lo + CNT_PER < N ? lo + CNT_PER : N;
+  unsigned long long viol = 0, accs = 0, ont_all = 0;
+  for (int d = 0; d <= D; d++) {
+    const int64_t a0 = devOff[d] > lo ? devOff[d] : lo, a1 = devOff[d + 1] < hi ? devOff[d + 1] : hi;
+    if (a0 >= a1) continue;
+    if (d == D) {  // the sink: dropped (R7)
+      if (threadIdx.x == 0) viol += (unsigned long long)(a1 - a0);
+      continue;
     }
-#pragma unroll
-    for (int k = 0; k < 4; k++) {
-      const int64_t p = p0 + threadIdx.x + (int64_t)k * blockDim.x;
-      if (p >= hi) continue;
-      int dd = d;
-      while (dd < D && sOff[dd + 1] <= p) dd++;
-      if ((int64_t)l[k] > sL[dd]) viol++;
-      else { ont++; accs += sA[dd]; }
+    const LaneParam q = lp[(size_t)s * D + d];
+    const uint32_t L = q.L < 0 ? 0u : q.L > 0xFFFFFFFEll ? 0xFFFFFFFFu : (uint32_t)q.L;
+    const bool all_on = q.L >= 0xFFFFFFFFll;  // every latency (<= UINT32_MAX) is on time
+    unsigned ont = 0;
+    // scalar head up to a 16-byte boundary, uint4 body, scalar tail
+    const int64_t a0r = (a0 + 3) & ~(int64_t)3;  // row starts are 16-byte aligned (NS % 32 == 0)
+    const int64_t b0 = a0r < a1 ? a0r : a1;
+    const int64_t b1 = b0 + ((a1 - b0) & ~(int64_t)3);
+    for (int64_t p = a0 + threadIdx.x; p < b0; p += blockDim.x) ont += all_on || row[p] <= L;
+    for (int64_t p = b0 + 4 * (int64_t)threadIdx.x; p < b1; p += 4 * (int64_t)blockDim.x) {
+      const uint4 v = *(const uint4 *)(row + p);
+      ont += all_on ? 4u : (unsigned)(v.x <= L) + (v.y <= L) + (v.z <= L) + (v.w <= L);
     }
+    for (int64_t p = b1 + threadIdx.x; p < a1; p += blockDim.x) ont += all_on || row[p] <= L;
+    // q.L < 0 cannot happen for a routed device (L = mult * base / 1000 >= 0)
+    ont_all += ont;
+    accs += (unsigned long long)ont * q.A;
+    if (threadIdx.x == 0) viol += (unsigned long long)(a1 - a0);  // minus the on-time ones below
   }
   for (int o = 16; o; o >>= 1) {
     viol += __shfl_xor_sync(0xffffffffu, viol, o);
-    ont += __shfl_xor_sync(0xffffffffu, ont, o);
+    ont_all += __shfl_xor_sync(0xffffffffu, ont_all, o);
     accs += __shfl_xor_sync(0xffffffffu, accs, o);
   }
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (lane == 0) { red[0][w] = viol; red[1][w] = ont; red[2][w] = accs; }
+  if (lane == 0) { red[0][w] = viol; red[1][w] = ont_all; red[2][w] = accs; }
   __syncthreads();
   if (threadIdx.x == 0) {
     unsigned long long v = 0, o2 = 0, a2 = 0;
     for (int k = 0; k < (int)(blockDim.x >> 5); k++) { v += red[0][k]; o2 += red[1][k]; a2 += red[2][k]; }
+    v -= o2;
     if (v) atomicAdd((unsigned long long *)&agg[s], v);
     if (o2) atomicAdd((unsigned long long *)&agg[S + s], o2);
     if (a2) atomicAdd((unsigned long long *)&agg[2 * S + s], a2);
@@ -1074,7 +1467,7 @@ __global__ void k_count(int64_t N, int S, int D, const int32_t *__restrict__ sc_
 // per-query order: out[s][i] = latd[s][inv(i)] (coalesced stores, gathered loads
 // that walk ~D sequential streams)
 #define UNP_PER 16
-__global__ void __launch_bounds__(256) k_unpermute(int64_t N, int S, const proteus_scenario *__restrict__ sc,
+__global__ void __launch_bounds__(256) k_unpermute(int64_t N, int64_t NS, int S, const proteus_scenario *__restrict__ sc,
                                                    const uint32_t *__restrict__ inv0, const uint32_t *__restrict__ inv1,
                                                    const uint32_t *__restrict__ latd, uint32_t *out) {
   // one block per chunk of 256 * UNP_PER queries, all scenario rows: every
@@ -1092,12 +1485,12 @@ __global__ void __launch_bounds__(256) k_unpermute(int64_t N, int S, const prote
     p1[k] = (inv1 && i < N) ? inv1[i] : 0;
   }
   for (int s = 0; s < S; s++) {
-    const size_t r = (size_t)s * N;
+    const size_t r = (size_t)s * N, rs = (size_t)s * NS;
     const bool m1 = rt[s] != 0;
     uint32_t v[UNP_PER];
 #pragma unroll
     for (int k = 0; k < UNP_PER; k++)
-      if (i0 + 256 * k < N) v[k] = latd[r + (m1 ? p1[k] : p0[k])];
+      if (i0 + 256 * k < N) v[k] = latd[rs + (m1 ? p1[k] : p0[k])];
 #pragma unroll
     for (int k = 0; k < UNP_PER; k++)
       if (i0 + 256 * k < N) out[r + i0 + 256 * k] = v[k];
@@ -1122,7 +1515,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   if (!sb) return px_fail(ctx, PROTEUS_ENOMEM, "replay scratch");
   int32_t *d_opt = (int32_t *)sb, *d_z = d_opt + D, *d_dev = d_z + D, *d_dem = d_dev + D, *d_slo = d_dem + Q;
   int32_t *d_pat_off = d_slo + Q, *d_pat_len = d_pat_off + PX_MAXQ;
-  uint32_t *d_flags = (uint32_t *)(d_pat_len + PX_MAXQ);
+  uint32_t *d_flags = (uint32_t *)(d_pat_len + PX_MAXQ);  // [0] trace checks, [4] fix-up changes
   int32_t *d_scl = (int32_t *)(d_flags + 8);              // [2][S] scenario lists per routing mode
   int32_t *d_goff = d_scl + 2 * S;                        // [2][PX_MAXD + 2]
   int64_t *d_choff = (int64_t *)(((uintptr_t)(d_goff + 2 * (PX_MAXD + 2)) + 15) & ~(uintptr_t)15);  // [2][PX_MAXD + 2]
@@ -1164,7 +1557,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     int32_t *hist = (int32_t *)px_buf(ctx, B_R_HIST, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
     int32_t *fbase = (int32_t *)px_buf(ctx, B_R_BASE, (size_t)(ntiles + 1) * (PX_MAXQ + 2) * 4);
     int32_t *dbase = (int32_t *)px_buf(ctx, B_R_DBASE0, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
-    uint8_t *tgt = (uint8_t *)px_buf(ctx, B_R_TGT, (size_t)N + 16);
+    uint8_t *tgt = (uint8_t *)px_buf(ctx, rt ? B_R_TGT1 : B_R_TGT, (size_t)N + 16);
     int64_t *off = (int64_t *)px_buf(ctx, rt ? B_R_OFF1 : B_R_OFF, (size_t)2 * (PX_MAXD + 2) * 8);
     // + whole trailing ring segment: k_stitch bulk-copies 4 KB segments
     uint32_t *darr = (uint32_t *)px_buf(ctx, rt ? B_R_DEVARR1 : B_R_DEVARR, ((size_t)N + 2 * RSEG) * 4);
@@ -1172,7 +1565,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     if (!pat || !hist || !fbase || !dbase || !tgt || !off || !darr || !dinv)
       return px_fail(ctx, PROTEUS_ENOMEM, "routing buffers");
     int64_t *totals = off + (PX_MAXD + 2);
-    PX_LAUNCH(ctx, "route_prepare", k_route_prepare, 1, 32, 0, rt, Q, D, M, ctx->bmax, d_opt, d_z, d_dev, d_dem,
+    PX_LAUNCH(ctx, "route_prepare", k_route_prepare, Q, 32, 0, rt, Q, D, M, ctx->bmax, d_opt, d_z, d_dev, d_dem,
               ctx->d_fam, ctx->d_lat, pat, d_pat_off, d_pat_len);
     if (N > 0) {
       PX_LAUNCH(ctx, "route_count", k_tile_count, tblocks, TILE_WARPS * 32, 0, d_fam, N, Q, hist);
@@ -1190,9 +1583,11 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   }
   if (N == 0) return 0;
   // chunk layout per routing mode (sizes only): the host reads the per-device counts
-  int CH = env_int("PROTEUS_REPLAY_CHUNK", 1024);
-  CH = CH < 1 ? 1 : CH > SPECCAP ? SPECCAP : CH;  // the stitch caches one chunk
+  int CH = env_int("PROTEUS_REPLAY_CHUNK", 4096);
+  CH = CH < 1 ? 1 : CH > (1 << 20) ? (1 << 20) : CH;
   const bool simple = env_int("PROTEUS_REPLAY_SIMPLE", 0) != 0;
+  // fix-up rounds before the sequential stitch finishes whatever is left
+  const int max_rounds = env_int("PROTEUS_REPLAY_ROUNDS", 0);
   int64_t h_off[2][PX_MAXD + 2];
   for (int rt = 0; rt < 2; rt++)
     if (devOff[rt])
@@ -1214,98 +1609,162 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   }
   PX_CUDA(ctx, cudaMemcpyAsync(d_choff, choff.data(), choff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_goff, goff.data(), goff.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
-  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * N * 4 + 64);  // B_R_LAT stages host outputs
+  const int64_t NS = (N + 31) & ~(int64_t)31;  // latd row stride
+  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * NS * 4 + 8192);  // B_R_LAT stages host outputs
   if (!latd) return px_fail(ctx, PROTEUS_ENOMEM, "latency scratch");
-  SpecExit *ex = nullptr;
-  // phase runs (k_spec): lanes with 2 <= Bmax <= rmax also speculate each
-  // chunk from its (r + 1)-th query, r < Bmax, so the true run (which enters
-  // a chunk up to Bmax - 1 queries late) always has a run that starts with it
-  const int rmax = simple ? 1 : env_int("PROTEUS_REPLAY_PHASES", 1);
-  uint32_t *vlat = nullptr;
-  SpecExit *vex = nullptr;
-  int64_t *d_voff = nullptr;
-  int rz = 1;
+  const int64_t nmax = NCH[0] > NCH[1] ? NCH[0] : NCH[1];
+  ChunkSt *csb[2] = {nullptr, nullptr};  // chunk runs, double-buffered across fix-up rounds
+  unsigned *d_changed = d_flags + 4;  // [0] chunk exits changed, [1] lanes left to the stitch
+  unsigned *d_lstat = (unsigned *)px_buf(ctx, B_R_VOFF, (size_t)S * D * 24 + 64);
+  if (!d_lstat) return px_fail(ctx, PROTEUS_ENOMEM, "lane statistics");
+  int64_t *d_lstart = (int64_t *)(((uintptr_t)(d_lstat + 2 * (size_t)S * D) + 15) & ~(uintptr_t)15);
+  PX_CUDA(ctx, cudaMemsetAsync(d_lstat, 0, (size_t)S * D * 8, ctx->stream));
+  PX_CUDA(ctx, cudaMemsetAsync(d_lstart, 0xFF, (size_t)S * D * 16, ctx->stream));  // head -1: not scanned
+  const bool use_bscan = !simple && env_int("PROTEUS_REPLAY_BSCAN", 0) != 0;
   if (!simple) {
-    std::vector<int64_t> voff(2 * (size_t)S * D, 0);
-    int64_t vtot = 0, vxtot = 0;
-    for (int s = 0; s < S; s++) {
-      const int rt = h_sc[s].routing;
-      for (int d = 0; d < D; d++) {
-        int Bmax = 0;
-        if (h_option[d] > 0) {
-          const int32_t *Tr = ctx->lat.data() + ((size_t)h_dev_type[d] * M + (h_option[d] - 1)) * ctx->bmax;
-          int depth = 0;
-          while (depth < ctx->bmax && Tr[depth] > 0) depth++;
-          const int cap = h_sc[s].batch_cap;
-          Bmax = (cap > 0 && cap < depth) ? cap : depth;  // as k_lane_params
-        }
-        const int R = n_phase_runs(Bmax, rmax);
-        const int64_t nd = h_off[rt][d + 1] - h_off[rt][d], nchd = (nd + CH - 1) / CH;
-        voff[(size_t)s * D + d] = vtot;
-        voff[(size_t)S * D + (size_t)s * D + d] = vxtot;
-        vtot += (int64_t)(R - 1) * nd;
-        vxtot += (int64_t)(R - 1) * nchd;
-        if (R > rz && nchd > 1) rz = R;
-      }
-    }
-    if (rz > 1) {
-      vlat = (uint32_t *)px_buf(ctx, B_R_VLAT, (size_t)vtot * 4 + 16);
-      vex = (SpecExit *)px_buf(ctx, B_R_VEX, sizeof(SpecExit) * (size_t)(vxtot + 1));
-      d_voff = (int64_t *)px_buf(ctx, B_R_VOFF, voff.size() * 8);
-      if (!vlat || !vex || !d_voff) return px_fail(ctx, PROTEUS_ENOMEM, "phase-run buffers");
-      PX_CUDA(ctx, cudaMemcpyAsync(d_voff, voff.data(), voff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
-    }
-    const int64_t nmax = NCH[0] > NCH[1] ? NCH[0] : NCH[1];
-    ex = (SpecExit *)px_buf(ctx, B_R_LANE, sizeof(SpecExit) * (size_t)S * (nmax + 1));
-    if (!ex) return px_fail(ctx, PROTEUS_ENOMEM, "speculation states");
+    csb[0] = (ChunkSt *)px_buf(ctx, B_R_LANE, sizeof(ChunkSt) * (size_t)S * (nmax + 1));
+    csb[1] = (ChunkSt *)px_buf(ctx, B_R_VEX, sizeof(ChunkSt) * (size_t)S * (nmax + 1));
+    if (!csb[0] || !csb[1]) return px_fail(ctx, PROTEUS_ENOMEM, "chunk states");
     PX_CUDA(ctx, cudaFuncSetAttribute(k_stitch, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)stitch_smem(ctx->bmax)));
   }
+  // Bmax per (scenario, device), as k_lane_params (R4)
+  std::vector<int32_t> hB((size_t)S * D, 0), hT1(D, 0);
+  for (int d = 0; d < D; d++) {
+    if (h_option[d] <= 0) continue;
+    const int32_t *Tr = ctx->lat.data() + ((size_t)h_dev_type[d] * M + (h_option[d] - 1)) * ctx->bmax;
+    int depth = 0;
+    while (depth < ctx->bmax && Tr[depth] > 0) depth++;
+    hT1[d] = Tr[0];
+    for (int s = 0; s < S; s++) {
+      const int cap = h_sc[s].batch_cap;
+      hB[(size_t)s * D + d] = (cap > 0 && cap < depth) ? cap : depth;
+    }
+  }
+  const bool use_scan1 = !simple && env_int("PROTEUS_REPLAY_SCAN1", 1) != 0;
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
     LaneArgs la;
     memset(&la, 0, sizeof la);
     la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.nsc = (int)scl[rt].size(); la.CH = CH;
-    la.N = N; la.NCH = NCH[0] > NCH[1] ? NCH[0] : NCH[1];  // one row stride for both routing modes
+    la.N = N; la.NS = NS; la.NCH = nmax;  // one row stride for both routing modes
     la.option = d_opt; la.dev_type = d_dev; la.lat = ctx->d_lat; la.sc_list = d_scl + rt * S; la.lp = d_lp;
     la.devOff = devOff[rt]; la.choff = d_choff + rt * (PX_MAXD + 2); la.goff = d_goff + rt * (PX_MAXD + 2);
-    la.devArr = devArr[rt]; la.latd = latd; la.ex = ex; la.agg = d_agg;
+    la.devArr = devArr[rt]; la.latd = latd; la.cs = csb[0]; la.csp = nullptr; la.agg = d_agg;
     la.debug = env_int("PROTEUS_REPLAY_DEBUG", 0);
     la.maxchk = env_int("PROTEUS_REPLAY_CHECKS", 1 << 30);
-    la.rmax = rz > 1 ? rmax : 1;
-    la.vlat = vlat; la.vex = vex; la.voff = d_voff;
+    la.scan1 = use_scan1 ? 1 : 0;
+    la.lstat = d_lstat;
+    la.lstart = d_lstart;
+    if (use_scan1) {  // Bmax = 1 lanes: exact prefix-maximum scan
+      Scan1Args sa;
+      memset(&sa, 0, sizeof sa);
+      sa.D = D; sa.nsc = la.nsc; sa.N = N; sa.NS = NS;
+      std::vector<int32_t> t1(D, 0);
+      int64_t nb = 0;
+      for (int d = 0; d < D; d++) {
+        sa.boff[d] = nb;
+        bool any = false;
+        for (int k : scl[rt]) any |= hB[(size_t)k * D + d] == 1;
+        if (!any) continue;
+        t1[d] = hT1[d];
+        nb += (h_off[rt][d + 1] - h_off[rt][d] + SCAN_BLK - 1) / SCAN_BLK;
+      }
+      sa.boff[D] = nb;
+      if (nb > 0) {
+        char *sb2 = (char *)px_buf(ctx, B_R_SCAN, (size_t)nb * 16 + (size_t)D * 4 + 64);
+        if (!sb2) return px_fail(ctx, PROTEUS_ENOMEM, "scan buffers");
+        sa.bmx = (int64_t *)sb2;
+        sa.bpre = sa.bmx + nb;
+        int32_t *d_t1 = (int32_t *)(sa.bpre + nb);
+        PX_CUDA(ctx, cudaMemcpyAsync(d_t1, t1.data(), D * 4, cudaMemcpyHostToDevice, ctx->stream));
+        sa.T1 = d_t1; sa.devOff = devOff[rt]; sa.devArr = devArr[rt]; sa.sc_list = d_scl + rt * S; sa.lp = d_lp;
+        sa.latd = latd;
+        if (nb > 0x7fffffff) return px_fail(ctx, PROTEUS_ERANGE, "scan blocks");
+        PX_LAUNCH(ctx, "replay_scan1", k_scan1_reduce, (unsigned)nb, 256, 0, sa);
+        PX_LAUNCH(ctx, "replay_scan1", k_scan1_prefix, D, 32, 0, sa);
+        PX_LAUNCH(ctx, "replay_scan1", k_scan1_apply, (unsigned)nb, 256, 0, sa);
+      }
+    }
     if (simple) {
       const int nl = la.nsc * D;
       PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
-    } else {
-      if (ngroups[rt] > 0) {
-        if ((ngroups[rt] + 3) / 4 > 65535) return px_fail(ctx, PROTEUS_ERANGE, "too many replay chunks");
-        dim3 grid((unsigned)la.nsc, (unsigned)((ngroups[rt] + 3) / 4));
-        PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la, 0);
-        if (rz > 1) {
-          dim3 gv(grid.x, grid.y, (unsigned)(rz - 1));
-          PX_LAUNCH(ctx, "replay_spec_phase", k_spec, gv, 128, 0, la, 1);
+    } else if (ngroups[rt] > 0) {
+      if ((ngroups[rt] + 3) / 4 > 65535 || (NCH[rt] + 3) / 4 > 65535)
+        return px_fail(ctx, PROTEUS_ERANGE, "too many replay chunks");
+      dim3 grid((unsigned)la.nsc, (unsigned)((ngroups[rt] + 3) / 4));
+      PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la);
+      // backlogged lanes (k_spec's statistics): full-batch prefix-maximum scan
+      if (use_bscan) {
+        std::vector<int32_t> lid;
+        std::vector<int64_t> loff(1, 0);
+        for (int k : scl[rt])
+          for (int d = 0; d < D; d++) {
+            const int B = hB[(size_t)k * D + d];
+            const int64_t nd = h_off[rt][d + 1] - h_off[rt][d];
+            if (B < 2 || nd < B) continue;
+            lid.push_back(k * D + d);
+            loff.push_back(loff.back() + (nd / B + BSCAN_BLK - 1) / BSCAN_BLK);
+          }
+        const int nl = (int)lid.size();
+        const int64_t nb = loff.back();
+        if (nl > 0 && nb > 0) {
+          if (nb > 0x7fffffff) return px_fail(ctx, PROTEUS_ERANGE, "scan blocks");
+          char *bb = (char *)px_buf(ctx, B_R_BSCAN, (size_t)(nl + 1) * 8 + (size_t)nl * 4 + (size_t)nb * 16 +
+                                                        (size_t)nl * 8 + 256);
+          if (!bb) return px_fail(ctx, PROTEUS_ENOMEM, "scan buffers");
+          BScanArgs ba;
+          memset(&ba, 0, sizeof ba);
+          int64_t *d_loff = (int64_t *)bb;
+          ba.bmx = d_loff + (nl + 1);
+          ba.bpre = ba.bmx + nb;
+          ba.vio = (unsigned long long *)(ba.bpre + nb);
+          int32_t *d_lid = (int32_t *)(ba.vio + nl);
+          PX_CUDA(ctx, cudaMemcpyAsync(d_loff, loff.data(), loff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
+          PX_CUDA(ctx, cudaMemcpyAsync(d_lid, lid.data(), lid.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+          PX_CUDA(ctx, cudaMemsetAsync(ba.vio, 0xFF, (size_t)nl * 8, ctx->stream));
+          ba.D = D; ba.nl = nl; ba.NS = NS; ba.loff = d_loff; ba.lid = d_lid; ba.devOff = devOff[rt];
+          ba.devArr = devArr[rt]; ba.lat = ctx->d_lat; ba.option = d_opt; ba.dev_type = d_dev; ba.M = M;
+          ba.bmax = ctx->bmax; ba.lp = d_lp; ba.lstat = d_lstat; ba.latd = latd; ba.lstart = d_lstart;
+          PX_LAUNCH(ctx, "replay_bscan", k_bscan_reduce, (unsigned)nb, 256, 0, ba);
+          PX_LAUNCH(ctx, "replay_bscan", k_bscan_prefix, nl, 32, 0, ba);
+          PX_LAUNCH(ctx, "replay_bscan", k_bscan_verify, (unsigned)nb, 256, 0, ba);
+          PX_LAUNCH(ctx, "replay_bscan", k_bscan_apply, (unsigned)nb, 256, 0, ba);
         }
       }
-      const int64_t warps = (int64_t)la.nsc * D;
-      PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128,
-                stitch_smem(ctx->bmax), la);
+      // fix-up rounds until no chunk exit changes (then every chunk is exact)
+      int cur = 0;
+      bool done = false;
+      for (int r = 1; r <= max_rounds; r++) {
+        la.csp = csb[cur];
+        la.cs = csb[cur ^ 1];
+        PX_CUDA(ctx, cudaMemsetAsync(d_changed, 0, 8, ctx->stream));
+        dim3 gf((unsigned)la.nsc, (unsigned)((NCH[rt] + 3) / 4));
+        PX_LAUNCH(ctx, "replay_fix", k_fix, gf, 128, 0, la, d_changed);
+        cur ^= 1;
+        unsigned changed[2] = {0, 0};
+        PX_CUDA(ctx, cudaMemcpyAsync(changed, d_changed, 8, cudaMemcpyDeviceToHost, ctx->stream));
+        PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+        if (la.debug) fprintf(stderr, "replay routing %d fix-up round %d: %u chunk exits changed\n", rt, r, changed[0]);
+        if (changed[0] == 0) { done = changed[1] == 0; break; }
+      }
+      la.cs = csb[cur];
+      la.csp = nullptr;
+      if (!done) {  // the sequential stitch carries the true state through the rest
+        const int64_t warps = (int64_t)la.nsc * D;
+        PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, stitch_smem(ctx->bmax), la);
+      }
     }
     dim3 g(32, la.nsc < 65535 ? la.nsc : 65535);
-    PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, N, S, D, d_scl + rt * S, la.nsc, devOff[rt], latd, d_agg);
-    int nsm = 0;
-    PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
-    int64_t cbx = (N + 4095) / 4096;
-    const int64_t cap_bx = ((int64_t)nsm * 64 + la.nsc - 1) / la.nsc;
-    if (cbx > cap_bx) cbx = cap_bx > 0 ? cap_bx : 1;
-    dim3 cg((unsigned)cbx, (unsigned)la.nsc);
-    PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, S, D, d_scl + rt * S, devOff[rt], d_lp, latd, d_agg);
+    PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, NS, S, D, d_scl + rt * S, la.nsc, devOff[rt], latd, d_agg);
+    dim3 cg((unsigned)((N + CNT_PER - 1) / CNT_PER), (unsigned)la.nsc);
+    PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, NS, S, D, d_scl + rt * S, devOff[rt], d_lp, latd, d_agg);
   }
   if (d_lat_out) {
     int nsm = 0;
     PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
     const int64_t nb = (N + 256 * UNP_PER - 1) / (256 * UNP_PER);
-    PX_LAUNCH(ctx, "replay_unpermute", k_unpermute, (unsigned)nb, 256, 0, N, S, d_sc, inv[0], inv[1], latd, d_lat_out);
+    PX_LAUNCH(ctx, "replay_unpermute", k_unpermute, (unsigned)nb, 256, 0, N, NS, S, d_sc, inv[0], inv[1], latd, d_lat_out);
   }
   return 0;
 }

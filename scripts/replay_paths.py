@@ -13,10 +13,9 @@ arr = torch.from_numpy(cfg["arrival_us"]).cuda(); fam = torch.from_numpy(cfg["fa
 sc = cfg["scenarios"]
 lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
 px.set_timing(True)
-KEYS = ("PROTEUS_REPLAY_SIMPLE", "PROTEUS_REPLAY_CHUNK", "PROTEUS_REPLAY_CHECKS", "PROTEUS_REPLAY_PHASES", "PROTEUS_REPLAY_DEBUG")
-variants = [{}, {"PROTEUS_REPLAY_PHASES": "4"}]
-variants += [{"PROTEUS_REPLAY_CHUNK": str(c)} for c in (256, 512)]
-
+KEYS = ("PROTEUS_REPLAY_SIMPLE", "PROTEUS_REPLAY_CHUNK", "PROTEUS_REPLAY_CHECKS", "PROTEUS_REPLAY_ROUNDS", "PROTEUS_REPLAY_DEBUG", "PROTEUS_REPLAY_SCAN1")
+variants = [{}, {"PROTEUS_REPLAY_ROUNDS": "2"}, {"PROTEUS_REPLAY_ROUNDS": "0"}, {"PROTEUS_REPLAY_SCAN1": "0"}]
+variants += [{"PROTEUS_REPLAY_CHUNK": str(c)} for c in (1024, 16384)]
 variants += [eval(v) for v in sys.argv[1:]]
 ref = None
 for env in variants:
@@ -26,7 +25,12 @@ for env in variants:
         torch.cuda.synchronize(); t0 = time.perf_counter()
         r = px.replay(arr, fam, a.option, a.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
         torch.cuda.synchronize(); t1 = time.perf_counter()
-    kt = {n: round(ms, 2) for n, ms in px.kernel_times() if n.startswith("replay")}
+    kt = {}
+    for n, ms in px.kernel_times():
+        if n.startswith("replay"):
+            kt[n] = round(kt.get(n, 0) + ms, 2)
+    nfix = sum(1 for n, _ in px.kernel_times() if n == "replay_fix")
+    kt["fix_rounds"] = nfix
     h = int(torch.sum(lat.view(torch.int32).to(torch.int64) * 2654435761 % 1000003).item())
     if ref is None: ref = h
     print(env, f"{(t1-t0)*1e3:.1f} ms", kt, int(r["violations"].sum()), "same" if h == ref else "DIFFERENT", flush=True)

@@ -26,6 +26,9 @@ def main():
     sc = np.array([[1000, 1, 0], [2000, 4, 0], [3500, 0, 0], [1500, 0, 1]], np.int32)
     os.environ["PROTEUS_REPLAY_CHUNK"] = "16"
     px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
+    os.environ["PROTEUS_REPLAY_ROUNDS"] = "1"  # one fix-up round, then the stitch
+    px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
+    os.environ.pop("PROTEUS_REPLAY_ROUNDS")
     os.environ["PROTEUS_REPLAY_SIMPLE"] = "1"
     px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
     print("sanitize target done")

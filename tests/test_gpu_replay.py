@@ -33,8 +33,13 @@ def _compare(px, oracle_mod, prof, cl, option, z, demand, arr, fam, sc):
 
 
 PATHS = {"chunked": {}, "small_chunks": {"PROTEUS_REPLAY_CHUNK": "16"}, "odd_chunks": {"PROTEUS_REPLAY_CHUNK": "37"},
-         "phase_runs": {"PROTEUS_REPLAY_PHASES": "8", "PROTEUS_REPLAY_CHUNK": "37"},
-         "all_phase_runs": {"PROTEUS_REPLAY_PHASES": "64", "PROTEUS_REPLAY_CHUNK": "100"},
+         "stitch_only": {"PROTEUS_REPLAY_ROUNDS": "0", "PROTEUS_REPLAY_CHUNK": "37"},
+         "one_round_then_stitch": {"PROTEUS_REPLAY_ROUNDS": "1", "PROTEUS_REPLAY_CHUNK": "100"},
+         "rounds_to_convergence": {"PROTEUS_REPLAY_ROUNDS": "1000000", "PROTEUS_REPLAY_CHUNK": "64"},
+         "no_scans": {"PROTEUS_REPLAY_SCAN1": "0", "PROTEUS_REPLAY_BSCAN": "0", "PROTEUS_REPLAY_CHUNK": "512"},
+         "scans_small_chunks_rounds": {"PROTEUS_REPLAY_ROUNDS": "3", "PROTEUS_REPLAY_CHUNK": "200",
+                                       "PROTEUS_REPLAY_BSCAN": "1"},
+         "backlog_scan": {"PROTEUS_REPLAY_BSCAN": "1"},
          "simple": {"PROTEUS_REPLAY_SIMPLE": "1"}}
 
 
@@ -42,9 +47,11 @@ PATHS = {"chunked": {}, "small_chunks": {"PROTEUS_REPLAY_CHUNK": "16"}, "odd_chu
 @pytest.mark.parametrize("kind", ["poisson", "gamma", "uniform"])
 def test_replay_small_all_scenarios(px, oracle_mod, kind, path, monkeypatch):
     """60k queries x 64 scenarios x both routings; `small_chunks` /
-    `odd_chunks` cut the device arrays every 16 / 37 queries so the stitch
-    (backlogged jumps, re-walks, meeting tests) runs at every chunk; `simple`
-    is one thread per (device, scenario) lane."""
+    `odd_chunks` cut the device arrays every 16 / 37 queries so the fix-up
+    rounds and the stitch (backlogged jumps, re-walks, meeting tests) run at
+    every chunk; `stitch_only` / `one_round_then_stitch` /
+    `rounds_to_convergence` take each finishing path alone; `simple` is one
+    thread per (device, scenario) lane."""
     for k, v in PATHS[path].items():
         monkeypatch.setenv(k, v)
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
@@ -119,3 +126,19 @@ def test_replay_c5_full_size(px, oracle_mod):
         assert np.array_equal(g[k], o[k]), k
     glat = lat.cpu().numpy()
     assert np.array_equal(glat, o["latency"])
+
+
+def test_replay_aggregates_without_latencies(px, oracle_mod):
+    """latency=None (aggregates only: the separate count pass) equals the
+    oracle's aggregates, as the fused count in the un-permute pass does."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    r = _alloc(oracle_mod, cfg, 1)
+    arr, fam = W.query_trace(50_000, float(cfg["demand"][1].sum()), cfg["weights"], 12, "gamma")
+    sc = np.concatenate([W.scenarios_64(0)[::3], W.scenarios_64(1)[::5]])
+    px.load_profiles(prof)
+    g = px.replay(arr, fam, r["option"], r["z"], cl.device_type, cfg["demand"][1], cl.slo_us, sc, latency=None)
+    o = oracle_mod.replay(prof, cl.device_type, r["option"], r["z"], cfg["demand"][1], cl.slo_us, arr, fam, sc)
+    for k in ("violations", "on_time", "acc_sum"):
+        assert np.array_equal(g[k], o[k]), k
