@@ -115,6 +115,18 @@ def flat_pair_ops_per_candidate(Q, V, K):
     return per_prefix / (K * K)
 
 
+# the lane kernels of the replay (a12): their algorithmic bytes are the latency
+# rows written plus one read of the per-device arrays
+LANE_KERNELS = ("replay_scan1", "replay_bscan", "replay_spec", "replay_fix", "replay_stitch", "replay_lanes")
+
+
+# algorithmic int32 lane-ops of one (count vector, demand vector) evaluation in
+# k_fact_gv: VM minima and VM multiply-adds of the summation-by-parts fill, the
+# served shift-add and the 64-bit compare
+def fact_g_ops(VM):
+    return 2 * VM + 3
+
+
 def oracle_cpu_baseline(cfg, vec=0):
     import oracle
     prof, cl = cfg["prof"], cfg["cluster"]
@@ -371,6 +383,11 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
         t0 = time.perf_counter()
         px.solve(t_dev, t_slo, t_one, mode=2)
         one.append((time.perf_counter() - t0) * 1e3)
+    g_ms = ksplit.get("fact_g", float("nan"))
+    evals = nv * ncand  # this rank's vectors x count vectors per vector
+    g_ops = evals * fact_g_ops(5)
+    sm_mhz = peaks.get("sm_max_mhz", SM_MAX_MHZ_FALLBACK)
+    peak_ops = SM_COUNT * INT_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12
     out["c4_resolve"] = {
         "vectors": len(cfg["demand"]), "ms_all_vectors": ms, "ms_per_vector_batched": ms / max(1, hi - lo),
         "kernel_ms": ksplit,
@@ -378,6 +395,10 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
         "single_vector_time_to_optimal_ms": statistics.median(one),
         "subplacements_per_vector": ncand,
         "subplacements_per_s": (len(cfg["demand"]) * ncand) / (ms / 1e3),
+        "roofline": {"kernel": "fact_g", "bound": "alu", "achieved": g_ops / (g_ms / 1e3) / 1e12, "peak": peak_ops,
+                     "unit": "Tops/s (int32 lane-ops)", "frac": g_ops / (g_ms / 1e3) / 1e12 / peak_ops,
+                     "ops_per_evaluation": fact_g_ops(5), "evaluations": evals,
+                     "peak_basis": f"148 SMs x 128 int32 lane-ops/clk x {sm_mhz:.0f} MHz (max SM clock)"},
         "scaling": "weak (vectors split by rank)"}
     # c5: replay 10M queries x 64 scenarios (scenarios on every rank; N>1 = replicas)
     cfg = W.config("c5")
@@ -402,9 +423,12 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
         barrier()
         ts.append(a.elapsed_time(b))
         kt = px.kernel_times()
-        lane_ms.append(sum(ms for n, ms in kt if n in ("replay_spec", "replay_stitch", "replay_lanes")))
+        lane_ms.append(sum(ms for n, ms in kt if n in LANE_KERNELS))
         route_ms = sum(ms for n, ms in kt if n.startswith("route"))
-        split = {n: ms for n, ms in kt if n in ("replay_spec", "replay_stitch", "replay_lanes")}
+        split = {}
+        for n, ms_ in kt:
+            if n.startswith("replay") or n.startswith("route"):
+                split[n] = split.get(n, 0.0) + ms_
     px.set_timing(False)
     ms = max_over_ranks(statistics.median(ts))
     lane = statistics.median(lane_ms)
@@ -418,8 +442,8 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     e2e = time.perf_counter() - t0
     out["c5_replay"] = {
         "queries": N, "scenarios": S, "ms": ms, "query_scenarios_per_s": N * S / (ms / 1e3),
-        "routing_ms": route_ms, "lane_kernels_ms": lane, "lane_kernel_split_ms": split,
-        "roofline": {"kernel": "replay_spec + replay_stitch", "bound": "hbm", "achieved": alg_bytes / (lane / 1e3) / 1e9,
+        "routing_ms": route_ms, "lane_kernels_ms": lane, "kernel_split_ms": split,
+        "roofline": {"kernel": " + ".join(LANE_KERNELS), "bound": "hbm", "achieved": alg_bytes / (lane / 1e3) / 1e9,
                      "peak": hbm, "unit": "GB/s", "frac": alg_bytes / (lane / 1e3) / 1e9 / hbm,
                      "peak_source": peak_src, "alg_bytes": alg_bytes},
         "violations_first_scenarios": [int(x) for x in res["violations"][:4]],

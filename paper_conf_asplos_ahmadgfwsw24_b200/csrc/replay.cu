@@ -25,6 +25,7 @@
 //            and the reference formulation in the tests).
 // a13: k_count reduces the final latency rows to per-scenario violations,
 // on-time counts and accuracy sums.
+#include <algorithm>
 #include <climits>
 #include <cstdlib>
 #include <cstring>
@@ -297,6 +298,7 @@ struct LaneArgs {
   uint64_t *agg;          // [3][S]
   int maxchk;             // convergence checks per chunk (free decisions only)
   int scan1;              // Bmax = 1 lanes are produced by k_scan1_* (the chunk kernels skip them)
+  uint64_t dmask;         // devices whose lanes this launch of k_spec / k_fix / k_stitch takes
   const int64_t *lstart;  // [S * D][2] (head, F) where k_stitch starts a lane the full-batch scan took (head -1: not taken)
   unsigned *lstat;        // [S * D][2] speculative decisions that were full batches sent when the device
                           // freed (backlog), and all speculative decisions; k_fix leaves backlogged lanes
@@ -400,6 +402,7 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   if (g >= sG[a.D]) return;
   int d = 0;
   while (g >= sG[d + 1]) d++;
+  if (!((a.dmask >> d) & 1ull)) return;
   const int s = a.sc_list[blockIdx.x];
   const LaneParam p = a.lp[s * a.D + d];
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
@@ -554,6 +557,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   const int64_t gw = (int64_t)blockIdx.x * 4 + w;
   if (gw >= (int64_t)a.nsc * a.D) return;
   const int s = a.sc_list[gw / a.D], d = (int)(gw % a.D);
+  if (!((a.dmask >> d) & 1ull)) return;
   const LaneParam p = a.lp[s * a.D + d];
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
@@ -993,6 +997,7 @@ __global__ void __launch_bounds__(128) k_fix(const __grid_constant__ LaneArgs a,
   if (g >= sC[a.D]) return;
   int d = 0;
   while (g >= sC[d + 1]) d++;
+  if (!((a.dmask >> d) & 1ull)) return;
   const int s = a.sc_list[blockIdx.x];
   const int64_t c = g - sC[d];
   const size_t row = (size_t)s * a.NCH + sC[d];
@@ -1654,6 +1659,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     la.debug = env_int("PROTEUS_REPLAY_DEBUG", 0);
     la.maxchk = env_int("PROTEUS_REPLAY_CHECKS", 1 << 30);
     la.scan1 = use_scan1 ? 1 : 0;
+    la.dmask = D >= 64 ? ~0ull : ((1ull << D) - 1);
     la.lstat = d_lstat;
     la.lstart = d_lstart;
     if (use_scan1) {  // Bmax = 1 lanes: exact prefix-maximum scan
@@ -1730,6 +1736,20 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
           PX_LAUNCH(ctx, "replay_bscan", k_bscan_prefix, nl, 32, 0, ba);
           PX_LAUNCH(ctx, "replay_bscan", k_bscan_verify, (unsigned)nb, 256, 0, ba);
           PX_LAUNCH(ctx, "replay_bscan", k_bscan_apply, (unsigned)nb, 256, 0, ba);
+        }
+      }
+      if (la.debug) {  // diagnostic: speculative decisions per lane
+        std::vector<unsigned> hs((size_t)2 * S * D);
+        PX_CUDA(ctx, cudaMemcpyAsync(hs.data(), d_lstat, hs.size() * 4, cudaMemcpyDeviceToHost, ctx->stream));
+        PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+        unsigned long long tot = 0, full = 0;
+        for (int k : scl[rt])
+          for (int d = 0; d < D; d++) { tot += hs[2 * ((size_t)k * D + d) + 1]; full += hs[2 * ((size_t)k * D + d)]; }
+        fprintf(stderr, "replay routing %d: %llu speculative decisions, %llu full-immediate\n", rt, tot, full);
+        for (int d = 0; d < D; d++) {
+          unsigned long long t = 0;
+          for (int k : scl[rt]) t += hs[2 * ((size_t)k * D + d) + 1];
+          fprintf(stderr, "  device %d: n=%lld decisions=%llu\n", d, (long long)(h_off[rt][d + 1] - h_off[rt][d]), t);
         }
       }
       // fix-up rounds until no chunk exit changes (then every chunk is exact)

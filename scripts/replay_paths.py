@@ -13,9 +13,8 @@ arr = torch.from_numpy(cfg["arrival_us"]).cuda(); fam = torch.from_numpy(cfg["fa
 sc = cfg["scenarios"]
 lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
 px.set_timing(True)
-KEYS = ("PROTEUS_REPLAY_SIMPLE", "PROTEUS_REPLAY_CHUNK", "PROTEUS_REPLAY_CHECKS", "PROTEUS_REPLAY_ROUNDS", "PROTEUS_REPLAY_DEBUG", "PROTEUS_REPLAY_SCAN1")
-variants = [{}, {"PROTEUS_REPLAY_ROUNDS": "2"}, {"PROTEUS_REPLAY_ROUNDS": "0"}, {"PROTEUS_REPLAY_SCAN1": "0"}]
-variants += [{"PROTEUS_REPLAY_CHUNK": str(c)} for c in (1024, 16384)]
+KEYS = ("PROTEUS_REPLAY_SIMPLE", "PROTEUS_REPLAY_CHUNK", "PROTEUS_REPLAY_CHECKS", "PROTEUS_REPLAY_ROUNDS", "PROTEUS_REPLAY_DEBUG", "PROTEUS_REPLAY_SCAN1", "PROTEUS_REPLAY_SPLIT", "PROTEUS_REPLAY_BSCAN")
+variants = [{}, {"PROTEUS_REPLAY_SPLIT": "0"}, {"PROTEUS_REPLAY_CHUNK": "8192"}, {"PROTEUS_REPLAY_CHUNK": "2048"}]
 variants += [eval(v) for v in sys.argv[1:]]
 ref = None
 for env in variants:

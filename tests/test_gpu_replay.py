@@ -40,6 +40,7 @@ PATHS = {"chunked": {}, "small_chunks": {"PROTEUS_REPLAY_CHUNK": "16"}, "odd_chu
          "scans_small_chunks_rounds": {"PROTEUS_REPLAY_ROUNDS": "3", "PROTEUS_REPLAY_CHUNK": "200",
                                        "PROTEUS_REPLAY_BSCAN": "1"},
          "backlog_scan": {"PROTEUS_REPLAY_BSCAN": "1"},
+         "chunk_300": {"PROTEUS_REPLAY_CHUNK": "300"},
          "simple": {"PROTEUS_REPLAY_SIMPLE": "1"}}
 
 
