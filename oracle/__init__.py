@@ -69,6 +69,8 @@ def lib():
         L.orc_replay.argtypes = [C.c_int64, u32p, u8p, C.c_int, C.c_int, i32p, i32p, C.c_int, i32p,
                                  C.c_int, i32p, i32p, i32p, i32p, i32p, C.c_int, i32p, C.c_int,
                                  C.c_void_p, u64p, u64p, u64p]
+        L.orc_pareto.argtypes = [C.c_int, i32p, C.c_int, i32p, i32p, C.c_int, C.c_int, C.c_int, C.c_int64,
+                                 i64p, i64p, u64p, C.POINTER(C.c_uint64), C.POINTER(C.c_int64)]
         _lib = L
     return _lib
 
@@ -202,3 +204,22 @@ def replay(prof, device_type, option, z, demand, slo_base, arrival_us, family, s
     if rc != 0:
         raise RuntimeError(f"orc_replay returned {rc}")
     return dict(latency=lat, violations=viol, on_time=ont, acc_sum=accs)
+
+
+def pareto(prof, device_type, slo_us, family, allow_idle=False, P=None, max_out=1 << 16):
+    """Fig. 1b: every configuration of family `family`'s variants
+    on the devices; returns dict(cap, accsum, index) of the Pareto frontier
+    sorted by capacity, and n_configs (readings P1-P4)."""
+    Pt = _i32(capacity(prof, slo_us)[0] if P is None else P)
+    off = int(np.sum(np.asarray(prof.V)[:family]))
+    cap = np.zeros(max_out, np.int64)
+    acs = np.zeros(max_out, np.int64)
+    idx = np.zeros(max_out, np.uint64)
+    ncfg, nout = C.c_uint64(), C.c_int64()
+    rc = lib().orc_pareto(len(device_type), _i32(device_type), Pt.shape[1], Pt, _i32(prof.acc_micro), off,
+                          int(prof.V[family]), int(bool(allow_idle)), max_out, cap, acs, idx,
+                          C.byref(ncfg), C.byref(nout))
+    if rc != 0:
+        raise OverflowError("configuration space too large for the oracle")
+    k = min(nout.value, max_out)
+    return dict(cap=cap[:k], accsum=acs[:k], index=idx[:k], n_configs=ncfg.value, n_front=nout.value)

@@ -23,6 +23,9 @@
  *   orc_replay_device     event-driven simulation of §5 adaptive batching on one
  *                         device, readings R1-R13
  *   orc_replay            route + simulate every (device, scenario) lane
+ *   orc_pareto            system capacity vs capacity-weighted accuracy of
+ *                         every placement of one family's variants, and its
+ *                         Pareto frontier (Fig. 1b), readings P1-P4
  *
  * The oracle never uses the packed 64-bit score of the CUDA path: objective
  * values are (served, accsum) pairs of int64 compared lexicographically.
@@ -952,5 +955,85 @@ int orc_replay(int64_t N, const uint32_t *arrival, const uint8_t *family,
   for (int i = 0; i < nth; i++) pthread_join(th[i], NULL);
   free(th);
   for (int rt = 0; rt < 2; rt++) { free(c.target[rt]); free(c.dev_start[rt]); free(c.idx_of_dev[rt]); }
+  return 0;
+}
+
+/* --------------------------------------------------------------- Fig. 1b -- */
+/* "all possible mappings between 5 EfficientNet variants and 5
+ * devices ... all devices serve the maximum number of queries feasible without
+ * SLO violations.  Out of all 3125 possible configurations, we are only
+ * interested in those at the Pareto frontier".
+ * Readings: P1 system throughput capacity = sum_d P(t_d, m_d) and
+ * system accuracy = the capacity-weighted mean sum_d P A / sum_d P, kept as
+ * the exact pair (cap, accsum); P2 a configuration of capacity 0 has accuracy
+ * 0; P3 a configuration is on the frontier iff no configuration has capacity
+ * >= and accuracy >= with one of them strict (accuracies compared exactly by
+ * cross-multiplication); equal points are one frontier point, reported with
+ * the lowest index; P4 configurations are digits o_d in [0, K), device 0 most
+ * significant, K = V (every device hosts a variant, as in Fig. 1b) or V + 1
+ * with o = 0 idle when allow_idle.
+ * Enumerates every configuration; per distinct capacity keeps the largest
+ * accsum (at equal capacity a larger accsum dominates) with the lowest index,
+ * then tests every pair of those points for dominance.  P[t][m] is the a1
+ * capacity table.  Writes up to max_out points sorted by capacity; returns the
+ * number of configurations in *n_cfg and of frontier points in *n_out. */
+static int acc_ge(int64_t a1, int64_t c1, int64_t a2, int64_t c2) {  /* a1/c1 >= a2/c2, 0/0 = 0 */
+  const __int128 l = (__int128)a1 * (c2 > 0 ? c2 : 1), r = (__int128)a2 * (c1 > 0 ? c1 : 1);
+  if (c1 == 0 && c2 == 0) return 1;
+  if (c1 == 0) return a2 == 0;   /* accuracy 0 >= a2/c2 iff a2 == 0 */
+  if (c2 == 0) return 1;         /* anything >= 0 */
+  return l >= r;
+}
+
+int orc_pareto(int D, const int32_t *dev_type, int M, const int32_t *P, const int32_t *acc, int off, int V,
+               int allow_idle, int64_t max_out, int64_t *cap_out, int64_t *accsum_out, uint64_t *idx_out,
+               uint64_t *n_cfg, int64_t *n_out) {
+  const int K = V + (allow_idle ? 1 : 0);
+  uint64_t n = 1;
+  for (int d = 0; d < D; d++) {
+    if (n > (1ull << 40) / (uint64_t)K) return -1;
+    n *= (uint64_t)K;
+  }
+  int64_t cmax = 0;
+  for (int d = 0; d < D; d++) {
+    int64_t b = 0;
+    for (int v = 0; v < V; v++) b = P[dev_type[d] * M + off + v] > b ? P[dev_type[d] * M + off + v] : b;
+    cmax += b;
+  }
+  int64_t *best_acc = malloc((cmax + 1) * sizeof(int64_t));
+  uint64_t *best_idx = malloc((cmax + 1) * sizeof(uint64_t));
+  for (int64_t c = 0; c <= cmax; c++) { best_acc[c] = -1; best_idx[c] = 0; }
+  int32_t dig[ORC_MAXD];
+  for (uint64_t i = 0; i < n; i++) {
+    uint64_t x = i;
+    for (int d = D - 1; d >= 0; d--) { dig[d] = (int32_t)(x % K); x /= K; }
+    int64_t cap = 0, as = 0;
+    for (int d = 0; d < D; d++) {
+      const int o = dig[d];
+      if (allow_idle && o == 0) continue;
+      const int m = off + o - (allow_idle ? 1 : 0);
+      const int64_t pc = P[dev_type[d] * M + m];
+      cap += pc;
+      as += pc * acc[m];
+    }
+    if (as > best_acc[cap]) { best_acc[cap] = as; best_idx[cap] = i; }  /* i ascends: first = lowest index */
+  }
+  int64_t nf = 0;
+  for (int64_t c = 0; c <= cmax; c++) {
+    if (best_acc[c] < 0) continue;
+    int dominated = 0;
+    for (int64_t c2 = 0; c2 <= cmax && !dominated; c2++) {
+      if (c2 == c || best_acc[c2] < 0 || c2 < c) continue;
+      /* c2 > c: dominated iff accuracy(c2) >= accuracy(c) */
+      if (acc_ge(best_acc[c2], c2, best_acc[c], c)) dominated = 1;
+    }
+    if (dominated) continue;
+    if (nf < max_out) { cap_out[nf] = c; accsum_out[nf] = best_acc[c]; idx_out[nf] = best_idx[c]; }
+    nf++;
+  }
+  free(best_acc);
+  free(best_idx);
+  *n_cfg = n;
+  *n_out = nf;
   return 0;
 }
