@@ -400,6 +400,34 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
                      "ops_per_evaluation": fact_g_ops(5), "evaluations": evals,
                      "peak_basis": f"148 SMs x 128 int32 lane-ops/clk x {sm_mhz:.0f} MHz (max SM clock)"},
         "scaling": "weak (vectors split by rank)"}
+    # f3: Fig. 1b Pareto frontier, EfficientNet (5 variants) on 12 devices of the
+    # c3 types (4 each): 5^12 = 244 140 625 configurations (index-range shards)
+    cfg = W.config("c3")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    pdev = np.repeat(np.arange(3, dtype=np.int32), 4)
+    t_pdev = torch.as_tensor(pdev, device=dev)
+    t_pslo = torch.as_tensor(cl.slo_us, dtype=torch.int32, device=dev)
+    for _ in range(2):
+        px.pareto(t_pdev, t_pslo, 3, shard_rank=rank, shard_world=world)
+    pts, pk = [], []
+    px.set_timing(True)
+    for _ in range(3):
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        pr = px.pareto(t_pdev, t_pslo, 3, shard_rank=rank, shard_world=world)
+        b.record(stream)
+        barrier()
+        pts.append(a.elapsed_time(b))
+        pk.append(sum(ms for n, ms in px.kernel_times() if n in ("pareto_best", "pareto_index")))
+    px.set_timing(False)
+    pms = max_over_ranks(statistics.median(pts))
+    out["f3_pareto"] = {
+        "workload": "Fig. 1b frontier: 5 EfficientNet variants on 12 devices (cpu/gpu_a/gpu_b x4), 5^12 configurations",
+        "configs": 5 ** 12, "ms": pms, "configs_per_s": 5 ** 12 / (pms / 1e3),
+        "scan_kernels_ms": statistics.median(pk), "frontier_points": int(pr["n_front"]),
+        "scaling": "strong (index-range shards)" if world > 1 else "1 GPU"}
     # c5: replay 10M queries x 64 scenarios (scenarios on every rank; N>1 = replicas)
     cfg = W.config("c5")
     prof, cl = cfg["prof"], cfg["cluster"]

@@ -198,6 +198,50 @@ int proteus_materialize(proteus_ctx *ctx, const proteus_solve_args *args, int32_
 /* Size of the candidate space of args (modes 0/1), or PROTEUS_ERANGE. */
 int proteus_candidate_count(proteus_ctx *ctx, const proteus_solve_args *args, uint64_t *count);
 
+/* -------------------------------------------------------------- pareto --
+ * Fig. 1b: every configuration of family `family`'s variants on
+ * the D devices ("all possible mappings"), each device serving its capacity
+ * P (the a1 estimate under slo_us, "the maximum number of queries feasible
+ * without SLO violations"), and the Pareto frontier of system throughput
+ * capacity C = sum_d P against system accuracy = the capacity-weighted mean
+ * sum_d P A / C (readings P1-P4).
+ *   D, device_type[D], slo_us[Q]   as proteus_solve (host or device)
+ *   family        the family q whose variants are placed
+ *   allow_idle    0: every device hosts one of the V_q variants (K = V_q, as
+ *                 Fig. 1b's 5^5 = 3125); 1: a device may also idle (digit 0,
+ *                 K = V_q + 1)
+ *   shard_rank, shard_world   scan slice shard_rank of shard_world contiguous
+ *                 slices of the index space; the union of the slices'
+ *                 frontiers contains the whole space's, so the frontier of
+ *                 that union (dist.py: pareto_merge) is the whole answer
+ * A configuration is the mixed-radix number of its digits o_d in [0, K),
+ * device 0 most significant.  A point is on the frontier iff no
+ * configuration has capacity >= and accuracy >= with one of them strict
+ * (accuracies compared exactly; capacity 0 has accuracy 0); each point is
+ * reported once with the lowest index reaching it.
+ * Output: up to max_points points sorted by increasing capacity (accuracy
+ * strictly decreasing) in out[]; *n_points = the frontier size (may exceed
+ * max_points: then only the first max_points are written); *n_configs = the
+ * configurations scanned.  PROTEUS_ERANGE if the space exceeds 2^63 or the
+ * capacity range 2^26. */
+typedef struct {
+  int32_t D;
+  const int32_t *device_type;
+  const int32_t *slo_us;
+  int32_t family;
+  int32_t allow_idle;
+  int32_t shard_rank, shard_world;
+} proteus_pareto_args;
+
+typedef struct {
+  int64_t capacity;  /* sum of P over the devices, QPS */
+  int64_t accsum;    /* sum of P * A (accuracy = accsum / capacity, 1e-6 units) */
+  uint64_t index;    /* lowest configuration index at this point */
+} proteus_pareto_point;
+
+int proteus_pareto(proteus_ctx *ctx, const proteus_pareto_args *args, proteus_pareto_point *out, int32_t max_points,
+                   int32_t *n_points, uint64_t *n_configs);
+
 /* -------------------------------------------------------------- replay --
  * §5 adaptive batching over an allocation, per scenario.
  *   arrival_us[N]   query arrival times, sorted non-decreasing, uint32 us

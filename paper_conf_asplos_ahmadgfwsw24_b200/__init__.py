@@ -182,6 +182,22 @@ class Proteus:
         return Solution(s.score, s.index, s.served, s.unmet, s.accsum, s.eff_acc_micro, s.n_candidates,
                         opt.copy(), z.copy())
 
+    # -------------------------------------------------------------- pareto --
+    def pareto(self, device_type, slo_us, family, allow_idle=False, shard_rank=0, shard_world=1, max_points=65536):
+        """Fig. 1b Pareto frontier (proteus_pareto): dict of numpy arrays
+        cap, accsum, index sorted by capacity, plus n_configs."""
+        keep = []
+        a = N.proteus_pareto_args(len(device_type), _arg(device_type, np.int32, keep), _arg(slo_us, np.int32, keep),
+                                  int(family), int(bool(allow_idle)), int(shard_rank), int(shard_world))
+        pts = (N.proteus_pareto_point * max(1, max_points))()
+        npts, ncfg = C.c_int32(), C.c_uint64()
+        self._check(self._lib.proteus_pareto(self._h, C.byref(a), pts, int(max_points), C.byref(npts), C.byref(ncfg)))
+        k = min(npts.value, max_points)
+        cap = np.array([pts[i].capacity for i in range(k)], np.int64)
+        acs = np.array([pts[i].accsum for i in range(k)], np.int64)
+        idx = np.array([pts[i].index for i in range(k)], np.uint64)
+        return dict(cap=cap, accsum=acs, index=idx, n_configs=ncfg.value, n_front=npts.value)
+
     # -------------------------------------------------------------- replay --
     def replay(self, arrival_us, family, option, z, device_type, demand, slo_base_us, scenarios,
                latency=True, aggregates_out=None):

@@ -21,7 +21,7 @@ PROTEUS_SOLVE_GENERIC = 1
 EXPORTED = (
     "proteus_abi_version", "proteus_create", "proteus_destroy", "proteus_set_stream", "proteus_last_error",
     "proteus_load_profiles", "proteus_solve", "proteus_solve_batch", "proteus_materialize", "proteus_candidate_count",
-    "proteus_replay", "proteus_set_timing", "proteus_kernel_times", "proteus_launch_count",
+    "proteus_pareto", "proteus_replay", "proteus_set_timing", "proteus_kernel_times", "proteus_launch_count",
 )
 
 
@@ -46,6 +46,15 @@ class proteus_batch(C.Structure):
     _fields_ = [("score", C.c_void_p), ("index", C.c_void_p), ("served", C.c_void_p), ("unmet", C.c_void_p),
                 ("accsum", C.c_void_p), ("eff_acc_micro", C.c_void_p), ("option", C.c_void_p),
                 ("z_qps", C.c_void_p), ("n_candidates", C.c_uint64)]
+
+
+class proteus_pareto_args(C.Structure):
+    _fields_ = [("D", C.c_int32), ("device_type", C.c_void_p), ("slo_us", C.c_void_p), ("family", C.c_int32),
+                ("allow_idle", C.c_int32), ("shard_rank", C.c_int32), ("shard_world", C.c_int32)]
+
+
+class proteus_pareto_point(C.Structure):
+    _fields_ = [("capacity", C.c_int64), ("accsum", C.c_int64), ("index", C.c_uint64)]
 
 
 class proteus_scenario(C.Structure):
@@ -83,6 +92,8 @@ def load(path: str = LIB_PATH):
     L.proteus_solve_batch.argtypes = [vp, C.POINTER(proteus_solve_args), C.POINTER(proteus_batch)]
     L.proteus_materialize.argtypes = [vp, C.POINTER(proteus_solve_args), i32, u64, C.POINTER(proteus_solution)]
     L.proteus_candidate_count.argtypes = [vp, C.POINTER(proteus_solve_args), C.POINTER(u64)]
+    L.proteus_pareto.argtypes = [vp, C.POINTER(proteus_pareto_args), C.POINTER(proteus_pareto_point), i32,
+                                 C.POINTER(i32), C.POINTER(u64)]
     L.proteus_replay.argtypes = [vp, vp, vp, i64, vp, vp, vp, i32, vp, vp, C.POINTER(proteus_scenario), i32,
                                  vp, vp, vp, vp]
     L.proteus_set_timing.argtypes = [vp, C.c_int]

@@ -498,6 +498,45 @@ int proteus_candidate_count(proteus_ctx *ctx, const proteus_solve_args *a, uint6
   return ovf ? px_fail(ctx, PROTEUS_ERANGE, "candidate space exceeds 2^64") : PROTEUS_OK;
 }
 
+// ------------------------------------------------------------- pareto -----
+int proteus_pareto(proteus_ctx *ctx, const proteus_pareto_args *a, proteus_pareto_point *out, int32_t max_points,
+                   int32_t *n_points, uint64_t *n_configs) {
+  if (!ctx) return PROTEUS_EINVAL;
+  ctx->err.clear();
+  if (!a || !n_points || !n_configs || max_points < 0 || (max_points > 0 && !out))
+    return px_fail(ctx, PROTEUS_EINVAL, "null argument");
+  if (!ctx->have_prof) return px_fail(ctx, PROTEUS_EINVAL, "no profiles loaded");
+  if (a->D < 1 || a->D > PX_MAXD || !a->device_type || !a->slo_us)
+    return px_fail(ctx, PROTEUS_EINVAL, "D=%d out of range or null array", a->D);
+  if (a->family < 0 || a->family >= ctx->Q) return px_fail(ctx, PROTEUS_EINVAL, "family %d", a->family);
+  const int world = a->shard_world > 0 ? a->shard_world : 1, rank = a->shard_world > 0 ? a->shard_rank : 0;
+  if (rank < 0 || rank >= world) return px_fail(ctx, PROTEUS_EINVAL, "shard %d/%d", rank, world);
+  PX_CUDA(ctx, cudaSetDevice(ctx->device));
+  timing_reset(ctx);
+  std::vector<int32_t> dev, slo;
+  int rc;
+  if ((rc = to_host(ctx, a->device_type, a->D, dev)) || (rc = to_host(ctx, a->slo_us, ctx->Q, slo))) return rc;
+  for (int d = 0; d < a->D; d++)
+    if (dev[d] < 0 || dev[d] >= ctx->T) return px_fail(ctx, PROTEUS_EINVAL, "device_type[%d]=%d", d, dev[d]);
+  for (int q = 0; q < ctx->Q; q++)
+    if (slo[q] < 0) return px_fail(ctx, PROTEUS_EINVAL, "slo_us[%d] < 0", q);
+  const int32_t *d_dev = to_device(ctx, dev.data(), dev.size(), B_IN0, &rc);
+  if (rc) return rc;
+  const int32_t *d_slo = to_device(ctx, slo.data(), slo.size(), B_IN1, &rc);
+  if (rc) return rc;
+  std::vector<proteus_pareto_point> h(max_points > 0 ? max_points : 1);
+  int32_t np = 0;
+  uint64_t nc = 0;
+  if ((rc = px_pareto(ctx, a->D, dev.data(), d_dev, d_slo, a->family, a->allow_idle != 0, rank, world, h.data(),
+                      max_points, &np, &nc)))
+    return rc;
+  if ((rc = timing_collect(ctx))) return rc;
+  for (int i = 0; i < np && i < max_points; i++) out[i] = h[i];
+  *n_points = np;
+  *n_configs = nc;
+  return PROTEUS_OK;
+}
+
 // ------------------------------------------------------------- replay -----
 int proteus_replay(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *family, int64_t N,
                    const int32_t *option, const int32_t *z_qps, const int32_t *device_type, int32_t D,

@@ -88,3 +88,33 @@ def solve_vectors_sharded(px, device_type, slo_us, demand_vectors, group=None):
     if hi <= lo:
         return lo, []
     return lo, px.solve(device_type, slo_us, demand_vectors[lo:hi], mode=2)
+
+
+def pareto_merge(parts):
+    """Frontier of the union of shard frontiers (Fig. 1b, proteus_pareto with
+    shard_rank/shard_world): a point dominated inside a shard is dominated in
+    the whole space, so the union holds every frontier point; keep the points
+    strictly more accurate than everything of higher capacity (exact integer
+    cross-multiplication), the lowest index among equal points.  Host-side
+    combination of <= a few hundred points per shard, like pick_best."""
+    pts = {}
+    for p in parts:
+        for c, a, i in zip(p["cap"].tolist(), p["accsum"].tolist(), p["index"].tolist()):
+            key = (int(c), int(a))
+            if key not in pts or int(i) < pts[key]:
+                pts[key] = int(i)
+    by_cap = {}
+    for (c, a), i in pts.items():  # at one capacity only the largest accuracy sum can survive
+        if c not in by_cap or a > by_cap[c][0] or (a == by_cap[c][0] and i < by_cap[c][1]):
+            by_cap[c] = (a, i)
+    out, ra, rc = [], 0, 0
+    for c in sorted(by_cap, reverse=True):
+        a, i = by_cap[c]
+        above = a * rc > ra * c if (c > 0 and rc > 0) else (a > 0 if c > 0 else (rc == 0 and ra == 0))
+        if above:
+            out.append((c, a, i))
+            ra, rc = a, c
+    out.reverse()
+    return dict(cap=np.array([o[0] for o in out], np.int64), accsum=np.array([o[1] for o in out], np.int64),
+                index=np.array([o[2] for o in out], np.uint64),
+                n_configs=sum(int(p["n_configs"]) for p in parts), n_front=len(out))

@@ -19,6 +19,9 @@ def main():
     px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=0, generic=True)
     px.solve(cl.device_type, cl.slo_us, np.repeat(cfg["demand"], 9, axis=0), mode=2)  # batched kernel
     cfg = W.config("c3", totals=(3000,))
+    px.load_profiles(cfg["prof"])
+    px.pareto(np.array([0, 1, 1, 2, 2], np.int32), cfg["cluster"].slo_us, 3)
+    px.pareto(np.array([0, 1, 2], np.int32), cfg["cluster"].slo_us, 1, allow_idle=True)
     prof, cl = cfg["prof"], cfg["cluster"]
     px.load_profiles(prof)
     sol = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=2)[0]

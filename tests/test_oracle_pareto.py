@@ -114,3 +114,41 @@ def test_scaling_capacity_keeps_frontier(allow_idle):
     assert (3 * a["cap"]).tolist() == b["cap"].tolist()
     assert (3 * a["accsum"]).tolist() == b["accsum"].tolist()
     assert a["index"].tolist() == b["index"].tolist()
+
+
+def test_pareto_merge_of_shards():
+    """dist.pareto_merge: the frontier of the union of per-shard frontiers
+    (each computed by the oracle on a sub-inventory's configurations would need
+    index slices, so the shards here are slices of the full configuration list
+    reduced by the definition) equals the oracle's frontier of the whole."""
+    import oracle
+    from paper_conf_asplos_ahmadgfwsw24_b200.dist import pareto_merge
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    dev = np.array([0, 1, 1, 2], np.int32)
+    q = 3
+    whole = oracle.pareto(prof, dev, cl.slo_us, q)
+    P, _, _ = oracle.capacity(prof, cl.slo_us)
+    off = int(np.sum(prof.V[:q]))
+    pts = []
+    for i, c_ in enumerate(itertools.product(range(5), repeat=4)):
+        c = sum(int(P[dev[d], off + o]) for d, o in enumerate(c_))
+        a = sum(int(P[dev[d], off + o]) * int(prof.acc_micro[off + o]) for d, o in enumerate(c_))
+        pts.append((c, a, i))
+
+    def front(sub):  # definition of the frontier on a slice (exact fractions)
+        keep = []
+        for c, a, i in sub:
+            fa = Fraction(a, c) if c else Fraction(0)
+            dom = any(c2 >= c and (Fraction(a2, c2) if c2 else Fraction(0)) >= fa and
+                      (c2 > c or (Fraction(a2, c2) if c2 else Fraction(0)) > fa) for c2, a2, _ in sub)
+            if not dom:
+                keep.append((c, a, i))
+        return dict(cap=np.array([k[0] for k in keep], np.int64), accsum=np.array([k[1] for k in keep], np.int64),
+                    index=np.array([k[2] for k in keep], np.uint64), n_configs=len(sub))
+    parts = [front(pts[k * 625 // 3:(k + 1) * 625 // 3]) for k in range(3)]
+    m = pareto_merge(parts)
+    assert m["n_configs"] == 625 == whole["n_configs"]
+    for k in ("cap", "accsum", "index"):
+        assert m[k].tolist() == whole[k].tolist(), k
