@@ -66,6 +66,8 @@ def lib():
                                          i32p, i32p, i32p]
         L.orc_route_swrr.argtypes = [C.c_int64, u8p, C.c_int, C.c_int, i32p, i32p, i32p, i32p]
         L.orc_replay_device.argtypes = [C.c_int64, u32p, i32p, C.c_int, C.c_int64, u32p]
+        L.orc_replay_device_nexus.argtypes = [C.c_int64, u32p, i32p, C.c_int, C.c_int64, u32p]
+        L.orc_replay_device_aimd.argtypes = [C.c_int64, u32p, i32p, C.c_int, C.c_int64, u32p]
         L.orc_replay.argtypes = [C.c_int64, u32p, u8p, C.c_int, C.c_int, i32p, i32p, C.c_int, i32p,
                                  C.c_int, i32p, i32p, i32p, i32p, i32p, C.c_int, i32p, C.c_int,
                                  C.c_void_p, u64p, u64p, u64p]
@@ -185,13 +187,42 @@ def replay_device(arrival_us, Tproc, Bmax, L):
     return lat
 
 
+def replay_device_nexus(arrival_us, Tproc, B, L):
+    """§8(f2) Nexus early-drop batching on one device (reading R14); B = the
+    window / batch size.  Dropped queries get UINT32_MAX."""
+    a = np.ascontiguousarray(arrival_us, dtype=np.uint32)
+    lat = np.zeros(len(a), np.uint32)
+    rc = lib().orc_replay_device_nexus(len(a), a, _i32(Tproc), int(B), int(L), lat)
+    assert rc == 0
+    return lat
+
+
+def replay_device_aimd(arrival_us, Tproc, Bmax, L):
+    """§8(f2) Clipper AIMD batching on one device (reading R15)."""
+    a = np.ascontiguousarray(arrival_us, dtype=np.uint32)
+    lat = np.zeros(len(a), np.uint32)
+    rc = lib().orc_replay_device_aimd(len(a), a, _i32(Tproc), int(Bmax), int(L), lat)
+    assert rc == 0
+    return lat
+
+
+def scenario_rows(scenarios):
+    """[S][3] (policy 0) or [S][4] scenario rows -> int32[S][4]
+    (slo_mult_milli, batch_cap, routing, policy)."""
+    sc = np.asarray(scenarios, dtype=np.int32)
+    sc = sc.reshape(-1, sc.shape[-1]) if sc.size else sc.reshape(0, 4)
+    if sc.shape[1] == 3:
+        sc = np.concatenate([sc, np.zeros((sc.shape[0], 1), np.int32)], axis=1)
+    return np.ascontiguousarray(sc)
+
+
 def replay(prof, device_type, option, z, demand, slo_base, arrival_us, family, scenarios,
            want_latency=True, threads=0):
     """a11-a13: route + simulate.  Returns dict(latency [S][N] or None,
     violations, on_time, acc_sum) per scenario."""
     a = np.ascontiguousarray(arrival_us, dtype=np.uint32)
     f = np.ascontiguousarray(family, dtype=np.uint8)
-    sc = _i32(scenarios).reshape(-1, 3)
+    sc = scenario_rows(scenarios)
     S, N = sc.shape[0], len(a)
     lat = np.zeros((S, N), np.uint32) if want_latency else None
     viol = np.zeros(S, np.uint64)

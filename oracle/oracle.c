@@ -22,6 +22,10 @@
  *   orc_route_swrr        literal smooth weighted round-robin router (R8)
  *   orc_replay_device     event-driven simulation of §5 adaptive batching on one
  *                         device, readings R1-R13
+ *   orc_replay_device_nexus / _aimd
+ *                         §8(f2) baseline batchers of §6.4:
+ *                         Nexus early drop and Clipper AIMD, work-conserving,
+ *                         event-driven; readings R14-R15
  *   orc_replay            route + simulate every (device, scenario) lane
  *   orc_pareto            system capacity vs capacity-weighted accuracy of
  *                         every placement of one family's variants, and its
@@ -833,9 +837,101 @@ int orc_replay_device(int64_t n, const uint32_t *a, const int32_t *Tproc, int Bm
   return 0;
 }
 
+/* §8(f2) baseline batchers, P:1535-1630 (§6.4, Fig. 6): "we implement each of
+ * these batching algorithms on top of Proteus".  Both are work-conserving
+ * ("dispatches an inference batch to each device as soon as the previous
+ * batch is finished"): whenever the device is free and the queue
+ * is non-empty, a batch leaves at once.  Event-driven like orc_replay_device
+ * (events: arrivals and batch completions; no timer).  DROPPED = UINT32_MAX.
+ *
+ * Nexus early drop (reading R14).  Batch size B (the
+ * caller passes it: the largest b <= Bmax with 2 T(b) <= L, at least 1 -- the
+ * capacity rule of P:923-928 that sizes Nexus's batches).  At a decision time t
+ * the dispatcher slides a window of min(B, queued from i) queries from the
+ * head: the first query i whose deadline a_i + L is met by the window's
+ * completion t + T(w) starts the batch; every query before it is dropped. */
+int orc_replay_device_nexus(int64_t n, const uint32_t *a, const int32_t *Tproc, int B, int64_t L,
+                            uint32_t *lat) {
+  if (n == 0) return 0;
+  if (B < 1) return -1;
+  const int64_t INF = INT64_MAX / 4;
+  int64_t head = 0, tail = 0;
+  int64_t F = 0;
+  int busy = 0;
+  while (head < n) {
+    int64_t t = INF;
+    if (tail < n) t = a[tail];
+    if (busy && F < t) t = F;
+    while (tail < n && (int64_t)a[tail] <= t) tail++;
+    if (busy && F <= t) busy = 0;
+    if (busy || tail == head) continue;
+    /* sliding window over the queue [head, tail) */
+    int64_t i = head, w = 0;
+    for (; i < tail; i++) {
+      w = tail - i < B ? tail - i : B;
+      if (t + Tproc[w] <= (int64_t)a[i] + L) break;
+      lat[i] = UINT32_MAX;          /* dropped early */
+    }
+    head = i;
+    if (head == tail) continue;     /* everything queued was dropped */
+    F = t + Tproc[w];
+    for (int64_t j = head; j < head + w; j++) {
+      int64_t l = F - (int64_t)a[j];
+      lat[j] = l >= (int64_t)UINT32_MAX ? UINT32_MAX - 1 : (uint32_t)l;
+    }
+    head += w;
+    busy = 1;
+  }
+  return 0;
+}
+
+/* Clipper AIMD (reading R15).  The batch-size limit
+ * starts at 1; a batch takes min(queued, limit) queries.  When it completes,
+ * the limit grows by 1 (additive increase, at most Bmax) if none of its
+ * queries timed out (latency > L), else it shrinks to max(1, floor(9 limit /
+ * 10)) (Clipper's 10 % multiplicative back-off).  No query is dropped. */
+int orc_replay_device_aimd(int64_t n, const uint32_t *a, const int32_t *Tproc, int Bmax, int64_t L,
+                           uint32_t *lat) {
+  if (n == 0) return 0;
+  if (Bmax < 1) return -1;
+  const int64_t INF = INT64_MAX / 4;
+  int64_t head = 0, tail = 0;
+  int64_t F = 0;
+  int busy = 0, limit = 1, pend = 0;  /* pend: the running batch's feedback is still to apply */
+  int timed_out = 0;
+  while (head < n) {
+    int64_t t = INF;
+    if (tail < n) t = a[tail];
+    if (busy && F < t) t = F;
+    while (tail < n && (int64_t)a[tail] <= t) tail++;
+    if (busy && F <= t) {
+      busy = 0;
+      if (pend) {                   /* completion: AIMD update */
+        if (timed_out) limit = limit * 9 / 10 < 1 ? 1 : limit * 9 / 10;
+        else limit = limit + 1 > Bmax ? Bmax : limit + 1;
+        pend = 0;
+      }
+    }
+    if (busy || tail == head) continue;
+    int64_t b = tail - head < limit ? tail - head : limit;
+    F = t + Tproc[b];
+    timed_out = 0;
+    for (int64_t j = head; j < head + b; j++) {
+      int64_t l = F - (int64_t)a[j];
+      lat[j] = l >= (int64_t)UINT32_MAX ? UINT32_MAX - 1 : (uint32_t)l;
+      if (l > L) timed_out = 1;
+    }
+    head += b;
+    busy = 1;
+    pend = 1;
+  }
+  return 0;
+}
+
 /* Full replay (a11-a13).  Scenario s: slo_mult_milli, batch_cap (0 = table
  * depth), routing (0 = SWRR over z with the unmet demand to the sink, 1 =
- * uniform over the hosting devices that fit batch 1, no sink).
+ * uniform over the hosting devices that fit batch 1, no sink), policy (0 = §5
+ * adaptive batching, 1 = Nexus early drop, 2 = Clipper AIMD; §8(f2)).
  * SLO_q(s) = floor(mult * slo_base[q] / 1000) (R12); Bmax = min(cap, depth).
  * Outputs per scenario: violations (latency > SLO, R6, plus dropped), on_time,
  * acc_sum (sum of the serving variant's accuracy over on-time queries, R9);
@@ -860,7 +956,7 @@ static void *rep_worker(void *arg) {
     int64_t lane = __sync_fetch_and_add(&c->next, 1);
     if (lane >= (int64_t)c->S * (c->D + 1)) break;
     int s = (int)(lane / (c->D + 1)), d = (int)(lane % (c->D + 1));
-    int rt = c->sc[s * 3 + 2];
+    int rt = c->sc[s * 4 + 2];
     int64_t st = c->dev_start[rt][d], en = c->dev_start[rt][d + 1];
     uint64_t viol = 0, ont = 0, accs = 0;
     if (d == c->D) { /* sink: dropped */
@@ -872,16 +968,25 @@ static void *rep_worker(void *arg) {
       const int32_t *row = c->lat_tab + ((size_t)t * c->M + m) * c->bmax;
       int dep = 0;
       while (dep < c->bmax && row[dep] > 0) dep++;
-      int cap = c->sc[s * 3 + 1];
+      int cap = c->sc[s * 4 + 1];
       int Bmax = (cap > 0 && cap < dep) ? cap : dep;
-      int64_t L = (int64_t)c->sc[s * 3 + 0] * c->slo_base[q] / 1000;
+      int64_t L = (int64_t)c->sc[s * 4 + 0] * c->slo_base[q] / 1000;
       int64_t n = en - st;
       uint32_t *a = (uint32_t *)malloc(sizeof(uint32_t) * n), *l = (uint32_t *)malloc(sizeof(uint32_t) * n);
       for (int64_t k = 0; k < n; k++) a[k] = c->arr[c->idx_of_dev[rt][st + k]];
       int32_t Tp[1025];
       Tp[0] = 0;
       for (int b = 1; b <= Bmax && b <= 1024; b++) Tp[b] = row[b - 1];
-      orc_replay_device(n, a, Tp, Bmax, L, l);
+      const int policy = c->sc[s * 4 + 3];
+      if (policy == 1) {          /* Nexus: batch size by the capacity rule (R14) */
+        int B = 1;
+        for (int b = 1; b <= Bmax && b <= 1024; b++) if (2LL * Tp[b] <= L) B = b;
+        orc_replay_device_nexus(n, a, Tp, B, L, l);
+      } else if (policy == 2) {
+        orc_replay_device_aimd(n, a, Tp, Bmax, L, l);
+      } else {
+        orc_replay_device(n, a, Tp, Bmax, L, l);
+      }
       for (int64_t k = 0; k < n; k++) {
         if ((int64_t)l[k] > L) viol++;
         else { ont++; accs += (uint64_t)c->acc[m]; }
@@ -900,7 +1005,7 @@ int orc_replay(int64_t N, const uint32_t *arrival, const uint8_t *family,
                int T, int Q, const int32_t *V, const int32_t *acc, int bmax, const int32_t *lat_tab,
                int D, const int32_t *option, const int32_t *z, const int32_t *dev_type,
                const int32_t *demand, const int32_t *slo_base,
-               int S, const int32_t *sc /* [S][3] */, int nthreads,
+               int S, const int32_t *sc /* [S][4] */, int nthreads,
                uint32_t *latency, uint64_t *viol, uint64_t *ontime, uint64_t *accsum) {
   int M = 0;
   for (int q = 0; q < Q; q++) M += V[q];
@@ -919,7 +1024,7 @@ int orc_replay(int64_t N, const uint32_t *arrival, const uint8_t *family,
   for (int s = 0; s < S; s++) { viol[s] = 0; ontime[s] = 0; accsum[s] = 0; }
   for (int rt = 0; rt < 2; rt++) {
     int used = 0;
-    for (int s = 0; s < S; s++) used |= sc[s * 3 + 2] == rt;
+    for (int s = 0; s < S; s++) used |= sc[s * 4 + 2] == rt;
     if (!used) continue;
     int32_t wdev[ORC_MAXD], wsink[ORC_MAXQ];
     for (int q = 0; q < Q; q++) wsink[q] = 0;
