@@ -478,6 +478,36 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
         "e2e": {"value": N * S / e2e, "unit": "query-scenarios/s", "h2d_bytes_per_step": int(N * 5),
                 "d2h_bytes_per_step": int(N * S * 4)},
         "scaling": "replicas" if world > 1 else "1 GPU"}
+    # f2: the §6.4 baseline batchers (Nexus early drop, Clipper AIMD) on the same
+    # trace and allocation, 64 scenarios each (k_wc_lanes), plus the Fig. 6-style
+    # violation ratios of all three policies at SLO 2x, batch cap = table depth
+    f2 = {}
+    for pol, name in ((1, "nexus"), (2, "aimd")):
+        scp = W.scenarios_64(0, pol)
+        px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, scp, latency=lat)
+        px.set_timing(True)
+        ts, kms = [], []
+        for _ in range(3):
+            barrier()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            rp = px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, scp,
+                           latency=lat)
+            b.record(stream)
+            barrier()
+            ts.append(a.elapsed_time(b))
+            kms.append(sum(ms_ for n, ms_ in px.kernel_times() if n == "replay_baseline"))
+        px.set_timing(False)
+        pms = max_over_ranks(statistics.median(ts))
+        km = statistics.median(kms)
+        sel = [i for i, r in enumerate(scp) if r[0] == 2000 and r[1] == 0][0]
+        f2[name] = {"ms": pms, "query_scenarios_per_s": N * len(scp) / (pms / 1e3), "lane_kernel_ms": km,
+                    "lane_kernel_hbm_frac": (N * len(scp) * 4 + N * 8) / (km / 1e3) / 1e9 / hbm,
+                    "violation_ratio_slo2x_depth": float(rp["violations"][sel]) / N}
+    sel = [i for i, r in enumerate(sc) if r[0] == 2000 and r[1] == 0][0]
+    f2["proteus_violation_ratio_slo2x_depth"] = float(res["violations"][sel]) / N
+    f2["workload"] = "c5 trace (10M Poisson queries) and allocation, 64 (SLO x batch cap) scenarios per policy"
+    out["f2_baseline_batchers"] = f2
     return out
 
 

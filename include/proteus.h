@@ -42,7 +42,7 @@
 extern "C" {
 #endif
 
-#define PROTEUS_ABI_VERSION 1
+#define PROTEUS_ABI_VERSION 2
 
 enum {
   PROTEUS_OK = 0,
@@ -256,13 +256,27 @@ int proteus_pareto(proteus_ctx *ctx, const proteus_pareto_args *args, proteus_pa
  *                   (0 = table depth; Bmax = min(cap, depth), R4), routing
  *                   (0 = smooth weighted round-robin over z with the sink,
  *                   1 = uniform over hosting devices that fit batch 1, no
- *                   sink; reading R8)
+ *                   sink; reading R8), policy (the batching rule on every
+ *                   device: 0 = §5 adaptive batching below; 1 = Nexus early
+ *                   drop, 2 = Clipper AIMD -- the §6.4 baselines, P:1535-1630,
+ *                   readings R14-R15 below)
  * Routing (R8): per family, query k goes to pattern_q[k mod W_q] of the SWRR
  * sequence over the members (hosting devices ascending, then the sink).
  * Batching per device (R1-R5): at decision time t with q queued, dispatch
  * Bmax if q >= Bmax, else q once t >= a_head + SLO - T(q+1), else wait for the
  * next arrival or that time; a batch of b dispatched at t finishes at t+T(b),
  * T(b) = lat_us of the device's variant (R10).
+ * Baseline policies (§8(f2); work-conserving: a batch leaves at
+ * t = max(F, a_head), the moment the device is free and a query waits):
+ *   1 Nexus early drop (R14): batch size B = the
+ *     largest b <= Bmax with 2 T(b) <= SLO (the capacity rule), at
+ *     least 1; from the head, the first queued query i whose deadline
+ *     a_i + SLO is met by t + T(min(B, queued from i)) starts the batch and
+ *     the queries before it are dropped (latency UINT32_MAX).
+ *   2 Clipper AIMD (R15): a batch takes
+ *     min(queued, limit); limit starts at 1, grows by 1 (up to Bmax) after a
+ *     batch with no query latency > SLO, else becomes max(1, floor(9 limit /
+ *     10)).  Nothing is dropped.
  * Outputs (each may be NULL):
  *   latency_us[S][N]  per-query latency F - a (UINT32_MAX = dropped)
  *   violations[S]     latency > SLO (strict, R6) plus dropped
@@ -273,7 +287,12 @@ typedef struct {
   int32_t slo_mult_milli;
   int32_t batch_cap;
   int32_t routing;
+  int32_t policy;  /* 0 = §5 adaptive batching, 1 = Nexus early drop, 2 = Clipper AIMD (ABI 2) */
 } proteus_scenario;
+
+#define PROTEUS_POLICY_PROTEUS 0
+#define PROTEUS_POLICY_NEXUS 1
+#define PROTEUS_POLICY_AIMD 2
 
 int proteus_replay(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *family, int64_t N,
                    const int32_t *option, const int32_t *z_qps, const int32_t *device_type, int32_t D,

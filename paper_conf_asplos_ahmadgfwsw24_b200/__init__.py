@@ -203,9 +203,15 @@ class Proteus:
                latency=True, aggregates_out=None):
         """Adaptive-batching replay (proteus_replay).  latency: True -> host
         numpy [S][N]; a CUDA uint32 tensor [S][N] -> written in place; None ->
-        not produced."""
+        not produced.  scenarios: int32 rows (slo_mult_milli, batch_cap,
+        routing[, policy]); a missing policy column means 0 (§5 batching)."""
         keep = []
-        sc = np.ascontiguousarray(np.asarray(scenarios, dtype=np.int32).reshape(-1, 3))
+        sc = np.asarray(scenarios, dtype=np.int32)
+        sc = sc.reshape(-1, sc.shape[-1])
+        if sc.shape[1] == 3:
+            sc = np.concatenate([sc, np.zeros((sc.shape[0], 1), np.int32)], axis=1)
+        if sc.shape[1] != 4:
+            raise ValueError("scenario rows have 3 or 4 columns")
         S = sc.shape[0]
         scs = (N.proteus_scenario * S)(*[N.proteus_scenario(*map(int, row)) for row in sc])
         n = int(arrival_us.shape[0]) if hasattr(arrival_us, "shape") else len(arrival_us)

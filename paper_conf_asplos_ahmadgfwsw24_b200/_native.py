@@ -58,7 +58,8 @@ class proteus_pareto_point(C.Structure):
 
 
 class proteus_scenario(C.Structure):
-    _fields_ = [("slo_mult_milli", C.c_int32), ("batch_cap", C.c_int32), ("routing", C.c_int32)]
+    _fields_ = [("slo_mult_milli", C.c_int32), ("batch_cap", C.c_int32), ("routing", C.c_int32),
+                ("policy", C.c_int32)]
 
 
 class ProteusError(RuntimeError):
@@ -100,7 +101,7 @@ def load(path: str = LIB_PATH):
     L.proteus_kernel_times.argtypes = [vp, C.POINTER(C.c_char_p), C.POINTER(C.c_float), C.c_int]
     L.proteus_launch_count.argtypes = [vp]
     L.proteus_launch_count.restype = u64
-    if L.proteus_abi_version() != 1:
+    if L.proteus_abi_version() != 2:
         raise ImportError("libproteus ABI version mismatch")
     _lib = L
     return L

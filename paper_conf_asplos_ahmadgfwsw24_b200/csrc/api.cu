@@ -575,7 +575,8 @@ int proteus_replay(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *
   for (int q = 0; q < ctx->Q; q++)
     if (zsum[q] > dem[q]) return px_fail(ctx, PROTEUS_EINVAL, "sum z of family %d exceeds its demand", q);
   for (int s = 0; s < S; s++)
-    if (scv[s].slo_mult_milli < 0 || scv[s].batch_cap < 0 || scv[s].routing < 0 || scv[s].routing > 1)
+    if (scv[s].slo_mult_milli < 0 || scv[s].batch_cap < 0 || scv[s].routing < 0 || scv[s].routing > 1 ||
+        scv[s].policy < 0 || scv[s].policy > 2)
       return px_fail(ctx, PROTEUS_EINVAL, "scenario %d", s);
   const uint32_t *d_arr = to_device(ctx, arrival_us, (size_t)N, B_IN0, &rc);
   if (rc) return rc;

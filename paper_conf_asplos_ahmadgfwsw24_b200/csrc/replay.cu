@@ -258,6 +258,8 @@ struct LaneParam {  // per (scenario, device)
   int32_t Bmax;     // min(cap, depth) (R4); 0 for idle devices
   uint32_t A;       // accuracy of the hosted variant
   int64_t L;        // scenario SLO of the hosted family (R12)
+  int32_t policy;   // 0 §5, 1 Nexus early drop, 2 Clipper AIMD (§8(f2))
+  int32_t Bn;       // Nexus batch size: largest b <= Bmax with 2 T(b) <= L, at least 1 (R14)
 };
 
 __global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__restrict__ option,
@@ -268,7 +270,7 @@ __global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__re
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= S * D) return;
   const int s = i / D, d = i % D;
-  LaneParam p = {0, 0, 0};
+  LaneParam p = {0, 0, 0, sc[s].policy, 0};
   const int o = option[d];
   if (o > 0) {
     const int32_t *T = lat + ((size_t)dev_type[d] * M + (o - 1)) * bmax;
@@ -278,6 +280,9 @@ __global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__re
     p.Bmax = (cap > 0 && cap < depth) ? cap : depth;
     p.A = (uint32_t)acc[o - 1];
     p.L = (int64_t)sc[s].slo_mult_milli * slo_base[fam_of_m[o - 1]] / 1000;
+    p.Bn = 1;
+    for (int b = 1; b <= p.Bmax; b++)
+      if (2 * (int64_t)T[b - 1] <= p.L) p.Bn = b;
   }
   lp[i] = p;
 }
@@ -382,6 +387,71 @@ __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ 
     F = t + T[b - 1];
     for (int j = 0; j < b; j++) out[h + j] = sat_lat(F - (int64_t)arr(h + j));
     h += b;
+  }
+}
+
+// ---- §8(f2) work-conserving baseline batchers, readings R14-R15
+// Warp per (device, scenario).  Both rules decide at t = max(F, a_head) (the
+// device is free and a query waits); the queue at t is
+// [h, tail), tail advanced 32 arrivals per ballot (t never decreases, so tail
+// only moves forward).  Nexus: the window test t + T(min(B, tail - i)) <=
+// a_i + L for 32 candidate heads i per ballot, the first pass starts the batch
+// and the lanes below it write the drops; AIMD: b = min(queued, limit) and the
+// limit update at completion.  Latencies are written 32 per store
+// (coalesced).
+__global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneArgs a) {
+  const int wid = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) >> 5), lane = threadIdx.x & 31;
+  if (wid >= a.nsc * a.D) return;
+  const int s = a.sc_list[wid / a.D], d = wid % a.D;
+  const LaneParam p = a.lp[s * a.D + d];
+  const int64_t st = a.devOff[d], n = a.devOff[d + 1] - st;
+  if (n == 0) return;
+  uint32_t *out = a.latd + (size_t)s * a.NS + st;
+  if (p.Bmax < 1) {  // never routed to (z = 0 / depth 0); kept for safety
+    for (int64_t j = lane; j < n; j += 32) out[j] = 0xFFFFFFFFu;
+    return;
+  }
+  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  const uint32_t *arr = a.devArr + st;
+  const bool nexus = p.policy == 1;
+  const int B = nexus ? p.Bn : p.Bmax;
+  int64_t h = 0, tail = 0, F = 0;  // R13
+  int limit = 1;                   // AIMD batch-size limit
+  while (h < n) {
+    const int64_t ah = __ldg(arr + h);
+    const int64_t t = F > ah ? F : ah;
+    if (tail <= h) tail = h + 1;
+    for (;;) {  // queued at t: arrivals <= t (sorted: the ballot is a prefix)
+      const int64_t j = tail + lane;
+      const unsigned m = __ballot_sync(0xffffffffu, j < n && (int64_t)__ldg(arr + j) <= t);
+      tail += __popc(m);
+      if (m != 0xffffffffu) break;
+    }
+    int64_t first = h;
+    if (nexus) {
+      first = -1;
+      for (int64_t i0 = h; i0 < tail; i0 += 32) {
+        const int64_t i = i0 + lane;
+        bool pass = false;
+        if (i < tail) {
+          const int64_t w = tail - i < B ? tail - i : B;
+          pass = t + __ldg(T + w - 1) <= (int64_t)__ldg(arr + i) + p.L;
+        }
+        const unsigned m = __ballot_sync(0xffffffffu, pass);
+        const int nd = m ? __ffs(m) - 1 : 32;
+        if (lane < nd && i < tail) out[i] = 0xFFFFFFFFu;  // dropped early
+        if (m) { first = i0 + nd; break; }
+      }
+      if (first < 0) { h = tail; continue; }  // everything queued was dropped
+    }
+    const int b = (int)(tail - first < (nexus ? B : limit) ? tail - first : (nexus ? B : limit));
+    F = t + __ldg(T + b - 1);
+    for (int k = lane; k < b; k += 32) out[first + k] = sat_lat(F - (int64_t)__ldg(arr + first + k));
+    if (!nexus) {  // completion feedback (the next decision is at >= F)
+      if (F - ah > p.L) limit = limit * 9 / 10 < 1 ? 1 : limit * 9 / 10;
+      else limit = limit + 1 > p.Bmax ? p.Bmax : limit + 1;
+    }
+    h = first + b;
   }
 }
 
@@ -1513,7 +1583,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
               const proteus_scenario *h_sc, int S, uint32_t *d_lat_out, uint64_t *d_agg) {
   const int Q = ctx->Q, M = ctx->M;
   PX_CUDA(ctx, cudaMemsetAsync(d_agg, 0, ((size_t)3 * S + 1) * 8, ctx->stream));
-  const size_t small = (size_t)(4 * D + 2 * Q + 2 * PX_MAXQ + 8 + 2 * S + 4 * (PX_MAXD + 2)) * 4 +
+  const size_t small = (size_t)(4 * D + 2 * Q + 2 * PX_MAXQ + 8 + 6 * S + 4 * (PX_MAXD + 2)) * 4 +
                        (size_t)S * sizeof(proteus_scenario) + (size_t)S * D * sizeof(LaneParam) +
                        (size_t)2 * (PX_MAXD + 2) * 8;
   char *sb = (char *)px_buf(ctx, B_R_MISC, small + 4096);
@@ -1521,22 +1591,27 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   int32_t *d_opt = (int32_t *)sb, *d_z = d_opt + D, *d_dev = d_z + D, *d_dem = d_dev + D, *d_slo = d_dem + Q;
   int32_t *d_pat_off = d_slo + Q, *d_pat_len = d_pat_off + PX_MAXQ;
   uint32_t *d_flags = (uint32_t *)(d_pat_len + PX_MAXQ);  // [0] trace checks, [4] fix-up changes
-  int32_t *d_scl = (int32_t *)(d_flags + 8);              // [2][S] scenario lists per routing mode
-  int32_t *d_goff = d_scl + 2 * S;                        // [2][PX_MAXD + 2]
+  // [6][S] scenario lists: per routing mode rt, row rt = every scenario, row 2 + rt = the §5
+  // scenarios (chunk / scan kernels), row 4 + rt = the baseline batchers (k_wc_lanes)
+  int32_t *d_scl = (int32_t *)(d_flags + 8);
+  int32_t *d_goff = d_scl + 6 * S;                        // [2][PX_MAXD + 2]
   int64_t *d_choff = (int64_t *)(((uintptr_t)(d_goff + 2 * (PX_MAXD + 2)) + 15) & ~(uintptr_t)15);  // [2][PX_MAXD + 2]
   proteus_scenario *d_sc = (proteus_scenario *)(d_choff + 2 * (PX_MAXD + 2));
   LaneParam *d_lp = (LaneParam *)(((uintptr_t)(d_sc + S) + 15) & ~(uintptr_t)15);
-  std::vector<int32_t> scl[2];
-  for (int s = 0; s < S; s++) scl[h_sc[s].routing].push_back(s);
-  std::vector<int32_t> scl_all(2 * S, 0);
-  for (int rt = 0; rt < 2; rt++)
-    for (size_t k = 0; k < scl[rt].size(); k++) scl_all[rt * S + k] = scl[rt][k];
+  std::vector<int32_t> scl[6];
+  for (int s = 0; s < S; s++) {
+    scl[h_sc[s].routing].push_back(s);
+    scl[(h_sc[s].policy == 0 ? 2 : 4) + h_sc[s].routing].push_back(s);
+  }
+  std::vector<int32_t> scl_all(6 * S, 0);
+  for (int r = 0; r < 6; r++)
+    for (size_t k = 0; k < scl[r].size(); k++) scl_all[r * S + k] = scl[r][k];
   PX_CUDA(ctx, cudaMemcpyAsync(d_opt, h_option, D * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_z, h_z, D * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_dev, h_dev_type, D * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_dem, h_demand, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_slo, h_slo, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
-  PX_CUDA(ctx, cudaMemcpyAsync(d_scl, scl_all.data(), 2 * S * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_scl, scl_all.data(), 6 * S * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_sc, h_sc, S * sizeof(proteus_scenario), cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemsetAsync(d_flags, 0, 4, ctx->stream));
   if (N > 0) {
@@ -1651,9 +1726,9 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     if (scl[rt].empty()) continue;
     LaneArgs la;
     memset(&la, 0, sizeof la);
-    la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.nsc = (int)scl[rt].size(); la.CH = CH;
+    la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.nsc = (int)scl[2 + rt].size(); la.CH = CH;
     la.N = N; la.NS = NS; la.NCH = nmax;  // one row stride for both routing modes
-    la.option = d_opt; la.dev_type = d_dev; la.lat = ctx->d_lat; la.sc_list = d_scl + rt * S; la.lp = d_lp;
+    la.option = d_opt; la.dev_type = d_dev; la.lat = ctx->d_lat; la.sc_list = d_scl + (2 + rt) * S; la.lp = d_lp;
     la.devOff = devOff[rt]; la.choff = d_choff + rt * (PX_MAXD + 2); la.goff = d_goff + rt * (PX_MAXD + 2);
     la.devArr = devArr[rt]; la.latd = latd; la.cs = csb[0]; la.csp = nullptr; la.agg = d_agg;
     la.debug = env_int("PROTEUS_REPLAY_DEBUG", 0);
@@ -1662,6 +1737,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     la.dmask = D >= 64 ? ~0ull : ((1ull << D) - 1);
     la.lstat = d_lstat;
     la.lstart = d_lstart;
+    if (la.nsc > 0) {  // §5 scenarios
     if (use_scan1) {  // Bmax = 1 lanes: exact prefix-maximum scan
       Scan1Args sa;
       memset(&sa, 0, sizeof sa);
@@ -1671,7 +1747,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       for (int d = 0; d < D; d++) {
         sa.boff[d] = nb;
         bool any = false;
-        for (int k : scl[rt]) any |= hB[(size_t)k * D + d] == 1;
+        for (int k : scl[2 + rt]) any |= hB[(size_t)k * D + d] == 1;
         if (!any) continue;
         t1[d] = hT1[d];
         nb += (h_off[rt][d + 1] - h_off[rt][d] + SCAN_BLK - 1) / SCAN_BLK;
@@ -1684,7 +1760,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
         sa.bpre = sa.bmx + nb;
         int32_t *d_t1 = (int32_t *)(sa.bpre + nb);
         PX_CUDA(ctx, cudaMemcpyAsync(d_t1, t1.data(), D * 4, cudaMemcpyHostToDevice, ctx->stream));
-        sa.T1 = d_t1; sa.devOff = devOff[rt]; sa.devArr = devArr[rt]; sa.sc_list = d_scl + rt * S; sa.lp = d_lp;
+        sa.T1 = d_t1; sa.devOff = devOff[rt]; sa.devArr = devArr[rt]; sa.sc_list = d_scl + (2 + rt) * S; sa.lp = d_lp;
         sa.latd = latd;
         if (nb > 0x7fffffff) return px_fail(ctx, PROTEUS_ERANGE, "scan blocks");
         PX_LAUNCH(ctx, "replay_scan1", k_scan1_reduce, (unsigned)nb, 256, 0, sa);
@@ -1704,7 +1780,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       if (use_bscan) {
         std::vector<int32_t> lid;
         std::vector<int64_t> loff(1, 0);
-        for (int k : scl[rt])
+        for (int k : scl[2 + rt])
           for (int d = 0; d < D; d++) {
             const int B = hB[(size_t)k * D + d];
             const int64_t nd = h_off[rt][d + 1] - h_off[rt][d];
@@ -1743,12 +1819,12 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
         PX_CUDA(ctx, cudaMemcpyAsync(hs.data(), d_lstat, hs.size() * 4, cudaMemcpyDeviceToHost, ctx->stream));
         PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
         unsigned long long tot = 0, full = 0;
-        for (int k : scl[rt])
+        for (int k : scl[2 + rt])
           for (int d = 0; d < D; d++) { tot += hs[2 * ((size_t)k * D + d) + 1]; full += hs[2 * ((size_t)k * D + d)]; }
         fprintf(stderr, "replay routing %d: %llu speculative decisions, %llu full-immediate\n", rt, tot, full);
         for (int d = 0; d < D; d++) {
           unsigned long long t = 0;
-          for (int k : scl[rt]) t += hs[2 * ((size_t)k * D + d) + 1];
+          for (int k : scl[2 + rt]) t += hs[2 * ((size_t)k * D + d) + 1];
           fprintf(stderr, "  device %d: n=%lld decisions=%llu\n", d, (long long)(h_off[rt][d + 1] - h_off[rt][d]), t);
         }
       }
@@ -1775,9 +1851,18 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
         PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, stitch_smem(ctx->bmax), la);
       }
     }
-    dim3 g(32, la.nsc < 65535 ? la.nsc : 65535);
-    PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, NS, S, D, d_scl + rt * S, la.nsc, devOff[rt], latd, d_agg);
-    dim3 cg((unsigned)((N + CNT_PER - 1) / CNT_PER), (unsigned)la.nsc);
+    }  // §5 scenarios
+    if (!scl[4 + rt].empty()) {  // §8(f2) baseline batchers: warp per (device, scenario)
+      LaneArgs lb = la;
+      lb.nsc = (int)scl[4 + rt].size();
+      lb.sc_list = d_scl + (4 + rt) * S;
+      const int64_t warps = (int64_t)lb.nsc * D;
+      PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes, (unsigned)((warps + 3) / 4), 128, 0, lb);
+    }
+    const int nall = (int)scl[rt].size();
+    dim3 g(32, nall < 65535 ? nall : 65535);
+    PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, NS, S, D, d_scl + rt * S, nall, devOff[rt], latd, d_agg);
+    dim3 cg((unsigned)((N + CNT_PER - 1) / CNT_PER), (unsigned)nall);
     PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, NS, S, D, d_scl + rt * S, devOff[rt], d_lp, latd, d_agg);
   }
   if (d_lat_out) {

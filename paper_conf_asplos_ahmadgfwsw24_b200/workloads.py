@@ -201,10 +201,21 @@ SLO_MULTS_MILLI = (1000, 1500, 2000, 2500, 3000, 3500, 4000, 5000)   # covers P:
 BATCH_CAPS = (1, 2, 4, 8, 16, 32, 64, 0)                               # 1 = "w/o AB"; 0 = table depth
 
 
-def scenarios_64(routing: int = 0) -> np.ndarray:
+def scenarios_64(routing: int = 0, policy: int | None = None) -> np.ndarray:
     """64 (SLO multiplier, batch cap) scenarios as an int32[S][3] array of
-    (slo_mult_milli, batch_cap, routing)."""
-    rows = [(m, c, routing) for m in SLO_MULTS_MILLI for c in BATCH_CAPS]
+    (slo_mult_milli, batch_cap, routing), or int32[S][4] with a policy column
+    (0 §5 batching, 1 Nexus early drop, 2 Clipper AIMD; §6.4)."""
+    if policy is None:
+        rows = [(m, c, routing) for m in SLO_MULTS_MILLI for c in BATCH_CAPS]
+    else:
+        rows = [(m, c, routing, policy) for m in SLO_MULTS_MILLI for c in BATCH_CAPS]
+    return np.array(rows, dtype=np.int32)
+
+
+def scenarios_fig6(routing: int = 0) -> np.ndarray:
+    """Fig. 6 / §6.4 comparison grid: the three batching
+    policies x SLO multipliers x batch caps {8, 32, depth}: int32[72][4]."""
+    rows = [(m, c, routing, p) for p in (0, 1, 2) for m in SLO_MULTS_MILLI for c in (8, 32, 0)]
     return np.array(rows, dtype=np.int32)
 
 

@@ -143,3 +143,46 @@ def test_replay_aggregates_without_latencies(px, oracle_mod):
     o = oracle_mod.replay(prof, cl.device_type, r["option"], r["z"], cfg["demand"][1], cl.slo_us, arr, fam, sc)
     for k in ("violations", "on_time", "acc_sum"):
         assert np.array_equal(g[k], o[k]), k
+
+
+@pytest.mark.parametrize("kind", ["poisson", "gamma", "uniform"])
+@pytest.mark.parametrize("policy", [1, 2])
+def test_replay_baseline_policies(px, oracle_mod, kind, policy):
+    """§8(f2): Nexus early drop (1) and Clipper AIMD (2) lanes (k_wc_lanes)
+    bit-exact against the oracle's event-driven simulators, 64 scenarios x
+    both routings, light load and overload (sink)."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    for v, n in ((0, 60_000), (1, 40_000)):
+        r = _alloc(oracle_mod, cfg, v)
+        arr, fam = W.query_trace(n, float(cfg["demand"][v].sum()), cfg["weights"], 11 + v, kind)
+        for routing in (0, 1):
+            g = _compare(px, oracle_mod, cfg["prof"], cfg["cluster"], r["option"], r["z"], cfg["demand"][v], arr,
+                         fam, W.scenarios_64(routing, policy))
+            assert np.all(g["violations"] + g["on_time"] == len(arr))
+
+
+def test_replay_mixed_policies_one_call(px, oracle_mod):
+    """All three policies in one call (Fig. 6 grid, both routings): the §5
+    scenarios take the chunk/stitch path, the baselines k_wc_lanes, and the
+    counts / sink / un-permute see every scenario."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    r = _alloc(oracle_mod, cfg, 1)
+    arr, fam = W.query_trace(50_000, float(cfg["demand"][1].sum()), cfg["weights"], 13, "gamma")
+    sc = np.concatenate([W.scenarios_fig6(0), W.scenarios_fig6(1)])
+    rng = np.random.default_rng(5)
+    sc = sc[rng.permutation(len(sc))]
+    _compare(px, oracle_mod, cfg["prof"], cfg["cluster"], r["option"], r["z"], cfg["demand"][1], arr, fam, sc)
+
+
+def test_replay_baseline_edge_cases(px, oracle_mod):
+    """Tiny traces: one query, all simultaneous, and a tight SLO that drops
+    nearly everything under Nexus."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    r = _alloc(oracle_mod, cfg, 0)
+    for arr in (np.array([5], np.uint32), np.zeros(300, np.uint32), np.arange(0, 3000, 10, dtype=np.uint32)):
+        fam = np.zeros(len(arr), np.uint8)
+        sc = np.array([(m, c, 0, p) for m in (100, 1000) for c in (1, 4, 0) for p in (0, 1, 2)], np.int32)
+        _compare(px, oracle_mod, cfg["prof"], cfg["cluster"], r["option"], r["z"], cfg["demand"][0], arr, fam, sc)
