@@ -289,6 +289,7 @@ __global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__re
 
 struct LaneArgs {
   int S, D, M, bmax, nsc, CH;
+  int WU;                 // k_spec warm-up: queries replayed before each chunk (0 = start at the chunk)
   int64_t N, NCH;
   int64_t NS;             // row stride of latd (N rounded up to 32: 16-byte aligned rows for bulk copies)
   const int32_t *option, *dev_type, *lat, *sc_list;
@@ -397,10 +398,16 @@ __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ 
 // only moves forward).  Nexus: the window test t + T(min(B, tail - i)) <=
 // a_i + L for 32 candidate heads i per ballot, the first pass starts the batch
 // and the lanes below it write the drops; AIMD: b = min(queued, limit) and the
-// limit update at completion.  Latencies are written 32 per store
-// (coalesced).
+// limit update at completion.  The lane's arrivals are staged in a per-warp
+// shared-memory ring covering [b0, b0 + WC_RW) (refilled by halves with
+// coalesced loads as the head advances; reads past it go to global memory),
+// T(b) in shared memory; latencies are written 32 per store (coalesced).
+#define WC_RW 1024
 __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneArgs a) {
+  __shared__ uint32_t sA[4][WC_RW];
+  __shared__ int32_t sT[4][PX_MAXB];
   const int wid = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) >> 5), lane = threadIdx.x & 31;
+  const int w = threadIdx.x >> 5;
   if (wid >= a.nsc * a.D) return;
   const int s = a.sc_list[wid / a.D], d = wid % a.D;
   const LaneParam p = a.lp[s * a.D + d];
@@ -411,19 +418,68 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
     for (int64_t j = lane; j < n; j += 32) out[j] = 0xFFFFFFFFu;
     return;
   }
-  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  int32_t *T = sT[w];
+  for (int k = lane; k < p.Bmax; k += 32) T[k] = __ldg(Tg + k);
   const uint32_t *arr = a.devArr + st;
+  uint32_t *ring = sA[w];
+  int64_t b0 = 0;
+  auto fill = [&](int64_t from, int cnt) {
+    for (int k = lane; k < cnt; k += 32) {
+      const int64_t j = from + k;
+      ring[j & (WC_RW - 1)] = j < n ? __ldg(arr + j) : 0xFFFFFFFFu;
+    }
+  };
+  fill(0, WC_RW);
+  __syncwarp();
+  // arrival j >= b0 (every index read is >= the head >= b0)
+  auto A = [&](int64_t j) -> int64_t {
+    return j - b0 < WC_RW ? (int64_t)ring[j & (WC_RW - 1)] : (int64_t)__ldg(arr + j);
+  };
   const bool nexus = p.policy == 1;
   const int B = nexus ? p.Bn : p.Bmax;
   int64_t h = 0, tail = 0, F = 0;  // R13
   int limit = 1;                   // AIMD batch-size limit
+  const int64_t T1 = T[0];
+  const bool fast = T1 <= p.L;     // isolated queries are on time
   while (h < n) {
-    const int64_t ah = __ldg(arr + h);
+    if (h - b0 >= WC_RW / 2) {     // slide the ring
+      const int64_t nb = h & ~(int64_t)(WC_RW / 2 - 1);
+      __syncwarp();
+      if (nb == b0 + WC_RW / 2) fill(b0 + WC_RW, WC_RW / 2);
+      else fill(nb, WC_RW);
+      b0 = nb;
+      __syncwarp();
+    }
+    const int64_t ah = A(h);
+    if (fast && ah >= F) {
+      // Isolated queries, 32 per ballot: query j finds the device free (a_j >=
+      // F, resp. a_j >= a_{j-1} + T(1) after its predecessor went alone) and no
+      // other query queued (a_{j+1} > a_j), so it leaves alone at a_j: latency
+      // T(1) <= L -- the Nexus window test passes and AIMD sees no timeout.
+      const int64_t j = h + lane;
+      const int64_t aj = j < n ? A(j) : 0;
+      const int64_t ap = __shfl_up_sync(0xffffffffu, aj, 1);
+      int64_t an = __shfl_down_sync(0xffffffffu, aj, 1);
+      if (lane == 31) an = j + 1 < n ? A(j + 1) : INT64_MAX;
+      if (j + 1 >= n) an = INT64_MAX;
+      const bool iso = j < n && an > aj && (lane == 0 || aj >= ap + T1);
+      const unsigned m = __ballot_sync(0xffffffffu, iso);
+      const int r = __ffs(~m) - 1 < 0 ? 32 : __ffs(~m) - 1;
+      if (r > 0) {
+        if (lane < r) out[j] = (uint32_t)T1;
+        F = __shfl_sync(0xffffffffu, aj, r - 1) + T1;
+        if (!nexus) limit = limit + r > p.Bmax ? p.Bmax : limit + r;
+        h += r;
+        if (tail < h) tail = h;
+        continue;
+      }
+    }
     const int64_t t = F > ah ? F : ah;
     if (tail <= h) tail = h + 1;
     for (;;) {  // queued at t: arrivals <= t (sorted: the ballot is a prefix)
       const int64_t j = tail + lane;
-      const unsigned m = __ballot_sync(0xffffffffu, j < n && (int64_t)__ldg(arr + j) <= t);
+      const unsigned m = __ballot_sync(0xffffffffu, j < n && A(j) <= t);
       tail += __popc(m);
       if (m != 0xffffffffu) break;
     }
@@ -434,8 +490,8 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
         const int64_t i = i0 + lane;
         bool pass = false;
         if (i < tail) {
-          const int64_t w = tail - i < B ? tail - i : B;
-          pass = t + __ldg(T + w - 1) <= (int64_t)__ldg(arr + i) + p.L;
+          const int64_t wl = tail - i < B ? tail - i : B;
+          pass = t + T[wl - 1] <= A(i) + p.L;
         }
         const unsigned m = __ballot_sync(0xffffffffu, pass);
         const int nd = m ? __ffs(m) - 1 : 32;
@@ -444,9 +500,10 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
       }
       if (first < 0) { h = tail; continue; }  // everything queued was dropped
     }
-    const int b = (int)(tail - first < (nexus ? B : limit) ? tail - first : (nexus ? B : limit));
-    F = t + __ldg(T + b - 1);
-    for (int k = lane; k < b; k += 32) out[first + k] = sat_lat(F - (int64_t)__ldg(arr + first + k));
+    const int cap = nexus ? B : limit;
+    const int b = (int)(tail - first < cap ? tail - first : cap);
+    F = t + T[b - 1];
+    for (int k = lane; k < b; k += 32) out[first + k] = sat_lat(F - A(first + k));
     if (!nexus) {  // completion feedback (the next decision is at >= F)
       if (F - ah > p.L) limit = limit * 9 / 10 < 1 ? 1 : limit * 9 / 10;
       else limit = limit + 1 > p.Bmax ? p.Bmax : limit + 1;
@@ -481,7 +538,7 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   if (c >= nch || (a.scan1 && p.Bmax == 1)) return;
   const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
   uint32_t *out = a.latd + (size_t)s * a.NS + off;
-  int64_t h = st, F = 0;
+  int64_t h = st, F = 0, eF = 0, edh = 0;
   if (p.Bmax < 1) {
     for (int64_t j = st; j < en; j++) out[j] = 0xFFFFFFFFu;
     h = en;
@@ -489,17 +546,24 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
     const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
     GArr arr{a.devArr + off};
     unsigned nfull = 0, ndec = 0;
+    // warm-up: the run starts idle WU queries before the chunk, so that by the
+    // chunk it has usually merged with the true run; the chunk's stored run is
+    // the part from its first batch head >= st (entry st + edh, free time eF);
+    // a batch straddling st writes the chunk's positions it covers
+    h = c > 0 ? (st - a.WU > 0 ? st - a.WU : 0) : st;
+    bool entered = h == st;
     while (h < en) {
+      if (!entered && h >= st) { entered = true; edh = h - st; eF = F; }
       int64_t t;
       const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
-      nfull += b == p.Bmax && t == F;
-      ndec++;
+      if (entered) { nfull += b == p.Bmax && t == F; ndec++; }
       const int64_t Fn = t + T[b - 1];
-      const int64_t jend = h + b < en ? h + b : en;
-      for (int64_t j = h; j < jend; j++) out[j] = sat_lat(Fn - (int64_t)arr(j));
+      const int64_t jlo = h > st ? h : st, jend = h + b < en ? h + b : en;
+      for (int64_t j = jlo; j < jend; j++) out[j] = sat_lat(Fn - (int64_t)arr(j));
       F = Fn;
       h += b;
     }
+    if (!entered) { edh = h - st; eF = F; }  // a warm-up batch covered the whole chunk
     unsigned *ls = a.lstat + 2 * ((size_t)s * a.D + d);
     if (nfull) atomicAdd(ls, nfull);
     atomicAdd(ls + 1, ndec);
@@ -507,8 +571,8 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   ChunkSt e;
   e.xF = F;
   e.xov = (int32_t)(h - en);
-  e.eF = 0;
-  e.edh = 0;
+  e.eF = eF;
+  e.edh = (int32_t)edh;
   a.cs[(size_t)s * a.NCH + a.choff[d] + c] = e;
 }
 
@@ -1728,6 +1792,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     memset(&la, 0, sizeof la);
     la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.nsc = (int)scl[2 + rt].size(); la.CH = CH;
     la.N = N; la.NS = NS; la.NCH = nmax;  // one row stride for both routing modes
+    la.WU = env_int("PROTEUS_REPLAY_WARMUP", 0);
+    la.WU = la.WU < 0 ? 0 : la.WU;
     la.option = d_opt; la.dev_type = d_dev; la.lat = ctx->d_lat; la.sc_list = d_scl + (2 + rt) * S; la.lp = d_lp;
     la.devOff = devOff[rt]; la.choff = d_choff + rt * (PX_MAXD + 2); la.goff = d_goff + rt * (PX_MAXD + 2);
     la.devArr = devArr[rt]; la.latd = latd; la.cs = csb[0]; la.csp = nullptr; la.agg = d_agg;

@@ -41,7 +41,12 @@ PATHS = {"chunked": {}, "small_chunks": {"PROTEUS_REPLAY_CHUNK": "16"}, "odd_chu
                                        "PROTEUS_REPLAY_BSCAN": "1"},
          "backlog_scan": {"PROTEUS_REPLAY_BSCAN": "1"},
          "chunk_300": {"PROTEUS_REPLAY_CHUNK": "300"},
-         "simple": {"PROTEUS_REPLAY_SIMPLE": "1"}}
+         "simple": {"PROTEUS_REPLAY_SIMPLE": "1"},
+         "warmup": {"PROTEUS_REPLAY_WARMUP": "4096"},
+         "warmup_small_chunks": {"PROTEUS_REPLAY_CHUNK": "37", "PROTEUS_REPLAY_WARMUP": "50"},
+         "warmup_long_small_chunks": {"PROTEUS_REPLAY_CHUNK": "16", "PROTEUS_REPLAY_WARMUP": "1000"},
+         "warmup_rounds": {"PROTEUS_REPLAY_ROUNDS": "3", "PROTEUS_REPLAY_CHUNK": "64", "PROTEUS_REPLAY_WARMUP": "100"},
+         "warmup_bscan": {"PROTEUS_REPLAY_BSCAN": "1", "PROTEUS_REPLAY_CHUNK": "200", "PROTEUS_REPLAY_WARMUP": "300"}}
 
 
 @pytest.mark.parametrize("path", sorted(PATHS))
