@@ -71,6 +71,9 @@ def lib():
         L.orc_replay.argtypes = [C.c_int64, u32p, u8p, C.c_int, C.c_int, i32p, i32p, C.c_int, i32p,
                                  C.c_int, i32p, i32p, i32p, i32p, i32p, C.c_int, i32p, C.c_int,
                                  C.c_void_p, u64p, u64p, u64p]
+        L.orc_replay_epochs.argtypes = [C.c_int64, u32p, u8p, C.c_int, C.c_int64, C.c_int, C.c_int, i32p, i32p,
+                                        C.c_int, i32p, C.c_int, i32p, i32p, i32p, i32p, i32p, C.c_int, i32p,
+                                        C.c_void_p, u64p, u64p, u64p]
         L.orc_pareto.argtypes = [C.c_int, i32p, C.c_int, i32p, i32p, C.c_int, C.c_int, C.c_int, C.c_int64,
                                  i64p, i64p, u64p, C.POINTER(C.c_uint64), C.POINTER(C.c_int64)]
         _lib = L
@@ -234,6 +237,44 @@ def replay(prof, device_type, option, z, demand, slo_base, arrival_us, family, s
                           lat.ctypes.data if lat is not None else None, viol, ont, accs)
     if rc != 0:
         raise RuntimeError(f"orc_replay returned {rc}")
+    return dict(latency=lat, violations=viol, on_time=ont, acc_sum=accs)
+
+
+def replay_device_epochs(arrival_us, epoch, Tprocs, Bmaxs, Ls):
+    """§8(f4) one device across allocation epochs (readings F3-F4): epoch[j]
+    of query j, Tprocs[e] = T(b) row (index b), Bmaxs[e], Ls[e]."""
+    a = np.ascontiguousarray(arrival_us, dtype=np.uint32)
+    ep = _i32(epoch)
+    E = len(Bmaxs)
+    rows = [_i32(t) for t in Tprocs]
+    ptrs = (C.POINTER(C.c_int32) * E)(*[r.ctypes.data_as(C.POINTER(C.c_int32)) for r in rows])
+    lat = np.zeros(len(a), np.uint32)
+    L = np.ascontiguousarray(np.asarray(Ls, dtype=np.int64))
+    f = lib().orc_replay_device_epochs
+    f.argtypes = [C.c_int64, u32p, i32p, C.POINTER(C.POINTER(C.c_int32)), i32p, i64p, u32p]
+    rc = f(len(a), a, ep, ptrs, _i32(Bmaxs), L, lat)
+    assert rc == 0
+    return lat
+
+
+def replay_epochs(prof, device_type, option, z, demand, slo_base, arrival_us, family, epoch_us, scenarios,
+                  want_latency=True):
+    """§8(f4) closed-loop replay: option/z [E][D] and demand [E][Q] per epoch
+    (readings F1-F4).  Returns dict(latency, violations, on_time, acc_sum)."""
+    a = np.ascontiguousarray(arrival_us, dtype=np.uint32)
+    f = np.ascontiguousarray(family, dtype=np.uint8)
+    sc = scenario_rows(scenarios)
+    opt = _i32(option)
+    E, D = opt.shape
+    S, N = sc.shape[0], len(a)
+    lat = np.zeros((S, N), np.uint32) if want_latency else None
+    viol, ont, accs = np.zeros(S, np.uint64), np.zeros(S, np.uint64), np.zeros(S, np.uint64)
+    rc = lib().orc_replay_epochs(N, a, f, E, int(epoch_us), prof.T, prof.Q, _i32(prof.V), _i32(prof.acc_micro),
+                                 prof.bmax, _i32(prof.lat_us), D, opt, _i32(z), _i32(device_type), _i32(demand),
+                                 _i32(slo_base), S, sc, lat.ctypes.data if lat is not None else None,
+                                 viol, ont, accs)
+    if rc != 0:
+        raise RuntimeError(f"orc_replay_epochs returned {rc}")
     return dict(latency=lat, violations=viol, on_time=ont, acc_sum=accs)
 
 

@@ -27,6 +27,9 @@
  *                         Nexus early drop and Clipper AIMD, work-conserving,
  *                         event-driven; readings R14-R15
  *   orc_replay            route + simulate every (device, scenario) lane
+ *   orc_replay_device_epochs / orc_replay_epochs
+ *                         §8(f4) closed loop: one allocation per epoch (the
+ *                         per-second re-solve), epoch-aware queues; F1-F4
  *   orc_pareto            system capacity vs capacity-weighted accuracy of
  *                         every placement of one family's variants, and its
  *                         Pareto frontier (Fig. 1b), readings P1-P4
@@ -1060,6 +1063,159 @@ int orc_replay(int64_t N, const uint32_t *arrival, const uint8_t *family,
   for (int i = 0; i < nth; i++) pthread_join(th[i], NULL);
   free(th);
   for (int rt = 0; rt < 2; rt++) { free(c.target[rt]); free(c.dev_start[rt]); free(c.idx_of_dev[rt]); }
+  return 0;
+}
+
+/* ------------------------------------------------------- §8(f4) loop -- */
+/* Closed loop (P:707-723 re-allocation, P:1369-1370 period,
+ * P:192-203 per-second demand changes).  Readings F1-F4:
+ *   F1  time is cut into epochs of epoch_us; query i belongs to epoch
+ *       floor(a_i / epoch_us), which must be < E;
+ *   F2  epoch e runs allocation e (option[e][D], z[e][D]) solved by the
+ *       caller for demand[e][Q] (the controller's estimate: the bench uses the
+ *       previous epoch's observed counts); routing restarts each epoch: SWRR
+ *       over z[e] with the sink weight demand[e][q] - sum z (R8), its state
+ *       reset at the epoch start;
+ *   F3  switching costs nothing (C14) but a device finishes the queue of one
+ *       epoch with that epoch's variant before serving queries of the next:
+ *       a batch holds queries of one epoch only, later-epoch queries wait;
+ *   F4  the §5 rule (R1-R13) applies to the head's epoch: q counts the queued
+ *       queries of the head's epoch, T, Bmax and L are that epoch's.
+ *
+ * One device, event-driven like orc_replay_device.  ep[j] = epoch of query j
+ * (non-decreasing); Tp[e] = that epoch's T(b) row (index b), Bm[e], L[e]. */
+int orc_replay_device_epochs(int64_t n, const uint32_t *a, const int32_t *ep, const int32_t *const *Tp,
+                             const int32_t *Bm, const int64_t *L, uint32_t *lat) {
+  if (n == 0) return 0;
+  const int64_t INF = INT64_MAX / 4;
+  int64_t head = 0, tail = 0;
+  int64_t F = 0;
+  int busy = 0, armed = 0;
+  int64_t timer = 0;
+  while (head < n) {
+    int64_t te = INF;
+    if (tail < n && (int64_t)a[tail] < te) te = a[tail];
+    if (busy && F < te) te = F;
+    if (armed && timer < te) te = timer;
+    int64_t t = te;
+    while (tail < n && (int64_t)a[tail] <= t) tail++;
+    if (busy && F <= t) busy = 0;
+    if (busy || tail == head) continue;
+    const int e = ep[head];
+    if (Bm[e] < 1) return -1;
+    int64_t q = 0;                   /* queued queries of the head's epoch */
+    while (head + q < tail && ep[head + q] == e) q++;
+    int64_t b = 0;
+    if (q >= Bm[e]) b = Bm[e];
+    else {
+      int64_t W = (int64_t)a[head] + L[e] - Tp[e][q + 1];
+      if (t >= W) b = q;
+      else { armed = 1; timer = W; }
+    }
+    if (b) {
+      F = t + Tp[e][b];
+      for (int64_t j = head; j < head + b; j++) {
+        int64_t l = F - (int64_t)a[j];
+        lat[j] = l >= (int64_t)UINT32_MAX ? UINT32_MAX - 1 : (uint32_t)l;
+      }
+      head += b;
+      busy = 1;
+      armed = 0;
+    }
+  }
+  return 0;
+}
+
+/* Full closed-loop replay: route every epoch, simulate every (device,
+ * scenario) lane across the epochs, count per scenario (violation: latency >
+ * the query's epoch SLO, R6; accuracy of the serving epoch's variant, R9).
+ * Scenarios as orc_replay ([S][4]); routing must be 0 and policy 0. */
+int orc_replay_epochs(int64_t N, const uint32_t *arrival, const uint8_t *family, int E, int64_t epoch_us,
+                      int T, int Q, const int32_t *V, const int32_t *acc, int bmax, const int32_t *lat_tab,
+                      int D, const int32_t *option, const int32_t *z, const int32_t *dev_type,
+                      const int32_t *demand, const int32_t *slo_base, int S, const int32_t *sc,
+                      uint32_t *latency, uint64_t *viol, uint64_t *ontime, uint64_t *accsum) {
+  (void)T;
+  int M = 0;
+  for (int q = 0; q < Q; q++) M += V[q];
+  if (M > 4096 || D > ORC_MAXD || E < 1 || epoch_us < 1) return -1;
+  for (int s = 0; s < S; s++) if (sc[s * 4 + 2] != 0 || sc[s * 4 + 3] != 0) return -1;
+  for (int64_t i = 1; i < N; i++) if (arrival[i] < arrival[i - 1]) return -5;
+  int32_t *fam_m = (int32_t *)malloc(sizeof(int32_t) * M);
+  { int m = 0; for (int q = 0; q < Q; q++) for (int v = 0; v < V[q]; v++) fam_m[m++] = q; }
+  int32_t *ep = (int32_t *)malloc(sizeof(int32_t) * (N ? N : 1));
+  int32_t *target = (int32_t *)malloc(sizeof(int32_t) * (N ? N : 1));
+  for (int64_t i = 0; i < N; i++) {
+    int64_t e = (int64_t)arrival[i] / epoch_us;
+    if (e >= E) { free(fam_m); free(ep); free(target); return -5; }
+    ep[i] = (int32_t)e;
+  }
+  /* F2: route each epoch's queries with a fresh SWRR over that epoch's weights */
+  for (int64_t i0 = 0; i0 < N;) {
+    int64_t i1 = i0;
+    while (i1 < N && ep[i1] == ep[i0]) i1++;
+    const int e = ep[i0];
+    int32_t dev_family[ORC_MAXD], wdev[ORC_MAXD], wsink[ORC_MAXQ];
+    for (int q = 0; q < Q; q++) wsink[q] = demand[(size_t)e * Q + q];
+    for (int d = 0; d < D; d++) {
+      const int o = option[(size_t)e * D + d];
+      dev_family[d] = o > 0 ? fam_m[o - 1] : -1;
+      wdev[d] = o > 0 ? z[(size_t)e * D + d] : 0;
+      if (o > 0) wsink[dev_family[d]] -= wdev[d];
+    }
+    for (int q = 0; q < Q; q++) if (wsink[q] < 0) { free(fam_m); free(ep); free(target); return -1; }
+    orc_route_swrr(i1 - i0, family + i0, Q, D, dev_family, wdev, wsink, target + i0);
+    i0 = i1;
+  }
+  for (int s = 0; s < S; s++) { viol[s] = 0; ontime[s] = 0; accsum[s] = 0; }
+  uint32_t *a = (uint32_t *)malloc(sizeof(uint32_t) * (N ? N : 1));
+  uint32_t *l = (uint32_t *)malloc(sizeof(uint32_t) * (N ? N : 1));
+  int32_t *eq = (int32_t *)malloc(sizeof(int32_t) * (N ? N : 1));
+  int64_t *idx = (int64_t *)malloc(sizeof(int64_t) * (N ? N : 1));
+  const int32_t **Tp = (const int32_t **)malloc(sizeof(int32_t *) * E);
+  int32_t *Tbuf = (int32_t *)malloc(sizeof(int32_t) * (size_t)E * (bmax + 1));
+  int32_t *Bm = (int32_t *)malloc(sizeof(int32_t) * E);
+  int64_t *Lv = (int64_t *)malloc(sizeof(int64_t) * E);
+  for (int s = 0; s < S; s++) {
+    for (int d = 0; d <= D; d++) {
+      int64_t n = 0;
+      for (int64_t i = 0; i < N; i++)
+        if (target[i] == d) { a[n] = arrival[i]; eq[n] = ep[i]; idx[n] = i; n++; }
+      if (d == D) {                  /* the sinks: dropped (R7) */
+        viol[s] += (uint64_t)n;
+        if (latency) for (int64_t k = 0; k < n; k++) latency[(size_t)s * N + idx[k]] = UINT32_MAX;
+        continue;
+      }
+      if (n == 0) continue;
+      for (int e = 0; e < E; e++) {  /* this device's variant in every epoch */
+        const int o = option[(size_t)e * D + d];
+        int32_t *row = Tbuf + (size_t)e * (bmax + 1);
+        Tp[e] = row;
+        Bm[e] = 0; Lv[e] = 0; row[0] = 0;
+        if (o <= 0) continue;
+        const int32_t *tr = lat_tab + ((size_t)dev_type[d] * M + o - 1) * bmax;
+        int dep = 0;
+        while (dep < bmax && tr[dep] > 0) dep++;
+        for (int b = 1; b <= dep; b++) row[b] = tr[b - 1];
+        const int cap = sc[s * 4 + 1];
+        Bm[e] = (cap > 0 && cap < dep) ? cap : dep;
+        Lv[e] = (int64_t)sc[s * 4 + 0] * slo_base[fam_m[o - 1]] / 1000;
+      }
+      if (orc_replay_device_epochs(n, a, eq, Tp, Bm, Lv, l) != 0) {
+        free(fam_m); free(ep); free(target); free(a); free(l); free(eq); free(idx); free(Tp); free(Tbuf);
+        free(Bm); free(Lv);
+        return -1;
+      }
+      for (int64_t k = 0; k < n; k++) {
+        const int e = eq[k], m = option[(size_t)e * D + d] - 1;
+        if ((int64_t)l[k] > Lv[e]) viol[s]++;
+        else { ontime[s]++; accsum[s] += (uint64_t)acc[m]; }
+        if (latency) latency[(size_t)s * N + idx[k]] = l[k];
+      }
+    }
+  }
+  free(fam_m); free(ep); free(target); free(a); free(l); free(eq); free(idx); free(Tp); free(Tbuf); free(Bm);
+  free(Lv);
   return 0;
 }
 

@@ -196,6 +196,31 @@ def query_trace(n: int, rate_qps: float, weights: np.ndarray, seed: int, kind: s
     return arr.astype(np.uint32), fam
 
 
+def epoch_trace(counts: np.ndarray, epoch_us: int, seed: int):
+    """Arrivals for per-epoch family counts [E][Q] (§8(f4)): counts[e][q]
+    queries of family q uniformly at random in epoch e (a Poisson process
+    conditioned on its count: "Poisson inter-arrivals within each second",
+    P:1155-1157), merged and sorted.  Returns (uint32 us, uint8 family)."""
+    rng = np.random.default_rng(seed)
+    E, Q = counts.shape
+    if E * epoch_us >= UINT32_MAX:
+        raise ValueError("trace longer than 2^32 us")
+    tot = counts.sum(axis=1)
+    ep = np.repeat(np.arange(E, dtype=np.int64), tot)
+    fam = np.concatenate([np.repeat(np.arange(Q, dtype=np.uint8), counts[e]) for e in range(E)]) if E else \
+        np.zeros(0, np.uint8)
+    t = ep * epoch_us + rng.integers(0, epoch_us, size=len(ep))
+    order = np.lexsort((rng.random(len(ep)), t))
+    return t[order].astype(np.uint32), fam[order].astype(np.uint8)
+
+
+def controller_demand(counts: np.ndarray) -> np.ndarray:
+    """The controller's estimate for epoch e: the counts observed in epoch
+    e - 1 (epoch 0: its own), per-second re-solve on the last second's
+    statistics (P:707-719)."""
+    return np.concatenate([counts[:1], counts[:-1]]).astype(np.int32)
+
+
 # -------------------------------------------------------------- scenarios --
 SLO_MULTS_MILLI = (1000, 1500, 2000, 2500, 3000, 3500, 4000, 5000)   # covers P:1817-1818
 BATCH_CAPS = (1, 2, 4, 8, 16, 32, 64, 0)                               # 1 = "w/o AB" (P:1789); 0 = table depth
@@ -270,6 +295,20 @@ def config(name: str, **kw) -> dict:
         arr, fam = query_trace(n, rate, w, 505, kw.get("kind", "poisson"))
         return dict(name=name, prof=prof, cluster=cl, demand=dem, arrival_us=arr, family=fam,
                     scenarios=scenarios_64(kw.get("routing", 0)), weights=w)
+    elif name == "f4":
+        # §8(f4) closed loop on the c4 demand: every epoch's true counts make
+        # the trace; the controller solves epoch e on epoch e - 1's counts
+        prof = make_profiles(303, ("cpu", "gpu_a", "gpu_b"), C3_FAMILIES, bmax=64)
+        cl = Cluster(cluster_types((10, 5, 5)), slo_from_cpu_rule(prof))
+        w = zipf_weights(prof.Q, 303)
+        E = kw.get("n_seconds", 3600)
+        counts = demand_trace(E, kw.get("lam_mid", C4_LAM_MID), w, 404)
+        epoch_us = kw.get("epoch_us", 1_000_000)
+        arr, fam = epoch_trace(counts, epoch_us, 606)
+        return dict(name=name, prof=prof, cluster=cl, counts=counts, demand=controller_demand(counts),
+                    arrival_us=arr, family=fam, epoch_us=epoch_us, weights=w,
+                    scenarios=np.array([(m, c, 0, 0) for m in (1000, 2000, 3000, 5000) for c in (8, 32, 0)],
+                                       np.int32))
     else:
         raise ValueError(name)
     return dict(name=name, prof=prof, cluster=cl, demand=dem, weights=w)
