@@ -300,6 +300,33 @@ int proteus_replay(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *
                    const proteus_scenario *sc, int32_t S,
                    uint32_t *latency_us, uint64_t *violations, uint64_t *on_time, uint64_t *acc_sum);
 
+/* ------------------------------------------------------ closed loop --
+ * §8(f4): the per-second re-solve (the paper re-solves
+ * every 30 s) feeding the replay.  Time is cut into E epochs of
+ * epoch_us; epoch e runs allocation e (typically proteus_solve_batch's
+ * outputs for the controller's demand estimates, left on the device).
+ * Readings F1-F4:
+ *   F1  query i belongs to epoch floor(arrival_us[i] / epoch_us) < E
+ *       (PROTEUS_ERANGE otherwise);
+ *   F2  routing restarts every epoch: SWRR over z[e] of the devices hosting
+ *       the family with the sink weight demand[e][q] - sum z (R8);
+ *   F3  switching is free (C14) but a device finishes the queue of one epoch
+ *       with that epoch's variant before serving the next epoch's queries: a
+ *       batch holds queries of one epoch;
+ *   F4  the §5 rule (R1-R13) with the head's epoch's variant T(b), Bmax and
+ *       SLO; violations and accuracy use the query's epoch's variant.
+ *   arrival_us[N], family[N]   as proteus_replay
+ *   option[E][D], z_qps[E][D]  allocation per epoch (row-major)
+ *   demand_qps[E][Q]           the demand each allocation was solved for
+ *   device_type[D], slo_base_us[Q], sc[S]   as proteus_replay; every scenario
+ *                  must have routing 0 and policy 0 (PROTEUS_EINVAL otherwise)
+ * Outputs as proteus_replay. */
+int proteus_replay_epochs(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *family, int64_t N,
+                          int32_t E, int64_t epoch_us, const int32_t *option, const int32_t *z_qps,
+                          const int32_t *device_type, int32_t D, const int32_t *demand_qps,
+                          const int32_t *slo_base_us, const proteus_scenario *sc, int32_t S, uint32_t *latency_us,
+                          uint64_t *violations, uint64_t *on_time, uint64_t *acc_sum);
+
 /* ------------------------------------------------------- instrumentation --
  * proteus_set_timing(ctx, 1) makes later calls record CUDA events around
  * every kernel they launch (on the context's stream).  proteus_kernel_times

@@ -242,6 +242,64 @@ class Proteus:
             res.update(violations=out[0], on_time=out[1], acc_sum=out[2])
         return res
 
+    # --------------------------------------------------------- closed loop --
+    def replay_epochs(self, arrival_us, family, epoch_us, option, z, device_type, demand, slo_base_us, scenarios,
+                      latency=True, aggregates_out=None):
+        """§8(f4) closed-loop replay (proteus_replay_epochs): option / z
+        [E][D] and demand [E][Q], one allocation per epoch of epoch_us
+        (numpy or CUDA tensors).  latency / aggregates_out as replay()."""
+        keep = []
+        sc = np.asarray(scenarios, dtype=np.int32)
+        sc = sc.reshape(-1, sc.shape[-1])
+        if sc.shape[1] == 3:
+            sc = np.concatenate([sc, np.zeros((sc.shape[0], 1), np.int32)], axis=1)
+        S = sc.shape[0]
+        scs = (N.proteus_scenario * S)(*[N.proteus_scenario(*map(int, row)) for row in sc])
+        n = int(arrival_us.shape[0]) if hasattr(arrival_us, "shape") else len(arrival_us)
+        E, D = int(option.shape[0]), int(option.shape[1])
+        lat_np = None
+        if latency is True:
+            lat_np = np.empty((S, n), np.uint32)
+            lat_ptr = lat_np.ctypes.data
+        elif latency is None or latency is False:
+            lat_ptr = None
+        else:
+            lat_ptr = _arg(latency, np.uint32, keep)
+        if aggregates_out is not None:
+            viol, ont, accs = (_arg(aggregates_out[k], np.uint64, keep) for k in range(3))
+            out = None
+        else:
+            out = np.zeros((3, S), np.uint64)
+            viol, ont, accs = out[0].ctypes.data, out[1].ctypes.data, out[2].ctypes.data
+        rc = self._lib.proteus_replay_epochs(
+            self._h, _arg(arrival_us, np.uint32, keep), _arg(family, np.uint8, keep), n, E, int(epoch_us),
+            _arg(option, np.int32, keep), _arg(z, np.int32, keep), _arg(device_type, np.int32, keep), D,
+            _arg(demand, np.int32, keep), _arg(slo_base_us, np.int32, keep), scs, S, lat_ptr, viol, ont, accs)
+        self._check(rc)
+        res = {"latency": lat_np if latency is True else latency}
+        if out is not None:
+            res.update(violations=out[0], on_time=out[1], acc_sum=out[2])
+        return res
+
+    def closed_loop(self, arrival_us, family, epoch_us, demand, device_type, slo_us, scenarios, latency=True,
+                    device=None):
+        """§8(f4): per-epoch re-solve (factored, batched) of the controller's
+        demand estimates [E][Q] feeding the closed-loop replay; with CUDA
+        tensors (or `device`) the allocations stay on the GPU between the two
+        calls.  Returns (replay result dict, allocation dict)."""
+        E = int(demand.shape[0])
+        D = len(device_type)
+        if device is not None:
+            import torch
+            alloc = {"option": torch.empty((E, D), dtype=torch.int32, device=device),
+                     "z_qps": torch.empty((E, D), dtype=torch.int32, device=device)}
+        else:
+            alloc = {"option": np.empty((E, D), np.int32), "z_qps": np.empty((E, D), np.int32)}
+        self.solve_batch(device_type, slo_us, demand, mode=MODE_FACTORED, out=alloc)
+        res = self.replay_epochs(arrival_us, family, epoch_us, alloc["option"], alloc["z_qps"], device_type, demand,
+                                 slo_us, scenarios, latency=latency)
+        return res, alloc
+
     # ----------------------------------------------------- instrumentation --
     def set_timing(self, on=True):
         self._check(self._lib.proteus_set_timing(self._h, 1 if on else 0))

@@ -21,7 +21,7 @@ PROTEUS_SOLVE_GENERIC = 1
 EXPORTED = (
     "proteus_abi_version", "proteus_create", "proteus_destroy", "proteus_set_stream", "proteus_last_error",
     "proteus_load_profiles", "proteus_solve", "proteus_solve_batch", "proteus_materialize", "proteus_candidate_count",
-    "proteus_pareto", "proteus_replay", "proteus_set_timing", "proteus_kernel_times", "proteus_launch_count",
+    "proteus_pareto", "proteus_replay", "proteus_replay_epochs", "proteus_set_timing", "proteus_kernel_times", "proteus_launch_count",
 )
 
 
@@ -97,6 +97,8 @@ def load(path: str = LIB_PATH):
                                  C.POINTER(i32), C.POINTER(u64)]
     L.proteus_replay.argtypes = [vp, vp, vp, i64, vp, vp, vp, i32, vp, vp, C.POINTER(proteus_scenario), i32,
                                  vp, vp, vp, vp]
+    L.proteus_replay_epochs.argtypes = [vp, vp, vp, i64, i32, i64, vp, vp, vp, i32, vp, vp,
+                                        C.POINTER(proteus_scenario), i32, vp, vp, vp, vp]
     L.proteus_set_timing.argtypes = [vp, C.c_int]
     L.proteus_kernel_times.argtypes = [vp, C.POINTER(C.c_char_p), C.POINTER(C.c_float), C.c_int]
     L.proteus_launch_count.argtypes = [vp]

@@ -617,4 +617,86 @@ int proteus_replay(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *
   return PROTEUS_OK;
 }
 
+// -------------------------------------------------------- closed loop -----
+int proteus_replay_epochs(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *family, int64_t N,
+                          int32_t E, int64_t epoch_us, const int32_t *option, const int32_t *z_qps,
+                          const int32_t *device_type, int32_t D, const int32_t *demand_qps,
+                          const int32_t *slo_base_us, const proteus_scenario *sc, int32_t S, uint32_t *latency_us,
+                          uint64_t *violations, uint64_t *on_time, uint64_t *acc_sum) {
+  if (!ctx) return PROTEUS_EINVAL;
+  ctx->err.clear();
+  if (!ctx->have_prof) return px_fail(ctx, PROTEUS_EINVAL, "no profiles loaded");
+  if (N < 0 || (N > 0 && (!arrival_us || !family))) return px_fail(ctx, PROTEUS_EINVAL, "trace");
+  if (N >= (1ll << 32)) return px_fail(ctx, PROTEUS_ERANGE, "N >= 2^32");
+  if (E < 1 || E > (1 << 24) || epoch_us < 1) return px_fail(ctx, PROTEUS_EINVAL, "E=%d epoch_us=%lld", E, (long long)epoch_us);
+  if (D < 1 || D > PX_MAXD || !option || !z_qps || !device_type || !demand_qps || !slo_base_us)
+    return px_fail(ctx, PROTEUS_EINVAL, "allocation arguments");
+  if (S < 1 || S > 4096 || !sc) return px_fail(ctx, PROTEUS_EINVAL, "S=%d", S);
+  PX_CUDA(ctx, cudaSetDevice(ctx->device));
+  timing_reset(ctx);
+  int rc;
+  std::vector<int32_t> opt, z, dev, dem, slo;
+  std::vector<proteus_scenario> scv;
+  if ((rc = to_host(ctx, option, (size_t)E * D, opt)) || (rc = to_host(ctx, z_qps, (size_t)E * D, z)) ||
+      (rc = to_host(ctx, device_type, D, dev)) || (rc = to_host(ctx, demand_qps, (size_t)E * ctx->Q, dem)) ||
+      (rc = to_host(ctx, slo_base_us, ctx->Q, slo)) || (rc = to_host(ctx, sc, S, scv)))
+    return rc;
+  for (int q = 0; q < ctx->Q; q++)
+    if (slo[q] < 0) return px_fail(ctx, PROTEUS_EINVAL, "negative slo");
+  for (int d = 0; d < D; d++)
+    if (dev[d] < 0 || dev[d] >= ctx->T) return px_fail(ctx, PROTEUS_EINVAL, "device_type[%d]", d);
+  std::vector<int64_t> zsum(ctx->Q);
+  for (int e = 0; e < E; e++) {
+    int64_t dsum = 0;
+    for (int q = 0; q < ctx->Q; q++) {
+      if (dem[(size_t)e * ctx->Q + q] < 0) return px_fail(ctx, PROTEUS_EINVAL, "negative demand");
+      dsum += dem[(size_t)e * ctx->Q + q];
+      zsum[q] = 0;
+    }
+    if (dsum >= (1 << 22)) return px_fail(ctx, PROTEUS_ERANGE, "sum of demand >= 2^22 (epoch %d)", e);
+    for (int d = 0; d < D; d++) {
+      const int32_t o = opt[(size_t)e * D + d], zz = z[(size_t)e * D + d];
+      if (o < 0 || o > ctx->M) return px_fail(ctx, PROTEUS_EINVAL, "option[%d][%d]=%d", e, d, o);
+      if (zz < 0 || (o == 0 && zz != 0)) return px_fail(ctx, PROTEUS_EINVAL, "z[%d][%d]=%d", e, d, zz);
+      if (o) zsum[ctx->fam[o - 1]] += zz;
+    }
+    for (int q = 0; q < ctx->Q; q++)
+      if (zsum[q] > dem[(size_t)e * ctx->Q + q])
+        return px_fail(ctx, PROTEUS_EINVAL, "sum z of family %d exceeds its demand (epoch %d)", q, e);
+  }
+  for (int s = 0; s < S; s++)
+    if (scv[s].slo_mult_milli < 0 || scv[s].batch_cap < 0 || scv[s].routing != 0 || scv[s].policy != 0)
+      return px_fail(ctx, PROTEUS_EINVAL, "scenario %d (closed loop: routing 0, policy 0)", s);
+  const uint32_t *d_arr = to_device(ctx, arrival_us, (size_t)N, B_IN0, &rc);
+  if (rc) return rc;
+  const uint8_t *d_fam = to_device(ctx, family, (size_t)N, B_IN1, &rc);
+  if (rc) return rc;
+  uint32_t *d_lat = nullptr;
+  bool lat_dev = latency_us && px_is_device_ptr(latency_us);
+  if (latency_us) {
+    d_lat = lat_dev ? latency_us : (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S * N * 4);
+    if (!d_lat) return px_fail(ctx, PROTEUS_ENOMEM, "latency buffer");
+  }
+  uint64_t *d_agg = (uint64_t *)px_buf(ctx, B_R_AGG, (size_t)3 * S * 8 + 8);
+  if (!d_agg) return px_fail(ctx, PROTEUS_ENOMEM, "aggregate buffer");
+  rc = px_replay_epochs(ctx, d_arr, d_fam, N, E, epoch_us, opt.data(), z.data(), dev.data(), D, dem.data(),
+                        slo.data(), scv.data(), S, d_lat, d_agg);
+  if (rc) return rc;
+  std::vector<uint64_t> agg((size_t)3 * S + 1);
+  PX_CUDA(ctx, cudaMemcpyAsync(agg.data(), d_agg, ((size_t)3 * S + 1) * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  if (latency_us && !lat_dev)
+    PX_CUDA(ctx, cudaMemcpyAsync(latency_us, d_lat, (size_t)S * N * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  if ((rc = timing_collect(ctx))) return rc;
+  uint64_t *outs[3] = {violations, on_time, acc_sum};
+  for (int k = 0; k < 3; k++) {
+    if (!outs[k]) continue;
+    if (px_is_device_ptr(outs[k]))
+      PX_CUDA(ctx, cudaMemcpy(outs[k], &agg[(size_t)k * S], (size_t)S * 8, cudaMemcpyHostToDevice));
+    else
+      memcpy(outs[k], &agg[(size_t)k * S], (size_t)S * 8);
+  }
+  return PROTEUS_OK;
+}
+
 }  // extern "C"

@@ -111,7 +111,7 @@ struct proteus_ctx {
 enum {
   B_TABLES = 0, B_BEST, B_SOL, B_IN0, B_IN1, B_IN2, B_IN3, B_FACT0, B_FACT1, B_FACT2, B_FACT3,
   B_R_PAT, B_R_TGT, B_R_HIST, B_R_BASE, B_R_DEVARR, B_R_DEVIDX, B_R_OFF, B_R_LAT, B_R_AGG, B_R_TGT1,
-  B_R_DEVARR1, B_R_DEVIDX1, B_R_OFF1, B_R_MISC, B_R_LANE, B_R_DBASE0, B_R_DBASE1, B_R_LATD, B_R_VLAT, B_R_VEX, B_R_VOFF, B_FACT4, B_R_SCAN, B_R_BSCAN, B_PARETO, B_NBUF
+  B_R_DEVARR1, B_R_DEVIDX1, B_R_OFF1, B_R_MISC, B_R_LANE, B_R_DBASE0, B_R_DBASE1, B_R_LATD, B_R_VLAT, B_R_VEX, B_R_VOFF, B_FACT4, B_R_SCAN, B_R_BSCAN, B_PARETO, B_E_MISC, B_E_PAT, B_E_EXIT, B_NBUF
 };
 static_assert(B_NBUF <= 48, "proteus_ctx::bufs is too small");
 
@@ -157,3 +157,7 @@ int px_pareto(proteus_ctx *ctx, int D, const int32_t *h_dev_type, const int32_t 
 int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int64_t N, const int32_t *h_option,
               const int32_t *h_z, const int32_t *h_dev_type, int D, const int32_t *h_demand, const int32_t *h_slo,
               const proteus_scenario *h_sc, int S, uint32_t *d_lat_out, uint64_t *d_agg /* [3][S] */);
+int px_replay_epochs(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int64_t N, int E,
+                     int64_t epoch_us, const int32_t *h_option, const int32_t *h_z, const int32_t *h_dev_type, int D,
+                     const int32_t *h_demand, const int32_t *h_slo, const proteus_scenario *h_sc, int S,
+                     uint32_t *d_lat_out, uint64_t *d_agg /* [3][S] */);

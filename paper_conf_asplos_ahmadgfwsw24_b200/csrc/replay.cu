@@ -1939,3 +1939,346 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   }
   return 0;
 }
+
+// ============================================================ §8(f4) ======
+// Closed loop (readings F1-F4): allocation e serves the queries
+// arriving in epoch e = floor(a / epoch_us) (the per-second re-solve,
+// P:707-723).  Routing restarts every epoch (SWRR over z[e] with
+// the sink, R8); a device finishes one epoch's queue with that epoch's variant
+// before serving the next epoch's queries (a batch holds one epoch), so a
+// device's array is a sequence of (device, epoch) segments replayed with the
+// §5 rule, the device state F carried from segment to segment.
+//   phase A  every segment from an idle device, in parallel (k_ep_spec);
+//   phase B  per (device, scenario), the true F carried over the epochs: a
+//            segment whose first query arrives at or after F takes exactly the
+//            idle run's decisions (t = max(F, a_head) = a_head) and is kept,
+//            otherwise it is replayed from F (k_ep_stitch).
+
+// SWRR pattern per (epoch, family): weights w[(e * Q + q) * (D + 1) + d] (the
+// sink is member D), one warp per pattern (as k_route_prepare)
+__global__ void k_ep_patterns(int EQ, int D, const int32_t *__restrict__ w, const int64_t *__restrict__ poff,
+                              const int32_t *__restrict__ plen, uint8_t *pattern) {
+  const int eq = blockIdx.x, lane = threadIdx.x;
+  if (eq >= EQ) return;
+  const int32_t Wq = plen[eq];
+  int32_t wl[3], cur[3];
+#pragma unroll
+  for (int i = 0; i < 3; i++) {
+    const int d = lane + 32 * i;
+    wl[i] = d <= D ? w[(size_t)eq * (D + 1) + d] : 0;
+    cur[i] = 0;
+  }
+  uint8_t *pat = pattern + poff[eq];
+  for (int32_t k = 0; k < Wq; k++) {
+    long long key = LLONG_MIN;
+#pragma unroll
+    for (int i = 0; i < 3; i++) {
+      if (wl[i] == 0) continue;
+      cur[i] += wl[i];
+      const long long kk = ((long long)cur[i] << 32) | (0xFFFFFFFFu - (uint32_t)(lane + 32 * i));
+      key = kk > key ? kk : key;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      const long long v = __shfl_xor_sync(0xffffffffu, key, o);
+      key = v > key ? v : key;
+    }
+    const int best = (int)(0xFFFFFFFFu - (uint32_t)(key & 0xFFFFFFFFll));
+#pragma unroll
+    for (int i = 0; i < 3; i++)
+      if (best == lane + 32 * i) cur[i] -= Wq;
+    if (lane == 0) pat[k] = (uint8_t)best;
+  }
+}
+
+// per (epoch, family) counts; flags bit 3: an arrival beyond the last epoch
+__global__ void k_ep_hist(const uint32_t *__restrict__ arr, const uint8_t *__restrict__ fam, int64_t N, int E,
+                          int64_t epoch_us, int Q, int32_t *cntEQ, uint32_t *flags) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t e = (int64_t)arr[i] / epoch_us;
+    if (e >= E) { atomicOr(flags, 8u); continue; }
+    atomicAdd(cntEQ + e * Q + fam[i], 1);
+  }
+}
+
+// family ordinal within the epoch -> target (as k_route_target, the ordinal
+// made epoch-relative by the family's count before the epoch)
+__global__ void k_ep_target(const uint8_t *__restrict__ fam, const uint32_t *__restrict__ arr, int64_t N, int Q,
+                            int64_t epoch_us, const int32_t *__restrict__ famBase, const int32_t *__restrict__ fbEQ,
+                            const uint8_t *__restrict__ pattern, const int64_t *__restrict__ poff,
+                            const int32_t *__restrict__ plen, int D, uint8_t *target, int32_t *histDev) {
+  __shared__ int32_t run[TILE_WARPS][PX_MAXQ];
+  __shared__ int32_t cnt[TILE_WARPS][PX_MAXD + 2];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t tile = (int64_t)blockIdx.x * TILE_WARPS + w;
+  const int64_t t0 = tile * TILE;
+  if (t0 < N)
+    for (int k = lane; k < Q; k += 32) run[w][k] = famBase[tile * Q + k];
+  for (int k = lane; k <= D; k += 32) cnt[w][k] = 0;
+  __syncthreads();
+  if (t0 >= N) return;
+  for (int c = 0; c < TILE; c += 32) {
+    const int64_t i = t0 + c + lane;
+    const bool valid = i < N;
+    const int key = valid ? fam[i] : 255;
+    const unsigned peers = __match_any_sync(0xffffffffu, key);
+    const int rank = __popc(peers & ((1u << lane) - 1));
+    int ord = 0;
+    if (valid) ord = run[w][key] + rank;
+    __syncwarp();
+    if (valid && lane == __ffs(peers) - 1) run[w][key] += __popc(peers);
+    int tgt = D;
+    if (valid) {
+      const int64_t eq = ((int64_t)arr[i] / epoch_us) * Q + key;
+      const int len = plen[eq];
+      tgt = len > 0 ? pattern[poff[eq] + ((ord - fbEQ[eq]) % len)] : D;
+      target[i] = (uint8_t)tgt;
+    }
+    const unsigned tp = __match_any_sync(0xffffffffu, valid ? tgt : 255);
+    if (valid && lane == __ffs(tp) - 1) cnt[w][tgt] += __popc(tp);
+    __syncwarp();
+  }
+  for (int k = lane; k <= D; k += 32) histDev[tile * (D + 1) + k] = cnt[w][k];
+}
+
+// per (epoch, device) segment sizes (the sink is not a segment)
+__global__ void k_ep_seghist(const uint8_t *__restrict__ target, const uint32_t *__restrict__ arr, int64_t N,
+                             int64_t epoch_us, int D, int32_t *cntED) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < N; i += (int64_t)gridDim.x * blockDim.x) {
+    const int d = target[i];
+    if (d < D) atomicAdd(cntED + ((int64_t)arr[i] / epoch_us) * D + d, 1);
+  }
+}
+
+struct EpArgs {
+  int E, D, M, bmax, S;
+  int64_t NS;
+  const int32_t *option;  // [E][D]
+  const int32_t *dev_type, *lat, *acc, *fam_of_m, *slo;
+  const proteus_scenario *sc;
+  const int64_t *devOff;  // [D + 2]
+  const int32_t *cntED, *segBase;  // [E][D]
+  const uint32_t *devArr;
+  uint32_t *latd;         // [S][NS]
+  int64_t *exitF;         // [S][E][D]
+};
+
+struct EpLane {
+  const int32_t *T;
+  int Bmax;
+  int64_t L;
+};
+
+__device__ __forceinline__ EpLane ep_lane(const EpArgs &a, int s, int e, int d) {
+  EpLane r;
+  const int o = a.option[(size_t)e * a.D + d];
+  r.T = a.lat + ((size_t)a.dev_type[d] * a.M + (o - 1)) * a.bmax;
+  int depth = 0;
+  while (depth < a.bmax && r.T[depth] > 0) depth++;
+  const int cap = a.sc[s].batch_cap;
+  r.Bmax = (cap > 0 && cap < depth) ? cap : depth;
+  r.L = (int64_t)a.sc[s].slo_mult_milli * a.slo[a.fam_of_m[o - 1]] / 1000;
+  return r;
+}
+
+// replay one segment [st, st + n) of the device array from free time F; returns the exit F
+__device__ __forceinline__ int64_t ep_walk(const EpArgs &a, int s, int e, int d, int64_t st, int64_t n, int64_t F) {
+  const EpLane p = ep_lane(a, s, e, d);
+  uint32_t *out = a.latd + (size_t)s * a.NS + st;
+  if (p.Bmax < 1) {  // never routed to (z = 0 / depth 0); kept for safety
+    for (int64_t j = 0; j < n; j++) out[j] = 0xFFFFFFFFu;
+    return F;
+  }
+  GArr arr{a.devArr + st};
+  int64_t h = 0;
+  while (h < n) {
+    int64_t t;
+    const int b = decide(arr, n, h, F, p.Bmax, p.L, p.T, &t);
+    F = t + p.T[b - 1];
+    for (int j = 0; j < b; j++) out[h + j] = sat_lat(F - (int64_t)arr(h + j));
+    h += b;
+  }
+  return F;
+}
+
+// phase A: thread per (scenario, epoch, device) segment, from an idle device
+__global__ void __launch_bounds__(128) k_ep_spec(const __grid_constant__ EpArgs a) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int s = blockIdx.y;
+  if (i >= (int64_t)a.E * a.D) return;
+  const int e = (int)(i / a.D), d = (int)(i % a.D);
+  const int32_t n = a.cntED[i];
+  if (n == 0) return;
+  const int64_t st = a.devOff[d] + a.segBase[i];
+  a.exitF[(size_t)s * a.E * a.D + i] = ep_walk(a, s, e, d, st, n, 0);
+}
+
+// phase B: thread per (scenario, device), the true state across the epochs
+__global__ void __launch_bounds__(64) k_ep_stitch(const __grid_constant__ EpArgs a) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= a.S * a.D) return;
+  const int s = i / a.D, d = i % a.D;
+  int64_t F = 0;  // R13
+  for (int e = 0; e < a.E; e++) {
+    const int64_t k = (int64_t)e * a.D + d;
+    const int32_t n = a.cntED[k];
+    if (n == 0) continue;
+    const int64_t st = a.devOff[d] + a.segBase[k];
+    if (F <= (int64_t)a.devArr[st]) F = a.exitF[(size_t)s * a.E * a.D + k];  // idle at the head: kept
+    else F = ep_walk(a, s, e, d, st, n, F);
+  }
+}
+
+// per-scenario counts over the device-major rows (each position's epoch
+// variant gives its SLO and accuracy); the sink segment is written dropped
+__global__ void __launch_bounds__(256) k_ep_count(const __grid_constant__ EpArgs a, int64_t N, int64_t epoch_us,
+                                                  uint64_t *agg) {
+  __shared__ int64_t sOff[PX_MAXD + 2];
+  __shared__ unsigned long long red[3][8];
+  for (int k = threadIdx.x; k <= a.D + 1; k += blockDim.x) sOff[k] = a.devOff[k];
+  __syncthreads();
+  const int s = blockIdx.y;
+  uint32_t *row = a.latd + (size_t)s * a.NS;
+  unsigned long long v = 0, o = 0, ac = 0;
+  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < N; p += (int64_t)gridDim.x * blockDim.x) {
+    int d = 0;
+    while (p >= sOff[d + 1]) d++;
+    if (d == a.D) { row[p] = 0xFFFFFFFFu; v++; continue; }
+    const int e = (int)((int64_t)a.devArr[p] / epoch_us);
+    const int opt = a.option[(size_t)e * a.D + d];
+    const int64_t L = (int64_t)a.sc[s].slo_mult_milli * a.slo[a.fam_of_m[opt - 1]] / 1000;
+    if ((int64_t)row[p] > L) v++;
+    else { o++; ac += (unsigned long long)a.acc[opt - 1]; }
+  }
+  for (int k = 16; k; k >>= 1) {
+    v += __shfl_xor_sync(0xffffffffu, v, k);
+    o += __shfl_xor_sync(0xffffffffu, o, k);
+    ac += __shfl_xor_sync(0xffffffffu, ac, k);
+  }
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) { red[0][w] = v; red[1][w] = o; red[2][w] = ac; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long t[3] = {0, 0, 0};
+    for (int k = 0; k < (int)(blockDim.x >> 5); k++) { t[0] += red[0][k]; t[1] += red[1][k]; t[2] += red[2][k]; }
+    if (t[0]) atomicAdd((unsigned long long *)&agg[s], t[0]);
+    if (t[1]) atomicAdd((unsigned long long *)&agg[a.S + s], t[1]);
+    if (t[2]) atomicAdd((unsigned long long *)&agg[2 * a.S + s], t[2]);
+  }
+}
+
+int px_replay_epochs(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int64_t N, int E,
+                     int64_t epoch_us, const int32_t *h_option, const int32_t *h_z, const int32_t *h_dev_type, int D,
+                     const int32_t *h_demand, const int32_t *h_slo, const proteus_scenario *h_sc, int S,
+                     uint32_t *d_lat_out, uint64_t *d_agg) {
+  const int Q = ctx->Q, M = ctx->M;
+  PX_CUDA(ctx, cudaMemsetAsync(d_agg, 0, ((size_t)3 * S + 1) * 8, ctx->stream));
+  // F2: SWRR weights per (epoch, family) -- members z[e][d] of the hosting devices, the sink
+  const size_t EQ = (size_t)E * Q;
+  std::vector<int32_t> w(EQ * (D + 1), 0), plen(EQ, 0);
+  std::vector<int64_t> poff(EQ + 1, 0);
+  for (int e = 0; e < E; e++) {
+    for (int q = 0; q < Q; q++) w[((size_t)e * Q + q) * (D + 1) + D] = h_demand[(size_t)e * Q + q];
+    for (int d = 0; d < D; d++) {
+      const int o = h_option[(size_t)e * D + d];
+      if (o <= 0) continue;
+      const int q = ctx->fam[o - 1];
+      w[((size_t)e * Q + q) * (D + 1) + d] = h_z[(size_t)e * D + d];
+      w[((size_t)e * Q + q) * (D + 1) + D] -= h_z[(size_t)e * D + d];
+    }
+  }
+  for (size_t k = 0; k < EQ; k++) {
+    int64_t t = 0;
+    for (int d = 0; d <= D; d++) t += w[k * (D + 1) + d];
+    plen[k] = (int32_t)t;
+    poff[k + 1] = poff[k] + t;
+  }
+  const size_t small = EQ * (D + 1) * 4 + EQ * 4 + (EQ + 1) * 8 + (size_t)E * D * 4 * 4 + EQ * 4 * 2 + (size_t)Q * 4 +
+                       (size_t)E * D * 4 + (size_t)S * sizeof(proteus_scenario) + 256 + 64 * 8;
+  char *sb = (char *)px_buf(ctx, B_E_MISC, small + 4096);
+  uint8_t *pat = (uint8_t *)px_buf(ctx, B_E_PAT, (size_t)poff[EQ] + 16);
+  int64_t *exitF = (int64_t *)px_buf(ctx, B_E_EXIT, (size_t)S * E * D * 8 + 8);
+  if (!sb || !pat || !exitF) return px_fail(ctx, PROTEUS_ENOMEM, "closed-loop buffers");
+  char *cur = sb;
+  auto take = [&](size_t bytes) { char *r = cur; cur += (bytes + 15) & ~(size_t)15; return r; };
+  int32_t *d_w = (int32_t *)take(EQ * (D + 1) * 4);
+  int32_t *d_plen = (int32_t *)take(EQ * 4);
+  int64_t *d_poff = (int64_t *)take((EQ + 1) * 8);
+  int32_t *d_opt = (int32_t *)take((size_t)E * D * 4);
+  int32_t *d_dev = (int32_t *)take((size_t)D * 4);
+  int32_t *d_slo = (int32_t *)take((size_t)Q * 4);
+  int32_t *d_cntEQ = (int32_t *)take(EQ * 4);
+  int32_t *d_fbEQ = (int32_t *)take((EQ + Q) * 4);
+  int32_t *d_cntED = (int32_t *)take((size_t)E * D * 4);
+  int32_t *d_segBase = (int32_t *)take(((size_t)E + 1) * D * 4);
+  int64_t *d_tot = (int64_t *)take(64 * 8);
+  uint32_t *d_flags = (uint32_t *)take(16);
+  proteus_scenario *d_sc = (proteus_scenario *)take((size_t)S * sizeof(proteus_scenario));
+  if ((size_t)(cur - sb) > small + 4096) return px_fail(ctx, PROTEUS_EINTERNAL, "closed-loop scratch layout");
+  PX_CUDA(ctx, cudaMemcpyAsync(d_w, w.data(), w.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_plen, plen.data(), EQ * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_poff, poff.data(), (EQ + 1) * 8, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_opt, h_option, (size_t)E * D * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_dev, h_dev_type, (size_t)D * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_slo, h_slo, (size_t)Q * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_sc, h_sc, (size_t)S * sizeof(proteus_scenario), cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemsetAsync(d_flags, 0, 16, ctx->stream));
+  PX_CUDA(ctx, cudaMemsetAsync(d_cntEQ, 0, EQ * 4, ctx->stream));
+  PX_CUDA(ctx, cudaMemsetAsync(d_cntED, 0, (size_t)E * D * 4, ctx->stream));
+  if (EQ > 0x7fffffff) return px_fail(ctx, PROTEUS_ERANGE, "epochs x families");
+  PX_LAUNCH(ctx, "loop_patterns", k_ep_patterns, (unsigned)EQ, 32, 0, (int)EQ, D, d_w, d_poff, d_plen, pat);
+  if (N > 0) {
+    PX_LAUNCH(ctx, "replay_check", k_check_trace, 1184, 256, 0, d_arr, d_fam, N, Q, d_flags);
+    PX_LAUNCH(ctx, "loop_hist", k_ep_hist, 1184, 256, 0, d_arr, d_fam, N, E, epoch_us, Q, d_cntEQ, d_flags);
+    uint32_t flags = 0;
+    PX_CUDA(ctx, cudaMemcpyAsync(&flags, d_flags, 4, cudaMemcpyDeviceToHost, ctx->stream));
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+    if (flags & 1) return px_fail(ctx, PROTEUS_ERANGE, "arrival timestamps not sorted");
+    if (flags & 2) return px_fail(ctx, PROTEUS_EINVAL, "family id >= Q");
+    if (flags & 8) return px_fail(ctx, PROTEUS_ERANGE, "an arrival lies beyond the last epoch");
+  }
+  const int64_t ntiles = (N + TILE - 1) / TILE;
+  const unsigned tblocks = (unsigned)((ntiles + TILE_WARPS - 1) / TILE_WARPS);
+  int32_t *hist = (int32_t *)px_buf(ctx, B_R_HIST, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
+  int32_t *fbase = (int32_t *)px_buf(ctx, B_R_BASE, (size_t)(ntiles + 1) * (PX_MAXQ + 2) * 4);
+  int32_t *dbase = (int32_t *)px_buf(ctx, B_R_DBASE0, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
+  uint8_t *tgt = (uint8_t *)px_buf(ctx, B_R_TGT, (size_t)N + 16);
+  int64_t *off = (int64_t *)px_buf(ctx, B_R_OFF, (size_t)2 * (PX_MAXD + 2) * 8);
+  uint32_t *darr = (uint32_t *)px_buf(ctx, B_R_DEVARR, (size_t)N * 4 + 16);
+  uint32_t *dinv = (uint32_t *)px_buf(ctx, B_R_DEVIDX, (size_t)N * 4 + 16);
+  const int64_t NS = (N + 31) & ~(int64_t)31;
+  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * NS * 4 + 8192);
+  if (!hist || !fbase || !dbase || !tgt || !off || !darr || !dinv || !latd)
+    return px_fail(ctx, PROTEUS_ENOMEM, "routing buffers");
+  int64_t *totals = off + (PX_MAXD + 2);
+  if (N == 0) {
+    PX_CUDA(ctx, cudaMemsetAsync(off, 0, (size_t)(PX_MAXD + 2) * 8, ctx->stream));
+    return 0;
+  }
+  PX_LAUNCH(ctx, "loop_route", k_tile_scan, Q, 1024, 0, d_cntEQ, (int64_t)E, Q, d_fbEQ, d_tot);
+  PX_LAUNCH(ctx, "loop_route", k_tile_count, tblocks, TILE_WARPS * 32, 0, d_fam, N, Q, hist);
+  PX_LAUNCH(ctx, "loop_route", k_tile_scan, Q, 1024, 0, hist, ntiles, Q, fbase, totals);
+  PX_LAUNCH(ctx, "loop_route", k_ep_target, tblocks, TILE_WARPS * 32, 0, d_fam, d_arr, N, Q, epoch_us, fbase, d_fbEQ,
+            pat, d_poff, d_plen, D, tgt, hist);
+  PX_LAUNCH(ctx, "loop_route", k_tile_scan, D + 1, 1024, 0, hist, ntiles, D + 1, dbase, totals);
+  PX_LAUNCH(ctx, "loop_route", k_dev_offsets, 1, 32, 0, totals, D + 1, off);
+  PX_LAUNCH(ctx, "loop_route", k_scatter, tblocks, TILE_WARPS * 32, 0, tgt, d_arr, N, D, dbase, off, darr, dinv);
+  PX_LAUNCH(ctx, "loop_route", k_ep_seghist, 1184, 256, 0, tgt, d_arr, N, epoch_us, D, d_cntED);
+  PX_LAUNCH(ctx, "loop_route", k_tile_scan, D, 1024, 0, d_cntED, (int64_t)E, D, d_segBase, d_tot);
+  EpArgs ea;
+  memset(&ea, 0, sizeof ea);
+  ea.E = E; ea.D = D; ea.M = M; ea.bmax = ctx->bmax; ea.S = S; ea.NS = NS;
+  ea.option = d_opt; ea.dev_type = d_dev; ea.lat = ctx->d_lat; ea.acc = ctx->d_acc; ea.fam_of_m = ctx->d_fam;
+  ea.slo = d_slo; ea.sc = d_sc; ea.devOff = off; ea.cntED = d_cntED; ea.segBase = d_segBase; ea.devArr = darr;
+  ea.latd = latd; ea.exitF = exitF;
+  if (S > 65535) return px_fail(ctx, PROTEUS_EINVAL, "S");
+  const int64_t nseg = (int64_t)E * D;
+  PX_LAUNCH(ctx, "loop_spec", k_ep_spec, dim3((unsigned)((nseg + 127) / 128), (unsigned)S), 128, 0, ea);
+  PX_LAUNCH(ctx, "loop_stitch", k_ep_stitch, (unsigned)((S * D + 63) / 64), 64, 0, ea);
+  PX_LAUNCH(ctx, "loop_count", k_ep_count, dim3(296, (unsigned)S), 256, 0, ea, N, epoch_us, d_agg);
+  if (d_lat_out) {
+    const int64_t nb = (N + 256 * UNP_PER - 1) / (256 * UNP_PER);
+    PX_LAUNCH(ctx, "loop_unpermute", k_unpermute, (unsigned)nb, 256, 0, N, NS, S, d_sc, dinv, dinv, latd, d_lat_out);
+  }
+  return 0;
+}
