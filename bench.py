@@ -508,6 +508,56 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     f2["proteus_violation_ratio_slo2x_depth"] = float(res["violations"][sel]) / N
     f2["workload"] = "c5 trace (10M Poisson queries) and allocation, 64 (SLO x batch cap) scenarios per policy"
     out["f2_baseline_batchers"] = f2
+    # f4: closed loop over the c4 hour -- 3600 per-second re-solves (on the
+    # previous second's counts) feeding the replay of that hour's queries
+    cfg = W.config("f4")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    E, D = len(cfg["demand"]), len(cl.device_type)
+    arr = torch.from_numpy(cfg["arrival_us"]).to(dev)
+    fam = torch.from_numpy(cfg["family"]).to(dev)
+    dem = torch.from_numpy(cfg["demand"]).to(dev)
+    t_dev = torch.as_tensor(cl.device_type, dtype=torch.int32, device=dev)
+    t_slo = torch.as_tensor(cl.slo_us, dtype=torch.int32, device=dev)
+    scl = cfg["scenarios"]
+    Nl = len(cfg["arrival_us"])
+    lat4 = torch.empty((len(scl), Nl), dtype=torch.uint32, device=dev)
+    alloc = {"option": torch.empty((E, D), dtype=torch.int32, device=dev),
+             "z_qps": torch.empty((E, D), dtype=torch.int32, device=dev)}
+    for _ in range(2):
+        px.solve_batch(t_dev, t_slo, dem, mode=2, out=alloc)
+        rl = px.replay_epochs(arr, fam, cfg["epoch_us"], alloc["option"], alloc["z_qps"], t_dev, dem, t_slo, scl,
+                              latency=lat4)
+    px.set_timing(True)
+    ts, kts = [], []
+    for _ in range(3):
+        flush.zero_()
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        px.solve_batch(t_dev, t_slo, dem, mode=2, out=alloc)
+        k1 = px.kernel_times()
+        rl = px.replay_epochs(arr, fam, cfg["epoch_us"], alloc["option"], alloc["z_qps"], t_dev, dem, t_slo, scl,
+                              latency=lat4)
+        b.record(stream)
+        barrier()
+        ts.append(a.elapsed_time(b))
+        kts.append(k1 + px.kernel_times())
+    px.set_timing(False)
+    lms = max_over_ranks(statistics.median(ts))
+    ksplit = {}
+    for kt in kts:
+        for n_, v in kt:
+            ksplit.setdefault(n_, []).append(v)
+    ksplit = {k: statistics.median(v) for k, v in ksplit.items()}
+    out["f4_closed_loop"] = {
+        "workload": f"c4 hour: {E} one-second epochs, {Nl} queries (Poisson within each second), allocation e "
+                    f"solved on epoch e-1's counts, {len(scl)} (SLO x batch cap) scenarios",
+        "epochs": E, "queries": Nl, "scenarios": len(scl), "ms": lms,
+        "query_scenarios_per_s": Nl * len(scl) / (lms / 1e3), "kernel_ms": ksplit,
+        "violation_ratio_slo2x_depth": float(rl["violations"][[i for i, r in enumerate(scl)
+                                                                 if r[0] == 2000 and r[1] == 0][0]]) / Nl,
+        "scaling": "replicas" if world > 1 else "1 GPU"}
     return out
 
 

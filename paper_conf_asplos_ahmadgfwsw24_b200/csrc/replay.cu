@@ -2101,6 +2101,39 @@ __device__ __forceinline__ int64_t ep_walk(const EpArgs &a, int s, int e, int d,
   return F;
 }
 
+// re-walk a segment from the true free time F until the true run meets the
+// segment's idle run (phase A's latencies, still in the row at positions >=
+// the true head): at a true decision head h where the idle run also starts a
+// batch, with both devices free by a_h, both take the idle decision from h
+// and agree from there on -- the rest of the row and the exit (xF) are the
+// idle run's.  specPrev = the idle run's finish of the batch holding h - 1,
+// read before the true run overwrites that position.
+__device__ __forceinline__ int64_t ep_rewalk(const EpArgs &a, int s, int e, int d, int64_t st, int64_t n, int64_t F,
+                                             int64_t xF) {
+  const EpLane p = ep_lane(a, s, e, d);
+  uint32_t *out = a.latd + (size_t)s * a.NS + st;
+  if (p.Bmax < 1) {
+    for (int64_t j = 0; j < n; j++) out[j] = 0xFFFFFFFFu;
+    return F;
+  }
+  GArr arr{a.devArr + st};
+  int64_t h = 0, specPrev = 0;
+  while (h < n) {
+    const int64_t ah = arr(h);
+    if (h > 0 && F <= ah && specPrev <= ah) {
+      const int64_t specH = ah + (int64_t)out[h];
+      if (specH != specPrev) return xF;  // the idle run starts a batch at h: met
+    }
+    int64_t t;
+    const int b = decide(arr, n, h, F, p.Bmax, p.L, p.T, &t);
+    F = t + p.T[b - 1];
+    specPrev = (int64_t)arr(h + b - 1) + (int64_t)out[h + b - 1];
+    for (int j = 0; j < b; j++) out[h + j] = sat_lat(F - (int64_t)arr(h + j));
+    h += b;
+  }
+  return F;
+}
+
 // phase A: thread per (scenario, epoch, device) segment, from an idle device
 __global__ void __launch_bounds__(128) k_ep_spec(const __grid_constant__ EpArgs a) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -2124,8 +2157,9 @@ __global__ void __launch_bounds__(64) k_ep_stitch(const __grid_constant__ EpArgs
     const int32_t n = a.cntED[k];
     if (n == 0) continue;
     const int64_t st = a.devOff[d] + a.segBase[k];
-    if (F <= (int64_t)a.devArr[st]) F = a.exitF[(size_t)s * a.E * a.D + k];  // idle at the head: kept
-    else F = ep_walk(a, s, e, d, st, n, F);
+    const int64_t xF = a.exitF[(size_t)s * a.E * a.D + k];
+    if (F <= (int64_t)a.devArr[st]) F = xF;  // idle at the head: the idle run is the true one
+    else F = ep_rewalk(a, s, e, d, st, n, F, xF);
   }
 }
 
