@@ -2101,39 +2101,6 @@ __device__ __forceinline__ int64_t ep_walk(const EpArgs &a, int s, int e, int d,
   return F;
 }
 
-// re-walk a segment from the true free time F until the true run meets the
-// segment's idle run (phase A's latencies, still in the row at positions >=
-// the true head): at a true decision head h where the idle run also starts a
-// batch, with both devices free by a_h, both take the idle decision from h
-// and agree from there on -- the rest of the row and the exit (xF) are the
-// idle run's.  specPrev = the idle run's finish of the batch holding h - 1,
-// read before the true run overwrites that position.
-__device__ __forceinline__ int64_t ep_rewalk(const EpArgs &a, int s, int e, int d, int64_t st, int64_t n, int64_t F,
-                                             int64_t xF) {
-  const EpLane p = ep_lane(a, s, e, d);
-  uint32_t *out = a.latd + (size_t)s * a.NS + st;
-  if (p.Bmax < 1) {
-    for (int64_t j = 0; j < n; j++) out[j] = 0xFFFFFFFFu;
-    return F;
-  }
-  GArr arr{a.devArr + st};
-  int64_t h = 0, specPrev = 0;
-  while (h < n) {
-    const int64_t ah = arr(h);
-    if (h > 0 && F <= ah && specPrev <= ah) {
-      const int64_t specH = ah + (int64_t)out[h];
-      if (specH != specPrev) return xF;  // the idle run starts a batch at h: met
-    }
-    int64_t t;
-    const int b = decide(arr, n, h, F, p.Bmax, p.L, p.T, &t);
-    F = t + p.T[b - 1];
-    specPrev = (int64_t)arr(h + b - 1) + (int64_t)out[h + b - 1];
-    for (int j = 0; j < b; j++) out[h + j] = sat_lat(F - (int64_t)arr(h + j));
-    h += b;
-  }
-  return F;
-}
-
 // phase A: thread per (scenario, epoch, device) segment, from an idle device
 __global__ void __launch_bounds__(128) k_ep_spec(const __grid_constant__ EpArgs a) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -2146,20 +2113,99 @@ __global__ void __launch_bounds__(128) k_ep_spec(const __grid_constant__ EpArgs 
   a.exitF[(size_t)s * a.E * a.D + i] = ep_walk(a, s, e, d, st, n, 0);
 }
 
-// phase B: thread per (scenario, device), the true state across the epochs
-__global__ void __launch_bounds__(64) k_ep_stitch(const __grid_constant__ EpArgs a) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= a.S * a.D) return;
-  const int s = i / a.D, d = i % a.D;
+// phase B: warp per (scenario, device), the true state across the epochs.
+// A re-walk takes one §5 decision per step with the lanes in parallel: lane j
+// (queue size q = j, 1 <= j < Bmax) tests whether the rule stops at q -- q
+// is a stable count (a_q > t_q = max(t0, a_{q-1}), t0 = max(F, a_0)) and
+// either t_q >= Tmax_wait(q+1) = a_0 + L - T(q+1) (dispatch now) or the next
+// arrival a_q comes after it (dispatch at Tmax_wait) -- and the first stop
+// is the decision (Case 2 moves through exactly the stable counts in order);
+// no stop below Bmax dispatches Bmax once the Bmax-th query is there.
+// Arrivals come from a per-warp shared-memory ring over the device array.
+__global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArgs a) {
+  __shared__ uint32_t sA[4][WC_RW];
+  __shared__ int32_t sT[4][PX_MAXB];
+  const int wid = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) >> 5), lane = threadIdx.x & 31;
+  const int w = threadIdx.x >> 5;
+  if (wid >= a.S * a.D) return;
+  const int s = wid / a.D, d = wid % a.D;
+  uint32_t *ring = sA[w];
+  int32_t *T = sT[w];
+  const int64_t dbase = a.devOff[d], dn = a.devOff[d + 1] - dbase;  // the device's array
+  const uint32_t *arr = a.devArr + dbase;
+  uint32_t *row = a.latd + (size_t)s * a.NS + dbase;
+  int64_t b0 = -(int64_t)WC_RW;  // ring covers device positions [b0, b0 + WC_RW)
+  auto fill = [&](int64_t from, int cnt) {
+    for (int k = lane; k < cnt; k += 32) {
+      const int64_t j = from + k;
+      ring[j & (WC_RW - 1)] = j < dn ? __ldg(arr + j) : 0xFFFFFFFFu;
+    }
+  };
+  auto A = [&](int64_t j) -> int64_t {  // j >= b0
+    return j - b0 < WC_RW ? (int64_t)ring[j & (WC_RW - 1)] : (int64_t)__ldg(arr + j);
+  };
+  const int64_t INF = INT64_MAX / 4;
   int64_t F = 0;  // R13
   for (int e = 0; e < a.E; e++) {
     const int64_t k = (int64_t)e * a.D + d;
     const int32_t n = a.cntED[k];
     if (n == 0) continue;
-    const int64_t st = a.devOff[d] + a.segBase[k];
+    const int64_t st = a.segBase[k];  // segment start in the device array
     const int64_t xF = a.exitF[(size_t)s * a.E * a.D + k];
-    if (F <= (int64_t)a.devArr[st]) F = xF;  // idle at the head: the idle run is the true one
-    else F = ep_rewalk(a, s, e, d, st, n, F, xF);
+    if (F <= (int64_t)__ldg(arr + st)) { F = xF; continue; }  // idle at the head: the idle run is the true one
+    const EpLane p = ep_lane(a, s, e, d);
+    __syncwarp();
+    for (int i = lane; i < p.Bmax; i += 32) T[i] = p.T[i];
+    __syncwarp();
+    int64_t h = st, specPrev = 0;
+    const int64_t en = st + n;
+    bool met = false;
+    while (h < en) {
+      if (h - b0 >= WC_RW / 2 || h < b0) {  // slide / reload the ring
+        const int64_t nb = h & ~(int64_t)(WC_RW / 2 - 1);
+        __syncwarp();
+        if (nb == b0 + WC_RW / 2) fill(b0 + WC_RW, WC_RW / 2);
+        else fill(nb, WC_RW);
+        b0 = nb;
+        __syncwarp();
+      }
+      const int64_t a0 = A(h);
+      if (h > st && F <= a0 && specPrev <= a0 && a0 + (int64_t)row[h] != specPrev) { met = true; break; }
+      const int64_t t0 = F > a0 ? F : a0;
+      int b = p.Bmax;
+      int64_t t = -1;
+      for (int r = 0; 1 + 32 * r < p.Bmax; r++) {
+        const int j = 1 + 32 * r + lane;
+        bool stop = false;
+        int64_t tj = 0;
+        if (j < p.Bmax) {
+          const int64_t am = h + j - 1 < en ? A(h + j - 1) : INF;
+          const int64_t aj = h + j < en ? A(h + j) : INF;
+          const int64_t tq = t0 > am ? t0 : am;
+          const int64_t W = a0 + p.L - T[j];
+          stop = aj > tq && (tq >= W || aj > W);
+          tj = tq >= W ? tq : W;
+        }
+        const unsigned m = __ballot_sync(0xffffffffu, stop);
+        if (m) {
+          const int f = __ffs(m) - 1;
+          b = 1 + 32 * r + f;
+          t = __shfl_sync(0xffffffffu, tj, f);
+          break;
+        }
+      }
+      if (t < 0) {  // Bmax queued: dispatch once the Bmax-th query is there
+        const int64_t al = A(h + p.Bmax - 1);
+        t = t0 > al ? t0 : al;
+      }
+      const int64_t Fn = t + T[b - 1];
+      specPrev = A(h + b - 1) + (int64_t)row[h + b - 1];
+      __syncwarp();
+      for (int i = lane; i < b; i += 32) row[h + i] = sat_lat(Fn - A(h + i));
+      F = Fn;
+      h += b;
+    }
+    if (met) F = xF;
   }
 }
 
@@ -2308,7 +2354,7 @@ int px_replay_epochs(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_f
   if (S > 65535) return px_fail(ctx, PROTEUS_EINVAL, "S");
   const int64_t nseg = (int64_t)E * D;
   PX_LAUNCH(ctx, "loop_spec", k_ep_spec, dim3((unsigned)((nseg + 127) / 128), (unsigned)S), 128, 0, ea);
-  PX_LAUNCH(ctx, "loop_stitch", k_ep_stitch, (unsigned)((S * D + 63) / 64), 64, 0, ea);
+  PX_LAUNCH(ctx, "loop_stitch", k_ep_stitch, (unsigned)((S * D + 3) / 4), 128, 0, ea);
   PX_LAUNCH(ctx, "loop_count", k_ep_count, dim3(296, (unsigned)S), 256, 0, ea, N, epoch_us, d_agg);
   if (d_lat_out) {
     const int64_t nb = (N + 256 * UNP_PER - 1) / (256 * UNP_PER);

@@ -20,6 +20,9 @@
 #include "internal.cuh"
 
 #define FLAT_THREADS 256
+#ifndef FLAT_MINB
+#define FLAT_MINB 2  // blocks per SM the register budget is sized for
+#endif
 #define GEN_THREADS 128
 
 // ------------------------------------------------------------ reduce ----
@@ -199,7 +202,7 @@ __device__ __forceinline__ uint64_t fill(const int (&caps)[QM * VM], const FlatA
 }
 
 template <int QM, int VM>
-__global__ void __launch_bounds__(FLAT_THREADS, 2) k_flat_pair(const __grid_constant__ FlatArgs<QM, VM> a) {
+__global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __grid_constant__ FlatArgs<QM, VM> a) {
   constexpr int S = QM * VM;
   extern __shared__ int32_t smem[];
   const int D = a.D, K = a.K;
