@@ -32,8 +32,21 @@ def main():
     os.environ["PROTEUS_REPLAY_ROUNDS"] = "1"  # one fix-up round, then the stitch
     px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
     os.environ.pop("PROTEUS_REPLAY_ROUNDS")
+    os.environ["PROTEUS_REPLAY_WARMUP"] = "40"  # chunk runs entered after a warm-up
+    px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
+    os.environ.pop("PROTEUS_REPLAY_WARMUP")
+    # §8(f2) baseline batchers (k_wc_lanes), mixed with §5 scenarios
+    scb = np.array([[1000, 4, 0, 1], [2000, 0, 0, 2], [1500, 8, 1, 1], [3000, 0, 0, 0]], np.int32)
+    px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, scb)
     os.environ["PROTEUS_REPLAY_SIMPLE"] = "1"
     px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
+    os.environ.pop("PROTEUS_REPLAY_SIMPLE")
+    # §8(f4) closed loop (k_ep_*), 5 short epochs with switching allocations
+    lc = W.config("f4", n_seconds=5, lam_mid=3000.0)
+    dem = np.ascontiguousarray(lc["demand"])
+    px.load_profiles(lc["prof"])
+    px.closed_loop(lc["arrival_us"], lc["family"], lc["epoch_us"], dem, lc["cluster"].device_type,
+                   lc["cluster"].slo_us, np.array([[1000, 4, 0, 0], [3000, 0, 0, 0]], np.int32))
     print("sanitize target done")
 
 
