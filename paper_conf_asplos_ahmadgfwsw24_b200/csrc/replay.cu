@@ -576,6 +576,45 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   a.cs[(size_t)s * a.NCH + a.choff[d] + c] = e;
 }
 
+// ---- one §5 decision by a whole warp (lane-parallel form of decide()):
+// lane j (queue size q = j, 1 <= j < Bmax, rounds of 32) tests whether the
+// rule stops at q -- q is a stable count (a_q > t_q = max(t0, a_{q-1}),
+// t0 = max(F, a_h)) and either t_q >= Tmax_wait(q+1) = a_h + L - T(q+1)
+// (dispatch now, Case 1) or the next arrival a_q comes after Tmax_wait(q+1)
+// (dispatch then).  Case 2 walks through exactly the stable counts in
+// increasing order, so the first stop is decide()'s batch; no stop below
+// Bmax dispatches Bmax once the Bmax-th query is there (R4).  Arr(j) is the
+// arrival of position j (< n); returns b, *t_out = dispatch time.
+template <class Arr, class Tab>
+__device__ __forceinline__ int decide_warp(const Arr &A, int64_t n, int64_t h, int64_t F, int Bmax, int64_t L,
+                                           const Tab &T, int lane, int64_t *t_out) {
+  const int64_t INF = INT64_MAX / 4;
+  const int64_t a0 = A(h);
+  const int64_t t0 = F > a0 ? F : a0;
+  for (int r = 0; 1 + 32 * r < Bmax; r++) {
+    const int j = 1 + 32 * r + lane;
+    bool stop = false;
+    int64_t tj = 0;
+    if (j < Bmax) {
+      const int64_t am = h + j - 1 < n ? A(h + j - 1) : INF;
+      const int64_t aj = h + j < n ? A(h + j) : INF;
+      const int64_t tq = t0 > am ? t0 : am;
+      const int64_t W = a0 + L - T(j);
+      stop = aj > tq && (tq >= W || aj > W);
+      tj = tq >= W ? tq : W;
+    }
+    const unsigned m = __ballot_sync(0xffffffffu, stop);
+    if (m) {
+      const int f = __ffs(m) - 1;
+      *t_out = __shfl_sync(0xffffffffu, tj, f);
+      return 1 + 32 * r + f;
+    }
+  }
+  const int64_t al = A(h + Bmax - 1);
+  *t_out = t0 > al ? t0 : al;
+  return Bmax;
+}
+
 // ---- phase B: exact stitch, one warp per (device, scenario)
 // The true state (h, F) is carried from chunk to chunk.  A chunk whose
 // speculative start (its first query, device idle) equals the true state is
@@ -2114,14 +2153,9 @@ __global__ void __launch_bounds__(128) k_ep_spec(const __grid_constant__ EpArgs 
 }
 
 // phase B: warp per (scenario, device), the true state across the epochs.
-// A re-walk takes one §5 decision per step with the lanes in parallel: lane j
-// (queue size q = j, 1 <= j < Bmax) tests whether the rule stops at q -- q
-// is a stable count (a_q > t_q = max(t0, a_{q-1}), t0 = max(F, a_0)) and
-// either t_q >= Tmax_wait(q+1) = a_0 + L - T(q+1) (dispatch now) or the next
-// arrival a_q comes after it (dispatch at Tmax_wait) -- and the first stop
-// is the decision (Case 2 moves through exactly the stable counts in order);
-// no stop below Bmax dispatches Bmax once the Bmax-th query is there.
-// Arrivals come from a per-warp shared-memory ring over the device array.
+// A re-walk takes one §5 decision per step with the lanes in parallel
+// (decide_warp); arrivals come from a per-warp shared-memory ring over the
+// device array.
 __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArgs a) {
   __shared__ uint32_t sA[4][WC_RW];
   __shared__ int32_t sT[4][PX_MAXB];
@@ -2144,7 +2178,6 @@ __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArg
   auto A = [&](int64_t j) -> int64_t {  // j >= b0
     return j - b0 < WC_RW ? (int64_t)ring[j & (WC_RW - 1)] : (int64_t)__ldg(arr + j);
   };
-  const int64_t INF = INT64_MAX / 4;
   int64_t F = 0;  // R13
   for (int e = 0; e < a.E; e++) {
     const int64_t k = (int64_t)e * a.D + d;
@@ -2171,33 +2204,9 @@ __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArg
       }
       const int64_t a0 = A(h);
       if (h > st && F <= a0 && specPrev <= a0 && a0 + (int64_t)row[h] != specPrev) { met = true; break; }
-      const int64_t t0 = F > a0 ? F : a0;
-      int b = p.Bmax;
-      int64_t t = -1;
-      for (int r = 0; 1 + 32 * r < p.Bmax; r++) {
-        const int j = 1 + 32 * r + lane;
-        bool stop = false;
-        int64_t tj = 0;
-        if (j < p.Bmax) {
-          const int64_t am = h + j - 1 < en ? A(h + j - 1) : INF;
-          const int64_t aj = h + j < en ? A(h + j) : INF;
-          const int64_t tq = t0 > am ? t0 : am;
-          const int64_t W = a0 + p.L - T[j];
-          stop = aj > tq && (tq >= W || aj > W);
-          tj = tq >= W ? tq : W;
-        }
-        const unsigned m = __ballot_sync(0xffffffffu, stop);
-        if (m) {
-          const int f = __ffs(m) - 1;
-          b = 1 + 32 * r + f;
-          t = __shfl_sync(0xffffffffu, tj, f);
-          break;
-        }
-      }
-      if (t < 0) {  // Bmax queued: dispatch once the Bmax-th query is there
-        const int64_t al = A(h + p.Bmax - 1);
-        t = t0 > al ? t0 : al;
-      }
+      int64_t t;
+      auto Tl = [&](int j) -> int64_t { return (int64_t)T[j]; };
+      const int b = decide_warp(A, en, h, F, p.Bmax, p.L, Tl, lane, &t);
       const int64_t Fn = t + T[b - 1];
       specPrev = A(h + b - 1) + (int64_t)row[h + b - 1];
       __syncwarp();
