@@ -451,6 +451,43 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
       b0 = nb;
       __syncwarp();
     }
+    if (nexus ? B == 1 : limit == 1) {
+      // Batches of one, 32 per step: query h + k leaves at max(F_{k-1}, a)
+      // (work-conserving), F_k = max(F_{k-1}, a_{h+k}) + T(1), i.e. F_k - (k+1) T(1)
+      // = max(F, max_{i<=k} a_{h+i} - i T(1)) -- a warp max-scan.  AIMD keeps
+      // limit 1 while batches time out (and always when Bmax = 1): the step
+      // ends after the first on-time batch (the limit becomes 2).  Nexus
+      // (B = 1) serves a query iff it finishes on time; the first one that
+      // would not is dropped (F unchanged) and ends the step.
+      const int64_t j = h + lane;
+      const bool valid = j < n;
+      const int64_t aj = valid ? A(j) : 0;
+      int64_t x = valid ? aj - (int64_t)lane * T1 : INT64_MIN / 4;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t v = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x = v > x ? v : x;
+      }
+      const int64_t Fk = (F > x ? F : x) + (int64_t)(lane + 1) * T1;
+      const bool late = valid && Fk - aj > p.L;
+      const int nval = n - h < 32 ? (int)(n - h) : 32;
+      int r = nval;        // queries this step handles
+      bool drop_last = false;
+      if (nexus) {
+        const unsigned m = __ballot_sync(0xffffffffu, late);
+        if (m) { r = __ffs(m); drop_last = true; }
+      } else if (p.Bmax > 1) {
+        const unsigned m = __ballot_sync(0xffffffffu, valid && !late);
+        if (m) { r = __ffs(m); limit = 2; }
+      }
+      const int served = drop_last ? r - 1 : r;
+      if (lane < served) out[j] = sat_lat(Fk - aj);
+      if (drop_last && lane == r - 1) out[j] = 0xFFFFFFFFu;
+      if (served > 0) F = __shfl_sync(0xffffffffu, Fk, served - 1);
+      h += r;
+      if (tail < h) tail = h;
+      continue;
+    }
     const int64_t ah = A(h);
     if (fast && ah >= F) {
       // Isolated queries, 32 per ballot: query j finds the device free (a_j >=
