@@ -3,6 +3,8 @@
     python scripts/profile_target.py c2      # flat search over 13^8 candidates
     python scripts/profile_target.py c4      # factored re-solve, 3600 vectors
     python scripts/profile_target.py c5      # replay 10M queries x 64 scenarios
+    python scripts/profile_target.py f2      # c5 trace, Nexus + AIMD, 32 scenarios each
+    python scripts/profile_target.py f4      # closed loop, 3600 epochs x 12 scenarios
 """
 import os
 import sys
@@ -38,6 +40,27 @@ def main(what):
         lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
         r = px.replay(arr, fam, a.option, a.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
         print("c5", r["violations"][:8])
+    elif what == "f2":
+        cfg = W.config("c5")
+        prof, cl = cfg["prof"], cfg["cluster"]
+        px.load_profiles(prof)
+        a = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=2)[0]
+        arr = torch.from_numpy(cfg["arrival_us"]).cuda()
+        fam = torch.from_numpy(cfg["family"]).cuda()
+        sc = np.concatenate([W.scenarios_64(0, 1)[::2], W.scenarios_64(0, 2)[::2]])
+        lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
+        r = px.replay(arr, fam, a.option, a.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
+        print("f2", r["violations"][:8])
+    elif what == "f4":
+        cfg = W.config("f4")
+        px.load_profiles(cfg["prof"])
+        cl = cfg["cluster"]
+        arr = torch.from_numpy(cfg["arrival_us"]).cuda()
+        fam = torch.from_numpy(cfg["family"]).cuda()
+        dem = torch.from_numpy(cfg["demand"]).cuda()
+        res, _ = px.closed_loop(arr, fam, cfg["epoch_us"], dem, cl.device_type, cl.slo_us, cfg["scenarios"],
+                                latency=None, device=torch.device("cuda:0"))
+        print("f4", res["violations"][:8])
     torch.cuda.synchronize()
 
 
