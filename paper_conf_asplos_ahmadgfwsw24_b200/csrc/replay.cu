@@ -2241,6 +2241,32 @@ __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArg
       }
       const int64_t a0 = A(h);
       if (h > st && F <= a0 && specPrev <= a0 && a0 + (int64_t)row[h] != specPrev) { met = true; break; }
+      const int B = p.Bmax;
+      if (h + B <= en && A(h + B - 1) <= F) {
+        // backlog: Bmax queued when the device frees -> a full batch leaves at
+        // once (R4), so batch k of the stretch finishes at F + (k+1) T(Bmax)
+        // while a_{h + (k+1) Bmax - 1} <= F + k T(Bmax); 32 batches per ballot
+        const int64_t TB = T[B - 1];
+        int done = 0;
+        for (;;) {
+          const int64_t hk = h + (int64_t)(done + lane) * B;
+          const bool full = hk + B <= en && A(hk + B - 1) <= F + (int64_t)(done + lane) * TB;
+          const unsigned m = __ballot_sync(0xffffffffu, full);
+          const int r = m == 0xffffffffu ? 32 : __ffs(~m) - 1;
+          const int64_t hs = h + (int64_t)done * B, ns = (int64_t)r * B;
+          if (ns > 0) specPrev = A(hs + ns - 1) + (int64_t)row[hs + ns - 1];
+          __syncwarp();
+          for (int64_t i = lane; i < ns; i += 32) {
+            const int64_t kb = i / B;
+            row[hs + i] = sat_lat(F + (done + kb + 1) * TB - A(hs + i));
+          }
+          done += r;
+          if (r < 32 || h + (int64_t)(done + 32) * B - 1 - b0 >= WC_RW) break;  // stretch ends / ring edge
+        }
+        F += (int64_t)done * TB;
+        h += (int64_t)done * B;
+        continue;
+      }
       int64_t t;
       auto Tl = [&](int j) -> int64_t { return (int64_t)T[j]; };
       const int b = decide_warp(A, en, h, F, p.Bmax, p.L, Tl, lane, &t);
