@@ -10,7 +10,10 @@ GPUs: each rank its contiguous slice + one NCCL slot all-reduce + the winner's
 materialisation), inputs resident in HBM.  The same run also measures, as
 `extra`, the other two parts of BASELINE.json's metric: the per-second
 re-solve of the paper-scale cluster (c4, 3600 demand vectors, factored search)
-and the adaptive-batching replay (c5, 10M queries x 64 scenarios).
+and the adaptive-batching replay (c5, 10M queries x 64 scenarios), plus the
+§8(f) rows: the Fig. 1b frontier (f3), the baseline batchers on the c5 trace
+(f2) and the closed loop of per-second re-solves feeding the replay (f4).  At
+N > 1 the replays split their scenarios by rank (strong scaling).
 
 --impl reference times the CPU oracle (oracle/, test infrastructure) on the
 same workload: the paper ships no code, so the oracle is the reference arm.
@@ -435,8 +438,13 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     alloc = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=2)[0]
     arr = torch.from_numpy(cfg["arrival_us"]).to(dev)
     fam = torch.from_numpy(cfg["family"]).to(dev)
-    sc = cfg["scenarios"]
+    # N > 1: the scenarios are split by rank (dist.replay_sharded);
+    # value = all ranks' query-scenarios / the slowest rank's time
+    sc_all = cfg["scenarios"]
+    slo_, shi_ = shard_range(len(sc_all), rank, world)
+    sc = sc_all[slo_:shi_]
     S, N = len(sc), len(cfg["arrival_us"])
+    S_all = len(sc_all)
     lat = torch.empty((S, N), dtype=torch.uint32, device=dev)
     for _ in range(2):
         px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
@@ -469,21 +477,23 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     px.replay(arr_h, fam_h, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=True)
     e2e = time.perf_counter() - t0
     out["c5_replay"] = {
-        "queries": N, "scenarios": S, "ms": ms, "query_scenarios_per_s": N * S / (ms / 1e3),
+        "queries": N, "scenarios": S_all, "ms": ms, "query_scenarios_per_s": N * S_all / (ms / 1e3),
         "routing_ms": route_ms, "lane_kernels_ms": lane, "kernel_split_ms": split,
         "roofline": {"kernel": " + ".join(LANE_KERNELS), "bound": "hbm", "achieved": alg_bytes / (lane / 1e3) / 1e9,
                      "peak": hbm, "unit": "GB/s", "frac": alg_bytes / (lane / 1e3) / 1e9 / hbm,
                      "peak_source": peak_src, "alg_bytes": alg_bytes},
         "violations_first_scenarios": [int(x) for x in res["violations"][:4]],
-        "e2e": {"value": N * S / e2e, "unit": "query-scenarios/s", "h2d_bytes_per_step": int(N * 5),
-                "d2h_bytes_per_step": int(N * S * 4)},
-        "scaling": "replicas" if world > 1 else "1 GPU"}
+        "e2e": {"value": N * S_all / max_over_ranks(e2e), "unit": "query-scenarios/s",
+                "h2d_bytes_per_step": int(N * 5), "d2h_bytes_per_step": int(N * S * 4)},
+        "scaling": "strong (scenarios split by rank)" if world > 1 else "1 GPU"}
     # f2: the §6.4 baseline batchers (Nexus early drop, Clipper AIMD) on the same
     # trace and allocation, 64 scenarios each (k_wc_lanes), plus the Fig. 6-style
     # violation ratios of all three policies at SLO 2x, batch cap = table depth
     f2 = {}
     for pol, name in ((1, "nexus"), (2, "aimd")):
-        scp = W.scenarios_64(0, pol)
+        scp_all = W.scenarios_64(0, pol)
+        plo, phi = shard_range(len(scp_all), rank, world)
+        scp = scp_all[plo:phi]
         px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, scp, latency=lat)
         px.set_timing(True)
         ts, kms = [], []
@@ -500,12 +510,12 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
         px.set_timing(False)
         pms = max_over_ranks(statistics.median(ts))
         km = statistics.median(kms)
-        sel = [i for i, r in enumerate(scp) if r[0] == 2000 and r[1] == 0][0]
-        f2[name] = {"ms": pms, "query_scenarios_per_s": N * len(scp) / (pms / 1e3), "lane_kernel_ms": km,
+        sel = [i for i, r in enumerate(scp) if r[0] == 2000 and r[1] == 0]
+        f2[name] = {"ms": pms, "query_scenarios_per_s": N * len(scp_all) / (pms / 1e3), "lane_kernel_ms": km,
                     "lane_kernel_hbm_frac": (N * len(scp) * 4 + N * 8) / (km / 1e3) / 1e9 / hbm,
-                    "violation_ratio_slo2x_depth": float(rp["violations"][sel]) / N}
-    sel = [i for i, r in enumerate(sc) if r[0] == 2000 and r[1] == 0][0]
-    f2["proteus_violation_ratio_slo2x_depth"] = float(res["violations"][sel]) / N
+                    "violation_ratio_slo2x_depth": float(rp["violations"][sel[0]]) / N if sel else None}
+    sel = [i for i, r in enumerate(sc) if r[0] == 2000 and r[1] == 0]
+    f2["proteus_violation_ratio_slo2x_depth"] = float(res["violations"][sel[0]]) / N if sel else None
     f2["workload"] = "c5 trace (10M Poisson queries) and allocation, 64 (SLO x batch cap) scenarios per policy"
     out["f2_baseline_batchers"] = f2
     # f4: closed loop over the c4 hour -- 3600 per-second re-solves (on the
@@ -519,7 +529,9 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     dem = torch.from_numpy(cfg["demand"]).to(dev)
     t_dev = torch.as_tensor(cl.device_type, dtype=torch.int32, device=dev)
     t_slo = torch.as_tensor(cl.slo_us, dtype=torch.int32, device=dev)
-    scl = cfg["scenarios"]
+    scl_all = cfg["scenarios"]
+    llo, lhi = shard_range(len(scl_all), rank, world)
+    scl = scl_all[llo:lhi]
     Nl = len(cfg["arrival_us"])
     lat4 = torch.empty((len(scl), Nl), dtype=torch.uint32, device=dev)
     alloc = {"option": torch.empty((E, D), dtype=torch.int32, device=dev),
@@ -553,11 +565,11 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     out["f4_closed_loop"] = {
         "workload": f"c4 hour: {E} one-second epochs, {Nl} queries (Poisson within each second), allocation e "
                     f"solved on epoch e-1's counts, {len(scl)} (SLO x batch cap) scenarios",
-        "epochs": E, "queries": Nl, "scenarios": len(scl), "ms": lms,
-        "query_scenarios_per_s": Nl * len(scl) / (lms / 1e3), "kernel_ms": ksplit,
-        "violation_ratio_slo2x_depth": float(rl["violations"][[i for i, r in enumerate(scl)
-                                                                 if r[0] == 2000 and r[1] == 0][0]]) / Nl,
-        "scaling": "replicas" if world > 1 else "1 GPU"}
+        "epochs": E, "queries": Nl, "scenarios": len(scl_all), "ms": lms,
+        "query_scenarios_per_s": Nl * len(scl_all) / (lms / 1e3), "kernel_ms": ksplit,
+        "violation_ratio_slo2x_depth": (float(rl["violations"][sel4[0]]) / Nl) if (sel4 := [
+            i for i, r in enumerate(scl) if r[0] == 2000 and r[1] == 0]) else None,
+        "scaling": "strong (scenarios split by rank; every rank re-solves all epochs)" if world > 1 else "1 GPU"}
     return out
 
 

@@ -118,3 +118,41 @@ def pareto_merge(parts):
     return dict(cap=np.array([o[0] for o in out], np.int64), accsum=np.array([o[1] for o in out], np.int64),
                 index=np.array([o[2] for o in out], np.uint64),
                 n_configs=sum(int(p["n_configs"]) for p in parts), n_front=len(out))
+
+
+def gather_aggregates(lo: int, hi: int, S: int, parts: dict, group=None, device=None) -> dict:
+    """Per-scenario aggregates of scenarios [lo, hi) from every rank into full
+    [S] arrays on every rank: each rank writes its slice into a zero
+    int64[3][S] tensor, one SUM all-reduce assembles it (scenario slices are
+    disjoint, so the sum is a gather).  768 bytes per 32 scenarios."""
+    import torch
+    import torch.distributed as dist
+    v = np.zeros((3, S), np.int64)
+    for k, name in enumerate(("violations", "on_time", "acc_sum")):
+        v[k, lo:hi] = np.asarray(parts[name], dtype=np.uint64).astype(np.int64)
+    t = torch.from_numpy(v)
+    if device is not None:
+        t = t.to(device)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    out = t.cpu().numpy().astype(np.uint64)
+    return dict(violations=out[0], on_time=out[1], acc_sum=out[2])
+
+
+def replay_sharded(replay, scenarios, group=None, comm_device=None, **kw):
+    """Replay (c5) / closed loop (f4) with the scenarios split by rank
+    (scenarios are independent): this rank runs slice
+    shard_range(S) through `replay(scenarios=..., **kw)` (Proteus.replay or
+    Proteus.replay_epochs, keyword arguments) and the per-scenario aggregates
+    are gathered to every rank; per-query latencies stay on their rank.
+    Returns (aggregates over all S, this rank's result, (lo, hi))."""
+    import torch.distributed as dist
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    sc = np.asarray(scenarios, dtype=np.int32)
+    S = len(sc)
+    lo, hi = shard_range(S, rank, world)
+    if hi > lo:
+        local = replay(scenarios=sc[lo:hi], **kw)
+    else:
+        local = dict(latency=None, violations=np.zeros(0, np.uint64), on_time=np.zeros(0, np.uint64),
+                     acc_sum=np.zeros(0, np.uint64))
+    return gather_aggregates(lo, hi, S, local, group, comm_device), local, (lo, hi)

@@ -90,3 +90,58 @@ def test_pick_best_order_and_sign():
     assert pick_best(v) == (big, 3, 1)
     v = slot_vector(0, 2, 4, 9) + slot_vector(1, 2, 4, 9)
     assert pick_best(v)[:2] == (4, 9)
+
+
+def _replay_worker(rank, world, port, q):
+    """Scenario-split replay: the per-rank replay is stood in for by the
+    oracle over this rank's scenario slice."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import torch.distributed as dist
+    import oracle
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    from paper_conf_asplos_ahmadgfwsw24_b200.dist import replay_sharded
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    try:
+        cfg = W.config("c3", totals=(12000,))
+        prof, cl = cfg["prof"], cfg["cluster"]
+        r = oracle.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][0], 2)
+        a, f = W.query_trace(8000, 12000.0, cfg["weights"], 17, "gamma")
+        sc = np.concatenate([W.scenarios_64(0, 0)[::9], W.scenarios_fig6(0)[::13]])
+
+        def rep(scenarios):
+            return oracle.replay(prof, cl.device_type, r["option"], r["z"], cfg["demand"][0], cl.slo_us, a, f,
+                                 scenarios, want_latency=False)
+
+        agg, _, (lo, hi) = replay_sharded(rep, sc)
+        q.put((rank, lo, hi, {k: v.tolist() for k, v in agg.items()}))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_world2_scenario_split_replay(oracle_mod):
+    """§8(e) replay: scenarios split by rank, aggregates gathered by one SUM
+    all-reduce -- every rank ends with the single-process aggregates."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3", totals=(12000,))
+    prof, cl = cfg["prof"], cfg["cluster"]
+    r = oracle_mod.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][0], 2)
+    a, f = W.query_trace(8000, 12000.0, cfg["weights"], 17, "gamma")
+    sc = np.concatenate([W.scenarios_64(0, 0)[::9], W.scenarios_fig6(0)[::13]])
+    ref = oracle_mod.replay(prof, cl.device_type, r["option"], r["z"], cfg["demand"][0], cl.slo_us, a, f, sc,
+                            want_latency=False)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_replay_worker, args=(rk, 2, port, q)) for rk in range(2)]
+    for p in ps:
+        p.start()
+    out = [q.get(timeout=300) for _ in ps]
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    spans = sorted((lo, hi) for _, lo, hi, _ in out)
+    assert spans[0][0] == 0 and spans[0][1] == spans[1][0] and spans[1][1] == len(sc)
+    for _, _, _, agg in out:
+        for k in ("violations", "on_time", "acc_sum"):
+            assert agg[k] == ref[k].tolist(), k
