@@ -110,10 +110,11 @@ def flat_pair_ops_per_candidate(Q, V, K):
     per_prefix = (S                       # add device D-3's capacity to its slot
                   + Q * fill              # family values of the prefix
                   + S * (fill + 2)        # deltas Fb of every option of device D-1
-                  + 2 + 2 + 2 * S         # idle row: threshold, (idle, idle), (idle, sb) compares
+                  + 2 * S + 4 * Q         # largest delta per family (64-bit max), top two families
+                  + 2 + 2 + 2             # idle row: threshold, (idle, idle), best other-family compare
                   + S * ((fill + 4)       # row sa: delta of device D-2's option, ba
                          + 2 + 2          #   threshold, (sa, idle) compare
-                         + 2 * (S - V)    #   other-family candidates: one 64-bit compare each
+                         + 3              #   other-family candidates: select M1/M2, one 64-bit compare
                          + V * (fill + 6)))  # same-family candidates: joint fill, combine, compare
     return per_prefix / (K * K)
 

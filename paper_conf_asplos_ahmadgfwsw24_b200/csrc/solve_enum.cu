@@ -254,28 +254,35 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
 #pragma unroll
       for (int s = 0; s < S; s++) Fb[s] = fill<QM, VM>(caps, a, s / VM, s % VM, a.PB[s], -1, 0) - Fq[s / VM];
       // The K^2 candidates of this prefix, one row per option of device D-2
-      // (idle first).  Fast path per row: every candidate is scored and
-      // compared with the running best lb -- a candidate of another family
-      // than the row's as Fb[sb] > lb - ba (its score is ba + Fb[sb], Fb >= 0),
-      // a same-family candidate through its joint water-fill -- and the
-      // compares are only OR-ed into flags.  A flagged row (it holds a better
+      // (idle first).  Fast path per row: a candidate of another family than
+      // the row's scores ba + Fb[sb] (Fb >= 0), so the row holds one above the
+      // running best lb iff the largest such Fb exceeds lb - ba (M1 / M2
+      // below: one compare for all of them); a same-family candidate is
+      // scored through its joint water-fill.  The compares only flag the row.  A flagged row (it holds a better
       // candidate) is re-scanned in index order with strict >, so the first
       // (lowest-index) maximum is kept.  If lb < ba the row's first candidate
       // (sa, idle) = ba already flags the row, so the unsigned threshold never
       // matters when it wraps.  Pad slots (code 0, capacity 0) score exactly
       // like the idle option with the same index and never change the result.
+      // Largest delta of device D-1 over all its options (M1, family fm1) and
+      // over the options outside family fm1 (M2): a row of family qa holds an
+      // other-family candidate above lb iff (qa == fm1 ? M2 : M1) > lb - ba.
+      uint64_t M1 = 0, M2 = 0;
+      int fm1 = -1;
+#pragma unroll
+      for (int q = 0; q < QM; q++) {
+        uint64_t mq = Fb[q * VM];
+#pragma unroll
+        for (int j = 1; j < VM; j++) mq = Fb[q * VM + j] > mq ? Fb[q * VM + j] : mq;
+        if (mq > M1) { M2 = M1; M1 = mq; fm1 = q; }
+        else if (mq > M2) M2 = mq;
+      }
       uint64_t lb = best_s;
       int lp = -1;
       if (best_i == ~0ull) { lb = base; lp = 0; }  // the thread's first candidate
       {
         const uint64_t thr = lb - base;
-        bool f0 = base > lb, f1 = false, f2 = false, f3 = false;
-#pragma unroll
-        for (int sb = 0; sb < S; sb++) {
-          const bool g = Fb[sb] > thr;
-          if ((sb & 3) == 0) f0 |= g; else if ((sb & 3) == 1) f1 |= g; else if ((sb & 3) == 2) f2 |= g; else f3 |= g;
-        }
-        if (f0 | f1 | f2 | f3) {
+        if (base > lb || M1 > thr) {
           if (base > lb) { lb = base; lp = 0; }
 #pragma unroll
           for (int sb = 0; sb < S; sb++)
@@ -291,13 +298,10 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
         for (int jb = 0; jb < VM; jb++)
           jv[jb] = base - Fq[qa] + fill<QM, VM>(caps, a, qa, sa % VM, a.PA[sa], jb, a.PB[qa * VM + jb]);
         const uint64_t thr = lb - ba;
-        bool f0 = ba > lb, f1 = false, f2 = false, f3 = false;
+        bool f0 = ba > lb || (qa == fm1 ? M2 : M1) > thr;
 #pragma unroll
-        for (int sb = 0; sb < S; sb++) {
-          const bool g = (qa == sb / VM) ? jv[sb % VM] > lb : Fb[sb] > thr;
-          if ((sb & 3) == 0) f0 |= g; else if ((sb & 3) == 1) f1 |= g; else if ((sb & 3) == 2) f2 |= g; else f3 |= g;
-        }
-        if (f0 | f1 | f2 | f3) {
+        for (int jb = 0; jb < VM; jb++) f0 |= jv[jb] > lb;
+        if (f0) {
           if (ba > lb) { lb = ba; lp = a.code[sa] * K; }
 #pragma unroll
           for (int sb = 0; sb < S; sb++) {
@@ -328,6 +332,13 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
 // a6 (grid level) is folded in: the block first reduces the per-block winners.
 __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const BestRec *__restrict__ blocks, int nb,
                                    uint64_t fixed_index, int use_fixed, uint64_t n_candidates, SolRec *out) {
+  // the tables thread 0 walks, staged in shared memory (its loop is serial)
+  __shared__ int32_t sPdev[8192];
+  __shared__ int32_t sCode[PX_MAXQ * PX_MAXV], sAcc[PX_MAXQ * PX_MAXV];
+  const bool staged = a.D * a.K <= 8192;
+  if (staged)
+    for (int k = threadIdx.x; k < a.D * a.K; k += blockDim.x) sPdev[k] = a.Pdev[k];
+  for (int k = threadIdx.x; k < a.Q * a.VM; k += blockDim.x) { sCode[k] = a.slot_code[k]; sAcc[k] = a.slot_acc[k]; }
   uint64_t bs = 0, bi = ~0ull;
   if (!use_fixed)
     for (int k = threadIdx.x; k < nb; k += blockDim.x)
@@ -357,11 +368,11 @@ __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const Bes
     uint64_t acc = 0;
     stot += a.s[q];
     for (int j = 0; j < a.V[q]; j++) {
-      const int code = __ldg(&a.slot_code[q * a.VM + j]);
-      const int A = __ldg(&a.slot_acc[q * a.VM + j]);
+      const int code = sCode[q * a.VM + j];
+      const int A = sAcc[q * a.VM + j];
       for (int d = 0; d < a.D; d++) {
         if (o[d] != code) continue;
-        const int t = min(rem, __ldg(&a.Pdev[d * a.K + code]));
+        const int t = min(rem, staged ? sPdev[d * a.K + code] : __ldg(&a.Pdev[d * a.K + code]));
         z[d] = t;
         rem -= t;
         acc += (uint64_t)A * (uint64_t)t;
@@ -408,7 +419,15 @@ static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p
   if (smem > 48 * 1024) PX_CUDA(ctx, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int nsm = 0, occ = 0;
   PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
-  PX_CUDA(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, FLAT_THREADS, smem));
+  {  // occupancy per (instantiation, shared-memory size), queried once
+    static size_t occ_smem = ~(size_t)0;
+    static int occ_val = 0;
+    if (occ_smem != smem) {
+      PX_CUDA(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_val, kern, FLAT_THREADS, smem));
+      occ_smem = smem;
+    }
+    occ = occ_val;
+  }
   if (occ < 1) occ = 1;
   const uint64_t np = p_hi - p_lo;
   uint64_t nb = (uint64_t)nsm * occ;

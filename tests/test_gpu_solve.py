@@ -254,3 +254,17 @@ def test_c4_solve_batch_outputs(px, oracle_mod):
         r = oracle_mod.solve(prof, cl.device_type, cl.slo_us, dem[v], 2)
         assert (host["served"][v], host["accsum"][v]) == (r["served"], r["accsum"])
         assert host["option"][v].tolist() == r["option"].tolist()
+
+
+def test_random_flat_kernel(px, oracle_mod):
+    """The specialised flat kernel (sorted accuracies, D >= 3) on random toys
+    (row filters by the largest other-family delta, flagged rows re-scanned),
+    incl. tied accuracies and P = 0 holes."""
+    rng = np.random.default_rng(4321)
+    for trial in range(80):
+        T = int(rng.integers(1, 4))
+        Q = int(rng.integers(1, 5))
+        D = int(rng.integers(3, 7))
+        prof, dev, slo, P = random_instance(rng, T=T, Q=Q, Vmax=3, D=D, Pmax=40, tie_acc=trial % 3 == 0)
+        s = rng.integers(0, 60, size=(3, prof.Q)).astype(np.int32)
+        check(px, oracle_mod, prof, dev, slo, s, 0, False, threads=2)

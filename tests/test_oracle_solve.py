@@ -347,3 +347,4 @@ def test_c1_c2_regimes(oracle_mod):
     cfg = W.config("c1")
     r = oracle_mod.solve(cfg["prof"], cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"][0], 0)
     assert r["unmet"] == 0 and r["eff"] < 1_000_000 and r["n_candidates"] == 7**4
+
