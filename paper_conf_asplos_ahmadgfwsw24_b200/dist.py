@@ -156,3 +156,60 @@ def replay_sharded(replay, scenarios, group=None, comm_device=None, **kw):
         local = dict(latency=None, violations=np.zeros(0, np.uint64), on_time=np.zeros(0, np.uint64),
                      acc_sum=np.zeros(0, np.uint64))
     return gather_aggregates(lo, hi, S, local, group, comm_device), local, (lo, hi)
+
+
+# ------------------------------------------------ batched flat search --
+SOL_HEAD = 7  # score, index, served, unmet, accsum, eff, n_candidates per solution, then option[D], z[D]
+
+
+def pack_solutions(sols, D: int) -> np.ndarray:
+    """Per-vector solutions of this rank as int64 rows [n][SOL_HEAD + 2D]
+    (uint64 score / index as their bit patterns)."""
+    out = np.zeros((len(sols), SOL_HEAD + 2 * D), np.int64)
+    for v, s in enumerate(sols):
+        out[v, :SOL_HEAD] = [_to_i64(s.score), _to_i64(s.index), s.served, s.unmet, s.accsum, s.eff_acc_micro,
+                             s.n_candidates]
+        out[v, SOL_HEAD:SOL_HEAD + D] = np.asarray(s.option, np.int64)
+        out[v, SOL_HEAD + D:] = np.asarray(s.z, np.int64)
+    return out
+
+
+def pick_solutions(gathered: np.ndarray, D: int):
+    """gathered [world][n][SOL_HEAD + 2D]: per vector the rank with the
+    lexicographic maximum (score desc, index asc) -- its local winner is the
+    global one, already materialised (placement, z, value); n_candidates
+    sums the ranks' slices."""
+    from . import Solution
+    world, n = gathered.shape[0], gathered.shape[1]
+    out = []
+    for v in range(n):
+        best = None
+        for r in range(world):
+            s, i = _to_u64(gathered[r, v, 0]), _to_u64(gathered[r, v, 1])
+            if best is None or s > best[0] or (s == best[0] and i < best[1]):
+                best = (s, i, r)
+        row = gathered[best[2], v]
+        out.append(Solution(best[0], best[1], int(row[2]), int(row[3]), int(row[4]), int(row[5]),
+                            int(gathered[:, v, 6].sum()),
+                            row[SOL_HEAD:SOL_HEAD + D].astype(np.int32), row[SOL_HEAD + D:].astype(np.int32)))
+    return out
+
+
+def solve_sharded_batch(px, device_type, slo_us, demand, mode=0, group=None, comm_device=None):
+    """Modes 0/1 for a batch of demand vectors on every rank of `group`: one
+    library call scans this rank's index slice for every vector (one host
+    synchronisation per call), then ONE all-gather of the per-rank winners,
+    each already materialised, and the per-vector (score desc, index asc)
+    pick -- no re-materialisation.  Returns (solutions, local solutions)."""
+    import torch
+    import torch.distributed as dist
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    D = len(device_type)
+    local = px.solve(device_type, slo_us, demand, mode=mode, shard_rank=rank, shard_world=world)
+    t = torch.from_numpy(pack_solutions(local, D))
+    if comm_device is not None:
+        t = t.to(comm_device)
+    parts = [torch.empty_like(t) for _ in range(world)]
+    dist.all_gather(parts, t, group=group)
+    gathered = np.stack([p.cpu().numpy() for p in parts])
+    return pick_solutions(gathered, D), local

@@ -145,3 +145,66 @@ def test_world2_scenario_split_replay(oracle_mod):
     for _, _, _, agg in out:
         for k in ("violations", "on_time", "acc_sum"):
             assert agg[k] == ref[k].tolist(), k
+
+
+def _batch_worker(rank, world, port, q):
+    """Batched flat search split by index range: the per-rank library call is
+    stood in for by a fake `px` whose solve() returns, per demand vector, the
+    oracle's best over the rank's index slice, materialised by the oracle."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import torch.distributed as dist
+    import oracle
+    from paper_conf_asplos_ahmadgfwsw24_b200 import Solution, workloads as W
+    from paper_conf_asplos_ahmadgfwsw24_b200.dist import shard_range, solve_sharded_batch
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    try:
+        cfg = W.config("c1")
+        prof, cl = cfg["prof"], cfg["cluster"]
+        dems = np.array([[0, 0], [300, 100], [600, 0], [800, 700]], np.int32)
+        K, D = 1 + prof.M, len(cl.device_type)
+
+        class FakePx:
+            def solve(self, device_type, slo_us, demand, mode, shard_rank, shard_world):
+                n = K ** D
+                lo, hi = shard_range(n, shard_rank, shard_world)
+                out = []
+                for dem in demand:
+                    s, i = _rank_best(prof, device_type, slo_us, dem, lo, hi)
+                    opt = np.array([(i // K ** (D - 1 - d)) % K for d in range(D)], np.int32)
+                    r = oracle.score_placement(prof, device_type, slo_us, dem, opt)
+                    out.append(Solution(s, i, r["served"], r["unmet"], r["accsum"], r["eff"], hi - lo, opt, r["z"]))
+                return out
+
+        sols, _ = solve_sharded_batch(FakePx(), cl.device_type, cl.slo_us, dems, mode=0)
+        q.put((rank, [(s.score, s.index, s.served, s.accsum, s.n_candidates, s.option.tolist(), s.z.tolist())
+                      for s in sols]))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_world2_batched_flat_search(oracle_mod):
+    """One all-gather of the per-rank winners (already materialised) per
+    batch of demand vectors: every rank ends with the single-process optimum,
+    placement and z of every vector."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c1")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    dems = np.array([[0, 0], [300, 100], [600, 0], [800, 700]], np.int32)
+    refs = [oracle_mod.solve(prof, cl.device_type, cl.slo_us, d, 0) for d in dems]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_batch_worker, args=(rk, 2, port, q)) for rk in range(2)]
+    for p in ps:
+        p.start()
+    out = [q.get(timeout=600) for _ in ps]
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for _, sols in out:
+        for (sc, idx, served, accsum, ncand, opt, z), r in zip(sols, refs):
+            assert idx == r["index"] and sc == (r["served"] << 42) | r["accsum"]
+            assert (served, accsum) == (r["served"], r["accsum"])
+            assert ncand == r["n_candidates"]
+            assert opt == r["option"].tolist() and z == r["z"].tolist()
