@@ -436,10 +436,10 @@ static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_s
     rc = px_solve_factored(ctx, a, in.dev_type.data(), d_dev, d_dem, VM, tab, h_P, d_sol);
   } else if (mat_only) {
     rc = px_solve_enum(ctx, a, in.dev_type.data(), in.slo.data(), in.demand.data(), VM, tab, h_P, h_slot_code,
-                       d_sol, mat_vec, mat_vec + 1, true, mat_index, use_flat);
+                       d_sol, mat_vec, mat_vec + 1, true, mat_index, use_flat, d_dem);
   } else {
     rc = px_solve_enum(ctx, a, in.dev_type.data(), in.slo.data(), in.demand.data(), VM, tab, h_P, h_slot_code,
-                       d_sol, 0, a->n_vec, false, 0, use_flat);
+                       d_sol, 0, a->n_vec, false, 0, use_flat, d_dem);
   }
   if (rc) return rc;
   if (bout) return batch_out(ctx, a, d_sol, nout, bout);

@@ -143,7 +143,7 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *a, const int32_t *
                   const int32_t *h_slo, const int32_t *h_demand, int VM, const Tables &tab,
                   const std::vector<int32_t> &h_P, const std::vector<int32_t> &h_slot_code,
                   SolRec *d_sol, int32_t vec_lo, int32_t vec_hi, bool materialize_only, uint64_t mat_index,
-                  bool use_flat);
+                  bool use_flat, const int32_t *d_demand /* [n_vec][Q] on the device */);
 int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32_t *h_dev_type,
                       const int32_t *d_dev, const int32_t *d_demand, int VM, const Tables &tab, const std::vector<int32_t> &h_P,
                       SolRec *d_sol);

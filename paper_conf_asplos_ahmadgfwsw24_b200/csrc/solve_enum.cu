@@ -330,8 +330,15 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
 // a9: decode the winner, water-fill z in (accuracy desc, code asc, device asc)
 // order (reading C10), report served / unmet / accsum / eff; re-check the score.
 // a6 (grid level) is folded in: the block first reduces the per-block winners.
+// Block v materialises vector v of a batch: its per-block results start at
+// blocks + v * stride, its demand at dem_all + v * Q (dem_all NULL: a.s).
 __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const BestRec *__restrict__ blocks, int nb,
-                                   uint64_t fixed_index, int use_fixed, uint64_t n_candidates, SolRec *out) {
+                                   uint64_t fixed_index, int use_fixed, uint64_t n_candidates, SolRec *out,
+                                   int64_t stride, const int32_t *__restrict__ dem_all) {
+  blocks += (int64_t)blockIdx.x * stride;
+  out += blockIdx.x;
+  __shared__ int32_t sS[PX_MAXQ];
+  for (int q = threadIdx.x; q < a.Q; q += blockDim.x) sS[q] = dem_all ? dem_all[(int64_t)blockIdx.x * a.Q + q] : a.s[q];
   // the tables thread 0 walks, staged in shared memory (its loop is serial)
   __shared__ int32_t sPdev[8192];
   __shared__ int32_t sCode[PX_MAXQ * PX_MAXV], sAcc[PX_MAXQ * PX_MAXV];
@@ -352,7 +359,7 @@ __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const Bes
   if (idx == ~0ull) {  // empty shard: nothing scored
     for (int d = 0; d < a.D; d++) { r.option[d] = 0; r.z[d] = 0; }
     int64_t stot = 0;
-    for (int q = 0; q < a.Q; q++) stot += a.s[q];
+    for (int q = 0; q < a.Q; q++) stot += sS[q];
     r.score = 0; r.index = idx; r.served = 0; r.unmet = stot; r.accsum = 0; r.eff = 0;
     r.n_candidates = n_candidates; r.status = 0;
     return;
@@ -364,9 +371,9 @@ __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const Bes
   int64_t served = 0, accsum = 0, stot = 0;
   uint64_t score = 0;
   for (int q = 0; q < a.Q; q++) {
-    int rem = a.s[q];
+    int rem = sS[q];
     uint64_t acc = 0;
-    stot += a.s[q];
+    stot += sS[q];
     for (int j = 0; j < a.V[q]; j++) {
       const int code = sCode[q * a.VM + j];
       const int A = sAcc[q * a.VM + j];
@@ -378,9 +385,9 @@ __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const Bes
         acc += (uint64_t)A * (uint64_t)t;
       }
     }
-    served += a.s[q] - rem;
+    served += sS[q] - rem;
     accsum += (int64_t)acc;
-    score += px_pack((uint32_t)(a.s[q] - rem), acc);
+    score += px_pack((uint32_t)(sS[q] - rem), acc);
   }
   for (int d = 0; d < a.D; d++) { r.option[d] = o[d]; r.z[d] = z[d]; }
   r.score = score;
@@ -477,7 +484,7 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
                   const int32_t *h_slo, const int32_t *h_demand, int VM, const Tables &tab,
                   const std::vector<int32_t> &h_P, const std::vector<int32_t> &h_slot_code,
                   SolRec *d_sol, int32_t vec_lo, int32_t vec_hi, bool materialize_only, uint64_t mat_index,
-                  bool use_flat) {
+                  bool use_flat, const int32_t *d_demand) {
   (void)h_slo;
   const int D = args->D, K = 1 + ctx->M, Q = ctx->Q, T = ctx->T;
   const int mode = args->mode;
@@ -517,9 +524,16 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
   int nsm = 0;
   PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
   const size_t max_blocks = (size_t)nsm * 64;
-  BestRec *d_blocks = (BestRec *)px_buf(ctx, B_BEST, sizeof(BestRec) * (max_blocks + 1));
-  if (!d_blocks) return px_fail(ctx, PROTEUS_ENOMEM, "block results");
+  // per-block winners of every vector of the batch (one row each); one
+  // materialise launch for the whole batch at the end (block = vector)
+  const int64_t stride = (int64_t)max_blocks + 1;
+  const int nv = materialize_only ? 1 : vec_hi - vec_lo;
+  BestRec *d_blocks0 = (BestRec *)px_buf(ctx, B_BEST, sizeof(BestRec) * (size_t)stride * nv);
+  if (!d_blocks0) return px_fail(ctx, PROTEUS_ENOMEM, "block results");
+  uint64_t ncand_all = 0;
+  int nb_all = 0;
   for (int v = vec_lo; v < vec_hi; v++) {
+    BestRec *d_blocks = d_blocks0 + (materialize_only ? 0 : (int64_t)(v - vec_lo) * stride);
     const int32_t *dem = h_demand + (size_t)v * Q;
     for (int q = 0; q < Q; q++) ea.s[q] = dem[q];
     SolRec *rec = d_sol + (materialize_only ? 0 : v - vec_lo);
@@ -551,8 +565,17 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
       }
       nb_used = nb;
     }
-    PX_LAUNCH(ctx, "argmax_materialize", k_materialize_enum, 1, 1024, 0, ea, d_blocks, nb_used, mat_index,
-              materialize_only ? 1 : 0, ncand, rec);
+    if (materialize_only) {
+      PX_LAUNCH(ctx, "argmax_materialize", k_materialize_enum, 1, 1024, 0, ea, d_blocks, nb_used, mat_index, 1,
+                ncand, rec, (int64_t)0, (const int32_t *)nullptr);
+    } else {
+      (void)rec;
+      ncand_all = ncand;  // the same slice for every vector
+      nb_all = nb_used;
+    }
   }
+  if (!materialize_only && nv > 0)
+    PX_LAUNCH(ctx, "argmax_materialize", k_materialize_enum, (unsigned)nv, 1024, 0, ea, d_blocks0, nb_all,
+              (uint64_t)0, 0, ncand_all, d_sol, stride, d_demand + (size_t)vec_lo * Q);
   return 0;
 }
