@@ -266,7 +266,9 @@ def main():
     # roofline of the dominant kernel (score_flat_pair, one launch per demand vector)
     peaks, peak_src = measured_peaks()
     k_ms = statistics.mean(kern_ms) if kern_ms else float("nan")
-    cand_per_launch = loc[0].n_candidates
+    # one launch scores the rank's slice for up to 32 vectors of the batch (grid.y = vector)
+    launches_per_step = max(1, len(kern_ms) // args.steps)
+    cand_per_launch = loc[0].n_candidates * NVEC / launches_per_step
     ops = flat_pair_ops_per_candidate(4, 3, 13) * cand_per_launch
     sm_mhz = clocks["sm_mhz"] or peaks.get("sm_max_mhz", SM_MAX_MHZ_FALLBACK)
     peak_ops = SM_COUNT * INT_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12

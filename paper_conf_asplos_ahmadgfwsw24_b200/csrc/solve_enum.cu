@@ -20,6 +20,7 @@
 #include "internal.cuh"
 
 #define FLAT_THREADS 256
+#define FLAT_NV 32  // demand vectors per flat launch (grid.y)
 #ifndef FLAT_MINB
 #define FLAT_MINB 2  // blocks per SM the register budget is sized for
 #endif
@@ -179,7 +180,8 @@ struct FlatArgs {
   int32_t PA[QM * VM];  // capacity of slot on device D-2
   int32_t PB[QM * VM];  // capacity of slot on device D-1
   int32_t code[QM * VM];
-  int32_t s[QM];
+  int32_t s[FLAT_NV][QM];  // demand of each vector of the launch (grid.y)
+  int64_t out_stride;      // rows of block winners per vector
   const int32_t *Pdev, *code_slot;
   BestRec *out;
 };
@@ -187,9 +189,9 @@ struct FlatArgs {
 // water-fill of family q over slots q*VM..q*VM+VM-1, with capacity pa added
 // to slot ja and pb to slot jb (compile-time; -1 = none) -> packed score
 template <int QM, int VM>
-__device__ __forceinline__ uint64_t fill(const int (&caps)[QM * VM], const FlatArgs<QM, VM> &a, int q, int ja,
-                                         int pa, int jb, int pb) {
-  int rem = a.s[q];
+__device__ __forceinline__ uint64_t fill(const int (&caps)[QM * VM], const FlatArgs<QM, VM> &a,
+                                         const int32_t *sd, int q, int ja, int pa, int jb, int pb) {
+  int rem = sd[q];
   uint64_t acc = 0;
 #pragma unroll
   for (int j = 0; j < VM; j++) {
@@ -198,7 +200,7 @@ __device__ __forceinline__ uint64_t fill(const int (&caps)[QM * VM], const FlatA
     acc += (uint64_t)(uint32_t)a.A[q * VM + j] * (uint32_t)t;
     rem -= t;
   }
-  return px_pack((uint32_t)(a.s[q] - rem), acc);
+  return px_pack((uint32_t)(sd[q] - rem), acc);
 }
 
 template <int QM, int VM>
@@ -210,6 +212,8 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
   int32_t *sCS = smem + D * K; // [K]
   for (int i = threadIdx.x; i < D * K; i += blockDim.x) sP[i] = a.Pdev[i];
   for (int i = threadIdx.x; i < K; i += blockDim.x) sCS[i] = a.code_slot[i];
+  __shared__ int32_t sDem[QM];  // this launch row's demand vector (grid.y)
+  if (threadIdx.x < QM) sDem[threadIdx.x] = a.s[blockIdx.y][threadIdx.x];
   __syncthreads();
   const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   uint64_t p = a.p_lo + tid * a.per_thread;
@@ -249,10 +253,10 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
       uint64_t Fq[QM];
       uint64_t base = 0;
 #pragma unroll
-      for (int q = 0; q < QM; q++) { Fq[q] = fill<QM, VM>(caps, a, q, -1, 0, -1, 0); base += Fq[q]; }
+      for (int q = 0; q < QM; q++) { Fq[q] = fill<QM, VM>(caps, a, sDem, q, -1, 0, -1, 0); base += Fq[q]; }
       uint64_t Fb[S];
 #pragma unroll
-      for (int s = 0; s < S; s++) Fb[s] = fill<QM, VM>(caps, a, s / VM, s % VM, a.PB[s], -1, 0) - Fq[s / VM];
+      for (int s = 0; s < S; s++) Fb[s] = fill<QM, VM>(caps, a, sDem, s / VM, s % VM, a.PB[s], -1, 0) - Fq[s / VM];
       // The K^2 candidates of this prefix, one row per option of device D-2
       // (idle first).  Fast path per row: a candidate of another family than
       // the row's scores ba + Fb[sb] (Fb >= 0), so the row holds one above the
@@ -292,11 +296,11 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
 #pragma unroll
       for (int sa = 0; sa < S; sa++) {
         const int qa = sa / VM;
-        const uint64_t ba = base + fill<QM, VM>(caps, a, qa, sa % VM, a.PA[sa], -1, 0) - Fq[qa];
+        const uint64_t ba = base + fill<QM, VM>(caps, a, sDem, qa, sa % VM, a.PA[sa], -1, 0) - Fq[qa];
         uint64_t jv[VM];  // same-family candidates (joint fills)
 #pragma unroll
         for (int jb = 0; jb < VM; jb++)
-          jv[jb] = base - Fq[qa] + fill<QM, VM>(caps, a, qa, sa % VM, a.PA[sa], jb, a.PB[qa * VM + jb]);
+          jv[jb] = base - Fq[qa] + fill<QM, VM>(caps, a, sDem, qa, sa % VM, a.PA[sa], jb, a.PB[qa * VM + jb]);
         const uint64_t thr = lb - ba;
         bool f0 = ba > lb || (qa == fm1 ? M2 : M1) > thr;
 #pragma unroll
@@ -323,7 +327,11 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
     }
   }
   block_best(best_s, best_i);
-  if (threadIdx.x == 0) { a.out[blockIdx.x].score = best_s; a.out[blockIdx.x].index = best_i; }
+  if (threadIdx.x == 0) {
+    BestRec &o = a.out[(int64_t)blockIdx.y * a.out_stride + blockIdx.x];
+    o.score = best_s;
+    o.index = best_i;
+  }
 }
 
 // ------------------------------------------------------- materialise ----
@@ -403,8 +411,9 @@ __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const Bes
 // ------------------------------------------------------------- host -----
 template <int QM, int VM>
 static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p_hi, const int32_t *dev_type,
-                       const int32_t *demand, const std::vector<int32_t> &h_P, const std::vector<int32_t> &h_slot_code,
-                       const Tables &tab, BestRec *d_blocks, int *nblocks_out) {
+                       const int32_t *demand, int nvec, const std::vector<int32_t> &h_P,
+                       const std::vector<int32_t> &h_slot_code, const Tables &tab, BestRec *d_blocks,
+                       int64_t out_stride, int *nblocks_out) {
   FlatArgs<QM, VM> a;
   memset(&a, 0, sizeof a);
   a.D = D; a.K = K;
@@ -417,7 +426,9 @@ static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p
     a.PA[s] = code ? h_P[dev_type[D - 2] * M + code - 1] : 0;
     a.PB[s] = code ? h_P[dev_type[D - 1] * M + code - 1] : 0;
   }
-  for (int q = 0; q < QM; q++) a.s[q] = q < ctx->Q ? demand[q] : 0;
+  for (int v = 0; v < nvec; v++)
+    for (int q = 0; q < QM; q++) a.s[v][q] = q < ctx->Q ? demand[(size_t)v * ctx->Q + q] : 0;
+  a.out_stride = out_stride;
   a.Pdev = tab.Pdev;
   a.code_slot = tab.code_slot;
   a.out = d_blocks;
@@ -448,13 +459,14 @@ static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p
   if (a.per_thread > (uint64_t)K) a.per_thread = (a.per_thread + K - 1) / K * K;
   nb = (np + a.per_thread * FLAT_THREADS - 1) / (a.per_thread * FLAT_THREADS);
   if (nb == 0) nb = 1;
-  PX_LAUNCH(ctx, "score_flat_pair", kern, (unsigned)nb, FLAT_THREADS, smem, a);
+  PX_LAUNCH(ctx, "score_flat_pair", kern, dim3((unsigned)nb, (unsigned)nvec), FLAT_THREADS, smem, a);
   *nblocks_out = (int)nb;
   return 0;
 }
 
-typedef int (*flat_fn)(proteus_ctx *, int, int, uint64_t, uint64_t, const int32_t *, const int32_t *,
-                       const std::vector<int32_t> &, const std::vector<int32_t> &, const Tables &, BestRec *, int *);
+typedef int (*flat_fn)(proteus_ctx *, int, int, uint64_t, uint64_t, const int32_t *, const int32_t *, int,
+                       const std::vector<int32_t> &, const std::vector<int32_t> &, const Tables &, BestRec *, int64_t,
+                       int *);
 
 struct FlatInst { int QM, VM; flat_fn fn; };
 static const FlatInst kFlat[] = {
@@ -531,7 +543,7 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
   BestRec *d_blocks0 = (BestRec *)px_buf(ctx, B_BEST, sizeof(BestRec) * (size_t)stride * nv);
   if (!d_blocks0) return px_fail(ctx, PROTEUS_ENOMEM, "block results");
   uint64_t ncand_all = 0;
-  int nb_all = 0;
+  int nb_all = 0, flat_nb = 0;
   for (int v = vec_lo; v < vec_hi; v++) {
     BestRec *d_blocks = d_blocks0 + (materialize_only ? 0 : (int64_t)(v - vec_lo) * stride);
     const int32_t *dem = h_demand + (size_t)v * Q;
@@ -545,9 +557,14 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
         const uint64_t NP = N / ((uint64_t)K * K);
         const uint64_t plo = mul_div(NP, rank, world), phi = mul_div(NP, rank + 1, world);
         ncand = (phi - plo) * (uint64_t)K * K;
-        const FlatInst *f = pick_flat(Q, *std::max_element(ctx->V.begin(), ctx->V.end()));
-        int rc = f->fn(ctx, D, K, plo, phi, h_dev_type, dem, h_P, h_slot_code, tab, d_blocks, &nb);
-        if (rc) return rc;
+        if ((v - vec_lo) % FLAT_NV == 0) {  // one launch per FLAT_NV vectors (grid.y = vector)
+          const int nvec = vec_hi - v < FLAT_NV ? vec_hi - v : FLAT_NV;
+          const FlatInst *f = pick_flat(Q, *std::max_element(ctx->V.begin(), ctx->V.end()));
+          int rc = f->fn(ctx, D, K, plo, phi, h_dev_type, dem, nvec, h_P, h_slot_code, tab, d_blocks, stride,
+                         &flat_nb);
+          if (rc) return rc;
+        }
+        nb = flat_nb;
       } else {
         const uint64_t lo = mul_div(N, rank, world), hi = mul_div(N, rank + 1, world);
         ncand = hi - lo;
