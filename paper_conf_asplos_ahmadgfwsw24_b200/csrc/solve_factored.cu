@@ -187,9 +187,11 @@ __global__ void __launch_bounds__(FG_WARPS * 32) k_fact_g(const __grid_constant_
 // instructions per slot and no serial dependence between slots.  Each lane
 // keeps the first maximum in candidate order (= lowest lexicographic rank)
 // as a candidate ordinal and decodes its rank once at the end.
+#ifndef GV_TILE
 #define GV_TILE 64
+#endif
 #ifndef GV_NV
-#define GV_NV 4  // demand vectors per lane
+#define GV_NV 2  // demand vectors per lane (2: 5.54 ms on c4; 1: 6.28, 4: 5.90, 8: 6.73)
 #endif
 __device__ __forceinline__ uint64_t madw(uint32_t a, uint32_t b, uint64_t c) {
   uint64_t r;
