@@ -18,7 +18,7 @@ import sys
 METRICS = {
     "duration_us": ("gpu__time_duration.sum", 1e-3),
     "ipc_per_sm": ("sm__inst_executed.avg.per_cycle_active", 1),
-    "issue_active_pct": ("sm__issue_active.avg.pct_of_peak_sustained_active", 1),
+    "issue_active_pct": ("smsp__issue_active.avg.pct_of_peak_sustained_active", 1),
     "warps_active_per_sm": ("sm__warps_active.avg.per_cycle_active", 1),
     "alu_pipe_pct": ("sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active", 1),
     "fma_pipe_pct": ("sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active", 1),
@@ -54,12 +54,14 @@ def raw(rep):
                 if units[i] in UNIT and name.endswith(("bytes", "_us")):
                     v *= UNIT[units[i]]
                 k[name] = v * scale if name != "duration_us" else v / 1e3
-        stalls = {}
+        stalls = {}  # warp-cycles stalled per issued instruction, by reason
         for i, h in enumerate(hdr):
-            if h.startswith("smsp__average_warp_latency_issue_stalled_") or \
-               (h.startswith("smsp__warp_issue_stalled_") and h.endswith("_per_warp_active.pct")):
+            if h.startswith("smsp__average_warps_issue_stalled_") and h.endswith("_per_issue_active.ratio"):
+                reason = h[len("smsp__average_warps_issue_stalled_"):-len("_per_issue_active.ratio")]
+                if reason in ("selected",):
+                    continue
                 try:
-                    stalls[h.split("stalled_")[1].replace("_per_warp_active.pct", "")] = float(r[i])
+                    stalls[reason] = float(r[i])
                 except ValueError:
                     pass
         k["top_stalls_pct"] = dict(sorted(stalls.items(), key=lambda x: -x[1])[:5])
@@ -85,7 +87,7 @@ def main():
     os.makedirs("profiles", exist_ok=True)
     kern, md = [], [f"# ncu per-kernel counters ({tag})\n", "Full captures (`ncu --set full --clock-control none`,"
                     " one launch each, replayed; times are cold-cache and serialised).\n",
-                    "| kernel | us | IPC/SM | issue % | warps/SM | ALU % | FMA % | DRAM R+W GB | regs | top stalls |",
+                    "| kernel | us | IPC/SM | issue % | warps/SM | ALU % | FMA % | DRAM R+W GB | regs | top stalls (cycles per issue) |",
                     "|---|---|---|---|---|---|---|---|---|---|"]
     lmd = [f"# ncu launch lists ({tag})\n", "`ncu --metrics gpu__time_duration.sum --clock-control none`: per-launch "
            "times are cold-cache and serialised -- compare the shares, not the absolutes.\n"]
@@ -96,7 +98,7 @@ def main():
                 kern.append(k)
                 g = lambda n, f="{:.1f}": f.format(k[n]) if n in k else "-"
                 dr = (k.get("dram_read_bytes", 0) + k.get("dram_write_bytes", 0)) / 1e9
-                st = ", ".join(f"{a} {b:.0f}" for a, b in list(k["top_stalls_pct"].items())[:3])
+                st = ", ".join(f"{a} {b:.2f}" for a, b in list(k["top_stalls_pct"].items())[:3])
                 md.append(f"| {k['kernel'][:40]} | {g('duration_us')} | {g('ipc_per_sm', '{:.2f}')} | "
                           f"{g('issue_active_pct')} | {g('warps_active_per_sm')} | {g('alu_pipe_pct')} | "
                           f"{g('fma_pipe_pct')} | {dr:.3f} | {g('registers', '{:.0f}')} | {st} |")

@@ -268,3 +268,29 @@ def test_random_flat_kernel(px, oracle_mod):
         prof, dev, slo, P = random_instance(rng, T=T, Q=Q, Vmax=3, D=D, Pmax=40, tie_acc=trial % 3 == 0)
         s = rng.integers(0, 60, size=(3, prof.Q)).astype(np.int32)
         check(px, oracle_mod, prof, dev, slo, s, 0, False, threads=2)
+
+
+def test_c2_bench_batch_sampled(px, oracle_mod):
+    """The bench's launch configuration: the 32-vector c2 batch in one call
+    (one flat launch, grid.y = vector) with device-resident inputs.  Sampled
+    vectors against the exhaustive oracle; every vector's placement re-scored
+    by the oracle, and the batch equal to one-vector calls."""
+    import torch
+    import bench
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c2", totals=bench.C2_TOTALS)
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    dev = torch.device("cuda:0")
+    sols = px.solve(torch.as_tensor(cl.device_type, device=dev), torch.as_tensor(cl.slo_us, device=dev),
+                    torch.as_tensor(cfg["demand"], device=dev), mode=0)
+    assert len(sols) == bench.NVEC
+    for v in (0, 13, bench.NVEC - 1):
+        r = oracle_mod.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][v], 0)
+        assert (sols[v].index, sols[v].served, sols[v].accsum) == (r["index"], r["served"], r["accsum"])
+        assert sols[v].z.tolist() == r["z"].tolist()
+    for v, sol in enumerate(sols):
+        chk = oracle_mod.score_placement(prof, cl.device_type, cl.slo_us, cfg["demand"][v], sol.option)
+        assert (chk["served"], chk["accsum"]) == (sol.served, sol.accsum)
+        one = px.solve(cl.device_type, cl.slo_us, cfg["demand"][v:v + 1], mode=0)[0]
+        assert (one.score, one.index) == (sol.score, sol.index)
