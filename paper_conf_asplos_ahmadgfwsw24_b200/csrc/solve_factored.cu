@@ -26,7 +26,9 @@
 #include "internal.cuh"
 
 #define FG_WARPS 8
-#define DP_THREADS 512
+#ifndef DP_THREADS
+#define DP_THREADS 256  // c4 fact_dp: 128 1.95 ms, 256 1.97, 512 2.20 (barrier stalls)
+#endif
 
 struct FactLayout {
   int32_t Q, T, VM, U;
