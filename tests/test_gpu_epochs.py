@@ -123,3 +123,33 @@ def test_closed_loop_errors(px):
         px.replay_epochs(cfg["arrival_us"], cfg["family"], cfg["epoch_us"], np.zeros((3, D), np.int32),
                          np.zeros((3, D), np.int32), cl.device_type, cfg["demand"], cl.slo_us,
                          np.array([[1000, 0, 1, 0]], np.int32))
+
+
+def test_closed_loop_full_hour(px, oracle_mod):
+    """§8(f4) at the bench's size and launch configuration: the whole c4 hour
+    (3600 one-second epochs, ~10.6M queries) in one proteus_replay_epochs
+    call.  Allocations (inputs of the replay) come from the oracle: 48
+    demand levels of the hour solved exactly, epoch e running level e mod 48
+    with that level's demand as its routing demand (any valid allocation is a
+    valid input); every latency and aggregate compared with the oracle."""
+    import torch
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("f4")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    E = len(cfg["demand"])
+    lv = np.linspace(0, E - 1, 48).astype(int)
+    sols = [oracle_mod.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][e], 2) for e in lv]
+    pick = np.arange(E) % 48
+    opts = np.array([sols[k]["option"] for k in pick], np.int32)
+    zs = np.array([sols[k]["z"] for k in pick], np.int32)
+    dem = np.ascontiguousarray(cfg["demand"][lv][pick])
+    sc = np.array([(1000, 8, 0, 0), (3000, 0, 0, 0)], np.int32)
+    px.load_profiles(prof)
+    a, f = cfg["arrival_us"], cfg["family"]
+    lat = torch.empty((len(sc), len(a)), dtype=torch.uint32, device="cuda")
+    g = px.replay_epochs(torch.from_numpy(a).cuda(), torch.from_numpy(f).cuda(), cfg["epoch_us"], opts, zs,
+                         cl.device_type, dem, cl.slo_us, sc, latency=lat)
+    o = oracle_mod.replay_epochs(prof, cl.device_type, opts, zs, dem, cl.slo_us, a, f, cfg["epoch_us"], sc)
+    for k in ("violations", "on_time", "acc_sum"):
+        assert np.array_equal(g[k], o[k]), k
+    assert np.array_equal(lat.cpu().numpy(), o["latency"])
