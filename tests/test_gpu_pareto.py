@@ -68,3 +68,14 @@ def test_large_10_devices_and_shards(px, oracle_mod):
     assert m["n_configs"] == g["n_configs"]
     for k in ("cap", "accsum", "index"):
         assert m[k].tolist() == g[k].tolist(), k
+
+
+def test_bench_size_5_pow_12(px, oracle_mod):
+    """The bench's f3 workload: EfficientNet's 5 variants on 12 devices (4 of
+    each c3 type), 5^12 = 244 140 625 configurations, against the oracle's
+    brute force (every configuration, pairwise dominance)."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    dev = np.repeat(np.arange(3, dtype=np.int32), 4)
+    g = check(px, oracle_mod, cfg["prof"], dev, cfg["cluster"].slo_us, 3, False)
+    assert g["n_configs"] == 5 ** 12
