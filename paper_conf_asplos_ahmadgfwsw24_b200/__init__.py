@@ -139,13 +139,15 @@ class Proteus:
         self._check(self._lib.proteus_solve(self._h, C.byref(a), sols))
         return [self._sol(sols[i], opts[i], zs[i]) for i in range(n_vec)]
 
-    def solve_batch(self, device_type, slo_us, demand, mode=MODE_FACTORED, out=None, fields=None):
+    def solve_batch(self, device_type, slo_us, demand, mode=MODE_FACTORED, out=None, fields=None, shard_rank=0,
+                    shard_world=1):
         """Many demand vectors at once (proteus_solve_batch).  out: dict of
         preallocated arrays (numpy or CUDA torch) keyed by field name, written
         in place; else host numpy arrays are returned for `fields` (default
-        all).  Returns (dict of arrays, n_candidates per vector)."""
+        all).  Modes 0/1 may scan one slice of shard_world (as solve()).
+        Returns (dict of arrays, n_candidates per vector)."""
         keep = []
-        a, n_vec, D = self._solve_args(device_type, slo_us, demand, mode, 0, 1, 0, False, keep)
+        a, n_vec, D = self._solve_args(device_type, slo_us, demand, mode, shard_rank, shard_world, 0, False, keep)
         shapes = {"score": ((n_vec,), np.uint64), "index": ((n_vec,), np.uint64), "served": ((n_vec,), np.int64),
                   "unmet": ((n_vec,), np.int64), "accsum": ((n_vec,), np.int64),
                   "eff_acc_micro": ((n_vec,), np.int32), "option": ((n_vec, D), np.int32),

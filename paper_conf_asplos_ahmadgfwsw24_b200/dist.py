@@ -159,57 +159,57 @@ def replay_sharded(replay, scenarios, group=None, comm_device=None, **kw):
 
 
 # ------------------------------------------------ batched flat search --
-SOL_HEAD = 7  # score, index, served, unmet, accsum, eff, n_candidates per solution, then option[D], z[D]
+BATCH_HEAD = ("score", "index", "served", "unmet", "accsum", "eff_acc_micro")
 
 
-def pack_solutions(sols, D: int) -> np.ndarray:
-    """Per-vector solutions of this rank as int64 rows [n][SOL_HEAD + 2D]
-    (uint64 score / index as their bit patterns)."""
-    out = np.zeros((len(sols), SOL_HEAD + 2 * D), np.int64)
-    for v, s in enumerate(sols):
-        out[v, :SOL_HEAD] = [_to_i64(s.score), _to_i64(s.index), s.served, s.unmet, s.accsum, s.eff_acc_micro,
-                             s.n_candidates]
-        out[v, SOL_HEAD:SOL_HEAD + D] = np.asarray(s.option, np.int64)
-        out[v, SOL_HEAD + D:] = np.asarray(s.z, np.int64)
-    return out
+def pack_batch(out: dict, D: int, ncand: int) -> np.ndarray:
+    """proteus_solve_batch arrays of this rank -> int64 rows [n][7 + 2D]:
+    the BATCH_HEAD fields (uint64 score / index as their bit patterns), the
+    rank's slice size, option[D], z[D]."""
+    n = len(out["score"])
+    cols = [np.asarray(out[k]).astype(np.uint64).view(np.int64).reshape(n, 1) if k in ("score", "index")
+            else np.asarray(out[k], np.int64).reshape(n, 1) for k in BATCH_HEAD]
+    cols.append(np.full((n, 1), ncand, np.int64))
+    cols += [np.asarray(out["option"], np.int64).reshape(n, D), np.asarray(out["z_qps"], np.int64).reshape(n, D)]
+    return np.ascontiguousarray(np.concatenate(cols, axis=1))
 
 
-def pick_solutions(gathered: np.ndarray, D: int):
-    """gathered [world][n][SOL_HEAD + 2D]: per vector the rank with the
+def pick_batch(gathered: np.ndarray, D: int):
+    """gathered [world][n][7 + 2D]: per vector the rank with the
     lexicographic maximum (score desc, index asc) -- its local winner is the
-    global one, already materialised (placement, z, value); n_candidates
-    sums the ranks' slices."""
-    from . import Solution
-    world, n = gathered.shape[0], gathered.shape[1]
-    out = []
-    for v in range(n):
-        best = None
-        for r in range(world):
-            s, i = _to_u64(gathered[r, v, 0]), _to_u64(gathered[r, v, 1])
-            if best is None or s > best[0] or (s == best[0] and i < best[1]):
-                best = (s, i, r)
-        row = gathered[best[2], v]
-        out.append(Solution(best[0], best[1], int(row[2]), int(row[3]), int(row[4]), int(row[5]),
-                            int(gathered[:, v, 6].sum()),
-                            row[SOL_HEAD:SOL_HEAD + D].astype(np.int32), row[SOL_HEAD + D:].astype(np.int32)))
-    return out
+    global one, already materialised (placement, z, value).  Returns (dict of
+    arrays, candidates of the whole space per vector)."""
+    s = gathered[:, :, 0].view(np.uint64)
+    i = gathered[:, :, 1].view(np.uint64)
+    best = s.max(axis=0)
+    r = np.where(s == best[None, :], i, np.uint64(U64)).argmin(axis=0)
+    rows = gathered[r, np.arange(gathered.shape[1])]
+    out = {k: rows[:, c] for c, k in enumerate(BATCH_HEAD)}
+    out["score"] = rows[:, 0].view(np.uint64)
+    out["index"] = rows[:, 1].view(np.uint64)
+    out["option"] = rows[:, 7:7 + D].astype(np.int32)
+    out["z_qps"] = rows[:, 7 + D:].astype(np.int32)
+    return out, int(gathered[:, 0, 6].sum()) if gathered.shape[1] else 0
 
 
 def solve_sharded_batch(px, device_type, slo_us, demand, mode=0, group=None, comm_device=None):
     """Modes 0/1 for a batch of demand vectors on every rank of `group`: one
-    library call scans this rank's index slice for every vector (one host
-    synchronisation per call), then ONE all-gather of the per-rank winners,
+    proteus_solve_batch call scans this rank's index slice for every vector
+    (one host synchronisation), then ONE all-gather of the per-rank winners,
     each already materialised, and the per-vector (score desc, index asc)
-    pick -- no re-materialisation.  Returns (solutions, local solutions)."""
+    pick, all in numpy -- no re-materialisation, no per-vector host objects.
+    Returns (dict of arrays over the batch, this rank's dict, candidates of
+    the whole space per vector, candidates of this rank's slice per vector)."""
     import torch
     import torch.distributed as dist
     world, rank = dist.get_world_size(group), dist.get_rank(group)
     D = len(device_type)
-    local = px.solve(device_type, slo_us, demand, mode=mode, shard_rank=rank, shard_world=world)
-    t = torch.from_numpy(pack_solutions(local, D))
+    local, ncand = px.solve_batch(device_type, slo_us, demand, mode=mode, shard_rank=rank, shard_world=world)
+    t = torch.from_numpy(pack_batch(local, D, ncand))
     if comm_device is not None:
         t = t.to(comm_device)
     parts = [torch.empty_like(t) for _ in range(world)]
     dist.all_gather(parts, t, group=group)
     gathered = np.stack([p.cpu().numpy() for p in parts])
-    return pick_solutions(gathered, D), local
+    best, n_all = pick_batch(gathered, D)
+    return best, local, n_all, ncand

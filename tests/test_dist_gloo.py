@@ -155,7 +155,7 @@ def _batch_worker(rank, world, port, q):
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import torch.distributed as dist
     import oracle
-    from paper_conf_asplos_ahmadgfwsw24_b200 import Solution, workloads as W
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
     from paper_conf_asplos_ahmadgfwsw24_b200.dist import shard_range, solve_sharded_batch
     dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
     try:
@@ -165,20 +165,26 @@ def _batch_worker(rank, world, port, q):
         K, D = 1 + prof.M, len(cl.device_type)
 
         class FakePx:
-            def solve(self, device_type, slo_us, demand, mode, shard_rank, shard_world):
+            def solve_batch(self, device_type, slo_us, demand, mode, shard_rank, shard_world):
                 n = K ** D
                 lo, hi = shard_range(n, shard_rank, shard_world)
-                out = []
+                out = {k: [] for k in ("score", "index", "served", "unmet", "accsum", "eff_acc_micro", "option",
+                                       "z_qps")}
                 for dem in demand:
                     s, i = _rank_best(prof, device_type, slo_us, dem, lo, hi)
                     opt = np.array([(i // K ** (D - 1 - d)) % K for d in range(D)], np.int32)
                     r = oracle.score_placement(prof, device_type, slo_us, dem, opt)
-                    out.append(Solution(s, i, r["served"], r["unmet"], r["accsum"], r["eff"], hi - lo, opt, r["z"]))
-                return out
+                    for k, v in (("score", s), ("index", i), ("served", r["served"]), ("unmet", r["unmet"]),
+                                 ("accsum", r["accsum"]), ("eff_acc_micro", r["eff"]), ("option", opt),
+                                 ("z_qps", r["z"])):
+                        out[k].append(v)
+                out = {k: np.array(v, np.uint64 if k in ("score", "index") else np.int64) for k, v in out.items()}
+                return out, hi - lo
 
-        sols, _ = solve_sharded_batch(FakePx(), cl.device_type, cl.slo_us, dems, mode=0)
-        q.put((rank, [(s.score, s.index, s.served, s.accsum, s.n_candidates, s.option.tolist(), s.z.tolist())
-                      for s in sols]))
+        best, _, ncand, _ = solve_sharded_batch(FakePx(), cl.device_type, cl.slo_us, dems, mode=0)
+        q.put((rank, [(int(best["score"][v]), int(best["index"][v]), int(best["served"][v]),
+                       int(best["accsum"][v]), ncand, best["option"][v].tolist(), best["z_qps"][v].tolist())
+                      for v in range(len(dems))]))
     finally:
         dist.destroy_process_group()
 

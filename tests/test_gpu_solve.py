@@ -294,3 +294,27 @@ def test_c2_bench_batch_sampled(px, oracle_mod):
         assert (chk["served"], chk["accsum"]) == (sol.served, sol.accsum)
         one = px.solve(cl.device_type, cl.slo_us, cfg["demand"][v:v + 1], mode=0)[0]
         assert (one.score, one.index) == (sol.score, sol.index)
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_c2_batch_shards_combine(px, world):
+    """The bench's N-GPU path without NCCL: every rank's proteus_solve_batch
+    over its index slice for the 32-vector batch, packed as dist.pack_batch
+    and combined by dist.pick_batch (the all-gather's result), equals the
+    one-GPU batch -- score, index, value, placement and z of every vector."""
+    import bench
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    from paper_conf_asplos_ahmadgfwsw24_b200.dist import pack_batch, pick_batch
+    cfg = W.config("c2", totals=bench.C2_TOTALS)
+    prof, cl = cfg["prof"], cfg["cluster"]
+    px.load_profiles(prof)
+    D = len(cl.device_type)
+    ref, n = px.solve_batch(cl.device_type, cl.slo_us, cfg["demand"], mode=0)
+    parts = []
+    for r in range(world):
+        loc, nc = px.solve_batch(cl.device_type, cl.slo_us, cfg["demand"], mode=0, shard_rank=r, shard_world=world)
+        parts.append(pack_batch(loc, D, nc))
+    best, n_all = pick_batch(np.stack(parts), D)
+    assert n_all == n == 13**8
+    for k in ("score", "index", "served", "unmet", "accsum", "eff_acc_micro", "option", "z_qps"):
+        assert np.array_equal(np.asarray(best[k]).astype(np.int64), np.asarray(ref[k]).astype(np.int64)), k
