@@ -488,11 +488,17 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     alg_bytes = N * S * 4 + N * 8   # latency writes + one read of the per-device arrays
     hbm = peaks.get("hbm_gbs", 6650.0)
     # e2e with host buffers: H2D of the trace, D2H of all latencies
+    # (the first call also page-locks the 2.56 GB host output: untimed)
     arr_h, fam_h = cfg["arrival_us"], cfg["family"]
-    barrier()
-    t0 = time.perf_counter()
-    px.replay(arr_h, fam_h, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=True)
-    e2e = time.perf_counter() - t0
+    e2e_ts = []
+    for _ in range(3):
+        barrier()
+        t0 = time.perf_counter()
+        r_h = px.replay(arr_h, fam_h, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc,
+                        latency=True)
+        e2e_ts.append(time.perf_counter() - t0)
+        del r_h
+    e2e = statistics.median(e2e_ts[1:])
     out["c5_replay"] = {
         "queries": N, "scenarios": S_all, "ms": ms, "query_scenarios_per_s": N * S_all / (ms / 1e3),
         "routing_ms": route_ms, "lane_kernels_ms": lane, "kernel_split_ms": split,
