@@ -212,3 +212,20 @@ def test_replay_baseline_edge_cases(px, oracle_mod):
         fam = np.zeros(len(arr), np.uint8)
         sc = np.array([(m, c, 0, p) for m in (100, 1000) for c in (1, 4, 0) for p in (0, 1, 2)], np.int32)
         _compare(px, oracle_mod, cfg["prof"], cfg["cluster"], r["option"], r["z"], cfg["demand"][0], arr, fam, sc)
+
+
+def test_replay_scenario_errors(px, oracle_mod):
+    """Invalid scenario rows are rejected before any output is written:
+    policy outside 0..2, routing outside 0..1, negative multiplier or cap."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import ProteusError, workloads as W
+    cfg = W.config("c3")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    r = oracle_mod.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][0], 2)
+    a, f = W.query_trace(1000, 3000.0, cfg["weights"], 3, "poisson")
+    px.load_profiles(prof)
+    for bad in ([1000, 0, 0, 3], [1000, 0, 2, 0], [-1, 0, 0, 0], [1000, -2, 0, 1]):
+        lat = np.full((1, len(a)), 7, np.uint32)
+        with pytest.raises(ProteusError):
+            px.replay(a, f, r["option"], r["z"], cl.device_type, cfg["demand"][0], cl.slo_us,
+                      np.array([bad], np.int32), latency=lat)
+        assert np.all(lat == 7)
