@@ -310,6 +310,15 @@ struct LaneArgs {
                           // freed (backlog), and all speculative decisions; k_fix leaves backlogged lanes
                           // (a quarter or more) to the stitch's max-plus stretches
   long long debug;        // > 0: k_stitch prints lanes slower than this many cycles (diagnostic)
+  uint8_t *wst;           // baseline chunk runs: [S][NS] 0, or 1 + the run's AIMD limit (Nexus: 1) at a
+                          // decision whose head found the device free (NULL: no chunk runs)
+  struct WcExit *wx;      // baseline chunk runs: [S][NCH] exit state
+};
+
+struct WcExit {  // a baseline chunk run left its chunk at head h (>= chunk end), device free at F;
+  int64_t h, F;    // its last decision dropped [.., first) and served [first, h) (Nexus drops can
+  int64_t first;   // reach past the chunk end)
+  int32_t limit, pad;
 };
 
 __device__ __forceinline__ uint32_t sat_lat(int64_t l) { return l >= 0xFFFFFFFFll ? 0xFFFFFFFEu : (uint32_t)l; }
@@ -403,6 +412,77 @@ __global__ void __launch_bounds__(LANE_THREADS) k_lanes(const __grid_constant__ 
 // coalesced loads as the head advances; reads past it go to global memory),
 // T(b) in shared memory; latencies are written 32 per store (coalesced).
 #define WC_RW 1024
+// Chunk runs of the baseline batchers (thread per (scenario, chunk of CH
+// queries of a device)): the rule replayed from an idle device at the chunk's
+// first query, latencies / drops written for the chunk's positions, and at
+// every decision whose head finds the device free the mark 1 + limit (AIMD;
+// Nexus: 1).  A decision from head h with the device free at a_h depends on h
+// (and AIMD's limit) only, so the true run that reaches such a head in the
+// same state continues exactly as this run: k_wc_lanes jumps to its exit.
+__global__ void __launch_bounds__(128) k_wc_spec(const __grid_constant__ LaneArgs a) {
+  const int64_t cg = (int64_t)blockIdx.y * blockDim.x + threadIdx.x;  // chunk over all devices
+  if (cg >= a.choff[a.D]) return;
+  int d = 0;
+  while (cg >= a.choff[d + 1]) d++;
+  const int s = a.sc_list[blockIdx.x];
+  const LaneParam p = a.lp[s * a.D + d];
+  const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+  const int64_t c = cg - a.choff[d];
+  const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
+  uint32_t *out = a.latd + (size_t)s * a.NS + off;
+  uint8_t *mk = a.wst + (size_t)s * a.NS + off;
+  WcExit e = {en, 0, en, 1, 0};
+  if (p.Bmax >= 1) {
+    const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+    const uint32_t *arr = a.devArr + off;
+    const bool nexus = p.policy == 1;
+    const int B = nexus ? p.Bn : p.Bmax;
+    int64_t h = st, F = 0, last_first = st;
+    int limit = 1;
+    while (h < en) {
+      const int64_t ah = __ldg(arr + h);
+      const int64_t t = F > ah ? F : ah;
+      if (F <= ah) mk[h] = (uint8_t)(nexus ? 1 : (limit < 254 ? limit + 1 : 255));
+      int64_t first = h;
+      int b;
+      if (nexus) {
+        int64_t i = h;
+        int w = 0;
+        for (;; i++) {  // sliding window from the head (R14)
+          if (i >= n || (int64_t)__ldg(arr + i) > t) break;  // past the queue: all dropped
+          w = 1;
+          while (w < B && i + w < n && (int64_t)__ldg(arr + i + w) <= t) w++;
+          if (t + T[w - 1] <= (int64_t)__ldg(arr + i) + p.L) break;
+          if (i < en) out[i] = 0xFFFFFFFFu;
+          w = 0;
+        }
+        if (w == 0) { h = i; last_first = i; continue; }  // everything queued was dropped
+        first = i;
+        b = w;
+      } else {
+        int q = 1;
+        while (q < limit && h + q < n && (int64_t)__ldg(arr + h + q) <= t) q++;
+        b = q;
+      }
+      const int64_t Fn = t + T[b - 1];
+      for (int64_t j = first; j < first + b && j < en; j++) out[j] = sat_lat(Fn - (int64_t)__ldg(arr + j));
+      if (!nexus) {
+        if (Fn - ah > p.L) limit = limit * 9 / 10 < 1 ? 1 : limit * 9 / 10;
+        else limit = limit + 1 > p.Bmax ? p.Bmax : limit + 1;
+      }
+      F = Fn;
+      h = first + b;
+      last_first = first;
+    }
+    e.h = h;
+    e.F = F;
+    e.first = last_first;
+    e.limit = limit;
+  }
+  a.wx[(size_t)s * a.NCH + cg] = e;
+}
+
+template <bool CHUNKS>  // CHUNKS: meet the chunk runs of k_wc_spec (a.wst, a.wx)
 __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneArgs a) {
   __shared__ uint32_t sA[4][WC_RW];
   __shared__ int32_t sT[4][PX_MAXB];
@@ -442,6 +522,8 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
   int limit = 1;                   // AIMD batch-size limit
   const int64_t T1 = T[0];
   const bool fast = T1 <= p.L;     // isolated queries are on time
+  int64_t cc = 0, cend = a.CH < n ? a.CH : n;  // chunk of the head
+  const uint8_t *wrow = CHUNKS ? a.wst + (size_t)s * a.NS + st : nullptr;
   while (h < n) {
     if (h - b0 >= WC_RW / 2) {     // slide the ring
       const int64_t nb = h & ~(int64_t)(WC_RW / 2 - 1);
@@ -450,6 +532,21 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
       else fill(nb, WC_RW);
       b0 = nb;
       __syncwarp();
+    }
+    if (CHUNKS) {  // chunk runs: meet one at a free head in the same state, jump to its exit
+      while (h >= cend) { cc++; cend = (cc + 1) * a.CH < n ? (cc + 1) * a.CH : n; }
+      const uint8_t mkh = wrow[h];
+      if (mkh && F <= A(h) && (nexus || (int)mkh == limit + 1)) {
+        const WcExit e = a.wx[(size_t)s * a.NCH + a.choff[d] + cc];
+        // the run's last batch may reach into the next chunks: their rows hold
+        // those chunks' own runs there, so this batch's latencies are rewritten
+        for (int64_t j = cend + lane; j < e.h; j += 32) out[j] = j < e.first ? 0xFFFFFFFFu : sat_lat(e.F - A(j));
+        h = e.h;
+        F = e.F;
+        limit = e.limit;
+        if (tail < h) tail = h;
+        continue;
+      }
     }
     if (nexus ? B == 1 : limit == 1) {
       // Batches of one, 32 per step: query h + k leaves at max(F_{k-1}, a)
@@ -1723,7 +1820,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
               const proteus_scenario *h_sc, int S, uint32_t *d_lat_out, uint64_t *d_agg) {
   const int Q = ctx->Q, M = ctx->M;
   PX_CUDA(ctx, cudaMemsetAsync(d_agg, 0, ((size_t)3 * S + 1) * 8, ctx->stream));
-  const size_t small = (size_t)(4 * D + 2 * Q + 2 * PX_MAXQ + 8 + 6 * S + 4 * (PX_MAXD + 2)) * 4 +
+  const size_t small = (size_t)(4 * D + 2 * Q + 2 * PX_MAXQ + 8 + 8 * S + 4 * (PX_MAXD + 2)) * 4 +
                        (size_t)S * sizeof(proteus_scenario) + (size_t)S * D * sizeof(LaneParam) +
                        (size_t)2 * (PX_MAXD + 2) * 8;
   char *sb = (char *)px_buf(ctx, B_R_MISC, small + 4096);
@@ -1731,27 +1828,29 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   int32_t *d_opt = (int32_t *)sb, *d_z = d_opt + D, *d_dev = d_z + D, *d_dem = d_dev + D, *d_slo = d_dem + Q;
   int32_t *d_pat_off = d_slo + Q, *d_pat_len = d_pat_off + PX_MAXQ;
   uint32_t *d_flags = (uint32_t *)(d_pat_len + PX_MAXQ);  // [0] trace checks, [4] fix-up changes
-  // [6][S] scenario lists: per routing mode rt, row rt = every scenario, row 2 + rt = the §5
-  // scenarios (chunk / scan kernels), row 4 + rt = the baseline batchers (k_wc_lanes)
+  // [8][S] scenario lists: per routing mode rt, row rt = every scenario, row 2 + rt = the §5
+  // scenarios (chunk / scan kernels), row 4 + rt = the baseline batchers (k_wc_lanes), row
+  // 6 + rt = the AIMD ones (k_wc_spec chunk runs)
   int32_t *d_scl = (int32_t *)(d_flags + 8);
-  int32_t *d_goff = d_scl + 6 * S;                        // [2][PX_MAXD + 2]
+  int32_t *d_goff = d_scl + 8 * S;                        // [2][PX_MAXD + 2]
   int64_t *d_choff = (int64_t *)(((uintptr_t)(d_goff + 2 * (PX_MAXD + 2)) + 15) & ~(uintptr_t)15);  // [2][PX_MAXD + 2]
   proteus_scenario *d_sc = (proteus_scenario *)(d_choff + 2 * (PX_MAXD + 2));
   LaneParam *d_lp = (LaneParam *)(((uintptr_t)(d_sc + S) + 15) & ~(uintptr_t)15);
-  std::vector<int32_t> scl[6];
+  std::vector<int32_t> scl[8];
   for (int s = 0; s < S; s++) {
     scl[h_sc[s].routing].push_back(s);
     scl[(h_sc[s].policy == 0 ? 2 : 4) + h_sc[s].routing].push_back(s);
+    if (h_sc[s].policy == 2) scl[6 + h_sc[s].routing].push_back(s);
   }
-  std::vector<int32_t> scl_all(6 * S, 0);
-  for (int r = 0; r < 6; r++)
+  std::vector<int32_t> scl_all(8 * S, 0);
+  for (int r = 0; r < 8; r++)
     for (size_t k = 0; k < scl[r].size(); k++) scl_all[r * S + k] = scl[r][k];
   PX_CUDA(ctx, cudaMemcpyAsync(d_opt, h_option, D * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_z, h_z, D * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_dev, h_dev_type, D * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_dem, h_demand, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_slo, h_slo, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
-  PX_CUDA(ctx, cudaMemcpyAsync(d_scl, scl_all.data(), 6 * S * 4, cudaMemcpyHostToDevice, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(d_scl, scl_all.data(), 8 * S * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_sc, h_sc, S * sizeof(proteus_scenario), cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemsetAsync(d_flags, 0, 4, ctx->stream));
   if (N > 0) {
@@ -1994,12 +2093,32 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       }
     }
     }  // §5 scenarios
-    if (!scl[4 + rt].empty()) {  // §8(f2) baseline batchers: warp per (device, scenario)
+    if (!scl[4 + rt].empty()) {  // §8(f2) baseline batchers: chunk runs, then warp per (device, scenario)
       LaneArgs lb = la;
       lb.nsc = (int)scl[4 + rt].size();
       lb.sc_list = d_scl + (4 + rt) * S;
+      lb.wst = nullptr;
+      lb.wx = nullptr;
+      // chunk runs for the AIMD scenarios only: an overloaded Nexus lane never finds the
+      // device free, so its runs never meet (measured: no gain, +6 % for the runs)
+      if (env_int("PROTEUS_REPLAY_WCSPEC", 1) && !scl[6 + rt].empty() && (NCH[rt] + 127) / 128 <= 65535 &&
+          NCH[rt] > 0) {
+        uint8_t *wst = (uint8_t *)px_buf(ctx, B_R_WST, (size_t)S * NS + 16);
+        WcExit *wx = (WcExit *)px_buf(ctx, B_R_WEX, sizeof(WcExit) * (size_t)S * nmax + 16);
+        if (!wst || !wx) return px_fail(ctx, PROTEUS_ENOMEM, "baseline chunk runs");
+        for (int k : scl[4 + rt])
+          PX_CUDA(ctx, cudaMemsetAsync(wst + (size_t)k * NS, 0, (size_t)NS, ctx->stream));
+        lb.wst = wst;
+        lb.wx = wx;
+        LaneArgs la2 = lb;
+        la2.nsc = (int)scl[6 + rt].size();
+        la2.sc_list = d_scl + (6 + rt) * S;
+        dim3 gs((unsigned)la2.nsc, (unsigned)((NCH[rt] + 127) / 128));
+        PX_LAUNCH(ctx, "replay_baseline", k_wc_spec, gs, 128, 0, la2);
+      }
       const int64_t warps = (int64_t)lb.nsc * D;
-      PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes, (unsigned)((warps + 3) / 4), 128, 0, lb);
+      if (lb.wst) PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<true>, (unsigned)((warps + 3) / 4), 128, 0, lb);
+      else PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<false>, (unsigned)((warps + 3) / 4), 128, 0, lb);
     }
     const int nall = (int)scl[rt].size();
     dim3 g(32, nall < 65535 ? nall : 65535);

@@ -229,3 +229,20 @@ def test_replay_scenario_errors(px, oracle_mod):
             px.replay(a, f, r["option"], r["z"], cl.device_type, cfg["demand"][0], cl.slo_us,
                       np.array([bad], np.int32), latency=lat)
         assert np.all(lat == 7)
+
+
+@pytest.mark.parametrize("env", [{"PROTEUS_REPLAY_CHUNK": "16"}, {"PROTEUS_REPLAY_CHUNK": "37"},
+                                 {"PROTEUS_REPLAY_CHUNK": "1000"}, {"PROTEUS_REPLAY_WCSPEC": "0"}])
+def test_replay_baseline_chunk_runs(px, oracle_mod, env, monkeypatch):
+    """AIMD lanes meeting k_wc_spec's chunk runs at free heads in the same
+    limit (tiny chunks: batches straddling chunk ends, exits several chunks
+    ahead), and the walk without chunk runs; light load and overload."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    for v, kind in ((0, "poisson"), (1, "gamma")):
+        r = _alloc(oracle_mod, cfg, v)
+        arr, fam = W.query_trace(40_000, float(cfg["demand"][v].sum()), cfg["weights"], 21 + v, kind)
+        sc = np.concatenate([W.scenarios_64(0, 2), W.scenarios_64(0, 1)[::5]])
+        _compare(px, oracle_mod, cfg["prof"], cfg["cluster"], r["option"], r["z"], cfg["demand"][v], arr, fam, sc)
