@@ -522,9 +522,12 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
   int limit = 1;                   // AIMD batch-size limit
   const int64_t T1 = T[0];
   const bool fast = T1 <= p.L;     // isolated queries are on time
+  bool try_stretch = true;         // Nexus: look for an overload stretch at the next busy decision
+  long long dbg_t0 = clock64(), dbg_steps = 0, dbg_st = 0, dbg_stb = 0;
   int64_t cc = 0, cend = a.CH < n ? a.CH : n;  // chunk of the head
   const uint8_t *wrow = CHUNKS ? a.wst + (size_t)s * a.NS + st : nullptr;
   while (h < n) {
+    dbg_steps++;
     if (h - b0 >= WC_RW / 2) {     // slide the ring
       const int64_t nb = h & ~(int64_t)(WC_RW / 2 - 1);
       __syncwarp();
@@ -586,6 +589,54 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
       continue;
     }
     const int64_t ah = A(h);
+    if (nexus && B > 1 && F > ah && try_stretch) {
+      // Overload stretch (Nexus): the device is busy at every decision and the
+      // queue holds a full window, so batch k of the stretch is decided at
+      // t_k = F + k T(B): the window of B from the head passes iff a_i >=
+      // t_k + T(B) - L, so its head is i_k = max(p_k, g_k), g_k = the first
+      // arrival >= that threshold, p_k = i_{k-1} + B (p_0 = h): i_k = k B +
+      // max(h, max_{j<=k} g_j - j B), a prefix maximum over the lanes.  The
+      // queries in [p_k, i_k) are dropped.  Batch k is valid while the device
+      // is busy (a_{p_k} <= t_k) and the window is full (a_{i_k + B - 1} <=
+      // t_k); the stretch ends before the first invalid one (32 per step).
+      const int64_t TB = T[B - 1];
+      const int k = lane;
+      const int64_t tk = F + (int64_t)k * TB;
+      const int64_t thr = tk + TB - p.L;
+      int64_t x = h + (int64_t)k * B;  // g_k clamped below by h + k B (only larger values matter)
+      if (x < n && A(x) < thr) {       // gallop, then bisect: first index >= x with a >= thr
+        int64_t lo = x, step = 1, hi = x + 1;
+        while (hi < n && A(hi) < thr) { lo = hi; step <<= 1; hi = x + step; }
+        if (hi > n) hi = n;
+        while (hi - lo > 1) { const int64_t mid = (lo + hi) >> 1; if (A(mid) < thr) lo = mid; else hi = mid; }
+        x = hi;
+      }
+      int64_t m = x - (int64_t)k * B;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int64_t v = __shfl_up_sync(0xffffffffu, m, o);
+        if (lane >= o) m = v > m ? v : m;
+      }
+      const int64_t ik = (int64_t)k * B + (m > h ? m : h);
+      int64_t pk = __shfl_up_sync(0xffffffffu, ik + B, 1);
+      if (lane == 0) pk = h;
+      const bool ok = ik + B <= n && pk < n && A(pk) <= tk && A(ik + B - 1) <= tk;
+      const unsigned vm = __ballot_sync(0xffffffffu, ok);
+      const int r = vm == 0xffffffffu ? 32 : __ffs(~vm) - 1;
+      if (r > 0) {
+        dbg_st++; dbg_stb += r;
+        if (lane < r) {
+          for (int64_t j = pk; j < ik; j++) out[j] = 0xFFFFFFFFu;  // dropped early
+          const int64_t Fk = tk + TB;
+          for (int q = 0; q < B; q++) out[ik + q] = sat_lat(Fk - A(ik + q));
+        }
+        F += (int64_t)r * TB;
+        h = __shfl_sync(0xffffffffu, ik + B, r - 1);
+        if (tail < h) tail = h;
+        continue;
+      }
+      try_stretch = false;  // not in a stretch here: test again after a busy full-window batch
+    }
     if (fast && ah >= F) {
       // Isolated queries, 32 per ballot: query j finds the device free (a_j >=
       // F, resp. a_j >= a_{j-1} + T(1) after its predecessor went alone) and no
@@ -636,6 +687,7 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
     }
     const int cap = nexus ? B : limit;
     const int b = (int)(tail - first < cap ? tail - first : cap);
+    if (nexus && b == B && t == F) try_stretch = true;  // busy, full window: a stretch may follow
     F = t + T[b - 1];
     for (int k = lane; k < b; k += 32) out[first + k] = sat_lat(F - A(first + k));
     if (!nexus) {  // completion feedback (the next decision is at >= F)
@@ -644,6 +696,9 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
     }
     h = first + b;
   }
+  if (a.debug && lane == 0 && clock64() - dbg_t0 > a.debug)
+    printf("wc s=%d d=%d n=%lld pol=%d B=%d cycles=%lld steps=%lld stretches=%lld stretch_batches=%lld\n", s, d,
+           (long long)n, p.policy, B, clock64() - dbg_t0, dbg_steps, dbg_st, dbg_stb);
 }
 
 // ---- phase A: speculative chunks
