@@ -348,3 +348,32 @@ def test_c1_c2_regimes(oracle_mod):
     r = oracle_mod.solve(cfg["prof"], cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"][0], 0)
     assert r["unmet"] == 0 and r["eff"] < 1_000_000 and r["n_candidates"] == 7**4
 
+
+
+def test_optimum_dominates_clipper_ht_ha(oracle_mod):
+    """(vi) The joint optimum is at least the value of the static Clipper
+    placements: Clipper-HT allocates with only each family's
+    least accurate variant, Clipper-HA with only its most accurate one -- the
+    same search over a subset of the options (the other variants made
+    infeasible: latency 0 = does not fit, reading C7).  Also: with a single
+    variant per family the restricted and full searches coincide."""
+    from paper_conf_asplos_ahmadgfwsw24_b200.workloads import Profiles
+    rng = np.random.default_rng(31)
+    for _ in range(25):
+        prof, dev, slo, P = random_instance(rng, T=2, Q=2, Vmax=3, D=3, Pmax=25)
+        s = rng.integers(0, 70, size=prof.Q)
+        full = oracle_mod.solve(prof, dev, slo, s, 0)
+        off = np.concatenate([[0], np.cumsum(prof.V)[:-1]])
+        for pick in ("HT", "HA"):
+            lat = prof.lat_us.copy()
+            for q in range(prof.Q):
+                accs = prof.acc_micro[off[q]:off[q] + prof.V[q]]
+                keep = off[q] + (int(np.argmin(accs)) if pick == "HT" else int(np.argmax(accs)))
+                for m in range(off[q], off[q] + prof.V[q]):
+                    if m != keep:
+                        lat[:, m, :] = 0
+            sub = Profiles(T=prof.T, Q=prof.Q, V=prof.V, acc_micro=prof.acc_micro, bmax=prof.bmax, lat_us=lat)
+            r = oracle_mod.solve(sub, dev, slo, s, 0)
+            assert (full["served"], full["accsum"]) >= (r["served"], r["accsum"]), pick
+            if all(v == 1 for v in prof.V):
+                assert (full["served"], full["accsum"]) == (r["served"], r["accsum"])
