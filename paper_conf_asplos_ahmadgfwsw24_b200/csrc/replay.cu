@@ -2369,12 +2369,14 @@ __global__ void __launch_bounds__(128) k_ep_spec(const __grid_constant__ EpArgs 
 // device array.
 __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArgs a) {
   __shared__ uint32_t sA[4][WC_RW];
+  __shared__ uint32_t sL[4][WC_RW];  // the idle runs' latencies of the same positions
   __shared__ int32_t sT[4][PX_MAXB];
   const int wid = (int)((blockIdx.x * (unsigned)blockDim.x + threadIdx.x) >> 5), lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   if (wid >= a.S * a.D) return;
   const int s = wid / a.D, d = wid % a.D;
   uint32_t *ring = sA[w];
+  uint32_t *lring = sL[w];
   int32_t *T = sT[w];
   const int64_t dbase = a.devOff[d], dn = a.devOff[d + 1] - dbase;  // the device's array
   const uint32_t *arr = a.devArr + dbase;
@@ -2384,10 +2386,14 @@ __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArg
     for (int k = lane; k < cnt; k += 32) {
       const int64_t j = from + k;
       ring[j & (WC_RW - 1)] = j < dn ? __ldg(arr + j) : 0xFFFFFFFFu;
+      lring[j & (WC_RW - 1)] = j < dn ? row[j] : 0u;  // positions >= the head: not rewritten yet
     }
   };
   auto A = [&](int64_t j) -> int64_t {  // j >= b0
     return j - b0 < WC_RW ? (int64_t)ring[j & (WC_RW - 1)] : (int64_t)__ldg(arr + j);
+  };
+  auto Lspec = [&](int64_t j) -> int64_t {  // the idle run's latency at j >= the head
+    return j - b0 < WC_RW ? (int64_t)lring[j & (WC_RW - 1)] : (int64_t)row[j];
   };
   int64_t F = 0;  // R13
   for (int e = 0; e < a.E; e++) {
@@ -2414,7 +2420,7 @@ __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArg
         __syncwarp();
       }
       const int64_t a0 = A(h);
-      if (h > st && F <= a0 && specPrev <= a0 && a0 + (int64_t)row[h] != specPrev) { met = true; break; }
+      if (h > st && F <= a0 && specPrev <= a0 && a0 + Lspec(h) != specPrev) { met = true; break; }
       const int B = p.Bmax;
       if (h + B <= en && A(h + B - 1) <= F) {
         // backlog: Bmax queued when the device frees -> a full batch leaves at
@@ -2428,7 +2434,7 @@ __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArg
           const unsigned m = __ballot_sync(0xffffffffu, full);
           const int r = m == 0xffffffffu ? 32 : __ffs(~m) - 1;
           const int64_t hs = h + (int64_t)done * B, ns = (int64_t)r * B;
-          if (ns > 0) specPrev = A(hs + ns - 1) + (int64_t)row[hs + ns - 1];
+          if (ns > 0) specPrev = A(hs + ns - 1) + Lspec(hs + ns - 1);
           __syncwarp();
           for (int64_t i = lane; i < ns; i += 32) {
             const int64_t kb = i / B;
@@ -2445,7 +2451,7 @@ __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArg
       auto Tl = [&](int j) -> int64_t { return (int64_t)T[j]; };
       const int b = decide_warp(A, en, h, F, p.Bmax, p.L, Tl, lane, &t);
       const int64_t Fn = t + T[b - 1];
-      specPrev = A(h + b - 1) + (int64_t)row[h + b - 1];
+      specPrev = A(h + b - 1) + Lspec(h + b - 1);
       __syncwarp();
       for (int i = lane; i < b; i += 32) row[h + i] = sat_lat(Fn - A(h + i));
       F = Fn;
