@@ -523,6 +523,7 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
   const int64_t T1 = T[0];
   const bool fast = T1 <= p.L;     // isolated queries are on time
   bool try_stretch = true;         // Nexus: look for an overload stretch at the next busy decision
+  int stretch_wait = 0;            // decisions to let pass before the next stretch test
   long long dbg_t0 = clock64(), dbg_steps = 0, dbg_st = 0, dbg_stb = 0;
   int64_t cc = 0, cend = a.CH < n ? a.CH : n;  // chunk of the head
   const uint8_t *wrow = CHUNKS ? a.wst + (size_t)s * a.NS + st : nullptr;
@@ -538,8 +539,8 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
     }
     if (CHUNKS) {  // chunk runs: meet one at a free head in the same state, jump to its exit
       while (h >= cend) { cc++; cend = (cc + 1) * a.CH < n ? (cc + 1) * a.CH : n; }
-      const uint8_t mkh = wrow[h];
-      if (mkh && F <= A(h) && (nexus || (int)mkh == limit + 1)) {
+      const uint8_t mkh = F <= A(h) ? wrow[h] : 0;  // a global read only when the device is free
+      if (mkh && (nexus || (int)mkh == limit + 1)) {
         const WcExit e = a.wx[(size_t)s * a.NCH + a.choff[d] + cc];
         // the run's last batch may reach into the next chunks: their rows hold
         // those chunks' own runs there, so this batch's latencies are rewritten
@@ -589,7 +590,7 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
       continue;
     }
     const int64_t ah = A(h);
-    if (nexus && B > 1 && F > ah && try_stretch) {
+    if (nexus && B > 1 && F > ah && try_stretch && --stretch_wait <= 0) {
       // Overload stretch (Nexus): the device is busy at every decision and the
       // queue holds a full window, so batch k of the stretch is decided at
       // t_k = F + k T(B): the window of B from the head passes iff a_i >=
@@ -625,6 +626,7 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
       const int r = vm == 0xffffffffu ? 32 : __ffs(~vm) - 1;
       if (r > 0) {
         dbg_st++; dbg_stb += r;
+        stretch_wait = r < 4 ? 8 : 0;  // short stretches do not pay for the test: back off
         if (lane < r) {
           for (int64_t j = pk; j < ik; j++) out[j] = 0xFFFFFFFFu;  // dropped early
           const int64_t Fk = tk + TB;
@@ -636,6 +638,7 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
         continue;
       }
       try_stretch = false;  // not in a stretch here: test again after a busy full-window batch
+      stretch_wait = 8;
     }
     if (fast && ah >= F) {
       // Isolated queries, 32 per ballot: query j finds the device free (a_j >=
