@@ -208,8 +208,13 @@ def solve_sharded_batch(px, device_type, slo_us, demand, mode=0, group=None, com
     t = torch.from_numpy(pack_batch(local, D, ncand))
     if comm_device is not None:
         t = t.to(comm_device)
-    parts = [torch.empty_like(t) for _ in range(world)]
-    dist.all_gather(parts, t, group=group)
-    gathered = np.stack([p.cpu().numpy() for p in parts])
+    if t.is_cuda:  # NCCL: one flat buffer, one device-to-host copy
+        flat = torch.empty((world,) + tuple(t.shape), dtype=t.dtype, device=t.device)
+        dist.all_gather_into_tensor(flat, t, group=group)
+        gathered = flat.cpu().numpy()
+    else:
+        parts = [torch.empty_like(t) for _ in range(world)]
+        dist.all_gather(parts, t, group=group)
+        gathered = np.stack([p.numpy() for p in parts])
     best, n_all = pick_batch(gathered, D)
     return best, local, n_all, ncand
