@@ -318,3 +318,20 @@ def test_c2_batch_shards_combine(px, world):
     assert n_all == n == 13**8
     for k in ("score", "index", "served", "unmet", "accsum", "eff_acc_micro", "option", "z_qps"):
         assert np.array_equal(np.asarray(best[k]).astype(np.int64), np.asarray(ref[k]).astype(np.int64)), k
+
+
+def test_nccl_collective_paths_world1():
+    """The NCCL code paths of dist.solve_sharded_batch (all_gather_into_tensor)
+    and dist.replay_sharded (all-reduce gather) in a world-1 NCCL process
+    group on cuda:0 (subprocess): results equal the direct calls."""
+    import os
+    import socket
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    with socket.socket() as s_:
+        s_.bind(("127.0.0.1", 0))
+        port = s_.getsockname()[1]
+    r = subprocess.run([sys.executable, os.path.join(root, "scripts", "nccl_world1.py"), str(port)],
+                       capture_output=True, text=True, timeout=600, cwd=root)
+    assert r.returncode == 0 and "nccl world-1 ok" in r.stdout, (r.stdout + r.stderr)[-3000:]
