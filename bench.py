@@ -39,7 +39,7 @@ INT_LANES_PER_SM_CLK = 128   # 4 SMSPs x 1 warp-instruction/clk x 32 lanes (DESI
 SM_MAX_MHZ_FALLBACK = 1965.0
 # one step = the exhaustive c2 search for a batch of NVEC demand vectors (totals
 # 1500..7500 QPS, Zipf split: from the all-most-accurate regime to overload)
-NVEC = 32
+NVEC = 64
 C2_TOTALS = tuple(int(t) for t in np.linspace(1500, 7500, NVEC))
 WORKLOAD = (f"c2: exhaustive flat mixed-radix allocation search, 4 families x 3 variants on 8 devices "
             f"(types cpu x2, gpu_a x3, gpu_b x3), 13^8 = 815730721 candidates per demand vector, a batch of "
@@ -169,7 +169,7 @@ def run_reference(args, rank, world):
         "config": {"workload": WORKLOAD},
         "cpu_baseline": {"value": value, "unit": "candidates/s", "cores": cores, "kind": "oracle",
                          "sample": "per step the full c2 search for one demand vector of the batch (vector "
-                                   "step mod 32, 815730721 candidates), exhaustive enumeration + memoised "
+                                   "step mod 64, 815730721 candidates), exhaustive enumeration + memoised "
                                    "vertex-enumeration LP per family"},
         "e2e": {"value": value, "unit": "candidates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }

@@ -271,7 +271,7 @@ def test_random_flat_kernel(px, oracle_mod):
 
 
 def test_c2_bench_batch_sampled(px, oracle_mod):
-    """The bench's launch configuration: the 32-vector c2 batch in one call
+    """The bench's launch configuration: the 64-vector c2 batch in one call
     (one flat launch, grid.y = vector) with device-resident inputs.  Sampled
     vectors against the exhaustive oracle; every vector's placement re-scored
     by the oracle, and the batch equal to one-vector calls."""
@@ -299,7 +299,7 @@ def test_c2_bench_batch_sampled(px, oracle_mod):
 @pytest.mark.parametrize("world", [2, 3, 8])
 def test_c2_batch_shards_combine(px, world):
     """The bench's N-GPU path without NCCL: every rank's proteus_solve_batch
-    over its index slice for the 32-vector batch, packed as dist.pack_batch
+    over its index slice for the 64-vector batch, packed as dist.pack_batch
     and combined by dist.pick_batch (the all-gather's result), equals the
     one-GPU batch -- score, index, value, placement and z of every vector."""
     import bench
