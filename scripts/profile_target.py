@@ -19,11 +19,12 @@ from paper_conf_asplos_ahmadgfwsw24_b200 import Proteus, workloads as W  # noqa:
 
 def main(what):
     px = Proteus(0)
-    if what == "c2":
-        cfg = W.config("c2")
+    if what == "c2":  # the bench's step: the c2 batch (flat launches of 32 vectors)
+        import bench
+        cfg = W.config("c2", totals=bench.C2_TOTALS)
         px.load_profiles(cfg["prof"])
-        s = px.solve(cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"][:1], mode=0)[0]
-        print("c2", s.index, s.served, s.accsum)
+        out, n = px.solve_batch(cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"], mode=0)
+        print("c2", int(out["index"][0]), n)
     elif what == "c4":
         cfg = W.config("c4")
         px.load_profiles(cfg["prof"])
