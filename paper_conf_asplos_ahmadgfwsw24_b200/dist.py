@@ -9,9 +9,19 @@ all-reduce assembles all slots, and every rank picks the lexicographic maximum
 argmax, so the result is identical for every world size.  128 bytes at 8
 ranks; NCCL over NVLink on GPUs, gloo in the CPU tests.
 
+Batched flat search (the bench step): every rank scans its slice for every
+demand vector of the batch in one library call, and ONE all-gather of the
+per-rank winners -- each already materialised -- gives every rank the batch's
+optima (solve_sharded_batch; no re-materialisation).
+
 Factored batched re-solve (mode 2, config c4): demand vectors are
 independent; rank r solves vectors [r*n/world, (r+1)*n/world) -- no collective
 on the data path (weak scaling).
+
+Replay / closed loop (c5, f2, f4): scenarios are independent; rank r replays
+its slice and one SUM all-reduce of a zero-padded [3][S] vector gathers the
+per-scenario aggregates (replay_sharded).  Fig. 1b: index-range slices and a
+host-side frontier merge (pareto_merge).
 """
 
 from __future__ import annotations
