@@ -20,7 +20,7 @@
 #include "internal.cuh"
 
 #define FLAT_THREADS 256
-#define FLAT_NV 32  // demand vectors per flat launch (grid.y)
+#define FLAT_NV 64  // demand vectors per flat launch (grid.y)
 #ifndef FLAT_MINB
 #define FLAT_MINB 2  // blocks per SM the register budget is sized for
 #endif

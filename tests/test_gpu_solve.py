@@ -272,7 +272,7 @@ def test_random_flat_kernel(px, oracle_mod):
 
 def test_c2_bench_batch_sampled(px, oracle_mod):
     """The bench's launch configuration: the 64-vector c2 batch in one call
-    (flat launches of up to 32 vectors, grid.y = vector) with device-resident inputs.  Sampled
+    (one flat launch, grid.y = vector) with device-resident inputs.  Sampled
     vectors against the exhaustive oracle; every vector's placement re-scored
     by the oracle, and the batch equal to one-vector calls."""
     import torch
