@@ -189,6 +189,7 @@ struct FlatArgs {
   int64_t out_stride;      // rows of block winners per vector
   const int32_t *Pdev, *code_slot;
   BestRec *out;
+  unsigned long long *gbound;  // per vector of the launch: best score any thread has found (0 at launch)
 };
 
 // water-fill of family q over slots q*VM..q*VM+VM-1, with capacity pa added
@@ -249,7 +250,12 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
       for (int s = 0; s < S; s++) sCapsB[s][threadIdx.x] = cb[s];
     };
     rebuild();
+    unsigned long long *gb = a.gbound + blockIdx.y;
     for (;;) {
+      // grid-wide lower bound: the best score any thread of this vector has
+      // recorded so far (relaxed load, issued early; a stale value is only lower)
+      uint64_t G;
+      asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(G) : "l"(gb));
       const int o3 = dig[D - 3];
       const int sl3 = sCS[o3], p3 = sP[(D - 3) * K + o3];
       int caps[S];
@@ -289,6 +295,13 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
       uint64_t lb = best_s;
       int lp = -1;
       if (best_i == ~0ull) { lb = base; lp = 0; }  // the thread's first candidate
+      // Candidates below G cannot be the answer (G is the score of a real
+      // candidate), so the threshold is raised to G - 1: the rows still flag
+      // every candidate >= G (ties with G keep the lowest index), and the thread
+      // that holds the first maximum records it -- its score M >= G always
+      // exceeds the threshold until the thread has recorded M.  A thread that
+      // records nothing reports (0, ~0), the neutral element of the argmax.
+      if (G > 0 && G - 1 > lb) { lb = G - 1; lp = -1; }
       {
         const uint64_t thr = lb - base;
         if (base > lb || M1 > thr) {
@@ -319,7 +332,11 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
           }
         }
       }
-      if (lp >= 0) { best_s = lb; best_i = p * KK + (uint64_t)lp; }
+      if (lp >= 0) {
+        best_s = lb;
+        best_i = p * KK + (uint64_t)lp;
+        if (lb > G) atomicMax(gb, (unsigned long long)lb);
+      }
       if (++p >= pend) break;
       if (++dig[D - 3] == K) {
         dig[D - 3] = 0;
@@ -418,7 +435,7 @@ template <int QM, int VM>
 static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p_hi, const int32_t *dev_type,
                        const int32_t *demand, int nvec, const std::vector<int32_t> &h_P,
                        const std::vector<int32_t> &h_slot_code, const Tables &tab, BestRec *d_blocks,
-                       int64_t out_stride, int *nblocks_out) {
+                       int64_t out_stride, unsigned long long *gbound, int *nblocks_out) {
   FlatArgs<QM, VM> a;
   memset(&a, 0, sizeof a);
   a.D = D; a.K = K;
@@ -437,6 +454,8 @@ static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p
   a.Pdev = tab.Pdev;
   a.code_slot = tab.code_slot;
   a.out = d_blocks;
+  a.gbound = gbound;
+  PX_CUDA(ctx, cudaMemsetAsync(gbound, 0, sizeof(unsigned long long) * (size_t)nvec, ctx->stream));
   const size_t smem = (size_t)(D * K + K) * 4;
   auto kern = k_flat_pair<QM, VM>;
   if (smem > 48 * 1024) PX_CUDA(ctx, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -471,7 +490,7 @@ static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p
 
 typedef int (*flat_fn)(proteus_ctx *, int, int, uint64_t, uint64_t, const int32_t *, const int32_t *, int,
                        const std::vector<int32_t> &, const std::vector<int32_t> &, const Tables &, BestRec *, int64_t,
-                       int *);
+                       unsigned long long *, int *);
 
 struct FlatInst { int QM, VM; flat_fn fn; };
 static const FlatInst kFlat[] = {
@@ -545,7 +564,8 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
   // materialise launch for the whole batch at the end (block = vector)
   const int64_t stride = (int64_t)max_blocks + 1;
   const int nv = materialize_only ? 1 : vec_hi - vec_lo;
-  BestRec *d_blocks0 = (BestRec *)px_buf(ctx, B_BEST, sizeof(BestRec) * (size_t)stride * nv);
+  // per-block winners, then one grid-wide bound per vector (flat kernel)
+  BestRec *d_blocks0 = (BestRec *)px_buf(ctx, B_BEST, sizeof(BestRec) * (size_t)stride * nv + 8 * (size_t)nv);
   if (!d_blocks0) return px_fail(ctx, PROTEUS_ENOMEM, "block results");
   uint64_t ncand_all = 0;
   int nb_all = 0, flat_nb = 0;
@@ -565,8 +585,10 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
         if ((v - vec_lo) % FLAT_NV == 0) {  // one launch per FLAT_NV vectors (grid.y = vector)
           const int nvec = vec_hi - v < FLAT_NV ? vec_hi - v : FLAT_NV;
           const FlatInst *f = pick_flat(Q, *std::max_element(ctx->V.begin(), ctx->V.end()));
+          unsigned long long *gbound =
+              (unsigned long long *)(d_blocks0 + (size_t)stride * nv) + (v - vec_lo);
           int rc = f->fn(ctx, D, K, plo, phi, h_dev_type, dem, nvec, h_P, h_slot_code, tab, d_blocks, stride,
-                         &flat_nb);
+                         gbound, &flat_nb);
           if (rc) return rc;
         }
         nb = flat_nb;
