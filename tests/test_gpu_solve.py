@@ -101,6 +101,19 @@ def test_c2_flat_full(px, oracle_mod):
     assert sols[1].unmet > 0
 
 
+def test_c2_flat_full_ties(px, oracle_mod):
+    """Config 2 at full size with tiny demands: millions of candidates tie at
+    the maximum, spread over every thread of the launch, so the flat kernel's
+    grid-wide score bound (threshold G - 1) must still return the lowest index
+    among the maxima (reading C9); the all-zero vector ties everywhere at 0
+    (answer: index 0).  Oracle = exhaustive enumeration."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c2")
+    dem = np.array([[5, 5, 5, 5], [0, 0, 0, 0], [1, 0, 0, 0]], dtype=np.int32)
+    sols = check(px, oracle_mod, cfg["prof"], cfg["cluster"].device_type, cfg["cluster"].slo_us, dem, 0)
+    assert sols[1].index == 0 and sols[1].score == 0
+
+
 def test_c2_generic_kernel_and_multiset(px, oracle_mod):
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
     cfg = W.config("c2")
