@@ -20,10 +20,12 @@
 #include "internal.cuh"
 
 #ifndef FLAT_THREADS
-// 384 x 1 block per SM: 168 registers (fewer spills than 256 x 2 at 128) and
-// 12 warps/SM; measured on the c2 batch (ms per 64 vectors): 384x1 16.8,
-// 256x2 18.1, 512x1 17.3, 448x1 19.5, 352x1 18.5, 192x2 18.3, 128x4 18.9
-#define FLAT_THREADS 384
+// 512 x 1 block per SM (128 registers, 16 warps/SM).  Measured on the c2 batch
+// (ms per 64 vectors) before the grid-wide bound: 384x1 16.8, 256x2 18.1,
+// 512x1 17.3, 448x1 19.5, 352x1 18.5, 192x2 18.3, 128x4 18.9; with it (fewer
+// flagged rows, so the spill-heavy re-scans matter less): 512x1 16.0,
+// 384x1 16.4, 256x2 16.4
+#define FLAT_THREADS 512
 #endif
 #define FLAT_NV 64  // demand vectors per flat launch (grid.y)
 #ifndef FLAT_MINB
