@@ -27,7 +27,7 @@
 // 384x1 16.4, 256x2 16.4
 #define FLAT_THREADS 512
 #endif
-#define FLAT_NV 64  // demand vectors per flat launch (grid.y)
+#define FLAT_NV 64  // demand vectors per flat launch (grid.x)
 #ifndef FLAT_MINB
 #define FLAT_MINB 1  // blocks per SM the register budget is sized for
 #endif
@@ -187,7 +187,7 @@ struct FlatArgs {
   int32_t PA[QM * VM];  // capacity of slot on device D-2
   int32_t PB[QM * VM];  // capacity of slot on device D-1
   int32_t code[QM * VM];
-  int32_t s[FLAT_NV][QM];  // demand of each vector of the launch (grid.y)
+  int32_t s[FLAT_NV][QM];  // demand of each vector of the launch (grid.x)
   int64_t out_stride;      // rows of block winners per vector
   const int32_t *Pdev, *code_slot;
   BestRec *out;
@@ -220,10 +220,14 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
   int32_t *sCS = smem + D * K; // [K]
   for (int i = threadIdx.x; i < D * K; i += blockDim.x) sP[i] = a.Pdev[i];
   for (int i = threadIdx.x; i < K; i += blockDim.x) sCS[i] = a.code_slot[i];
-  __shared__ int32_t sDem[QM];  // this launch row's demand vector (grid.y)
-  if (threadIdx.x < QM) sDem[threadIdx.x] = a.s[blockIdx.y][threadIdx.x];
+  __shared__ int32_t sDem[QM];  // this block's demand vector (grid.x)
+  // grid.x = vector (fastest), grid.y = prefix range: the blocks of one vector
+  // are spread over the whole launch, so most of them start with the
+  // grid-wide bound of their vector already raised by the earlier ones
+  const int vec = blockIdx.x, blk = blockIdx.y;
+  if (threadIdx.x < QM) sDem[threadIdx.x] = a.s[vec][threadIdx.x];
   __syncthreads();
-  const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t tid = (uint64_t)blk * blockDim.x + threadIdx.x;
   uint64_t p = a.p_lo + tid * a.per_thread;
   const uint64_t pend = p + a.per_thread < a.p_hi ? p + a.per_thread : a.p_hi;
   const uint64_t KK = (uint64_t)K * K;
@@ -252,7 +256,7 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
       for (int s = 0; s < S; s++) sCapsB[s][threadIdx.x] = cb[s];
     };
     rebuild();
-    unsigned long long *gb = a.gbound + blockIdx.y;
+    unsigned long long *gb = a.gbound + vec;
     for (;;) {
       // grid-wide lower bound: the best score any thread of this vector has
       // recorded so far (relaxed load, issued early; a stale value is only lower)
@@ -352,7 +356,7 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
   }
   block_best(best_s, best_i);
   if (threadIdx.x == 0) {
-    BestRec &o = a.out[(int64_t)blockIdx.y * a.out_stride + blockIdx.x];
+    BestRec &o = a.out[(int64_t)vec * a.out_stride + blk];
     o.score = best_s;
     o.index = best_i;
   }
@@ -485,7 +489,7 @@ static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p
   if (a.per_thread > (uint64_t)K) a.per_thread = (a.per_thread + K - 1) / K * K;
   nb = (np + a.per_thread * FLAT_THREADS - 1) / (a.per_thread * FLAT_THREADS);
   if (nb == 0) nb = 1;
-  PX_LAUNCH(ctx, "score_flat_pair", kern, dim3((unsigned)nb, (unsigned)nvec), FLAT_THREADS, smem, a);
+  PX_LAUNCH(ctx, "score_flat_pair", kern, dim3((unsigned)nvec, (unsigned)nb), FLAT_THREADS, smem, a);
   *nblocks_out = (int)nb;
   return 0;
 }
@@ -584,7 +588,7 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
         const uint64_t NP = N / ((uint64_t)K * K);
         const uint64_t plo = mul_div(NP, rank, world), phi = mul_div(NP, rank + 1, world);
         ncand = (phi - plo) * (uint64_t)K * K;
-        if ((v - vec_lo) % FLAT_NV == 0) {  // one launch per FLAT_NV vectors (grid.y = vector)
+        if ((v - vec_lo) % FLAT_NV == 0) {  // one launch per FLAT_NV vectors (grid.x = vector)
           const int nvec = vec_hi - v < FLAT_NV ? vec_hi - v : FLAT_NV;
           const FlatInst *f = pick_flat(Q, *std::max_element(ctx->V.begin(), ctx->V.end()));
           unsigned long long *gbound =
