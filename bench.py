@@ -268,7 +268,7 @@ def main():
     # roofline of the dominant kernel (score_flat_pair, one launch per demand vector)
     peaks, peak_src = measured_peaks()
     k_ms = statistics.mean(kern_ms) if kern_ms else float("nan")
-    # one launch scores the rank's slice for up to 64 vectors of the batch (grid.y = vector)
+    # one launch scores the rank's slice for up to 64 vectors of the batch (grid.x = vector)
     launches_per_step = max(1, len(kern_ms) // args.steps)
     cand_per_launch = ncl * NVEC / launches_per_step  # ncl: this rank's candidates per vector
     ops = flat_pair_ops_per_candidate(4, 3, 13) * cand_per_launch
