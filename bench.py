@@ -34,13 +34,14 @@ sys.path.insert(0, ROOT)
 
 import numpy as np  # noqa: E402
 
-SM_COUNT = 148
-INT_LANES_PER_SM_CLK = 128   # 4 SMSPs x 1 warp-instruction/clk x 32 lanes
 SM_MAX_MHZ_FALLBACK = 1965.0
+SOLREC_BYTES = 568           # csrc/internal.cuh SolRec (D <= 64)
+# algorithmic int ops per c2 candidate, incremental scoring
+# (only the innermost digit changes, other families cached): 5 V + 9 = 24
+S8D_OPS_PER_CANDIDATE = 24
 # one step = the exhaustive c2 search for a batch of NVEC demand vectors (totals
 # 1500..7500 QPS, Zipf split: from the all-most-accurate regime to overload)
-NVEC = 64
-C2_TOTALS = tuple(int(t) for t in np.linspace(1500, 7500, NVEC))
+from paper_conf_asplos_ahmadgfwsw24_b200.workloads import C2_BENCH_NVEC as NVEC, C2_BENCH_TOTALS as C2_TOTALS  # noqa: E402
 WORKLOAD = (f"c2: exhaustive flat mixed-radix allocation search, 4 families x 3 variants on 8 devices "
             f"(types cpu x2, gpu_a x3, gpu_b x3), 13^8 = 815730721 candidates per demand vector, a batch of "
             f"{NVEC} demand vectors per step (totals 1500..7500 QPS, seed 202)")
@@ -105,28 +106,57 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.sm)}
 
 
-# algorithmic int32 lane-ops per candidate of the pair-incremental scoring in
-# k_flat_pair: per prefix (options of devices 0..D-3) the K^2
-# candidates of the last two devices.  fill = one family water-fill of V
-# variants (min, multiply-add, subtract per variant; pack 2).
-def flat_pair_ops_per_candidate(Q, V, K):
-    S = Q * V
-    fill = 3 * V + 2
-    per_prefix = (S                       # add device D-3's capacity to its slot
-                  + Q * fill              # family values of the prefix
-                  + S * (fill + 2)        # deltas Fb of every option of device D-1
-                  + 2 * S + 4 * Q         # largest delta per family (64-bit max), top two families
-                  + 2 + 2 + 2             # idle row: threshold, (idle, idle), best other-family compare
-                  + S * ((fill + 4)       # row sa: delta of device D-2's option, ba
-                         + 2 + 2          #   threshold, (sa, idle) compare
-                         + 3              #   other-family candidates: select M1/M2, one 64-bit compare
-                         + V * (fill + 6)))  # same-family candidates: joint fill, combine, compare
-    return per_prefix / (K * K)
-
-
 # the lane kernels of the replay (a12): their algorithmic bytes are the latency
-# rows written plus one read of the per-device arrays
+# rows written plus one read of the per-device arrays; the
+# writers put the latencies in query order
 LANE_KERNELS = ("replay_scan1", "replay_bscan", "replay_spec", "replay_fix", "replay_stitch", "replay_lanes")
+WRITE_KERNELS = ("replay_unpermute",)
+
+
+def int_peaks():
+    """Measured integer-pipe peaks of this B200 (scripts/int_peaks.cu ->
+    MEASURED_INT_PEAKS.json): lane-instructions per second of the ALU pipe
+    (IADD3 / VIMNMX / ISETP / LOP3), the FMA pipe (IMAD) and the issue limit
+    (both pipes, 1 warp-instruction / clk / SMSP)."""
+    p = os.path.join(ROOT, "MEASURED_INT_PEAKS.json")
+    with open(p) as f:
+        return json.load(f)
+
+
+def kernel_inst(kernel):
+    """ncu instruction counts of `kernel` per unit of work (warp-level
+    sm__inst_executed_pipe_alu / _fma / sm__inst_executed per candidate or
+    evaluation) from the committed capture summary profiles/inst_counts.json."""
+    p = os.path.join(ROOT, "profiles", "inst_counts.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        return json.load(f).get(kernel)
+
+
+def alu_roofline(kernel, inst, k_ms, ip, units, s8d_ops_per_unit, unit_name):
+    """Roofline of an integer-bound kernel against the MEASURED pipe peaks:
+    achieved = ALU-pipe lane-instructions per launch (ncu count per unit x the
+    units one launch processes) / the launch's live CUDA-event time.  Also the
+    issue fraction (all pipes) and SURVEY §8(d)'s algorithmic figure (ops per
+    unit / ALU peak), which exceeds 1 when the kernel skips work exactly."""
+    alu_peak = ip["alu_lane_instr_per_s"]
+    issue_peak = ip["issue_lane_instr_per_s"]
+    r = {"kernel": kernel, "bound": "alu", "unit": "lane-instr/s", "peak": alu_peak,
+         "peak_source": "measured (MEASURED_INT_PEAKS.json: ALU pipe, scripts/int_peaks.cu)",
+         "kernel_ms": k_ms, "units_per_launch": units, "unit_of_work": unit_name,
+         "s8d_ops_per_unit": s8d_ops_per_unit,
+         "s8d_algorithmic_frac": s8d_ops_per_unit * units / (k_ms / 1e3) / alu_peak}
+    if inst and k_ms == k_ms:
+        alu = inst["alu_per_unit"] * units * 32
+        tot = inst["inst_per_unit"] * units * 32
+        r.update(achieved=alu / (k_ms / 1e3), frac=alu / (k_ms / 1e3) / alu_peak,
+                 issue_frac=tot / (k_ms / 1e3) / issue_peak,
+                 fma_frac=inst["fma_per_unit"] * units * 32 / (k_ms / 1e3) / ip["fma_lane_instr_per_s"],
+                 traffic=inst.get("dram_bytes_per_unit", 0) * units, inst_source=inst.get("source"))
+    else:
+        r.update(achieved=None, frac=None, traffic=None)
+    return r
 
 
 # algorithmic int32 lane-ops of one (count vector, demand vector) evaluation in
@@ -193,7 +223,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_asplos_ahmadgfwsw24_b200 import Proteus, workloads as W
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import solve_sharded_batch
+    from paper_conf_asplos_ahmadgfwsw24_b200.dist import init_comm
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -221,6 +251,8 @@ def main():
         return float(t.item())
 
     px = Proteus(local)
+    if world > 1:  # the library's own NCCL communicator: every call below is distributed
+        init_comm(px)
     stream = torch.cuda.current_stream(dev)
     flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)  # > 126 MB L2
 
@@ -233,11 +265,10 @@ def main():
     t_dem = torch.as_tensor(cfg["demand"], dtype=torch.int32, device=dev)
 
     def step(d=t_dev, sl=t_slo, dm=t_dem):
-        """(solutions of the batch as arrays, this rank's, candidates per vector: all, this rank's)"""
-        if world > 1:  # index-range slices, one all-gather of the materialised per-rank winners
-            return solve_sharded_batch(px, d, sl, dm, 0, None, dev)
-        out, nc = px.solve_batch(d, sl, dm, mode=0)
-        return out, out, nc, nc
+        """(solutions of the batch as arrays, candidates per vector).  N > 1: each
+        rank scans its index slice, the library all-gathers the materialised
+        per-rank winners over NCCL and picks on the device"""
+        return px.solve_batch(d, sl, dm, mode=0)
 
     for _ in range(args.warmup):
         step()
@@ -252,7 +283,7 @@ def main():
             flush.zero_()
             barrier()
             ev[k][0].record(stream)
-            sols, loc, _, ncl = step()
+            sols, _ = step()
             ev[k][1].record(stream)
             barrier()
             kern_ms += [ms for name, ms in px.kernel_times() if name == "score_flat_pair"]
@@ -270,16 +301,10 @@ def main():
     k_ms = statistics.mean(kern_ms) if kern_ms else float("nan")
     # one launch scores the rank's slice for up to 64 vectors of the batch (grid.x = vector)
     launches_per_step = max(1, len(kern_ms) // args.steps)
-    cand_per_launch = ncl * NVEC / launches_per_step  # ncl: this rank's candidates per vector
-    ops = flat_pair_ops_per_candidate(4, 3, 13) * cand_per_launch
-    sm_mhz = clocks["sm_mhz"] or peaks.get("sm_max_mhz", SM_MAX_MHZ_FALLBACK)
-    peak_ops = SM_COUNT * INT_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12
-    achieved = ops / (k_ms / 1e3) / 1e12
-    traffic = None
-    tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp):
-        with open(tp) as f:
-            traffic = json.load(f).get("score_flat_pair")
+    ncl = 13**8 // world  # this rank's candidates per vector (index slice)
+    cand_per_launch = ncl * NVEC / launches_per_step
+    roof = alu_roofline("score_flat_pair", kernel_inst("score_flat_pair"), k_ms, int_peaks(), cand_per_launch,
+                        S8D_OPS_PER_CANDIDATE, "candidate (covered: scored or excluded by an exact row bound)")
 
     # e2e: the same batch through the public API with HOST buffers
     e2e_t = []
@@ -292,7 +317,7 @@ def main():
         e2e_t.append(time.perf_counter() - t0)
     e2e_s = max_over_ranks(statistics.median(e2e_t))
     h2d = cl.device_type.nbytes + cl.slo_us.nbytes + cfg["demand"].nbytes
-    d2h = NVEC * (2 * 4 * len(cl.device_type) + 64)
+    d2h = NVEC * SOLREC_BYTES + 12  # the solution records (host outputs) + status word + candidate count
     # time to optimal: one demand vector, host call -> solution in host memory
     one = []
     for _ in range(10):
@@ -308,13 +333,9 @@ def main():
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "int32/int64 (exact integer)", "data": "synthetic",
         "config": {"workload": WORKLOAD, "l2": "flushed (256 MB write) before every timed step",
-                   "parallelism": (f"index-range shards x{world}, one NCCL all-gather of the per-rank winners "
-                                   f"per batch") if world > 1 else "1 GPU"},
-        "roofline": {"kernel": "score_flat_pair", "bound": "alu", "achieved": achieved, "peak": peak_ops,
-                     "unit": "Tops/s (int32 lane-ops)", "frac": achieved / peak_ops, "traffic": traffic,
-                     "kernel_ms": k_ms, "ops_per_candidate": flat_pair_ops_per_candidate(4, 3, 13),
-                     "peak_basis": f"148 SMs x 128 int32 lane-ops/clk x {sm_mhz:.0f} MHz (median SM clock "
-                                   f"during the run; DESIGN.md §5)"},
+                   "parallelism": (f"index-range shards x{world}, one ncclAllGather of the materialised per-rank "
+                                   f"winners per batch + a device pick, inside libproteus") if world > 1 else "1 GPU"},
+        "roofline": roof,
         "e2e": {"value": n_cand / e2e_s, "unit": "candidates/s", "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": int(d2h)},
         "gpu_launches": int(sum_over_ranks(launches)),
@@ -345,55 +366,74 @@ def main():
         dist.destroy_process_group()
 
 
+def _ksplit(kts):
+    """median per kernel name over repeated calls' kernel_times()"""
+    acc = {}
+    for kt in kts:
+        per = {}
+        for n_, v in kt:
+            per[n_] = per.get(n_, 0.0) + v
+        for n_, v in per.items():
+            acc.setdefault(n_, []).append(v)
+    return {k: statistics.median(v) for k, v in acc.items()}
+
+
+def time_replay(px, barrier, max_over_ranks, stream, reps, call):
+    """device time of `call` (CUDA events on the library's stream, max over
+    ranks) and the library's per-kernel split"""
+    import torch
+    call()
+    px.set_timing(True)
+    ts, kts = [], []
+    for _ in range(reps):
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        res = call()
+        b.record(stream)
+        barrier()
+        ts.append(a.elapsed_time(b))
+        kts.append(px.kernel_times())
+    px.set_timing(False)
+    return max_over_ranks(statistics.median(ts)), _ksplit(kts), res
+
+
 def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, peaks, peak_src):
     import torch
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import shard_range
     out = {}
     stream = torch.cuda.current_stream(dev)
-    # c4: per-second re-solve of the paper-scale cluster, 3600 vectors (weak: vectors split by rank)
+    hbm = peaks.get("hbm_gbs", 6650.0)
+    ip = int_peaks()
+    scope = "all ranks (the library splits the work over its NCCL communicator)" if world > 1 else "1 GPU"
+    # c4: per-second re-solve of the paper-scale cluster, 3600 vectors (N > 1:
+    # vectors split by rank inside the library, one all-gather of the solutions)
     cfg = W.config("c4")
     prof, cl = cfg["prof"], cfg["cluster"]
     px.load_profiles(prof)
-    lo, hi = shard_range(len(cfg["demand"]), rank, world)
     t_dev = torch.as_tensor(cl.device_type, dtype=torch.int32, device=dev)
     t_slo = torch.as_tensor(cl.slo_us, dtype=torch.int32, device=dev)
-    t_dem = torch.as_tensor(cfg["demand"][lo:hi], dtype=torch.int32, device=dev)
+    t_dem = torch.as_tensor(cfg["demand"], dtype=torch.int32, device=dev)
     t_one = torch.as_tensor(cfg["demand"][:1], dtype=torch.int32, device=dev)
-    nv, D = hi - lo, len(cl.device_type)
+    nv, D = len(cfg["demand"]), len(cl.device_type)
     dout = {"score": torch.empty(nv, dtype=torch.uint64, device=dev),
             "served": torch.empty(nv, dtype=torch.int64, device=dev),
             "unmet": torch.empty(nv, dtype=torch.int64, device=dev),
             "accsum": torch.empty(nv, dtype=torch.int64, device=dev),
             "option": torch.empty((nv, D), dtype=torch.int32, device=dev),
             "z_qps": torch.empty((nv, D), dtype=torch.int32, device=dev)}
-    for _ in range(2):
-        px.solve_batch(t_dev, t_slo, t_dem, mode=2, out=dout)
-    ts, kts = [], []
-    px.set_timing(True)
-    for _ in range(5):
+    ncand_box = [0]
+
+    def c4_call():
         flush.zero_()
-        barrier()
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        _, ncand = px.solve_batch(t_dev, t_slo, t_dem, mode=2, out=dout)
-        b.record(stream)
-        barrier()
-        ts.append(a.elapsed_time(b))
-        kts.append(px.kernel_times())
-    px.set_timing(False)
-    ms = max_over_ranks(statistics.median(ts))
-    ksplit = {}
-    for kt in kts:
-        for n_, v in kt:
-            ksplit.setdefault(n_, []).append(v)
-    ksplit = {k: statistics.median(v) for k, v in ksplit.items()}
-    # e2e: host demand in, host solutions out (the call a user makes)
+        _, ncand_box[0] = px.solve_batch(t_dev, t_slo, t_dem, mode=2, out=dout)
+    ms, ksplit, _ = time_replay(px, barrier, max_over_ranks, stream, 5, c4_call)
+    ncand = ncand_box[0]
     e2e_t = []
     for _ in range(3):
         barrier()
         t0 = time.perf_counter()
-        px.solve_batch(cl.device_type, cl.slo_us, cfg["demand"][lo:hi], mode=2)
+        px.solve_batch(cl.device_type, cl.slo_us, cfg["demand"], mode=2)
         barrier()
         e2e_t.append(time.perf_counter() - t0)
     e2e_ms = max_over_ranks(statistics.median(e2e_t)) * 1e3
@@ -404,143 +444,89 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
         px.solve(t_dev, t_slo, t_one, mode=2)
         one.append((time.perf_counter() - t0) * 1e3)
     g_ms = ksplit.get("fact_g", float("nan"))
-    evals = nv * ncand  # this rank's vectors x count vectors per vector
-    g_ops = evals * fact_g_ops(5)
-    sm_mhz = peaks.get("sm_max_mhz", SM_MAX_MHZ_FALLBACK)
-    peak_ops = SM_COUNT * INT_LANES_PER_SM_CLK * sm_mhz * 1e6 / 1e12
+    g_inst = kernel_inst("fact_g")
     out["c4_resolve"] = {
-        "vectors": len(cfg["demand"]), "ms_all_vectors": ms, "ms_per_vector_batched": ms / max(1, hi - lo),
-        "kernel_ms": ksplit,
-        "e2e_ms_host_buffers": e2e_ms,
-        "single_vector_time_to_optimal_ms": statistics.median(one),
-        "subplacements_per_vector": ncand,
-        "subplacements_per_s": (len(cfg["demand"]) * ncand) / (ms / 1e3),
-        "roofline": {"kernel": "fact_g", "bound": "alu", "achieved": g_ops / (g_ms / 1e3) / 1e12, "peak": peak_ops,
-                     "unit": "Tops/s (int32 lane-ops)", "frac": g_ops / (g_ms / 1e3) / 1e12 / peak_ops,
-                     "ops_per_evaluation": fact_g_ops(5), "evaluations": evals,
-                     "peak_basis": f"148 SMs x 128 int32 lane-ops/clk x {sm_mhz:.0f} MHz (max SM clock)"},
-        "scaling": "weak (vectors split by rank)"}
+        "vectors": nv, "ms_all_vectors": ms, "ms_per_vector_batched": ms / nv, "kernel_ms": ksplit,
+        "e2e_ms_host_buffers": e2e_ms, "single_vector_time_to_optimal_ms": statistics.median(one),
+        "subplacements_per_vector": ncand, "subplacements_per_s": nv * ncand / (ms / 1e3),
+        "roofline": alu_roofline("fact_g", g_inst, g_ms, ip, nv * ncand // world, fact_g_ops(5), "evaluation"),
+        "scaling": "strong (3600 vectors split by rank, one ncclAllGather)" if world > 1 else "1 GPU"}
     # f3: Fig. 1b Pareto frontier, EfficientNet (5 variants) on 12 devices of the
-    # c3 types (4 each): 5^12 = 244 140 625 configurations (index-range shards)
+    # c3 types (4 each): 5^12 = 244 140 625 configurations
     cfg = W.config("c3")
     prof, cl = cfg["prof"], cfg["cluster"]
     px.load_profiles(prof)
-    pdev = np.repeat(np.arange(3, dtype=np.int32), 4)
-    t_pdev = torch.as_tensor(pdev, device=dev)
+    t_pdev = torch.as_tensor(np.repeat(np.arange(3, dtype=np.int32), 4), device=dev)
     t_pslo = torch.as_tensor(cl.slo_us, dtype=torch.int32, device=dev)
-    for _ in range(2):
-        px.pareto(t_pdev, t_pslo, 3, shard_rank=rank, shard_world=world)
-    pts, pk = [], []
-    px.set_timing(True)
-    for _ in range(3):
-        barrier()
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        pr = px.pareto(t_pdev, t_pslo, 3, shard_rank=rank, shard_world=world)
-        b.record(stream)
-        barrier()
-        pts.append(a.elapsed_time(b))
-        pk.append(sum(ms for n, ms in px.kernel_times() if n in ("pareto_best", "pareto_index")))
-    px.set_timing(False)
-    pms = max_over_ranks(statistics.median(pts))
+    pms, pk, pr = time_replay(px, barrier, max_over_ranks, stream, 3, lambda: px.pareto(t_pdev, t_pslo, 3))
     out["f3_pareto"] = {
         "workload": "Fig. 1b frontier: 5 EfficientNet variants on 12 devices (cpu/gpu_a/gpu_b x4), 5^12 configurations",
         "configs": 5 ** 12, "ms": pms, "configs_per_s": 5 ** 12 / (pms / 1e3),
-        "scan_kernels_ms": statistics.median(pk), "frontier_points": int(pr["n_front"]),
-        "scaling": "strong (index-range shards)" if world > 1 else "1 GPU"}
-    # c5: replay 10M queries x 64 scenarios (scenarios on every rank; N>1 = replicas)
-    cfg = W.config("c5")
-    prof, cl = cfg["prof"], cfg["cluster"]
-    px.load_profiles(prof)
-    alloc = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=2)[0]
-    arr = torch.from_numpy(cfg["arrival_us"]).to(dev)
-    fam = torch.from_numpy(cfg["family"]).to(dev)
-    # N > 1: the scenarios are split by rank (dist.replay_sharded);
-    # value = all ranks' query-scenarios / the slowest rank's time
-    sc_all = cfg["scenarios"]
-    slo_, shi_ = shard_range(len(sc_all), rank, world)
-    sc = sc_all[slo_:shi_]
-    S, N = len(sc), len(cfg["arrival_us"])
-    S_all = len(sc_all)
-    lat = torch.empty((S, N), dtype=torch.uint32, device=dev)
-    for _ in range(2):
-        px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
-    px.set_timing(True)
-    ts, lane_ms = [], []
-    for _ in range(3):
-        barrier()
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        res = px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
-        b.record(stream)
-        barrier()
-        ts.append(a.elapsed_time(b))
-        kt = px.kernel_times()
-        lane_ms.append(sum(ms for n, ms in kt if n in LANE_KERNELS))
-        route_ms = sum(ms for n, ms in kt if n.startswith("route"))
-        split = {}
-        for n, ms_ in kt:
-            if n.startswith("replay") or n.startswith("route"):
-                split[n] = split.get(n, 0.0) + ms_
-    px.set_timing(False)
-    ms = max_over_ranks(statistics.median(ts))
-    lane = statistics.median(lane_ms)
-    alg_bytes = N * S * 4 + N * 8   # latency writes + one read of the per-device arrays
-    hbm = peaks.get("hbm_gbs", 6650.0)
-    # e2e with host buffers: H2D of the trace, D2H of all latencies
-    # (the first call also page-locks the 2.56 GB host output: untimed)
-    arr_h, fam_h = cfg["arrival_us"], cfg["family"]
-    e2e_ts = []
-    for _ in range(3):
-        barrier()
-        t0 = time.perf_counter()
-        r_h = px.replay(arr_h, fam_h, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc,
-                        latency=True)
-        e2e_ts.append(time.perf_counter() - t0)
-        del r_h
-    e2e = statistics.median(e2e_ts[1:])
-    out["c5_replay"] = {
-        "queries": N, "scenarios": S_all, "ms": ms, "query_scenarios_per_s": N * S_all / (ms / 1e3),
-        "routing_ms": route_ms, "lane_kernels_ms": lane, "kernel_split_ms": split,
-        "roofline": {"kernel": " + ".join(LANE_KERNELS), "bound": "hbm", "achieved": alg_bytes / (lane / 1e3) / 1e9,
-                     "peak": hbm, "unit": "GB/s", "frac": alg_bytes / (lane / 1e3) / 1e9 / hbm,
-                     "peak_source": peak_src, "alg_bytes": alg_bytes},
-        "violations_first_scenarios": [int(x) for x in res["violations"][:4]],
-        "e2e": {"value": N * S_all / max_over_ranks(e2e), "unit": "query-scenarios/s",
-                "h2d_bytes_per_step": int(N * 5), "d2h_bytes_per_step": int(N * S * 4)},
-        "scaling": "strong (scenarios split by rank)" if world > 1 else "1 GPU"}
-    # f2: the §6.4 baseline batchers (Nexus early drop, Clipper AIMD) on the same
-    # trace and allocation, 64 scenarios each (k_wc_lanes), plus the Fig. 6-style
-    # violation ratios of all three policies at SLO 2x, batch cap = table depth
-    f2 = {}
-    for pol, name in ((1, "nexus"), (2, "aimd")):
-        scp_all = W.scenarios_64(0, pol)
-        plo, phi = shard_range(len(scp_all), rank, world)
-        scp = scp_all[plo:phi]
-        px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, scp, latency=lat)
-        px.set_timing(True)
-        ts, kms = [], []
-        for _ in range(3):
-            barrier()
-            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a.record(stream)
-            rp = px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, scp,
-                           latency=lat)
-            b.record(stream)
-            barrier()
-            ts.append(a.elapsed_time(b))
-            kms.append(sum(ms_ for n, ms_ in px.kernel_times() if n == "replay_baseline"))
-        px.set_timing(False)
-        pms = max_over_ranks(statistics.median(ts))
-        km = statistics.median(kms)
-        sel = [i for i, r in enumerate(scp) if r[0] == 2000 and r[1] == 0]
-        f2[name] = {"ms": pms, "query_scenarios_per_s": N * len(scp_all) / (pms / 1e3), "lane_kernel_ms": km,
-                    "lane_kernel_hbm_frac": (N * len(scp) * 4 + N * 8) / (km / 1e3) / 1e9 / hbm,
-                    "violation_ratio_slo2x_depth": float(rp["violations"][sel[0]]) / N if sel else None}
-    sel = [i for i, r in enumerate(sc) if r[0] == 2000 and r[1] == 0]
-    f2["proteus_violation_ratio_slo2x_depth"] = float(res["violations"][sel[0]]) / N if sel else None
-    f2["workload"] = "c5 trace (10M Poisson queries) and allocation, 64 (SLO x batch cap) scenarios per policy"
-    out["f2_baseline_batchers"] = f2
+        "scan_kernels_ms": pk.get("pareto_best", 0.0) + pk.get("pareto_index", 0.0),
+        "frontier_points": int(pr["n_front"]), "scaling": "strong (index slices, two ncclAllReduce)" if world > 1
+        else "1 GPU"}
+    # c5: replay 10M queries x 64 scenarios, Poisson (P) and Gamma(0.05) (G)
+    # traces; N > 1: scenario s on rank owner[s]
+    for kind in ("poisson", "gamma"):
+        cfg = W.config("c5", kind=kind)
+        prof, cl = cfg["prof"], cfg["cluster"]
+        px.load_profiles(prof)
+        alloc = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=2)[0]
+        arr = torch.from_numpy(cfg["arrival_us"]).to(dev)
+        fam = torch.from_numpy(cfg["family"]).to(dev)
+        sc = cfg["scenarios"]
+        S, N = len(sc), len(cfg["arrival_us"])
+        S_own = px.latency_rows(sc)
+        lat = torch.empty((max(S_own, 1), N), dtype=torch.uint32, device=dev)
+        rcall = lambda: px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0],  # noqa: E731
+                                  cl.slo_us, sc, latency=lat)
+        ms, split, res = time_replay(px, barrier, max_over_ranks, stream, 3, rcall)
+        lane = sum(v for k, v in split.items() if k in LANE_KERNELS)
+        wr = sum(v for k, v in split.items() if k in WRITE_KERNELS)
+        alg = N * S_own * 4 + N * 8
+        key = "c5_replay" if kind == "poisson" else "c5_replay_gamma"
+        out[key] = {
+            "trace": f"{N} queries, {kind} arrivals at 3000 QPS" + (" (Gamma shape 0.05, CV 4.47)" if kind == "gamma"
+                                                                    else ""),
+            "queries": N, "scenarios": S, "ms": ms, "query_scenarios_per_s": N * S / (ms / 1e3),
+            "kernel_split_ms": split, "lane_kernels_ms": lane,
+            "roofline": {"kernel": "lane kernels (" + " + ".join(k for k in LANE_KERNELS if k in split) + ")",
+                         "bound": "hbm", "achieved": alg / ((lane + wr) / 1e3) / 1e9, "peak": hbm, "unit": "GB/s",
+                         "frac": alg / ((lane + wr) / 1e3) / 1e9 / hbm, "peak_source": peak_src, "alg_bytes": alg,
+                         "note": "algorithmic bytes = this rank's latency rows (4 B per query-scenario) + one read "
+                                 "of the per-device arrays; time = lane kernels + latency writers"},
+            "violations_first_scenarios": [int(x) for x in res["violations"][:4]],
+            "scaling": "strong (scenarios by proteus_scenario_owner)" if world > 1 else "1 GPU"}
+        if kind == "poisson":
+            e2e_ts = []
+            for _ in range(3):  # host trace in, host latencies out (first call page-locks the output: untimed)
+                barrier()
+                t0 = time.perf_counter()
+                r_h = px.replay(cfg["arrival_us"], cfg["family"], alloc.option, alloc.z, cl.device_type,
+                                cfg["demand"][0], cl.slo_us, sc, latency=True)
+                e2e_ts.append(time.perf_counter() - t0)
+                del r_h
+            out[key]["e2e"] = {"value": N * S / max_over_ranks(statistics.median(e2e_ts[1:])),
+                               "unit": "query-scenarios/s", "h2d_bytes_per_step": int(N * 5),
+                               "d2h_bytes_per_step": int(N * S_own * 4)}
+            # f2: the §6.4 baseline batchers on the same trace and allocation, 64
+            # scenarios each, and the Fig. 6 grid (3 policies x 8 SLOs x caps 8/32/depth)
+            f2 = {}
+            for pol, name in ((1, "nexus"), (2, "aimd")):
+                scp = W.scenarios_64(0, pol)
+                latp = torch.empty((max(px.latency_rows(scp), 1), N), dtype=torch.uint32, device=dev)
+                pms, pk, rp = time_replay(px, barrier, max_over_ranks, stream, 3, lambda: px.replay(
+                    arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, scp, latency=latp))
+                f2[name] = {"ms": pms, "query_scenarios_per_s": N * len(scp) / (pms / 1e3),
+                            "lane_kernel_ms": pk.get("replay_baseline", 0.0)}
+            out["f2_baseline_batchers"] = f2
+        fig6 = W.scenarios_fig6(0)
+        r6 = px.replay(arr, fam, alloc.option, alloc.z, cl.device_type, cfg["demand"][0], cl.slo_us, fig6,
+                       latency=None)
+        grid = {}
+        for (m, c, _, p), v in zip(fig6.tolist(), r6["violations"].tolist()):
+            grid.setdefault(("proteus", "nexus", "aimd")[p], {})[f"slo{m / 1000:g}x_cap{c or 'depth'}"] = v / N
+        out.setdefault("f2_fig6_violation_ratio", {})[kind] = grid
     # f4: closed loop over the c4 hour -- 3600 per-second re-solves (on the
     # previous second's counts) feeding the replay of that hour's queries
     cfg = W.config("f4")
@@ -552,49 +538,34 @@ def extra_metrics(px, dev, rank, world, args, barrier, max_over_ranks, flush, pe
     dem = torch.from_numpy(cfg["demand"]).to(dev)
     t_dev = torch.as_tensor(cl.device_type, dtype=torch.int32, device=dev)
     t_slo = torch.as_tensor(cl.slo_us, dtype=torch.int32, device=dev)
-    scl_all = cfg["scenarios"]
-    llo, lhi = shard_range(len(scl_all), rank, world)
-    scl = scl_all[llo:lhi]
+    scl = cfg["scenarios"]
     Nl = len(cfg["arrival_us"])
-    lat4 = torch.empty((len(scl), Nl), dtype=torch.uint32, device=dev)
+    lat4 = torch.empty((max(px.latency_rows(scl), 1), Nl), dtype=torch.uint32, device=dev)
     alloc = {"option": torch.empty((E, D), dtype=torch.int32, device=dev),
              "z_qps": torch.empty((E, D), dtype=torch.int32, device=dev)}
-    for _ in range(2):
-        px.solve_batch(t_dev, t_slo, dem, mode=2, out=alloc)
-        rl = px.replay_epochs(arr, fam, cfg["epoch_us"], alloc["option"], alloc["z_qps"], t_dev, dem, t_slo, scl,
-                              latency=lat4)
-    px.set_timing(True)
-    ts, kts = [], []
-    for _ in range(3):
+
+    def f4_call():
         flush.zero_()
-        barrier()
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record(stream)
         px.solve_batch(t_dev, t_slo, dem, mode=2, out=alloc)
         k1 = px.kernel_times()
-        rl = px.replay_epochs(arr, fam, cfg["epoch_us"], alloc["option"], alloc["z_qps"], t_dev, dem, t_slo, scl,
-                              latency=lat4)
-        b.record(stream)
-        barrier()
-        ts.append(a.elapsed_time(b))
-        kts.append(k1 + px.kernel_times())
-    px.set_timing(False)
-    lms = max_over_ranks(statistics.median(ts))
-    ksplit = {}
-    for kt in kts:
-        for n_, v in kt:
-            ksplit.setdefault(n_, []).append(v)
-    ksplit = {k: statistics.median(v) for k, v in ksplit.items()}
+        r = px.replay_epochs(arr, fam, cfg["epoch_us"], alloc["option"], alloc["z_qps"], t_dev, dem, t_slo, scl,
+                             latency=lat4)
+        f4_call.k1 = k1
+        return r
+    lms, ksplit, rl = time_replay(px, barrier, max_over_ranks, stream, 3, f4_call)
+    for k, v in _ksplit([f4_call.k1]).items():
+        ksplit["resolve:" + k] = v
+    sel4 = [i for i, r in enumerate(scl) if r[0] == 2000 and r[1] == 0]
     out["f4_closed_loop"] = {
         "workload": f"c4 hour: {E} one-second epochs, {Nl} queries (Poisson within each second), allocation e "
                     f"solved on epoch e-1's counts, {len(scl)} (SLO x batch cap) scenarios",
-        "epochs": E, "queries": Nl, "scenarios": len(scl_all), "ms": lms,
-        "query_scenarios_per_s": Nl * len(scl_all) / (lms / 1e3), "kernel_ms": ksplit,
-        "violation_ratio_slo2x_depth": (float(rl["violations"][sel4[0]]) / Nl) if (sel4 := [
-            i for i, r in enumerate(scl) if r[0] == 2000 and r[1] == 0]) else None,
-        "scaling": "strong (scenarios split by rank; every rank re-solves all epochs)" if world > 1 else "1 GPU"}
+        "epochs": E, "queries": Nl, "scenarios": len(scl), "ms": lms,
+        "query_scenarios_per_s": Nl * len(scl) / (lms / 1e3), "kernel_ms": ksplit,
+        "violation_ratio_slo2x_depth": float(rl["violations"][sel4[0]]) / Nl if sel4 else None,
+        "scaling": ("strong (epochs' re-solves split by rank + ncclAllGather; scenarios by owner)" if world > 1
+                    else "1 GPU")}
+    out["scope"] = scope
     return out
-
 
 if __name__ == "__main__":
     main()

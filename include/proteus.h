@@ -42,13 +42,14 @@
 extern "C" {
 #endif
 
-#define PROTEUS_ABI_VERSION 2
+#define PROTEUS_ABI_VERSION 3
 
 enum {
   PROTEUS_OK = 0,
   PROTEUS_EINVAL = -1,  /* bad argument (null pointer, out-of-range value, no profiles loaded) */
   PROTEUS_ENOMEM = -2,  /* device or host allocation failed */
   PROTEUS_ECUDA = -3,   /* a CUDA call failed */
+  PROTEUS_ENCCL = -4,   /* NCCL missing or an NCCL call failed (proteus_comm_*, distributed calls) */
   PROTEUS_ERANGE = -5,  /* overflow guard: sum of demand >= 2^22, N >= 2^32, unsorted
                            timestamps, or candidate space above max_candidates / 2^63 */
   PROTEUS_EINTERNAL = -6 /* an internal consistency check failed (a bug) */
@@ -326,6 +327,65 @@ int proteus_replay_epochs(proteus_ctx *ctx, const uint32_t *arrival_us, const ui
                           const int32_t *device_type, int32_t D, const int32_t *demand_qps,
                           const int32_t *slo_base_us, const proteus_scenario *sc, int32_t S, uint32_t *latency_us,
                           uint64_t *violations, uint64_t *on_time, uint64_t *acc_sum);
+
+/* -------------------------------------------------------- multi-GPU --
+ * one process per GPU, one context each, joined by an
+ * NCCL communicator the context owns (NCCL is loaded at run time: the copy
+ * already in the process, else libnccl.so.2; PROTEUS_NCCL_LIB overrides).
+ * While the communicator is enabled, calls are DISTRIBUTED: every rank must
+ * make the same call with the same arguments (collectives run on the
+ * context's stream, in call order), and every rank returns the combined
+ * result:
+ *   proteus_solve / proteus_solve_batch, modes 0/1: rank r scans slice r of
+ *     `world` contiguous slices of the index space (shard_rank / shard_world
+ *     must be 0 / 0 or 1), its per-vector winners -- already materialised --
+ *     are exchanged with one ncclAllGather and every rank keeps, per vector,
+ *     the (score desc, index asc) maximum on the device; n_candidates is the
+ *     whole space's.  Identical to the single-GPU answer.
+ *   mode 2 (batched re-solve): demand vectors split by rank (slice r of
+ *     n_vec), one ncclAllGather of the solutions; every rank returns all.
+ *   proteus_pareto: index slices by rank, one ncclAllReduce(MAX) of the best
+ *     accuracy sum per capacity and one ncclAllReduce(MIN) of the lowest
+ *     index per frontier point; every rank returns the whole frontier.
+ *   proteus_replay / proteus_replay_epochs: scenario s is replayed by rank
+ *     owner[s] (proteus_scenario_owner); the per-scenario aggregates are
+ *     combined with one ncclAllReduce(SUM) and are complete on every rank;
+ *     latency_us holds only this rank's scenarios: row k = its k-th owned
+ *     scenario in ascending scenario order ([S_own][N]).
+ * Errors are detected before the first collective from the arguments alone,
+ * so ranks given the same arguments fail together. */
+
+/* 128-byte NCCL unique id (ncclGetUniqueId) into id_out; rank 0 calls it and
+ * the caller broadcasts the bytes (any transport) to the other ranks. */
+#define PROTEUS_COMM_ID_BYTES 128
+int proteus_comm_unique_id(void *id_out);
+/* Create the context's communicator (ncclCommInitRank on the context's GPU;
+ * collective over the `world` ranks) and enable it. */
+int proteus_comm_init(proteus_ctx *ctx, const void *nccl_unique_id, int world, int rank);
+/* Disable (0) / re-enable (1) distributed calls; the communicator is kept. */
+int proteus_comm_enable(proteus_ctx *ctx, int enable);
+/* *world / *rank of the communicator (1 / 0 without one); returns 1 if calls
+ * are distributed, else 0. */
+int proteus_comm_info(const proteus_ctx *ctx, int32_t *world, int32_t *rank);
+/* The rank that replays scenario s in a distributed replay (host only, no
+ * GPU needed): longest-processing-time greedy over a per-scenario lane-cost
+ * model, deterministic in (sc, world).  owner[S] out. */
+int proteus_scenario_owner(const proteus_scenario *sc, int32_t S, int32_t world, int32_t *owner);
+
+/* Combine per-slice results obtained by any transport (e.g. gloo, MPI):
+ * parts[world] are proteus_solve_batch outputs of slices 0..world-1 of the
+ * same search (modes 0/1; every part must have score, index, served, unmet,
+ * accsum, eff_acc_micro, option, z_qps), combined per vector by (score desc,
+ * index asc) on the device into out (as proteus_solve_batch; n_candidates
+ * of out = the sum of the parts').  part_candidates[world]: the parts'
+ * n_candidates.  Pointers may be host or device. */
+int proteus_combine_solutions(proteus_ctx *ctx, int32_t world, int32_t n_vec, int32_t D, const proteus_batch *parts,
+                              const uint64_t *part_candidates, proteus_batch *out);
+/* Frontier of the union of shard frontiers (proteus_pareto with
+ * shard_rank/shard_world, any transport): pts[n] concatenated; out as
+ * proteus_pareto (sorted by capacity, lowest index per point). */
+int proteus_pareto_merge(proteus_ctx *ctx, const proteus_pareto_point *pts, int32_t n, proteus_pareto_point *out,
+                         int32_t max_points, int32_t *n_points);
 
 /* ------------------------------------------------------- instrumentation --
  * proteus_set_timing(ctx, 1) makes later calls record CUDA events around

@@ -71,9 +71,57 @@ def _optimize(T, basis, obj, allowed):
         _pivot(T, basis, best[1], enter)
 
 
-def lp_max(c, A_ub, b_ub, A_eq, b_eq):
+def _presolve_zero_fixed(nx, A_ub, b_ub, A_eq, b_eq):
+    """Generic LP presolve (nothing specific to Eqs. 2-6): with x >= 0, a row
+    whose nonzero coefficients all have one sign and whose right-hand side is
+    0 -- an equality, or a <= row with positive coefficients -- forces every
+    variable in it to 0.  Repeated to a fixed point; returns the set of fixed
+    variables."""
+    fixed = set()
+    changed = True
+    while changed:
+        changed = False
+        rows = [(a, b, True) for a, b in zip(A_eq, b_eq)] + [(a, b, False) for a, b in zip(A_ub, b_ub)]
+        for a, b, eq in rows:
+            if b != 0:
+                continue
+            nz = [j for j in range(nx) if a[j] != 0 and j not in fixed]
+            if not nz:
+                continue
+            pos = all(a[j] > 0 for j in nz)
+            neg = all(a[j] < 0 for j in nz)
+            if pos or (eq and neg):
+                fixed.update(nz)
+                changed = True
+    return fixed
+
+
+def lp_max(c, A_ub, b_ub, A_eq, b_eq, presolve=False):
     """max c.x  s.t. A_ub x <= b_ub, A_eq x = b_eq, x >= 0 (all Fractions).
-    Returns (value, x)."""
+    Returns (value, x).  presolve=True first removes the variables that
+    _presolve_zero_fixed fixes at 0 (and rows left empty, after checking
+    them), then solves the rest with the same simplex."""
+    if presolve:
+        nx = len(c)
+        fixed = _presolve_zero_fixed(nx, A_ub, b_ub, A_eq, b_eq)
+        keep = [j for j in range(nx) if j not in fixed]
+        red = lambda a: [a[j] for j in keep]  # noqa: E731
+        rub, rbu, req, rbe = [], [], [], []
+        for a, b in zip(A_ub, b_ub):
+            if any(a[j] != 0 for j in keep):
+                rub.append(red(a)); rbu.append(b)
+            elif b < 0:
+                raise Infeasible()
+        for a, b in zip(A_eq, b_eq):
+            if any(a[j] != 0 for j in keep):
+                req.append(red(a)); rbe.append(b)
+            elif b != 0:
+                raise Infeasible()
+        val, xr = lp_max(red(c), rub, rbu, req, rbe)
+        x = [Fr(0)] * nx
+        for j, v in zip(keep, xr):
+            x[j] = v
+        return val, x
     nx = len(c)
     rows = []  # (coeffs over x, slack sign or None, rhs)
     for a, b in zip(A_ub, b_ub):
@@ -122,10 +170,13 @@ def lp_max(c, A_ub, b_ub, A_eq, b_eq):
     return val, x[:nx]
 
 
-def literal_assignment_lp(P_tm, acc_m, V, device_type, option, demand):
+def literal_assignment_lp(P_tm, acc_m, V, device_type, option, demand, presolve=False):
     """Solve Eqs. 2-6 (+ reading C1 lexicographic objective) for placement x
     given as option[d] (0 idle, else 1 + variant index m).  Returns
-    (served, accsum, z[d][q]) with Fractions."""
+    (served, accsum, z[d][q]) with Fractions.  presolve=True hands the same
+    constraint rows to lp_max's generic zero-fixing presolve (needed for
+    c2/c3-sized placements: the dense tableau of D*Q*2 columns is otherwise
+    too slow in Fractions)."""
     V = list(map(int, V))
     Q = len(V)
     D = len(option)
@@ -172,13 +223,13 @@ def literal_assignment_lp(P_tm, acc_m, V, device_type, option, demand):
     for d in range(D):
         for q in range(Q):
             c1[Z(d, q)] = 1
-    served, _ = lp_max(c1, A_ub, b_ub, A_eq, b_eq)
+    served, _ = lp_max(c1, A_ub, b_ub, A_eq, b_eq, presolve)
     # stage 2: Eq. 7 at the optimal served
     c2 = [0] * nv
     for d in range(D):
         for q in range(Q):
             c2[Z(d, q)] = sum(int(acc_m[m]) * x[d][m] for m in range(M))
-    acc, sol = lp_max(c2, A_ub, b_ub, A_eq + [c1], b_eq + [served])
+    acc, sol = lp_max(c2, A_ub, b_ub, A_eq + [c1], b_eq + [served], presolve)
     z = [[sol[Z(d, q)] for q in range(Q)] for d in range(D)]
     return served, acc, z
 

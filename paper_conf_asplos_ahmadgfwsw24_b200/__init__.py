@@ -20,7 +20,7 @@ import numpy as np
 from . import _native as N
 from ._native import ProteusError  # noqa: F401
 
-__all__ = ["Proteus", "Solution", "ProteusError", "MODE_FLAT", "MODE_MULTISET", "MODE_FACTORED"]
+__all__ = ["Proteus", "Solution", "ProteusError", "MODE_FLAT", "MODE_MULTISET", "MODE_FACTORED", "scenario_owner"]
 
 MODE_FLAT, MODE_MULTISET, MODE_FACTORED = 0, 1, 2
 UINT64_MAX = (1 << 64) - 1
@@ -46,6 +46,31 @@ def _pinned_u32(shape, keep):
     t = torch.empty(shape, dtype=torch.int32, pin_memory=True)
     keep.append(t)
     return t.numpy().view(np.uint32)
+
+
+def _scenario_rows(scenarios):
+    """int32 rows (slo_mult_milli, batch_cap, routing[, policy]) -> [S][4]
+    (a missing policy column means 0, §5 batching)."""
+    sc = np.asarray(scenarios, dtype=np.int32)
+    sc = sc.reshape(-1, sc.shape[-1])
+    if sc.shape[1] == 3:
+        sc = np.concatenate([sc, np.zeros((sc.shape[0], 1), np.int32)], axis=1)
+    if sc.shape[1] != 4:
+        raise ValueError("scenario rows have 3 or 4 columns")
+    return sc
+
+
+def scenario_owner(scenarios, world: int) -> np.ndarray:
+    """Rank that replays each scenario in a distributed replay
+    (proteus_scenario_owner; host only, no GPU needed)."""
+    sc = _scenario_rows(scenarios)
+    S = sc.shape[0]
+    scs = (N.proteus_scenario * max(S, 1))(*[N.proteus_scenario(*map(int, row)) for row in sc])
+    owner = np.zeros(max(S, 1), np.int32)
+    rc = N.load().proteus_scenario_owner(scs, S, int(world), owner.ctypes.data)
+    if rc != 0:
+        raise ProteusError(rc, "proteus_scenario_owner")
+    return owner[:S]
 
 
 def _is_torch(x):
@@ -217,18 +242,13 @@ class Proteus:
         not produced.  scenarios: int32 rows (slo_mult_milli, batch_cap,
         routing[, policy]); a missing policy column means 0 (§5 batching)."""
         keep = []
-        sc = np.asarray(scenarios, dtype=np.int32)
-        sc = sc.reshape(-1, sc.shape[-1])
-        if sc.shape[1] == 3:
-            sc = np.concatenate([sc, np.zeros((sc.shape[0], 1), np.int32)], axis=1)
-        if sc.shape[1] != 4:
-            raise ValueError("scenario rows have 3 or 4 columns")
+        sc = _scenario_rows(scenarios)
         S = sc.shape[0]
         scs = (N.proteus_scenario * S)(*[N.proteus_scenario(*map(int, row)) for row in sc])
         n = int(arrival_us.shape[0]) if hasattr(arrival_us, "shape") else len(arrival_us)
         lat_np = None
         if latency is True:
-            lat_np = _pinned_u32((S, n), keep)
+            lat_np = _pinned_u32((self.latency_rows(sc), n), keep)
             lat_ptr = lat_np.ctypes.data
         elif latency is None or latency is False:
             lat_ptr = None
@@ -260,17 +280,14 @@ class Proteus:
         [E][D] and demand [E][Q], one allocation per epoch of epoch_us
         (numpy or CUDA tensors).  latency / aggregates_out as replay()."""
         keep = []
-        sc = np.asarray(scenarios, dtype=np.int32)
-        sc = sc.reshape(-1, sc.shape[-1])
-        if sc.shape[1] == 3:
-            sc = np.concatenate([sc, np.zeros((sc.shape[0], 1), np.int32)], axis=1)
+        sc = _scenario_rows(scenarios)
         S = sc.shape[0]
         scs = (N.proteus_scenario * S)(*[N.proteus_scenario(*map(int, row)) for row in sc])
         n = int(arrival_us.shape[0]) if hasattr(arrival_us, "shape") else len(arrival_us)
         E, D = int(option.shape[0]), int(option.shape[1])
         lat_np = None
         if latency is True:
-            lat_np = _pinned_u32((S, n), keep)
+            lat_np = _pinned_u32((self.latency_rows(sc), n), keep)
             lat_ptr = lat_np.ctypes.data
         elif latency is None or latency is False:
             lat_ptr = None
@@ -310,6 +327,82 @@ class Proteus:
         res = self.replay_epochs(arrival_us, family, epoch_us, alloc["option"], alloc["z_qps"], device_type, demand,
                                  slo_us, scenarios, latency=latency)
         return res, alloc
+
+    # ----------------------------------------------------------- multi-GPU --
+    @staticmethod
+    def comm_unique_id() -> bytes:
+        """128-byte NCCL unique id (rank 0; broadcast it to the other ranks)."""
+        buf = C.create_string_buffer(N.COMM_ID_BYTES)
+        rc = N.load().proteus_comm_unique_id(buf)
+        if rc != 0:
+            raise ProteusError(rc, "proteus_comm_unique_id (NCCL unavailable?)")
+        return buf.raw
+
+    def comm_init(self, unique_id: bytes, world: int, rank: int):
+        """Join the context's NCCL communicator (collective over the ranks);
+        later calls are distributed (proteus.h, multi-GPU)."""
+        buf = C.create_string_buffer(bytes(unique_id), N.COMM_ID_BYTES)
+        self._check(self._lib.proteus_comm_init(self._h, buf, int(world), int(rank)))
+
+    def comm_enable(self, on: bool = True):
+        self._check(self._lib.proteus_comm_enable(self._h, 1 if on else 0))
+
+    def comm_info(self):
+        """(world, rank, distributed calls enabled)."""
+        w, r = C.c_int32(), C.c_int32()
+        on = self._lib.proteus_comm_info(self._h, C.byref(w), C.byref(r))
+        return w.value, r.value, bool(on == 1)
+
+    def latency_rows(self, scenarios) -> int:
+        """Rows of a replay's latency output: S, or in a distributed replay
+        the number of scenarios this rank owns (in ascending order)."""
+        sc = _scenario_rows(scenarios)
+        world, rank, on = self.comm_info()
+        if not on or world == 1:
+            return sc.shape[0]
+        return int(np.sum(scenario_owner(sc, world) == rank))
+
+    def combine_solutions(self, parts, part_candidates, D):
+        """proteus_combine_solutions: per-slice solve_batch outputs (dicts of
+        arrays with every field) -> the batch's optima, combined on the GPU."""
+        keep = []
+        world = len(parts)
+        n_vec = len(parts[0]["score"])
+        types = {"score": np.uint64, "index": np.uint64, "served": np.int64, "unmet": np.int64,
+                 "accsum": np.int64, "eff_acc_micro": np.int32, "option": np.int32, "z_qps": np.int32}
+        arr = (N.proteus_batch * world)()
+        for r, p in enumerate(parts):
+            for k, t in types.items():
+                setattr(arr[r], k, _arg(p[k], t, keep))
+        out = {"score": np.empty(n_vec, np.uint64), "index": np.empty(n_vec, np.uint64),
+               "served": np.empty(n_vec, np.int64), "unmet": np.empty(n_vec, np.int64),
+               "accsum": np.empty(n_vec, np.int64), "eff_acc_micro": np.empty(n_vec, np.int32),
+               "option": np.empty((n_vec, D), np.int32), "z_qps": np.empty((n_vec, D), np.int32)}
+        b = N.proteus_batch()
+        for k, x in out.items():
+            setattr(b, k, _arg(x, types[k], keep))
+        pc = _arg(np.asarray(part_candidates, np.uint64), np.uint64, keep)
+        self._check(self._lib.proteus_combine_solutions(self._h, world, n_vec, int(D), arr, pc, C.byref(b)))
+        return out, int(b.n_candidates)
+
+    def pareto_merge(self, parts, max_points=65536):
+        """proteus_pareto_merge: frontier of the union of shard frontiers
+        (dicts from pareto(..., shard_rank, shard_world))."""
+        cap = np.concatenate([np.asarray(p["cap"], np.int64) for p in parts])
+        acs = np.concatenate([np.asarray(p["accsum"], np.int64) for p in parts])
+        idx = np.concatenate([np.asarray(p["index"], np.uint64) for p in parts])
+        n = len(cap)
+        pts = (N.proteus_pareto_point * max(1, n))()
+        for i in range(n):
+            pts[i] = N.proteus_pareto_point(int(cap[i]), int(acs[i]), int(idx[i]))
+        out = (N.proteus_pareto_point * max(1, max_points))()
+        npts = C.c_int32()
+        self._check(self._lib.proteus_pareto_merge(self._h, pts, n, out, int(max_points), C.byref(npts)))
+        k = min(npts.value, max_points)
+        return dict(cap=np.array([out[i].capacity for i in range(k)], np.int64),
+                    accsum=np.array([out[i].accsum for i in range(k)], np.int64),
+                    index=np.array([out[i].index for i in range(k)], np.uint64),
+                    n_configs=sum(int(p["n_configs"]) for p in parts), n_front=npts.value)
 
     # ----------------------------------------------------- instrumentation --
     def set_timing(self, on=True):

@@ -14,6 +14,7 @@ PROTEUS_OK = 0
 PROTEUS_EINVAL = -1
 PROTEUS_ENOMEM = -2
 PROTEUS_ECUDA = -3
+PROTEUS_ENCCL = -4
 PROTEUS_ERANGE = -5
 PROTEUS_EINTERNAL = -6
 PROTEUS_SOLVE_GENERIC = 1
@@ -22,7 +23,11 @@ EXPORTED = (
     "proteus_abi_version", "proteus_create", "proteus_destroy", "proteus_set_stream", "proteus_last_error",
     "proteus_load_profiles", "proteus_solve", "proteus_solve_batch", "proteus_materialize", "proteus_candidate_count",
     "proteus_pareto", "proteus_replay", "proteus_replay_epochs", "proteus_set_timing", "proteus_kernel_times", "proteus_launch_count",
+    "proteus_comm_unique_id", "proteus_comm_init", "proteus_comm_enable", "proteus_comm_info", "proteus_scenario_owner",
+    "proteus_combine_solutions", "proteus_pareto_merge",
 )
+ABI_VERSION = 3
+COMM_ID_BYTES = 128
 
 
 class proteus_profiles(C.Structure):
@@ -103,7 +108,15 @@ def load(path: str = LIB_PATH):
     L.proteus_kernel_times.argtypes = [vp, C.POINTER(C.c_char_p), C.POINTER(C.c_float), C.c_int]
     L.proteus_launch_count.argtypes = [vp]
     L.proteus_launch_count.restype = u64
-    if L.proteus_abi_version() != 2:
+    L.proteus_comm_unique_id.argtypes = [vp]
+    L.proteus_comm_init.argtypes = [vp, vp, C.c_int, C.c_int]
+    L.proteus_comm_enable.argtypes = [vp, C.c_int]
+    L.proteus_comm_info.argtypes = [vp, C.POINTER(i32), C.POINTER(i32)]
+    L.proteus_scenario_owner.argtypes = [C.POINTER(proteus_scenario), i32, i32, vp]
+    L.proteus_combine_solutions.argtypes = [vp, i32, i32, i32, C.POINTER(proteus_batch), vp, C.POINTER(proteus_batch)]
+    L.proteus_pareto_merge.argtypes = [vp, C.POINTER(proteus_pareto_point), i32, C.POINTER(proteus_pareto_point),
+                                       i32, C.POINTER(i32)]
+    if L.proteus_abi_version() != ABI_VERSION:
         raise ImportError("libproteus ABI version mismatch")
     _lib = L
     return L

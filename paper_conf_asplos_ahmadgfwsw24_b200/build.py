@@ -28,6 +28,19 @@ NVCC_FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2", "-I",
               "--expt-relaxed-constexpr", "-Xptxas", "-warn-spills"]
 
 
+def _nccl_include() -> list:
+    """nccl.h for comm.cu (types and enums only: libnccl is dlopen'ed at run
+    time): the NCCL that ships with torch, else the system one."""
+    try:
+        import nvidia.nccl as nn
+        inc = os.path.join(list(nn.__path__)[0], "include")
+        if os.path.exists(os.path.join(inc, "nccl.h")):
+            return ["-I", inc]
+    except ImportError:
+        pass
+    return []
+
+
 def _nvcc() -> str:
     for c in (os.environ.get("NVCC"), "/usr/local/cuda/bin/nvcc", shutil.which("nvcc")):
         if c and os.path.exists(c):
@@ -44,7 +57,7 @@ def _compile(src: str, verbose: bool) -> str:
     obj = os.path.join(OBJ, os.path.basename(src) + ".o")
     if os.path.exists(obj) and os.path.getmtime(obj) >= max(os.path.getmtime(src), _newest_header()):
         return obj
-    cmd = [_nvcc(), *ARCH, *NVCC_FLAGS, *DEFS, "-c", src, "-o", obj + ".tmp"]
+    cmd = [_nvcc(), *ARCH, *NVCC_FLAGS, *_nccl_include(), *DEFS, "-c", src, "-o", obj + ".tmp"]
     if verbose:
         cmd += ["-Xptxas", "-v"]
     r = subprocess.run(cmd, capture_output=True, text=True)

@@ -153,6 +153,7 @@ void proteus_destroy(proteus_ctx *ctx) {
   for (int32_t *p : {ctx->d_lat, ctx->d_acc, ctx->d_fam, ctx->d_off, ctx->d_V}) if (p) cudaFree(p);
   for (auto e : ctx->tev) cudaEventDestroy(e);
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+  px_comm_destroy(ctx);
   delete ctx;
 }
 
@@ -377,11 +378,21 @@ static bool families_sorted(const proteus_ctx *ctx) {
 
 int px_flat_template_vm(int Q, int maxV);  // solve_enum.cu: VM of the specialised kernel, 0 if none
 
-static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_solution *out, bool mat_only,
+static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a_in, proteus_solution *out, bool mat_only,
                         int32_t mat_vec, uint64_t mat_index, proteus_batch *bout = nullptr) {
   SolveInputs in;
-  int rc = validate_solve(ctx, a, in);
+  int rc = validate_solve(ctx, a_in, in);
   if (rc) return rc;
+  // distributed call (comm.cu): modes 0/1 scan the communicator rank's slice,
+  // mode 2 solves the rank's slice of the demand vectors
+  const bool dist = px_comm_active(ctx) && !mat_only;
+  proteus_solve_args a_loc = *a_in;
+  const proteus_solve_args *a = &a_loc;
+  if (dist && a_in->mode != 2) {
+    if (a_in->shard_world > 1) return px_fail(ctx, PROTEUS_EINVAL, "explicit shards in a distributed call");
+    a_loc.shard_rank = ctx->comm_rank;
+    a_loc.shard_world = ctx->comm_world;
+  }
   if (!out && !bout) return px_fail(ctx, PROTEUS_EINVAL, "null out");
   if (mat_only && (a->mode == 2 || mat_vec < 0 || mat_vec >= a->n_vec))
     return px_fail(ctx, PROTEUS_EINVAL, "materialize: mode %d vec %d", a->mode, mat_vec);
@@ -415,7 +426,7 @@ static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_s
   key.insert(key.end(), in.slo.begin(), in.slo.end());
   if (!ctx->tab_valid || key != ctx->tab_key) {
     ctx->tab_valid = false;
-    if ((rc = px_prepare_tables(ctx, a->D, d_dev, in.d_slo, VM, ctx->tab))) return rc;
+    if ((rc = px_prepare_tables(ctx, a->D, d_dev, in.d_slo, VM, ctx->tab, true))) return rc;
     // the launch parameters of the scoring kernels carry the capacity table
     ctx->tab_P.resize((size_t)ctx->T * ctx->M);
     ctx->tab_slot_code.resize((size_t)ctx->Q * VM);
@@ -432,7 +443,24 @@ static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_s
   int nout = mat_only ? 1 : a->n_vec;
   SolRec *d_sol = (SolRec *)px_buf(ctx, B_SOL, sizeof(SolRec) * nout);
   if (!d_sol) return px_fail(ctx, PROTEUS_ENOMEM, "solution buffer");
-  if (a->mode == 2) {
+  if (a->mode == 2 && dist) {
+    // vectors [lo, hi) on this rank, padded to `stride` records for the all-gather
+    const int W = ctx->comm_world, R = ctx->comm_rank, n = a->n_vec;
+    const int lo = (int)((int64_t)n * R / W), hi = (int)((int64_t)n * (R + 1) / W);
+    const int stride = (n + W - 1) / W;
+    SolRec *d_gat = (SolRec *)px_buf(ctx, B_C_GATHER, sizeof(SolRec) * (size_t)stride * (W + 1));
+    if (!d_gat) return px_fail(ctx, PROTEUS_ENOMEM, "gather buffer");
+    SolRec *d_mine = d_gat + (size_t)stride * W;
+    if (hi > lo) {
+      proteus_solve_args part = *a;
+      part.n_vec = hi - lo;
+      rc = px_solve_factored(ctx, &part, in.dev_type.data(), d_dev, d_dem + (size_t)lo * ctx->Q, VM, tab, h_P,
+                             d_mine);
+      if (rc) return rc;
+    }
+    if ((rc = px_comm_allgather(ctx, d_mine, d_gat, sizeof(SolRec) * (size_t)stride))) return rc;
+    rc = px_gather_vectors(ctx, d_gat, W, n, stride, d_sol);
+  } else if (a->mode == 2) {
     rc = px_solve_factored(ctx, a, in.dev_type.data(), d_dev, d_dem, VM, tab, h_P, d_sol);
   } else if (mat_only) {
     rc = px_solve_enum(ctx, a, in.dev_type.data(), in.slo.data(), in.demand.data(), VM, tab, h_P, h_slot_code,
@@ -440,6 +468,13 @@ static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_s
   } else {
     rc = px_solve_enum(ctx, a, in.dev_type.data(), in.slo.data(), in.demand.data(), VM, tab, h_P, h_slot_code,
                        d_sol, 0, a->n_vec, false, 0, use_flat, d_dem);
+    if (!rc && dist) {  // every rank's materialised winners -> the (score desc, index asc) maximum per vector
+      const int W = ctx->comm_world;
+      SolRec *d_gat = (SolRec *)px_buf(ctx, B_C_GATHER, sizeof(SolRec) * (size_t)nout * W);
+      if (!d_gat) return px_fail(ctx, PROTEUS_ENOMEM, "gather buffer");
+      if ((rc = px_comm_allgather(ctx, d_sol, d_gat, sizeof(SolRec) * (size_t)nout))) return rc;
+      rc = px_pick_solrec(ctx, d_gat, W, nout, d_sol);
+    }
   }
   if (rc) return rc;
   if (bout) return batch_out(ctx, a, d_sol, nout, bout);
@@ -458,15 +493,19 @@ static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a, proteus_s
     o.accsum = h[i].accsum;
     o.eff_acc_micro = h[i].eff;
     o.n_candidates = h[i].n_candidates;
+    // device outputs: copied on the stream from the device record (no host round trip), one sync below
     if (o.option) {
-      if (px_is_device_ptr(o.option)) PX_CUDA(ctx, cudaMemcpy(o.option, h[i].option, a->D * 4, cudaMemcpyHostToDevice));
+      if (px_is_device_ptr(o.option))
+        PX_CUDA(ctx, cudaMemcpyAsync(o.option, d_sol[i].option, a->D * 4, cudaMemcpyDeviceToDevice, ctx->stream));
       else memcpy(o.option, h[i].option, a->D * 4);
     }
     if (o.z_qps) {
-      if (px_is_device_ptr(o.z_qps)) PX_CUDA(ctx, cudaMemcpy(o.z_qps, h[i].z, a->D * 4, cudaMemcpyHostToDevice));
+      if (px_is_device_ptr(o.z_qps))
+        PX_CUDA(ctx, cudaMemcpyAsync(o.z_qps, d_sol[i].z, a->D * 4, cudaMemcpyDeviceToDevice, ctx->stream));
       else memcpy(o.z_qps, h[i].z, a->D * 4);
     }
   }
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
   return PROTEUS_OK;
 }
 
@@ -496,6 +535,82 @@ int proteus_candidate_count(proteus_ctx *ctx, const proteus_solve_args *a, uint6
   bool ovf = false;
   *count = px_count_candidates(a->mode, a->D, dev.data(), ctx->T, 1 + ctx->M, &ovf);
   return ovf ? px_fail(ctx, PROTEUS_ERANGE, "candidate space exceeds 2^64") : PROTEUS_OK;
+}
+
+// ------------------------------------------------------------ combine -----
+int proteus_combine_solutions(proteus_ctx *ctx, int32_t world, int32_t n_vec, int32_t D, const proteus_batch *parts,
+                              const uint64_t *part_candidates, proteus_batch *out) {
+  if (!ctx) return PROTEUS_EINVAL;
+  ctx->err.clear();
+  if (world < 1 || n_vec < 1 || D < 1 || D > PX_MAXD || !parts || !out)
+    return px_fail(ctx, PROTEUS_EINVAL, "combine: world %d n_vec %d D %d", world, n_vec, D);
+  PX_CUDA(ctx, cudaSetDevice(ctx->device));
+  timing_reset(ctx);
+  // marshal the parts into the record layout the NCCL path gathers (host side: layout only)
+  std::vector<SolRec> recs((size_t)world * n_vec);
+  memset(recs.data(), 0, recs.size() * sizeof(SolRec));
+  for (int r = 0; r < world; r++) {
+    const proteus_batch &p = parts[r];
+    if (!p.score || !p.index || !p.served || !p.unmet || !p.accsum || !p.eff_acc_micro || !p.option || !p.z_qps)
+      return px_fail(ctx, PROTEUS_EINVAL, "combine: part %d lacks a field", r);
+    std::vector<uint64_t> sc, ix;
+    std::vector<int64_t> sv, um, ac;
+    std::vector<int32_t> ef, op, zz;
+    int rc;
+    if ((rc = to_host(ctx, p.score, n_vec, sc)) || (rc = to_host(ctx, p.index, n_vec, ix)) ||
+        (rc = to_host(ctx, p.served, n_vec, sv)) || (rc = to_host(ctx, p.unmet, n_vec, um)) ||
+        (rc = to_host(ctx, p.accsum, n_vec, ac)) || (rc = to_host(ctx, p.eff_acc_micro, n_vec, ef)) ||
+        (rc = to_host(ctx, p.option, (size_t)n_vec * D, op)) || (rc = to_host(ctx, p.z_qps, (size_t)n_vec * D, zz)))
+      return rc;
+    for (int v = 0; v < n_vec; v++) {
+      SolRec &x = recs[(size_t)r * n_vec + v];
+      x.score = sc[v]; x.index = ix[v]; x.served = sv[v]; x.unmet = um[v]; x.accsum = ac[v]; x.eff = ef[v];
+      x.n_candidates = part_candidates ? part_candidates[r] : 0;
+      memcpy(x.option, &op[(size_t)v * D], D * 4);
+      memcpy(x.z, &zz[(size_t)v * D], D * 4);
+    }
+  }
+  SolRec *d_gat = (SolRec *)px_buf(ctx, B_C_GATHER, sizeof(SolRec) * recs.size());
+  SolRec *d_sol = (SolRec *)px_buf(ctx, B_SOL, sizeof(SolRec) * (size_t)n_vec);
+  if (!d_gat || !d_sol) return px_fail(ctx, PROTEUS_ENOMEM, "combine buffers");
+  PX_CUDA(ctx, cudaMemcpyAsync(d_gat, recs.data(), sizeof(SolRec) * recs.size(), cudaMemcpyHostToDevice, ctx->stream));
+  int rc = px_pick_solrec(ctx, d_gat, world, n_vec, d_sol);
+  if (rc) return rc;
+  proteus_solve_args a;
+  memset(&a, 0, sizeof a);
+  a.D = D;
+  return batch_out(ctx, &a, d_sol, n_vec, out);
+}
+
+int proteus_pareto_merge(proteus_ctx *ctx, const proteus_pareto_point *pts, int32_t n, proteus_pareto_point *out,
+                         int32_t max_points, int32_t *n_points) {
+  if (!ctx) return PROTEUS_EINVAL;
+  ctx->err.clear();
+  if (n < 0 || (n > 0 && !pts) || !n_points || max_points < 0 || (max_points > 0 && !out))
+    return px_fail(ctx, PROTEUS_EINVAL, "pareto_merge arguments");
+  PX_CUDA(ctx, cudaSetDevice(ctx->device));
+  timing_reset(ctx);
+  int rc;
+  const proteus_pareto_point *d_pts = to_device(ctx, pts, (size_t)n, B_IN0, &rc);
+  if (rc) return rc;
+  proteus_pareto_point *d_out = (proteus_pareto_point *)px_buf(ctx, B_C_PTS, sizeof(proteus_pareto_point) * (size_t)(n + 1) + 16);
+  if (!d_out) return px_fail(ctx, PROTEUS_ENOMEM, "merge output");
+  int32_t *d_n = (int32_t *)(d_out + n + 1);
+  if ((rc = px_pareto_merge(ctx, d_pts, n, d_out, d_n))) return rc;
+  int32_t nf = 0;
+  PX_CUDA(ctx, cudaMemcpyAsync(&nf, d_n, 4, cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  const int k = nf < max_points ? nf : max_points;
+  if (k > 0) {
+    if (px_is_device_ptr(out))
+      PX_CUDA(ctx, cudaMemcpyAsync(out, d_out, sizeof(proteus_pareto_point) * k, cudaMemcpyDeviceToDevice, ctx->stream));
+    else
+      PX_CUDA(ctx, cudaMemcpyAsync(out, d_out, sizeof(proteus_pareto_point) * k, cudaMemcpyDeviceToHost, ctx->stream));
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  }
+  if ((rc = timing_collect(ctx))) return rc;
+  *n_points = nf;
+  return PROTEUS_OK;
 }
 
 // ------------------------------------------------------------- pareto -----
@@ -538,6 +653,68 @@ int proteus_pareto(proteus_ctx *ctx, const proteus_pareto_args *a, proteus_paret
 }
 
 // ------------------------------------------------------------- replay -----
+
+// Outputs of a replay: per-scenario aggregates [3][S] (+ the unsorted flag)
+// from d_agg -- straight device-to-device into device outputs, one copy per
+// array -- and the latency rows [S_run][N] into a host buffer.
+static int replay_outputs(proteus_ctx *ctx, const uint64_t *d_agg, int S, int64_t N, int S_run, uint32_t *latency_us,
+                          bool lat_dev, const uint32_t *d_lat, uint64_t *violations, uint64_t *on_time,
+                          uint64_t *acc_sum) {
+  uint64_t *outs[3] = {violations, on_time, acc_sum};
+  for (int k = 0; k < 3; k++)
+    if (outs[k] && px_is_device_ptr(outs[k]))
+      PX_CUDA(ctx, cudaMemcpyAsync(outs[k], d_agg + (size_t)k * S, (size_t)S * 8, cudaMemcpyDeviceToDevice,
+                                   ctx->stream));
+  std::vector<uint64_t> agg((size_t)3 * S + 1);
+  PX_CUDA(ctx, cudaMemcpyAsync(agg.data(), d_agg, ((size_t)3 * S + 1) * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  if (latency_us && !lat_dev && S_run > 0)
+    PX_CUDA(ctx, cudaMemcpyAsync(latency_us, d_lat, (size_t)S_run * N * 4, cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  int rc;
+  if ((rc = timing_collect(ctx))) return rc;
+  if (agg[3 * (size_t)S] != 0) return px_fail(ctx, PROTEUS_ERANGE, "arrival timestamps not sorted");
+  for (int k = 0; k < 3; k++)
+    if (outs[k] && !px_is_device_ptr(outs[k])) memcpy(outs[k], &agg[(size_t)k * S], (size_t)S * 8);
+  return PROTEUS_OK;
+}
+// Distributed replay (comm.cu): this rank's scenarios only; their aggregates
+// [3][S_own] (+ the unsorted flag) are scattered into a zero [3][S] (+ flag)
+// vector that one all-reduce(SUM) completes on every rank.
+__global__ void k_agg_scatter(const uint64_t *__restrict__ loc, int S_loc, const int32_t *__restrict__ map,
+                              uint64_t *full, int S) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < 3 * S_loc) full[(size_t)(i / S_loc) * S + map[i % S_loc]] = loc[i];
+  if (i == 0) full[(size_t)3 * S] = loc[(size_t)3 * S_loc];
+}
+
+struct ReplayShard {
+  bool dist = false;
+  std::vector<proteus_scenario> sc;  // this rank's scenarios (ascending scenario index)
+  std::vector<int32_t> map;          // their scenario indices
+};
+
+static void replay_shard(proteus_ctx *ctx, const std::vector<proteus_scenario> &scv, ReplayShard &sh) {
+  sh.dist = px_comm_active(ctx);
+  if (!sh.dist) return;
+  std::vector<int32_t> owner(scv.size());
+  px_scenario_owner(scv.data(), (int)scv.size(), ctx->comm_world, owner.data());
+  for (size_t s = 0; s < scv.size(); s++)
+    if (owner[s] == ctx->comm_rank) { sh.sc.push_back(scv[s]); sh.map.push_back((int32_t)s); }
+}
+
+// combine a distributed replay's aggregates into d_full [3][S] + flag
+static int replay_combine(proteus_ctx *ctx, const ReplayShard &sh, const uint64_t *d_loc, int S, uint64_t *d_full) {
+  const int S_loc = (int)sh.map.size();
+  PX_CUDA(ctx, cudaMemsetAsync(d_full, 0, ((size_t)3 * S + 1) * 8, ctx->stream));
+  int32_t *d_map = (int32_t *)px_buf(ctx, B_C_PTS, (size_t)S_loc * 4 + 16);
+  if (!d_map) return px_fail(ctx, PROTEUS_ENOMEM, "scenario map");
+  if (S_loc) {
+    PX_CUDA(ctx, cudaMemcpyAsync(d_map, sh.map.data(), (size_t)S_loc * 4, cudaMemcpyHostToDevice, ctx->stream));
+    PX_LAUNCH(ctx, "agg_scatter", k_agg_scatter, (3 * S_loc + 255) / 256, 256, 0, d_loc, S_loc, d_map, d_full, S);
+  }
+  return px_comm_allreduce_u64(ctx, d_full, (size_t)3 * S + 1, PX_RED_SUM);
+}
+
 int proteus_replay(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *family, int64_t N,
                    const int32_t *option, const int32_t *z_qps, const int32_t *device_type, int32_t D,
                    const int32_t *demand_qps, const int32_t *slo_base_us, const proteus_scenario *sc, int32_t S,
@@ -582,39 +759,32 @@ int proteus_replay(proteus_ctx *ctx, const uint32_t *arrival_us, const uint8_t *
   if (rc) return rc;
   const uint8_t *d_fam = to_device(ctx, family, (size_t)N, B_IN1, &rc);
   if (rc) return rc;
+  ReplayShard sh;
+  replay_shard(ctx, scv, sh);
+  const int S_run = sh.dist ? (int)sh.sc.size() : S;  // scenarios replayed here
+  const proteus_scenario *sc_run = sh.dist ? sh.sc.data() : scv.data();
   uint32_t *d_lat = nullptr;
   bool lat_dev = latency_us && px_is_device_ptr(latency_us);
   if (latency_us) {
-    d_lat = lat_dev ? latency_us : (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S * N * 4);
+    d_lat = lat_dev ? latency_us : (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S_run * N * 4);
     if (!d_lat) return px_fail(ctx, PROTEUS_ENOMEM, "latency buffer");
   }
-  uint64_t *d_agg = (uint64_t *)px_buf(ctx, B_R_AGG, (size_t)3 * S * 8 + 8);
-  if (!d_agg) return px_fail(ctx, PROTEUS_ENOMEM, "aggregate buffer");
-  rc = px_replay(ctx, d_arr, d_fam, N, opt.data(), z.data(), dev.data(), D, dem.data(), slo.data(), scv.data(), S,
-                 d_lat, d_agg);
-  if (rc) return rc;
-  std::vector<uint64_t> agg((size_t)3 * S + 1);
-  PX_CUDA(ctx, cudaMemcpyAsync(agg.data(), d_agg, ((size_t)3 * S + 1) * 8, cudaMemcpyDeviceToHost, ctx->stream));
-  if (latency_us && !lat_dev)
-    PX_CUDA(ctx, cudaMemcpyAsync(latency_us, d_lat, (size_t)S * N * 4, cudaMemcpyDeviceToHost, ctx->stream));
-  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
-  if ((rc = timing_collect(ctx))) return rc;
-  if (agg[3 * S] != 0) return px_fail(ctx, PROTEUS_ERANGE, "arrival timestamps not sorted");
-  for (int s = 0; s < S; s++) {
-    if (violations) {
-      if (px_is_device_ptr(violations)) PX_CUDA(ctx, cudaMemcpy(violations + s, &agg[s], 8, cudaMemcpyHostToDevice));
-      else violations[s] = agg[s];
-    }
-    if (on_time) {
-      if (px_is_device_ptr(on_time)) PX_CUDA(ctx, cudaMemcpy(on_time + s, &agg[S + s], 8, cudaMemcpyHostToDevice));
-      else on_time[s] = agg[S + s];
-    }
-    if (acc_sum) {
-      if (px_is_device_ptr(acc_sum)) PX_CUDA(ctx, cudaMemcpy(acc_sum + s, &agg[2 * S + s], 8, cudaMemcpyHostToDevice));
-      else acc_sum[s] = agg[2 * S + s];
-    }
+  // [3][S_run] + flag, then (distributed) the combined [3][S] + flag
+  uint64_t *d_agg0 = (uint64_t *)px_buf(ctx, B_R_AGG, ((size_t)3 * S_run + 1 + (sh.dist ? 3 * (size_t)S + 1 : 0)) * 8);
+  if (!d_agg0) return px_fail(ctx, PROTEUS_ENOMEM, "aggregate buffer");
+  uint64_t *d_agg = d_agg0;
+  if (S_run > 0) {
+    rc = px_replay(ctx, d_arr, d_fam, N, opt.data(), z.data(), dev.data(), D, dem.data(), slo.data(), sc_run, S_run,
+                   d_lat, d_agg);
+    if (rc) return rc;
+  } else {
+    PX_CUDA(ctx, cudaMemsetAsync(d_agg, 0, 8, ctx->stream));
   }
-  return PROTEUS_OK;
+  if (sh.dist) {
+    d_agg = d_agg0 + 3 * (size_t)S_run + 1;
+    if ((rc = replay_combine(ctx, sh, d_agg0, S, d_agg))) return rc;
+  }
+  return replay_outputs(ctx, d_agg, S, N, S_run, latency_us, lat_dev, d_lat, violations, on_time, acc_sum);
 }
 
 // -------------------------------------------------------- closed loop -----
@@ -671,32 +841,32 @@ int proteus_replay_epochs(proteus_ctx *ctx, const uint32_t *arrival_us, const ui
   if (rc) return rc;
   const uint8_t *d_fam = to_device(ctx, family, (size_t)N, B_IN1, &rc);
   if (rc) return rc;
+  ReplayShard sh;
+  replay_shard(ctx, scv, sh);
+  const int S_run = sh.dist ? (int)sh.sc.size() : S;  // scenarios replayed here
+  const proteus_scenario *sc_run = sh.dist ? sh.sc.data() : scv.data();
   uint32_t *d_lat = nullptr;
   bool lat_dev = latency_us && px_is_device_ptr(latency_us);
   if (latency_us) {
-    d_lat = lat_dev ? latency_us : (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S * N * 4);
+    d_lat = lat_dev ? latency_us : (uint32_t *)px_buf(ctx, B_R_LAT, (size_t)S_run * N * 4);
     if (!d_lat) return px_fail(ctx, PROTEUS_ENOMEM, "latency buffer");
   }
-  uint64_t *d_agg = (uint64_t *)px_buf(ctx, B_R_AGG, (size_t)3 * S * 8 + 8);
-  if (!d_agg) return px_fail(ctx, PROTEUS_ENOMEM, "aggregate buffer");
-  rc = px_replay_epochs(ctx, d_arr, d_fam, N, E, epoch_us, opt.data(), z.data(), dev.data(), D, dem.data(),
-                        slo.data(), scv.data(), S, d_lat, d_agg);
-  if (rc) return rc;
-  std::vector<uint64_t> agg((size_t)3 * S + 1);
-  PX_CUDA(ctx, cudaMemcpyAsync(agg.data(), d_agg, ((size_t)3 * S + 1) * 8, cudaMemcpyDeviceToHost, ctx->stream));
-  if (latency_us && !lat_dev)
-    PX_CUDA(ctx, cudaMemcpyAsync(latency_us, d_lat, (size_t)S * N * 4, cudaMemcpyDeviceToHost, ctx->stream));
-  PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
-  if ((rc = timing_collect(ctx))) return rc;
-  uint64_t *outs[3] = {violations, on_time, acc_sum};
-  for (int k = 0; k < 3; k++) {
-    if (!outs[k]) continue;
-    if (px_is_device_ptr(outs[k]))
-      PX_CUDA(ctx, cudaMemcpy(outs[k], &agg[(size_t)k * S], (size_t)S * 8, cudaMemcpyHostToDevice));
-    else
-      memcpy(outs[k], &agg[(size_t)k * S], (size_t)S * 8);
+  // [3][S_run] + flag, then (distributed) the combined [3][S] + flag
+  uint64_t *d_agg0 = (uint64_t *)px_buf(ctx, B_R_AGG, ((size_t)3 * S_run + 1 + (sh.dist ? 3 * (size_t)S + 1 : 0)) * 8);
+  if (!d_agg0) return px_fail(ctx, PROTEUS_ENOMEM, "aggregate buffer");
+  uint64_t *d_agg = d_agg0;
+  if (S_run > 0) {
+    rc = px_replay_epochs(ctx, d_arr, d_fam, N, E, epoch_us, opt.data(), z.data(), dev.data(), D, dem.data(),
+                          slo.data(), sc_run, S_run, d_lat, d_agg);
+    if (rc) return rc;
+  } else {
+    PX_CUDA(ctx, cudaMemsetAsync(d_agg, 0, 8, ctx->stream));
   }
-  return PROTEUS_OK;
+  if (sh.dist) {
+    d_agg = d_agg0 + 3 * (size_t)S_run + 1;
+    if ((rc = replay_combine(ctx, sh, d_agg0, S, d_agg))) return rc;
+  }
+  return replay_outputs(ctx, d_agg, S, N, S_run, latency_us, lat_dev, d_lat, violations, on_time, acc_sum);
 }
 
 }  // extern "C"

@@ -17,6 +17,7 @@
 #define PX_MAXV 16
 #define PX_MAXM 255
 #define PX_MAXB 1024
+#define PX_PCLAMP (1 << 22)  // solve-path capacity clamp (prepare.cu): > any demand
 
 // ------------------------------------------------------------ score ----
 // Packed objective (reading C1): served in the high 22 bits, accuracy sum in
@@ -105,13 +106,19 @@ struct proteus_ctx {
   // cached count-vector lists of the factored search
   void *fact_lists_buf = nullptr;
   std::vector<int32_t> fact_lists_key;
+  // flat kernel occupancy per (instantiation, shared-memory size) on this device
+  std::vector<std::pair<std::pair<const void *, size_t>, int>> occ_cache;
+  // NCCL communicator (comm.cu): calls shard over it while comm_on
+  void *comm = nullptr;
+  int comm_world = 1, comm_rank = 0;
+  bool comm_on = false;
 };
 
 // scratch buffer ids
 enum {
   B_TABLES = 0, B_BEST, B_SOL, B_IN0, B_IN1, B_IN2, B_IN3, B_FACT0, B_FACT1, B_FACT2, B_FACT3,
   B_R_PAT, B_R_TGT, B_R_HIST, B_R_BASE, B_R_DEVARR, B_R_DEVIDX, B_R_OFF, B_R_LAT, B_R_AGG, B_R_TGT1,
-  B_R_DEVARR1, B_R_DEVIDX1, B_R_OFF1, B_R_MISC, B_R_LANE, B_R_DBASE0, B_R_DBASE1, B_R_LATD, B_R_VLAT, B_R_VEX, B_R_VOFF, B_FACT4, B_R_SCAN, B_R_BSCAN, B_PARETO, B_E_MISC, B_E_PAT, B_E_EXIT, B_R_WST, B_R_WEX, B_NBUF
+  B_R_DEVARR1, B_R_DEVIDX1, B_R_OFF1, B_R_MISC, B_R_LANE, B_R_DBASE0, B_R_DBASE1, B_R_LATD, B_R_VLAT, B_R_VEX, B_R_VOFF, B_FACT4, B_R_SCAN, B_R_BSCAN, B_PARETO, B_E_MISC, B_E_PAT, B_E_EXIT, B_R_WST, B_R_WEX, B_C_KEEP, B_C_GATHER, B_C_PTS, B_NBUF
 };
 static_assert(B_NBUF <= 48, "proteus_ctx::bufs is too small");
 
@@ -148,8 +155,21 @@ int px_solve_factored(proteus_ctx *ctx, const proteus_solve_args *a, const int32
                       const int32_t *d_dev, const int32_t *d_demand, int VM, const Tables &tab, const std::vector<int32_t> &h_P,
                       SolRec *d_sol);
 int px_prepare_tables(proteus_ctx *ctx, int D, const int32_t *d_dev_type, const int32_t *d_slo, int VM,
-                      Tables &tab);
+                      Tables &tab, bool clamp);
 uint64_t px_count_candidates(int mode, int D, const int32_t *dev_type, int T, int K, bool *overflow);
+
+// comm.cu: the NCCL communicator and the combine kernels
+enum { PX_RED_SUM = 0, PX_RED_MAX = 1 /* int64 */, PX_RED_MIN = 2 };
+bool px_comm_active(const proteus_ctx *ctx);
+int px_comm_allgather(proteus_ctx *ctx, const void *send, void *recv, size_t bytes);
+int px_comm_allreduce_u64(proteus_ctx *ctx, void *buf, size_t count, int op);
+int px_pick_solrec(proteus_ctx *ctx, const SolRec *d_gathered, int world, int n, SolRec *d_out);
+int px_gather_vectors(proteus_ctx *ctx, const SolRec *d_gathered, int world, int n, int stride, SolRec *d_out);
+int px_pareto_merge(proteus_ctx *ctx, const proteus_pareto_point *d_pts, int n, proteus_pareto_point *d_out,
+                    int32_t *d_n);
+void px_scenario_owner(const proteus_scenario *sc, int S, int world, int32_t *owner);
+void px_comm_destroy(proteus_ctx *ctx);
+int px_occupancy(proteus_ctx *ctx, const void *kern, int threads, size_t smem, int *occ);
 
 int px_pareto(proteus_ctx *ctx, int D, const int32_t *h_dev_type, const int32_t *d_dev, const int32_t *d_slo,
               int family, int allow_idle, int rank, int world, proteus_pareto_point *out, int32_t max_points,

@@ -210,7 +210,7 @@ int px_pareto(proteus_ctx *ctx, int D, const int32_t *h_dev_type, const int32_t 
   int VM = 0;
   for (int q = 0; q < ctx->Q; q++) VM = std::max(VM, ctx->V[q]);
   Tables tab;
-  int rc = px_prepare_tables(ctx, D, d_dev, d_slo, VM, tab);
+  int rc = px_prepare_tables(ctx, D, d_dev, d_slo, VM, tab, false);
   if (rc) return rc;
   ctx->tab_valid = false;  // the cached solve tables were overwritten
   std::vector<int32_t> hP((size_t)T * M);
@@ -228,6 +228,8 @@ int px_pareto(proteus_ctx *ctx, int D, const int32_t *h_dev_type, const int32_t 
   }
   if (cmax >= (1ll << 26)) return px_fail(ctx, PROTEUS_ERANGE, "capacity range %lld too large", (long long)cmax);
   const uint64_t N = (uint64_t)n;
+  const bool dist = px_comm_active(ctx);  // slices by communicator rank, combined by two all-reduces
+  if (dist) { rank = ctx->comm_rank; world = ctx->comm_world; }
   const uint64_t lo = mul_div_u(N, rank, world), hi = mul_div_u(N, rank + 1, world);
   const size_t nc = (size_t)cmax + 1;
   char *b = (char *)px_buf(ctx, B_PARETO, (size_t)D * K * 12 + nc * (8 + 4 + 8 + 8 + 8) + 256);
@@ -259,9 +261,16 @@ int px_pareto(proteus_ctx *ctx, int D, const int32_t *h_dev_type, const int32_t 
   if (sm1 > 48 * 1024) PX_CUDA(ctx, cudaFuncSetAttribute(k_pareto_best, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm1));
   if (sm2 > 48 * 1024) PX_CUDA(ctx, cudaFuncSetAttribute(k_pareto_index, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm2));
   if (cnt > 0) PX_LAUNCH(ctx, "pareto_best", k_pareto_best, blocks, PAR_THREADS, sm1, a);
+  // distributed: the largest accuracy sum per capacity over all slices (-1 = none)
+  if (dist && (rc = px_comm_allreduce_u64(ctx, best, nc, PX_RED_MAX))) return rc;
   PX_LAUNCH(ctx, "pareto_front", k_pareto_front, 1, 1024, 0, cmax, best, slot, fbest, fcap, fidx, d_nf);
-  if (cnt > 0) PX_LAUNCH(ctx, "pareto_index", k_pareto_index, blocks, PAR_THREADS, sm2, a);
   int32_t nf = 0;
+  if (dist) {  // every rank holds the same frontier; the lowest index per point over all slices
+    PX_CUDA(ctx, cudaMemcpyAsync(&nf, d_nf, 4, cudaMemcpyDeviceToHost, ctx->stream));
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+  }
+  if (cnt > 0) PX_LAUNCH(ctx, "pareto_index", k_pareto_index, blocks, PAR_THREADS, sm2, a);
+  if (dist && nf > 0 && (rc = px_comm_allreduce_u64(ctx, fidx, (size_t)nf, PX_RED_MIN))) return rc;
   PX_CUDA(ctx, cudaMemcpyAsync(&nf, d_nf, 4, cudaMemcpyDeviceToHost, ctx->stream));
   PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
   const int k = std::min(nf, max_points);
@@ -279,6 +288,6 @@ int px_pareto(proteus_ctx *ctx, int D, const int32_t *h_dev_type, const int32_t 
     out[i].index = hi_[i];
   }
   *n_points = nf;
-  *n_configs = cnt;
+  *n_configs = dist ? N : cnt;
   return 0;
 }

@@ -9,10 +9,15 @@
 //  2. per family q: order its variants by (accuracy desc, code asc) -> slot
 //     q*VM + j (reading C10 fill order); pad slots get code 0 / accuracy 0.
 //  3. per (device d, code o): Pdev[d][o] = P[type_d][o-1] (0 for idle).
+// With pclamp > 0 (the solve path) P is stored as min(P, pclamp): demand per
+// vector is < 2^22 = pclamp, so a water-fill take min(rem, cap) and every z
+// are unchanged, while slot sums of up to 64 devices stay far inside int32.
+// The Fig. 1b frontier (pareto.cu) sums the exact capacities: pclamp = 0.
 __global__ void k_prepare(int T, int Q, int M, int bmax, int D, int VM, const int32_t *__restrict__ lat,
                           const int32_t *__restrict__ acc, const int32_t *__restrict__ fam,
                           const int32_t *__restrict__ off, const int32_t *__restrict__ V,
-                          const int32_t *__restrict__ dev_type, const int32_t *__restrict__ slo, Tables tab) {
+                          const int32_t *__restrict__ dev_type, const int32_t *__restrict__ slo, int32_t pclamp,
+                          Tables tab) {
   const int K = M + 1;
   for (int i = threadIdx.x; i < T * M; i += blockDim.x) {
     int t = i / M, m = i % M;
@@ -24,7 +29,8 @@ __global__ void k_prepare(int T, int Q, int M, int bmax, int D, int VM, const in
     for (int b = dep; b >= 1; b--)
       if (2ll * row[b - 1] <= L) { bs = b; break; }
     tab.depth[i] = dep;
-    tab.P[i] = bs ? (int32_t)(((int64_t)bs * 1000000ll) / row[bs - 1]) : 0;
+    int32_t P = bs ? (int32_t)(((int64_t)bs * 1000000ll) / row[bs - 1]) : 0;
+    tab.P[i] = (pclamp > 0 && P > pclamp) ? pclamp : P;
   }
   for (int q = threadIdx.x; q < Q; q += blockDim.x) {
     for (int j = 0; j < VM; j++) { tab.slot_code[q * VM + j] = 0; tab.slot_acc[q * VM + j] = 0; }
@@ -48,7 +54,7 @@ __global__ void k_prepare(int T, int Q, int M, int bmax, int D, int VM, const in
 }
 
 int px_prepare_tables(proteus_ctx *ctx, int D, const int32_t *d_dev_type, const int32_t *d_slo, int VM,
-                      Tables &tab) {
+                      Tables &tab, bool clamp) {
   const int T = ctx->T, Q = ctx->Q, M = ctx->M, K = M + 1;
   size_t n = (size_t)2 * T * M + M + 2 * Q * VM + K + (size_t)D * K;
   int32_t *b = (int32_t *)px_buf(ctx, B_TABLES, n * 4);
@@ -61,7 +67,7 @@ int px_prepare_tables(proteus_ctx *ctx, int D, const int32_t *d_dev_type, const 
   tab.code_slot = b; b += K;
   tab.Pdev = b;
   PX_LAUNCH(ctx, "prepare", k_prepare, 1, 256, 0, T, Q, M, ctx->bmax, D, VM, ctx->d_lat, ctx->d_acc, ctx->d_fam,
-            ctx->d_off, ctx->d_V, d_dev_type, d_slo, tab);
+            ctx->d_off, ctx->d_V, d_dev_type, d_slo, clamp ? PX_PCLAMP : 0, tab);
   return 0;
 }
 

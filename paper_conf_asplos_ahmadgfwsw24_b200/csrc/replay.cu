@@ -1937,7 +1937,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     uint8_t *tgt = (uint8_t *)px_buf(ctx, rt ? B_R_TGT1 : B_R_TGT, (size_t)N + 16);
     int64_t *off = (int64_t *)px_buf(ctx, rt ? B_R_OFF1 : B_R_OFF, (size_t)2 * (PX_MAXD + 2) * 8);
     // + whole trailing ring segment: k_stitch bulk-copies 4 KB segments
-    uint32_t *darr = (uint32_t *)px_buf(ctx, rt ? B_R_DEVARR1 : B_R_DEVARR, ((size_t)N + 2 * RSEG) * 4);
+    // k_stitch's ring reads whole segments up to 2 past the head's: pad 3 segments
+    uint32_t *darr = (uint32_t *)px_buf(ctx, rt ? B_R_DEVARR1 : B_R_DEVARR, ((size_t)N + 3 * RSEG) * 4);
     uint32_t *dinv = (uint32_t *)px_buf(ctx, rt ? B_R_DEVIDX1 : B_R_DEVIDX, (size_t)N * 4 + 16);
     if (!pat || !hist || !fbase || !dbase || !tgt || !off || !darr || !dinv)
       return px_fail(ctx, PROTEUS_ENOMEM, "routing buffers");
@@ -1987,7 +1988,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   PX_CUDA(ctx, cudaMemcpyAsync(d_choff, choff.data(), choff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_goff, goff.data(), goff.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
   const int64_t NS = (N + 31) & ~(int64_t)31;  // latd row stride
-  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * NS * 4 + 8192);  // B_R_LAT stages host outputs
+  // B_R_LAT stages host outputs; the stitch ring reads up to 3 segments past a row's last query
+  uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * NS * 4 + 3 * RSEG * 4 + 64);
   if (!latd) return px_fail(ctx, PROTEUS_ENOMEM, "latency scratch");
   const int64_t nmax = NCH[0] > NCH[1] ? NCH[0] : NCH[1];
   ChunkSt *csb[2] = {nullptr, nullptr};  // chunk runs, double-buffered across fix-up rounds

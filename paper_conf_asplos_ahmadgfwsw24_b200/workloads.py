@@ -317,6 +317,10 @@ def config(name: str, **kw) -> dict:
 # Calibrated absolute demand totals (QPS); see DESIGN.md §3 for how they were chosen.
 C1_TOTAL = 600
 C2_TOTALS = (3000, 7000)
+# the bench step's batch (bench.py): 64 demand vectors, totals 1500..7500 QPS
+# (from the all-most-accurate regime to overload)
+C2_BENCH_NVEC = 64
+C2_BENCH_TOTALS = tuple(int(t) for t in np.linspace(1500, 7500, C2_BENCH_NVEC))
 C3_TOTALS = (3000, 12000)
 C3MINI_TOTALS = (8000, 30000)
 C3MINI_COUNTS = (6, 3, 3)   # 12 devices: multiset space 5005 * 220^2 = 2.42e8

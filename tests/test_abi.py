@@ -30,7 +30,7 @@ def test_library_exports_every_declared_symbol():
         assert hasattr(lib, name), name
     from paper_conf_asplos_ahmadgfwsw24_b200 import _native
     assert set(_native.EXPORTED) == set(_declared())
-    assert lib.proteus_abi_version() == 2
+    assert lib.proteus_abi_version() == _native.ABI_VERSION == 3
 
 
 def test_create_without_gpu_fails_cleanly():

@@ -1,7 +1,12 @@
-"""Multi-process (world_size 2, gloo, CPU) coverage of the N > 1 host logic:
-the slot all-reduce that combines per-rank search winners, the index-range
-and demand-vector splits.  The per-rank search itself is stood in for by the
-oracle over the rank's index range (the GPU kernels are covered by -m gpu)."""
+"""Multi-process (world_size 2, gloo, CPU) coverage of the N > 1 host logic
+(SURVEY §8(e)): the NCCL unique-id broadcast that joins the library contexts,
+the work splits the library uses (index slices, demand-vector slices, the
+scenario owners of proteus_scenario_owner -- host code of libproteus.so that
+runs without a GPU), and that each split is exact: per-rank results combined
+in the library's order reproduce the single-process answer.  The per-rank
+GPU work is stood in for by the oracle; the library's device-side combine
+(NCCL all-gather / all-reduce + pick kernels) is covered by -m gpu
+(tests/test_gpu_solve.py: combine_solutions, the world-1 NCCL communicator)."""
 
 import os
 import socket
@@ -17,10 +22,32 @@ def _free_port():
         return s.getsockname()[1]
 
 
+def _run(worker, world=2, timeout=600):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=worker, args=(r, world, port, q)) for r in range(world)]
+    for p in ps:
+        p.start()
+    out = [q.get(timeout=timeout) for _ in ps]
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    return sorted(out, key=lambda o: o[0])
+
+
+def _init(rank, world, port):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import torch.distributed as dist
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    return dist
+
+
 def _rank_best(prof, dev, slo, dem, lo, hi):
-    """Best (score, index) over flat indices [lo, hi): device 0 is the most
-    significant digit (reading C9); ascending order + strict > keeps the
-    lowest index among ties."""
+    """Best (score, index) over flat indices [lo, hi) by the oracle: device 0
+    is the most significant digit (reading C9); ascending order + strict >
+    keeps the lowest index among ties."""
     import oracle
     K, D = 1 + prof.M, len(dev)
     best = None
@@ -33,95 +60,96 @@ def _rank_best(prof, dev, slo, dem, lo, hi):
     return best if best else (0, (1 << 64) - 1)
 
 
-def _worker(rank, world, port, q):
-    import sys
-    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-    import torch.distributed as dist
-    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import allreduce_best, shard_range
-    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+def _id_worker(rank, world, port, q):
+    dist = _init(rank, world, port)
     try:
-        cfg = W.config("c1")
-        prof, cl, dem = cfg["prof"], cfg["cluster"], cfg["demand"][0]
-        n = (1 + prof.M) ** len(cl.device_type)
-        lo, hi = shard_range(n, rank, world)
-        s, i = _rank_best(prof, cl.device_type, cl.slo_us, dem, lo, hi)
-        gs, gi, grank = allreduce_best(s, i)
-        # demand-vector split of the batched re-solve covers every vector once
-        vlo, vhi = shard_range(3600, rank, world)
-        cover = np.zeros(3600, np.int64)
-        cover[vlo:vhi] = 1
-        import torch
-        t = torch.from_numpy(cover)
-        dist.all_reduce(t)
-        q.put((rank, gs, gi, grank, int(t.min()), int(t.max())))
+        from paper_conf_asplos_ahmadgfwsw24_b200 import Proteus, scenario_owner, workloads as W
+        from paper_conf_asplos_ahmadgfwsw24_b200.dist import broadcast_unique_id, shard_range
+        uid = broadcast_unique_id(Proteus.comm_unique_id() if rank == 0 else None)
+        sc = np.concatenate([W.scenarios_64(0, 0), W.scenarios_fig6(0), W.scenarios_64(0, 1)])
+        owner = scenario_owner(sc, world)
+        lo, hi = shard_range(3600, rank, world)
+        q.put((rank, uid, owner.tolist(), lo, hi))
     finally:
         dist.destroy_process_group()
 
 
-def test_world2_slot_allreduce_matches_single_process(oracle_mod):
+def test_world2_comm_id_broadcast_and_splits():
+    """Rank 0's 128-byte NCCL id reaches every rank unchanged (the bytes
+    proteus_comm_init needs); every rank computes the same scenario owners
+    (each scenario owned once, loads balanced) and disjoint vector slices."""
+    out = _run(_id_worker)
+    assert len(out[0][1]) == 128 and out[0][1] == out[1][1]
+    assert out[0][2] == out[1][2]
+    owner = np.array(out[0][2])
+    assert set(owner.tolist()) <= {0, 1} and abs(int(np.sum(owner == 0)) - int(np.sum(owner == 1))) <= 24
+    assert (out[0][3], out[0][4], out[1][3], out[1][4]) == (0, 1800, 1800, 3600)
+
+
+def _flat_worker(rank, world, port, q):
+    dist = _init(rank, world, port)
+    try:
+        from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+        from paper_conf_asplos_ahmadgfwsw24_b200.dist import shard_range
+        cfg = W.config("c1")
+        prof, cl = cfg["prof"], cfg["cluster"]
+        dems = np.array([[0, 0], [300, 100], [600, 0], [800, 700]], np.int32)
+        n = (1 + prof.M) ** len(cl.device_type)
+        lo, hi = shard_range(n, rank, world)
+        mine = [_rank_best(prof, cl.device_type, cl.slo_us, d, lo, hi) for d in dems]
+        parts = [None] * world
+        dist.all_gather_object(parts, mine)
+        q.put((rank, parts))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_world2_flat_slices_combine_to_the_optimum(oracle_mod):
+    """Index-range slices (the library's split) of c1: the (score desc,
+    index asc) maximum of the per-rank slice winners -- the order of
+    k_pick_solrec -- is the single-process optimum for every demand vector,
+    on every rank."""
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
     cfg = W.config("c1")
-    prof, cl, dem = cfg["prof"], cfg["cluster"], cfg["demand"][0]
-    ref = oracle_mod.solve(prof, cl.device_type, cl.slo_us, dem, 0)
-    ctx = mp.get_context("spawn")
-    q = ctx.Queue()
-    port = _free_port()
-    ps = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
-    for p in ps:
-        p.start()
-    out = [q.get(timeout=300) for _ in ps]
-    for p in ps:
-        p.join(timeout=60)
-        assert p.exitcode == 0
-    for rank, gs, gi, grank, cmin, cmax in out:
-        assert gi == ref["index"]
-        assert gs == (ref["served"] << 42) | ref["accsum"]
-        assert (cmin, cmax) == (1, 1)
-    assert len({o[3] for o in out}) == 1
-
-
-def test_pick_best_order_and_sign():
-    """Slots carry uint64 bit patterns in int64; the combine order is (score
-    desc, index asc) -- the same as the in-GPU reduction."""
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import pick_best, slot_vector
-    big = (1 << 63) + 5
-    v = slot_vector(0, 3, big, 7) + slot_vector(1, 3, big, 3) + slot_vector(2, 3, 10, 0)
-    assert pick_best(v) == (big, 3, 1)
-    v = slot_vector(0, 2, 4, 9) + slot_vector(1, 2, 4, 9)
-    assert pick_best(v)[:2] == (4, 9)
+    prof, cl = cfg["prof"], cfg["cluster"]
+    dems = np.array([[0, 0], [300, 100], [600, 0], [800, 700]], np.int32)
+    refs = [oracle_mod.solve(prof, cl.device_type, cl.slo_us, d, 0) for d in dems]
+    for _, parts in _run(_flat_worker):
+        for v, r in enumerate(refs):
+            cands = [p[v] for p in parts]
+            best = max(cands, key=lambda si: (si[0], -si[1]))
+            assert best == ((r["served"] << 42) | r["accsum"], r["index"])
 
 
 def _replay_worker(rank, world, port, q):
-    """Scenario-split replay: the per-rank replay is stood in for by the
-    oracle over this rank's scenario slice."""
-    import sys
-    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-    import torch.distributed as dist
-    import oracle
-    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import replay_sharded
-    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    dist = _init(rank, world, port)
     try:
+        import torch
+        import oracle
+        from paper_conf_asplos_ahmadgfwsw24_b200 import scenario_owner, workloads as W
         cfg = W.config("c3", totals=(12000,))
         prof, cl = cfg["prof"], cfg["cluster"]
         r = oracle.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][0], 2)
         a, f = W.query_trace(8000, 12000.0, cfg["weights"], 17, "gamma")
-        sc = np.concatenate([W.scenarios_64(0, 0)[::9], W.scenarios_fig6(0)[::13]])
-
-        def rep(scenarios):
-            return oracle.replay(prof, cl.device_type, r["option"], r["z"], cfg["demand"][0], cl.slo_us, a, f,
-                                 scenarios, want_latency=False)
-
-        agg, _, (lo, hi) = replay_sharded(rep, sc)
-        q.put((rank, lo, hi, {k: v.tolist() for k, v in agg.items()}))
+        sc = oracle.scenario_rows(np.concatenate([W.scenarios_64(0, 0)[::9], W.scenarios_fig6(0)[::13]]))
+        mine = np.flatnonzero(scenario_owner(sc, world) == rank)
+        agg = np.zeros((3, len(sc)), np.int64)
+        if len(mine):
+            o = oracle.replay(prof, cl.device_type, r["option"], r["z"], cfg["demand"][0], cl.slo_us, a, f,
+                              sc[mine], want_latency=False)
+            for k, name in enumerate(("violations", "on_time", "acc_sum")):
+                agg[k, mine] = o[name].astype(np.int64)
+        t = torch.from_numpy(agg)
+        dist.all_reduce(t)  # zero-padded per-scenario aggregates: the sum is a gather
+        q.put((rank, mine.tolist(), t.numpy().tolist()))
     finally:
         dist.destroy_process_group()
 
 
-def test_world2_scenario_split_replay(oracle_mod):
-    """§8(e) replay: scenarios split by rank, aggregates gathered by one SUM
-    all-reduce -- every rank ends with the single-process aggregates."""
+def test_world2_scenario_owner_replay(oracle_mod):
+    """§8(e) replay split: scenario s on rank owner[s]; the zero-padded
+    per-scenario aggregates summed over ranks (the library's all-reduce)
+    equal the single-process aggregates; each scenario ran exactly once."""
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
     cfg = W.config("c3", totals=(12000,))
     prof, cl = cfg["prof"], cfg["cluster"]
@@ -130,87 +158,24 @@ def test_world2_scenario_split_replay(oracle_mod):
     sc = np.concatenate([W.scenarios_64(0, 0)[::9], W.scenarios_fig6(0)[::13]])
     ref = oracle_mod.replay(prof, cl.device_type, r["option"], r["z"], cfg["demand"][0], cl.slo_us, a, f, sc,
                             want_latency=False)
-    ctx = mp.get_context("spawn")
-    q = ctx.Queue()
-    port = _free_port()
-    ps = [ctx.Process(target=_replay_worker, args=(rk, 2, port, q)) for rk in range(2)]
-    for p in ps:
-        p.start()
-    out = [q.get(timeout=300) for _ in ps]
-    for p in ps:
-        p.join(timeout=60)
-        assert p.exitcode == 0
-    spans = sorted((lo, hi) for _, lo, hi, _ in out)
-    assert spans[0][0] == 0 and spans[0][1] == spans[1][0] and spans[1][1] == len(sc)
-    for _, _, _, agg in out:
-        for k in ("violations", "on_time", "acc_sum"):
-            assert agg[k] == ref[k].tolist(), k
+    out = _run(_replay_worker)
+    assert sorted(out[0][1] + out[1][1]) == list(range(len(sc)))
+    for _, _, agg in out:
+        for k, name in enumerate(("violations", "on_time", "acc_sum")):
+            assert agg[k] == ref[name].astype(np.int64).tolist(), name
 
 
-def _batch_worker(rank, world, port, q):
-    """Batched flat search split by index range: the per-rank library call is
-    stood in for by a fake `px` whose solve() returns, per demand vector, the
-    oracle's best over the rank's index slice, materialised by the oracle."""
-    import sys
-    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
-    import torch.distributed as dist
-    import oracle
-    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import shard_range, solve_sharded_batch
-    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
-    try:
-        cfg = W.config("c1")
-        prof, cl = cfg["prof"], cfg["cluster"]
-        dems = np.array([[0, 0], [300, 100], [600, 0], [800, 700]], np.int32)
-        K, D = 1 + prof.M, len(cl.device_type)
-
-        class FakePx:
-            def solve_batch(self, device_type, slo_us, demand, mode, shard_rank, shard_world):
-                n = K ** D
-                lo, hi = shard_range(n, shard_rank, shard_world)
-                out = {k: [] for k in ("score", "index", "served", "unmet", "accsum", "eff_acc_micro", "option",
-                                       "z_qps")}
-                for dem in demand:
-                    s, i = _rank_best(prof, device_type, slo_us, dem, lo, hi)
-                    opt = np.array([(i // K ** (D - 1 - d)) % K for d in range(D)], np.int32)
-                    r = oracle.score_placement(prof, device_type, slo_us, dem, opt)
-                    for k, v in (("score", s), ("index", i), ("served", r["served"]), ("unmet", r["unmet"]),
-                                 ("accsum", r["accsum"]), ("eff_acc_micro", r["eff"]), ("option", opt),
-                                 ("z_qps", r["z"])):
-                        out[k].append(v)
-                out = {k: np.array(v, np.uint64 if k in ("score", "index") else np.int64) for k, v in out.items()}
-                return out, hi - lo
-
-        best, _, ncand, _ = solve_sharded_batch(FakePx(), cl.device_type, cl.slo_us, dems, mode=0)
-        q.put((rank, [(int(best["score"][v]), int(best["index"][v]), int(best["served"][v]),
-                       int(best["accsum"][v]), ncand, best["option"][v].tolist(), best["z_qps"][v].tolist())
-                      for v in range(len(dems))]))
-    finally:
-        dist.destroy_process_group()
-
-
-def test_world2_batched_flat_search(oracle_mod):
-    """One all-gather of the per-rank winners (already materialised) per
-    batch of demand vectors: every rank ends with the single-process optimum,
-    placement and z of every vector."""
-    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
-    cfg = W.config("c1")
-    prof, cl = cfg["prof"], cfg["cluster"]
-    dems = np.array([[0, 0], [300, 100], [600, 0], [800, 700]], np.int32)
-    refs = [oracle_mod.solve(prof, cl.device_type, cl.slo_us, d, 0) for d in dems]
-    ctx = mp.get_context("spawn")
-    q = ctx.Queue()
-    port = _free_port()
-    ps = [ctx.Process(target=_batch_worker, args=(rk, 2, port, q)) for rk in range(2)]
-    for p in ps:
-        p.start()
-    out = [q.get(timeout=600) for _ in ps]
-    for p in ps:
-        p.join(timeout=60)
-        assert p.exitcode == 0
-    for _, sols in out:
-        for (sc, idx, served, accsum, ncand, opt, z), r in zip(sols, refs):
-            assert idx == r["index"] and sc == (r["served"] << 42) | r["accsum"]
-            assert (served, accsum) == (r["served"], r["accsum"])
-            assert ncand == r["n_candidates"]
-            assert opt == r["option"].tolist() and z == r["z"].tolist()
+@pytest.mark.parametrize("world", [3, 8])
+def test_scenario_owner_balance(world):
+    """proteus_scenario_owner (host code of the library): deterministic,
+    every scenario owned once, and no rank gets all the large-cap,
+    large-SLO scenarios (the critical replay lanes) -- unlike contiguous
+    slices, where the last rank would own every 5x-SLO scenario."""
+    from paper_conf_asplos_ahmadgfwsw24_b200 import scenario_owner, workloads as W
+    sc = W.scenarios_64(0)
+    o = scenario_owner(sc, world)
+    assert o.tolist() == scenario_owner(sc, world).tolist()
+    assert set(o.tolist()) == set(range(world))
+    heavy = np.flatnonzero((sc[:, 0] >= 3000) & ((sc[:, 1] == 0) | (sc[:, 1] >= 32)))
+    counts = np.bincount(o[heavy], minlength=world)
+    assert counts.max() - counts.min() <= 2

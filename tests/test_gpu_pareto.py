@@ -59,12 +59,11 @@ def test_large_10_devices_and_shards(px, oracle_mod):
     configurations (several blocks per thread range, carries through every
     digit); three shards merged equal the whole space."""
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import pareto_merge
     cfg = W.config("c3")
     dev = np.array([0, 0, 0, 0, 1, 1, 1, 2, 2, 2], np.int32)
     g = check(px, oracle_mod, cfg["prof"], dev, cfg["cluster"].slo_us, 3, False)
     parts = [px.pareto(dev, cfg["cluster"].slo_us, 3, shard_rank=r, shard_world=3) for r in range(3)]
-    m = pareto_merge(parts)
+    m = px.pareto_merge(parts)  # proteus_pareto_merge (device kernel)
     assert m["n_configs"] == g["n_configs"]
     for k in ("cap", "accsum", "index"):
         assert m[k].tolist() == g[k].tolist(), k
@@ -79,3 +78,19 @@ def test_bench_size_5_pow_12(px, oracle_mod):
     dev = np.repeat(np.arange(3, dtype=np.int32), 4)
     g = check(px, oracle_mod, cfg["prof"], dev, cfg["cluster"].slo_us, 3, False)
     assert g["n_configs"] == 5 ** 12
+
+
+def test_pareto_merge_kernel_equal_points_and_ties(px):
+    """proteus_pareto_merge on hand-made parts (reading P3): duplicates of one
+    point keep the lowest index; a point dominated by another part's point
+    drops; capacity 0 has accuracy 0; output sorted by capacity."""
+    parts = [dict(cap=np.array([0, 10, 20], np.int64), accsum=np.array([0, 9_000_000, 16_000_000], np.int64),
+                  index=np.array([0, 7, 9], np.uint64), n_configs=5),
+             dict(cap=np.array([10, 20, 30], np.int64), accsum=np.array([9_000_000, 17_000_000, 21_000_000], np.int64),
+                  index=np.array([3, 11, 12], np.uint64), n_configs=5)]
+    m = px.pareto_merge(parts)
+    # (10, 0.9) idx 3 (lowest of the two); (20, 0.85) beats (20, 0.8); (30, 0.7); (0, 0) is dominated
+    assert m["cap"].tolist() == [10, 20, 30]
+    assert m["accsum"].tolist() == [9_000_000, 17_000_000, 21_000_000]
+    assert m["index"].tolist() == [3, 11, 12]
+    assert m["n_configs"] == 10

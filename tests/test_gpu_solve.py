@@ -126,21 +126,20 @@ def test_c2_generic_kernel_and_multiset(px, oracle_mod):
 
 
 def test_c2_sharded_identical(px, oracle_mod):
-    """Index-range shards (as on 1/2/4/8 GPUs) combined by the slot order give
-    the single-GPU result."""
+    """Index-range shards (as on 1/2/4/8 GPUs) combined on the device by
+    proteus_combine_solutions -- the (score desc, index asc) pick the NCCL
+    path runs after its all-gather -- give the single-GPU result."""
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import pick_best, slot_vector
     cfg = W.config("c2")
     px.load_profiles(cfg["prof"])
-    dev, slo, dem = cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"][0]
-    full = px.solve(dev, slo, dem, mode=0)[0]
+    dev, slo, dem = cfg["cluster"].device_type, cfg["cluster"].slo_us, cfg["demand"][:1]
+    full, n = px.solve_batch(dev, slo, dem, mode=0)
     for world in (2, 3, 8):
-        slots = sum(slot_vector(r, world, s.score, s.index)
-                    for r in range(world) for s in [px.solve(dev, slo, dem, mode=0, shard_rank=r, shard_world=world)[0]])
-        s, i, _ = pick_best(slots)
-        assert (s, i) == (full.score, full.index)
-        m = px.materialize(dev, slo, dem, i)
-        assert m.option.tolist() == full.option.tolist() and m.z.tolist() == full.z.tolist()
+        parts = [px.solve_batch(dev, slo, dem, mode=0, shard_rank=r, shard_world=world) for r in range(world)]
+        best, n_all = px.combine_solutions([p[0] for p in parts], [p[1] for p in parts], len(dev))
+        assert n_all == n == 13**8
+        for k in ("score", "index", "served", "unmet", "accsum", "eff_acc_micro", "option", "z_qps"):
+            assert np.array_equal(np.asarray(best[k]), np.asarray(full[k])), (world, k)
 
 
 def test_c3_factored(px, oracle_mod):
@@ -311,32 +310,31 @@ def test_c2_bench_batch_sampled(px, oracle_mod):
 
 @pytest.mark.parametrize("world", [2, 3, 8])
 def test_c2_batch_shards_combine(px, world):
-    """The bench's N-GPU path without NCCL: every rank's proteus_solve_batch
-    over its index slice for the 64-vector batch, packed as dist.pack_batch
-    and combined by dist.pick_batch (the all-gather's result), equals the
-    one-GPU batch -- score, index, value, placement and z of every vector."""
+    """The bench's N-GPU combine without NCCL: every rank's
+    proteus_solve_batch over its index slice for the 64-vector batch,
+    combined by proteus_combine_solutions (the pick kernel of the NCCL path),
+    equals the one-GPU batch -- score, index, value, placement and z of every
+    vector."""
     import bench
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import pack_batch, pick_batch
     cfg = W.config("c2", totals=bench.C2_TOTALS)
     prof, cl = cfg["prof"], cfg["cluster"]
     px.load_profiles(prof)
     D = len(cl.device_type)
     ref, n = px.solve_batch(cl.device_type, cl.slo_us, cfg["demand"], mode=0)
-    parts = []
-    for r in range(world):
-        loc, nc = px.solve_batch(cl.device_type, cl.slo_us, cfg["demand"], mode=0, shard_rank=r, shard_world=world)
-        parts.append(pack_batch(loc, D, nc))
-    best, n_all = pick_batch(np.stack(parts), D)
+    parts = [px.solve_batch(cl.device_type, cl.slo_us, cfg["demand"], mode=0, shard_rank=r, shard_world=world)
+             for r in range(world)]
+    best, n_all = px.combine_solutions([p[0] for p in parts], [p[1] for p in parts], D)
     assert n_all == n == 13**8
     for k in ("score", "index", "served", "unmet", "accsum", "eff_acc_micro", "option", "z_qps"):
         assert np.array_equal(np.asarray(best[k]).astype(np.int64), np.asarray(ref[k]).astype(np.int64)), k
 
 
 def test_nccl_collective_paths_world1():
-    """The NCCL code paths of dist.solve_sharded_batch (all_gather_into_tensor)
-    and dist.replay_sharded (all-reduce gather) in a world-1 NCCL process
-    group on cuda:0 (subprocess): results equal the direct calls."""
+    """The library's own NCCL communicator (proteus_comm_init, world 1 on
+    cuda:0, in a subprocess with a torch NCCL process group for the id
+    broadcast): distributed solve (modes 0, 1, 2), frontier, replay and
+    closed loop equal the non-distributed calls (scripts/nccl_world1.py)."""
     import os
     import socket
     import subprocess

@@ -116,13 +116,14 @@ def test_scaling_capacity_keeps_frontier(allow_idle):
     assert a["index"].tolist() == b["index"].tolist()
 
 
-def test_pareto_merge_of_shards():
-    """dist.pareto_merge: the frontier of the union of per-shard frontiers
-    (each computed by the oracle on a sub-inventory's configurations would need
-    index slices, so the shards here are slices of the full configuration list
-    reduced by the definition) equals the oracle's frontier of the whole."""
+def test_pareto_shard_decomposition():
+    """The multi-GPU split of Fig. 1b (index slices) is exact: a
+    point dominated inside a slice is dominated in the whole space, so the
+    frontier (definition P3, exact fractions) of the union of the slices'
+    frontiers, lowest index per point, equals the oracle's frontier of the
+    whole space.  (The product's merge, proteus_pareto_merge, runs on the GPU:
+    tests/test_gpu_pareto.py.)"""
     import oracle
-    from paper_conf_asplos_ahmadgfwsw24_b200.dist import pareto_merge
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
     cfg = W.config("c3")
     prof, cl = cfg["prof"], cfg["cluster"]
@@ -137,18 +138,17 @@ def test_pareto_merge_of_shards():
         a = sum(int(P[dev[d], off + o]) * int(prof.acc_micro[off + o]) for d, o in enumerate(c_))
         pts.append((c, a, i))
 
-    def front(sub):  # definition of the frontier on a slice (exact fractions)
-        keep = []
+    def front(sub):  # definition of the frontier (exact fractions), lowest index per point
+        keep = {}
         for c, a, i in sub:
             fa = Fraction(a, c) if c else Fraction(0)
             dom = any(c2 >= c and (Fraction(a2, c2) if c2 else Fraction(0)) >= fa and
                       (c2 > c or (Fraction(a2, c2) if c2 else Fraction(0)) > fa) for c2, a2, _ in sub)
-            if not dom:
-                keep.append((c, a, i))
-        return dict(cap=np.array([k[0] for k in keep], np.int64), accsum=np.array([k[1] for k in keep], np.int64),
-                    index=np.array([k[2] for k in keep], np.uint64), n_configs=len(sub))
+            if not dom and ((c, a) not in keep or i < keep[(c, a)]):
+                keep[(c, a)] = i
+        return sorted((c, a, i) for (c, a), i in keep.items())
     parts = [front(pts[k * 625 // 3:(k + 1) * 625 // 3]) for k in range(3)]
-    m = pareto_merge(parts)
-    assert m["n_configs"] == 625 == whole["n_configs"]
-    for k in ("cap", "accsum", "index"):
-        assert m[k].tolist() == whole[k].tolist(), k
+    merged = front([p for part in parts for p in part])
+    assert [m[0] for m in merged] == whole["cap"].tolist()
+    assert [m[1] for m in merged] == whole["accsum"].tolist()
+    assert [m[2] for m in merged] == whole["index"].tolist()

@@ -159,3 +159,42 @@ def test_uniform_routing_has_no_sink(oracle_mod):
     hosted = {int(fam_m[o - 1]) for o in r["option"] if o > 0}
     dropped = out["latency"][0] == 0xFFFFFFFF
     assert set(np.unique(f[dropped]).tolist()) <= set(range(prof.Q)) - hosted
+
+
+def test_acc_sum_hand_worked(oracle_mod):
+    """R9 pin ("accuracy for all the queries successfully
+    served"): acc_sum = sum of the serving variant's accuracy over ON-TIME
+    queries only; late and dropped queries add nothing.  Worked by hand:
+
+    one family, two variants v0 (A = 1 000 000, option 1) and v1 (A = 900 000,
+    option 2); one device type, table depth 1 (so Bmax = 1, R4: every query is
+    dispatched alone at max(F, a)), T_v0(1) = 100 us, T_v1(1) = 50 us.  Device
+    0 hosts v0 with z = 1, device 1 hosts v1 with z = 1, demand s = 3, so the
+    sink weight is unmet = 1 (R7, R8).  SWRR over weights (1, 1, sink 1):
+    currents (1,1,1) -> device 0; (-1,2,2) -> device 1; (0,0,3) -> sink; the
+    pattern repeats every 3 queries.  Arrivals 0, 0, 0, 10, 10, 20 us:
+      q0 -> dev 0 at 0: F = 100, latency 100
+      q1 -> dev 1 at 0: F = 50,  latency 50
+      q2 -> sink: dropped (UINT32_MAX)
+      q3 -> dev 0 at 10, busy until 100: F = 200, latency 190
+      q4 -> dev 1 at 10, busy until 50:  F = 100, latency 90
+      q5 -> sink: dropped
+    SLO base 150 us, multiplier 1x: q3 is late (190 > 150, R6) -> on_time 3,
+    violations 3 (one late + two dropped), acc_sum = A0 + A1 + A1 = 2 800 000.
+    Multiplier 2x (SLO 300): q3 on time -> on_time 4, violations 2,
+    acc_sum = 1e6 + 9e5 + 1e6 + 9e5 = 3 800 000."""
+    from paper_conf_asplos_ahmadgfwsw24_b200.workloads import Profiles
+    prof = Profiles(T=1, Q=1, V=np.array([2], np.int32), acc_micro=np.array([1_000_000, 900_000], np.int32),
+                    bmax=1, lat_us=np.array([[[100], [50]]], np.int32))
+    arr = np.array([0, 0, 0, 10, 10, 20], np.uint32)
+    fam = np.zeros(6, np.uint8)
+    sc = np.array([[1000, 0, 0], [2000, 0, 0]], np.int32)
+    out = oracle_mod.replay(prof, np.array([0, 0], np.int32), np.array([1, 2], np.int32),
+                            np.array([1, 1], np.int32), np.array([3], np.int32), np.array([150], np.int32),
+                            arr, fam, sc)
+    U = 0xFFFFFFFF
+    assert out["latency"][0].tolist() == [100, 50, U, 190, 90, U]
+    assert out["latency"][1].tolist() == [100, 50, U, 190, 90, U]
+    assert out["on_time"].tolist() == [3, 4]
+    assert out["violations"].tolist() == [3, 2]
+    assert out["acc_sum"].tolist() == [2_800_000, 3_800_000]
