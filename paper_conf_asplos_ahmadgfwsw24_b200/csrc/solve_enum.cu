@@ -31,6 +31,9 @@
 #ifndef FLAT_MINB
 #define FLAT_MINB 1  // blocks per SM the register budget is sized for
 #endif
+#ifndef FLAT_RK
+#define FLAT_RK 1    // outer prefixes per thread per work item, in units of K
+#endif
 #define GEN_THREADS 128
 
 // ------------------------------------------------------------ reduce ----
@@ -179,10 +182,38 @@ __global__ void __launch_bounds__(GEN_THREADS) k_enum_generic(const __grid_const
 }
 
 // -------------------------------------------- specialised flat kernel ----
+// k_flat_fam<QM, VM>: mode 0 with families supplied in accuracy order and
+// Q <= QM, V_q <= VM.  The index is split as
+//   idx = o K^3 + o3 K^2 + oA K + oB,
+// o = the options of devices 0..D-4 ("outer prefix"), o3, oA, oB those of
+// devices D-3, D-2, D-1.  A placement's value is the sum over families of
+// the family's water-fill value (Eqs. 1, 3, 5 make a device serve only its
+// variant's family), so for the K^2 candidates of a block (o, o3) everything
+// is a function of per-family quantities of the block's capacities c_q:
+//   F_q   = fill_q(c_q)                            (the (idle, idle) value)
+//   MA_q  = max_j fill_q(c_q + PA_j e_j) - F_q       (device D-2 joins family q)
+//   MB_q  = max_j fill_q(c_q + PB_j e_j) - F_q       (device D-1 joins family q)
+//   J_q   = max_{i,j} fill_q(c_q + PA_i e_i + PB_j e_j) - F_q   (both join q)
+// and the block's maximum is EXACT:
+//   sum_q F_q + max(0, max_q MA_q, max_q MB_q, max_{qa != qb} MA_qa + MB_qb, max_q J_q)
+// (a candidate with oA, oB in different families scores the separable sum).
+// Devices D-3 and D-4 change one family's capacities per step, so between
+// consecutive blocks only one family's state is recomputed ("incremental
+// family carry"): the thread keeps the states of the outer prefix (devices
+// 0..D-4) for every family, and per block recomputes only the family of o3.
+// A block is skipped with one compare unless its maximum beats the running
+// threshold; then (rarely) its lowest index reaching the maximum is found by
+// a re-scan in index order, so the thread keeps its first maximum (reading
+// C9).  Capacities of the outer prefix live in shared memory ([slot][thread],
+// conflict-free), the per-family states in registers (compile-time indices),
+// the last two devices' capacities and the accuracies in the constant bank.
 template <int QM, int VM>
 struct FlatArgs {
-  int32_t D, K;
-  uint64_t p_lo, p_hi, per_thread;
+  int32_t D, K, nvec;
+  uint64_t o_lo, o_hi, per_thread;  // outer prefixes [o_lo, o_hi); per thread per work item (a multiple of K)
+  uint64_t n_items;                 // work items: (item / nvec)-th span of FLAT_THREADS * per_thread outer
+                                    // prefixes of vector item % nvec
+  unsigned long long *counter;      // work-item counter (0 at launch)
   int32_t A[QM * VM];   // accuracy per slot
   int32_t PA[QM * VM];  // capacity of slot on device D-2
   int32_t PB[QM * VM];  // capacity of slot on device D-1
@@ -194,25 +225,113 @@ struct FlatArgs {
   unsigned long long *gbound;  // per vector of the launch: best score any thread has found (0 at launch)
 };
 
-// water-fill of family q over slots q*VM..q*VM+VM-1, with capacity pa added
-// to slot ja and pb to slot jb (compile-time; -1 = none) -> packed score
+// water-fill of one family: capacities c[0..VM) in fill order (reading C10),
+// demand s -> packed (served << 42) + accsum
 template <int QM, int VM>
-__device__ __forceinline__ uint64_t fill(const int (&caps)[QM * VM], const FlatArgs<QM, VM> &a,
-                                         const int32_t *sd, int q, int ja, int pa, int jb, int pb) {
-  int rem = sd[q];
+__device__ __forceinline__ uint64_t fam_fill(const int (&c)[VM], int s, const FlatArgs<QM, VM> &a, int q) {
+  int rem = s;
   uint64_t acc = 0;
 #pragma unroll
   for (int j = 0; j < VM; j++) {
-    int c = caps[q * VM + j] + (j == ja ? pa : 0) + (j == jb ? pb : 0);
-    int t = min(rem, c);
+    const int t = min(rem, c[j]);
     acc += (uint64_t)(uint32_t)a.A[q * VM + j] * (uint32_t)t;
     rem -= t;
   }
-  return px_pack((uint32_t)(sd[q] - rem), acc);
+  return px_pack((uint32_t)(s - rem), acc);
 }
 
+struct FamState {
+  uint64_t F, MA, MB, J;
+};
+
+// SYM: devices D-2 and D-1 have the same capacities (same device type), so
+// MB = MA and the joint fills are symmetric: 1 + V + V(V+1)/2 fills instead
+// of 1 + 2V + V^2
+template <int QM, int VM, bool SYM>
+__device__ __forceinline__ FamState fam_state(const int (&c)[VM], int s, const FlatArgs<QM, VM> &a, int q) {
+  FamState st;
+  st.F = fam_fill<QM, VM>(c, s, a, q);
+  uint64_t ma = st.F, mb = st.F, jm = st.F;
+#pragma unroll
+  for (int i = 0; i < VM; i++) {
+    int ci[VM];
+#pragma unroll
+    for (int k = 0; k < VM; k++) ci[k] = c[k] + (k == i ? a.PA[q * VM + i] : 0);
+    const uint64_t fa = fam_fill<QM, VM>(ci, s, a, q);
+    ma = fa > ma ? fa : ma;
+    if (!SYM) {
+      int cb[VM];
+#pragma unroll
+      for (int k = 0; k < VM; k++) cb[k] = c[k] + (k == i ? a.PB[q * VM + i] : 0);
+      const uint64_t fb = fam_fill<QM, VM>(cb, s, a, q);
+      mb = fb > mb ? fb : mb;
+    }
+#pragma unroll
+    for (int j = SYM ? i : 0; j < VM; j++) {
+      int cj[VM];
+#pragma unroll
+      for (int k = 0; k < VM; k++) cj[k] = ci[k] + (k == j ? a.PB[q * VM + j] : 0);
+      const uint64_t fj = fam_fill<QM, VM>(cj, s, a, q);
+      jm = fj > jm ? fj : jm;
+    }
+  }
+  st.MA = ma - st.F;
+  st.MB = (SYM ? ma : mb) - st.F;
+  st.J = jm - st.F;
+  return st;
+}
+
+// The block's first candidate (index order: oA-major, then oB, idle first,
+// slots = codes in order) scoring Mx; returns its oA * K + oB, -1 if none
+// (an internal error, caught by the materialise check).  Rare: called when a
+// block beats the thread's running maximum, so it is kept out of line.
 template <int QM, int VM>
-__global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __grid_constant__ FlatArgs<QM, VM> a) {
+__device__ __noinline__ int flat_rescan(const FlatArgs<QM, VM> &a, const int *sCaps /* [S][FLAT_THREADS] */,
+                                        const int32_t *sDem, int s3, int p3, uint64_t base, const uint64_t *Fq,
+                                        uint64_t Mx) {
+  constexpr int S = QM * VM;
+  const int K = a.K;
+  int c3[S];
+#pragma unroll
+  for (int k = 0; k < S; k++) c3[k] = sCaps[k * FLAT_THREADS + threadIdx.x] + (k == s3 ? p3 : 0);
+  uint64_t dB[S];
+#pragma unroll
+  for (int sb = 0; sb < S; sb++) {
+    const int qb = sb / VM;
+    int cb[VM];
+#pragma unroll
+    for (int j = 0; j < VM; j++) cb[j] = c3[qb * VM + j] + (j == sb % VM ? a.PB[sb] : 0);
+    dB[sb] = fam_fill<QM, VM>(cb, sDem[qb], a, qb) - Fq[qb];
+  }
+  if (base == Mx) return 0;  // (idle, idle)
+  for (int sb = 0; sb < S; sb++)
+    if (base + dB[sb] == Mx) return a.code[sb];
+  for (int sa = 0; sa < S; sa++) {
+    const int qa = sa / VM;
+    int ca[VM];
+#pragma unroll
+    for (int j = 0; j < VM; j++) ca[j] = c3[qa * VM + j] + (j == sa % VM ? a.PA[sa] : 0);
+    const uint64_t ba = base - Fq[qa] + fam_fill<QM, VM>(ca, sDem[qa], a, qa);
+    if (ba == Mx) return a.code[sa] * K;
+    for (int sb = 0; sb < S; sb++) {
+      const int qb = sb / VM;
+      uint64_t v;
+      if (qb == qa) {
+        int cj[VM];
+#pragma unroll
+        for (int j = 0; j < VM; j++) cj[j] = ca[j] + (j == sb % VM ? a.PB[sb] : 0);
+        v = base - Fq[qa] + fam_fill<QM, VM>(cj, sDem[qa], a, qa);
+      } else {
+        v = ba + dB[sb];
+      }
+      if (v == Mx) return a.code[sa] * K + a.code[sb];
+    }
+  }
+  return -1;
+}
+
+template <int QM, int VM, bool SYM>
+__global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_fam(const __grid_constant__ FlatArgs<QM, VM> a) {
   constexpr int S = QM * VM;
   extern __shared__ int32_t smem[];
   const int D = a.D, K = a.K;
@@ -220,145 +339,146 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_pair(const __g
   int32_t *sCS = smem + D * K; // [K]
   for (int i = threadIdx.x; i < D * K; i += blockDim.x) sP[i] = a.Pdev[i];
   for (int i = threadIdx.x; i < K; i += blockDim.x) sCS[i] = a.code_slot[i];
-  __shared__ int32_t sDem[QM];  // this block's demand vector (grid.x)
-  // grid.x = vector (fastest), grid.y = prefix range: the blocks of one vector
-  // are spread over the whole launch, so most of them start with the
-  // grid-wide bound of their vector already raised by the earlier ones
-  const int vec = blockIdx.x, blk = blockIdx.y;
-  if (threadIdx.x < QM) sDem[threadIdx.x] = a.s[vec][threadIdx.x];
-  __syncthreads();
-  const uint64_t tid = (uint64_t)blk * blockDim.x + threadIdx.x;
-  uint64_t p = a.p_lo + tid * a.per_thread;
-  const uint64_t pend = p + a.per_thread < a.p_hi ? p + a.per_thread : a.p_hi;
-  const uint64_t KK = (uint64_t)K * K;
+  __shared__ int32_t sDem[QM];  // the work item's demand vector
+  __shared__ unsigned long long sItem;
+  // capacities of devices 0..D-4 per slot ([slot][thread]: conflict-free)
+  __shared__ int sCaps[S][FLAT_THREADS];
+  const uint64_t K2 = (uint64_t)K * K, K3 = K2 * K;
+  const int ND = D - 3;  // outer digits: devices 0..D-4
+  // persistent blocks: work items taken in order, vectors interleaved (item %
+  // nvec), so every vector's items spread over the launch and most start with
+  // the grid-wide bound of their vector already raised by earlier items
+  for (;;) {
+    if (threadIdx.x == 0) sItem = atomicAdd(a.counter, 1ull);
+    __syncthreads();
+    const uint64_t item = sItem;
+    if (item >= a.n_items) break;
+    const int vec = (int)(item % a.nvec);
+    const uint64_t chunk = item / a.nvec;
+    if (threadIdx.x < QM) sDem[threadIdx.x] = a.s[vec][threadIdx.x];
+    __syncthreads();
+  uint64_t o = a.o_lo + (chunk * FLAT_THREADS + threadIdx.x) * a.per_thread;
+  const uint64_t oend = o + a.per_thread < a.o_hi ? o + a.per_thread : a.o_hi;
   uint64_t best_s = 0, best_i = ~0ull;
-  if (p < pend) {
-    int dig[PX_MAXD];
+  bool rec = false;
+  if (o < oend) {
+    int dig[PX_MAXD];  // touched on carries only
     {
-      uint64_t x = p;
-      for (int i = D - 3; i >= 0; i--) { dig[i] = (int)(x % K); x /= K; }
+      uint64_t x = o;
+      for (int i = ND - 1; i >= 0; i--) { dig[i] = (int)(x % K); x /= K; }
     }
-    // capacities of devices 0..D-4 per slot: rebuilt only when a digit above
-    // D-3 changes, kept in shared memory ([slot][thread], conflict-free) to
-    // leave the registers to the candidate loop
-    __shared__ int sCapsB[S][FLAT_THREADS];
-    auto rebuild = [&]() {
+    FamState st[QM];
+    uint64_t Fsum = 0;
+    auto fam_from_smem = [&](int q) -> FamState {
+      int c[VM];
+#pragma unroll
+      for (int j = 0; j < VM; j++) c[j] = sCaps[q * VM + j][threadIdx.x];
+      return fam_state<QM, VM, SYM>(c, sDem[q], a, q);
+    };
+    auto rebuild = [&]() {  // all families from the outer digits
       int cb[S];
 #pragma unroll
-      for (int s = 0; s < S; s++) cb[s] = 0;
-      for (int i = 0; i < D - 3; i++) {
-        const int o = dig[i];
-        const int sl = sCS[o], pv = sP[i * K + o];
+      for (int k = 0; k < S; k++) cb[k] = 0;
+      for (int i = 0; i < ND; i++) {
+        const int oo = dig[i];
+        const int sl = sCS[oo], pv = sP[i * K + oo];
 #pragma unroll
-        for (int s = 0; s < S; s++) cb[s] += (sl == s) ? pv : 0;
+        for (int k = 0; k < S; k++) cb[k] += (sl == k) ? pv : 0;
       }
 #pragma unroll
-      for (int s = 0; s < S; s++) sCapsB[s][threadIdx.x] = cb[s];
+      for (int k = 0; k < S; k++) sCaps[k][threadIdx.x] = cb[k];
+      Fsum = 0;
+#pragma unroll
+      for (int q = 0; q < QM; q++) { st[q] = fam_from_smem(q); Fsum += st[q].F; }
     };
     rebuild();
     unsigned long long *gb = a.gbound + vec;
     for (;;) {
-      // grid-wide lower bound: the best score any thread of this vector has
-      // recorded so far (relaxed load, issued early; a stale value is only lower)
-      uint64_t G;
-      asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(G) : "l"(gb));
-      const int o3 = dig[D - 3];
-      const int sl3 = sCS[o3], p3 = sP[(D - 3) * K + o3];
-      int caps[S];
+      // the K blocks (o, o3) of this outer prefix
+      for (int o3 = 0; o3 < K; o3++) {
+        uint64_t G;  // best score any thread of this vector has recorded (relaxed; stale = lower)
+        asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(G) : "l"(gb));
+        const int s3 = sCS[o3];  // warp-uniform (-1: idle)
+        const int q3 = s3 >= 0 ? s3 / VM : -1;
+        FamState m;  // family q3 with device D-3's capacity added
+        if (q3 >= 0) {
+          int c[VM];
 #pragma unroll
-      for (int s = 0; s < S; s++) caps[s] = sCapsB[s][threadIdx.x] + (sl3 == s ? p3 : 0);
-      uint64_t Fq[QM];
-      uint64_t base = 0;
+          for (int j = 0; j < VM; j++) c[j] = sCaps[q3 * VM + j][threadIdx.x] + (q3 * VM + j == s3 ? sP[(D - 3) * K + o3] : 0);
+          m = fam_state<QM, VM, SYM>(c, sDem[q3], a, q3);
+        }
+        uint64_t base = Fsum;
+        uint64_t mB1 = 0, mB2 = 0, mJ = 0;
+        int fB1 = -1;
 #pragma unroll
-      for (int q = 0; q < QM; q++) { Fq[q] = fill<QM, VM>(caps, a, sDem, q, -1, 0, -1, 0); base += Fq[q]; }
-      uint64_t Fb[S];
+        for (int q = 0; q < QM; q++) {
+          const bool mod = q == q3;
+          const uint64_t MBq = mod ? m.MB : st[q].MB, Jq = mod ? m.J : st[q].J;
+          if (mod) base = base - st[q].F + m.F;
+          mJ = Jq > mJ ? Jq : mJ;
+          if (MBq > mB1) { mB2 = mB1; mB1 = MBq; fB1 = q; }
+          else if (MBq > mB2) mB2 = MBq;
+        }
+        uint64_t dmax = mJ > mB1 ? mJ : mB1;  // J covers both-in-one-family; (idle, b) rows: mB1
 #pragma unroll
-      for (int s = 0; s < S; s++) Fb[s] = fill<QM, VM>(caps, a, sDem, s / VM, s % VM, a.PB[s], -1, 0) - Fq[s / VM];
-      // The K^2 candidates of this prefix, one row per option of device D-2
-      // (idle first).  Fast path per row: a candidate of another family than
-      // the row's scores ba + Fb[sb] (Fb >= 0), so the row holds one above the
-      // running best lb iff the largest such Fb exceeds lb - ba (M1 / M2
-      // below: one compare for all of them); a same-family candidate is
-      // scored through its joint water-fill.  The compares only flag the row.  A flagged row (it holds a better
-      // candidate) is re-scanned in index order with strict >, so the first
-      // (lowest-index) maximum is kept.  If lb < ba the row's first candidate
-      // (sa, idle) = ba already flags the row, so the unsigned threshold never
-      // matters when it wraps.  Pad slots (code 0, capacity 0) score exactly
-      // like the idle option with the same index and never change the result.
-      // Largest delta of device D-1 over all its options (M1, family fm1) and
-      // over the options outside family fm1 (M2): a row of family qa holds an
-      // other-family candidate above lb iff (qa == fm1 ? M2 : M1) > lb - ba.
-      uint64_t M1 = 0, M2 = 0;
-      int fm1 = -1;
+        for (int q = 0; q < QM; q++) {
+          const uint64_t MAq = q == q3 ? m.MA : st[q].MA;
+          const uint64_t v = MAq + (q == fB1 ? mB2 : mB1);  // (a in q, b outside q or idle)
+          dmax = v > dmax ? v : dmax;
+        }
+        const uint64_t Mx = base + dmax;
+        // threshold: the thread's best so far (strict >: the first maximum is
+        // kept), raised to G - 1 (nothing below the score G of a real
+        // candidate can win; ties with G still record, reading C9)
+        bool take;
+        if (!rec) take = G == 0 || Mx > G - 1;
+        else take = Mx > best_s && (G == 0 || Mx > G - 1);
+        if (take) {
+          uint64_t Fq[QM];
 #pragma unroll
-      for (int q = 0; q < QM; q++) {
-        uint64_t mq = Fb[q * VM];
-#pragma unroll
-        for (int j = 1; j < VM; j++) mq = Fb[q * VM + j] > mq ? Fb[q * VM + j] : mq;
-        if (mq > M1) { M2 = M1; M1 = mq; fm1 = q; }
-        else if (mq > M2) M2 = mq;
-      }
-      uint64_t lb = best_s;
-      int lp = -1;
-      if (best_i == ~0ull) { lb = base; lp = 0; }  // the thread's first candidate
-      // Candidates below G cannot be the answer (G is the score of a real
-      // candidate), so the threshold is raised to G - 1: the rows still flag
-      // every candidate >= G (ties with G keep the lowest index), and the thread
-      // that holds the first maximum records it -- its score M >= G always
-      // exceeds the threshold until the thread has recorded M.  A thread that
-      // records nothing reports (0, ~0), the neutral element of the argmax.
-      if (G > 0 && G - 1 > lb) { lb = G - 1; lp = -1; }
-      {
-        const uint64_t thr = lb - base;
-        if (base > lb || M1 > thr) {
-          if (base > lb) { lb = base; lp = 0; }
-#pragma unroll
-          for (int sb = 0; sb < S; sb++)
-            if (base + Fb[sb] > lb) { lb = base + Fb[sb]; lp = a.code[sb]; }
+          for (int q = 0; q < QM; q++) Fq[q] = q == q3 ? m.F : st[q].F;
+          const int lp = flat_rescan<QM, VM>(a, &sCaps[0][0], sDem, s3, s3 >= 0 ? sP[(D - 3) * K + o3] : 0, base,
+                                             Fq, Mx);
+          best_s = Mx;
+          best_i = o * K3 + (uint64_t)o3 * K2 + (uint64_t)(lp < 0 ? 0 : lp);
+          rec = true;
+          if (Mx > G) atomicMax(gb, (unsigned long long)Mx);
         }
       }
-#pragma unroll
-      for (int sa = 0; sa < S; sa++) {
-        const int qa = sa / VM;
-        const uint64_t ba = base + fill<QM, VM>(caps, a, sDem, qa, sa % VM, a.PA[sa], -1, 0) - Fq[qa];
-        uint64_t jv[VM];  // same-family candidates (joint fills)
-#pragma unroll
-        for (int jb = 0; jb < VM; jb++)
-          jv[jb] = base - Fq[qa] + fill<QM, VM>(caps, a, sDem, qa, sa % VM, a.PA[sa], jb, a.PB[qa * VM + jb]);
-        const uint64_t thr = lb - ba;
-        bool f0 = ba > lb || (qa == fm1 ? M2 : M1) > thr;
-#pragma unroll
-        for (int jb = 0; jb < VM; jb++) f0 |= jv[jb] > lb;
-        if (f0) {
-          if (ba > lb) { lb = ba; lp = a.code[sa] * K; }
-#pragma unroll
-          for (int sb = 0; sb < S; sb++) {
-            const uint64_t c = (qa == sb / VM) ? jv[sb % VM] : ba + Fb[sb];
-            if (c > lb) { lb = c; lp = a.code[sa] * K + a.code[sb]; }
-          }
-        }
-      }
-      if (lp >= 0) {
-        best_s = lb;
-        best_i = p * KK + (uint64_t)lp;
-        if (lb > G) atomicMax(gb, (unsigned long long)lb);
-      }
-      if (++p >= pend) break;
-      if (++dig[D - 3] == K) {
-        dig[D - 3] = 0;
-        for (int i = D - 4; i >= 0; i--) {
+      if (++o >= oend) break;
+      if (ND == 0) break;
+      // next outer prefix: device D-4 advances (one or two families change)
+      const int i4 = ND - 1;
+      const int old = dig[i4];
+      if (++dig[i4] == K) {
+        dig[i4] = 0;
+        for (int i = i4 - 1; i >= 0; i--) {
           if (++dig[i] < K) break;
           dig[i] = 0;
         }
         rebuild();
+      } else {
+        const int s_old = sCS[old], s_new = sCS[old + 1];
+        if (s_old >= 0) sCaps[s_old][threadIdx.x] -= sP[i4 * K + old];
+        sCaps[s_new][threadIdx.x] += sP[i4 * K + old + 1];
+        const int q_old = s_old >= 0 ? s_old / VM : -1, q_new = s_new / VM;
+#pragma unroll
+        for (int q = 0; q < QM; q++)
+          if (q == q_old || q == q_new) {
+            Fsum -= st[q].F;
+            st[q] = fam_from_smem(q);
+            Fsum += st[q].F;
+          }
       }
     }
   }
   block_best(best_s, best_i);
   if (threadIdx.x == 0) {
-    BestRec &o = a.out[(int64_t)vec * a.out_stride + blk];
-    o.score = best_s;
-    o.index = best_i;
+    BestRec &r = a.out[(int64_t)vec * a.out_stride + (int64_t)chunk];
+    r.score = best_s;
+    r.index = best_i;
+  }
+  __syncthreads();  // sItem / sDem / block_best's shared arrays are rewritten by the next item
   }
 }
 
@@ -437,8 +557,18 @@ __global__ void k_materialize_enum(const __grid_constant__ EnumArgs a, const Bes
 }
 
 // ------------------------------------------------------------- host -----
+int px_occupancy(proteus_ctx *ctx, const void *kern, int threads, size_t smem, int *occ) {
+  // per context and device: cached by (kernel, shared memory)
+  for (auto &e : ctx->occ_cache)
+    if (e.first.first == kern && e.first.second == smem) { *occ = e.second; return 0; }
+  PX_CUDA(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(occ, kern, threads, smem));
+  ctx->occ_cache.push_back({{kern, smem}, *occ});
+  return 0;
+}
+
+// o_lo, o_hi: outer prefixes (devices 0..D-4) of this slice
 template <int QM, int VM>
-static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p_hi, const int32_t *dev_type,
+static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t o_lo, uint64_t o_hi, const int32_t *dev_type,
                        const int32_t *demand, int nvec, const std::vector<int32_t> &h_P,
                        const std::vector<int32_t> &h_slot_code, const Tables &tab, BestRec *d_blocks,
                        int64_t out_stride, unsigned long long *gbound, int *nblocks_out) {
@@ -461,36 +591,40 @@ static int launch_flat(proteus_ctx *ctx, int D, int K, uint64_t p_lo, uint64_t p
   a.code_slot = tab.code_slot;
   a.out = d_blocks;
   a.gbound = gbound;
-  PX_CUDA(ctx, cudaMemsetAsync(gbound, 0, sizeof(unsigned long long) * (size_t)nvec, ctx->stream));
   const size_t smem = (size_t)(D * K + K) * 4;
-  auto kern = k_flat_pair<QM, VM>;
+  bool sym = true;  // devices D-2 and D-1 of one type: the symmetric family states
+  for (int s = 0; s < QM * VM; s++) sym &= a.PA[s] == a.PB[s];
+  auto kern = sym ? k_flat_fam<QM, VM, true> : k_flat_fam<QM, VM, false>;
   if (smem > 48 * 1024) PX_CUDA(ctx, cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   int nsm = 0, occ = 0;
   PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
-  {  // occupancy per (instantiation, shared-memory size), queried once
-    static size_t occ_smem = ~(size_t)0;
-    static int occ_val = 0;
-    if (occ_smem != smem) {
-      PX_CUDA(ctx, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_val, kern, FLAT_THREADS, smem));
-      occ_smem = smem;
-    }
-    occ = occ_val;
-  }
+  int rc = px_occupancy(ctx, (const void *)kern, FLAT_THREADS, smem, &occ);
+  if (rc) return rc;
   if (occ < 1) occ = 1;
-  const uint64_t np = p_hi - p_lo;
+  const uint64_t np = o_hi - o_lo;
+  // work items of FLAT_THREADS threads x per_thread outer prefixes; per_thread
+  // a multiple of K (o_lo is one too, px_solve_enum), so every thread's
+  // device D-4 digit carries in the same iteration
+  a.o_lo = o_lo; a.o_hi = o_hi;
+  a.nvec = nvec;
+  uint64_t pt = (uint64_t)K * FLAT_RK;
+  const uint64_t per_vec_threads = (np + pt - 1) / pt;
+  if (per_vec_threads * nvec < (uint64_t)nsm * occ * FLAT_THREADS) {  // small spaces: finer items
+    pt = (np * nvec + (uint64_t)nsm * occ * FLAT_THREADS - 1) / ((uint64_t)nsm * occ * FLAT_THREADS);
+    if (pt < 1) pt = 1;
+  }
+  a.per_thread = pt;
+  const uint64_t span = pt * FLAT_THREADS;
+  const uint64_t items_per_vec = (np + span - 1) / span;
+  if (items_per_vec > (uint64_t)out_stride) return px_fail(ctx, PROTEUS_EINTERNAL, "flat: %llu work items per vector",
+                                                           (unsigned long long)items_per_vec);
+  a.n_items = items_per_vec * nvec;
+  a.counter = gbound + nvec;
+  PX_CUDA(ctx, cudaMemsetAsync(gbound, 0, sizeof(unsigned long long) * ((size_t)nvec + 1), ctx->stream));
   uint64_t nb = (uint64_t)nsm * occ;
-  const uint64_t need = (np + FLAT_THREADS - 1) / FLAT_THREADS;
-  if (need < nb) nb = need ? need : 1;
-  a.p_lo = p_lo; a.p_hi = p_hi;
-  a.per_thread = (np + nb * FLAT_THREADS - 1) / (nb * FLAT_THREADS);
-  if (a.per_thread == 0) a.per_thread = 1;
-  // a multiple of K: every thread's prefix counter then carries (and rebuilds
-  // the capacities of devices 0..D-4) in the same iteration -- no divergence
-  if (a.per_thread > (uint64_t)K) a.per_thread = (a.per_thread + K - 1) / K * K;
-  nb = (np + a.per_thread * FLAT_THREADS - 1) / (a.per_thread * FLAT_THREADS);
-  if (nb == 0) nb = 1;
-  PX_LAUNCH(ctx, "score_flat_pair", kern, dim3((unsigned)nvec, (unsigned)nb), FLAT_THREADS, smem, a);
-  *nblocks_out = (int)nb;
+  if (nb > a.n_items) nb = a.n_items;
+  PX_LAUNCH(ctx, "score_flat_pair", kern, (unsigned)nb, FLAT_THREADS, smem, a);
+  *nblocks_out = (int)items_per_vec;
   return 0;
 }
 
@@ -571,7 +705,7 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
   const int64_t stride = (int64_t)max_blocks + 1;
   const int nv = materialize_only ? 1 : vec_hi - vec_lo;
   // per-block winners, then one grid-wide bound per vector (flat kernel)
-  BestRec *d_blocks0 = (BestRec *)px_buf(ctx, B_BEST, sizeof(BestRec) * (size_t)stride * nv + 8 * (size_t)nv);
+  BestRec *d_blocks0 = (BestRec *)px_buf(ctx, B_BEST, sizeof(BestRec) * (size_t)stride * nv + 8 * ((size_t)nv + 1));
   if (!d_blocks0) return px_fail(ctx, PROTEUS_ENOMEM, "block results");
   uint64_t ncand_all = 0;
   int nb_all = 0, flat_nb = 0;
@@ -585,9 +719,19 @@ int px_solve_enum(proteus_ctx *ctx, const proteus_solve_args *args, const int32_
     if (!materialize_only) {
       int nb = 0;
       if (flat_ok) {
-        const uint64_t NP = N / ((uint64_t)K * K);
-        const uint64_t plo = mul_div(NP, rank, world), phi = mul_div(NP, rank + 1, world);
-        ncand = (phi - plo) * (uint64_t)K * K;
+        // outer prefixes (devices 0..D-4), K^3 candidates each; rank slices
+        // start on a multiple of K when there are enough
+        const uint64_t K3 = (uint64_t)K * K * K;
+        const uint64_t NO = N / K3;
+        uint64_t plo, phi;
+        if (NO % (uint64_t)K == 0 && NO / K >= (uint64_t)world) {
+          plo = mul_div(NO / K, rank, world) * K;
+          phi = mul_div(NO / K, rank + 1, world) * K;
+        } else {
+          plo = mul_div(NO, rank, world);
+          phi = mul_div(NO, rank + 1, world);
+        }
+        ncand = (phi - plo) * K3;
         if ((v - vec_lo) % FLAT_NV == 0) {  // one launch per FLAT_NV vectors (grid.x = vector)
           const int nvec = vec_hi - v < FLAT_NV ? vec_hi - v : FLAT_NV;
           const FlatInst *f = pick_flat(Q, *std::max_element(ctx->V.begin(), ctx->V.end()));

@@ -67,7 +67,7 @@ a, b = both(lambda: px.pareto(pdev, c3["cluster"].slo_us, 3))
 same(a, b, "pareto")
 sol = px.solve(c3["cluster"].device_type, c3["cluster"].slo_us, c3["demand"][:1], mode=2)[0]
 arr, fam = W.query_trace(20000, 3000.0, c3["weights"], 5, "gamma")
-sc = np.concatenate([W.scenarios_64(0)[::7], W.scenarios_64(0, 1)[::16], W.scenarios_64(0, 2)[::16]])
+sc = np.concatenate([W.scenarios_64(0, 0)[::7], W.scenarios_64(0, 1)[::16], W.scenarios_64(0, 2)[::16]])
 a, b = both(lambda: px.replay(arr, fam, sol.option, sol.z, c3["cluster"].device_type, c3["demand"][0],
                               c3["cluster"].slo_us, sc))
 same(a, b, "replay")
