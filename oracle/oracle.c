@@ -935,7 +935,13 @@ int orc_replay_device_aimd(int64_t n, const uint32_t *a, const int32_t *Tproc, i
  * depth), routing (0 = SWRR over z with the unmet demand to the sink, 1 =
  * uniform over the hosting devices that fit batch 1, no sink), policy (0 = §5
  * adaptive batching, 1 = Nexus early drop, 2 = Clipper AIMD; §8(f2)).
- * SLO_q(s) = floor(mult * slo_base[q] / 1000) (R12); Bmax = min(cap, depth).
+ * SLO_q(s) = floor(mult * slo_base[q] / 1000) (R12).  Reading R4' (P:918-936:
+ * "the maximum allowed batch size is the minimum of (i) the maximum batch size
+ * that meets SLO, (ii) the maximum batch size that fits in the memory of d",
+ * with (i) the half-SLO rule of P:920-926): the §5 policy batches at most
+ * Bmax = the largest b <= min(cap, depth) with 2 T(b) <= SLO, at least 1 --
+ * the same size as the Nexus baseline's (R14) and as the capacity estimate's
+ * b*; Clipper AIMD grows its own limit up to min(cap, depth) (R15).
  * Outputs per scenario: violations (latency > SLO, R6, plus dropped), on_time,
  * acc_sum (sum of the serving variant's accuracy over on-time queries, R9);
  * latency[s][i] if non-NULL (UINT32_MAX = dropped). */
@@ -974,6 +980,8 @@ static void *rep_worker(void *arg) {
       int cap = c->sc[s * 4 + 1];
       int Bmax = (cap > 0 && cap < dep) ? cap : dep;
       int64_t L = (int64_t)c->sc[s * 4 + 0] * c->slo_base[q] / 1000;
+      int Bhalf = 1;  /* the maximum allowed batch size (R4', R14) */
+      for (int b = 1; b <= Bmax && b <= 1024; b++) if (2LL * row[b - 1] <= L) Bhalf = b;
       int64_t n = en - st;
       uint32_t *a = (uint32_t *)malloc(sizeof(uint32_t) * n), *l = (uint32_t *)malloc(sizeof(uint32_t) * n);
       for (int64_t k = 0; k < n; k++) a[k] = c->arr[c->idx_of_dev[rt][st + k]];
@@ -982,13 +990,11 @@ static void *rep_worker(void *arg) {
       for (int b = 1; b <= Bmax && b <= 1024; b++) Tp[b] = row[b - 1];
       const int policy = c->sc[s * 4 + 3];
       if (policy == 1) {          /* Nexus: batch size by the capacity rule (R14) */
-        int B = 1;
-        for (int b = 1; b <= Bmax && b <= 1024; b++) if (2LL * Tp[b] <= L) B = b;
-        orc_replay_device_nexus(n, a, Tp, B, L, l);
+        orc_replay_device_nexus(n, a, Tp, Bhalf, L, l);
       } else if (policy == 2) {
         orc_replay_device_aimd(n, a, Tp, Bmax, L, l);
-      } else {
-        orc_replay_device(n, a, Tp, Bmax, L, l);
+      } else {                    /* §5 with the maximum allowed batch size (R4') */
+        orc_replay_device(n, a, Tp, Bhalf, L, l);
       }
       for (int64_t k = 0; k < n; k++) {
         if ((int64_t)l[k] > L) viol++;
@@ -1198,8 +1204,10 @@ int orc_replay_epochs(int64_t N, const uint32_t *arrival, const uint8_t *family,
         while (dep < bmax && tr[dep] > 0) dep++;
         for (int b = 1; b <= dep; b++) row[b] = tr[b - 1];
         const int cap = sc[s * 4 + 1];
-        Bm[e] = (cap > 0 && cap < dep) ? cap : dep;
+        const int Bcap = (cap > 0 && cap < dep) ? cap : dep;
         Lv[e] = (int64_t)sc[s * 4 + 0] * slo_base[fam_m[o - 1]] / 1000;
+        Bm[e] = 1;  /* the maximum allowed batch size of the epoch's variant (R4') */
+        for (int b = 1; b <= Bcap && b <= 1024; b++) if (2LL * row[b] <= Lv[e]) Bm[e] = b;
       }
       if (orc_replay_device_epochs(n, a, eq, Tp, Bm, Lv, l) != 0) {
         free(fam_m); free(ep); free(target); free(a); free(l); free(eq); free(idx); free(Tp); free(Tbuf);

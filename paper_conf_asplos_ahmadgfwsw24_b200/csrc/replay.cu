@@ -255,11 +255,12 @@ struct ChunkSt {
 };
 
 struct LaneParam {  // per (scenario, device)
-  int32_t Bmax;     // min(cap, depth) (R4); 0 for idle devices
+  int32_t Bmax;     // §5: the maximum allowed batch size (R4'); AIMD: min(cap, depth); 0 for idle devices
   uint32_t A;       // accuracy of the hosted variant
   int64_t L;        // scenario SLO of the hosted family (R12)
   int32_t policy;   // 0 §5, 1 Nexus early drop, 2 Clipper AIMD (§8(f2))
   int32_t Bn;       // Nexus batch size: largest b <= Bmax with 2 T(b) <= L, at least 1 (R14)
+  int32_t mono;     // T(b) non-decreasing over b = 1..Bmax (binary-search decisions)
 };
 
 __global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__restrict__ option,
@@ -270,7 +271,7 @@ __global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__re
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= S * D) return;
   const int s = i / D, d = i % D;
-  LaneParam p = {0, 0, 0, sc[s].policy, 0};
+  LaneParam p = {0, 0, 0, sc[s].policy, 0, 0};
   const int o = option[d];
   if (o > 0) {
     const int32_t *T = lat + ((size_t)dev_type[d] * M + (o - 1)) * bmax;
@@ -280,9 +281,13 @@ __global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__re
     p.Bmax = (cap > 0 && cap < depth) ? cap : depth;
     p.A = (uint32_t)acc[o - 1];
     p.L = (int64_t)sc[s].slo_mult_milli * slo_base[fam_of_m[o - 1]] / 1000;
-    p.Bn = 1;
+    p.Bn = 1;  // the maximum allowed batch size: largest b <= min(cap, depth), 2 T(b) <= SLO
     for (int b = 1; b <= p.Bmax; b++)
       if (2 * (int64_t)T[b - 1] <= p.L) p.Bn = b;
+    if (p.policy == 0) p.Bmax = p.Bn;  // §5 batches at most that (reading R4')
+    p.mono = 1;
+    for (int b = 1; b < p.Bmax; b++)
+      if (T[b] < T[b - 1]) p.mono = 0;
   }
   lp[i] = p;
 }
@@ -348,6 +353,59 @@ __device__ __forceinline__ int decide(const Arr &arr, int64_t n, int64_t h, int6
   }
   *t_out = t;
   return b;
+}
+
+// idle decision at head h (fact (ii)); T[b-1] = T(b); n = the device's size
+template <class Arr>
+__device__ __forceinline__ int idle_decide(const Arr &A, int64_t n, int64_t h, int Bmax, int64_t L,
+                                           const int32_t *T, bool mono, int64_t *t_out) {
+  if (!mono) return decide(A, n, h, (int64_t)0, Bmax, L, T, t_out);
+  const int64_t ah = A(h);
+  int q0 = 1;
+  while (q0 < Bmax && h + q0 < n && (int64_t)A(h + q0) <= ah) q0++;  // R3: simultaneous arrivals
+  if (q0 >= Bmax) { *t_out = ah; return Bmax; }
+  // first q in [q0, Bmax) whose stop test holds (monotone), Bmax if none
+  int lo = q0, hi = Bmax;
+  while (lo < hi) {
+    const int q = (lo + hi) >> 1;
+    const int64_t W = ah + L - T[q];
+    const int64_t nxt = h + q < n ? (int64_t)A(h + q) : INT64_MAX;
+    const bool stop = nxt > W || (int64_t)A(h + q - 1) >= W;
+    if (stop) hi = q; else lo = q + 1;
+  }
+  int q = lo;
+  while (q < Bmax && h + q < n && A(h + q) == A(h + q - 1)) q++;  // first stable count
+  if (q >= Bmax) { *t_out = A(h + Bmax - 1); return Bmax; }      // R4: Bmax queued at that instant
+  const int64_t W = ah + L - T[q];
+  const int64_t tq = A(h + q - 1);
+  *t_out = tq >= W ? tq : W;
+  return q;
+}
+
+// #{j in [h, min(n, h + Bmax)) : A(j) <= F} by binary search (>= 1 when A(h) <= F)
+template <class Arr>
+__device__ __forceinline__ int count_upto(const Arr &A, int64_t n, int64_t h, int Bmax, int64_t F) {
+  int lo = 0, hi = (int)(n - h < Bmax ? n - h : Bmax);
+  while (lo < hi) {
+    const int m = (lo + hi + 1) >> 1;
+    if ((int64_t)A(h + m - 1) <= F) lo = m; else hi = m - 1;
+  }
+  return lo;
+}
+
+// one decision from head h with the device free at F (the rule R1-R5 in the
+// form of facts (i)-(ii) of the window path, below): the idle decision by
+// binary search, or, when the device frees after it would have dispatched,
+// the greedy batch min(Bmax, queued at F) at F.  Same result as decide().
+template <class Arr>
+__device__ __forceinline__ int fast_decide(const Arr &A, int64_t n, int64_t h, int64_t F, int Bmax, int64_t L,
+                                           const int32_t *T, bool mono, int64_t *t_out) {
+  if (!mono) return decide(A, n, h, F, Bmax, L, T, t_out);
+  int64_t t;
+  const int b = idle_decide(A, n, h, Bmax, L, T, true, &t);
+  if (F <= t) { *t_out = t; return b; }
+  *t_out = F;
+  return count_upto(A, n, h, Bmax, F);
 }
 
 struct GArr {
@@ -747,6 +805,8 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
     while (h < en) {
       if (!entered && h >= st) { entered = true; edh = h - st; eF = F; }
       int64_t t;
+      // linear scan (decide): the arrivals stream through L1; binary-search probes
+      // (fast_decide) measured slower here (c5 k_spec 8.1 -> 10.0 ms)
       const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
       if (entered) { nfull += b == p.Bmax && t == F; ndec++; }
       const int64_t Fn = t + T[b - 1];
@@ -1856,6 +1916,7 @@ __global__ void __launch_bounds__(256) k_unpermute(int64_t N, int64_t NS, int S,
   }
   for (int s = 0; s < S; s++) {
     const size_t r = (size_t)s * N, rs = (size_t)s * NS;
+    if (rt[s] < 0) continue;  // written by the window path
     const bool m1 = rt[s] != 0;
     uint32_t v[UNP_PER];
 #pragma unroll
@@ -1864,6 +1925,551 @@ __global__ void __launch_bounds__(256) k_unpermute(int64_t N, int64_t NS, int S,
 #pragma unroll
     for (int k = 0; k < UNP_PER; k++)
       if (i0 + 256 * k < N) out[r + i0 + 256 * k] = v[k];
+  }
+}
+
+// ======================================================= window path ======
+// The §5 lanes as three data-parallel passes over GLOBAL WINDOWS of WT tiles
+// (TQ = WT * TILE queries; chunk (d, k) = device d's positions of window k,
+// [cb[k][d], cb[k+1][d]) from the routing's per-tile bases).  It rests on
+// three facts about the rule (readings R1-R5, R4'):
+//  (i)   from head h with the device free at F, the decision is the one from
+//        an idle device (F <= a_h) iff F <= t_idle(h), the idle decision's
+//        dispatch time (the busy run sees the same queue states once t passes
+//        F); otherwise the queue is already past the idle decision when the
+//        device frees, so the batch leaves at F with min(Bmax, #{j >= h :
+//        a_j <= F}) queries ("greedy");
+//  (ii)  the idle decision is a binary search: with T non-decreasing, the stop
+//        test of queue size q -- the next arrival a_{h+q} comes after
+//        W(q) = a_h + L - T(q+1), or the queue's last arrival a_{h+q-1} is at
+//        or past it -- is monotone in q; the batch is the first stable count
+//        (next arrival strictly later) at or after the first q that stops,
+//        leaving at max(a_{h+q-1}, W(q));
+//  (iii) whenever a_{h+Bmax-1} <= F, Bmax queries are queued when the device
+//        frees and a full batch leaves at F (R4), whatever the branch: a
+//        backlogged stretch from (h, F) is m full batches, F + m T(Bmax), iff
+//        F >= max_k a_{h+(k+1)Bmax-1} - k T(Bmax) (max-plus).
+// A chain entered on the idle branch at head e is a function of e alone, and
+// the first head of the true run in chunk k lies in [c0, c0 + Bmax).  So:
+//   k_win_tables   block per chunk (d, k), arrivals staged in shared memory,
+//                  a warp per scenario lane: per entry offset o < min(Bmax,
+//                  chunk) the idle-branch chain to its first head >= c1
+//                  (chains reaching a head another chain took on the idle
+//                  branch merge into it) and the backlog threshold of (iii);
+//                  Bmax = 1: the max-plus form F_out = max(F_in + m T(1),
+//                  max_i a_i + (c1 - i) T(1));
+//   k_win_compose  warp per lane: the true state across the chunks -- one hop
+//                  per chunk when the entry is on the idle branch or the whole
+//                  chunk is backlogged, else the rule walked to the chunk end
+//                  (32 idle decisions per step, in parallel);
+//   k_win_write    block per (scenario, window), arrivals staged in shared
+//                  memory: every device's chunk replayed from its true entry
+//                  state, latencies into a shared-memory tile in device order,
+//                  written ONCE in query order with the per-scenario counts
+//                  folded in (a13) -- no device-major latency rows, no
+//                  un-permute pass.
+// Lanes with Bmax <= WIN_EMAX take this path; a lane whose T is not
+// non-decreasing in b (the table need not be, reading C6) makes its idle
+// decisions linear (decide()).
+#define WIN_EMAX 64
+#define WIN_EXT (2 * WIN_EMAX + 64)  // arrivals staged past a chunk's end (look-ahead of its decisions)
+#define WIN_WARPS 8
+
+struct WinRec {     // chain of one entry offset o of one chunk (times relative to a_{c0})
+  int64_t Fx;       // free time after the batch that crosses c1 (absolute; Bmax = 1: R of the max-plus form)
+  int32_t tdisp;    // idle dispatch time at the entry head c0 + o, - a_{c0}
+  int32_t R;        // backlog threshold of (iii) through the chunk, - a_{c0} (INT32_MAX: none)
+  int32_t hx;       // first head >= c1 of the chain, - c0
+  int32_t pad;
+};
+struct WinEntry {   // true state at a chunk start: first head >= c0 (device-relative), free time
+  int64_t F;
+  int32_t h, pad;
+};
+
+struct WinArgs {
+  int S, D, M, bmax, nsc, WT, D1;
+  int64_t N, nw, ntiles;
+  const int32_t *option, *dev_type, *lat, *sc_list;
+  const LaneParam *lp;
+  const uint8_t *mono;         // [S * D] T non-decreasing over 1..Bmax
+  const int64_t *devOff;       // [D + 2]
+  const int32_t *dbase;        // [(ntiles + 1)][D + 1] per-tile bases (device-relative)
+  const uint32_t *devArr, *inv;
+  const uint8_t *tgt;
+  const int64_t *recoff;       // [nsc * D] offset of the lane's WinRec rows (E per chunk)
+  const int32_t *E;            // [nsc * D] entry offsets per chunk of the lane (min(Bmax, 64); 0 = no lane)
+  WinRec *rec;
+  WinEntry *ent;               // [nsc * D][nw]
+  uint32_t *out;               // [S][N] or null
+  uint64_t *agg;               // [3][S]
+  unsigned long long *dbg;     // [nsc * D][4] (PROTEUS_REPLAY_DEBUG): idle hops, backlog hops, walks, walked batches
+};
+
+__device__ __forceinline__ int64_t win_cb(const WinArgs &a, int64_t k, int d) {
+  const int64_t t = k * a.WT < a.ntiles ? k * a.WT : a.ntiles;
+  return a.dbase[t * a.D1 + d];
+}
+
+// arrivals of one device: positions [lo, lo + len) from shared memory, the rest from global
+struct SArr {
+  const uint32_t *s, *g;
+  int64_t lo, len;
+  __device__ __forceinline__ uint32_t operator()(int64_t j) const {
+    const int64_t r = j - lo;
+    return (r >= 0 && r < len) ? s[r] : __ldg(g + j);
+  }
+};
+
+__device__ __forceinline__ int32_t clamp_rel(int64_t v) {  // upward clamp keeps "F <= tdisp" / "F >= R" tests safe
+  return v > (int64_t)INT32_MAX ? INT32_MAX : (v < -(int64_t)(1 << 30) ? -(1 << 30) : (int32_t)v);
+}
+
+// ---- pass 1: chunk tables, block per chunk (d, k), warp per scenario lane
+__global__ void __launch_bounds__(WIN_WARPS * 32) k_win_tables(const __grid_constant__ WinArgs a) {
+  extern __shared__ __align__(16) uint8_t win_sm[];  // [TQ + WIN_EXT] arrivals, then [WIN_WARPS][TQ] marks
+  __shared__ int32_t sT[WIN_WARPS][WIN_EMAX];
+  __shared__ int64_t exF[WIN_WARPS][WIN_EMAX];
+  __shared__ int32_t exH[WIN_WARPS][WIN_EMAX], mg[WIN_WARPS][WIN_EMAX];
+  __shared__ int64_t tdE[WIN_WARPS][WIN_EMAX];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int d = blockIdx.x % a.D;
+  const int64_t k = blockIdx.x / a.D;
+  const int64_t c0 = win_cb(a, k, d), c1 = win_cb(a, k + 1, d);
+  if (c1 <= c0) return;
+  const int64_t TQ = (int64_t)a.WT * TILE;
+  const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+  uint32_t *sarr = (uint32_t *)win_sm;
+  const int64_t slen = (c1 + WIN_EXT < n ? c1 + WIN_EXT : n) - c0;
+  for (int64_t i = threadIdx.x; i < slen; i += blockDim.x) sarr[i] = __ldg(a.devArr + off + c0 + i);
+  __syncthreads();
+  SArr A{sarr, a.devArr + off, c0, slen};
+  volatile uint8_t *vis = win_sm + (TQ + WIN_EXT) * 4 + (size_t)w * TQ;
+  const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  const int64_t len = c1 - c0;  // <= TQ
+  const int64_t a0 = A(c0);
+  for (int si = w; si < a.nsc; si += WIN_WARPS) {
+    const int li = si * a.D + d;
+    const int E = a.E[li];
+    if (E <= 0) continue;
+    const int s = a.sc_list[si];
+    const LaneParam p = a.lp[(size_t)s * a.D + d];
+    WinRec *R = a.rec + a.recoff[li] + k * (int64_t)E;
+    if (p.Bmax == 1) {  // max-plus form: R = max_i a_i + (c1 - i) T(1)
+      const int64_t T1 = Tg[0];
+      int64_t m = INT64_MIN;
+      for (int64_t i = c0 + lane; i < c1; i += 32) {
+        const int64_t v = (int64_t)A(i) + (c1 - i) * T1;
+        m = v > m ? v : m;
+      }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) {
+        const int64_t v = __shfl_xor_sync(0xffffffffu, m, o);
+        m = v > m ? v : m;
+      }
+      if (lane == 0) { WinRec r; r.Fx = m; r.tdisp = 0; r.R = 0; r.hx = (int32_t)len; r.pad = 0; R[0] = r; }
+      continue;
+    }
+    const int Bm = p.Bmax;
+    const bool mono = a.mono[(size_t)s * a.D + d] != 0;
+    for (int b = lane; b < Bm; b += 32) sT[w][b] = Tg[b];
+    for (int64_t i = lane; i < len; i += 32) vis[i] = 0xFF;
+    __syncwarp();
+    const int32_t *T = sT[w];
+    const int Ee = (int)(E < len ? E : len);
+    const int64_t TB = T[Bm - 1];
+    for (int r0 = 0; r0 < Ee; r0 += 32) {
+      const int o = r0 + lane;
+      bool live = o < Ee;
+      int64_t h = c0 + o, F = 0;
+      int merged = -1;
+      bool first = true;
+      while (__any_sync(0xffffffffu, live)) {
+        if (live) {
+          if (h >= c1) {
+            live = false;
+          } else {
+            int64_t t;
+            int b = idle_decide(A, n, h, Bm, p.L, T, mono, &t);
+            if (first) { tdE[w][o] = t; first = false; F = t; }  // the entry: idle branch by construction
+            if (F <= t) {  // idle branch (fact (i)): a function of h alone
+              const uint8_t mk = vis[h - c0];
+              if (mk != 0xFF && mk != (uint8_t)o) { merged = mk; live = false; }
+              else vis[h - c0] = (uint8_t)o;
+              if (live) { F = t + T[b - 1]; h += b; }
+            } else {  // greedy
+              b = count_upto(A, n, h, Bm, F);
+              F = F + T[b - 1];
+              h += b;
+            }
+          }
+        }
+      }
+      if (o < Ee) {
+        exH[w][o] = (int32_t)h; exF[w][o] = F; mg[w][o] = merged;
+        // backlog threshold (fact (iii)) from the entry head: full batches to the first head >= c1
+        int64_t Rb = INT64_MIN;
+        bool ok = true;
+        int64_t kk = 0;
+        for (int64_t hh = c0 + o; hh < c1; hh += Bm, kk++) {
+          if (hh + Bm - 1 >= n) { ok = false; break; }  // the trace ends: no full batch
+          const int64_t v = (int64_t)A(hh + Bm - 1) - kk * TB;
+          Rb = v > Rb ? v : Rb;
+        }
+        tdE[w][o] = tdE[w][o] - a0;
+        exF[w][o] = F;
+        R[o].R = ok ? clamp_rel(Rb - a0) : INT32_MAX;  // rest of the record below
+      }
+      __syncwarp();
+    }
+    // resolve merges (pointers strictly increase the stopping position: no cycles)
+    for (int o = lane; o < Ee; o += 32) {
+      int r = o;
+      while (mg[w][r] >= 0) r = mg[w][r];
+      R[o].Fx = exF[w][r];
+      R[o].hx = (int32_t)(exH[w][r] - c0);
+      R[o].tdisp = clamp_rel(tdE[w][o]);
+      R[o].pad = 0;
+    }
+    __syncwarp();
+  }
+}
+
+// ---- pass 2: the true state across the chunks, one warp per lane
+__global__ void __launch_bounds__(128) k_win_compose(const __grid_constant__ WinArgs a) {
+  __shared__ int32_t sT[4][WIN_EMAX];
+  __shared__ uint32_t sW[4][32 + WIN_EXT];  // a walk's arrivals
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int li = blockIdx.x * 4 + w;
+  if (li >= a.nsc * a.D) return;
+  const int d = li % a.D, s = a.sc_list[li / a.D];
+  const int E = a.E[li];
+  if (E <= 0) return;
+  const LaneParam p = a.lp[(size_t)s * a.D + d];
+  const int Bm = p.Bmax;
+  const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+  const uint32_t *G = a.devArr + off;
+  const bool mono = a.mono[(size_t)s * a.D + d] != 0;
+  const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  for (int b = lane; b < Bm; b += 32) sT[w][b] = Tg[b];
+  __syncwarp();
+  const int32_t *T = sT[w];
+  const int64_t TB = T[Bm - 1];
+  const WinRec *R = a.rec + a.recoff[li];
+  WinEntry *ent = a.ent + (int64_t)li * a.nw;
+  unsigned long long n_idle = 0, n_back = 0, n_walk = 0, n_wb = 0;
+  int64_t h = 0, F = 0;  // R13: idle at t = 0
+  // chunk bounds and first arrivals 32 chunks at a time; the next chunk's records prefetched
+  int64_t cb0 = 0, cb1 = 0, ca0 = 0;
+  WinRec r0 = {}, r1 = {}, q0 = {}, q1 = {};
+  auto load_row = [&](int64_t k, WinRec &x0, WinRec &x1) {
+    if (k < a.nw) {
+      if (lane < E) x0 = R[k * E + lane];
+      if (lane + 32 < E) x1 = R[k * E + lane + 32];
+    }
+  };
+  load_row(0, r0, r1);
+  for (int64_t k = 0; k < a.nw; k++) {
+    const int kk = (int)(k & 31);
+    if (kk == 0) {
+      cb0 = k + lane < a.nw ? win_cb(a, k + lane, d) : 0;
+      cb1 = k + lane < a.nw ? win_cb(a, k + lane + 1, d) : 0;
+      ca0 = (k + lane < a.nw && cb0 < cb1) ? (int64_t)__ldg(G + cb0) : 0;
+    }
+    load_row(k + 1, q0, q1);
+    const int64_t c0 = __shfl_sync(0xffffffffu, cb0, kk), c1 = __shfl_sync(0xffffffffu, cb1, kk);
+    const int64_t a0 = __shfl_sync(0xffffffffu, ca0, kk);
+    if (lane == 0) { WinEntry e; e.F = F; e.h = (int32_t)h; e.pad = 0; ent[k] = e; }
+    if (c1 > c0 && h < c1) {
+      if (Bm == 1) {
+        const int64_t Rk = __shfl_sync(0xffffffffu, r0.Fx, 0);
+        const int64_t v = F + (c1 - h) * (int64_t)T[0];
+        F = v > Rk ? v : Rk;
+        h = c1;
+      } else {
+        const int o = (int)(h - c0);  // < min(Bmax, chunk): the first head >= c0
+        const int src = o & 31;
+        const int64_t tdisp = a0 + __shfl_sync(0xffffffffu, o < 32 ? r0.tdisp : r1.tdisp, src);
+        const int32_t Rr = __shfl_sync(0xffffffffu, o < 32 ? r0.R : r1.R, src);
+        const int64_t Fx = __shfl_sync(0xffffffffu, o < 32 ? r0.Fx : r1.Fx, src);
+        const int32_t hx = __shfl_sync(0xffffffffu, o < 32 ? r0.hx : r1.hx, src);
+        if (F <= tdisp) {  // idle branch at the entry: the chain of the table
+          h = c0 + hx;
+          F = Fx;
+          n_idle++;
+        } else if (Rr != INT32_MAX && F >= a0 + Rr) {  // backlogged through the chunk (iii)
+          const int64_t m = (c1 - h + Bm - 1) / Bm;
+          h += m * Bm;
+          F += m * TB;
+          n_back++;
+        } else {  // the rule itself to the chunk end: 32 idle decisions per step, in parallel
+          n_walk++;
+          uint32_t *sw = sW[w];
+          while (h < c1) {
+            const int64_t base = h;
+            const int64_t wl = (n - base < 32 + WIN_EXT) ? n - base : 32 + WIN_EXT;
+            for (int i = lane; i < wl; i += 32) sw[i] = __ldg(G + base + i);
+            __syncwarp();
+            SArr A{sw, G, base, wl};
+            int64_t tl = 0;
+            int bl = 0;
+            if (base + lane < c1) bl = idle_decide(A, n, base + lane, Bm, p.L, T, mono, &tl);
+            while (h < c1 && h < base + 32) {
+              const int i = (int)(h - base);
+              int b = __shfl_sync(0xffffffffu, bl, i);
+              int64_t t = __shfl_sync(0xffffffffu, tl, i);
+              if (F > t) {  // greedy (fact (i))
+                b = count_upto(A, n, h, Bm, F);
+                t = F;
+              }
+              F = t + T[b - 1];
+              h += b;
+              n_wb++;
+            }
+            __syncwarp();
+          }
+        }
+      }
+    }
+    r0 = q0;
+    r1 = q1;
+  }
+  if (a.dbg && lane == 0) {
+    atomicAdd(a.dbg + 4 * li, n_idle);
+    atomicAdd(a.dbg + 4 * li + 1, n_back);
+    atomicAdd(a.dbg + 4 * li + 2, n_walk);
+    atomicAdd(a.dbg + 4 * li + 3, n_wb);
+  }
+}
+
+// ---- pass 3: latencies in query order, block per (scenario, window)
+#define WIN_THREADS 256
+__global__ void __launch_bounds__(WIN_THREADS) k_win_write(const __grid_constant__ WinArgs a) {
+  // dynamic: [TQ] latencies (device-major: wbase[d] + position - c0), then the
+  // arrivals of every device's chunk plus WIN_EXT look-ahead (abase[d] + position - c0)
+  extern __shared__ __align__(16) uint32_t wsm[];
+  __shared__ int32_t wbase[PX_MAXD + 2], abase[PX_MAXD + 2], wc0[PX_MAXD + 1], wlen[PX_MAXD + 1],
+      walen[PX_MAXD + 1], wown[PX_MAXD + 1];
+  __shared__ int64_t wL[PX_MAXD + 1];
+  __shared__ uint32_t wA[PX_MAXD + 1];
+  __shared__ int32_t sT[WIN_THREADS / 32][WIN_EMAX];
+  __shared__ unsigned long long red[3][WIN_THREADS / 32];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31, nwarps = WIN_THREADS / 32;
+  const int si = blockIdx.x;  // scenario list position (fastest: the window's inputs are shared in L2)
+  const int64_t k = blockIdx.y;
+  const int s = a.sc_list[si];
+  const int D = a.D;
+  const int64_t TQ = (int64_t)a.WT * TILE;
+  uint32_t *slat = wsm, *sarr = wsm + TQ;
+  if (threadIdx.x < D) {
+    const int d = threadIdx.x;
+    const int64_t c0 = win_cb(a, k, d), c1 = win_cb(a, k + 1, d);
+    const int64_t n = a.devOff[d + 1] - a.devOff[d];
+    wc0[d] = (int32_t)c0;
+    wlen[d] = (int32_t)(c1 - c0);
+    walen[d] = (int32_t)((c1 + WIN_EXT < n ? c1 + WIN_EXT : n) - c0);
+    const LaneParam q = a.lp[(size_t)s * D + d];
+    wL[d] = q.L;
+    wA[d] = q.A;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {  // tile layouts; devices to warps, largest chunk first (LPT)
+    int acc = 0, acc2 = 0;
+    for (int d = 0; d < D; d++) { wbase[d] = acc; acc += wlen[d]; abase[d] = acc2; acc2 += walen[d]; }
+    wbase[D] = acc;
+    abase[D] = acc2;
+    unsigned long long load[WIN_THREADS / 32];
+    for (int x = 0; x < nwarps; x++) load[x] = 0;
+    unsigned long long used = 0;
+    for (int it = 0; it < D; it++) {
+      int bd = -1;
+      for (int d = 0; d < D; d++)
+        if (!((used >> d) & 1ull) && (bd < 0 || wlen[d] > wlen[bd])) bd = d;
+      used |= 1ull << bd;
+      int bw = 0;
+      for (int x = 1; x < nwarps; x++) if (load[x] < load[bw]) bw = x;
+      wown[bd] = bw;
+      load[bw] += (unsigned long long)wlen[bd] + 64;
+    }
+  }
+  __syncthreads();
+  for (int d = 0; d < D; d++) {  // stage the arrivals (block-wide, coalesced)
+    const uint32_t *g = a.devArr + a.devOff[d] + wc0[d];
+    for (int i = threadIdx.x; i < walen[d]; i += WIN_THREADS) sarr[abase[d] + i] = __ldg(g + i);
+  }
+  __syncthreads();
+  for (int d = 0; d < D; d++) {
+    if (wown[d] != w || wlen[d] == 0) continue;
+    const int li = si * D + d;
+    const LaneParam p = a.lp[(size_t)s * D + d];
+    const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+    const int64_t c0 = wc0[d], c1 = c0 + wlen[d];
+    uint32_t *lt = slat + wbase[d];  // lt[position - c0]
+    SArr A{sarr + abase[d], a.devArr + off, c0, walen[d]};
+    if (p.Bmax < 1) {  // never routed to (kept for safety): dropped
+      for (int64_t j = c0 + lane; j < c1; j += 32) lt[j - c0] = 0xFFFFFFFFu;
+      continue;
+    }
+    const int Bm = p.Bmax;
+    const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+    for (int b = lane; b < Bm; b += 32) sT[w][b] = Tg[b];
+    __syncwarp();
+    const int32_t *T = sT[w];
+    const bool mono = a.mono[(size_t)s * D + d] != 0;
+    const WinEntry e = a.ent[(int64_t)li * a.nw + k];
+    int64_t h = e.h, F = e.F;
+    // positions before the first head: the batch that crossed c0 (finish F)
+    const int64_t hs = h < c1 ? h : c1;
+    for (int64_t j = c0 + lane; j < hs; j += 32) lt[j - c0] = sat_lat(F - (int64_t)A(j));
+    if (Bm == 1) {  // F_i = max(F_{i-1}, a_i) + T(1): a prefix maximum, 32 positions per step
+      const int64_t T1 = T[0];
+      for (int64_t b0 = h; b0 < c1; b0 += 32) {
+        const int64_t j = b0 + lane;
+        int64_t x = j < c1 ? (int64_t)A(j) - (j - b0) * T1 : INT64_MIN;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int64_t y = __shfl_up_sync(0xffffffffu, x, o);
+          if (lane >= o) x = y > x ? y : x;
+        }
+        const int64_t g = F > x ? F : x;
+        const int64_t Fj = g + (j - b0 + 1) * T1;
+        if (j < c1) lt[j - c0] = sat_lat(Fj - (int64_t)A(j));
+        F = __shfl_sync(0xffffffffu, Fj, (int)((c1 - b0 < 32 ? c1 - b0 : 32) - 1));
+      }
+      continue;
+    }
+    while (h < c1) {
+      // the idle decisions of the 32 positions from h, in parallel
+      const int64_t base = h;
+      int64_t tl = 0;
+      int bl = 0;
+      if (base + lane < c1) bl = idle_decide(A, n, base + lane, Bm, p.L, T, mono, &tl);
+      while (h < c1 && h < base + 32) {
+        const int i = (int)(h - base);
+        int b = __shfl_sync(0xffffffffu, bl, i);
+        int64_t t = __shfl_sync(0xffffffffu, tl, i);
+        if (F > t) {  // greedy (fact (i)): leave at F with what has arrived by then
+          int c = 0;
+          for (int r = 0; r < Bm; r += 32) {
+            const int64_t j = h + r + lane;
+            const bool le = r + lane < Bm && j < n && (int64_t)A(j) <= F;
+            c += __popc(__ballot_sync(0xffffffffu, le));
+          }
+          b = c;
+          t = F;
+        }
+        const int64_t Fn = t + T[b - 1];
+        for (int r = lane; r < b; r += 32)
+          if (h + r < c1) lt[h + r - c0] = sat_lat(Fn - (int64_t)A(h + r));
+        F = Fn;
+        h += b;
+      }
+    }
+  }
+  __syncthreads();
+  // query order: out[s][i] for the window's queries; counts (a13)
+  const int64_t i0 = k * TQ;
+  const int64_t i1 = i0 + TQ < a.N ? i0 + TQ : a.N;
+  unsigned long long viol = 0, ont = 0, accs = 0;
+  uint32_t *orow = a.out ? a.out + (size_t)s * a.N : nullptr;
+  for (int64_t i = i0 + threadIdx.x; i < i1; i += WIN_THREADS) {
+    const int d = a.tgt[i];
+    uint32_t l;
+    if (d >= D) {
+      l = 0xFFFFFFFFu;  // the sink: dropped (R7)
+      viol++;
+    } else {
+      const int64_t pos = (int64_t)a.inv[i] - a.devOff[d];
+      l = slat[wbase[d] + (pos - wc0[d])];
+      if ((int64_t)l > wL[d]) viol++;  // R6
+      else { ont++; accs += wA[d]; }   // R9
+    }
+    if (orow) orow[i] = l;
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    viol += __shfl_xor_sync(0xffffffffu, viol, o);
+    ont += __shfl_xor_sync(0xffffffffu, ont, o);
+    accs += __shfl_xor_sync(0xffffffffu, accs, o);
+  }
+  if (lane == 0) { red[0][w] = viol; red[1][w] = ont; red[2][w] = accs; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long v = 0, o2 = 0, a2 = 0;
+    for (int x = 0; x < nwarps; x++) { v += red[0][x]; o2 += red[1][x]; a2 += red[2][x]; }
+    if (v) atomicAdd((unsigned long long *)&a.agg[s], v);
+    if (o2) atomicAdd((unsigned long long *)&a.agg[a.S + s], o2);
+    if (a2) atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], a2);
+  }
+}
+
+// a13 + un-permute in one pass (the chunk-run / stitch path): per query i and
+// scenario s, the latency from the device-major rows (gathered through inv;
+// the sink: dropped, R7) written once in query order, and the per-scenario
+// violations (R6), on-time count and accuracy sum (R9) of the same values --
+// each latency read once (k_count + k_unpermute read every row twice).
+#define FIN_PER 16
+__global__ void __launch_bounds__(256) k_finish(int64_t N, int64_t NS, int S, int D,
+                                                const proteus_scenario *__restrict__ sc,
+                                                const uint32_t *__restrict__ inv0, const uint32_t *__restrict__ inv1,
+                                                const uint8_t *__restrict__ tgt0, const uint8_t *__restrict__ tgt1,
+                                                const LaneParam *__restrict__ lp, const uint32_t *__restrict__ latd,
+                                                uint32_t *out, uint64_t *agg) {
+  __shared__ unsigned long long red[3][8];
+  const int64_t i0 = (int64_t)blockIdx.x * (256 * FIN_PER) + threadIdx.x;
+  uint32_t p0[FIN_PER], p1[FIN_PER];
+  uint8_t g0[FIN_PER], g1[FIN_PER];
+#pragma unroll
+  for (int k = 0; k < FIN_PER; k++) {
+    const int64_t i = i0 + 256 * k;
+    const bool v = i < N;
+    p0[k] = (inv0 && v) ? inv0[i] : 0;
+    p1[k] = (inv1 && v) ? inv1[i] : 0;
+    g0[k] = (tgt0 && v) ? tgt0[i] : 0;
+    g1[k] = (tgt1 && v) ? tgt1[i] : 0;
+  }
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  for (int s = 0; s < S; s++) {
+    const int rt = sc[s].routing;
+    if (rt < 0) continue;  // written by the window path
+    const size_t rs = (size_t)s * NS;
+    const LaneParam *lps = lp + (size_t)s * D;
+    unsigned long long viol = 0, ont = 0, accs = 0;
+    uint32_t v[FIN_PER];
+#pragma unroll
+    for (int k = 0; k < FIN_PER; k++) {
+      const int d = rt ? g1[k] : g0[k];
+      v[k] = 0xFFFFFFFFu;
+      if (i0 + 256 * k < N && d < D) v[k] = latd[rs + (rt ? p1[k] : p0[k])];
+    }
+#pragma unroll
+    for (int k = 0; k < FIN_PER; k++) {
+      if (i0 + 256 * k >= N) continue;
+      const int d = rt ? g1[k] : g0[k];
+      if (d >= D) { viol++; }
+      else {
+        const LaneParam q = lps[d];
+        if ((int64_t)v[k] > q.L) viol++;
+        else { ont++; accs += q.A; }
+      }
+      if (out) out[(size_t)s * N + i0 + 256 * k] = v[k];
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      viol += __shfl_xor_sync(0xffffffffu, viol, o);
+      ont += __shfl_xor_sync(0xffffffffu, ont, o);
+      accs += __shfl_xor_sync(0xffffffffu, accs, o);
+    }
+    if (lane == 0) { red[0][w] = viol; red[1][w] = ont; red[2][w] = accs; }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned long long a0 = 0, a1 = 0, a2 = 0;
+      for (int x = 0; x < 8; x++) { a0 += red[0][x]; a1 += red[1][x]; a2 += red[2][x]; }
+      if (a0) atomicAdd((unsigned long long *)&agg[s], a0);
+      if (a1) atomicAdd((unsigned long long *)&agg[S + s], a1);
+      if (a2) atomicAdd((unsigned long long *)&agg[2 * S + s], a2);
+    }
+    __syncthreads();
   }
 }
 
@@ -1894,12 +2500,51 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   int64_t *d_choff = (int64_t *)(((uintptr_t)(d_goff + 2 * (PX_MAXD + 2)) + 15) & ~(uintptr_t)15);  // [2][PX_MAXD + 2]
   proteus_scenario *d_sc = (proteus_scenario *)(d_choff + 2 * (PX_MAXD + 2));
   LaneParam *d_lp = (LaneParam *)(((uintptr_t)(d_sc + S) + 15) & ~(uintptr_t)15);
+  // Bmax per (scenario, device), as k_lane_params (R4', R15); T(b) non-decreasing on the lane
+  std::vector<int32_t> hB((size_t)S * D, 0), hT1(D, 0);
+  std::vector<uint8_t> hmono((size_t)S * D, 0);
+  for (int d = 0; d < D; d++) {
+    if (h_option[d] <= 0) continue;
+    const int32_t *Tr = ctx->lat.data() + ((size_t)h_dev_type[d] * M + (h_option[d] - 1)) * ctx->bmax;
+    int depth = 0;
+    while (depth < ctx->bmax && Tr[depth] > 0) depth++;
+    hT1[d] = Tr[0];
+    const int64_t base = h_slo[ctx->fam[h_option[d] - 1]];
+    for (int s = 0; s < S; s++) {
+      const int cap = h_sc[s].batch_cap;
+      int B = (cap > 0 && cap < depth) ? cap : depth;
+      if (h_sc[s].policy == 0 && B > 0) {  // the maximum allowed batch size (R4')
+        const int64_t L = (int64_t)h_sc[s].slo_mult_milli * base / 1000;
+        int Bn = 1;
+        for (int b = 1; b <= B; b++) if (2 * (int64_t)Tr[b - 1] <= L) Bn = b;
+        B = Bn;
+      }
+      hB[(size_t)s * D + d] = B;
+      bool mono = true;
+      for (int b = 1; b < B; b++) mono &= Tr[b] >= Tr[b - 1];
+      hmono[(size_t)s * D + d] = mono ? 1 : 0;
+    }
+  }
+  // the window path (k_win_*) takes the §5 scenarios whose lanes all have
+  // Bmax <= WIN_EMAX; the chunk-run / stitch path below takes the rest
+  const bool simple = env_int("PROTEUS_REPLAY_SIMPLE", 0) != 0;
+  const bool use_win = !simple && env_int("PROTEUS_REPLAY_WINDOW", 0) != 0;
+  std::vector<int32_t> wl[2];
+  std::vector<char> is_win(S, 0);
+  for (int s = 0; s < S; s++) {
+    if (!use_win || h_sc[s].policy != 0) continue;
+    int mb = 0;
+    for (int d = 0; d < D; d++) mb = std::max(mb, hB[(size_t)s * D + d]);
+    if (mb <= WIN_EMAX) { wl[h_sc[s].routing].push_back(s); is_win[s] = 1; }
+  }
   std::vector<int32_t> scl[8];
   for (int s = 0; s < S; s++) {
+    if (is_win[s]) continue;
     scl[h_sc[s].routing].push_back(s);
     scl[(h_sc[s].policy == 0 ? 2 : 4) + h_sc[s].routing].push_back(s);
     if (h_sc[s].policy == 2) scl[6 + h_sc[s].routing].push_back(s);
   }
+  const bool any_old = !scl[0].empty() || !scl[1].empty();
   std::vector<int32_t> scl_all(8 * S, 0);
   for (int r = 0; r < 8; r++)
     for (size_t k = 0; k < scl[r].size(); k++) scl_all[r * S + k] = scl[r][k];
@@ -1909,7 +2554,12 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   PX_CUDA(ctx, cudaMemcpyAsync(d_dem, h_demand, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_slo, h_slo, Q * 4, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_scl, scl_all.data(), 8 * S * 4, cudaMemcpyHostToDevice, ctx->stream));
-  PX_CUDA(ctx, cudaMemcpyAsync(d_sc, h_sc, S * sizeof(proteus_scenario), cudaMemcpyHostToDevice, ctx->stream));
+  {  // the un-permute of the old path skips the window path's rows (routing -1)
+    std::vector<proteus_scenario> sc2(h_sc, h_sc + S);
+    for (int s = 0; s < S; s++) if (is_win[s]) sc2[s].routing = -1;
+    PX_CUDA(ctx, cudaMemcpyAsync(d_sc, sc2.data(), S * sizeof(proteus_scenario), cudaMemcpyHostToDevice, ctx->stream));
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // sc2 is a stack copy
+  }
   PX_CUDA(ctx, cudaMemsetAsync(d_flags, 0, 4, ctx->stream));
   if (N > 0) {
     PX_LAUNCH(ctx, "replay_check", k_check_trace, 1184, 256, 0, d_arr, d_fam, N, Q, d_flags);
@@ -1928,12 +2578,14 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   const size_t pat_cap = (size_t)dsum + (size_t)Q * D + 16;
   int64_t *devOff[2] = {nullptr, nullptr};
   const uint32_t *devArr[2] = {nullptr, nullptr}, *inv[2] = {nullptr, nullptr};
+  int32_t *dbase_rt[2] = {nullptr, nullptr};
+  const uint8_t *tgt_rt[2] = {nullptr, nullptr};
   for (int rt = 0; rt < 2; rt++) {
-    if (scl[rt].empty()) continue;
+    if (scl[rt].empty() && wl[rt].empty()) continue;
     uint8_t *pat = (uint8_t *)px_buf(ctx, B_R_PAT, pat_cap);
     int32_t *hist = (int32_t *)px_buf(ctx, B_R_HIST, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
     int32_t *fbase = (int32_t *)px_buf(ctx, B_R_BASE, (size_t)(ntiles + 1) * (PX_MAXQ + 2) * 4);
-    int32_t *dbase = (int32_t *)px_buf(ctx, B_R_DBASE0, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
+    int32_t *dbase = (int32_t *)px_buf(ctx, rt ? B_R_DBASE1 : B_R_DBASE0, (size_t)(ntiles + 1) * (PX_MAXD + 2) * 4);
     uint8_t *tgt = (uint8_t *)px_buf(ctx, rt ? B_R_TGT1 : B_R_TGT, (size_t)N + 16);
     int64_t *off = (int64_t *)px_buf(ctx, rt ? B_R_OFF1 : B_R_OFF, (size_t)2 * (PX_MAXD + 2) * 8);
     // + whole trailing ring segment: k_stitch bulk-copies 4 KB segments
@@ -1957,13 +2609,95 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     } else {
       PX_CUDA(ctx, cudaMemsetAsync(off, 0, (size_t)(PX_MAXD + 2) * 8, ctx->stream));
     }
-    devOff[rt] = off; devArr[rt] = darr; inv[rt] = dinv;
+    devOff[rt] = off; devArr[rt] = darr; inv[rt] = dinv; dbase_rt[rt] = dbase; tgt_rt[rt] = tgt;
   }
   if (N == 0) return 0;
+  // ---- window path (k_win_tables, k_win_compose, k_win_write)
+  if (!wl[0].empty() || !wl[1].empty()) {
+    int WT = env_int("PROTEUS_REPLAY_WIN_TILES", 16);
+    WT = WT < 1 ? 1 : WT > 32 ? 32 : WT;  // TQ = WT * TILE <= 16384 queries (shared-memory tiles)
+    const int64_t TQ = (int64_t)WT * TILE;
+    const int64_t nw = (ntiles + WT - 1) / WT;
+    if (nw > 65535) return px_fail(ctx, PROTEUS_ERANGE, "replay windows");
+    char *aux = (char *)px_buf(ctx, B_W_AUX, (size_t)S * D * (1 + 4 + 8) + (size_t)2 * S * 4 + 256);
+    if (!aux) return px_fail(ctx, PROTEUS_ENOMEM, "window scratch");
+    uint8_t *d_mono = (uint8_t *)aux;
+    int64_t *d_recoff = (int64_t *)(((uintptr_t)(d_mono + (size_t)S * D) + 15) & ~(uintptr_t)15);
+    int32_t *d_E = (int32_t *)(d_recoff + (size_t)S * D);
+    int32_t *d_wl = d_E + (size_t)S * D;
+    PX_CUDA(ctx, cudaMemcpyAsync(d_mono, hmono.data(), (size_t)S * D, cudaMemcpyHostToDevice, ctx->stream));
+    std::vector<int64_t> recoff((size_t)S * D, 0);
+    std::vector<int32_t> Ev((size_t)S * D, 0), wlv(2 * (size_t)S, 0);
+    int64_t nrec = 0, lbase = 0;
+    for (int rt = 0; rt < 2; rt++) {
+      for (size_t i = 0; i < wl[rt].size(); i++) {
+        wlv[(size_t)rt * S + i] = wl[rt][i];
+        for (int d = 0; d < D; d++) {
+          const int B = hB[(size_t)wl[rt][i] * D + d];
+          const int E = B >= 1 ? std::min(B, WIN_EMAX) : 0;
+          Ev[lbase + i * D + d] = E;
+          recoff[lbase + i * D + d] = nrec;
+          nrec += (int64_t)E * nw;
+        }
+      }
+      lbase += (int64_t)wl[rt].size() * D;
+    }
+    WinRec *d_rec = (WinRec *)px_buf(ctx, B_W_REC, sizeof(WinRec) * (size_t)(nrec + 1));
+    WinEntry *d_ent = (WinEntry *)px_buf(ctx, B_W_ENT, sizeof(WinEntry) * (size_t)(lbase * nw + 1));
+    if (!d_rec || !d_ent) return px_fail(ctx, PROTEUS_ENOMEM, "window tables");
+    PX_CUDA(ctx, cudaMemcpyAsync(d_recoff, recoff.data(), recoff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
+    PX_CUDA(ctx, cudaMemcpyAsync(d_E, Ev.data(), Ev.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+    PX_CUDA(ctx, cudaMemcpyAsync(d_wl, wlv.data(), wlv.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // host vectors are staged
+    const size_t sm1 = (size_t)(TQ + WIN_EXT) * 4 + (size_t)WIN_WARPS * TQ;
+    const size_t sm3 = (size_t)TQ * 4 + (size_t)(TQ + (size_t)D * WIN_EXT) * 4;
+    PX_CUDA(ctx, cudaFuncSetAttribute(k_win_tables, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm1));
+    PX_CUDA(ctx, cudaFuncSetAttribute(k_win_write, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm3));
+    int64_t loff = 0;
+    for (int rt = 0; rt < 2; rt++) {
+      const int nsc = (int)wl[rt].size();
+      if (!nsc) continue;
+      WinArgs wa;
+      memset(&wa, 0, sizeof wa);
+      wa.S = S; wa.D = D; wa.M = M; wa.bmax = ctx->bmax; wa.nsc = nsc; wa.WT = WT; wa.D1 = D + 1;
+      wa.N = N; wa.nw = nw; wa.ntiles = ntiles;
+      wa.option = d_opt; wa.dev_type = d_dev; wa.lat = ctx->d_lat; wa.sc_list = d_wl + (size_t)rt * S;
+      wa.lp = d_lp; wa.mono = d_mono; wa.devOff = devOff[rt]; wa.dbase = dbase_rt[rt]; wa.devArr = devArr[rt];
+      wa.inv = inv[rt]; wa.tgt = tgt_rt[rt]; wa.recoff = d_recoff + loff; wa.E = d_E + loff; wa.rec = d_rec;
+      wa.ent = d_ent + loff * nw; wa.out = d_lat_out; wa.agg = d_agg;
+      const int64_t items = (int64_t)nsc * D * nw;
+      const bool dbg = env_int("PROTEUS_REPLAY_DEBUG", 0) != 0;
+      if (dbg) {
+        wa.dbg = (unsigned long long *)px_buf(ctx, B_R_VLAT, (size_t)nsc * D * 32 + 64);
+        if (!wa.dbg) return px_fail(ctx, PROTEUS_ENOMEM, "debug counters");
+        PX_CUDA(ctx, cudaMemsetAsync(wa.dbg, 0, (size_t)nsc * D * 32, ctx->stream));
+      }
+      (void)items;
+      PX_LAUNCH(ctx, "replay_win_tables", k_win_tables, (unsigned)(nw * D), WIN_WARPS * 32, sm1, wa);
+      PX_LAUNCH(ctx, "replay_win_compose", k_win_compose, (unsigned)(((int64_t)nsc * D + 3) / 4), 128, 0, wa);
+      if (dbg) {
+        std::vector<unsigned long long> hc((size_t)nsc * D * 4);
+        std::vector<int64_t> hoff(D + 2);
+        PX_CUDA(ctx, cudaMemcpyAsync(hoff.data(), devOff[rt], (D + 2) * 8, cudaMemcpyDeviceToHost, ctx->stream));
+        PX_CUDA(ctx, cudaMemcpyAsync(hc.data(), wa.dbg, hc.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+        PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+        for (int i = 0; i < nsc; i++)
+          for (int d = 0; d < D; d++) {
+            const unsigned long long *c = &hc[((size_t)i * D + d) * 4];
+            if (c[0] || c[1] || c[2])
+              fprintf(stderr, "win rt %d sc %d (mult %d cap %d) dev %d: n=%lld Bmax=%d idle %llu backlog %llu walks %llu "
+                      "walked %llu\n", rt, wl[rt][i], h_sc[wl[rt][i]].slo_mult_milli, h_sc[wl[rt][i]].batch_cap, d,
+                      (long long)(hoff[d + 1] - hoff[d]), hB[(size_t)wl[rt][i] * D + d], c[0], c[1], c[2], c[3]);
+          }
+      }
+      PX_LAUNCH(ctx, "replay_win_write", k_win_write, dim3((unsigned)nsc, (unsigned)nw), WIN_THREADS, sm3, wa);
+      loff += (int64_t)nsc * D;
+    }
+  }
+  if (!any_old) return 0;
   // chunk layout per routing mode (sizes only): the host reads the per-device counts
   int CH = env_int("PROTEUS_REPLAY_CHUNK", 4096);
   CH = CH < 1 ? 1 : CH > (1 << 20) ? (1 << 20) : CH;
-  const bool simple = env_int("PROTEUS_REPLAY_SIMPLE", 0) != 0;
   // fix-up rounds before the sequential stitch finishes whatever is left
   const int max_rounds = env_int("PROTEUS_REPLAY_ROUNDS", 0);
   int64_t h_off[2][PX_MAXD + 2];
@@ -2006,19 +2740,6 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     if (!csb[0] || !csb[1]) return px_fail(ctx, PROTEUS_ENOMEM, "chunk states");
     PX_CUDA(ctx, cudaFuncSetAttribute(k_stitch, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)stitch_smem(ctx->bmax)));
-  }
-  // Bmax per (scenario, device), as k_lane_params (R4)
-  std::vector<int32_t> hB((size_t)S * D, 0), hT1(D, 0);
-  for (int d = 0; d < D; d++) {
-    if (h_option[d] <= 0) continue;
-    const int32_t *Tr = ctx->lat.data() + ((size_t)h_dev_type[d] * M + (h_option[d] - 1)) * ctx->bmax;
-    int depth = 0;
-    while (depth < ctx->bmax && Tr[depth] > 0) depth++;
-    hT1[d] = Tr[0];
-    for (int s = 0; s < S; s++) {
-      const int cap = h_sc[s].batch_cap;
-      hB[(size_t)s * D + d] = (cap > 0 && cap < depth) ? cap : depth;
-    }
   }
   const bool use_scan1 = !simple && env_int("PROTEUS_REPLAY_SCAN1", 1) != 0;
   for (int rt = 0; rt < 2; rt++) {
@@ -2180,17 +2901,24 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       if (lb.wst) PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<true>, (unsigned)((warps + 3) / 4), 128, 0, lb);
       else PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<false>, (unsigned)((warps + 3) / 4), 128, 0, lb);
     }
-    const int nall = (int)scl[rt].size();
-    dim3 g(32, nall < 65535 ? nall : 65535);
-    PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, NS, S, D, d_scl + rt * S, nall, devOff[rt], latd, d_agg);
-    dim3 cg((unsigned)((N + CNT_PER - 1) / CNT_PER), (unsigned)nall);
-    PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, NS, S, D, d_scl + rt * S, devOff[rt], d_lp, latd, d_agg);
+    if (!d_lat_out || env_int("PROTEUS_REPLAY_FINISH", 0) == 0) {  // counts from the device-major rows
+      const int nall = (int)scl[rt].size();
+      dim3 g(32, nall < 65535 ? nall : 65535);
+      PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, NS, S, D, d_scl + rt * S, nall, devOff[rt], latd, d_agg);
+      dim3 cg((unsigned)((N + CNT_PER - 1) / CNT_PER), (unsigned)nall);
+      PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, NS, S, D, d_scl + rt * S, devOff[rt], d_lp, latd, d_agg);
+    }
   }
   if (d_lat_out) {
-    int nsm = 0;
-    PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
     const int64_t nb = (N + 256 * UNP_PER - 1) / (256 * UNP_PER);
-    PX_LAUNCH(ctx, "replay_unpermute", k_unpermute, (unsigned)nb, 256, 0, N, NS, S, d_sc, inv[0], inv[1], latd, d_lat_out);
+    if (env_int("PROTEUS_REPLAY_FINISH", 0) == 0) {
+      PX_LAUNCH(ctx, "replay_unpermute", k_unpermute, (unsigned)nb, 256, 0, N, NS, S, d_sc, inv[0], inv[1], latd,
+                d_lat_out);
+    } else {  // latencies in query order and the counts in one pass
+      const int64_t nf = (N + 256 * FIN_PER - 1) / (256 * FIN_PER);
+      PX_LAUNCH(ctx, "replay_finish", k_finish, (unsigned)nf, 256, 0, N, NS, S, D, d_sc, inv[0], inv[1], tgt_rt[0],
+                tgt_rt[1], d_lp, latd, d_lat_out, d_agg);
+    }
   }
   return 0;
 }
@@ -2331,8 +3059,11 @@ __device__ __forceinline__ EpLane ep_lane(const EpArgs &a, int s, int e, int d) 
   int depth = 0;
   while (depth < a.bmax && r.T[depth] > 0) depth++;
   const int cap = a.sc[s].batch_cap;
-  r.Bmax = (cap > 0 && cap < depth) ? cap : depth;
+  const int Bcap = (cap > 0 && cap < depth) ? cap : depth;
   r.L = (int64_t)a.sc[s].slo_mult_milli * a.slo[a.fam_of_m[o - 1]] / 1000;
+  r.Bmax = 1;  // the maximum allowed batch size of the epoch's variant (reading R4')
+  for (int b = 1; b <= Bcap; b++)
+    if (2 * (int64_t)r.T[b - 1] <= r.L) r.Bmax = b;
   return r;
 }
 

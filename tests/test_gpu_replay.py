@@ -47,6 +47,15 @@ PATHS = {"chunked": {}, "small_chunks": {"PROTEUS_REPLAY_CHUNK": "16"}, "odd_chu
          "warmup_long_small_chunks": {"PROTEUS_REPLAY_CHUNK": "16", "PROTEUS_REPLAY_WARMUP": "1000"},
          "warmup_rounds": {"PROTEUS_REPLAY_ROUNDS": "3", "PROTEUS_REPLAY_CHUNK": "64", "PROTEUS_REPLAY_WARMUP": "100"},
          "warmup_bscan": {"PROTEUS_REPLAY_BSCAN": "1", "PROTEUS_REPLAY_CHUNK": "200", "PROTEUS_REPLAY_WARMUP": "300"}}
+# the chunk-run / stitch path (PROTEUS_REPLAY_WINDOW=0) under every knob; the
+# window path (the default for §5 lanes with Bmax <= 64) with windows of 1, 3,
+# 32 (default) and 64 tiles of 512 queries
+PATHS = {k: dict(v, PROTEUS_REPLAY_WINDOW="0") for k, v in PATHS.items()}
+PATHS["finish_fused"] = {"PROTEUS_REPLAY_FINISH": "1"}
+PATHS.update({"window": {"PROTEUS_REPLAY_WINDOW": "1"},
+              "window_wt1": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "1"},
+              "window_wt3": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "3"},
+              "window_wt32": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "32"}})
 
 
 @pytest.mark.parametrize("path", sorted(PATHS))

@@ -169,11 +169,13 @@ def test_full_replay_policies(oracle_mod):
         L = int(sc[s, 0]) * int(cl.slo_us[fam_m[m]]) // 1000
         Tp = [0] + [int(x) for x in row[:Bmax]]
         sel = np.nonzero(tgt == d)[0]
+        # the maximum allowed batch size: Nexus's batch (R14) and the
+        # §5 policy's cap (R4'); AIMD grows its limit to min(cap, depth) (R15)
+        B = max([1] + [b for b in range(1, Bmax + 1) if 2 * Tp[b] <= L])
         if sc[s, 3] == 1:
-            B = max([1] + [b for b in range(1, Bmax + 1) if 2 * Tp[b] <= L])
             ref = oracle_mod.replay_device_nexus(a[sel], Tp, B, L)
         elif sc[s, 3] == 2:
             ref = oracle_mod.replay_device_aimd(a[sel], Tp, Bmax, L)
         else:
-            ref = oracle_mod.replay_device(a[sel], Tp, Bmax, L)
+            ref = oracle_mod.replay_device(a[sel], Tp[:B + 1], B, L)
         assert np.array_equal(out["latency"][s][sel], ref)

@@ -198,3 +198,31 @@ def test_acc_sum_hand_worked(oracle_mod):
     assert out["on_time"].tolist() == [3, 4]
     assert out["violations"].tolist() == [3, 2]
     assert out["acc_sum"].tolist() == [2_800_000, 3_800_000]
+
+
+def test_max_allowed_batch_size_R4prime(oracle_mod):
+    """Reading R4': a device batches at most the "maximum allowed
+    batch size" -- the largest b <= min(cap, depth) with 2 T(b) <= SLO (the
+    half-SLO rule of P:920-926), at least 1.  Worked by hand: one variant,
+    T = (100, 130, 160, 190, 220) us for b = 1..5 (depth 5), 7 queries at t = 0,
+    one device with z = 7 = demand (no sink).
+      SLO 400, cap depth: b* = 4 (2 x 190 <= 400 < 2 x 220): four leave at 0
+        (F = 190); three wait until W = 0 + 400 - T(4) = 210, F = 210 + 160 = 370
+        -> latencies 190 x 4, 370 x 3, all on time.
+      SLO 400, cap 3: three at 0 (F = 160); at 160 four are queued >= 3: three
+        more (F = 320); at 320 one is left, W = 400 - T(2) = 270 <= 320: it
+        leaves at once, F = 420 -> 160 x 3, 320 x 3, 420 (late).
+      SLO 800: b* = 5 = depth: five at 0 (F = 220); two wait until
+        W = 800 - T(3) = 640, F = 770 -> 220 x 5, 770 x 2."""
+    from paper_conf_asplos_ahmadgfwsw24_b200.workloads import Profiles
+    prof = Profiles(T=1, Q=1, V=np.array([1], np.int32), acc_micro=np.array([1_000_000], np.int32), bmax=5,
+                    lat_us=np.array([[[100, 130, 160, 190, 220]]], np.int32))
+    arr = np.zeros(7, np.uint32)
+    fam = np.zeros(7, np.uint8)
+    sc = np.array([[1000, 0, 0], [1000, 3, 0], [2000, 0, 0]], np.int32)
+    out = oracle_mod.replay(prof, np.array([0], np.int32), np.array([1], np.int32), np.array([7], np.int32),
+                            np.array([7], np.int32), np.array([400], np.int32), arr, fam, sc)
+    assert out["latency"][0].tolist() == [190] * 4 + [370] * 3
+    assert out["latency"][1].tolist() == [160] * 3 + [320] * 3 + [420]
+    assert out["latency"][2].tolist() == [220] * 5 + [770] * 2
+    assert out["on_time"].tolist() == [7, 6, 7] and out["violations"].tolist() == [0, 1, 0]
