@@ -211,19 +211,15 @@ int px_pareto_merge(proteus_ctx *ctx, const proteus_pareto_point *d_pts, int n, 
 
 // ----------------------------------------------- scenario assignment ----
 // Relative cost of one replay scenario's lanes (host; a deterministic model
-// from measured 1-GPU per-scenario times): the §5 lanes with
-// Bmax = 1 are one exact prefix-max scan (cheap); larger batch caps and SLOs
-// make the stitch's critical lanes longer; the baseline batchers walk
-// sequential chains.
+// from the measured 1-GPU time of every c5 scenario replayed alone,
+// profiles/r02d_scenario_costs.json): §5 lanes with Bmax = 1
+// are one exact prefix-max scan (0.7 ms); every other §5 scenario costs about
+// the same (8-19 ms, set by its slowest stitch lane); Clipper AIMD 27-77 ms
+// and Nexus 220-440 ms (sequential chains of the overloaded lanes).
 static double scenario_cost(const proteus_scenario &s) {
-  const double mult = s.slo_mult_milli / 1000.0;
-  const int cap = s.batch_cap == 0 ? 64 : s.batch_cap;
-  if (s.policy == 1) return 8.0 + 2.0 * mult;               // Nexus early drop
-  if (s.policy == 2) return 2.0 + 0.2 * mult;               // Clipper AIMD
-  if (cap == 1) return 0.05;                                // Bmax = 1: one scan for all such scenarios
-  double c = 0.2 + 0.05 * mult * (cap >= 8 ? 8 : cap);      // chunk runs + stitch
-  if (cap >= 16) c += 0.15 * mult * (cap >= 32 ? 2.0 : 1.0); // slow-merging critical lanes
-  return c;
+  if (s.policy == 1) return 32.0;   // Nexus early drop
+  if (s.policy == 2) return 3.5;    // Clipper AIMD
+  return s.batch_cap == 1 ? 0.06 : 1.0;
 }
 
 // Longest-processing-time greedy: scenarios by decreasing cost (ties by

@@ -292,6 +292,18 @@ __global__ void k_lane_params(int S, int D, int M, int bmax, const int32_t *__re
   lp[i] = p;
 }
 
+struct WinRec {     // chain of one entry offset o of one chunk (times relative to a_{c0})
+  int64_t Fx;       // free time after the batch that crosses c1 (absolute; Bmax = 1: R of the max-plus form)
+  int32_t tdisp;    // idle dispatch time at the entry head c0 + o, - a_{c0}
+  int32_t R;        // backlog threshold of (iii) through the chunk, - a_{c0} (INT32_MAX: none)
+  int32_t hx;       // first head >= c1 of the chain, - c0
+  int32_t pad;
+};
+struct WinEntry {   // true state at a chunk start: first head >= c0 (device-relative), free time
+  int64_t F;
+  int32_t h, pad;
+};
+
 struct LaneArgs {
   int S, D, M, bmax, nsc, CH;
   int WU;                 // k_spec warm-up: queries replayed before each chunk (0 = start at the chunk)
@@ -318,6 +330,13 @@ struct LaneArgs {
   uint8_t *wst;           // baseline chunk runs: [S][NS] 0, or 1 + the run's AIMD limit (Nexus: 1) at a
                           // decision whose head found the device free (NULL: no chunk runs)
   struct WcExit *wx;      // baseline chunk runs: [S][NCH] exit state
+  // chunk tables of the idle-branch chains (k_win_tables over the CH chunks) for
+  // lanes with large Bmax: the stitch hops a chunk entered on the idle branch
+  // and k_rewrite replays it from the true entry (rw)
+  const WinRec *trec;
+  const int64_t *trecoff;  // [nsc * D] (list position * D + d)
+  const int32_t *tE;       // [nsc * D] entry offsets per chunk (0: no table)
+  WinEntry *rw;            // [nsc * D][NCH] true entry of a hopped chunk (pad = 1)
 };
 
 struct WcExit {  // a baseline chunk run left its chunk at head h (>= chunk end), device free at F;
@@ -1073,6 +1092,10 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   tbig = __reduce_max_sync(0xffffffffu, tbig);
   const int64_t SW = tbig <= TB ? (p.L - TB > 0 ? p.L - TB : 0) : INT64_MIN / 4;
   bool lastfull = true;
+  const int64_t li_t = (gw / a.D) * a.D + d;  // lane index of the chunk tables
+  const int tEl = a.tE ? a.tE[li_t] : 0;
+  const WinRec *trow = tEl ? a.trec + a.trecoff[li_t] : nullptr;
+  WinEntry *rwrow = tEl ? a.rw + li_t * a.NCH : nullptr;
   long long dbg_t0 = clock64(), dbg_dec = 0, dbg_jump = 0, dbg_match = 0, dbg_chk = 0;
   long long dbg_sec[5] = {0, 0, 0, 0, 0}, dbg_tk = 0;
   for (int64_t c0 = cstart; c0 < nch; c0 += 32) {
@@ -1100,6 +1123,15 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
         F = xF;
         PX_DBG(dbg_match++);
         continue;
+      }
+      if (tEl > h - st) {  // the chain table: an entry on the idle branch is a function of its head
+        const WinRec r = trow[c * tEl + (h - st)];
+        if (F <= AR(st) + r.tdisp) {
+          if (lane == 0) { WinEntry e; e.F = F; e.h = (int32_t)h; e.pad = 1; rwrow[c] = e; }
+          h = st + r.hx;
+          F = r.Fx;
+          continue;
+        }
       }
       int checks = a.maxchk;
       const bool spec_ready = true;  // stored latencies stream through lring (positions >= h)
@@ -1413,6 +1445,35 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
 // change leaves every chunk exact (chunk 0 starts at the true initial state,
 // R13, and by induction each chunk entry is the true one).  Reads of the
 // stored row happen before the round rewrites them (positions >= the head).
+// chunks the stitch hopped with a chain table: replay from the true entry
+// (head h >= chunk start, free time F) to the chunk end (the positions before
+// h were written by the stitch; those past the end belong to the next chunk,
+// whose entry F the stitch carried).  Thread per (lane, chunk).
+__global__ void __launch_bounds__(128) k_rewrite(const __grid_constant__ LaneArgs a) {
+  const int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (g >= (int64_t)a.nsc * a.D * a.NCH) return;
+  const int64_t li = g / a.NCH, c = g % a.NCH;
+  if (!a.tE || a.tE[li] == 0) return;
+  const WinEntry e = a.rw[li * a.NCH + c];
+  if (e.pad != 1) return;
+  const int d = (int)(li % a.D), s = a.sc_list[li / a.D];
+  const LaneParam p = a.lp[s * a.D + d];
+  const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
+  const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
+  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  GArr arr{a.devArr + off};
+  uint32_t *out = a.latd + (size_t)s * a.NS + off;
+  int64_t h = e.h, F = e.F;
+  while (h < en) {
+    int64_t t;
+    const int b = decide(arr, n, h, F, p.Bmax, p.L, T, &t);
+    F = t + T[b - 1];
+    const int64_t jend = h + b < en ? h + b : en;
+    for (int64_t j = h; j < jend; j++) out[j] = sat_lat(F - (int64_t)arr(j));
+    h += b;
+  }
+}
+
 __global__ void __launch_bounds__(128) k_fix(const __grid_constant__ LaneArgs a, unsigned *changed) {
   __shared__ int64_t sC[PX_MAXD + 1];
   for (int k = threadIdx.x; k <= a.D; k += blockDim.x) sC[k] = a.choff[k];
@@ -1975,20 +2036,9 @@ __global__ void __launch_bounds__(256) k_unpermute(int64_t N, int64_t NS, int S,
 #define WIN_EXT (2 * WIN_EMAX + 64)  // arrivals staged past a chunk's end (look-ahead of its decisions)
 #define WIN_WARPS 8
 
-struct WinRec {     // chain of one entry offset o of one chunk (times relative to a_{c0})
-  int64_t Fx;       // free time after the batch that crosses c1 (absolute; Bmax = 1: R of the max-plus form)
-  int32_t tdisp;    // idle dispatch time at the entry head c0 + o, - a_{c0}
-  int32_t R;        // backlog threshold of (iii) through the chunk, - a_{c0} (INT32_MAX: none)
-  int32_t hx;       // first head >= c1 of the chain, - c0
-  int32_t pad;
-};
-struct WinEntry {   // true state at a chunk start: first head >= c0 (device-relative), free time
-  int64_t F;
-  int32_t h, pad;
-};
-
 struct WinArgs {
   int S, D, M, bmax, nsc, WT, D1;
+  int64_t CHF;                 // > 0: chunks of CHF positions per device (the stitch's), not windows
   int64_t N, nw, ntiles;
   const int32_t *option, *dev_type, *lat, *sc_list;
   const LaneParam *lp;
@@ -2007,6 +2057,10 @@ struct WinArgs {
 };
 
 __device__ __forceinline__ int64_t win_cb(const WinArgs &a, int64_t k, int d) {
+  if (a.CHF > 0) {
+    const int64_t n = a.devOff[d + 1] - a.devOff[d];
+    return k * a.CHF < n ? k * a.CHF : n;
+  }
   const int64_t t = k * a.WT < a.ntiles ? k * a.WT : a.ntiles;
   return a.dbase[t * a.D1 + d];
 }
@@ -2037,7 +2091,7 @@ __global__ void __launch_bounds__(WIN_WARPS * 32) k_win_tables(const __grid_cons
   const int64_t k = blockIdx.x / a.D;
   const int64_t c0 = win_cb(a, k, d), c1 = win_cb(a, k + 1, d);
   if (c1 <= c0) return;
-  const int64_t TQ = (int64_t)a.WT * TILE;
+  const int64_t TQ = a.CHF > 0 ? a.CHF : (int64_t)a.WT * TILE;
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   uint32_t *sarr = (uint32_t *)win_sm;
   const int64_t slen = (c1 + WIN_EXT < n ? c1 + WIN_EXT : n) - c0;
@@ -2869,8 +2923,57 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       la.cs = csb[cur];
       la.csp = nullptr;
       if (!done) {  // the sequential stitch carries the true state through the rest
+        // chunk tables for the lanes with large Bmax (slow-merging runs): the
+        // stitch hops a chunk entered on the idle branch, k_rewrite replays it
+        const int minB = env_int("PROTEUS_REPLAY_TABLES_MINB", 8);
+        const bool tables = env_int("PROTEUS_REPLAY_TABLES", 0) != 0 && CH <= 8192;  // measured slower on c5
+        std::vector<int32_t> tEv((size_t)la.nsc * D, 0);
+        std::vector<int64_t> trecoff((size_t)la.nsc * D, 0);
+        int64_t ntrec = 0;
+        const int64_t nchd = nmax;
+        if (tables) {
+          for (int i = 0; i < la.nsc; i++)
+            for (int d = 0; d < D; d++) {
+              const int B = hB[(size_t)scl[2 + rt][i] * D + d];
+              const int E = (B >= minB && B <= WIN_EMAX && B > 1) ? B : 0;
+              tEv[(size_t)i * D + d] = E;
+              trecoff[(size_t)i * D + d] = ntrec;
+              ntrec += (int64_t)E * nchd;
+            }
+        }
+        if (ntrec > 0) {
+          char *aux = (char *)px_buf(ctx, B_W_AUX, (size_t)la.nsc * D * 12 + (size_t)S * D + 256);
+          WinRec *d_trec = (WinRec *)px_buf(ctx, B_W_REC, sizeof(WinRec) * (size_t)ntrec + 64);
+          WinEntry *d_rw = (WinEntry *)px_buf(ctx, B_W_ENT, sizeof(WinEntry) * (size_t)la.nsc * D * nchd + 64);
+          if (!aux || !d_trec || !d_rw) return px_fail(ctx, PROTEUS_ENOMEM, "chunk tables");
+          int64_t *d_trecoff = (int64_t *)aux;
+          int32_t *d_tE = (int32_t *)(d_trecoff + (size_t)la.nsc * D);
+          uint8_t *d_mono = (uint8_t *)(d_tE + (size_t)la.nsc * D);
+          PX_CUDA(ctx, cudaMemcpyAsync(d_trecoff, trecoff.data(), trecoff.size() * 8, cudaMemcpyHostToDevice,
+                                       ctx->stream));
+          PX_CUDA(ctx, cudaMemcpyAsync(d_tE, tEv.data(), tEv.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+          PX_CUDA(ctx, cudaMemcpyAsync(d_mono, hmono.data(), (size_t)S * D, cudaMemcpyHostToDevice, ctx->stream));
+          PX_CUDA(ctx, cudaMemsetAsync(d_rw, 0, sizeof(WinEntry) * (size_t)la.nsc * D * nchd, ctx->stream));
+          WinArgs wa;
+          memset(&wa, 0, sizeof wa);
+          wa.S = S; wa.D = D; wa.M = M; wa.bmax = ctx->bmax; wa.nsc = la.nsc; wa.WT = 1; wa.D1 = D + 1; wa.CHF = CH;
+          wa.N = N; wa.nw = nchd; wa.ntiles = ntiles;
+          wa.option = d_opt; wa.dev_type = d_dev; wa.lat = ctx->d_lat; wa.sc_list = la.sc_list; wa.lp = d_lp;
+          wa.mono = d_mono; wa.devOff = devOff[rt]; wa.devArr = devArr[rt]; wa.recoff = d_trecoff; wa.E = d_tE;
+          wa.rec = d_trec;
+          const size_t smt = (size_t)(CH + WIN_EXT) * 4 + (size_t)WIN_WARPS * CH;
+          PX_CUDA(ctx, cudaFuncSetAttribute(k_win_tables, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smt));
+          PX_LAUNCH(ctx, "replay_tables", k_win_tables, (unsigned)(nchd * D), WIN_WARPS * 32, smt, wa);
+          PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // host vectors staged
+          la.trec = d_trec; la.trecoff = d_trecoff; la.tE = d_tE; la.rw = d_rw;
+        }
         const int64_t warps = (int64_t)la.nsc * D;
         PX_LAUNCH(ctx, "replay_stitch", k_stitch, (unsigned)((warps + 3) / 4), 128, stitch_smem(ctx->bmax), la);
+        if (ntrec > 0) {
+          const int64_t nt = (int64_t)la.nsc * D * nchd;
+          PX_LAUNCH(ctx, "replay_rewrite", k_rewrite, (unsigned)((nt + 127) / 128), 128, 0, la);
+        }
+        la.trec = nullptr; la.trecoff = nullptr; la.tE = nullptr; la.rw = nullptr;
       }
     }
     }  // §5 scenarios

@@ -1,0 +1,10 @@
+#!/bin/bash
+# full pass: every GPU test, smoke, bench line, per-scenario costs
+cd "$(dirname "$0")/.."
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+timeout 2400 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
+timeout 900 python bench.py --steps 20 --warmup 5 > gpurun_out/bench.json 2> gpurun_out/bench.err
+timeout 1200 python scripts/scenario_costs.py > gpurun_out/scenario_costs.json 2> gpurun_out/scenario_costs.err
+tail -3 gpurun_out/pytest_gpu.log; tail -2 gpurun_out/smoke.log; head -c 400 gpurun_out/bench.json; tail -3 gpurun_out/bench.err

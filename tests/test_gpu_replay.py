@@ -52,6 +52,11 @@ PATHS = {"chunked": {}, "small_chunks": {"PROTEUS_REPLAY_CHUNK": "16"}, "odd_chu
 # 32 (default) and 64 tiles of 512 queries
 PATHS = {k: dict(v, PROTEUS_REPLAY_WINDOW="0") for k, v in PATHS.items()}
 PATHS["finish_fused"] = {"PROTEUS_REPLAY_FINISH": "1"}
+# the stitch with chunk tables for every lane with Bmax >= 2 / >= 4, and with none
+PATHS["tables_all"] = {"PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB": "2", "PROTEUS_REPLAY_CHUNK": "300"}
+PATHS["tables_min4_chunk64"] = {"PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB": "4",
+                                "PROTEUS_REPLAY_CHUNK": "64"}
+PATHS["tables_default"] = {"PROTEUS_REPLAY_TABLES": "1"}
 PATHS.update({"window": {"PROTEUS_REPLAY_WINDOW": "1"},
               "window_wt1": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "1"},
               "window_wt3": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "3"},
