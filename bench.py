@@ -275,7 +275,6 @@ def main():
     sols_ref = step()[0]
     key = lambda o: (o["score"].tolist(), o["index"].tolist())  # noqa: E731
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    px.set_timing(True)
     kern_ms = []
     launches0 = px.launch_count()
     with ClockSampler(local) as clk:
@@ -286,9 +285,17 @@ def main():
             sols, _ = step()
             ev[k][1].record(stream)
             barrier()
-            kern_ms += [ms for name, ms in px.kernel_times() if name == "score_flat_pair"]
             assert key(sols) == key(sols_ref)
     launches = px.launch_count() - launches0
+    # the scoring kernel's own time: the library's CUDA events around each launch,
+    # in extra steps after the timed ones (the events add host work to a step)
+    px.set_timing(True)
+    for k in range(max(3, args.steps // 4)):
+        flush.zero_()
+        barrier()
+        step()
+        barrier()
+        kern_ms += [ms for name, ms in px.kernel_times() if name == "score_flat_pair"]
     px.set_timing(False)
     step_ms = [a.elapsed_time(b) for a, b in ev]
     total_ms = max_over_ranks(sum(step_ms))
@@ -300,7 +307,7 @@ def main():
     peaks, peak_src = measured_peaks()
     k_ms = statistics.mean(kern_ms) if kern_ms else float("nan")
     # one launch scores the rank's slice for up to 64 vectors of the batch (grid.x = vector)
-    launches_per_step = max(1, len(kern_ms) // args.steps)
+    launches_per_step = max(1, len(kern_ms) // max(3, args.steps // 4))
     ncl = 13**8 // world  # this rank's candidates per vector (index slice)
     cand_per_launch = ncl * NVEC / launches_per_step
     roof = alu_roofline("score_flat_pair", kernel_inst("score_flat_pair"), k_ms, int_peaks(), cand_per_launch,
@@ -335,6 +342,9 @@ def main():
         "config": {"workload": WORKLOAD, "l2": "flushed (256 MB write) before every timed step",
                    "parallelism": (f"index-range shards x{world}, one ncclAllGather of the materialised per-rank "
                                    f"winners per batch + a device pick, inside libproteus") if world > 1 else "1 GPU"},
+        "metric_note": ("candidates covered per second by the exact exhaustive search: each candidate is scored "
+                        "or excluded by an exact block maximum (DESIGN.md §5); time_to_optimal_ms is the "
+                        "per-vector time"),
         "roofline": roof,
         "e2e": {"value": n_cand / e2e_s, "unit": "candidates/s", "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": int(d2h)},

@@ -3,8 +3,10 @@
 // validation (overflow guards) and kernel timing.  All arithmetic of the method
 // runs in the kernels of prepare.cu, solve_enum.cu, solve_factored.cu and
 // replay.cu.
+#include <chrono>
 #include <cstdarg>
 #include <cstddef>
+#include <cstdlib>
 #include <cstring>
 
 #include "internal.cuh"
@@ -154,6 +156,11 @@ void proteus_destroy(proteus_ctx *ctx) {
   for (auto e : ctx->tev) cudaEventDestroy(e);
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
   px_comm_destroy(ctx);
+  if (ctx->aux) cudaStreamDestroy(ctx->aux);
+  if (ctx->aux_hi) cudaStreamDestroy(ctx->aux_hi);
+  if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
+  if (ctx->ev_join) cudaEventDestroy(ctx->ev_join);
+  if (ctx->ev_join2) cudaEventDestroy(ctx->ev_join2);
   delete ctx;
 }
 
@@ -380,9 +387,18 @@ int px_flat_template_vm(int Q, int maxV);  // solve_enum.cu: VM of the specialis
 
 static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a_in, proteus_solution *out, bool mat_only,
                         int32_t mat_vec, uint64_t mat_index, proteus_batch *bout = nullptr) {
+  // PROTEUS_HOST_TIMING=1: host-side phase times of the call on stderr (diagnostic)
+  static const bool htime = getenv("PROTEUS_HOST_TIMING") && atoi(getenv("PROTEUS_HOST_TIMING"));
+  const auto ht0 = std::chrono::steady_clock::now();
+  auto hts = [&](const char *what) {
+    if (htime)
+      fprintf(stderr, "solve %s %.1f us\n", what,
+              std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - ht0).count());
+  };
   SolveInputs in;
   int rc = validate_solve(ctx, a_in, in);
   if (rc) return rc;
+  hts("validated");
   // distributed call (comm.cu): modes 0/1 scan the communicator rank's slice,
   // mode 2 solves the rank's slice of the demand vectors
   const bool dist = px_comm_active(ctx) && !mat_only;
@@ -477,7 +493,12 @@ static int solve_common(proteus_ctx *ctx, const proteus_solve_args *a_in, proteu
     }
   }
   if (rc) return rc;
-  if (bout) return batch_out(ctx, a, d_sol, nout, bout);
+  hts("launched");
+  if (bout) {
+    rc = batch_out(ctx, a, d_sol, nout, bout);
+    hts("returned");
+    return rc;
+  }
   std::vector<SolRec> h(nout);
   PX_CUDA(ctx, cudaMemcpyAsync(h.data(), d_sol, sizeof(SolRec) * nout, cudaMemcpyDeviceToHost, ctx->stream));
   PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));

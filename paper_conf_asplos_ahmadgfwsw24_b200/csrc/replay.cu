@@ -337,6 +337,12 @@ struct LaneArgs {
   const int64_t *trecoff;  // [nsc * D] (list position * D + d)
   const int32_t *tE;       // [nsc * D] entry offsets per chunk (0: no table)
   WinEntry *rw;            // [nsc * D][NCH] true entry of a hopped chunk (pad = 1)
+  // spec/stitch pipelining: k_spec sets cready[s][choff[d] + c] when chunk c's
+  // latencies and exit state are written; k_stitch (running concurrently on
+  // another stream) waits for the flags of the chunks it reads (null: no
+  // wait); cready[-1]: the wait watchdog fired
+  unsigned *cready;
+  const int32_t *lane_order;  // k_stitch: lane (list position * D + d) of warp i (null: identity)
 };
 
 struct WcExit {  // a baseline chunk run left its chunk at head h (>= chunk end), device free at F;
@@ -845,6 +851,24 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   e.eF = eF;
   e.edh = (int32_t)edh;
   a.cs[(size_t)s * a.NCH + a.choff[d] + c] = e;
+  if (a.cready) {  // publish: this chunk's latencies and exit state are written
+    __threadfence();
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(a.cready + (size_t)s * a.NCH + a.choff[d] + c), "r"(1u)
+                 : "memory");
+  }
+}
+
+// k_stitch side of the pipelining: wait until chunk c of (s, d) is published.
+// A watchdog bounds the wait (~8 s): on expiry it raises cready[-1] (the
+// host turns it into PROTEUS_EINTERNAL) instead of hanging the device.
+__device__ __forceinline__ void wait_chunk(unsigned *cready, int64_t idx) {
+  unsigned v;
+  for (uint32_t it = 0;; it++) {
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(cready + idx) : "memory");
+    if (v) break;
+    if (it > (1u << 25)) { atomicExch(cready - 1, 1u); break; }
+    __nanosleep(256);
+  }
 }
 
 // ---- one §5 decision by a whole warp (lane-parallel form of decide()):
@@ -998,8 +1022,9 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   // finishes [32 SUMAX], T [bmax]
   extern __shared__ __align__(16) uint32_t ssm[];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  const int64_t gw = (int64_t)blockIdx.x * 4 + w;
-  if (gw >= (int64_t)a.nsc * a.D) return;
+  const int64_t gw0 = (int64_t)blockIdx.x * 4 + w;
+  if (gw0 >= (int64_t)a.nsc * a.D) return;
+  const int64_t gw = a.lane_order ? a.lane_order[gw0] : gw0;  // pipelined: the longest lanes first
   const int s = a.sc_list[gw / a.D], d = (int)(gw % a.D);
   if (!((a.dmask >> d) & 1ull)) return;
   const LaneParam p = a.lp[s * a.D + d];
@@ -1020,6 +1045,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   uint32_t *out = a.latd + (size_t)s * a.NS + off;
   const ChunkSt *cst = a.cs + (size_t)s * a.NCH + a.choff[d];
   const int64_t CH = a.CH;
+  if (a.cready) wait_chunk(a.cready, (size_t)s * a.NCH + a.choff[d]);  // chunk 0's exit (pipelined k_spec)
   int64_t h = (CH < n ? CH : n) + cst[0].xov, F = cst[0].xF;
   int64_t cstart = 1;  // first chunk to stitch; a lane the full-batch scan took starts where it stopped
   bool fresh = false;  // ... with the positions below h of that chunk already written
@@ -1048,9 +1074,16 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
       __syncwarp();
       // arrivals and the stored latencies of the same positions (the row holds
       // the chunk runs' values at every position >= h: rewritten ones lie below)
-      if (lane == 0)
+      if (lane == 0) {
+        if (a.cready) {  // the segment's chunks of this device are published (pipelined k_spec)
+          const int64_t j0 = sg_iss * RSEG - off, j1 = j0 + RSEG - 1;
+          const int64_t ca = (j0 > 0 ? j0 : 0) / CH, cb = (j1 < n - 1 ? j1 : n - 1) / CH;
+          for (int64_t cc = ca; cc <= cb && cc < nch; cc++) wait_chunk(a.cready, (size_t)s * a.NCH + a.choff[d] + cc);
+          asm volatile("fence.proxy.async.global;" ::: "memory");  // generic-proxy writes -> the bulk copy
+        }
         bulk_load2(ring + (sg_iss & 3) * RSEG, a.devArr + sg_iss * RSEG, lring + (sg_iss & 3) * RSEG,
                    a.latd + (size_t)s * a.NS + sg_iss * RSEG, RSEG * 4, bars + (sg_iss & 3));
+      }
       sg_iss++;
     }
   };
@@ -1100,6 +1133,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   long long dbg_sec[5] = {0, 0, 0, 0, 0}, dbg_tk = 0;
   for (int64_t c0 = cstart; c0 < nch; c0 += 32) {
     ChunkSt cr = {0, 0, 0, 0};
+    if (a.cready && c0 + lane < nch) wait_chunk(a.cready, (size_t)s * a.NCH + a.choff[d] + c0 + lane);
     if (c0 + lane < nch) cr = cst[c0 + lane];
     const int cnt = nch - c0 < 32 ? (int)(nch - c0) : 32;
     for (int k = 0; k < cnt; k++) {
@@ -2851,6 +2885,74 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       if ((ngroups[rt] + 3) / 4 > 65535 || (NCH[rt] + 3) / 4 > 65535)
         return px_fail(ctx, PROTEUS_ERANGE, "too many replay chunks");
       dim3 grid((unsigned)la.nsc, (unsigned)((ngroups[rt] + 3) / 4));
+      // pipelining: the stitch runs on an auxiliary stream alongside the chunk
+      // runs and waits for each chunk it reads (ready flags), so the critical
+      // lanes start at once instead of after every chunk run of every lane
+      const bool overlap = env_int("PROTEUS_REPLAY_OVERLAP", 1) != 0 && max_rounds == 0 && !use_bscan && !la.debug &&
+                           env_int("PROTEUS_REPLAY_TABLES", 0) == 0;
+      if (overlap) {
+        unsigned *cready0 = (unsigned *)px_buf(ctx, B_R_READY, (size_t)S * nmax * 4 + (size_t)S * D * 4 + 64);
+        if (!cready0) return px_fail(ctx, PROTEUS_ENOMEM, "chunk flags");
+        unsigned *cready = cready0 + 4;  // cready[-1]: watchdog
+        PX_CUDA(ctx, cudaMemsetAsync(cready0, 0, (size_t)S * nmax * 4 + 16, ctx->stream));
+        if (!ctx->aux) {
+          // the stitch on the highest-priority stream, the chunk runs on the lowest
+          int lo = 0, hi = 0;
+          PX_CUDA(ctx, cudaDeviceGetStreamPriorityRange(&lo, &hi));
+          PX_CUDA(ctx, cudaStreamCreateWithPriority(&ctx->aux, cudaStreamNonBlocking, lo));
+          PX_CUDA(ctx, cudaStreamCreateWithPriority(&ctx->aux_hi, cudaStreamNonBlocking, hi));
+          PX_CUDA(ctx, cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming));
+          PX_CUDA(ctx, cudaEventCreateWithFlags(&ctx->ev_join, cudaEventDisableTiming));
+          PX_CUDA(ctx, cudaEventCreateWithFlags(&ctx->ev_join2, cudaEventDisableTiming));
+        }
+        la.cready = cready;
+        // stitch lanes longest first (device load, then Bmax): with the stitch on the
+        // high-priority stream they hold the SMs from the start while the chunk runs
+        // fill the rest (a stitch block needs > half an SM's shared memory, so an SM
+        // never holds two, and chunk-run blocks always fit beside it: no deadlock)
+        {
+          std::vector<int32_t> ord((size_t)la.nsc * D);
+          for (size_t i = 0; i < ord.size(); i++) ord[i] = (int32_t)i;
+          std::stable_sort(ord.begin(), ord.end(), [&](int32_t x, int32_t y) {
+            const int dx = x % D, dy = y % D;
+            const int64_t nx = h_off[rt][dx + 1] - h_off[rt][dx], ny = h_off[rt][dy + 1] - h_off[rt][dy];
+            if (nx != ny) return nx > ny;
+            return hB[(size_t)scl[2 + rt][x / D] * D + dx] > hB[(size_t)scl[2 + rt][y / D] * D + dy];
+          });
+          int32_t *d_ord = (int32_t *)(cready0 + 4 + (size_t)S * nmax);
+          PX_CUDA(ctx, cudaMemcpyAsync(d_ord, ord.data(), ord.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+          PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // ord is a host vector
+          la.lane_order = d_ord;
+        }
+        PX_CUDA(ctx, cudaEventRecord(ctx->ev_fork, ctx->stream));
+        PX_CUDA(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_fork, 0));
+        PX_CUDA(ctx, cudaStreamWaitEvent(ctx->aux_hi, ctx->ev_fork, 0));
+        cudaStream_t main = ctx->stream;
+        const int64_t warps = (int64_t)la.nsc * D;
+        int rcs = 0;
+        ctx->stream = ctx->aux;
+        px_launch_begin(ctx, "replay_spec");
+        k_spec<<<grid, 128, 0, ctx->stream>>>(la);
+        rcs = px_launch_end(ctx);
+        if (!rcs) {
+          ctx->stream = ctx->aux_hi;
+          px_launch_begin(ctx, "replay_stitch");
+          k_stitch<<<(unsigned)((warps + 3) / 4), 128, stitch_smem(ctx->bmax), ctx->stream>>>(la);
+          rcs = px_launch_end(ctx);
+        }
+        ctx->stream = main;
+        if (rcs) return rcs;
+        PX_CUDA(ctx, cudaEventRecord(ctx->ev_join, ctx->aux));
+        PX_CUDA(ctx, cudaEventRecord(ctx->ev_join2, ctx->aux_hi));
+        PX_CUDA(ctx, cudaStreamWaitEvent(ctx->stream, ctx->ev_join, 0));
+        PX_CUDA(ctx, cudaStreamWaitEvent(ctx->stream, ctx->ev_join2, 0));
+        unsigned wd = 0;
+        PX_CUDA(ctx, cudaMemcpyAsync(&wd, cready - 1, 4, cudaMemcpyDeviceToHost, ctx->stream));
+        PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+        if (wd) return px_fail(ctx, PROTEUS_EINTERNAL, "replay: pipelined stitch waited too long for a chunk run");
+        la.cready = nullptr;
+        la.lane_order = nullptr;
+      } else {
       PX_LAUNCH(ctx, "replay_spec", k_spec, grid, 128, 0, la);
       // backlogged lanes (k_spec's statistics): full-batch prefix-maximum scan
       if (use_bscan) {
@@ -2975,6 +3077,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
         }
         la.trec = nullptr; la.trecoff = nullptr; la.tE = nullptr; la.rw = nullptr;
       }
+      }  // not pipelined
     }
     }  // §5 scenarios
     if (!scl[4 + rt].empty()) {  // §8(f2) baseline batchers: chunk runs, then warp per (device, scenario)

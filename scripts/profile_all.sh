@@ -7,7 +7,7 @@ for t in c4 c5 f2 f4; do
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_$t.csv \
       python scripts/profile_target.py $t > /dev/null 2>&1; echo "list $t rc=$?"
 done
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_flat_pair -c 1 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_flat_fam -c 1 \
     -o gpurun_out/full_flat -f python scripts/profile_target.py c2 > /dev/null 2>&1; echo "full flat rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_fact_gv|k_fact_dp" -c 2 \
     -o gpurun_out/full_fact -f python scripts/profile_target.py c4 > /dev/null 2>&1; echo "full fact rc=$?"

@@ -20,9 +20,8 @@ for kind in ("poisson", "gamma"):
     sc = cfg["scenarios"]
     lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
     res = {}
-    for name, tab, minb in (("tables8", "1", "8"), ("tables4", "1", "4"), ("tables16", "1", "16"), ("no_tables", "0", "8")):
-        os.environ["PROTEUS_REPLAY_TABLES"] = tab
-        os.environ["PROTEUS_REPLAY_TABLES_MINB"] = minb
+    for name, ov in (("overlap", "1"), ("serial", "0")):
+        os.environ["PROTEUS_REPLAY_OVERLAP"] = ov
         r0 = px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
         px.set_timing(True)
         ts = []

@@ -57,6 +57,8 @@ PATHS["tables_all"] = {"PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB
 PATHS["tables_min4_chunk64"] = {"PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB": "4",
                                 "PROTEUS_REPLAY_CHUNK": "64"}
 PATHS["tables_default"] = {"PROTEUS_REPLAY_TABLES": "1"}
+PATHS["serial_spec_stitch"] = {"PROTEUS_REPLAY_OVERLAP": "0"}
+PATHS["pipelined_small_chunks"] = {"PROTEUS_REPLAY_CHUNK": "37"}
 PATHS.update({"window": {"PROTEUS_REPLAY_WINDOW": "1"},
               "window_wt1": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "1"},
               "window_wt3": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "3"},
