@@ -343,6 +343,7 @@ struct LaneArgs {
   // wait); cready[-1]: the wait watchdog fired
   unsigned *cready;
   const int32_t *lane_order;  // k_stitch: lane (list position * D + d) of warp i (null: identity)
+  int bsearch;                // k_stitch: binary-search decisions (fast_decide) on lanes with T non-decreasing
 };
 
 struct WcExit {  // a baseline chunk run left its chunk at head h (>= chunk end), device free at F;
@@ -1112,7 +1113,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   int32_t tmax = 0;
   for (int k = lane; k < p.Bmax; k += 32) tmax = T[k] > tmax ? T[k] : tmax;
   tmax = __reduce_max_sync(0xffffffffu, tmax);
-  const bool lean = p.L < LEAN_C / 2 && tmax < LEAN_C;
+  const bool lean = !(a.bsearch && p.mono) && p.L < LEAN_C / 2 && tmax < LEAN_C;
   const int32_t W0 = lane + 1 < p.Bmax ? (int32_t)p.L - T[lane + 1] : 0;
   const int32_t W1 = lane + 33 < p.Bmax ? (int32_t)p.L - T[lane + 33] : 0;
   const int32_t T0 = lane < p.Bmax ? T[lane] : 0;
@@ -1406,6 +1407,14 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
           Fn = ah + __shfl_sync(0xffffffffu, cand, sl);
           b = kb + sl + 1;
           isfree = fr < 0 || ((fb >> sl) & 1u);  // dispatched after the device freed (t > F)
+        } else if (a.bsearch && p.mono) {
+          // facts (i)-(ii) of the window path: the idle decision by binary search
+          // over the ring, or the greedy batch when the device frees after it
+          // (every lane the same probes: shared-memory broadcasts, no ballots)
+          int64_t t;
+          b = fast_decide(AR, n, h, F, p.Bmax, p.L, T, true, &t);
+          Fn = t + T[b - 1];
+          isfree = t > F;
         } else {
           const int64_t t0 = F > ah ? F : ah;
           int64_t t;
@@ -2847,6 +2856,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     la.dmask = D >= 64 ? ~0ull : ((1ull << D) - 1);
     la.lstat = d_lstat;
     la.lstart = d_lstart;
+    la.bsearch = env_int("PROTEUS_STITCH_BSEARCH", 0);
     if (la.nsc > 0) {  // §5 scenarios
     if (use_scan1) {  // Bmax = 1 lanes: exact prefix-maximum scan
       Scan1Args sa;

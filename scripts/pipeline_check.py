@@ -16,6 +16,7 @@ px.load_profiles(prof)
 sol = px.solve(cl.device_type, cl.slo_us, cfg["demand"][:1], mode=2)[0]
 arr, fam = W.query_trace(60_000, float(cfg["demand"][0].sum()), cfg["weights"], 9, "gamma")
 sc = W.scenarios_64(0)
+os.environ["PROTEUS_STITCH_BSEARCH"] = "1"
 for chunk in ("37", "64", "4096"):
     os.environ["PROTEUS_REPLAY_CHUNK"] = chunk
     os.environ["PROTEUS_REPLAY_OVERLAP"] = "0"
@@ -33,8 +34,9 @@ sol = px.solve(c5["cluster"].device_type, c5["cluster"].slo_us, c5["demand"], mo
 a = torch.from_numpy(c5["arrival_us"]).cuda()
 f = torch.from_numpy(c5["family"]).cuda()
 lat = torch.empty((64, len(a)), dtype=torch.uint32, device="cuda")
-for ov in ("0", "1"):
+for ov, bs in (("1", "0"), ("1", "1"), ("0", "1")):
     os.environ["PROTEUS_REPLAY_OVERLAP"] = ov
+    os.environ["PROTEUS_STITCH_BSEARCH"] = bs
     px.replay(a, f, sol.option, sol.z, c5["cluster"].device_type, c5["demand"][0], c5["cluster"].slo_us,
               c5["scenarios"], latency=lat)
     ts = []
@@ -46,4 +48,5 @@ for ov in ("0", "1"):
         e1.record()
         torch.cuda.synchronize()
         ts.append(e0.elapsed_time(e1))
-    print("c5 overlap", ov, "ms", [round(x, 2) for x in ts], r["violations"][:4].tolist(), flush=True)
+    print("c5 overlap", ov, "bsearch", bs, "ms", [round(x, 2) for x in ts], r["violations"][:4].tolist(),
+          int(lat[:, ::997].sum(dtype=torch.int64).item()), flush=True)

@@ -17,11 +17,20 @@ def main():
     for mode in (0, 1, 2):
         px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=mode)
     px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=0, generic=True)
+    # k_flat_fam without the symmetric states (last two devices of different types)
+    px.solve(np.array([1, 0, 1, 0], np.int32), cl.slo_us, cfg["demand"], mode=0)
+    # the device combines of the multi-GPU path (comm.cu) on 3 slices
+    parts = [px.solve_batch(cl.device_type, cl.slo_us, cfg["demand"], mode=0, shard_rank=r, shard_world=3)
+             for r in range(3)]
+    px.combine_solutions([q[0] for q in parts], [q[1] for q in parts], len(cl.device_type))
     px.solve(cl.device_type, cl.slo_us, np.repeat(cfg["demand"], 9, axis=0), mode=2)  # batched kernel
     cfg = W.config("c3", totals=(3000,))
     px.load_profiles(cfg["prof"])
     px.pareto(np.array([0, 1, 1, 2, 2], np.int32), cfg["cluster"].slo_us, 3)
     px.pareto(np.array([0, 1, 2], np.int32), cfg["cluster"].slo_us, 1, allow_idle=True)
+    pp = [px.pareto(np.array([0, 1, 1, 2], np.int32), cfg["cluster"].slo_us, 3, shard_rank=r, shard_world=2)
+          for r in range(2)]
+    px.pareto_merge(pp)
     prof, cl = cfg["prof"], cfg["cluster"]
     px.load_profiles(prof)
     sol = px.solve(cl.device_type, cl.slo_us, cfg["demand"], mode=2)[0]
@@ -38,6 +47,14 @@ def main():
     # §8(f2) baseline batchers (k_wc_lanes), mixed with §5 scenarios
     scb = np.array([[1000, 4, 0, 1], [2000, 0, 0, 2], [1500, 8, 1, 1], [3000, 0, 0, 0]], np.int32)
     px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, scb)
+    # opt-in replay paths: window path, stitch chunk tables, fused finish, binary-search stitch
+    for env in ({"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "2"},
+                {"PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB": "2"},
+                {"PROTEUS_REPLAY_FINISH": "1"}, {"PROTEUS_STITCH_BSEARCH": "1"}):
+        os.environ.update(env)
+        px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
+        for k in env:
+            os.environ.pop(k)
     os.environ["PROTEUS_REPLAY_SIMPLE"] = "1"
     px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
     os.environ.pop("PROTEUS_REPLAY_SIMPLE")
