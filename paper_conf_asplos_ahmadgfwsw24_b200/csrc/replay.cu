@@ -2169,6 +2169,7 @@ __global__ void __launch_bounds__(WIN_WARPS * 32) k_win_tables(const __grid_cons
     }
     const int Bm = p.Bmax;
     const bool mono = a.mono[(size_t)s * a.D + d] != 0;
+    __syncwarp();  // the previous lane's reads of sT / vis are done
     for (int b = lane; b < Bm; b += 32) sT[w][b] = Tg[b];
     for (int64_t i = lane; i < len; i += 32) vis[i] = 0xFF;
     __syncwarp();
@@ -2182,24 +2183,32 @@ __global__ void __launch_bounds__(WIN_WARPS * 32) k_win_tables(const __grid_cons
       int merged = -1;
       bool first = true;
       while (__any_sync(0xffffffffu, live)) {
+        // lockstep over the warp: decide, read the marks, __syncwarp, mark (one
+        // lane per head), __syncwarp -- no unordered shared-memory access
+        bool idle = false;
+        int b = 0;
+        int64_t t = 0;
+        if (live && h >= c1) live = false;
         if (live) {
-          if (h >= c1) {
-            live = false;
-          } else {
-            int64_t t;
-            int b = idle_decide(A, n, h, Bm, p.L, T, mono, &t);
-            if (first) { tdE[w][o] = t; first = false; F = t; }  // the entry: idle branch by construction
-            if (F <= t) {  // idle branch (fact (i)): a function of h alone
-              const uint8_t mk = vis[h - c0];
-              if (mk != 0xFF && mk != (uint8_t)o) { merged = mk; live = false; }
-              else vis[h - c0] = (uint8_t)o;
-              if (live) { F = t + T[b - 1]; h += b; }
-            } else {  // greedy
-              b = count_upto(A, n, h, Bm, F);
-              F = F + T[b - 1];
-              h += b;
-            }
+          b = idle_decide(A, n, h, Bm, p.L, T, mono, &t);
+          if (first) { tdE[w][o] = t; first = false; F = t; }  // the entry: idle branch by construction
+          idle = F <= t;  // idle branch (fact (i)): a function of h alone
+        }
+        const uint8_t mk = idle ? vis[h - c0] : (uint8_t)0xFF;
+        __syncwarp();
+        // another chain took h on the idle branch: the same future from here
+        if (idle && mk != 0xFF) { merged = mk; live = false; idle = false; }
+        const unsigned same = __match_any_sync(0xffffffffu, idle ? h : -1 - (int64_t)lane);
+        if (idle && lane == __ffs(same) - 1) vis[h - c0] = (uint8_t)o;
+        __syncwarp();
+        if (live) {
+          if (idle) {
+            F = t + T[b - 1];
+          } else {  // greedy
+            b = count_upto(A, n, h, Bm, F);
+            F = F + T[b - 1];
           }
+          h += b;
         }
       }
       if (o < Ee) {
@@ -2409,6 +2418,7 @@ __global__ void __launch_bounds__(WIN_THREADS) k_win_write(const __grid_constant
     }
     const int Bm = p.Bmax;
     const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+    __syncwarp();  // the previous device's reads of sT are done
     for (int b = lane; b < Bm; b += 32) sT[w][b] = Tg[b];
     __syncwarp();
     const int32_t *T = sT[w];

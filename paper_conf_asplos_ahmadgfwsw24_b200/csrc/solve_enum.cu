@@ -34,6 +34,9 @@
 #ifndef FLAT_RK
 #define FLAT_RK 1    // outer prefixes per thread per work item, in units of K
 #endif
+#ifndef FLAT_WAGG
+#define FLAT_WAGG 1  // one grid-bound atomic per warp (0: per thread)
+#endif
 #define GEN_THREADS 128
 
 // ------------------------------------------------------------ reduce ----
@@ -244,6 +247,8 @@ struct FamState {
   uint64_t F, MA, MB, J;
 };
 
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
 // SYM: devices D-2 and D-1 have the same capacities (same device type), so
 // MB = MA and the joint fills are symmetric: 1 + V + V(V+1)/2 fills instead
 // of 1 + 2V + V^2
@@ -442,7 +447,20 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_fam(const __gr
           best_s = Mx;
           best_i = o * K3 + (uint64_t)o3 * K2 + (uint64_t)(lp < 0 ? 0 : lp);
           rec = true;
-          if (Mx > G) atomicMax(gb, (unsigned long long)Mx);
+          if (Mx > G) {
+#if FLAT_WAGG
+            // raise the grid-wide bound once per warp (the largest new record
+            // among the lanes here): early in a launch every thread records,
+            // and one address per vector would serialise their atomics
+            const unsigned am = __activemask();
+            const uint32_t mh = __reduce_max_sync(am, (uint32_t)(Mx >> 32));
+            const uint32_t ml = __reduce_max_sync(am, (uint32_t)(Mx >> 32) == mh ? (uint32_t)Mx : 0u);
+            const uint64_t mv = ((uint64_t)mh << 32) | ml;
+            if (lane_id() == __ffs(__ballot_sync(am, Mx == mv)) - 1) atomicMax(gb, (unsigned long long)mv);
+#else
+            atomicMax(gb, (unsigned long long)Mx);
+#endif
+          }
         }
       }
       if (++o >= oend) break;
