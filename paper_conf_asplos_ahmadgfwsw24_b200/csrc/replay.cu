@@ -26,6 +26,8 @@
 // a13: k_count reduces the final latency rows to per-scenario violations,
 // on-time counts and accuracy sums.
 #include <algorithm>
+#include <array>
+#include <utility>
 #include <climits>
 #include <cstdlib>
 #include <cstring>
@@ -344,6 +346,7 @@ struct LaneArgs {
   unsigned *cready;
   const int32_t *lane_order;  // k_stitch: lane (list position * D + d) of warp i (null: identity)
   int bsearch;                // k_stitch: binary-search decisions (fast_decide) on lanes with T non-decreasing
+  const uint8_t *skip;        // [S * D] 1: the chunk / lane kernels leave the lane alone (a duplicate lane, or k_chain's)
 };
 
 struct WcExit {  // a baseline chunk run left its chunk at head h (>= chunk end), device free at F;
@@ -509,6 +512,7 @@ __global__ void __launch_bounds__(128) k_wc_spec(const __grid_constant__ LaneArg
   int d = 0;
   while (cg >= a.choff[d + 1]) d++;
   const int s = a.sc_list[blockIdx.x];
+  if (a.skip && a.skip[s * a.D + d]) return;
   const LaneParam p = a.lp[s * a.D + d];
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t c = cg - a.choff[d];
@@ -574,6 +578,7 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
   const int w = threadIdx.x >> 5;
   if (wid >= a.nsc * a.D) return;
   const int s = a.sc_list[wid / a.D], d = wid % a.D;
+  if (a.skip && a.skip[s * a.D + d]) return;
   const LaneParam p = a.lp[s * a.D + d];
   const int64_t st = a.devOff[d], n = a.devOff[d + 1] - st;
   if (n == 0) return;
@@ -811,7 +816,7 @@ __global__ void __launch_bounds__(128) k_spec(const __grid_constant__ LaneArgs a
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
   const int64_t c = (int64_t)(g - sG[d]) * 32 + lane;
-  if (c >= nch || (a.scan1 && p.Bmax == 1)) return;
+  if (c >= nch || (a.scan1 && p.Bmax == 1) || (a.skip && a.skip[s * a.D + d])) return;
   const int64_t st = c * a.CH, en = st + a.CH < n ? st + a.CH : n;
   uint32_t *out = a.latd + (size_t)s * a.NS + off;
   int64_t h = st, F = 0, eF = 0, edh = 0;
@@ -1031,7 +1036,7 @@ __global__ void __launch_bounds__(128) k_stitch(const __grid_constant__ LaneArgs
   const LaneParam p = a.lp[s * a.D + d];
   const int64_t off = a.devOff[d], n = a.devOff[d + 1] - off;
   const int64_t nch = a.choff[d + 1] - a.choff[d];
-  if (p.Bmax < 1 || nch < 2 || (a.scan1 && p.Bmax == 1)) return;
+  if (p.Bmax < 1 || nch < 2 || (a.scan1 && p.Bmax == 1) || (a.skip && a.skip[s * a.D + d])) return;
   uint32_t *wsm = ssm + (size_t)w * stitch_wstride(a.bmax);
   uint32_t *ring = wsm;
   uint32_t *lring = wsm + RING;
@@ -1948,10 +1953,10 @@ __global__ void k_sink(int64_t NS, int S, int D, const int32_t *__restrict__ sc_
 #define CNT_PER 16384
 __global__ void __launch_bounds__(256) k_count(int64_t N, int64_t NS, int S, int D, const int32_t *__restrict__ sc_list,
                                                const int64_t *__restrict__ devOff, const LaneParam *__restrict__ lp,
-                                               const uint32_t *__restrict__ latd, uint64_t *agg) {
+                                               const int32_t *__restrict__ rep, const uint32_t *__restrict__ latd,
+                                               uint64_t *agg) {
   __shared__ unsigned long long red[3][8];
   const int s = sc_list[blockIdx.y];
-  const uint32_t *row = latd + (size_t)s * NS;
   const int64_t lo = (int64_t)blockIdx.x * CNT_PER, hi = lo + CNT_PER < N ? lo + CNT_PER : N;
   unsigned long long viol = 0, accs = 0, ont_all = 0;
   for (int d = 0; d <= D; d++) {
@@ -1962,6 +1967,7 @@ __global__ void __launch_bounds__(256) k_count(int64_t N, int64_t NS, int S, int
       continue;
     }
     const LaneParam q = lp[(size_t)s * D + d];
+    const uint32_t *row = latd + (size_t)(rep ? rep[(size_t)s * (D + 1) + d] : s) * NS;  // a duplicate lane: its row's
     const uint32_t L = q.L < 0 ? 0u : q.L > 0xFFFFFFFEll ? 0xFFFFFFFFu : (uint32_t)q.L;
     const bool all_on = q.L >= 0xFFFFFFFFll;  // every latency (<= UINT32_MAX) is on time
     unsigned ont = 0;
@@ -1996,6 +2002,24 @@ __global__ void __launch_bounds__(256) k_count(int64_t N, int64_t NS, int S, int
     if (o2) atomicAdd((unsigned long long *)&agg[S + s], o2);
     if (a2) atomicAdd((unsigned long long *)&agg[2 * S + s], a2);
   }
+}
+
+// duplicate lanes (same policy, Bmax and SLO on a device as an earlier
+// scenario): the representative's row segment copied into the duplicate's
+// row; blockIdx.y = pair k (dup[k], src[k], device dev[k]).  Both rows share
+// the segment's offset, so the body moves in 16-byte words.
+__global__ void __launch_bounds__(256) k_dupcopy(int64_t NS, const int32_t *__restrict__ pairs,
+                                                 const int64_t *__restrict__ devOff, uint32_t *latd) {
+  const int32_t dst = pairs[3 * blockIdx.y], src = pairs[3 * blockIdx.y + 1], d = pairs[3 * blockIdx.y + 2];
+  const int64_t a0 = devOff[d], a1 = devOff[d + 1];
+  const uint32_t *in = latd + (size_t)src * NS;
+  uint32_t *o = latd + (size_t)dst * NS;
+  const int64_t b0 = ((a0 + 3) & ~(int64_t)3) < a1 ? ((a0 + 3) & ~(int64_t)3) : a1;
+  const int64_t b1 = b0 + ((a1 - b0) & ~(int64_t)3);
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x, nt = (int64_t)gridDim.x * blockDim.x;
+  if (t < b0 - a0) o[a0 + t] = in[a0 + t];
+  if (t < a1 - b1) o[b1 + t] = in[b1 + t];
+  for (int64_t p = b0 + 4 * t; p < b1; p += 4 * nt) *(uint4 *)(o + p) = *(const uint4 *)(in + p);
 }
 
 // per-query order: out[s][i] = latd[s][inv(i)] (coalesced stores, gathered loads
@@ -2580,6 +2604,411 @@ __global__ void __launch_bounds__(256) k_finish(int64_t N, int64_t NS, int S, in
   }
 }
 
+// ---- chain path: the §5 lanes as a chained scan over chunk maps
+// For a lane with T(b) non-decreasing (facts (i)-(ii) of the window path), the
+// decision at head h with the device free at F is the idle decision
+// (b_i(h), t_i(h)) when F <= t_i(h), else the greedy batch min(Bmax, queued at
+// F) at F.  The idle decision depends on h only, so a chunk of C heads is
+// tabulated in parallel (one binary search per head), and so is, for every
+// head i, the rest of the run after an idle-branch decision at i: the next
+// head at which the run decides on the idle branch again (the greedy batches
+// between are a function of i too), or the state (head >= chunk end, free
+// time) in which it leaves the chunk.  A chunk's exit is then a function of
+// its entry: an entry on the idle branch at head h leaves where the chain of
+// h leaves (every chain's end is found beforehand by pointer jumping); a busy
+// entry first takes its greedy batches.  Units (lane, chunk) are taken in chunk-major ticket order by
+// persistent blocks; each builds its tables, then waits for the previous
+// chunk's exit (a single 64-bit word: ((F + 1) << 8) | (head - chunk start)),
+// publishes its own, and only then walks its chunk once from the true entry to
+// write the latencies (device-major rows, like the chunk runs).  The serial
+// dependency per lane is one table lookup per chunk.
+#define CHAIN_THREADS 256
+#define CHAIN_WARPS (CHAIN_THREADS / 32)
+#define CHAIN_CMAX 8192  // largest chunk (heads are int16 in the tables)
+#ifdef PX_CHAIN_DEBUG  // per-phase cycle totals of k_chain (thread 0), printed by the host
+#define CX_T(k) do { if (threadIdx.x == 0) { const long long t_ = clock64(); atomicAdd(a.dbg + (k), (unsigned long long)(t_ - cx_t)); cx_t = t_; } } while (0)
+#else
+#define CX_T(k) do { } while (0)
+#endif
+struct ChainArgs {
+  int D, M, bmax, nl, C;
+  int K;                       // greedy batches a head's chain follows in the tables
+  int64_t NS, maxch, nunits;   // tickets: c * nl + li (chunk-major)
+  const int32_t *lid;          // [nl] lane = s * D + d (device-major: consecutive tickets share arrivals)
+  const int32_t *nch;          // [nl] chunks of the lane
+  const uint8_t *cmode;        // [nl] 0: chunk tables, 1: near overload (full-batch walks, no tables)
+  const LaneParam *lp;
+  const int32_t *option, *dev_type, *lat;
+  const int64_t *devOff;
+  const uint32_t *devArr;
+  uint32_t *latd;
+  unsigned long long *ex;      // [nl][maxch] packed chunk exits, 0 = not yet published
+  unsigned long long *counter; // ticket counter
+  unsigned *watchdog;          // set when a wait for a previous chunk's exit times out
+  unsigned long long *dbg;     // PX_CHAIN_DEBUG: [16] phase cycles, units, batches, jump rounds
+};
+
+struct ShArr {  // arrivals of a chunk in shared memory, from its first head
+  const uint32_t *p;
+  __device__ __forceinline__ uint32_t operator()(int64_t j) const { return p[j]; }
+};
+
+// per routing mode: lid [nl] i32, nch [nl] i32, cmode [nl] u8, ticket + watchdog, exits [nl][maxch] u64
+static size_t chain_ctroff(size_t nl) { return (nl * 9 + 15) & ~(size_t)15; }
+static size_t chain_exoff(size_t nl) { return chain_ctroff(nl) + 16; }
+static size_t chain_smem(int C, int bmax) {
+  const size_t E = (size_t)C + bmax + 2;
+  return (size_t)C * 8 /* sFx */ + (size_t)bmax * 4 /* sT */ + E * 4 /* sA */ + (size_t)C * 4 /* sTi */ +
+         (size_t)C * 4 /* sFi */ + (size_t)C * 6 /* sNx, sJ[2] */ + (size_t)C /* sB */ + (size_t)C /* sHx */ + 64;
+}
+
+__global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__ ChainArgs a) {
+  extern __shared__ __align__(16) unsigned char csm[];
+  const int C = a.C;
+  int64_t *sFx = (int64_t *)csm;                    // [C] exit free time of an exiting chain
+  int32_t *sT = (int32_t *)(sFx + C);               // [bmax] T(b) at b - 1
+  uint32_t *sA = (uint32_t *)(sT + a.bmax);         // [C + bmax + 2] arrivals from the chunk start
+  int32_t *sTi = (int32_t *)(sA + C + a.bmax + 2);  // [C] t_i(h) - a_h
+  int32_t *sFi = sTi + C;                           // [C] t_i(h) + T(b_i(h)) - a_h: the idle batch's finish
+  int16_t *sNx = (int16_t *)(sFi + C);              // [C] next idle-branch head of the chain of h, -1: leaves, -2: left to the walk
+  int16_t *sJa = sNx + C, *sJb = sJa + C;          // [2][C] last idle-branch head of the chain of h (double buffer)
+  uint8_t *sB = (uint8_t *)(sJb + C);               // [C] b_i(h)
+  uint8_t *sHx = sB + C;                            // [C] exit head - chunk end of an exiting chain
+  __shared__ unsigned long long sTicket;
+  __shared__ uint32_t sVis[CHAIN_CMAX / 32];  // idle-branch batch starts of the speculative walks
+  __shared__ int sSx[CHAIN_WARPS], sEnt;       // speculative walks' exit heads; the true entry
+  __shared__ int64_t sSF[CHAIN_WARPS], sEntF;  // ... and free times
+  const int tid = threadIdx.x;
+  for (;;) {
+    if (tid == 0) sTicket = atomicAdd(a.counter, 1ull);
+    __syncthreads();
+    const unsigned long long tk = sTicket;
+    if (tk >= (unsigned long long)a.nunits) return;
+    const int li = (int)(tk % (unsigned long long)a.nl);
+    const int64_t c = (int64_t)(tk / (unsigned long long)a.nl);
+    if (c < a.nch[li]) {
+#ifdef PX_CHAIN_DEBUG
+      long long cx_t = clock64();
+#endif
+      const int lane_id = a.lid[li];
+      const int s = lane_id / a.D, d = lane_id % a.D;
+      const LaneParam p = a.lp[lane_id];
+      const int Bm = p.Bmax;
+      const int64_t off = a.devOff[d], nloc0 = a.devOff[d + 1] - off;
+      const int64_t c0 = c * C;
+      const int64_t nloc = nloc0 - c0;  // heads from the chunk start to the device's end
+      const int Cn = (int)(nloc < C ? nloc : C);
+      const int na = (int)(nloc < (int64_t)Cn + Bm + 1 ? nloc : (int64_t)Cn + Bm + 1);
+      const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+      for (int k = tid; k < Bm; k += CHAIN_THREADS) sT[k] = Tg[k];
+      const uint32_t *src = a.devArr + off + c0;
+      for (int j = tid; j < na; j += CHAIN_THREADS) sA[j] = src[j];
+      __syncthreads();
+      CX_T(0);
+      const ShArr A{sA};
+      const int w = tid >> 5, lane = tid & 31;
+      const int64_t TB = sT[Bm - 1];
+      uint32_t *out = a.latd + (size_t)s * a.NS + off + c0;
+      // full-batch stretch at (hh, FF): batch i (head hh + i Bm) leaves full at
+      // FF + i T(Bmax) while its last query has arrived by then -- with Bmax
+      // queued when the device frees, the decision is Bmax at that instant
+      // whether or not the idle run would have dispatched earlier.  Returns
+      // the number of such batches whose heads lie below lim (32 per ballot).
+      auto stretch = [&](int hh, int64_t FF, int lim) -> int {
+        int k = 0;
+        for (;;) {
+          const int i = k + lane;
+          const int64_t last = (int64_t)hh + (int64_t)(i + 1) * Bm - 1;
+          const bool full = (int64_t)hh + (int64_t)i * Bm < lim && last < nloc &&
+                            (int64_t)sA[last] <= FF + (int64_t)i * TB;
+          const unsigned bal = __ballot_sync(0xffffffffu, !full);
+          if (bal) return k + __ffs(bal) - 1;
+          k += 32;
+        }
+      };
+      // latencies of the batch [hh, hh + b) finishing at fin, positions < lim
+      auto put = [&](int hh, int b, int64_t fin, int lim) {
+        const int e = hh + b < lim ? hh + b : lim;
+        for (int j = hh + lane; j < e; j += 32) out[j] = sat_lat(fin - (int64_t)sA[j]);
+      };
+      // the chunk's entry (warp 0): R13 for the first chunk, else the previous
+      // chunk's exit, a single 64-bit word ((F + 1) << 8 | head - chunk start)
+      auto entry = [&](int &h, int64_t &F) {
+        if (c == 0) {
+          h = 0;
+          F = 0;  // R13: the device starts idle
+          return;
+        }
+        unsigned long long v = 0;
+        if (lane == 0) {
+          const unsigned long long *pe = a.ex + (size_t)li * a.maxch + (c - 1);
+          for (uint32_t it = 0;; it++) {
+            asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(pe) : "memory");
+            if (v) break;
+            if (it > (1u << 24)) { atomicExch(a.watchdog, 1u); v = 1ull << 8; break; }
+            __nanosleep(32);
+          }
+        }
+        v = __shfl_sync(0xffffffffu, v, 0);
+        h = (int)(v & 255u);
+        F = (int64_t)(v >> 8) - 1;
+      };
+      auto publish = [&](int hx, int64_t Fx) {
+        if (lane == 0) {
+          const unsigned long long v = ((unsigned long long)(Fx + 1) << 8) | (unsigned long long)hx;
+          asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(a.ex + (size_t)li * a.maxch + c), "l"(v) : "memory");
+        }
+      };
+      if (a.cmode[li]) {
+        // a lane near overload: mostly full batches back to back, taken 32 per
+        // ballot; the other decisions directly (idle decision by binary
+        // search, else the greedy batch).  No tables: warp 0 walks the chunk
+        // from its entry and then publishes the exit.
+        if (w == 0) {
+          int hh;
+          int64_t FF;
+          entry(hh, FF);
+          CX_T(4);
+          long long nbat = 0;
+          while (hh < Cn) {
+            const int k = stretch(hh, FF, Cn);
+            if (k > 0) {
+              const int np = k * Bm;
+              for (int j = lane; j < np; j += 32) out[hh + j] = sat_lat(FF + (int64_t)(j / Bm + 1) * TB - (int64_t)sA[hh + j]);
+              nbat += k;
+              hh += np;
+              FF += (int64_t)k * TB;
+              continue;
+            }
+            int64_t t;
+            int b = idle_decide(A, nloc, (int64_t)hh, Bm, p.L, sT, true, &t);
+            int64_t fin;
+            if (FF <= t) fin = t + sT[b - 1];
+            else { b = count_upto(A, nloc, (int64_t)hh, Bm, FF); fin = FF + sT[b - 1]; }
+            put(hh, b, fin, INT32_MAX);
+            nbat++;
+            hh += b;
+            FF = fin;
+          }
+          publish(hh - Cn, FF);
+          CX_T(6);
+#ifdef PX_CHAIN_DEBUG
+          if (lane == 0) {
+            atomicAdd(a.dbg + 8, 1ull);
+            atomicAdd(a.dbg + 9, (unsigned long long)nbat);
+            atomicAdd(a.dbg + 11, 1ull);
+          }
+#else
+          (void)nbat;
+#endif
+        }
+      } else {
+      // idle decisions of every head (fact (ii): binary search)
+      for (int i = tid; i < Cn; i += CHAIN_THREADS) {
+        int64_t t;
+        const int b = idle_decide(A, nloc, (int64_t)i, Bm, p.L, sT, true, &t);
+        sB[i] = (uint8_t)b;
+        sTi[i] = (int32_t)(t - (int64_t)sA[i]);
+        sFi[i] = (int32_t)(t + sT[b - 1] - (int64_t)sA[i]);
+      }
+      __syncthreads();
+      CX_T(1);
+      // greedy batch at (hh, F), the device free at F after the idle decision
+      // would have dispatched: min(Bmax, queued at F), Bmax without a search
+      // when the Bmax-th query is already there
+      auto greedy = [&](int hh, int64_t F) -> int {
+        return ((int64_t)hh + Bm - 1 < nloc && (int64_t)sA[hh + Bm - 1] <= F) ? Bm
+                                                                               : count_upto(A, nloc, (int64_t)hh, Bm, F);
+      };
+      // the chain of every head after its idle-branch decision (at most K
+      // greedy batches are followed here: -2 marks a head whose chain is left
+      // to the serial walk -- backlogged stretches would make this quadratic)
+      for (int i = tid; i < Cn; i += CHAIN_THREADS) {
+        int64_t F = (int64_t)sA[i] + sFi[i];
+        int hh = i + sB[i];
+        for (int st = 0;; st++) {
+          if (hh >= Cn) { sNx[i] = -1; sHx[i] = (uint8_t)(hh - Cn); sFx[i] = F; break; }
+          if (F <= (int64_t)sA[hh] + sTi[hh]) { sNx[i] = (int16_t)hh; break; }
+          if (st >= a.K) { sNx[i] = -2; break; }
+          const int g = greedy(hh, F);  // dispatched at F
+          F += sT[g - 1];
+          hh += g;
+        }
+      }
+      __syncthreads();
+      CX_T(2);
+      // the last idle-branch head of every chain (pointer jumping, double
+      // buffered: the last head is a fixed point)
+      int16_t *sJ = sJa, *sJn = sJb;
+      for (int i = tid; i < Cn; i += CHAIN_THREADS) sJ[i] = sNx[i] >= 0 ? sNx[i] : (int16_t)i;
+      for (bool more = true; more;) {
+        __syncthreads();
+        bool ch = false;
+        for (int i = tid; i < Cn; i += CHAIN_THREADS) {
+          const int j = sJ[i], jj = sJ[j];
+          sJn[i] = (int16_t)jj;
+          ch |= jj != j;
+        }
+        int16_t *t_ = sJ;
+        sJ = sJn;
+        sJn = t_;
+        more = __syncthreads_or(ch);
+#ifdef PX_CHAIN_DEBUG
+        if (tid == 0) atomicAdd(a.dbg + 10, 1ull);
+#endif
+      }
+      CX_T(3);
+      // segments for the speculative walks of warps 1..7 (the true run enters
+      // below Bmax, so segments starting at or past Bmax never hold positions
+      // of the previous chunk's last batch)
+      const bool spec = Cn / CHAIN_WARPS >= Bm;
+      auto seg0 = [&](int k) { return (int)(((int64_t)k * Cn) / CHAIN_WARPS); };
+      for (int k = tid; k < (Cn + 31) / 32; k += CHAIN_THREADS) sVis[k] = 0u;
+      __syncthreads();
+      if (w == 0) {  // the link: this chunk's exit from its entry
+        int h;
+        int64_t F;
+        entry(h, F);
+        CX_T(4);
+        // greedy batches, then the chain of the first idle-branch head (chains
+        // left to the serial walk are continued here)
+        int hh = h;
+        int64_t FF = F;
+        int hx;
+        int64_t Fx;
+        for (;;) {
+          if (hh >= Cn) { hx = hh - Cn; Fx = FF; break; }
+          const int64_t ti = (int64_t)sA[hh] + sTi[hh];
+          if (FF <= ti) {
+            const int r = sJ[hh];
+            if (sNx[r] == -1) { hx = sHx[r]; Fx = sFx[r]; break; }
+            FF = (int64_t)sA[r] + sFi[r];
+            hh = r + sB[r];
+            continue;
+          }
+          const int k = stretch(hh, FF, Cn);
+          if (k > 0) { hh += k * Bm; FF += (int64_t)k * TB; continue; }
+          const int g = count_upto(A, nloc, (int64_t)hh, Bm, FF);
+          FF += sT[g - 1];
+          hh += g;
+        }
+        publish(hx, Fx);
+        if (lane == 0) {
+          sEnt = h;
+          sEntF = F;
+        }
+        CX_T(5);
+      } else if (spec) {
+        // speculative walk of segment w from an idle device at its first head:
+        // latencies of its positions, its idle-branch batch starts (sVis) and
+        // its exit (first head past the segment, free time)
+        const int S0 = seg0(w), S1 = seg0(w + 1);
+        int hh = S0;
+        int64_t FF = INT64_MIN / 4;
+        while (hh < S1) {
+          if (FF <= (int64_t)sA[hh] + sTi[hh]) {
+            for (;;) {
+              const int b = sB[hh];
+              const int64_t fin = (int64_t)sA[hh] + sFi[hh];
+              if (lane == 0) atomicOr(&sVis[hh >> 5], 1u << (hh & 31));
+              put(hh, b, fin, S1);
+              const int nx = sNx[hh];
+              if (nx == hh + b && nx < S1) { hh = nx; continue; }
+              hh += b;
+              FF = fin;
+              break;
+            }
+            continue;
+          }
+          const int k = stretch(hh, FF, S1);
+          if (k > 0) {
+            const int np = k * Bm, e = hh + np < S1 ? hh + np : S1;
+            for (int j = hh + lane; j < e; j += 32) out[j] = sat_lat(FF + (int64_t)((j - hh) / Bm + 1) * TB - (int64_t)sA[j]);
+            hh += np;
+            FF += (int64_t)k * TB;
+            continue;
+          }
+          const int b = count_upto(A, nloc, (int64_t)hh, Bm, FF);
+          const int64_t fin = FF + sT[b - 1];
+          put(hh, b, fin, S1);
+          hh += b;
+          FF = fin;
+        }
+        if (lane == 0) { sSx[w] = hh; sSF[w] = FF; }
+      }
+      __syncthreads();
+      if (w == 0) {
+        // the true run through the chunk: latencies of [entry, exit head); in a
+        // segment of a speculative walk it stops at the first idle-branch batch
+        // start the walk also had (both then take the same decisions) and takes
+        // the walk's exit, writing the positions of the walk's last batch past
+        // the segment
+        long long nbat = 0;
+        int hh = sEnt;
+        int64_t FF = sEntF;
+        auto merge = [&](int x) -> int {  // segment whose speculative walk had an idle start at x, or 0
+          if (!spec || !((sVis[x >> 5] >> (x & 31)) & 1u)) return 0;
+          int k = (int)(((int64_t)x * CHAIN_WARPS) / Cn);
+          while (k + 1 < CHAIN_WARPS && seg0(k + 1) <= x) k++;
+          while (seg0(k) > x) k--;
+          return k;
+        };
+        while (hh < Cn) {
+          if (FF <= (int64_t)sA[hh] + sTi[hh]) {
+            const int m = merge(hh);
+            if (m > 0) {
+              const int S1 = seg0(m + 1), hx = sSx[m];
+              const int64_t Fx = sSF[m];
+              for (int j = S1 + lane; j < hx; j += 32) out[j] = sat_lat(Fx - (int64_t)sA[j]);
+              hh = hx;
+              FF = Fx;
+              continue;
+            }
+            for (;;) {
+              const int b = sB[hh];
+              const int64_t fin = (int64_t)sA[hh] + sFi[hh];
+              put(hh, b, fin, INT32_MAX);
+              nbat++;
+              const int nx = sNx[hh];
+              if (nx == hh + b && merge(nx) == 0) { hh = nx; continue; }
+              hh += b;
+              FF = fin;
+              break;
+            }
+            continue;
+          }
+          const int k = stretch(hh, FF, Cn);
+          if (k > 0) {
+            const int np = k * Bm;
+            for (int j = lane; j < np; j += 32) out[hh + j] = sat_lat(FF + (int64_t)(j / Bm + 1) * TB - (int64_t)sA[hh + j]);
+            nbat += k;
+            hh += np;
+            FF += (int64_t)k * TB;
+            continue;
+          }
+          const int b = count_upto(A, nloc, (int64_t)hh, Bm, FF);
+          const int64_t fin = FF + sT[b - 1];
+          put(hh, b, fin, INT32_MAX);
+          nbat++;
+          hh += b;
+          FF = fin;
+        }
+        CX_T(6);
+#ifdef PX_CHAIN_DEBUG
+        if (lane == 0) {
+          atomicAdd(a.dbg + 8, 1ull);
+          atomicAdd(a.dbg + 9, (unsigned long long)nbat);
+        }
+#else
+        (void)nbat;
+#endif
+      }
+      }  // tables
+    }
+    __syncthreads();  // shared tables and sTicket are rewritten by the next unit
+  }
+}
+
 // ---------------------------------------------------------------- host ----
 static int env_int(const char *name, int dflt) {
   const char *v = getenv(name);
@@ -2808,9 +3237,13 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   // fix-up rounds before the sequential stitch finishes whatever is left
   const int max_rounds = env_int("PROTEUS_REPLAY_ROUNDS", 0);
   int64_t h_off[2][PX_MAXD + 2];
+  memset(h_off, 0, sizeof h_off);
   for (int rt = 0; rt < 2; rt++)
     if (devOff[rt])
       PX_CUDA(ctx, cudaMemcpyAsync(h_off[rt], devOff[rt], (D + 2) * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  uint32_t h_span[2] = {0, 0};  // first and last arrival (the chain path's rate estimate)
+  PX_CUDA(ctx, cudaMemcpyAsync(&h_span[0], d_arr, 4, cudaMemcpyDeviceToHost, ctx->stream));
+  PX_CUDA(ctx, cudaMemcpyAsync(&h_span[1], d_arr + (N - 1), 4, cudaMemcpyDeviceToHost, ctx->stream));
   PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
   int64_t NCH[2] = {0, 0};
   int32_t ngroups[2] = {0, 0};
@@ -2828,6 +3261,154 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   }
   PX_CUDA(ctx, cudaMemcpyAsync(d_choff, choff.data(), choff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
   PX_CUDA(ctx, cudaMemcpyAsync(d_goff, goff.data(), goff.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+  // chain path (k_chain): the §5 lanes with T non-decreasing, 2 <= Bmax <= 255
+  // and L < 2^30; the chunk runs + stitch take the other lanes
+  const bool use_scan1 = !simple && env_int("PROTEUS_REPLAY_SCAN1", 1) != 0;
+  const bool use_chain = !simple && env_int("PROTEUS_REPLAY_CHAIN", 0) != 0 && max_rounds == 0 &&
+                         env_int("PROTEUS_REPLAY_BSCAN", 0) == 0 && env_int("PROTEUS_REPLAY_TABLES", 0) == 0;
+  int CHN = env_int("PROTEUS_REPLAY_CHAIN_C", 2048);
+  CHN = CHN < 256 ? 256 : CHN > CHAIN_CMAX ? CHAIN_CMAX : CHN;  // shared-memory tables (~24 B per head)
+  const int chain_minb = std::max(2, env_int("PROTEUS_REPLAY_CHAIN_MINB", 2));
+  std::vector<int32_t> clid[2], cnch[2];
+  std::vector<uint8_t> cmodev[2];
+  int64_t cmax[2] = {0, 0};
+  bool crest[2] = {true, true};  // lanes left to the chunk runs + stitch
+  uint8_t *d_chainf = nullptr;  // skip flags [S][D]
+  int32_t *d_rep = nullptr;      // row map [S][D + 1] (null: every lane its own row)
+  int32_t *d_pairs[2] = {nullptr, nullptr};  // (duplicate, representative, device) per routing mode
+  int64_t npair[2] = {0, 0};
+  char *cbuf[2] = {nullptr, nullptr};  // per routing mode (chain_exoff)
+  // Lanes (scenario, device) with the same policy, Bmax and SLO on a device
+  // see the same arrivals under the same rule: one of them (the first
+  // scenario) is replayed and the others read its row (rep[s][d], the row
+  // holding lane (s, d); rep[s][D] = s for the sink).  skip[s][d]: the chunk
+  // kernels leave the lane alone (a duplicate, or a chain lane).
+  const bool dedup = !simple && !use_win && max_rounds == 0 && env_int("PROTEUS_REPLAY_DEDUP", 1) != 0 &&
+                     env_int("PROTEUS_REPLAY_BSCAN", 0) == 0 && env_int("PROTEUS_REPLAY_TABLES", 0) == 0 &&
+                     env_int("PROTEUS_REPLAY_FINISH", 0) == 0 && env_int("PROTEUS_REPLAY_DEBUG", 0) == 0;
+  std::vector<int32_t> hrep((size_t)S * (D + 1));
+  std::vector<uint8_t> hskip((size_t)S * D, 0);
+  for (int s = 0; s < S; s++)
+    for (int d = 0; d <= D; d++) hrep[(size_t)s * (D + 1) + d] = s;
+  auto lane_L = [&](int s, int d) -> int64_t {
+    return (int64_t)h_sc[s].slo_mult_milli * h_slo[ctx->fam[h_option[d] - 1]] / 1000;
+  };
+  if (dedup) {
+    for (int rt = 0; rt < 2; rt++)
+      for (int d = 0; d < D; d++) {
+        if (h_option[d] <= 0) continue;
+        std::vector<std::pair<std::array<int64_t, 3>, int>> seen;
+        for (int s : scl[rt]) {
+          const int B = hB[(size_t)s * D + d];
+          if (h_sc[s].policy == 0 && B == 1 && use_scan1) continue;  // the Bmax = 1 scan writes every row
+          const std::array<int64_t, 3> key = {h_sc[s].policy, B, lane_L(s, d)};
+          int r = -1;
+          for (auto &e : seen) if (e.first == key) { r = e.second; break; }
+          if (r < 0) { seen.push_back({key, s}); continue; }
+          hrep[(size_t)s * (D + 1) + d] = r;
+          hskip[(size_t)s * D + d] = 1;
+        }
+      }
+  }
+  if (use_chain) {
+    // lanes whose idle batches are large: b^ = the largest b <= Bmax with
+    // 1 + lambda (L - T(b + 1)) >= b (the queries arriving while the head
+    // waits, lambda = the device's mean rate).  Small-batch lanes have long
+    // serial walks per chunk here, while their chunk runs meet the true run at
+    // once (the stitch accepts them), so they stay on the chunk runs + stitch.
+    const double minbatch = (double)env_int("PROTEUS_REPLAY_CHAIN_MINBATCH", 16);
+    const double minrho = (double)env_int("PROTEUS_REPLAY_CHAIN_RHO_PCT", 100) / 100.0;
+    const double span = (double)h_span[1] - (double)h_span[0];
+    std::vector<uint8_t> hchain((size_t)S * D, 0);
+    for (int s = 0; s < S; s++) {
+      if (is_win[s] || h_sc[s].policy != 0) continue;
+      for (int d = 0; d < D; d++) {
+        if (h_option[d] <= 0 || hskip[(size_t)s * D + d]) continue;
+        const int B = hB[(size_t)s * D + d];
+        const int64_t L = lane_L(s, d);
+        if (B < chain_minb || B > 255 || !hmono[(size_t)s * D + d] || L >= (1ll << 30)) continue;
+        const int32_t *Tr = ctx->lat.data() + ((size_t)h_dev_type[d] * M + (h_option[d] - 1)) * ctx->bmax;
+        if (Tr[B - 1] >= (1 << 30)) continue;  // 32-bit idle finishes in the chunk tables
+        const int rt = h_sc[s].routing;
+        const int64_t nd = h_off[rt][d + 1] - h_off[rt][d];
+        const double lam = span > 0 ? (double)nd / span : 1e30;
+        int bh = 1;
+        for (int b = 1; b <= B; b++)
+          if (1.0 + lam * (double)(L - Tr[b < B ? b : B - 1]) >= (double)b) bh = b;
+        // ... or lanes at or past overload at their batch cap (full batches
+        // back to back: the chain walks them 32 batches per ballot)
+        const double rho = lam * (double)Tr[B - 1] / (double)B;
+        if (rho >= minrho) hchain[(size_t)s * D + d] = 2;
+        else if (bh >= minbatch) hchain[(size_t)s * D + d] = 1;
+        if (hchain[(size_t)s * D + d]) hskip[(size_t)s * D + d] = 1;
+      }
+    }
+    for (int rt = 0; rt < 2; rt++) {
+      if (!devOff[rt]) continue;
+      bool rest = false;
+      for (int d = 0; d < D; d++) {
+        const int64_t nd = h_off[rt][d + 1] - h_off[rt][d];
+        for (int k : scl[2 + rt]) {
+          const size_t l = (size_t)k * D + d;
+          if (nd > 0 && hchain[l]) {
+            clid[rt].push_back((int32_t)l);
+            cnch[rt].push_back((int32_t)((nd + CHN - 1) / CHN));
+            cmodev[rt].push_back((uint8_t)(hchain[l] - 1));
+            cmax[rt] = std::max(cmax[rt], (int64_t)cnch[rt].back());
+          } else if (nd > 0 && !hskip[l] && !(use_scan1 && hB[l] == 1)) {
+            rest = true;
+          }
+        }
+      }
+      crest[rt] = rest;
+    }
+  }
+  if (!simple) {  // skip flags, row map and the chain lists in one buffer
+    const size_t o_rep = ((size_t)S * D + 15) & ~(size_t)15;
+    const size_t o_pr = o_rep + (((size_t)S * (D + 1) * 4 + 15) & ~(size_t)15);
+    std::vector<int32_t> hpairs[2];
+    for (int rt = 0; rt < 2; rt++)
+      for (int s : scl[rt])
+        for (int d = 0; d < D; d++)
+          if (hrep[(size_t)s * (D + 1) + d] != s) {
+            hpairs[rt].push_back(s);
+            hpairs[rt].push_back(hrep[(size_t)s * (D + 1) + d]);
+            hpairs[rt].push_back(d);
+          }
+    const size_t o_ch = o_pr + ((hpairs[0].size() + hpairs[1].size()) * 4 + 15) / 16 * 16;
+    size_t part[2] = {0, 0}, need = o_ch;
+    for (int rt = 0; rt < 2; rt++) {
+      const size_t nl = clid[rt].size();
+      if (nl) part[rt] = chain_exoff(nl) + nl * (size_t)cmax[rt] * 8;
+      need += part[rt];
+    }
+    char *cb = (char *)px_buf(ctx, B_R_CHAIN, need + 64);
+    if (!cb) return px_fail(ctx, PROTEUS_ENOMEM, "lane tables");
+    d_chainf = (uint8_t *)cb;
+    d_rep = (int32_t *)(cb + o_rep);
+    PX_CUDA(ctx, cudaMemcpyAsync(d_chainf, hskip.data(), hskip.size(), cudaMemcpyHostToDevice, ctx->stream));
+    PX_CUDA(ctx, cudaMemcpyAsync(d_rep, hrep.data(), hrep.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+    for (int rt = 0; rt < 2; rt++) {
+      d_pairs[rt] = (int32_t *)(cb + o_pr) + (rt ? hpairs[0].size() : 0);
+      npair[rt] = (int64_t)hpairs[rt].size() / 3;
+      if (npair[rt])
+        PX_CUDA(ctx, cudaMemcpyAsync(d_pairs[rt], hpairs[rt].data(), hpairs[rt].size() * 4, cudaMemcpyHostToDevice,
+                                     ctx->stream));
+    }
+    char *q = cb + o_ch;
+    for (int rt = 0; rt < 2; rt++) {
+      if (!part[rt]) continue;
+      cbuf[rt] = q;
+      const size_t nl = clid[rt].size();
+      PX_CUDA(ctx, cudaMemcpyAsync(q, clid[rt].data(), nl * 4, cudaMemcpyHostToDevice, ctx->stream));
+      PX_CUDA(ctx, cudaMemcpyAsync(q + nl * 4, cnch[rt].data(), nl * 4, cudaMemcpyHostToDevice, ctx->stream));
+      PX_CUDA(ctx, cudaMemcpyAsync(q + nl * 8, cmodev[rt].data(), nl, cudaMemcpyHostToDevice, ctx->stream));
+      PX_CUDA(ctx, cudaMemsetAsync(q + chain_ctroff(nl), 0, part[rt] - chain_ctroff(nl), ctx->stream));  // ticket, watchdog, exits
+      q += part[rt];
+    }
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // host vectors are staged
+    if (!dedup) d_rep = nullptr;
+  }
   const int64_t NS = (N + 31) & ~(int64_t)31;  // latd row stride
   // B_R_LAT stages host outputs; the stitch ring reads up to 3 segments past a row's last query
   uint32_t *latd = (uint32_t *)px_buf(ctx, B_R_LATD, (size_t)S * NS * 4 + 3 * RSEG * 4 + 64);
@@ -2848,7 +3429,6 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     PX_CUDA(ctx, cudaFuncSetAttribute(k_stitch, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)stitch_smem(ctx->bmax)));
   }
-  const bool use_scan1 = !simple && env_int("PROTEUS_REPLAY_SCAN1", 1) != 0;
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
     LaneArgs la;
@@ -2867,6 +3447,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     la.lstat = d_lstat;
     la.lstart = d_lstart;
     la.bsearch = env_int("PROTEUS_STITCH_BSEARCH", 0);
+    la.skip = d_chainf;
     if (la.nsc > 0) {  // §5 scenarios
     if (use_scan1) {  // Bmax = 1 lanes: exact prefix-maximum scan
       Scan1Args sa;
@@ -2898,10 +3479,52 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
         PX_LAUNCH(ctx, "replay_scan1", k_scan1_apply, (unsigned)nb, 256, 0, sa);
       }
     }
+    // chain lanes (k_chain): alongside the chunk runs + stitch when both have
+    // lanes (on the main stream after the fork, at most CHAIN_OCC blocks per SM
+    // so that stitch blocks still fit), else alone
+    ChainArgs ca;
+    memset(&ca, 0, sizeof ca);
+    const bool chain_now = use_chain && !clid[rt].empty();
+    size_t smc = 0;
+    int chain_nsm = 0, chain_occ = 0;
+    if (chain_now) {
+      const int nl = (int)clid[rt].size();
+      ca.D = D; ca.M = M; ca.bmax = ctx->bmax; ca.nl = nl; ca.C = CHN;
+      ca.K = std::max(0, env_int("PROTEUS_REPLAY_CHAIN_K", 8));
+      ca.NS = NS; ca.maxch = cmax[rt]; ca.nunits = (int64_t)nl * cmax[rt];
+      ca.lid = (const int32_t *)cbuf[rt]; ca.nch = ca.lid + nl; ca.cmode = (const uint8_t *)(cbuf[rt] + (size_t)nl * 8);
+      ca.counter = (unsigned long long *)(cbuf[rt] + chain_ctroff(nl));
+      ca.watchdog = (unsigned *)(ca.counter + 1);
+      ca.ex = (unsigned long long *)(cbuf[rt] + chain_exoff(nl));
+      ca.lp = d_lp; ca.option = d_opt; ca.dev_type = d_dev; ca.lat = ctx->d_lat;
+      ca.devOff = devOff[rt]; ca.devArr = devArr[rt]; ca.latd = latd;
+      smc = chain_smem(CHN, ctx->bmax);
+      PX_CUDA(ctx, cudaFuncSetAttribute(k_chain, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smc));
+      PX_CUDA(ctx, cudaDeviceGetAttribute(&chain_nsm, cudaDevAttrMultiProcessorCount, ctx->device));
+      const int orc = px_occupancy(ctx, (const void *)k_chain, CHAIN_THREADS, smc, &chain_occ);
+      if (orc) return orc;
+      chain_occ = chain_occ > 0 ? chain_occ : 1;
+#ifdef PX_CHAIN_DEBUG
+      ca.dbg = (unsigned long long *)px_buf(ctx, B_R_VLAT, 16 * 8);
+      PX_CUDA(ctx, cudaMemsetAsync(ca.dbg, 0, 16 * 8, ctx->stream));
+#endif
+    }
+    auto launch_chain = [&](int occ_cap) -> int {
+      const int64_t nb = std::min<int64_t>(ca.nunits, (int64_t)chain_nsm * std::min(chain_occ, occ_cap));
+      PX_LAUNCH(ctx, "replay_chain", k_chain, (unsigned)nb, CHAIN_THREADS, smc, ca);
+      return 0;
+    };
+    const bool chain_beside = chain_now && !simple && ngroups[rt] > 0 && crest[rt] &&
+                              env_int("PROTEUS_REPLAY_CHAIN_BESIDE", 0) != 0 &&
+                              env_int("PROTEUS_REPLAY_OVERLAP", 1) != 0 && max_rounds == 0 && !la.debug;
+    if (chain_now && !chain_beside) {
+      const int rc = launch_chain(1 << 20);
+      if (rc) return rc;
+    }
     if (simple) {
       const int nl = la.nsc * D;
       PX_LAUNCH(ctx, "replay_lanes", k_lanes, (nl + LANE_THREADS - 1) / LANE_THREADS, LANE_THREADS, 0, la);
-    } else if (ngroups[rt] > 0) {
+    } else if (ngroups[rt] > 0 && crest[rt]) {
       if ((ngroups[rt] + 3) / 4 > 65535 || (NCH[rt] + 3) / 4 > 65535)
         return px_fail(ctx, PROTEUS_ERANGE, "too many replay chunks");
       dim3 grid((unsigned)la.nsc, (unsigned)((ngroups[rt] + 3) / 4));
@@ -2947,6 +3570,10 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
         PX_CUDA(ctx, cudaEventRecord(ctx->ev_fork, ctx->stream));
         PX_CUDA(ctx, cudaStreamWaitEvent(ctx->aux, ctx->ev_fork, 0));
         PX_CUDA(ctx, cudaStreamWaitEvent(ctx->aux_hi, ctx->ev_fork, 0));
+        if (chain_beside) {
+          const int rc = launch_chain(std::max(1, env_int("PROTEUS_REPLAY_CHAIN_OCC", 2)));
+          if (rc) return rc;
+        }
         cudaStream_t main = ctx->stream;
         const int64_t warps = (int64_t)la.nsc * D;
         int rcs = 0;
@@ -3099,6 +3726,23 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       }
       }  // not pipelined
     }
+    if (chain_now) {
+#ifdef PX_CHAIN_DEBUG
+      {
+        unsigned long long hd[16];
+        PX_CUDA(ctx, cudaMemcpyAsync(hd, ca.dbg, 16 * 8, cudaMemcpyDeviceToHost, ctx->stream));
+        PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+        fprintf(stderr, "chain rt %d: lanes %d units %llu batches %llu jump rounds %llu | cycles/unit load %.0f "
+                "idle %.0f gwalk %.0f jump %.0f wait %.0f link %.0f walk %.0f write %.0f\n", rt, ca.nl, hd[8], hd[9],
+                hd[10], hd[0] / (double)hd[8], hd[1] / (double)hd[8], hd[2] / (double)hd[8], hd[3] / (double)hd[8],
+                hd[4] / (double)hd[8], hd[5] / (double)hd[8], hd[6] / (double)hd[8], hd[7] / (double)hd[8]);
+      }
+#endif
+      unsigned wd = 0;
+      PX_CUDA(ctx, cudaMemcpyAsync(&wd, ca.watchdog, 4, cudaMemcpyDeviceToHost, ctx->stream));
+      PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+      if (wd) return px_fail(ctx, PROTEUS_EINTERNAL, "replay: chain wait for a previous chunk timed out");
+    }
     }  // §5 scenarios
     if (!scl[4 + rt].empty()) {  // §8(f2) baseline batchers: chunk runs, then warp per (device, scenario)
       LaneArgs lb = la;
@@ -3132,7 +3776,17 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       dim3 g(32, nall < 65535 ? nall : 65535);
       PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, NS, S, D, d_scl + rt * S, nall, devOff[rt], latd, d_agg);
       dim3 cg((unsigned)((N + CNT_PER - 1) / CNT_PER), (unsigned)nall);
-      PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, NS, S, D, d_scl + rt * S, devOff[rt], d_lp, latd, d_agg);
+      PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, NS, S, D, d_scl + rt * S, devOff[rt], d_lp, d_rep, latd,
+                d_agg);
+    }
+    if (d_lat_out && d_rep && npair[rt] > 0) {  // the duplicate lanes' rows, for the un-permute
+      int64_t maxn = 1;
+      for (int d = 0; d < D; d++) maxn = std::max(maxn, h_off[rt][d + 1] - h_off[rt][d]);
+      const unsigned gx = (unsigned)std::min<int64_t>(64, (maxn + 4095) / 4096);
+      for (int64_t k0 = 0; k0 < npair[rt]; k0 += 65535) {
+        const unsigned gy = (unsigned)std::min<int64_t>(65535, npair[rt] - k0);
+        PX_LAUNCH(ctx, "replay_dupcopy", k_dupcopy, dim3(gx, gy), 256, 0, NS, d_pairs[rt] + 3 * k0, devOff[rt], latd);
+      }
     }
   }
   if (d_lat_out) {

@@ -1,4 +1,8 @@
-"""c5 replay timing, window path vs chunk-run/stitch path (diagnostic; the bench line is bench.py's)."""
+"""c5 replay timing per path variant (diagnostic; the bench line is bench.py's).
+
+    python scripts/replay_variants.py [NAME=ENV=VALUE[,ENV=VALUE] ...]
+
+Default variants: the chain path vs the chunk-run/stitch path."""
 import json
 import os
 import sys
@@ -8,6 +12,12 @@ import torch  # noqa: E402
 
 from paper_conf_asplos_ahmadgfwsw24_b200 import Proteus, workloads as W  # noqa: E402
 
+VARIANTS = [("chain", [("PROTEUS_REPLAY_CHAIN", "1")]), ("stitch", [("PROTEUS_REPLAY_CHAIN", "0")])]
+if len(sys.argv) > 1:
+    VARIANTS = []
+    for arg in sys.argv[1:]:
+        name, rest = arg.split("=", 1)
+        VARIANTS.append((name, [tuple(kv.split("=", 1)) for kv in rest.split(",")]))
 px = Proteus(0)
 out = {}
 for kind in ("poisson", "gamma"):
@@ -20,8 +30,9 @@ for kind in ("poisson", "gamma"):
     sc = cfg["scenarios"]
     lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
     res = {}
-    for name, ov in (("overlap", "1"), ("serial", "0")):
-        os.environ["PROTEUS_REPLAY_OVERLAP"] = ov
+    for name, envs in VARIANTS:
+        for k, v in envs:
+            os.environ[k] = v
         r0 = px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
         px.set_timing(True)
         ts = []

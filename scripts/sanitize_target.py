@@ -47,10 +47,17 @@ def main():
     # §8(f2) baseline batchers (k_wc_lanes), mixed with §5 scenarios
     scb = np.array([[1000, 4, 0, 1], [2000, 0, 0, 2], [1500, 8, 1, 1], [3000, 0, 0, 0]], np.int32)
     px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, scb)
-    # opt-in replay paths: window path, stitch chunk tables, fused finish, binary-search stitch
+    # duplicate lanes (caps past R4's bound give the same Bmax): one replayed, rows copied
+    scd = np.array([[2000, 32, 0], [2000, 64, 0], [2000, 0, 0], [1000, 1, 0], [3000, 16, 1], [3000, 0, 1]], np.int32)
+    px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, scd)
+    # opt-in replay paths: window path, stitch chunk tables, fused finish, binary-search stitch,
+    # the chain path (tables mode for every lane; full-batch walks for every lane)
     for env in ({"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "2"},
                 {"PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB": "2"},
-                {"PROTEUS_REPLAY_FINISH": "1"}, {"PROTEUS_STITCH_BSEARCH": "1"}):
+                {"PROTEUS_REPLAY_FINISH": "1"}, {"PROTEUS_STITCH_BSEARCH": "1"},
+                {"PROTEUS_REPLAY_CHAIN": "1", "PROTEUS_REPLAY_CHAIN_MINBATCH": "0", "PROTEUS_REPLAY_CHAIN_RHO_PCT": "100000",
+                 "PROTEUS_REPLAY_CHAIN_C": "256", "PROTEUS_REPLAY_CHAIN_K": "2"},
+                {"PROTEUS_REPLAY_CHAIN": "1", "PROTEUS_REPLAY_CHAIN_RHO_PCT": "0", "PROTEUS_REPLAY_CHAIN_C": "256"}):
         os.environ.update(env)
         px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc)
         for k in env:

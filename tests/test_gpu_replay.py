@@ -47,19 +47,39 @@ PATHS = {"chunked": {}, "small_chunks": {"PROTEUS_REPLAY_CHUNK": "16"}, "odd_chu
          "warmup_long_small_chunks": {"PROTEUS_REPLAY_CHUNK": "16", "PROTEUS_REPLAY_WARMUP": "1000"},
          "warmup_rounds": {"PROTEUS_REPLAY_ROUNDS": "3", "PROTEUS_REPLAY_CHUNK": "64", "PROTEUS_REPLAY_WARMUP": "100"},
          "warmup_bscan": {"PROTEUS_REPLAY_BSCAN": "1", "PROTEUS_REPLAY_CHUNK": "200", "PROTEUS_REPLAY_WARMUP": "300"}}
-# the chunk-run / stitch path (PROTEUS_REPLAY_WINDOW=0) under every knob; the
-# window path (the default for §5 lanes with Bmax <= 64) with windows of 1, 3,
-# 32 (default) and 64 tiles of 512 queries
-PATHS = {k: dict(v, PROTEUS_REPLAY_WINDOW="0") for k, v in PATHS.items()}
+# the chunk-run / stitch path (the default; PROTEUS_REPLAY_CHAIN=0) under every
+# knob, with duplicate lanes (same policy, Bmax and SLO on a device) replayed
+# once and copied (default) or each replayed; the window path with windows of
+# 1, 3, 16 (default) and 32 tiles of 512 queries; the opt-in chain path: chunk
+# tables for every lane (chunks of 256 / 300 / 2048 / 8192 heads, K = 0..8
+# greedy batches per chain), full-batch walks for every lane, mixed with the
+# chunk runs + stitch (serial or pipelined, or running beside them)
+PATHS = {k: dict(v, PROTEUS_REPLAY_WINDOW="0", PROTEUS_REPLAY_CHAIN="0") for k, v in PATHS.items()}
+PATHS["no_dedup"] = {"PROTEUS_REPLAY_DEDUP": "0"}
 PATHS["finish_fused"] = {"PROTEUS_REPLAY_FINISH": "1"}
+_T = {"PROTEUS_REPLAY_CHAIN": "1", "PROTEUS_REPLAY_CHAIN_MINBATCH": "0", "PROTEUS_REPLAY_CHAIN_RHO_PCT": "100000"}
+PATHS["chain"] = {"PROTEUS_REPLAY_CHAIN": "1"}
+PATHS["chain_tables_c256"] = dict(_T, PROTEUS_REPLAY_CHAIN_C="256")
+PATHS["chain_tables_c300_k0"] = dict(_T, PROTEUS_REPLAY_CHAIN_C="300", PROTEUS_REPLAY_CHAIN_K="0")
+PATHS["chain_tables_c8192"] = dict(_T, PROTEUS_REPLAY_CHAIN_C="8192")
+PATHS["chain_tables_no_dedup"] = dict(_T, PROTEUS_REPLAY_DEDUP="0", PROTEUS_REPLAY_CHAIN_K="3")
+PATHS["chain_backlog_all"] = {"PROTEUS_REPLAY_CHAIN": "1", "PROTEUS_REPLAY_CHAIN_RHO_PCT": "0",
+                              "PROTEUS_REPLAY_CHAIN_C": "256"}
+PATHS["chain_mixed_minb9"] = dict(_T, PROTEUS_REPLAY_CHAIN_MINB="9", PROTEUS_REPLAY_CHUNK="37")
+PATHS["chain_mixed_serial"] = {"PROTEUS_REPLAY_CHAIN": "1", "PROTEUS_REPLAY_CHAIN_MINBATCH": "0",
+                               "PROTEUS_REPLAY_CHAIN_RHO_PCT": "150", "PROTEUS_REPLAY_CHAIN_MINB": "17",
+                               "PROTEUS_REPLAY_OVERLAP": "0"}
+PATHS["chain_beside"] = {"PROTEUS_REPLAY_CHAIN": "1", "PROTEUS_REPLAY_CHAIN_MINBATCH": "4",
+                         "PROTEUS_REPLAY_CHAIN_BESIDE": "1"}
+PATHS["chain_no_scan1"] = dict(_T, PROTEUS_REPLAY_SCAN1="0", PROTEUS_REPLAY_CHAIN_C="256")
 # the stitch with chunk tables for every lane with Bmax >= 2 / >= 4, and with none
-PATHS["tables_all"] = {"PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB": "2", "PROTEUS_REPLAY_CHUNK": "300"}
-PATHS["tables_min4_chunk64"] = {"PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB": "4",
+PATHS["tables_all"] = {"PROTEUS_REPLAY_CHAIN": "0", "PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB": "2", "PROTEUS_REPLAY_CHUNK": "300"}
+PATHS["tables_min4_chunk64"] = {"PROTEUS_REPLAY_CHAIN": "0", "PROTEUS_REPLAY_TABLES": "1", "PROTEUS_REPLAY_TABLES_MINB": "4",
                                 "PROTEUS_REPLAY_CHUNK": "64"}
-PATHS["tables_default"] = {"PROTEUS_REPLAY_TABLES": "1"}
-PATHS["serial_spec_stitch"] = {"PROTEUS_REPLAY_OVERLAP": "0"}
-PATHS["pipelined_small_chunks"] = {"PROTEUS_REPLAY_CHUNK": "37"}
-PATHS.update({"window": {"PROTEUS_REPLAY_WINDOW": "1"},
+PATHS["tables_default"] = {"PROTEUS_REPLAY_CHAIN": "0", "PROTEUS_REPLAY_TABLES": "1"}
+PATHS["serial_spec_stitch"] = {"PROTEUS_REPLAY_CHAIN": "0", "PROTEUS_REPLAY_OVERLAP": "0"}
+PATHS["pipelined_small_chunks"] = {"PROTEUS_REPLAY_CHAIN": "0", "PROTEUS_REPLAY_CHUNK": "37"}
+PATHS.update({"window": {"PROTEUS_REPLAY_WINDOW": "1"},  # the window path takes its scenarios before the chain
               "window_wt1": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "1"},
               "window_wt3": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "3"},
               "window_wt32": {"PROTEUS_REPLAY_WINDOW": "1", "PROTEUS_REPLAY_WIN_TILES": "32"}})
