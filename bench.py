@@ -109,8 +109,8 @@ class ClockSampler:
 # the lane kernels of the replay (a12): their algorithmic bytes are the latency
 # rows written plus one read of the per-device arrays; the
 # writers put the latencies in query order
-LANE_KERNELS = ("replay_scan1", "replay_bscan", "replay_spec", "replay_fix", "replay_stitch", "replay_lanes")
-WRITE_KERNELS = ("replay_unpermute",)
+LANE_KERNELS = ("replay_scan1", "replay_bscan", "replay_spec", "replay_fix", "replay_stitch", "replay_lanes", "replay_chain")
+WRITE_KERNELS = ("replay_unpermute", "replay_dupcopy")
 
 
 def int_peaks():

@@ -3299,9 +3299,17 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
         if (h_option[d] <= 0) continue;
         std::vector<std::pair<std::array<int64_t, 3>, int>> seen;
         for (int s : scl[rt]) {
-          const int B = hB[(size_t)s * D + d];
+          int B = hB[(size_t)s * D + d];
           if (h_sc[s].policy == 0 && B == 1 && use_scan1) continue;  // the Bmax = 1 scan writes every row
-          const std::array<int64_t, 3> key = {h_sc[s].policy, B, lane_L(s, d)};
+          const int64_t L = lane_L(s, d);
+          if (h_sc[s].policy == 1) {  // Nexus batches Bn: the largest b <= Bmax with 2 T(b) <= L, at least 1 (R14)
+            const int32_t *Tr = ctx->lat.data() + ((size_t)h_dev_type[d] * M + (h_option[d] - 1)) * ctx->bmax;
+            int Bn = 1;
+            for (int b = 1; b <= B; b++)
+              if (2 * (int64_t)Tr[b - 1] <= L) Bn = b;
+            B = Bn;
+          }
+          const std::array<int64_t, 3> key = {h_sc[s].policy, B, L};
           int r = -1;
           for (auto &e : seen) if (e.first == key) { r = e.second; break; }
           if (r < 0) { seen.push_back({key, s}); continue; }

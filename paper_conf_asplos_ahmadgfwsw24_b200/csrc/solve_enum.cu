@@ -367,10 +367,19 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_fam(const __gr
   uint64_t best_s = 0, best_i = ~0ull;
   bool rec = false;
   if (o < oend) {
-    int dig[PX_MAXD];  // touched on carries only
+    // outer digits (touched at carries only): one byte each in a register when
+    // they fit (ND <= 8, K <= 256: c1, c2), else a local array
+    const bool pk = ND <= 8 && K <= 256;
+    uint64_t dpk = 0;
+    int dig_l[PX_MAXD];
+    auto DG = [&](int i) -> int { return pk ? (int)((dpk >> (8 * i)) & 255u) : dig_l[i]; };
+    auto DS = [&](int i, int v) {
+      if (pk) dpk = (dpk & ~(0xFFull << (8 * i))) | ((uint64_t)v << (8 * i));
+      else dig_l[i] = v;
+    };
     {
       uint64_t x = o;
-      for (int i = ND - 1; i >= 0; i--) { dig[i] = (int)(x % K); x /= K; }
+      for (int i = ND - 1; i >= 0; i--) { DS(i, (int)(x % K)); x /= K; }
     }
     FamState st[QM];
     uint64_t Fsum = 0;
@@ -385,7 +394,7 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_fam(const __gr
 #pragma unroll
       for (int k = 0; k < S; k++) cb[k] = 0;
       for (int i = 0; i < ND; i++) {
-        const int oo = dig[i];
+        const int oo = DG(i);
         const int sl = sCS[oo], pv = sP[i * K + oo];
 #pragma unroll
         for (int k = 0; k < S; k++) cb[k] += (sl == k) ? pv : 0;
@@ -467,15 +476,17 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_fam(const __gr
       if (ND == 0) break;
       // next outer prefix: device D-4 advances (one or two families change)
       const int i4 = ND - 1;
-      const int old = dig[i4];
-      if (++dig[i4] == K) {
-        dig[i4] = 0;
+      const int old = DG(i4);
+      if (old + 1 == K) {
+        DS(i4, 0);
         for (int i = i4 - 1; i >= 0; i--) {
-          if (++dig[i] < K) break;
-          dig[i] = 0;
+          const int v = DG(i) + 1;
+          if (v < K) { DS(i, v); break; }
+          DS(i, 0);
         }
         rebuild();
       } else {
+        DS(i4, old + 1);
         const int s_old = sCS[old], s_new = sCS[old + 1];
         if (s_old >= 0) sCaps[s_old][threadIdx.x] -= sP[i4 * K + old];
         sCaps[s_new][threadIdx.x] += sP[i4 * K + old + 1];
