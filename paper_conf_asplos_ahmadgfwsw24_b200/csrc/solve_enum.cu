@@ -408,37 +408,61 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_fam(const __gr
     rebuild();
     unsigned long long *gb = a.gbound + vec;
     for (;;) {
-      // the K blocks (o, o3) of this outer prefix
+      // the K blocks (o, o3) of this outer prefix.  Device D-3's option
+      // touches one family q3 (warp-uniform; options are grouped by family,
+      // so q3 changes QM + 1 times); the other families X are fixed, so their
+      // part of the block maximum is folded once per q3: JX = max J, b1 / b2 =
+      // the top two MB, MAX = max MA, CX = max over a != b in X of MA_a +
+      // MB_b (b may be idle: gains are >= 0)
+      int cq3 = -2;
+      uint64_t baseX = 0, JX = 0, b1X = 0, MAX = 0, CX = 0;
+      auto fold = [&](int q3) {
+        baseX = Fsum;
+        JX = 0;
+        b1X = 0;
+        MAX = 0;
+        uint64_t b2 = 0;
+        int f1 = -1;
+#pragma unroll
+        for (int q = 0; q < QM; q++) {
+          if (q == q3) { baseX -= st[q].F; continue; }
+          JX = st[q].J > JX ? st[q].J : JX;
+          MAX = st[q].MA > MAX ? st[q].MA : MAX;
+          if (st[q].MB > b1X) { b2 = b1X; b1X = st[q].MB; f1 = q; }
+          else if (st[q].MB > b2) b2 = st[q].MB;
+        }
+        CX = 0;
+#pragma unroll
+        for (int q = 0; q < QM; q++) {
+          if (q == q3) continue;
+          const uint64_t v = st[q].MA + (q == f1 ? b2 : b1X);
+          CX = v > CX ? v : CX;
+        }
+      };
       for (int o3 = 0; o3 < K; o3++) {
         uint64_t G;  // best score any thread of this vector has recorded (relaxed; stale = lower)
         asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(G) : "l"(gb));
         const int s3 = sCS[o3];  // warp-uniform (-1: idle)
         const int q3 = s3 >= 0 ? s3 / VM : -1;
+        if (q3 != cq3) { fold(q3); cq3 = q3; }
         FamState m;  // family q3 with device D-3's capacity added
+        uint64_t base = baseX, dmax;
         if (q3 >= 0) {
           int c[VM];
 #pragma unroll
           for (int j = 0; j < VM; j++) c[j] = sCaps[q3 * VM + j][threadIdx.x] + (q3 * VM + j == s3 ? sP[(D - 3) * K + o3] : 0);
           m = fam_state<QM, VM, SYM>(c, sDem[q3], a, q3);
-        }
-        uint64_t base = Fsum;
-        uint64_t mB1 = 0, mB2 = 0, mJ = 0;
-        int fB1 = -1;
-#pragma unroll
-        for (int q = 0; q < QM; q++) {
-          const bool mod = q == q3;
-          const uint64_t MBq = mod ? m.MB : st[q].MB, Jq = mod ? m.J : st[q].J;
-          if (mod) base = base - st[q].F + m.F;
-          mJ = Jq > mJ ? Jq : mJ;
-          if (MBq > mB1) { mB2 = mB1; mB1 = MBq; fB1 = q; }
-          else if (MBq > mB2) mB2 = MBq;
-        }
-        uint64_t dmax = mJ > mB1 ? mJ : mB1;  // J covers both-in-one-family; (idle, b) rows: mB1
-#pragma unroll
-        for (int q = 0; q < QM; q++) {
-          const uint64_t MAq = q == q3 ? m.MA : st[q].MA;
-          const uint64_t v = MAq + (q == fB1 ? mB2 : mB1);  // (a in q, b outside q or idle)
-          dmax = v > dmax ? v : dmax;
+          base += m.F;
+          // both in q3 (J), b alone, a in q3 with b in X or idle, a in X with b in q3, both in X
+          const uint64_t mj = m.J > JX ? m.J : JX, mb = m.MB > b1X ? m.MB : b1X;
+          const uint64_t c1 = m.MA + b1X, c2 = MAX + m.MB;
+          dmax = mj > mb ? mj : mb;
+          dmax = c1 > dmax ? c1 : dmax;
+          dmax = c2 > dmax ? c2 : dmax;
+          dmax = CX > dmax ? CX : dmax;
+        } else {
+          dmax = JX > b1X ? JX : b1X;
+          dmax = CX > dmax ? CX : dmax;
         }
         const uint64_t Mx = base + dmax;
         // threshold: the thread's best so far (strict >: the first maximum is
