@@ -240,7 +240,10 @@ __device__ __forceinline__ uint64_t fam_fill(const int (&c)[VM], int s, const Fl
     acc += (uint64_t)(uint32_t)a.A[q * VM + j] * (uint32_t)t;
     rem -= t;
   }
-  return px_pack((uint32_t)(s - rem), acc);
+  // px_pack(served, acc) with served << 42 added to the high word only
+  // (accsum < 2^42, so no carry crosses the halves)
+  const uint32_t hi = (uint32_t)(acc >> 32) + ((uint32_t)(s - rem) << (PX_ACC_BITS - 32));
+  return ((uint64_t)hi << 32) | (uint32_t)acc;
 }
 
 struct FamState {
