@@ -2610,21 +2610,24 @@ __global__ void __launch_bounds__(256) k_finish(int64_t N, int64_t NS, int S, in
 // (b_i(h), t_i(h)) when F <= t_i(h), else the greedy batch min(Bmax, queued at
 // F) at F.  The idle decision depends on h only, so a chunk of C heads is
 // tabulated in parallel (one binary search per head), and so is, for every
-// head i, the rest of the run after an idle-branch decision at i: the next
-// head at which the run decides on the idle branch again (the greedy batches
-// between are a function of i too), or the state (head >= chunk end, free
-// time) in which it leaves the chunk.  A chunk's exit is then a function of
-// its entry: an entry on the idle branch at head h leaves where the chain of
-// h leaves (every chain's end is found beforehand by pointer jumping); a busy
-// entry first takes its greedy batches.  Units (lane, chunk) are taken in chunk-major ticket order by
-// persistent blocks; each builds its tables, then waits for the previous
-// chunk's exit (a single 64-bit word: ((F + 1) << 8) | (head - chunk start)),
-// publishes its own, and only then walks its chunk once from the true entry to
-// write the latencies (device-major rows, like the chunk runs).  The serial
-// dependency per lane is one table lookup per chunk.
+// head i, the rest of the run after an idle-branch decision at i, up to the end
+// of i's segment (SEG heads): the next head at which the run decides on the
+// idle branch again (the greedy batches between are a function of i too), or
+// the state (first head past the segment, free time) in which it leaves the
+// segment.  Every head's last idle-branch head inside its segment follows by a
+// backward scan of the segment (thread per segment).  Units (lane, chunk) are
+// taken in chunk-major ticket order by persistent blocks; each builds its
+// tables, then warp 0 waits for the previous chunk's exit (a single 64-bit
+// word: ((F + 1) << 8) | (head - chunk start)), walks the chunk from the true
+// entry one segment per hop (greedy stretches in between, full batches 32 per
+// ballot), recording the true state at the first batch head of every segment,
+// and publishes the chunk's exit; then one thread per segment writes the
+// segment's latencies from its true state (device-major rows, like the chunk
+// runs).  The serial dependency per lane is one hop per segment.
 #define CHAIN_THREADS 256
 #define CHAIN_WARPS (CHAIN_THREADS / 32)
-#define CHAIN_CMAX 8192  // largest chunk (heads are int16 in the tables)
+#define CHAIN_CMAX 8192   // largest chunk (heads are int16 in the tables)
+#define CHAIN_SEGMIN 16   // smallest segment
 #ifdef PX_CHAIN_DEBUG  // per-phase cycle totals of k_chain (thread 0), printed by the host
 #define CX_T(k) do { if (threadIdx.x == 0) { const long long t_ = clock64(); atomicAdd(a.dbg + (k), (unsigned long long)(t_ - cx_t)); cx_t = t_; } } while (0)
 #else
@@ -2633,7 +2636,9 @@ __global__ void __launch_bounds__(256) k_finish(int64_t N, int64_t NS, int S, in
 struct ChainArgs {
   int D, M, bmax, nl, C;
   int K;                       // greedy batches a head's chain follows in the tables
-  int64_t NS, maxch, nunits;   // tickets: c * nl + li (chunk-major)
+  int SEG;                     // heads per segment (writer thread, link hop)
+  int64_t NS, maxch, nunits;   // tickets
+  const unsigned long long *units;  // [nunits] (lane index << 32) | chunk, in ticket order (host-built)
   const int32_t *lid;          // [nl] lane = s * D + d (device-major: consecutive tickets share arrivals)
   const int32_t *nch;          // [nl] chunks of the lane
   const uint8_t *cmode;        // [nl] 0: chunk tables, 1: near overload (full-batch walks, no tables)
@@ -2645,7 +2650,7 @@ struct ChainArgs {
   unsigned long long *ex;      // [nl][maxch] packed chunk exits, 0 = not yet published
   unsigned long long *counter; // ticket counter
   unsigned *watchdog;          // set when a wait for a previous chunk's exit times out
-  unsigned long long *dbg;     // PX_CHAIN_DEBUG: [16] phase cycles, units, batches, jump rounds
+  unsigned long long *dbg;     // PX_CHAIN_DEBUG: [16] phase cycles, units, batches, hops
 };
 
 struct ShArr {  // arrivals of a chunk in shared memory, from its first head
@@ -2659,33 +2664,34 @@ static size_t chain_exoff(size_t nl) { return chain_ctroff(nl) + 16; }
 static size_t chain_smem(int C, int bmax) {
   const size_t E = (size_t)C + bmax + 2;
   return (size_t)C * 8 /* sFx */ + (size_t)bmax * 4 /* sT */ + E * 4 /* sA */ + (size_t)C * 4 /* sTi */ +
-         (size_t)C * 4 /* sFi */ + (size_t)C * 6 /* sNx, sJ[2] */ + (size_t)C /* sB */ + (size_t)C /* sHx */ + 64;
+         (size_t)C * 8 /* sNx, sJ, sJc, sHx */ + (size_t)C /* sB */ + 64;
 }
 
 __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__ ChainArgs a) {
   extern __shared__ __align__(16) unsigned char csm[];
-  const int C = a.C;
-  int64_t *sFx = (int64_t *)csm;                    // [C] exit free time of an exiting chain
+  const int C = a.C, SEG = a.SEG;
+  int64_t *sFx = (int64_t *)csm;                    // [C] free time when a head's run leaves its segment
   int32_t *sT = (int32_t *)(sFx + C);               // [bmax] T(b) at b - 1
   uint32_t *sA = (uint32_t *)(sT + a.bmax);         // [C + bmax + 2] arrivals from the chunk start
   int32_t *sTi = (int32_t *)(sA + C + a.bmax + 2);  // [C] t_i(h) - a_h
-  int32_t *sFi = sTi + C;                           // [C] t_i(h) + T(b_i(h)) - a_h: the idle batch's finish
-  int16_t *sNx = (int16_t *)(sFi + C);              // [C] next idle-branch head of the chain of h, -1: leaves, -2: left to the walk
-  int16_t *sJa = sNx + C, *sJb = sJa + C;          // [2][C] last idle-branch head of the chain of h (double buffer)
-  uint8_t *sB = (uint8_t *)(sJb + C);               // [C] b_i(h)
-  uint8_t *sHx = sB + C;                            // [C] exit head - chunk end of an exiting chain
+  int16_t *sNx = (int16_t *)(sTi + C);              // [C] next idle-branch head in the segment, -1: leaves, -2: left to
+                                                    // the walk, -3: leaves onto an idle-branch head in the chunk
+  int16_t *sJ = sNx + C;                            // [C] last idle-branch head of h's run in its segment
+  int16_t *sJc = sJ + C;                            // [C] last idle-branch head of h's run in the chunk
+  int16_t *sHx = sJc + C;                           // [C] first head past the segment of a leaving run
+  uint8_t *sB = (uint8_t *)(sHx + C);               // [C] b_i(h)
   __shared__ unsigned long long sTicket;
-  __shared__ uint32_t sVis[CHAIN_CMAX / 32];  // idle-branch batch starts of the speculative walks
-  __shared__ int sSx[CHAIN_WARPS], sEnt;       // speculative walks' exit heads; the true entry
-  __shared__ int64_t sSF[CHAIN_WARPS], sEntF;  // ... and free times
+  __shared__ int sSegH[CHAIN_CMAX / CHAIN_SEGMIN];      // true state at the first batch head of each segment
+  __shared__ int64_t sSegF[CHAIN_CMAX / CHAIN_SEGMIN];
   const int tid = threadIdx.x;
   for (;;) {
     if (tid == 0) sTicket = atomicAdd(a.counter, 1ull);
     __syncthreads();
     const unsigned long long tk = sTicket;
     if (tk >= (unsigned long long)a.nunits) return;
-    const int li = (int)(tk % (unsigned long long)a.nl);
-    const int64_t c = (int64_t)(tk / (unsigned long long)a.nl);
+    const unsigned long long u = a.units[tk];
+    const int li = (int)(u >> 32);
+    const int64_t c = (int64_t)(u & 0xffffffffull);
     if (c < a.nch[li]) {
 #ifdef PX_CHAIN_DEBUG
       long long cx_t = clock64();
@@ -2699,10 +2705,12 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
       const int64_t nloc = nloc0 - c0;  // heads from the chunk start to the device's end
       const int Cn = (int)(nloc < C ? nloc : C);
       const int na = (int)(nloc < (int64_t)Cn + Bm + 1 ? nloc : (int64_t)Cn + Bm + 1);
+      const int nseg = (Cn + SEG - 1) / SEG;
       const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
       for (int k = tid; k < Bm; k += CHAIN_THREADS) sT[k] = Tg[k];
       const uint32_t *src = a.devArr + off + c0;
       for (int j = tid; j < na; j += CHAIN_THREADS) sA[j] = src[j];
+      for (int sg = tid; sg < nseg; sg += CHAIN_THREADS) sSegH[sg] = -1;  // not recorded yet
       __syncthreads();
       CX_T(0);
       const ShArr A{sA};
@@ -2796,7 +2804,6 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
           if (lane == 0) {
             atomicAdd(a.dbg + 8, 1ull);
             atomicAdd(a.dbg + 9, (unsigned long long)nbat);
-            atomicAdd(a.dbg + 11, 1ull);
           }
 #else
           (void)nbat;
@@ -2809,7 +2816,6 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
         const int b = idle_decide(A, nloc, (int64_t)i, Bm, p.L, sT, true, &t);
         sB[i] = (uint8_t)b;
         sTi[i] = (int32_t)(t - (int64_t)sA[i]);
-        sFi[i] = (int32_t)(t + sT[b - 1] - (int64_t)sA[i]);
       }
       __syncthreads();
       CX_T(1);
@@ -2820,14 +2826,22 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
         return ((int64_t)hh + Bm - 1 < nloc && (int64_t)sA[hh + Bm - 1] <= F) ? Bm
                                                                                : count_upto(A, nloc, (int64_t)hh, Bm, F);
       };
-      // the chain of every head after its idle-branch decision (at most K
-      // greedy batches are followed here: -2 marks a head whose chain is left
-      // to the serial walk -- backlogged stretches would make this quadratic)
+      // the run of every head after its idle-branch decision, inside the
+      // head's segment (at most K greedy batches are followed here: -2 marks a
+      // head whose run is left to the link walk -- backlogged stretches would
+      // make this quadratic)
       for (int i = tid; i < Cn; i += CHAIN_THREADS) {
-        int64_t F = (int64_t)sA[i] + sFi[i];
-        int hh = i + sB[i];
+        const int se = (i / SEG + 1) * SEG < Cn ? (i / SEG + 1) * SEG : Cn;
+        const int bi = sB[i];
+        int64_t F = (int64_t)sA[i] + sTi[i] + sT[bi - 1];
+        int hh = i + bi;
         for (int st = 0;; st++) {
-          if (hh >= Cn) { sNx[i] = -1; sHx[i] = (uint8_t)(hh - Cn); sFx[i] = F; break; }
+          if (hh >= se) {
+            sNx[i] = (hh < Cn && F <= (int64_t)sA[hh] + sTi[hh]) ? -3 : -1;
+            sHx[i] = (int16_t)hh;
+            sFx[i] = F;
+            break;
+          }
           if (F <= (int64_t)sA[hh] + sTi[hh]) { sNx[i] = (int16_t)hh; break; }
           if (st >= a.K) { sNx[i] = -2; break; }
           const int g = greedy(hh, F);  // dispatched at F
@@ -2837,53 +2851,52 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
       }
       __syncthreads();
       CX_T(2);
-      // the last idle-branch head of every chain (pointer jumping, double
-      // buffered: the last head is a fixed point)
-      int16_t *sJ = sJa, *sJn = sJb;
-      for (int i = tid; i < Cn; i += CHAIN_THREADS) sJ[i] = sNx[i] >= 0 ? sNx[i] : (int16_t)i;
+      // the last idle-branch head of every head's run inside its segment (sJ)
+      // and inside the chunk (sJc: a run leaving its segment onto an
+      // idle-branch head continues with that head's): pointer jumping, in
+      // place (a pointer only ever moves further along its own run)
+      for (int i = tid; i < Cn; i += CHAIN_THREADS) {
+        const int nx = sNx[i];
+        sJ[i] = nx >= 0 ? (int16_t)nx : (int16_t)i;
+        sJc[i] = nx >= 0 ? (int16_t)nx : nx == -3 ? sHx[i] : (int16_t)i;
+      }
       for (bool more = true; more;) {
         __syncthreads();
         bool ch = false;
         for (int i = tid; i < Cn; i += CHAIN_THREADS) {
           const int j = sJ[i], jj = sJ[j];
-          sJn[i] = (int16_t)jj;
-          ch |= jj != j;
+          const int k = sJc[i], kk = sJc[k];
+          if (jj != j) { sJ[i] = (int16_t)jj; ch = true; }
+          if (kk != k) { sJc[i] = (int16_t)kk; ch = true; }
         }
-        int16_t *t_ = sJ;
-        sJ = sJn;
-        sJn = t_;
         more = __syncthreads_or(ch);
-#ifdef PX_CHAIN_DEBUG
-        if (tid == 0) atomicAdd(a.dbg + 10, 1ull);
-#endif
       }
       CX_T(3);
-      // segments for the speculative walks of warps 1..7 (the true run enters
-      // below Bmax, so segments starting at or past Bmax never hold positions
-      // of the previous chunk's last batch)
-      const bool spec = Cn / CHAIN_WARPS >= Bm;
-      auto seg0 = [&](int k) { return (int)(((int64_t)k * Cn) / CHAIN_WARPS); };
-      for (int k = tid; k < (Cn + 31) / 32; k += CHAIN_THREADS) sVis[k] = 0u;
-      __syncthreads();
-      if (w == 0) {  // the link: this chunk's exit from its entry
+      if (w == 0) {
+        // the link: the true run through the chunk, one hop per run of
+        // idle-branch decisions (sJc), greedy batches between (full batches
+        // 32 per ballot); the chunk's exit is published at once.  Then the
+        // same run again, one hop per segment (sJ), recording the state at the
+        // first batch head of every segment for the writers.
         int h;
         int64_t F;
+#ifdef PX_CHAIN_DEBUG
+        const long long cx_w0 = clock64();
+#endif
         entry(h, F);
+#ifdef PX_CHAIN_DEBUG
+        if (lane == 0) atomicAdd(a.dbg + 18 + 3 * li, (unsigned long long)(clock64() - cx_w0));
+#endif
         CX_T(4);
-        // greedy batches, then the chain of the first idle-branch head (chains
-        // left to the serial walk are continued here)
         int hh = h;
         int64_t FF = F;
-        int hx;
-        int64_t Fx;
-        for (;;) {
-          if (hh >= Cn) { hx = hh - Cn; Fx = FF; break; }
-          const int64_t ti = (int64_t)sA[hh] + sTi[hh];
-          if (FF <= ti) {
-            const int r = sJ[hh];
-            if (sNx[r] == -1) { hx = sHx[r]; Fx = sFx[r]; break; }
-            FF = (int64_t)sA[r] + sFi[r];
-            hh = r + sB[r];
+        long long hops = 0;
+        while (hh < Cn) {
+          hops++;
+          if (FF <= (int64_t)sA[hh] + sTi[hh]) {
+            const int r = sJc[hh];
+            if (sNx[r] == -1) { FF = sFx[r]; hh = sHx[r]; }
+            else { const int br = sB[r]; FF = (int64_t)sA[r] + sTi[r] + sT[br - 1]; hh = r + br; }
             continue;
           }
           const int k = stretch(hh, FF, Cn);
@@ -2892,117 +2905,79 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
           FF += sT[g - 1];
           hh += g;
         }
-        publish(hx, Fx);
-        if (lane == 0) {
-          sEnt = h;
-          sEntF = F;
+        publish(hh - Cn, FF);
+#ifdef PX_CHAIN_DEBUG
+        if (lane == 0) {  // per lane: link cycles, hops, wait cycles
+          atomicAdd(a.dbg + 16 + 3 * li, (unsigned long long)(clock64() - cx_t));
+          atomicAdd(a.dbg + 17 + 3 * li, (unsigned long long)hops);
         }
+#endif
         CX_T(5);
-      } else if (spec) {
-        // speculative walk of segment w from an idle device at its first head:
-        // latencies of its positions, its idle-branch batch starts (sVis) and
-        // its exit (first head past the segment, free time)
-        const int S0 = seg0(w), S1 = seg0(w + 1);
-        int hh = S0;
-        int64_t FF = INT64_MIN / 4;
-        while (hh < S1) {
-          if (FF <= (int64_t)sA[hh] + sTi[hh]) {
-            for (;;) {
-              const int b = sB[hh];
-              const int64_t fin = (int64_t)sA[hh] + sFi[hh];
-              if (lane == 0) atomicOr(&sVis[hh >> 5], 1u << (hh & 31));
-              put(hh, b, fin, S1);
-              const int nx = sNx[hh];
-              if (nx == hh + b && nx < S1) { hh = nx; continue; }
-              hh += b;
-              FF = fin;
-              break;
-            }
-            continue;
+        int nrec = 0;  // segments [0, nrec) recorded (warp-uniform)
+        auto rec = [&](int hq, int64_t Fq) {  // free time first, then the head (the writers' flag)
+          const int upto = hq / SEG + 1 < nseg ? hq / SEG + 1 : nseg;
+          for (int sg = nrec + lane; sg < upto; sg += 32) {
+            sSegF[sg] = Fq;
+            __threadfence_block();
+            *(volatile int *)&sSegH[sg] = hq;
           }
-          const int k = stretch(hh, FF, S1);
-          if (k > 0) {
-            const int np = k * Bm, e = hh + np < S1 ? hh + np : S1;
-            for (int j = hh + lane; j < e; j += 32) out[j] = sat_lat(FF + (int64_t)((j - hh) / Bm + 1) * TB - (int64_t)sA[j]);
-            hh += np;
-            FF += (int64_t)k * TB;
-            continue;
-          }
-          const int b = count_upto(A, nloc, (int64_t)hh, Bm, FF);
-          const int64_t fin = FF + sT[b - 1];
-          put(hh, b, fin, S1);
-          hh += b;
-          FF = fin;
-        }
-        if (lane == 0) { sSx[w] = hh; sSF[w] = FF; }
-      }
-      __syncthreads();
-      if (w == 0) {
-        // the true run through the chunk: latencies of [entry, exit head); in a
-        // segment of a speculative walk it stops at the first idle-branch batch
-        // start the walk also had (both then take the same decisions) and takes
-        // the walk's exit, writing the positions of the walk's last batch past
-        // the segment
-        long long nbat = 0;
-        int hh = sEnt;
-        int64_t FF = sEntF;
-        auto merge = [&](int x) -> int {  // segment whose speculative walk had an idle start at x, or 0
-          if (!spec || !((sVis[x >> 5] >> (x & 31)) & 1u)) return 0;
-          int k = (int)(((int64_t)x * CHAIN_WARPS) / Cn);
-          while (k + 1 < CHAIN_WARPS && seg0(k + 1) <= x) k++;
-          while (seg0(k) > x) k--;
-          return k;
+          nrec = upto > nrec ? upto : nrec;
         };
+        hh = h;
+        FF = F;
+        rec(hh, FF);
         while (hh < Cn) {
           if (FF <= (int64_t)sA[hh] + sTi[hh]) {
-            const int m = merge(hh);
-            if (m > 0) {
-              const int S1 = seg0(m + 1), hx = sSx[m];
-              const int64_t Fx = sSF[m];
-              for (int j = S1 + lane; j < hx; j += 32) out[j] = sat_lat(Fx - (int64_t)sA[j]);
-              hh = hx;
-              FF = Fx;
-              continue;
-            }
-            for (;;) {
-              const int b = sB[hh];
-              const int64_t fin = (int64_t)sA[hh] + sFi[hh];
-              put(hh, b, fin, INT32_MAX);
-              nbat++;
-              const int nx = sNx[hh];
-              if (nx == hh + b && merge(nx) == 0) { hh = nx; continue; }
-              hh += b;
-              FF = fin;
-              break;
-            }
+            const int r = sJ[hh];
+            if (sNx[r] < -2 || sNx[r] == -1) { FF = sFx[r]; hh = sHx[r]; }
+            else { const int br = sB[r]; FF = (int64_t)sA[r] + sTi[r] + sT[br - 1]; hh = r + br; }
+            rec(hh, FF);
             continue;
           }
-          const int k = stretch(hh, FF, Cn);
-          if (k > 0) {
-            const int np = k * Bm;
-            for (int j = lane; j < np; j += 32) out[hh + j] = sat_lat(FF + (int64_t)(j / Bm + 1) * TB - (int64_t)sA[hh + j]);
-            nbat += k;
-            hh += np;
-            FF += (int64_t)k * TB;
-            continue;
-          }
-          const int b = count_upto(A, nloc, (int64_t)hh, Bm, FF);
-          const int64_t fin = FF + sT[b - 1];
-          put(hh, b, fin, INT32_MAX);
+          const int se = (hh / SEG + 1) * SEG < Cn ? (hh / SEG + 1) * SEG : Cn;
+          const int k = stretch(hh, FF, se);
+          if (k > 0) { hh += k * Bm; FF += (int64_t)k * TB; rec(hh, FF); continue; }
+          const int g = count_upto(A, nloc, (int64_t)hh, Bm, FF);
+          FF += sT[g - 1];
+          hh += g;
+          rec(hh, FF);
+        }
+        CX_T(7);
+#ifdef PX_CHAIN_DEBUG
+        if (lane == 0) { atomicAdd(a.dbg + 8, 1ull); atomicAdd(a.dbg + 10, (unsigned long long)hops); }
+#else
+        (void)hops;
+#endif
+      }
+      // the writers (warps 1..7, while warp 0 records): thread per segment,
+      // from the true state at its first batch head, as soon as it is
+      // recorded; a batch is written whole by the segment it starts in
+      long long nbat = 0;
+      for (int sg = tid - 32; sg < nseg; sg += CHAIN_THREADS - 32) {
+        if (sg < 0) break;
+        const int s1 = (sg + 1) * SEG < Cn ? (sg + 1) * SEG : Cn;
+        int hh;
+        while ((hh = *(volatile int *)&sSegH[sg]) < 0) __nanosleep(32);
+        __threadfence_block();
+        int64_t FF = *(volatile int64_t *)&sSegF[sg];
+        while (hh < s1) {
+          const int64_t ti = (int64_t)sA[hh] + sTi[hh];
+          int b;
+          int64_t fin;
+          if (FF <= ti) { b = sB[hh]; fin = ti + sT[b - 1]; }
+          else { b = greedy(hh, FF); fin = FF + sT[b - 1]; }
+          for (int j = 0; j < b; j++) out[hh + j] = sat_lat(fin - (int64_t)sA[hh + j]);
           nbat++;
           hh += b;
           FF = fin;
         }
-        CX_T(6);
-#ifdef PX_CHAIN_DEBUG
-        if (lane == 0) {
-          atomicAdd(a.dbg + 8, 1ull);
-          atomicAdd(a.dbg + 9, (unsigned long long)nbat);
-        }
-#else
-        (void)nbat;
-#endif
       }
+      CX_T(6);
+#ifdef PX_CHAIN_DEBUG
+      atomicAdd(a.dbg + 9, (unsigned long long)nbat);
+#else
+      (void)nbat;
+#endif
       }  // tables
     }
     __syncthreads();  // shared tables and sTicket are rewritten by the next unit
@@ -3265,11 +3240,13 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   // and L < 2^30; the chunk runs + stitch take the other lanes
   const bool use_scan1 = !simple && env_int("PROTEUS_REPLAY_SCAN1", 1) != 0;
   const bool use_chain = !simple && env_int("PROTEUS_REPLAY_CHAIN", 0) != 0 && max_rounds == 0 &&
-                         env_int("PROTEUS_REPLAY_BSCAN", 0) == 0 && env_int("PROTEUS_REPLAY_TABLES", 0) == 0;
+                         env_int("PROTEUS_REPLAY_TABLES", 0) == 0;
   int CHN = env_int("PROTEUS_REPLAY_CHAIN_C", 2048);
   CHN = CHN < 256 ? 256 : CHN > CHAIN_CMAX ? CHAIN_CMAX : CHN;  // shared-memory tables (~24 B per head)
   const int chain_minb = std::max(2, env_int("PROTEUS_REPLAY_CHAIN_MINB", 2));
   std::vector<int32_t> clid[2], cnch[2];
+  unsigned long long *d_units[2] = {nullptr, nullptr};  // chain ticket order per routing mode
+  int64_t nunits[2] = {0, 0};
   std::vector<uint8_t> cmodev[2];
   int64_t cmax[2] = {0, 0};
   bool crest[2] = {true, true};  // lanes left to the chunk runs + stitch
@@ -3284,7 +3261,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   // holding lane (s, d); rep[s][D] = s for the sink).  skip[s][d]: the chunk
   // kernels leave the lane alone (a duplicate, or a chain lane).
   const bool dedup = !simple && !use_win && max_rounds == 0 && env_int("PROTEUS_REPLAY_DEDUP", 1) != 0 &&
-                     env_int("PROTEUS_REPLAY_BSCAN", 0) == 0 && env_int("PROTEUS_REPLAY_TABLES", 0) == 0 &&
+                     env_int("PROTEUS_REPLAY_TABLES", 0) == 0 &&
                      env_int("PROTEUS_REPLAY_FINISH", 0) == 0 && env_int("PROTEUS_REPLAY_DEBUG", 0) == 0;
   std::vector<int32_t> hrep((size_t)S * (D + 1));
   std::vector<uint8_t> hskip((size_t)S * D, 0);
@@ -3412,6 +3389,36 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       PX_CUDA(ctx, cudaMemcpyAsync(q + nl * 4, cnch[rt].data(), nl * 4, cudaMemcpyHostToDevice, ctx->stream));
       PX_CUDA(ctx, cudaMemcpyAsync(q + nl * 8, cmodev[rt].data(), nl, cudaMemcpyHostToDevice, ctx->stream));
       PX_CUDA(ctx, cudaMemsetAsync(q + chain_ctroff(nl), 0, part[rt] - chain_ctroff(nl), ctx->stream));  // ticket, watchdog, exits
+      // ticket order: every lane's chunks spread over the run in proportion to
+      // its length (chunk c of a lane with n chunks at key c * maxch / n,
+      // counting sort), so that long lanes keep several chunks in flight; a
+      // chunk's predecessor always has a smaller key (an earlier ticket).
+      // Uploaded once per lane layout (cached in the context).
+      {
+        const int64_t mx = cmax[rt];
+        std::vector<int64_t> key;
+        key.reserve(nl + 2);
+        key.push_back((int64_t)nl);
+        key.push_back(mx);
+        size_t nu = 0;
+        for (size_t l = 0; l < nl; l++) { key.push_back(cnch[rt][l]); nu += (size_t)cnch[rt][l]; }
+        nunits[rt] = (int64_t)nu;
+        d_units[rt] = (unsigned long long *)px_buf(ctx, B_R_UNITS0 + rt, nu * 8 + 16);
+        if (!d_units[rt]) return px_fail(ctx, PROTEUS_ENOMEM, "chain tickets");
+        if (key != ctx->chain_ukey[rt]) {
+          std::vector<int64_t> cnt((size_t)mx + 1, 0);
+          for (size_t l = 0; l < nl; l++)
+            for (int64_t c = 0; c < cnch[rt][l]; c++) cnt[(size_t)(c * mx / cnch[rt][l]) + 1]++;
+          for (int64_t k = 0; k < mx; k++) cnt[(size_t)k + 1] += cnt[(size_t)k];
+          std::vector<unsigned long long> units(nu);
+          for (size_t l = 0; l < nl; l++)
+            for (int64_t c = 0; c < cnch[rt][l]; c++)
+              units[(size_t)cnt[(size_t)(c * mx / cnch[rt][l])]++] = ((unsigned long long)l << 32) | (unsigned long long)c;
+          PX_CUDA(ctx, cudaMemcpyAsync(d_units[rt], units.data(), nu * 8, cudaMemcpyHostToDevice, ctx->stream));
+          PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // units is a host vector
+          ctx->chain_ukey[rt] = key;
+        }
+      }
       q += part[rt];
     }
     PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // host vectors are staged
@@ -3499,11 +3506,13 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       const int nl = (int)clid[rt].size();
       ca.D = D; ca.M = M; ca.bmax = ctx->bmax; ca.nl = nl; ca.C = CHN;
       ca.K = std::max(0, env_int("PROTEUS_REPLAY_CHAIN_K", 8));
-      ca.NS = NS; ca.maxch = cmax[rt]; ca.nunits = (int64_t)nl * cmax[rt];
+      ca.SEG = std::min(CHN, std::max(CHAIN_SEGMIN, env_int("PROTEUS_REPLAY_CHAIN_SEG", 64)));
+      ca.NS = NS; ca.maxch = cmax[rt]; ca.nunits = nunits[rt];
       ca.lid = (const int32_t *)cbuf[rt]; ca.nch = ca.lid + nl; ca.cmode = (const uint8_t *)(cbuf[rt] + (size_t)nl * 8);
       ca.counter = (unsigned long long *)(cbuf[rt] + chain_ctroff(nl));
       ca.watchdog = (unsigned *)(ca.counter + 1);
       ca.ex = (unsigned long long *)(cbuf[rt] + chain_exoff(nl));
+      ca.units = d_units[rt];
       ca.lp = d_lp; ca.option = d_opt; ca.dev_type = d_dev; ca.lat = ctx->d_lat;
       ca.devOff = devOff[rt]; ca.devArr = devArr[rt]; ca.latd = latd;
       smc = chain_smem(CHN, ctx->bmax);
@@ -3513,8 +3522,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       if (orc) return orc;
       chain_occ = chain_occ > 0 ? chain_occ : 1;
 #ifdef PX_CHAIN_DEBUG
-      ca.dbg = (unsigned long long *)px_buf(ctx, B_R_VLAT, 16 * 8);
-      PX_CUDA(ctx, cudaMemsetAsync(ca.dbg, 0, 16 * 8, ctx->stream));
+      ca.dbg = (unsigned long long *)px_buf(ctx, B_R_VLAT, (16 + 3 * (size_t)nl) * 8);
+      PX_CUDA(ctx, cudaMemsetAsync(ca.dbg, 0, (16 + 3 * (size_t)nl) * 8, ctx->stream));
 #endif
     }
     auto launch_chain = [&](int occ_cap) -> int {
@@ -3740,10 +3749,22 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
         unsigned long long hd[16];
         PX_CUDA(ctx, cudaMemcpyAsync(hd, ca.dbg, 16 * 8, cudaMemcpyDeviceToHost, ctx->stream));
         PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
-        fprintf(stderr, "chain rt %d: lanes %d units %llu batches %llu jump rounds %llu | cycles/unit load %.0f "
-                "idle %.0f gwalk %.0f jump %.0f wait %.0f link %.0f walk %.0f write %.0f\n", rt, ca.nl, hd[8], hd[9],
+        fprintf(stderr, "chain rt %d: lanes %d units %llu batches %llu hops %llu | cycles/unit load %.0f "
+                "idle %.0f runs %.0f scan %.0f wait %.0f link %.0f rec %.0f write %.0f\n", rt, ca.nl, hd[8], hd[9],
                 hd[10], hd[0] / (double)hd[8], hd[1] / (double)hd[8], hd[2] / (double)hd[8], hd[3] / (double)hd[8],
-                hd[4] / (double)hd[8], hd[5] / (double)hd[8], hd[6] / (double)hd[8], hd[7] / (double)hd[8]);
+                hd[4] / (double)hd[8], hd[5] / (double)hd[8], hd[7] / (double)hd[8], hd[6] / (double)hd[8]);
+        std::vector<unsigned long long> pl(3 * (size_t)ca.nl);
+        PX_CUDA(ctx, cudaMemcpyAsync(pl.data(), ca.dbg + 16, pl.size() * 8, cudaMemcpyDeviceToHost, ctx->stream));
+        PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+        std::vector<int> ord(ca.nl);
+        for (int i = 0; i < ca.nl; i++) ord[i] = i;
+        std::sort(ord.begin(), ord.end(), [&](int x, int y) { return pl[3 * x] > pl[3 * y]; });
+        for (int k = 0; k < std::min(ca.nl, 12); k++) {
+          const int l = ord[k], lid = clid[rt][l];
+          fprintf(stderr, "  chain lane s=%d d=%d B=%d chunks=%d mode=%d: link Mcyc %.2f hops %llu wait Mcyc %.2f\n",
+                  lid / D, lid % D, hB[lid], cnch[rt][l], (int)cmodev[rt][l], pl[3 * l] / 1e6, pl[3 * l + 1],
+                  pl[3 * l + 2] / 1e6);
+        }
       }
 #endif
       unsigned wd = 0;

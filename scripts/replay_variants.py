@@ -30,7 +30,10 @@ for kind in ("poisson", "gamma"):
     sc = cfg["scenarios"]
     lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
     res = {}
+    keys = {k for _, envs in VARIANTS for k, _ in envs}
     for name, envs in VARIANTS:
+        for k in keys:  # every variant starts from the library defaults
+            os.environ.pop(k, None)
         for k, v in envs:
             os.environ[k] = v
         r0 = px.replay(arr, fam, sol.option, sol.z, cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
