@@ -2664,7 +2664,7 @@ static size_t chain_exoff(size_t nl) { return chain_ctroff(nl) + 16; }
 static size_t chain_smem(int C, int bmax) {
   const size_t E = (size_t)C + bmax + 2;
   return (size_t)C * 8 /* sFx */ + (size_t)bmax * 4 /* sT */ + E * 4 /* sA */ + (size_t)C * 4 /* sTi */ +
-         (size_t)C * 8 /* sNx, sJ, sJc, sHx */ + (size_t)C /* sB */ + 64;
+         (size_t)C * 10 /* sNx, sNc, sJ, sJc, sHx */ + (size_t)C /* sB */ + 64;
 }
 
 __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__ ChainArgs a) {
@@ -2676,7 +2676,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
   int32_t *sTi = (int32_t *)(sA + C + a.bmax + 2);  // [C] t_i(h) - a_h
   int16_t *sNx = (int16_t *)(sTi + C);              // [C] next idle-branch head in the segment, -1: leaves, -2: left to
                                                     // the walk, -3: leaves onto an idle-branch head in the chunk
-  int16_t *sJ = sNx + C;                            // [C] last idle-branch head of h's run in its segment
+  int16_t *sNc = sNx + C;                           // [C] next idle-branch head in the chunk, -1: leaves, -2: left to the walk
+  int16_t *sJ = sNc + C;                            // [C] last idle-branch head of h's run in its segment
   int16_t *sJc = sJ + C;                            // [C] last idle-branch head of h's run in the chunk
   int16_t *sHx = sJc + C;                           // [C] first head past the segment of a leaving run
   uint8_t *sB = (uint8_t *)(sHx + C);               // [C] b_i(h)
@@ -2826,24 +2827,38 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
         return ((int64_t)hh + Bm - 1 < nloc && (int64_t)sA[hh + Bm - 1] <= F) ? Bm
                                                                                : count_upto(A, nloc, (int64_t)hh, Bm, F);
       };
-      // the run of every head after its idle-branch decision, inside the
-      // head's segment (at most K greedy batches are followed here: -2 marks a
-      // head whose run is left to the link walk -- backlogged stretches would
-      // make this quadratic)
+      // the run of every head after its idle-branch decision (at most K
+      // greedy batches are followed here -- backlogged stretches would make
+      // this quadratic -- the rest is left to the link walk): inside the
+      // head's segment (sNx: the next idle-branch head, -1: the run leaves the
+      // segment at (sHx, sFx), -3: ... onto an idle-branch head, -2: left to
+      // the walk) and inside the chunk (sNc: the next idle-branch head, -1:
+      // the run leaves the chunk, -2: left to the walk)
       for (int i = tid; i < Cn; i += CHAIN_THREADS) {
         const int se = (i / SEG + 1) * SEG < Cn ? (i / SEG + 1) * SEG : Cn;
         const int bi = sB[i];
         int64_t F = (int64_t)sA[i] + sTi[i] + sT[bi - 1];
         int hh = i + bi;
+        bool segdone = false;
         for (int st = 0;; st++) {
-          if (hh >= se) {
-            sNx[i] = (hh < Cn && F <= (int64_t)sA[hh] + sTi[hh]) ? -3 : -1;
+          const bool node = hh < Cn && F <= (int64_t)sA[hh] + sTi[hh];
+          if (!segdone && hh >= se) {
+            sNx[i] = node ? -3 : -1;
             sHx[i] = (int16_t)hh;
             sFx[i] = F;
+            segdone = true;
+          }
+          if (hh >= Cn) { sNc[i] = -1; break; }
+          if (node) {
+            if (!segdone) sNx[i] = (int16_t)hh;
+            sNc[i] = (int16_t)hh;
             break;
           }
-          if (F <= (int64_t)sA[hh] + sTi[hh]) { sNx[i] = (int16_t)hh; break; }
-          if (st >= a.K) { sNx[i] = -2; break; }
+          if (st >= a.K) {
+            if (!segdone) sNx[i] = -2;
+            sNc[i] = -2;
+            break;
+          }
           const int g = greedy(hh, F);  // dispatched at F
           F += sT[g - 1];
           hh += g;
@@ -2852,13 +2867,12 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
       __syncthreads();
       CX_T(2);
       // the last idle-branch head of every head's run inside its segment (sJ)
-      // and inside the chunk (sJc: a run leaving its segment onto an
-      // idle-branch head continues with that head's): pointer jumping, in
-      // place (a pointer only ever moves further along its own run)
+      // and inside the chunk (sJc): pointer jumping, in place (a pointer only
+      // ever moves further along its own run)
       for (int i = tid; i < Cn; i += CHAIN_THREADS) {
-        const int nx = sNx[i];
+        const int nx = sNx[i], nc = sNc[i];
         sJ[i] = nx >= 0 ? (int16_t)nx : (int16_t)i;
-        sJc[i] = nx >= 0 ? (int16_t)nx : nx == -3 ? sHx[i] : (int16_t)i;
+        sJc[i] = nc >= 0 ? (int16_t)nc : (int16_t)i;
       }
       for (bool more = true; more;) {
         __syncthreads();
@@ -2894,9 +2908,18 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
         while (hh < Cn) {
           hops++;
           if (FF <= (int64_t)sA[hh] + sTi[hh]) {
+            // the run's last idle-branch head in the chunk; then its greedy
+            // batches (to the chunk's end when it leaves the chunk)
             const int r = sJc[hh];
-            if (sNx[r] == -1) { FF = sFx[r]; hh = sHx[r]; }
-            else { const int br = sB[r]; FF = (int64_t)sA[r] + sTi[r] + sT[br - 1]; hh = r + br; }
+            const int br = sB[r];
+            FF = (int64_t)sA[r] + sTi[r] + sT[br - 1];
+            hh = r + br;
+            if (sNc[r] == -1)
+              while (hh < Cn) {
+                const int g = greedy(hh, FF);
+                FF += sT[g - 1];
+                hh += g;
+              }
             continue;
           }
           const int k = stretch(hh, FF, Cn);
@@ -2929,9 +2952,16 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
         while (hh < Cn) {
           if (FF <= (int64_t)sA[hh] + sTi[hh]) {
             const int r = sJ[hh];
-            if (sNx[r] < -2 || sNx[r] == -1) { FF = sFx[r]; hh = sHx[r]; }
-            else { const int br = sB[r]; FF = (int64_t)sA[r] + sTi[r] + sT[br - 1]; hh = r + br; }
+            const int nx = sNx[r];
+            if (nx == -2) { const int br = sB[r]; FF = (int64_t)sA[r] + sTi[r] + sT[br - 1]; hh = r + br; rec(hh, FF); continue; }
+            FF = sFx[r];
+            hh = sHx[r];
             rec(hh, FF);
+            // a run leaving its segment busy: when its next idle-branch head
+            // (sNc) lies in the segment it entered, no other segment starts
+            // in between: continue there
+            const int nc = sNc[r];
+            if (nx == -1 && nc >= 0 && nc / SEG == hh / SEG) hh = nc;
             continue;
           }
           const int se = (hh / SEG + 1) * SEG < Cn ? (hh / SEG + 1) * SEG : Cn;
@@ -3239,9 +3269,9 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   // chain path (k_chain): the §5 lanes with T non-decreasing, 2 <= Bmax <= 255
   // and L < 2^30; the chunk runs + stitch take the other lanes
   const bool use_scan1 = !simple && env_int("PROTEUS_REPLAY_SCAN1", 1) != 0;
-  const bool use_chain = !simple && env_int("PROTEUS_REPLAY_CHAIN", 0) != 0 && max_rounds == 0 &&
+  const bool use_chain = !simple && env_int("PROTEUS_REPLAY_CHAIN", 1) != 0 && max_rounds == 0 &&
                          env_int("PROTEUS_REPLAY_TABLES", 0) == 0;
-  int CHN = env_int("PROTEUS_REPLAY_CHAIN_C", 2048);
+  int CHN = env_int("PROTEUS_REPLAY_CHAIN_C", 1024);
   CHN = CHN < 256 ? 256 : CHN > CHAIN_CMAX ? CHAIN_CMAX : CHN;  // shared-memory tables (~24 B per head)
   const int chain_minb = std::max(2, env_int("PROTEUS_REPLAY_CHAIN_MINB", 2));
   std::vector<int32_t> clid[2], cnch[2];
@@ -3301,7 +3331,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     // waits, lambda = the device's mean rate).  Small-batch lanes have long
     // serial walks per chunk here, while their chunk runs meet the true run at
     // once (the stitch accepts them), so they stay on the chunk runs + stitch.
-    const double minbatch = (double)env_int("PROTEUS_REPLAY_CHAIN_MINBATCH", 16);
+    const double minbatch = (double)env_int("PROTEUS_REPLAY_CHAIN_MINBATCH", 0);
     const double minrho = (double)env_int("PROTEUS_REPLAY_CHAIN_RHO_PCT", 100) / 100.0;
     const double span = (double)h_span[1] - (double)h_span[0];
     std::vector<uint8_t> hchain((size_t)S * D, 0);
@@ -3505,8 +3535,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     if (chain_now) {
       const int nl = (int)clid[rt].size();
       ca.D = D; ca.M = M; ca.bmax = ctx->bmax; ca.nl = nl; ca.C = CHN;
-      ca.K = std::max(0, env_int("PROTEUS_REPLAY_CHAIN_K", 8));
-      ca.SEG = std::min(CHN, std::max(CHAIN_SEGMIN, env_int("PROTEUS_REPLAY_CHAIN_SEG", 64)));
+      ca.K = std::max(0, env_int("PROTEUS_REPLAY_CHAIN_K", 16));
+      ca.SEG = std::min(CHN, std::max(CHAIN_SEGMIN, env_int("PROTEUS_REPLAY_CHAIN_SEG", 128)));
       ca.NS = NS; ca.maxch = cmax[rt]; ca.nunits = nunits[rt];
       ca.lid = (const int32_t *)cbuf[rt]; ca.nch = ca.lid + nl; ca.cmode = (const uint8_t *)(cbuf[rt] + (size_t)nl * 8);
       ca.counter = (unsigned long long *)(cbuf[rt] + chain_ctroff(nl));

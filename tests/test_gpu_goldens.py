@@ -107,14 +107,14 @@ def test_f4_bench_configuration_full_hour(px, oracle_mod):
             raise AssertionError(f"f4 scenario {sc[s]}: {len(bad)} latencies differ, first at {bad[0]}")
 
 
-@pytest.mark.parametrize("policies,env", [((0,), {}), ((1, 2), {}), ((0,), {"PROTEUS_REPLAY_CHAIN": "1"})],
-                         ids=["s5", "baselines", "s5_chain"])
+@pytest.mark.parametrize("policies,env", [((0,), {}), ((1, 2), {}), ((0,), {"PROTEUS_REPLAY_CHAIN": "0"})],
+                         ids=["s5", "baselines", "s5_stitch"])
 def test_c5_gamma_trace_full_size(px, oracle_mod, policies, env, monkeypatch):
     """Trace G of config 5: 10M queries with Gamma(shape 0.05) inter-arrivals
     (CV 4.47, the paper's bursty trace) at 3000 QPS on the c3
     allocation; the 64 (SLO x cap) scenarios of §5 batching (and, for f2, of
-    the two baseline batchers); every latency compared.  `s5_chain`: the
-    opt-in chain path for the §5 lanes it takes."""
+    the two baseline batchers); every latency compared.  `s5` runs the
+    default chain path, `s5_stitch` the chunk runs + stitch."""
     for k, v in env.items():
         monkeypatch.setenv(k, v)
     import torch

@@ -168,6 +168,18 @@ def test_replay_c5_full_size(px, oracle_mod):
         assert np.array_equal(g[k], o[k]), k
     glat = lat.cpu().numpy()
     assert np.array_equal(glat, o["latency"])
+    # the chunk runs + stitch on the same lanes (PROTEUS_REPLAY_CHAIN=0)
+    import os
+    os.environ["PROTEUS_REPLAY_CHAIN"] = "0"
+    try:
+        lat.fill_(0)
+        g = px.replay(torch.from_numpy(arr).cuda(), torch.from_numpy(fam).cuda(), r["option"], r["z"],
+                      cl.device_type, cfg["demand"][0], cl.slo_us, sc, latency=lat)
+    finally:
+        del os.environ["PROTEUS_REPLAY_CHAIN"]
+    for k in ("violations", "on_time", "acc_sum"):
+        assert np.array_equal(g[k], o[k]), k
+    assert np.array_equal(lat.cpu().numpy(), o["latency"])
 
 
 @pytest.mark.parametrize("policy", [1, 2])
