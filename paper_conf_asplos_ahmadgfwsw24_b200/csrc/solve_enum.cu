@@ -292,46 +292,38 @@ __device__ __forceinline__ FamState fam_state(const int (&c)[VM], int s, const F
 // The block's first candidate (index order: oA-major, then oB, idle first,
 // slots = codes in order) scoring Mx; returns its oA * K + oB, -1 if none
 // (an internal error, caught by the materialise check).  Rare: called when a
-// block beats the thread's running maximum, so it is kept out of line.
+// block beats the thread's running maximum, so it is kept out of line.  No
+// arrays indexed at run time (they would live in local memory): the block's
+// capacities are read from shared memory, family fills recomputed.
 template <int QM, int VM>
 __device__ __noinline__ int flat_rescan(const FlatArgs<QM, VM> &a, const int *sCaps /* [S][FLAT_THREADS] */,
-                                        const int32_t *sDem, int s3, int p3, uint64_t base, const uint64_t *Fq,
-                                        uint64_t Mx) {
+                                        const int32_t *sDem, int s3, int p3, uint64_t base, uint64_t Mx) {
   constexpr int S = QM * VM;
   const int K = a.K;
-  int c3[S];
+  // capacity of slot k with devices 0..D-3 placed, plus device D-2 (sa) / D-1 (sb) when given
+  auto cap = [&](int k, int sa, int sb) -> int {
+    return sCaps[k * FLAT_THREADS + threadIdx.x] + (k == s3 ? p3 : 0) + (k == sa ? a.PA[k] : 0) +
+           (k == sb ? a.PB[k] : 0);
+  };
+  auto fill = [&](int q, int sa, int sb) -> uint64_t {  // family q's water-fill value
+    int c[VM];
 #pragma unroll
-  for (int k = 0; k < S; k++) c3[k] = sCaps[k * FLAT_THREADS + threadIdx.x] + (k == s3 ? p3 : 0);
-  uint64_t dB[S];
-#pragma unroll
+    for (int j = 0; j < VM; j++) c[j] = cap(q * VM + j, sa, sb);
+    return fam_fill<QM, VM>(c, sDem[q], a, q);
+  };
+  if (base == Mx) return 0;  // (idle, idle)
   for (int sb = 0; sb < S; sb++) {
     const int qb = sb / VM;
-    int cb[VM];
-#pragma unroll
-    for (int j = 0; j < VM; j++) cb[j] = c3[qb * VM + j] + (j == sb % VM ? a.PB[sb] : 0);
-    dB[sb] = fam_fill<QM, VM>(cb, sDem[qb], a, qb) - Fq[qb];
+    if (base - fill(qb, -1, -1) + fill(qb, -1, sb) == Mx) return a.code[sb];
   }
-  if (base == Mx) return 0;  // (idle, idle)
-  for (int sb = 0; sb < S; sb++)
-    if (base + dB[sb] == Mx) return a.code[sb];
   for (int sa = 0; sa < S; sa++) {
     const int qa = sa / VM;
-    int ca[VM];
-#pragma unroll
-    for (int j = 0; j < VM; j++) ca[j] = c3[qa * VM + j] + (j == sa % VM ? a.PA[sa] : 0);
-    const uint64_t ba = base - Fq[qa] + fam_fill<QM, VM>(ca, sDem[qa], a, qa);
+    const uint64_t Fa = fill(qa, -1, -1);
+    const uint64_t ba = base - Fa + fill(qa, sa, -1);
     if (ba == Mx) return a.code[sa] * K;
     for (int sb = 0; sb < S; sb++) {
       const int qb = sb / VM;
-      uint64_t v;
-      if (qb == qa) {
-        int cj[VM];
-#pragma unroll
-        for (int j = 0; j < VM; j++) cj[j] = ca[j] + (j == sb % VM ? a.PB[sb] : 0);
-        v = base - Fq[qa] + fam_fill<QM, VM>(cj, sDem[qa], a, qa);
-      } else {
-        v = ba + dB[sb];
-      }
+      const uint64_t v = qb == qa ? base - Fa + fill(qa, sa, sb) : ba - fill(qb, -1, -1) + fill(qb, -1, sb);
       if (v == Mx) return a.code[sa] * K + a.code[sb];
     }
   }
@@ -475,11 +467,8 @@ __global__ void __launch_bounds__(FLAT_THREADS, FLAT_MINB) k_flat_fam(const __gr
         if (!rec) take = G == 0 || Mx > G - 1;
         else take = Mx > best_s && (G == 0 || Mx > G - 1);
         if (take) {
-          uint64_t Fq[QM];
-#pragma unroll
-          for (int q = 0; q < QM; q++) Fq[q] = q == q3 ? m.F : st[q].F;
           const int lp = flat_rescan<QM, VM>(a, &sCaps[0][0], sDem, s3, s3 >= 0 ? sP[(D - 3) * K + o3] : 0, base,
-                                             Fq, Mx);
+                                             Mx);
           best_s = Mx;
           best_i = o * K3 + (uint64_t)o3 * K2 + (uint64_t)(lp < 0 ? 0 : lp);
           rec = true;
