@@ -324,7 +324,8 @@ struct LaneArgs {
   int maxchk;             // convergence checks per chunk (free decisions only)
   int scan1;              // Bmax = 1 lanes are produced by k_scan1_* (the chunk kernels skip them)
   uint64_t dmask;         // devices whose lanes this launch of k_spec / k_fix / k_stitch takes
-  const int64_t *lstart;  // [S * D][2] (head, F) where k_stitch starts a lane the full-batch scan took (head -1: not taken)
+  int64_t *lstart;        // [S * D][2] (head, F) where k_stitch starts a lane the full-batch scan took (head -1: not taken);
+                          // also the Nexus scan's start / end states (k_wc_lanes, nxmode)
   unsigned *lstat;        // [S * D][2] speculative decisions that were full batches sent when the device
                           // freed (backlog), and all speculative decisions; k_fix leaves backlogged lanes
                           // (a quarter or more) to the stitch's max-plus stretches
@@ -347,6 +348,12 @@ struct LaneArgs {
   const int32_t *lane_order;  // k_stitch: lane (list position * D + d) of warp i (null: identity)
   int bsearch;                // k_stitch: binary-search decisions (fast_decide) on lanes with T non-decreasing
   const uint8_t *skip;        // [S * D] 1: the chunk / lane kernels leave the lane alone (a duplicate lane, or k_chain's)
+  // Nexus overload scan (k_nx_*): nxsel[s * D + d] = 1 for the lanes it takes;
+  // nxmode 1: k_wc_lanes walks those lanes only up to their first overload
+  // stretch and records the state there (lstart), the others whole; nxmode 2:
+  // only the selected lanes, from lstart (the state after the scan's batches)
+  const uint8_t *nxsel;
+  int nxmode;
 };
 
 struct WcExit {  // a baseline chunk run left its chunk at head h (>= chunk end), device free at F;
@@ -579,6 +586,8 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
   if (wid >= a.nsc * a.D) return;
   const int s = a.sc_list[wid / a.D], d = wid % a.D;
   if (a.skip && a.skip[s * a.D + d]) return;
+  const bool nxs = a.nxsel && a.nxsel[s * a.D + d];
+  if (a.nxmode == 2 && !nxs) return;
   const LaneParam p = a.lp[s * a.D + d];
   const int64_t st = a.devOff[d], n = a.devOff[d + 1] - st;
   if (n == 0) return;
@@ -608,6 +617,11 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
   const bool nexus = p.policy == 1;
   const int B = nexus ? p.Bn : p.Bmax;
   int64_t h = 0, tail = 0, F = 0;  // R13
+  if (nxs && a.nxmode == 2) {      // after the overload scan's batches
+    h = a.lstart[2 * ((size_t)s * a.D + d)];
+    F = a.lstart[2 * ((size_t)s * a.D + d) + 1];
+    tail = h;
+  }
   int limit = 1;                   // AIMD batch-size limit
   const int64_t T1 = T[0];
   const bool fast = T1 <= p.L;     // isolated queries are on time
@@ -641,7 +655,10 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
         continue;
       }
     }
-    if (nexus ? B == 1 : limit == 1) {
+    // Nexus with B = 1 takes the overload stretch below (when the device is
+    // busy) before the batches of one
+    const bool nx1 = nexus && B == 1 && try_stretch && F > A(h) && --stretch_wait <= 0;
+    if (!nx1 && (nexus ? B == 1 : limit == 1)) {
       // Batches of one, 32 per step: query h + k leaves at max(F_{k-1}, a)
       // (work-conserving), F_k = max(F_{k-1}, a_{h+k}) + T(1), i.e. F_k - (k+1) T(1)
       // = max(F, max_{i<=k} a_{h+i} - i T(1)) -- a warp max-scan.  AIMD keeps
@@ -671,6 +688,7 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
         if (m) { r = __ffs(m); limit = 2; }
       }
       const int served = drop_last ? r - 1 : r;
+      if (nexus && drop_last) try_stretch = true;  // dropping: overload, a stretch may follow
       if (lane < served) out[j] = sat_lat(Fk - aj);
       if (drop_last && lane == r - 1) out[j] = 0xFFFFFFFFu;
       if (served > 0) F = __shfl_sync(0xffffffffu, Fk, served - 1);
@@ -679,7 +697,7 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
       continue;
     }
     const int64_t ah = A(h);
-    if (nexus && B > 1 && F > ah && try_stretch && --stretch_wait <= 0) {
+    if (nexus && F > ah && try_stretch && (B == 1 ? nx1 : --stretch_wait <= 0)) {
       // Overload stretch (Nexus): the device is busy at every decision and the
       // queue holds a full window, so batch k of the stretch is decided at
       // t_k = F + k T(B): the window of B from the head passes iff a_i >=
@@ -713,6 +731,13 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
       const bool ok = ik + B <= n && pk < n && A(pk) <= tk && A(ik + B - 1) <= tk;
       const unsigned vm = __ballot_sync(0xffffffffu, ok);
       const int r = vm == 0xffffffffu ? 32 : __ffs(~vm) - 1;
+      if (r == 32 && nxs && a.nxmode == 1) {  // the state where the overload scan takes over
+        if (lane == 0) {
+          a.lstart[2 * ((size_t)s * a.D + d)] = h;
+          a.lstart[2 * ((size_t)s * a.D + d) + 1] = F;
+        }
+        return;
+      }
       if (r > 0) {
         dbg_st++; dbg_stb += r;
         stretch_wait = r < 4 ? 8 : 0;  // short stretches do not pay for the test: back off
@@ -787,6 +812,10 @@ __global__ void __launch_bounds__(128) k_wc_lanes(const __grid_constant__ LaneAr
       else limit = limit + 1 > p.Bmax ? p.Bmax : limit + 1;
     }
     h = first + b;
+  }
+  if (nxs && a.nxmode == 1 && lane == 0) {  // walked to the end: nothing left for the scan / the second walk
+    a.lstart[2 * ((size_t)s * a.D + d)] = n;
+    a.lstart[2 * ((size_t)s * a.D + d) + 1] = F;
   }
   if (a.debug && lane == 0 && clock64() - dbg_t0 > a.debug)
     printf("wc s=%d d=%d n=%lld pol=%d B=%d cycles=%lld steps=%lld stretches=%lld stretch_batches=%lld\n", s, d,
@@ -1929,6 +1958,224 @@ __global__ void __launch_bounds__(256) k_bscan_apply(const __grid_constant__ BSc
     a.lstart[2 * (size_t)L.lane] = kstar * L.B;
     a.lstart[2 * (size_t)L.lane + 1] = kstar == 0 ? 0 : Fs[kstar - 1 - kb];
   }
+}
+
+// ---- §8(f2) Nexus overload scan (reading R14)
+// In an overload stretch of a Nexus lane (the device busy at every decision,
+// a full window queued) batch k is decided at t_k = F + k T(B) from the state
+// (h, F) where the stretch starts; its window starts at i_k = max(p_k, g_k),
+// g_k = the first arrival >= t_k + T(B) - L, p_k = i_{k-1} + B (p_0 = h), and
+// [p_k, i_k) are dropped: i_k = k B + max(h, max_{j<=k} (g_j - j B)), a prefix
+// maximum (k_wc_lanes's stretch, 32 batches per warp step).  The scan takes the
+// whole lane at once from the state k_wc_lanes recorded at its first stretch
+// (nxmode 1): the g_k are independent searches, the prefix maximum a
+// two-level scan, and the stretch is exact up to the first batch that is not
+// valid (a_{p_k} <= t_k: busy; a_{i_k + B - 1} <= t_k: full window), where
+// the second walk of k_wc_lanes takes over.  Block = NX_BLK batches of a lane.
+#define NX_BLK 1024
+struct NxArgs {
+  int D, nl;
+  int64_t NS;
+  const int64_t *loff;       // [nl + 1] block offsets per lane
+  const int32_t *lid;        // [nl] lane = s * D + d
+  const int64_t *devOff;
+  const uint32_t *devArr;
+  const int32_t *lat, *option, *dev_type;
+  int M, bmax;
+  const LaneParam *lp;
+  int64_t *lstart;           // [S * D][2] (h, F): the scan's start, then the second walk's
+  uint32_t *latd;
+  int64_t *bmx, *bpre;       // [blocks]
+  int32_t *ik;               // [blocks * NX_BLK] window heads i_k (device-relative)
+  unsigned long long *vio;   // [nl] first invalid batch (init ~0)
+  int64_t *nxst;             // [nl][2] the second walk's start (k_nx_apply), copied to lstart by k_nx_commit
+};
+
+struct NxLane {
+  int64_t off, n, h0, F0, TB, L, nb;
+  int B, lane, blk;
+  bool on;
+};
+
+__device__ __forceinline__ NxLane nx_lane(const NxArgs &a, int64_t b) {
+  NxLane r;
+  int lo = 0, hi = a.nl;
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (__ldg(a.loff + mid) <= b) lo = mid; else hi = mid;
+  }
+  r.lane = a.lid[lo];
+  r.blk = (int)(b - a.loff[lo]);
+  const int d = r.lane % a.D;
+  const LaneParam p = a.lp[r.lane];
+  r.B = p.Bn;
+  r.L = p.L;
+  r.off = a.devOff[d];
+  r.n = a.devOff[d + 1] - r.off;
+  r.h0 = a.lstart[2 * (size_t)r.lane];
+  r.F0 = a.lstart[2 * (size_t)r.lane + 1];
+  r.on = r.h0 >= 0 && r.h0 < r.n && r.B >= 1;
+  const int32_t *T = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+  r.TB = T[r.B - 1];
+  r.nb = r.on ? (r.n - r.h0) / r.B : 0;  // at most this many batches (i_k >= h0 + k B)
+  return r;
+}
+
+// g_k - k B with g_k clamped below by h0 + k B (only larger values matter)
+__device__ __forceinline__ int64_t nx_m(const NxArgs &a, const NxLane &L, int64_t k) {
+  const uint32_t *arr = a.devArr + L.off;
+  const int64_t thr = L.F0 + (k + 1) * L.TB - L.L;
+  int64_t x = L.h0 + k * L.B;
+  if (x < L.n && (int64_t)__ldg(arr + x) < thr) {  // gallop, then bisect
+    int64_t lo = x, step = 1, hi = x + 1;
+    while (hi < L.n && (int64_t)__ldg(arr + hi) < thr) { lo = hi; step <<= 1; hi = x + step; }
+    if (hi > L.n) hi = L.n;
+    while (hi - lo > 1) {
+      const int64_t mid = (lo + hi) >> 1;
+      if ((int64_t)__ldg(arr + mid) < thr) lo = mid; else hi = mid;
+    }
+    x = hi;
+  }
+  return x - k * L.B;
+}
+
+__global__ void __launch_bounds__(256) k_nx_reduce(const __grid_constant__ NxArgs a) {
+  const NxLane L = nx_lane(a, blockIdx.x);
+  int64_t m = INT64_MIN;
+  if (L.on) {
+    const int64_t k0 = (int64_t)L.blk * NX_BLK;
+    for (int64_t k = k0 + threadIdx.x; k < k0 + NX_BLK && k < L.nb; k += blockDim.x) {
+      const int64_t v = nx_m(a, L, k);
+      m = v > m ? v : m;
+    }
+  }
+  __shared__ int64_t red[8];
+  for (int o = 16; o; o >>= 1) {
+    const int64_t v = __shfl_xor_sync(0xffffffffu, m, o);
+    m = v > m ? v : m;
+  }
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = m;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int k = 1; k < 8; k++) m = red[k] > m ? red[k] : m;
+    a.bmx[blockIdx.x] = m;
+  }
+}
+
+__global__ void k_nx_prefix(const __grid_constant__ NxArgs a) {  // warp per lane: exclusive block prefix
+  const int l = blockIdx.x, lane = threadIdx.x;
+  int64_t carry = INT64_MIN;
+  for (int64_t b0 = a.loff[l]; b0 < a.loff[l + 1]; b0 += 32) {
+    const int64_t b = b0 + lane;
+    int64_t v = b < a.loff[l + 1] ? a.bmx[b] : INT64_MIN;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t u = __shfl_up_sync(0xffffffffu, v, o);
+      if (lane >= o && u > v) v = u;
+    }
+    int64_t ex = __shfl_up_sync(0xffffffffu, v, 1);
+    if (lane == 0) ex = INT64_MIN;
+    if (b < a.loff[l + 1]) a.bpre[b] = ex > carry ? ex : carry;
+    const int64_t tot = __shfl_sync(0xffffffffu, v, 31);
+    carry = tot > carry ? tot : carry;
+  }
+}
+
+// window heads of the block's batches (block-wide inclusive max-scan with the
+// lane's prefix), then the validity test; the first invalid batch -> vio
+__global__ void __launch_bounds__(256) k_nx_verify(const __grid_constant__ NxArgs a) {
+  const NxLane L = nx_lane(a, blockIdx.x);
+  if (!L.on) return;
+  const int64_t k0 = (int64_t)L.blk * NX_BLK;
+  if (k0 >= L.nb) return;
+  constexpr int PER = NX_BLK / 256;
+  int64_t v[PER];
+  int64_t tm = INT64_MIN;
+#pragma unroll
+  for (int q = 0; q < PER; q++) {
+    const int64_t k = k0 + threadIdx.x * PER + q;
+    v[q] = k < L.nb ? nx_m(a, L, k) : INT64_MIN;
+    tm = v[q] > tm ? v[q] : tm;
+  }
+  // exclusive scan of the thread maxima across the block
+  __shared__ int64_t wsum[8];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  int64_t x = tm;
+  for (int o = 1; o < 32; o <<= 1) {
+    const int64_t u = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o && u > x) x = u;
+  }
+  if (lane == 31) wsum[w] = x;
+  int64_t ex = __shfl_up_sync(0xffffffffu, x, 1);
+  if (lane == 0) ex = INT64_MIN;
+  __syncthreads();
+  int64_t carry = a.bpre[blockIdx.x];
+  carry = carry > L.h0 ? carry : L.h0;
+  for (int k = 0; k < w; k++) carry = wsum[k] > carry ? wsum[k] : carry;
+  carry = ex > carry ? ex : carry;
+  const uint32_t *arr = a.devArr + L.off;
+  int32_t *ik = a.ik + (size_t)blockIdx.x * NX_BLK;
+#pragma unroll
+  for (int q = 0; q < PER; q++) {
+    const int64_t k = k0 + threadIdx.x * PER + q;
+    carry = v[q] > carry ? v[q] : carry;
+    if (k >= L.nb) break;
+    ik[threadIdx.x * PER + q] = (int32_t)(k * L.B + carry);  // i_k
+  }
+  __syncthreads();
+  // validity: p_k = i_{k-1} + B (p_0 = h0); a[p_k] <= t_k and a[i_k + B - 1] <= t_k
+  for (int j = threadIdx.x; j < NX_BLK; j += blockDim.x) {
+    const int64_t k = k0 + j;
+    if (k >= L.nb) break;
+    const int64_t i = ik[j];
+    // i_{k0 - 1} from the lane's exclusive block prefix (another block's)
+    const int64_t pb = a.bpre[blockIdx.x] > L.h0 ? a.bpre[blockIdx.x] : L.h0;
+    const int64_t pk = k == 0 ? L.h0 : (j > 0 ? (int64_t)ik[j - 1] : (k0 - 1) * L.B + pb) + L.B;
+    const int64_t tk = L.F0 + k * L.TB;
+    const bool ok = i + L.B <= L.n && pk < L.n && (int64_t)__ldg(arr + pk) <= tk &&
+                    (int64_t)__ldg(arr + i + L.B - 1) <= tk;
+    if (!ok) {
+      int l = 0, hi = a.nl;
+      while (hi - l > 1) { const int mid = (l + hi) >> 1; if (__ldg(a.loff + mid) <= (int64_t)blockIdx.x) l = mid; else hi = mid; }
+      atomicMin(a.vio + l, (unsigned long long)k);
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_nx_apply(const __grid_constant__ NxArgs a) {
+  const NxLane L = nx_lane(a, blockIdx.x);
+  if (!L.on) return;
+  int l = 0, hi = a.nl;
+  while (hi - l > 1) { const int mid = (l + hi) >> 1; if (__ldg(a.loff + mid) <= (int64_t)blockIdx.x) l = mid; else hi = mid; }
+  const unsigned long long v = a.vio[l];
+  const int64_t kstar = v < (unsigned long long)L.nb ? (int64_t)v : L.nb;  // batches taken
+  const int64_t k0 = (int64_t)L.blk * NX_BLK;
+  const uint32_t *arr = a.devArr + L.off;
+  uint32_t *out = a.latd + (size_t)(L.lane / a.D) * a.NS + L.off;
+  const int32_t *ik = a.ik + (size_t)blockIdx.x * NX_BLK;
+  for (int j = threadIdx.x; j < NX_BLK; j += blockDim.x) {
+    const int64_t k = k0 + j;
+    if (k >= kstar) break;
+    const int64_t i = ik[j];
+    const int64_t pb = a.bpre[blockIdx.x] > L.h0 ? a.bpre[blockIdx.x] : L.h0;
+    const int64_t pk = k == 0 ? L.h0 : (j > 0 ? (int64_t)ik[j - 1] : (k0 - 1) * L.B + pb) + L.B;
+    for (int64_t q = pk; q < i; q++) out[q] = 0xFFFFFFFFu;  // dropped early
+    const int64_t Fk = L.F0 + (k + 1) * L.TB;
+    for (int q = 0; q < L.B; q++) out[i + q] = sat_lat(Fk - (int64_t)__ldg(arr + i + q));
+  }
+  // the second walk starts at batch k* with the device free at F0 + k* T(B)
+  const bool mine = (kstar == 0 && L.blk == 0) || (kstar > k0 && kstar <= k0 + NX_BLK);
+  if (threadIdx.x == 0 && mine) {  // (lstart itself is the start every block of the lane reads)
+    a.nxst[2 * (size_t)l] = kstar == 0 ? L.h0 : (int64_t)ik[kstar - 1 - k0] + L.B;
+    a.nxst[2 * (size_t)l + 1] = L.F0 + kstar * L.TB;
+  }
+}
+
+__global__ void k_nx_commit(const __grid_constant__ NxArgs a) {
+  for (int l = blockIdx.x * blockDim.x + threadIdx.x; l < a.nl; l += gridDim.x * blockDim.x)
+    if (a.nxst[2 * (size_t)l] >= 0) {
+      a.lstart[2 * (size_t)a.lid[l]] = a.nxst[2 * (size_t)l];
+      a.lstart[2 * (size_t)a.lid[l] + 1] = a.nxst[2 * (size_t)l + 1];
+    }
 }
 
 // dropped queries (the sink segment, device index D): latency UINT32_MAX (R7)
@@ -3827,7 +4074,72 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
         PX_LAUNCH(ctx, "replay_baseline", k_wc_spec, gs, 128, 0, la2);
       }
       const int64_t warps = (int64_t)lb.nsc * D;
-      if (lb.wst) PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<true>, (unsigned)((warps + 3) / 4), 128, 0, lb);
+      // Nexus lanes predicted at or past overload at their batch size (rho =
+      // lambda T(B) / B, lambda the device's mean rate): k_wc_lanes walks them
+      // to their first overload stretch, the scan (k_nx_*) takes the stretch
+      // as far as it is valid, the second walk the rest
+      if (!simple && env_int("PROTEUS_REPLAY_NXSCAN", 0) != 0) {  // opt-in: measured slower on c5
+        const double rho_min = env_int("PROTEUS_REPLAY_NXSCAN_RHO_PCT", 95) / 100.0;
+        const double span = (double)h_span[1] - (double)h_span[0];
+        std::vector<uint8_t> sel((size_t)S * D, 0);
+        std::vector<int32_t> lid;
+        std::vector<int64_t> loff(1, 0);
+        for (int k : scl[4 + rt]) {
+          if (h_sc[k].policy != 1) continue;
+          for (int d = 0; d < D; d++) {
+            if (h_option[d] <= 0 || hskip[(size_t)k * D + d]) continue;
+            const int32_t *Tr = ctx->lat.data() + ((size_t)h_dev_type[d] * M + (h_option[d] - 1)) * ctx->bmax;
+            const int64_t L = lane_L(k, d);
+            int Bn = 1;
+            for (int b = 1; b <= hB[(size_t)k * D + d]; b++)
+              if (2 * (int64_t)Tr[b - 1] <= L) Bn = b;
+            const int64_t nd = h_off[rt][d + 1] - h_off[rt][d];
+            const double lam = span > 0 ? (double)nd / span : 0.0;
+            if (nd < 2 * Bn || lam * (double)Tr[Bn - 1] / (double)Bn < rho_min) continue;
+            sel[(size_t)k * D + d] = 1;
+            lid.push_back(k * D + d);
+            loff.push_back(loff.back() + (nd / Bn + NX_BLK) / NX_BLK);
+          }
+        }
+        const int nl = (int)lid.size();
+        const int64_t nb = loff.back();
+        if (nl > 0) {
+          if (nb > 0x7fffffff) return px_fail(ctx, PROTEUS_ERANGE, "scan blocks");
+          const size_t o_loff = ((size_t)S * D + 15) & ~(size_t)15, o_lid = o_loff + (size_t)(nl + 1) * 8,
+                       o_b = (o_lid + (size_t)nl * 4 + 15) & ~(size_t)15, o_vio = o_b + (size_t)nb * 16,
+                       o_st = o_vio + (size_t)nl * 8, o_ik = o_st + (size_t)nl * 16,
+                       tot = o_ik + (size_t)nb * NX_BLK * 4;
+          char *nx = (char *)px_buf(ctx, B_R_NX, tot + 64);
+          if (!nx) return px_fail(ctx, PROTEUS_ENOMEM, "Nexus scan buffers");
+          PX_CUDA(ctx, cudaMemcpyAsync(nx, sel.data(), sel.size(), cudaMemcpyHostToDevice, ctx->stream));
+          PX_CUDA(ctx, cudaMemcpyAsync(nx + o_loff, loff.data(), loff.size() * 8, cudaMemcpyHostToDevice, ctx->stream));
+          PX_CUDA(ctx, cudaMemcpyAsync(nx + o_lid, lid.data(), lid.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+          PX_CUDA(ctx, cudaMemsetAsync(nx + o_vio, 0xFF, (size_t)nl * 24, ctx->stream));  // vio, nxst
+          NxArgs na;
+          memset(&na, 0, sizeof na);
+          na.D = D; na.nl = nl; na.NS = NS; na.loff = (const int64_t *)(nx + o_loff); na.lid = (const int32_t *)(nx + o_lid);
+          na.devOff = devOff[rt]; na.devArr = devArr[rt]; na.lat = ctx->d_lat; na.option = d_opt; na.dev_type = d_dev;
+          na.M = M; na.bmax = ctx->bmax; na.lp = d_lp; na.lstart = d_lstart; na.latd = latd;
+          na.bmx = (int64_t *)(nx + o_b); na.bpre = na.bmx + nb; na.ik = (int32_t *)(nx + o_ik);
+          na.vio = (unsigned long long *)(nx + o_vio);
+          na.nxst = (int64_t *)(nx + o_st);
+          lb.nxsel = (const uint8_t *)nx;
+          lb.nxmode = 1;
+          if (lb.wst) PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<true>, (unsigned)((warps + 3) / 4), 128, 0, lb);
+          else PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<false>, (unsigned)((warps + 3) / 4), 128, 0, lb);
+          PX_LAUNCH(ctx, "replay_nxscan", k_nx_reduce, (unsigned)nb, 256, 0, na);
+          PX_LAUNCH(ctx, "replay_nxscan", k_nx_prefix, nl, 32, 0, na);
+          PX_LAUNCH(ctx, "replay_nxscan", k_nx_verify, (unsigned)nb, 256, 0, na);
+          PX_LAUNCH(ctx, "replay_nxscan", k_nx_apply, (unsigned)nb, 256, 0, na);
+          PX_LAUNCH(ctx, "replay_nxscan", k_nx_commit, 1, 256, 0, na);
+          lb.nxmode = 2;
+          PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<false>, (unsigned)((warps + 3) / 4), 128, 0, lb);
+          PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // sel / loff / lid are host vectors
+        }
+      }
+      if (lb.nxmode == 2) {
+        // done above
+      } else if (lb.wst) PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<true>, (unsigned)((warps + 3) / 4), 128, 0, lb);
       else PX_LAUNCH(ctx, "replay_baseline", k_wc_lanes<false>, (unsigned)((warps + 3) / 4), 128, 0, lb);
     }
     if (!d_lat_out || env_int("PROTEUS_REPLAY_FINISH", 0) == 0) {  // counts from the device-major rows

@@ -236,6 +236,25 @@ def test_replay_baseline_policies(px, oracle_mod, kind, policy):
             assert np.all(g["violations"] + g["on_time"] == len(arr))
 
 
+@pytest.mark.parametrize("kind", ["poisson", "gamma"])
+@pytest.mark.parametrize("rho", ["0", "95"])
+def test_replay_nexus_overload_scan(px, oracle_mod, kind, rho, monkeypatch):
+    """§8(f2) Nexus lanes through the opt-in overload scan (k_nx_*): the first
+    walk stops at a lane's first overload stretch, the scan takes the stretch
+    as far as it is valid, the second walk the rest (every Nexus lane selected
+    at rho 0); bit-exact against the oracle, light load and overload."""
+    monkeypatch.setenv("PROTEUS_REPLAY_NXSCAN", "1")
+    monkeypatch.setenv("PROTEUS_REPLAY_NXSCAN_RHO_PCT", rho)
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    for v, n in ((0, 60_000), (1, 80_000)):
+        r = _alloc(oracle_mod, cfg, v)
+        arr, fam = W.query_trace(n, float(cfg["demand"][v].sum()), cfg["weights"], 17 + v, kind)
+        for routing in (0, 1):
+            _compare(px, oracle_mod, cfg["prof"], cfg["cluster"], r["option"], r["z"], cfg["demand"][v], arr, fam,
+                     W.scenarios_64(routing, 1))
+
+
 def test_replay_mixed_policies_one_call(px, oracle_mod):
     """All three policies in one call (Fig. 6 grid, both routings): the §5
     scenarios take the chunk/stitch path, the baselines k_wc_lanes, and the
