@@ -212,14 +212,15 @@ int px_pareto_merge(proteus_ctx *ctx, const proteus_pareto_point *d_pts, int n, 
 // ----------------------------------------------- scenario assignment ----
 // Relative cost of one replay scenario's lanes (host; a deterministic model
 // from the measured 1-GPU time of every c5 scenario replayed alone,
-// profiles/r02d_scenario_costs.json): §5 lanes with Bmax = 1
+// profiles/r02g_scenario_costs.json): §5 lanes with Bmax = 1
 // are one exact prefix-max scan (0.7 ms); every other §5 scenario costs about
-// the same (8-19 ms, set by its slowest stitch lane); Clipper AIMD 27-77 ms
-// and Nexus 220-440 ms (sequential chains of the overloaded lanes).
+// the same (6-9.5 ms, the chain path's longest lane); Clipper AIMD 29-81 ms;
+// Nexus 58-250 ms at batch cap 1 (the overload stretches) and 230-475 ms
+// otherwise (sequential chains of the busy lanes).
 static double scenario_cost(const proteus_scenario &s) {
-  if (s.policy == 1) return 32.0;   // Nexus early drop
-  if (s.policy == 2) return 3.5;    // Clipper AIMD
-  return s.batch_cap == 1 ? 0.06 : 1.0;
+  if (s.policy == 1) return s.batch_cap == 1 ? 12.0 : 62.0;  // Nexus early drop
+  if (s.policy == 2) return 7.0;                              // Clipper AIMD
+  return s.batch_cap == 1 ? 0.11 : 1.0;
 }
 
 // Longest-processing-time greedy: scenarios by decreasing cost (ties by
