@@ -2875,6 +2875,9 @@ __global__ void __launch_bounds__(256) k_finish(int64_t N, int64_t NS, int S, in
 #define CHAIN_WARPS (CHAIN_THREADS / 32)
 #define CHAIN_CMAX 8192   // largest chunk (heads are int16 in the tables)
 #define CHAIN_SEGMIN 16   // smallest segment
+#ifndef CHAIN_MINB
+#define CHAIN_MINB 6      // blocks per SM (40 registers; 8 blocks at 32 registers measured slower)
+#endif
 #ifdef PX_CHAIN_DEBUG  // per-phase cycle totals of k_chain (thread 0), printed by the host
 #define CX_T(k) do { if (threadIdx.x == 0) { const long long t_ = clock64(); atomicAdd(a.dbg + (k), (unsigned long long)(t_ - cx_t)); cx_t = t_; } } while (0)
 #else
@@ -2908,20 +2911,25 @@ struct ShArr {  // arrivals of a chunk in shared memory, from its first head
 // per routing mode: lid [nl] i32, nch [nl] i32, cmode [nl] u8, ticket + watchdog, exits [nl][maxch] u64
 static size_t chain_ctroff(size_t nl) { return (nl * 9 + 15) & ~(size_t)15; }
 static size_t chain_exoff(size_t nl) { return chain_ctroff(nl) + 16; }
-static size_t chain_smem(int C, int bmax) {
+static size_t chain_smem(int C, int bmax, int SEG) {
   const size_t E = (size_t)C + bmax + 2;
-  return (size_t)C * 8 /* sFx */ + (size_t)bmax * 4 /* sT */ + E * 4 /* sA */ + (size_t)C * 4 /* sTi */ +
-         (size_t)C * 10 /* sNx, sNc, sJ, sJc, sHx */ + (size_t)C /* sB */ + 64;
+  const size_t nseg = ((size_t)C + SEG - 1) / SEG;
+  return (size_t)C * 8 /* sFx */ + nseg * 8 /* sSegF */ + (size_t)bmax * 4 /* sT */ + E * 4 /* sA */ +
+         (size_t)C * 4 /* sTi */ + nseg * 4 /* sSegH */ + (size_t)C * 10 /* sNx, sNc, sJ, sJc, sHx */ +
+         (size_t)C /* sB */ + 64;
 }
 
-__global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__ ChainArgs a) {
+__global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __grid_constant__ ChainArgs a) {
   extern __shared__ __align__(16) unsigned char csm[];
   const int C = a.C, SEG = a.SEG;
+  const int NSEG = (C + SEG - 1) / SEG;
   int64_t *sFx = (int64_t *)csm;                    // [C] free time when a head's run leaves its segment
-  int32_t *sT = (int32_t *)(sFx + C);               // [bmax] T(b) at b - 1
+  int64_t *sSegF = sFx + C;                         // [NSEG] true free time at the first batch head of a segment
+  int32_t *sT = (int32_t *)(sSegF + NSEG);          // [bmax] T(b) at b - 1
   uint32_t *sA = (uint32_t *)(sT + a.bmax);         // [C + bmax + 2] arrivals from the chunk start
   int32_t *sTi = (int32_t *)(sA + C + a.bmax + 2);  // [C] t_i(h) - a_h
-  int16_t *sNx = (int16_t *)(sTi + C);              // [C] next idle-branch head in the segment, -1: leaves, -2: left to
+  int *sSegH = (int *)(sTi + C);                    // [NSEG] ... and that head (-1: not recorded yet)
+  int16_t *sNx = (int16_t *)(sSegH + NSEG);              // [C] next idle-branch head in the segment, -1: leaves, -2: left to
                                                     // the walk, -3: leaves onto an idle-branch head in the chunk
   int16_t *sNc = sNx + C;                           // [C] next idle-branch head in the chunk, -1: leaves, -2: left to the walk
   int16_t *sJ = sNc + C;                            // [C] last idle-branch head of h's run in its segment
@@ -2929,8 +2937,6 @@ __global__ void __launch_bounds__(CHAIN_THREADS) k_chain(const __grid_constant__
   int16_t *sHx = sJc + C;                           // [C] first head past the segment of a leaving run
   uint8_t *sB = (uint8_t *)(sHx + C);               // [C] b_i(h)
   __shared__ unsigned long long sTicket;
-  __shared__ int sSegH[CHAIN_CMAX / CHAIN_SEGMIN];      // true state at the first batch head of each segment
-  __shared__ int64_t sSegF[CHAIN_CMAX / CHAIN_SEGMIN];
   const int tid = threadIdx.x;
   for (;;) {
     if (tid == 0) sTicket = atomicAdd(a.counter, 1ull);
@@ -3518,7 +3524,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   const bool use_scan1 = !simple && env_int("PROTEUS_REPLAY_SCAN1", 1) != 0;
   const bool use_chain = !simple && env_int("PROTEUS_REPLAY_CHAIN", 1) != 0 && max_rounds == 0 &&
                          env_int("PROTEUS_REPLAY_TABLES", 0) == 0;
-  int CHN = env_int("PROTEUS_REPLAY_CHAIN_C", 1024);
+  int CHN = env_int("PROTEUS_REPLAY_CHAIN_C", 1536);
   CHN = CHN < 256 ? 256 : CHN > CHAIN_CMAX ? CHAIN_CMAX : CHN;  // shared-memory tables (~24 B per head)
   const int chain_minb = std::max(2, env_int("PROTEUS_REPLAY_CHAIN_MINB", 2));
   std::vector<int32_t> clid[2], cnch[2];
@@ -3792,7 +3798,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       ca.units = d_units[rt];
       ca.lp = d_lp; ca.option = d_opt; ca.dev_type = d_dev; ca.lat = ctx->d_lat;
       ca.devOff = devOff[rt]; ca.devArr = devArr[rt]; ca.latd = latd;
-      smc = chain_smem(CHN, ctx->bmax);
+      smc = chain_smem(CHN, ctx->bmax, ca.SEG);
       PX_CUDA(ctx, cudaFuncSetAttribute(k_chain, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smc));
       PX_CUDA(ctx, cudaDeviceGetAttribute(&chain_nsm, cudaDevAttrMultiProcessorCount, ctx->device));
       const int orc = px_occupancy(ctx, (const void *)k_chain, CHAIN_THREADS, smc, &chain_occ);

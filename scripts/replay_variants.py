@@ -17,7 +17,7 @@ if len(sys.argv) > 1:
     VARIANTS = []
     for arg in sys.argv[1:]:
         name, rest = arg.split("=", 1)
-        VARIANTS.append((name, [tuple(kv.split("=", 1)) for kv in rest.split(",")]))
+        VARIANTS.append((name, [tuple(kv.split("=", 1)) for kv in rest.split(",")] if rest else []))
 px = Proteus(0)
 out = {}
 for kind in ("poisson", "gamma"):
