@@ -2197,11 +2197,29 @@ __global__ void k_sink(int64_t NS, int S, int D, const int32_t *__restrict__ sc_
 // per segment only the on-time count is accumulated (16-byte loads, one
 // compare per latency), then violations = length - on-time and the accuracy
 // sum = on-time x A.  The sink segment is all violations (nothing to read).
+// the counts of the lanes k_chain wrote (and of their duplicates): ccov[s * D
+// + d] = the chain lane index holding lane (s, d)'s latencies, -1 otherwise
+__global__ void k_chain_agg(int S, int D, int nsc, const int32_t *__restrict__ sc_list, const int32_t *__restrict__ ccov,
+                            const unsigned long long *__restrict__ lcnt, const int64_t *__restrict__ devOff,
+                            const LaneParam *__restrict__ lp, uint64_t *agg) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= nsc * D) return;
+  const int s = sc_list[i / D], d = i % D;
+  const int li = ccov[(size_t)s * D + d];
+  if (li < 0) return;
+  const unsigned long long on = lcnt[li], n = (unsigned long long)(devOff[d + 1] - devOff[d]);
+  if (n > on) atomicAdd((unsigned long long *)&agg[s], n - on);
+  if (on) {
+    atomicAdd((unsigned long long *)&agg[S + s], on);
+    atomicAdd((unsigned long long *)&agg[2 * S + s], on * lp[(size_t)s * D + d].A);
+  }
+}
+
 #define CNT_PER 16384
 __global__ void __launch_bounds__(256) k_count(int64_t N, int64_t NS, int S, int D, const int32_t *__restrict__ sc_list,
                                                const int64_t *__restrict__ devOff, const LaneParam *__restrict__ lp,
                                                const int32_t *__restrict__ rep, const uint32_t *__restrict__ latd,
-                                               uint64_t *agg) {
+                                               uint64_t *agg, const int32_t *__restrict__ ccov) {
   __shared__ unsigned long long red[3][8];
   const int s = sc_list[blockIdx.y];
   const int64_t lo = (int64_t)blockIdx.x * CNT_PER, hi = lo + CNT_PER < N ? lo + CNT_PER : N;
@@ -2213,6 +2231,7 @@ __global__ void __launch_bounds__(256) k_count(int64_t N, int64_t NS, int S, int
       if (threadIdx.x == 0) viol += (unsigned long long)(a1 - a0);
       continue;
     }
+    if (ccov && ccov[(size_t)s * D + d] >= 0) continue;  // counted by k_chain (k_chain_agg)
     const LaneParam q = lp[(size_t)s * D + d];
     const uint32_t *row = latd + (size_t)(rep ? rep[(size_t)s * (D + 1) + d] : s) * NS;  // a duplicate lane: its row's
     const uint32_t L = q.L < 0 ? 0u : q.L > 0xFFFFFFFEll ? 0xFFFFFFFFu : (uint32_t)q.L;
@@ -2901,6 +2920,7 @@ struct ChainArgs {
   unsigned long long *counter; // ticket counter
   unsigned *watchdog;          // set when a wait for a previous chunk's exit times out
   unsigned long long *dbg;     // PX_CHAIN_DEBUG: [16] phase cycles, units, batches, hops
+  unsigned long long *lcnt;    // [nl] on-time latencies per lane (the counts folded into the writers), or null
 };
 
 struct ShArr {  // arrivals of a chunk in shared memory, from its first head
@@ -2989,9 +3009,14 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
         }
       };
       // latencies of the batch [hh, hh + b) finishing at fin, positions < lim
+      unsigned long long ont = 0;  // on-time latencies this thread wrote (R6: latency <= SLO)
       auto put = [&](int hh, int b, int64_t fin, int lim) {
         const int e = hh + b < lim ? hh + b : lim;
-        for (int j = hh + lane; j < e; j += 32) out[j] = sat_lat(fin - (int64_t)sA[j]);
+        for (int j = hh + lane; j < e; j += 32) {
+          const uint32_t l = sat_lat(fin - (int64_t)sA[j]);
+          out[j] = l;
+          ont += (int64_t)l <= p.L;
+        }
       };
       // the chunk's entry (warp 0): R13 for the first chunk, else the previous
       // chunk's exit, a single 64-bit word ((F + 1) << 8 | head - chunk start)
@@ -3036,7 +3061,11 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
             const int k = stretch(hh, FF, Cn);
             if (k > 0) {
               const int np = k * Bm;
-              for (int j = lane; j < np; j += 32) out[hh + j] = sat_lat(FF + (int64_t)(j / Bm + 1) * TB - (int64_t)sA[hh + j]);
+              for (int j = lane; j < np; j += 32) {
+                const uint32_t l = sat_lat(FF + (int64_t)(j / Bm + 1) * TB - (int64_t)sA[hh + j]);
+                out[hh + j] = l;
+                ont += (int64_t)l <= p.L;
+              }
               nbat += k;
               hh += np;
               FF += (int64_t)k * TB;
@@ -3249,7 +3278,11 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
           int64_t fin;
           if (FF <= ti) { b = sB[hh]; fin = ti + sT[b - 1]; }
           else { b = greedy(hh, FF); fin = FF + sT[b - 1]; }
-          for (int j = 0; j < b; j++) out[hh + j] = sat_lat(fin - (int64_t)sA[hh + j]);
+          for (int j = 0; j < b; j++) {
+            const uint32_t l = sat_lat(fin - (int64_t)sA[hh + j]);
+            out[hh + j] = l;
+            ont += (int64_t)l <= p.L;
+          }
           nbat++;
           hh += b;
           FF = fin;
@@ -3262,6 +3295,10 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       (void)nbat;
 #endif
       }  // tables
+      if (a.lcnt) {  // the lane's on-time count (violations = positions - on time, R6; accuracy = on time x A, R9)
+        for (int o = 16; o; o >>= 1) ont += __shfl_xor_sync(0xffffffffu, ont, o);
+        if ((tid & 31) == 0 && ont) atomicAdd(a.lcnt + li, ont);
+      }
     }
     __syncthreads();  // shared tables and sTicket are rewritten by the next unit
   }
@@ -3729,6 +3766,8 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   }
   for (int rt = 0; rt < 2; rt++) {
     if (scl[rt].empty()) continue;
+    int32_t *d_ccov = nullptr;             // chain lanes whose counts k_chain folded (k_chain_agg)
+    unsigned long long *d_lcnt = nullptr;
     LaneArgs la;
     memset(&la, 0, sizeof la);
     la.S = S; la.D = D; la.M = M; la.bmax = ctx->bmax; la.nsc = (int)scl[2 + rt].size(); la.CH = CH;
@@ -3783,6 +3822,28 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     ChainArgs ca;
     memset(&ca, 0, sizeof ca);
     const bool chain_now = use_chain && !clid[rt].empty();
+    // the chain lanes' counts are folded into its writers (k_chain_agg adds
+    // them, k_count skips those lanes) when the counts come from the rows
+    const bool fold_counts = (!d_lat_out || env_int("PROTEUS_REPLAY_FINISH", 0) == 0) &&
+                             env_int("PROTEUS_REPLAY_CHAIN_COUNTS", 1) != 0;
+    if (chain_now && fold_counts) {
+      const int nl = (int)clid[rt].size();
+      char *cc = (char *)px_buf(ctx, B_R_CCNT, (size_t)S * D * 4 + (size_t)nl * 8 + 64);
+      if (!cc) return px_fail(ctx, PROTEUS_ENOMEM, "chain counts");
+      std::vector<int32_t> cov((size_t)S * D, -1);
+      for (int l = 0; l < nl; l++) cov[clid[rt][l]] = l;
+      for (int k : scl[2 + rt])  // duplicates read their representative's row
+        for (int d = 0; d < D; d++) {
+          const int r = hrep[(size_t)k * (D + 1) + d];
+          if (r != k && cov[(size_t)r * D + d] >= 0) cov[(size_t)k * D + d] = cov[(size_t)r * D + d];
+        }
+      ca.lcnt = (unsigned long long *)(cc + (((size_t)S * D * 4 + 15) & ~(size_t)15));
+      d_ccov = (int32_t *)cc;
+      d_lcnt = ca.lcnt;
+      PX_CUDA(ctx, cudaMemcpyAsync(d_ccov, cov.data(), cov.size() * 4, cudaMemcpyHostToDevice, ctx->stream));
+      PX_CUDA(ctx, cudaMemsetAsync(ca.lcnt, 0, (size_t)nl * 8, ctx->stream));
+      PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // cov is a host vector
+    }
     size_t smc = 0;
     int chain_nsm = 0, chain_occ = 0;
     if (chain_now) {
@@ -4153,8 +4214,13 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       dim3 g(32, nall < 65535 ? nall : 65535);
       PX_LAUNCH(ctx, "replay_sink", k_sink, g, 256, 0, NS, S, D, d_scl + rt * S, nall, devOff[rt], latd, d_agg);
       dim3 cg((unsigned)((N + CNT_PER - 1) / CNT_PER), (unsigned)nall);
+      if (d_ccov) {
+        const int n5 = (int)scl[2 + rt].size();
+        PX_LAUNCH(ctx, "replay_count", k_chain_agg, (n5 * D + 255) / 256, 256, 0, S, D, n5, d_scl + (2 + rt) * S, d_ccov,
+                  d_lcnt, devOff[rt], d_lp, d_agg);
+      }
       PX_LAUNCH(ctx, "replay_count", k_count, cg, 256, 0, N, NS, S, D, d_scl + rt * S, devOff[rt], d_lp, d_rep, latd,
-                d_agg);
+                d_agg, d_ccov);
     }
     if (d_lat_out && d_rep && npair[rt] > 0) {  // the duplicate lanes' rows, for the un-permute
       int64_t maxn = 1;
