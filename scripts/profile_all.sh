@@ -11,7 +11,7 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_fl
     -o gpurun_out/full_flat -f python scripts/profile_target.py c2 > /dev/null 2>&1; echo "full flat rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_fact_gv|k_fact_dp" -c 2 \
     -o gpurun_out/full_fact -f python scripts/profile_target.py c4 > /dev/null 2>&1; echo "full fact rc=$?"
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_spec|k_stitch|k_unpermute|k_count" -c 4 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_chain|k_unpermute|k_count" -c 3 \
     -o gpurun_out/full_replay -f python scripts/profile_target.py c5 > /dev/null 2>&1; echo "full replay rc=$?"
 timeout 1200 ncu --set full --clock-control none --import-source on -k regex:"k_wc_lanes" -c 1 \
     -o gpurun_out/full_wc -f python scripts/profile_target.py f2 > /dev/null 2>&1; echo "full wc rc=$?"
