@@ -3148,24 +3148,32 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       }
       __syncthreads();
       CX_T(2);
-      // the last idle-branch head of every head's run inside its segment (sJ)
-      // and inside the chunk (sJc): pointer jumping, in place (a pointer only
-      // ever moves further along its own run)
+      // the last idle-branch head of every head's run inside its segment
+      // (sJ): pointer jumping, in place (a pointer only ever moves further
+      // along its own run) ...
       for (int i = tid; i < Cn; i += CHAIN_THREADS) {
-        const int nx = sNx[i], nc = sNc[i];
+        const int nx = sNx[i];
         sJ[i] = nx >= 0 ? (int16_t)nx : (int16_t)i;
-        sJc[i] = nc >= 0 ? (int16_t)nc : (int16_t)i;
       }
       for (bool more = true; more;) {
         __syncthreads();
         bool ch = false;
         for (int i = tid; i < Cn; i += CHAIN_THREADS) {
           const int j = sJ[i], jj = sJ[j];
-          const int k = sJc[i], kk = sJc[k];
           if (jj != j) { sJ[i] = (int16_t)jj; ch = true; }
-          if (kk != k) { sJc[i] = (int16_t)kk; ch = true; }
         }
         more = __syncthreads_or(ch);
+      }
+      // ... and inside the chunk (sJc): a run whose last node r in its segment
+      // reaches an idle-branch head further on (sNc[r], a later segment)
+      // continues with that head's; segments from the last
+      for (int sg = nseg - 1; sg >= 0; sg--) {
+        const int s1 = (sg + 1) * SEG < Cn ? (sg + 1) * SEG : Cn;
+        for (int i = sg * SEG + tid; i < s1; i += CHAIN_THREADS) {
+          const int r = sJ[i], nc = sNc[r];
+          sJc[i] = nc >= 0 ? sJc[nc] : (int16_t)r;
+        }
+        __syncthreads();
       }
       CX_T(3);
       if (w == 0) {
