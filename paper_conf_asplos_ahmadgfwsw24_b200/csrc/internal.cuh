@@ -117,14 +117,14 @@ struct proteus_ctx {
   cudaStream_t aux = nullptr, aux_hi = nullptr;  // lowest / highest stream priority
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_join2 = nullptr;
   // replay chain path: the ticket order last uploaded per routing mode (its key: lanes, chunks per lane)
-  std::vector<int64_t> chain_ukey[2];
+  std::vector<int64_t> chain_ukey[3];  // [2]: the closed loop's
 };
 
 // scratch buffer ids
 enum {
   B_TABLES = 0, B_BEST, B_SOL, B_IN0, B_IN1, B_IN2, B_IN3, B_FACT0, B_FACT1, B_FACT2, B_FACT3,
   B_R_PAT, B_R_TGT, B_R_HIST, B_R_BASE, B_R_DEVARR, B_R_DEVIDX, B_R_OFF, B_R_LAT, B_R_AGG, B_R_TGT1,
-  B_R_DEVARR1, B_R_DEVIDX1, B_R_OFF1, B_R_MISC, B_R_LANE, B_R_DBASE0, B_R_DBASE1, B_R_LATD, B_R_VLAT, B_R_VEX, B_R_VOFF, B_FACT4, B_R_SCAN, B_R_BSCAN, B_PARETO, B_E_MISC, B_E_PAT, B_E_EXIT, B_R_WST, B_R_WEX, B_C_KEEP, B_C_GATHER, B_C_PTS, B_W_REC, B_W_ENT, B_W_AUX, B_R_READY, B_R_CHAIN, B_R_UNITS0, B_R_UNITS1, B_R_NX, B_R_CCNT, B_NBUF
+  B_R_DEVARR1, B_R_DEVIDX1, B_R_OFF1, B_R_MISC, B_R_LANE, B_R_DBASE0, B_R_DBASE1, B_R_LATD, B_R_VLAT, B_R_VEX, B_R_VOFF, B_FACT4, B_R_SCAN, B_R_BSCAN, B_PARETO, B_E_MISC, B_E_PAT, B_E_EXIT, B_R_WST, B_R_WEX, B_C_KEEP, B_C_GATHER, B_C_PTS, B_W_REC, B_W_ENT, B_W_AUX, B_R_READY, B_R_CHAIN, B_R_UNITS0, B_R_UNITS1, B_R_NX, B_R_CCNT, B_E_CHAIN, B_E_UNITS, B_NBUF
 };
 static_assert(B_NBUF <= 56, "proteus_ctx::bufs is too small");
 

@@ -2921,6 +2921,11 @@ struct ChainArgs {
   unsigned *watchdog;          // set when a wait for a previous chunk's exit times out
   unsigned long long *dbg;     // PX_CHAIN_DEBUG: [16] phase cycles, units, batches, hops
   unsigned long long *lcnt;    // [nl] on-time latencies per lane (the counts folded into the writers), or null
+  // EP (k_chain<true>, the closed loop): epochs of epoch_us, per (scenario, epoch, device) {Bmax, L, T row offset}
+  int E;
+  int64_t epoch_us;
+  const int32_t *epP;             // [S][E][D][3]
+  const int32_t *segBase, *cntED; // [E][D] segment of (epoch, device) in the device's array
 };
 
 struct ShArr {  // arrivals of a chunk in shared memory, from its first head
@@ -2931,14 +2936,15 @@ struct ShArr {  // arrivals of a chunk in shared memory, from its first head
 // per routing mode: lid [nl] i32, nch [nl] i32, cmode [nl] u8, ticket + watchdog, exits [nl][maxch] u64
 static size_t chain_ctroff(size_t nl) { return (nl * 9 + 15) & ~(size_t)15; }
 static size_t chain_exoff(size_t nl) { return chain_ctroff(nl) + 16; }
-static size_t chain_smem(int C, int bmax, int SEG) {
+static size_t chain_smem(int C, int bmax, int SEG, bool ep = false) {
   const size_t E = (size_t)C + bmax + 2;
   const size_t nseg = ((size_t)C + SEG - 1) / SEG;
   return (size_t)C * 8 /* sFx */ + nseg * 8 /* sSegF */ + (size_t)bmax * 4 /* sT */ + E * 4 /* sA */ +
          (size_t)C * 4 /* sTi */ + nseg * 4 /* sSegH */ + (size_t)C * 10 /* sNx, sNc, sJ, sJc, sHx */ +
-         (size_t)C /* sB */ + 64;
+         (size_t)C /* sB */ + 64 + (ep ? (size_t)C * 4 + 16 : 0) /* sEp, sEnd */;
 }
 
+template <bool EP>  // EP: the closed loop's lanes (§8(f4)): rule parameters and queue ends per epoch segment
 __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __grid_constant__ ChainArgs a) {
   extern __shared__ __align__(16) unsigned char csm[];
   const int C = a.C, SEG = a.SEG;
@@ -2956,6 +2962,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
   int16_t *sJc = sJ + C;                            // [C] last idle-branch head of h's run in the chunk
   int16_t *sHx = sJc + C;                           // [C] first head past the segment of a leaving run
   uint8_t *sB = (uint8_t *)(sHx + C);               // [C] b_i(h)
+  uint16_t *sEp = (uint16_t *)(sB + ((C + 15) & ~15));  // EP: [C] epoch of head h
+  int16_t *sEnd = (int16_t *)(sEp + C);             // EP: [C] end of h's epoch segment (chunk-relative, capped)
   __shared__ unsigned long long sTicket;
   const int tid = threadIdx.x;
   for (;;) {
@@ -2972,24 +2980,43 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
 #endif
       const int lane_id = a.lid[li];
       const int s = lane_id / a.D, d = lane_id % a.D;
-      const LaneParam p = a.lp[lane_id];
+      LaneParam p = {0, 0, 0, 0, 0, 0};
+      if (!EP) p = a.lp[lane_id];
       const int Bm = p.Bmax;
       const int64_t off = a.devOff[d], nloc0 = a.devOff[d + 1] - off;
       const int64_t c0 = c * C;
       const int64_t nloc = nloc0 - c0;  // heads from the chunk start to the device's end
       const int Cn = (int)(nloc < C ? nloc : C);
-      const int na = (int)(nloc < (int64_t)Cn + Bm + 1 ? nloc : (int64_t)Cn + Bm + 1);
+      const int Bst = EP ? a.bmax : Bm;  // look-ahead of a decision
+      const int na = (int)(nloc < (int64_t)Cn + Bst + 1 ? nloc : (int64_t)Cn + Bst + 1);
       const int nseg = (Cn + SEG - 1) / SEG;
-      const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
-      for (int k = tid; k < Bm; k += CHAIN_THREADS) sT[k] = Tg[k];
+      if (!EP) {
+        const int32_t *Tg = a.lat + ((size_t)a.dev_type[d] * a.M + (a.option[d] - 1)) * a.bmax;
+        for (int k = tid; k < Bm; k += CHAIN_THREADS) sT[k] = Tg[k];
+      }
       const uint32_t *src = a.devArr + off + c0;
       for (int j = tid; j < na; j += CHAIN_THREADS) sA[j] = src[j];
       for (int sg = tid; sg < nseg; sg += CHAIN_THREADS) sSegH[sg] = -1;  // not recorded yet
+      if (EP) {  // F1: query j belongs to epoch a_j / epoch_us; its segment ends where the epoch's queries end
+        __syncthreads();
+        for (int i = tid; i < Cn; i += CHAIN_THREADS) {
+          const int e = (int)((int64_t)sA[i] / a.epoch_us);
+          sEp[i] = (uint16_t)e;
+          const int64_t end = (int64_t)a.segBase[(size_t)e * a.D + d] + a.cntED[(size_t)e * a.D + d] - c0;
+          sEnd[i] = (int16_t)(end < (int64_t)Cn + Bst + 1 ? end : (int64_t)Cn + Bst + 1);
+        }
+      }
       __syncthreads();
       CX_T(0);
       const ShArr A{sA};
       const int w = tid >> 5, lane = tid & 31;
-      const int64_t TB = sT[Bm - 1];
+      const int64_t TB = EP ? 0 : sT[Bm - 1];
+      // the rule's parameters for a decision at head h: Bmax, SLO, T(b) row, queue end
+      auto epp = [&](int h) -> const int32_t * { return a.epP + ((size_t)(s * a.E + sEp[h]) * a.D + d) * 3; };
+      auto HB = [&](int h) -> int { if constexpr (EP) return epp(h)[0]; else return Bm; };
+      auto HL = [&](int h) -> int64_t { if constexpr (EP) return epp(h)[1]; else return p.L; };
+      auto HT = [&](int h) -> const int32_t * { if constexpr (EP) return a.lat + epp(h)[2]; else return sT; };
+      auto HN = [&](int h) -> int64_t { if constexpr (EP) return sEnd[h]; else return nloc; };
       uint32_t *out = a.latd + (size_t)s * a.NS + off + c0;
       // full-batch stretch at (hh, FF): batch i (head hh + i Bm) leaves full at
       // FF + i T(Bmax) while its last query has arrived by then -- with Bmax
@@ -2997,12 +3024,15 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       // whether or not the idle run would have dispatched earlier.  Returns
       // the number of such batches whose heads lie below lim (32 per ballot).
       auto stretch = [&](int hh, int64_t FF, int lim) -> int {
+        const int B_ = HB(hh);
+        const int64_t TB_ = HT(hh)[B_ - 1], N_ = HN(hh);
+        if (N_ < lim) lim = (int)N_;  // EP: a batch holds one epoch's queries (F3)
         int k = 0;
         for (;;) {
           const int i = k + lane;
-          const int64_t last = (int64_t)hh + (int64_t)(i + 1) * Bm - 1;
-          const bool full = (int64_t)hh + (int64_t)i * Bm < lim && last < nloc &&
-                            (int64_t)sA[last] <= FF + (int64_t)i * TB;
+          const int64_t last = (int64_t)hh + (int64_t)(i + 1) * B_ - 1;
+          const bool full = (int64_t)hh + (int64_t)i * B_ < lim && last < N_ &&
+                            (int64_t)sA[last] <= FF + (int64_t)i * TB_;
           const unsigned bal = __ballot_sync(0xffffffffu, !full);
           if (bal) return k + __ffs(bal) - 1;
           k += 32;
@@ -3046,7 +3076,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
           asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(a.ex + (size_t)li * a.maxch + c), "l"(v) : "memory");
         }
       };
-      if (a.cmode[li]) {
+      if (!EP && a.cmode[li]) {
         // a lane near overload: mostly full batches back to back, taken 32 per
         // ballot; the other decisions directly (idle decision by binary
         // search, else the greedy batch).  No tables: warp 0 walks the chunk
@@ -3096,7 +3126,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       // idle decisions of every head (fact (ii): binary search)
       for (int i = tid; i < Cn; i += CHAIN_THREADS) {
         int64_t t;
-        const int b = idle_decide(A, nloc, (int64_t)i, Bm, p.L, sT, true, &t);
+        const int b = idle_decide(A, HN(i), (int64_t)i, HB(i), HL(i), HT(i), true, &t);
         sB[i] = (uint8_t)b;
         sTi[i] = (int32_t)(t - (int64_t)sA[i]);
       }
@@ -3106,8 +3136,9 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       // would have dispatched: min(Bmax, queued at F), Bmax without a search
       // when the Bmax-th query is already there
       auto greedy = [&](int hh, int64_t F) -> int {
-        return ((int64_t)hh + Bm - 1 < nloc && (int64_t)sA[hh + Bm - 1] <= F) ? Bm
-                                                                               : count_upto(A, nloc, (int64_t)hh, Bm, F);
+        const int B_ = HB(hh);
+        const int64_t N_ = HN(hh);
+        return ((int64_t)hh + B_ - 1 < N_ && (int64_t)sA[hh + B_ - 1] <= F) ? B_ : count_upto(A, N_, (int64_t)hh, B_, F);
       };
       // the run of every head after its idle-branch decision (at most K
       // greedy batches are followed here -- backlogged stretches would make
@@ -3119,7 +3150,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       for (int i = tid; i < Cn; i += CHAIN_THREADS) {
         const int se = (i / SEG + 1) * SEG < Cn ? (i / SEG + 1) * SEG : Cn;
         const int bi = sB[i];
-        int64_t F = (int64_t)sA[i] + sTi[i] + sT[bi - 1];
+        int64_t F = (int64_t)sA[i] + sTi[i] + HT(i)[bi - 1];
         int hh = i + bi;
         bool segdone = false;
         for (int st = 0;; st++) {
@@ -3142,7 +3173,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
             break;
           }
           const int g = greedy(hh, F);  // dispatched at F
-          F += sT[g - 1];
+          F += HT(hh)[g - 1];
           hh += g;
         }
       }
@@ -3202,20 +3233,25 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
             // batches (to the chunk's end when it leaves the chunk)
             const int r = sJc[hh];
             const int br = sB[r];
-            FF = (int64_t)sA[r] + sTi[r] + sT[br - 1];
+            FF = (int64_t)sA[r] + sTi[r] + HT(r)[br - 1];
             hh = r + br;
             if (sNc[r] == -1)
               while (hh < Cn) {
                 const int g = greedy(hh, FF);
-                FF += sT[g - 1];
+                FF += HT(hh)[g - 1];
                 hh += g;
               }
             continue;
           }
           const int k = stretch(hh, FF, Cn);
-          if (k > 0) { hh += k * Bm; FF += (int64_t)k * TB; continue; }
-          const int g = count_upto(A, nloc, (int64_t)hh, Bm, FF);
-          FF += sT[g - 1];
+          if (k > 0) {
+            const int B_ = HB(hh);
+            FF += (int64_t)k * HT(hh)[B_ - 1];
+            hh += k * B_;
+            continue;
+          }
+          const int g = count_upto(A, HN(hh), (int64_t)hh, HB(hh), FF);
+          FF += HT(hh)[g - 1];
           hh += g;
         }
         publish(hh - Cn, FF);
@@ -3243,7 +3279,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
           if (FF <= (int64_t)sA[hh] + sTi[hh]) {
             const int r = sJ[hh];
             const int nx = sNx[r];
-            if (nx == -2) { const int br = sB[r]; FF = (int64_t)sA[r] + sTi[r] + sT[br - 1]; hh = r + br; rec(hh, FF); continue; }
+            if (nx == -2) { const int br = sB[r]; FF = (int64_t)sA[r] + sTi[r] + HT(r)[br - 1]; hh = r + br; rec(hh, FF); continue; }
             FF = sFx[r];
             hh = sHx[r];
             rec(hh, FF);
@@ -3256,9 +3292,15 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
           }
           const int se = (hh / SEG + 1) * SEG < Cn ? (hh / SEG + 1) * SEG : Cn;
           const int k = stretch(hh, FF, se);
-          if (k > 0) { hh += k * Bm; FF += (int64_t)k * TB; rec(hh, FF); continue; }
-          const int g = count_upto(A, nloc, (int64_t)hh, Bm, FF);
-          FF += sT[g - 1];
+          if (k > 0) {
+            const int B_ = HB(hh);
+            FF += (int64_t)k * HT(hh)[B_ - 1];
+            hh += k * B_;
+            rec(hh, FF);
+            continue;
+          }
+          const int g = count_upto(A, HN(hh), (int64_t)hh, HB(hh), FF);
+          FF += HT(hh)[g - 1];
           hh += g;
           rec(hh, FF);
         }
@@ -3284,8 +3326,8 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
           const int64_t ti = (int64_t)sA[hh] + sTi[hh];
           int b;
           int64_t fin;
-          if (FF <= ti) { b = sB[hh]; fin = ti + sT[b - 1]; }
-          else { b = greedy(hh, FF); fin = FF + sT[b - 1]; }
+          if (FF <= ti) { b = sB[hh]; fin = ti + HT(hh)[b - 1]; }
+          else { b = greedy(hh, FF); fin = FF + HT(hh)[b - 1]; }
           for (int j = 0; j < b; j++) {
             const uint32_t l = sat_lat(fin - (int64_t)sA[hh + j]);
             out[hh + j] = l;
@@ -3868,9 +3910,9 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
       ca.lp = d_lp; ca.option = d_opt; ca.dev_type = d_dev; ca.lat = ctx->d_lat;
       ca.devOff = devOff[rt]; ca.devArr = devArr[rt]; ca.latd = latd;
       smc = chain_smem(CHN, ctx->bmax, ca.SEG);
-      PX_CUDA(ctx, cudaFuncSetAttribute(k_chain, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smc));
+      PX_CUDA(ctx, cudaFuncSetAttribute(k_chain<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smc));
       PX_CUDA(ctx, cudaDeviceGetAttribute(&chain_nsm, cudaDevAttrMultiProcessorCount, ctx->device));
-      const int orc = px_occupancy(ctx, (const void *)k_chain, CHAIN_THREADS, smc, &chain_occ);
+      const int orc = px_occupancy(ctx, (const void *)k_chain<false>, CHAIN_THREADS, smc, &chain_occ);
       if (orc) return orc;
       chain_occ = chain_occ > 0 ? chain_occ : 1;
 #ifdef PX_CHAIN_DEBUG
@@ -3880,7 +3922,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
     }
     auto launch_chain = [&](int occ_cap) -> int {
       const int64_t nb = std::min<int64_t>(ca.nunits, (int64_t)chain_nsm * std::min(chain_occ, occ_cap));
-      PX_LAUNCH(ctx, "replay_chain", k_chain, (unsigned)nb, CHAIN_THREADS, smc, ca);
+      PX_LAUNCH(ctx, "replay_chain", k_chain<false>, (unsigned)nb, CHAIN_THREADS, smc, ca);
       return 0;
     };
     const bool chain_beside = chain_now && !simple && ngroups[rt] > 0 && crest[rt] &&
@@ -4418,6 +4460,28 @@ __device__ __forceinline__ int64_t ep_walk(const EpArgs &a, int s, int e, int d,
   return F;
 }
 
+// the chain path's rule parameters per (scenario, epoch, device) (ep_lane):
+// {Bmax, L, offset of the T(b) row in lat}; flags[0] |= 1 when a segment with
+// queries is outside the chain's domain (Bmax outside [1, 255], T(b) not
+// non-decreasing up to Bmax, L >= 2^30): the caller then takes the stitch
+__global__ void k_ep_chparams(const __grid_constant__ EpArgs a, int32_t *epP, unsigned *flags) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= (int64_t)a.S * a.E * a.D) return;
+  const int d = (int)(i % a.D), e = (int)((i / a.D) % a.E), s = (int)(i / ((int64_t)a.D * a.E));
+  const int o = a.option[(size_t)e * a.D + d];
+  int32_t *q = epP + i * 3;
+  if (o <= 0) { q[0] = 1; q[1] = 0; q[2] = 0; return; }
+  const EpLane p = ep_lane(a, s, e, d);
+  q[0] = p.Bmax;
+  q[1] = (int32_t)(p.L < (1ll << 30) ? p.L : 0);
+  q[2] = (int32_t)(((size_t)a.dev_type[d] * a.M + (o - 1)) * a.bmax);
+  if (a.cntED[(size_t)e * a.D + d] > 0) {
+    bool ok = p.Bmax >= 1 && p.Bmax <= 255 && p.L < (1ll << 30);
+    for (int b = 1; ok && b < p.Bmax; b++) ok = p.T[b] >= p.T[b - 1];
+    if (!ok) atomicOr(flags, 1u);
+  }
+}
+
 // phase A: thread per (scenario, epoch, device) segment, from an idle device
 __global__ void __launch_bounds__(128) k_ep_spec(const __grid_constant__ EpArgs a) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -4672,8 +4736,91 @@ int px_replay_epochs(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_f
   ea.latd = latd; ea.exitF = exitF;
   if (S > 65535) return px_fail(ctx, PROTEUS_EINVAL, "S");
   const int64_t nseg = (int64_t)E * D;
-  PX_LAUNCH(ctx, "loop_spec", k_ep_spec, dim3((unsigned)((nseg + 127) / 128), (unsigned)S), 128, 0, ea);
-  PX_LAUNCH(ctx, "loop_stitch", k_ep_stitch, (unsigned)((S * D + 3) / 4), 128, 0, ea);
+  // the chain path (k_chain<true>): per-chunk tables of the idle-branch
+  // decisions with each head's epoch parameters, a chained scan of chunk
+  // exits; the chunk runs + stitch otherwise
+  bool chained = false;
+  if (env_int("PROTEUS_LOOP_CHAIN", 1) != 0 && E <= 65535 && ctx->bmax <= 255 && N < (1ll << 31)) {
+    const int C = std::max(256, std::min(CHAIN_CMAX, env_int("PROTEUS_REPLAY_CHAIN_C", 1536)));
+    const int SEG = std::min(C, std::max(CHAIN_SEGMIN, env_int("PROTEUS_REPLAY_CHAIN_SEG", 128)));
+    int32_t *epP = (int32_t *)px_buf(ctx, B_E_CHAIN, (size_t)S * E * D * 12 + 64);
+    if (!epP) return px_fail(ctx, PROTEUS_ENOMEM, "closed-loop chain parameters");
+    PX_CUDA(ctx, cudaMemsetAsync(d_flags, 0, 4, ctx->stream));
+    const int64_t np = (int64_t)S * E * D;
+    PX_LAUNCH(ctx, "loop_chain", k_ep_chparams, (unsigned)((np + 255) / 256), 256, 0, ea, epP, d_flags);
+    int64_t h_off[PX_MAXD + 2];
+    uint32_t fl = 0;
+    PX_CUDA(ctx, cudaMemcpyAsync(h_off, off, (D + 2) * 8, cudaMemcpyDeviceToHost, ctx->stream));
+    PX_CUDA(ctx, cudaMemcpyAsync(&fl, d_flags, 4, cudaMemcpyDeviceToHost, ctx->stream));
+    PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+    if (!(fl & 1)) {
+      std::vector<int32_t> lid, nch;
+      int64_t mx = 1;
+      for (int sc = 0; sc < S; sc++)
+        for (int d = 0; d < D; d++) {
+          const int64_t nd = h_off[d + 1] - h_off[d];
+          if (nd <= 0) continue;
+          lid.push_back(sc * D + d);
+          nch.push_back((int32_t)((nd + C - 1) / C));
+          mx = std::max(mx, (int64_t)nch.back());
+        }
+      const size_t nl = lid.size();
+      if (nl > 0) {
+        const size_t part = chain_exoff(nl) + nl * (size_t)mx * 8;
+        char *q = (char *)px_buf(ctx, B_E_UNITS, part + 64);
+        if (!q) return px_fail(ctx, PROTEUS_ENOMEM, "closed-loop chain buffers");
+        std::vector<uint8_t> cm(nl, 0);
+        PX_CUDA(ctx, cudaMemcpyAsync(q, lid.data(), nl * 4, cudaMemcpyHostToDevice, ctx->stream));
+        PX_CUDA(ctx, cudaMemcpyAsync(q + nl * 4, nch.data(), nl * 4, cudaMemcpyHostToDevice, ctx->stream));
+        PX_CUDA(ctx, cudaMemcpyAsync(q + nl * 8, cm.data(), nl, cudaMemcpyHostToDevice, ctx->stream));
+        PX_CUDA(ctx, cudaMemsetAsync(q + chain_ctroff(nl), 0, part - chain_ctroff(nl), ctx->stream));
+        // ticket order (as px_replay's): chunks spread in proportion to the lane's length
+        size_t nu = 0;
+        for (size_t l = 0; l < nl; l++) nu += (size_t)nch[l];
+        std::vector<int64_t> cnt((size_t)mx + 1, 0);
+        for (size_t l = 0; l < nl; l++)
+          for (int64_t c = 0; c < nch[l]; c++) cnt[(size_t)(c * mx / nch[l]) + 1]++;
+        for (int64_t k = 0; k < mx; k++) cnt[(size_t)k + 1] += cnt[(size_t)k];
+        std::vector<unsigned long long> units(nu);
+        for (size_t l = 0; l < nl; l++)
+          for (int64_t c = 0; c < nch[l]; c++)
+            units[(size_t)cnt[(size_t)(c * mx / nch[l])]++] = ((unsigned long long)l << 32) | (unsigned long long)c;
+        unsigned long long *du = (unsigned long long *)px_buf(ctx, B_R_UNITS0, nu * 8 + 16);
+        if (!du) return px_fail(ctx, PROTEUS_ENOMEM, "closed-loop chain tickets");
+        ctx->chain_ukey[0].clear();  // B_R_UNITS0 now holds this order, not px_replay's
+        PX_CUDA(ctx, cudaMemcpyAsync(du, units.data(), nu * 8, cudaMemcpyHostToDevice, ctx->stream));
+        ChainArgs ca;
+        memset(&ca, 0, sizeof ca);
+        ca.D = D; ca.M = M; ca.bmax = ctx->bmax; ca.nl = (int)nl; ca.C = C; ca.SEG = SEG;
+        ca.K = std::max(0, env_int("PROTEUS_REPLAY_CHAIN_K", 16));
+        ca.NS = NS; ca.maxch = mx; ca.nunits = (int64_t)nu; ca.units = du;
+        ca.lid = (const int32_t *)q; ca.nch = ca.lid + nl; ca.cmode = (const uint8_t *)(q + nl * 8);
+        ca.counter = (unsigned long long *)(q + chain_ctroff(nl));
+        ca.watchdog = (unsigned *)(ca.counter + 1);
+        ca.ex = (unsigned long long *)(q + chain_exoff(nl));
+        ca.lat = ctx->d_lat; ca.devOff = off; ca.devArr = darr; ca.latd = latd;
+        ca.E = E; ca.epoch_us = epoch_us; ca.epP = epP; ca.segBase = d_segBase; ca.cntED = d_cntED;
+        const size_t smc = chain_smem(C, ctx->bmax, SEG, true);
+        PX_CUDA(ctx, cudaFuncSetAttribute(k_chain<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smc));
+        int nsm = 0, occ = 0;
+        PX_CUDA(ctx, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, ctx->device));
+        const int orc = px_occupancy(ctx, (const void *)k_chain<true>, CHAIN_THREADS, smc, &occ);
+        if (orc) return orc;
+        const int64_t nb = std::min<int64_t>((int64_t)nu, (int64_t)nsm * std::max(occ, 1));
+        PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));  // host vectors are staged
+        PX_LAUNCH(ctx, "loop_chain", k_chain<true>, (unsigned)nb, CHAIN_THREADS, smc, ca);
+        unsigned wd = 0;
+        PX_CUDA(ctx, cudaMemcpyAsync(&wd, ca.watchdog, 4, cudaMemcpyDeviceToHost, ctx->stream));
+        PX_CUDA(ctx, cudaStreamSynchronize(ctx->stream));
+        if (wd) return px_fail(ctx, PROTEUS_EINTERNAL, "closed loop: chain wait for a previous chunk timed out");
+      }
+      chained = true;
+    }
+  }
+  if (!chained) {
+    PX_LAUNCH(ctx, "loop_spec", k_ep_spec, dim3((unsigned)((nseg + 127) / 128), (unsigned)S), 128, 0, ea);
+    PX_LAUNCH(ctx, "loop_stitch", k_ep_stitch, (unsigned)((S * D + 3) / 4), 128, 0, ea);
+  }
   PX_LAUNCH(ctx, "loop_count", k_ep_count, dim3(296, (unsigned)S), 256, 0, ea, N, epoch_us, d_agg);
   if (d_lat_out) {
     const int64_t nb = (N + 256 * UNP_PER - 1) / (256 * UNP_PER);
