@@ -3612,7 +3612,13 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   const bool use_chain = !simple && env_int("PROTEUS_REPLAY_CHAIN", 1) != 0 && max_rounds == 0 &&
                          env_int("PROTEUS_REPLAY_TABLES", 0) == 0;
   int CHN = env_int("PROTEUS_REPLAY_CHAIN_C", 1536);
-  CHN = CHN < 256 ? 256 : CHN > CHAIN_CMAX ? CHAIN_CMAX : CHN;  // shared-memory tables (~24 B per head)
+  CHN = CHN < 256 ? 256 : CHN > CHAIN_CMAX ? CHAIN_CMAX : CHN;  // shared-memory tables (~28 B per head)
+  {
+    int smax = 0;
+    PX_CUDA(ctx, cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, ctx->device));
+    const int seg0 = std::max(CHAIN_SEGMIN, env_int("PROTEUS_REPLAY_CHAIN_SEG", 128));
+    while (CHN > 256 && chain_smem(CHN, ctx->bmax, std::min(CHN, seg0)) + 1024 > (size_t)smax) CHN -= 256;
+  }
   const int chain_minb = std::max(2, env_int("PROTEUS_REPLAY_CHAIN_MINB", 2));
   std::vector<int32_t> clid[2], cnch[2];
   unsigned long long *d_units[2] = {nullptr, nullptr};  // chain ticket order per routing mode
@@ -4741,8 +4747,13 @@ int px_replay_epochs(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_f
   // exits; the chunk runs + stitch otherwise
   bool chained = false;
   if (env_int("PROTEUS_LOOP_CHAIN", 1) != 0 && E <= 65535 && ctx->bmax <= 255 && N < (1ll << 31)) {
-    const int C = std::max(256, std::min(CHAIN_CMAX, env_int("PROTEUS_REPLAY_CHAIN_C", 1536)));
+    int C = std::max(256, std::min(CHAIN_CMAX, env_int("PROTEUS_REPLAY_CHAIN_C", 1536)));
     const int SEG = std::min(C, std::max(CHAIN_SEGMIN, env_int("PROTEUS_REPLAY_CHAIN_SEG", 128)));
+    {  // the chunk's tables must fit the block's shared memory (the per-head epoch arrays included)
+      int smax = 0;
+      PX_CUDA(ctx, cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, ctx->device));
+      while (C > 256 && chain_smem(C, ctx->bmax, SEG, true) + 1024 > (size_t)smax) C -= 256;
+    }
     int32_t *epP = (int32_t *)px_buf(ctx, B_E_CHAIN, (size_t)S * E * D * 12 + 64);
     if (!epP) return px_fail(ctx, PROTEUS_ENOMEM, "closed-loop chain parameters");
     PX_CUDA(ctx, cudaMemsetAsync(d_flags, 0, 4, ctx->stream));

@@ -55,6 +55,26 @@ def test_closed_loop_parity(px, oracle_mod, lam):
     assert np.all(g["violations"] + g["on_time"] == len(cfg["arrival_us"]))
 
 
+@pytest.mark.parametrize("env", [{"PROTEUS_LOOP_CHAIN": "0"},
+                                 {"PROTEUS_REPLAY_CHAIN_C": "256", "PROTEUS_REPLAY_CHAIN_SEG": "16"},
+                                 {"PROTEUS_REPLAY_CHAIN_C": "300", "PROTEUS_REPLAY_CHAIN_K": "0"},
+                                 {"PROTEUS_REPLAY_CHAIN_C": "8192", "PROTEUS_REPLAY_CHAIN_K": "64"}],
+                         ids=["stitch", "chain_c256_seg16", "chain_c300_k0", "chain_c8192_k64"])
+def test_closed_loop_paths(px, oracle_mod, env, monkeypatch):
+    """The closed loop's two replay paths: the chain path (default; small
+    chunks and segments put many epoch boundaries inside chunks, segments
+    and runs) and the chunk runs + stitch (PROTEUS_LOOP_CHAIN=0), light load
+    and overload, against the oracle's closed-loop simulator."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    for lam in (1500.0, 4000.0):
+        cfg = W.config("f4", n_seconds=12, lam_mid=lam)
+        opts, zs = _oracle_allocs(oracle_mod, cfg)
+        g = _compare(px, oracle_mod, cfg, opts, zs, SC)
+        assert np.all(g["violations"] + g["on_time"] == len(cfg["arrival_us"]))
+
+
 def test_closed_loop_short_epochs(px, oracle_mod):
     """100 ms epochs (allocations switching while queues are non-empty) and
     the epoch-boundary carry exercised on every device."""

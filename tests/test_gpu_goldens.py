@@ -66,10 +66,14 @@ def test_c4_all_3600_vectors(px):
             "z_qps": ref["z"]}, ("served", "accsum", "unmet", "option", "z_qps"), "c4")
 
 
-def test_f4_bench_configuration_full_hour(px, oracle_mod):
+@pytest.mark.parametrize("env", [{}, {"PROTEUS_LOOP_CHAIN": "0"}], ids=["chain", "stitch"])
+def test_f4_bench_configuration_full_hour(px, oracle_mod, env, monkeypatch):
     """bench.py's f4 step exactly: solve_batch(mode 2) of the controller's
     demand into device tensors, then replay_epochs of the 10.6M-query hour
-    with the 12 scenarios (SLO {1, 2, 3, 5}x x cap {8, 32, depth})."""
+    with the 12 scenarios (SLO {1, 2, 3, 5}x x cap {8, 32, depth}); the
+    default chain path and the chunk runs + stitch."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
     import torch
     from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
     ref = np.load(os.path.join(GOLDEN, "c4_oracle.npz"))
