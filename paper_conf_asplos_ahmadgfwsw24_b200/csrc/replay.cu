@@ -2939,8 +2939,8 @@ static size_t chain_exoff(size_t nl) { return chain_ctroff(nl) + 16; }
 static size_t chain_smem(int C, int bmax, int SEG, bool ep = false) {
   const size_t E = (size_t)C + bmax + 2;
   const size_t nseg = ((size_t)C + SEG - 1) / SEG;
-  return (size_t)C * 8 /* sFx */ + nseg * 8 /* sSegF */ + (size_t)bmax * 4 /* sT */ + E * 4 /* sA */ +
-         (size_t)C * 4 /* sTi */ + nseg * 4 /* sSegH */ + (size_t)C * 10 /* sNx, sNc, sJ, sJc, sHx */ +
+  return nseg * 8 /* sSegF */ + (size_t)bmax * 4 /* sT */ + E * 4 /* sA */ +
+         (size_t)C * 4 /* sTi */ + nseg * 4 /* sSegH */ + (size_t)C * 8 /* sNx, sNc, sJ, sJc */ +
          (size_t)C /* sB */ + 64 + (ep ? (size_t)C * 4 + 16 : 0) /* sEp, sEnd */;
 }
 
@@ -2949,8 +2949,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
   extern __shared__ __align__(16) unsigned char csm[];
   const int C = a.C, SEG = a.SEG;
   const int NSEG = (C + SEG - 1) / SEG;
-  int64_t *sFx = (int64_t *)csm;                    // [C] free time when a head's run leaves its segment
-  int64_t *sSegF = sFx + C;                         // [NSEG] true free time at the first batch head of a segment
+  int64_t *sSegF = (int64_t *)csm;                  // [NSEG] true free time at the first batch head of a segment
   int32_t *sT = (int32_t *)(sSegF + NSEG);          // [bmax] T(b) at b - 1
   uint32_t *sA = (uint32_t *)(sT + a.bmax);         // [C + bmax + 2] arrivals from the chunk start
   int32_t *sTi = (int32_t *)(sA + C + a.bmax + 2);  // [C] t_i(h) - a_h
@@ -2960,8 +2959,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
   int16_t *sNc = sNx + C;                           // [C] next idle-branch head in the chunk, -1: leaves, -2: left to the walk
   int16_t *sJ = sNc + C;                            // [C] last idle-branch head of h's run in its segment
   int16_t *sJc = sJ + C;                            // [C] last idle-branch head of h's run in the chunk
-  int16_t *sHx = sJc + C;                           // [C] first head past the segment of a leaving run
-  uint8_t *sB = (uint8_t *)(sHx + C);               // [C] b_i(h)
+  uint8_t *sB = (uint8_t *)(sJc + C);               // [C] b_i(h)
   uint16_t *sEp = (uint16_t *)(sB + ((C + 15) & ~15));  // EP: [C] epoch of head h
   int16_t *sEnd = (int16_t *)(sEp + C);             // EP: [C] end of h's epoch segment (chunk-relative, capped)
   __shared__ unsigned long long sTicket;
@@ -3144,7 +3142,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       // greedy batches are followed here -- backlogged stretches would make
       // this quadratic -- the rest is left to the link walk): inside the
       // head's segment (sNx: the next idle-branch head, -1: the run leaves the
-      // segment at (sHx, sFx), -3: ... onto an idle-branch head, -2: left to
+      // segment (its state there is recomputed by the record walk), -3: ... onto an idle-branch head, -2: left to
       // the walk) and inside the chunk (sNc: the next idle-branch head, -1:
       // the run leaves the chunk, -2: left to the walk)
       for (int i = tid; i < Cn; i += CHAIN_THREADS) {
@@ -3157,8 +3155,6 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
           const bool node = hh < Cn && F <= (int64_t)sA[hh] + sTi[hh];
           if (!segdone && hh >= se) {
             sNx[i] = node ? -3 : -1;
-            sHx[i] = (int16_t)hh;
-            sFx[i] = F;
             segdone = true;
           }
           if (hh >= Cn) { sNc[i] = -1; break; }
@@ -3280,8 +3276,17 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
             const int r = sJ[hh];
             const int nx = sNx[r];
             if (nx == -2) { const int br = sB[r]; FF = (int64_t)sA[r] + sTi[r] + HT(r)[br - 1]; hh = r + br; rec(hh, FF); continue; }
-            FF = sFx[r];
-            hh = sHx[r];
+            {  // the run of r to its segment's end (busy after r's batch, at most K greedy batches)
+              const int ser = (r / SEG + 1) * SEG < Cn ? (r / SEG + 1) * SEG : Cn;
+              const int br = sB[r];
+              FF = (int64_t)sA[r] + sTi[r] + HT(r)[br - 1];
+              hh = r + br;
+              while (hh < ser) {
+                const int g = greedy(hh, FF);
+                FF += HT(hh)[g - 1];
+                hh += g;
+              }
+            }
             rec(hh, FF);
             // a run leaving its segment busy: when its next idle-branch head
             // (sNc) lies in the segment it entered, no other segment starts
@@ -3611,7 +3616,7 @@ int px_replay(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_fam, int
   const bool use_scan1 = !simple && env_int("PROTEUS_REPLAY_SCAN1", 1) != 0;
   const bool use_chain = !simple && env_int("PROTEUS_REPLAY_CHAIN", 1) != 0 && max_rounds == 0 &&
                          env_int("PROTEUS_REPLAY_TABLES", 0) == 0;
-  int CHN = env_int("PROTEUS_REPLAY_CHAIN_C", 1536);
+  int CHN = env_int("PROTEUS_REPLAY_CHAIN_C", 2048);
   CHN = CHN < 256 ? 256 : CHN > CHAIN_CMAX ? CHAIN_CMAX : CHN;  // shared-memory tables (~28 B per head)
   {
     int smax = 0;
@@ -4747,7 +4752,7 @@ int px_replay_epochs(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_f
   // exits; the chunk runs + stitch otherwise
   bool chained = false;
   if (env_int("PROTEUS_LOOP_CHAIN", 1) != 0 && E <= 65535 && ctx->bmax <= 255 && N < (1ll << 31)) {
-    int C = std::max(256, std::min(CHAIN_CMAX, env_int("PROTEUS_REPLAY_CHAIN_C", 1536)));
+    int C = std::max(256, std::min(CHAIN_CMAX, env_int("PROTEUS_REPLAY_CHAIN_C", 2048)));
     const int SEG = std::min(C, std::max(CHAIN_SEGMIN, env_int("PROTEUS_REPLAY_CHAIN_SEG", 128)));
     {  // the chunk's tables must fit the block's shared memory (the per-head epoch arrays included)
       int smax = 0;
