@@ -2890,7 +2890,9 @@ __global__ void __launch_bounds__(256) k_finish(int64_t N, int64_t NS, int S, in
 // and publishes the chunk's exit; then one thread per segment writes the
 // segment's latencies from its true state (device-major rows, like the chunk
 // runs).  The serial dependency per lane is one hop per segment.
+#ifndef CHAIN_THREADS
 #define CHAIN_THREADS 256
+#endif
 #define CHAIN_WARPS (CHAIN_THREADS / 32)
 #define CHAIN_CMAX 8192   // largest chunk (heads are int16 in the tables)
 #define CHAIN_SEGMIN 16   // smallest segment
