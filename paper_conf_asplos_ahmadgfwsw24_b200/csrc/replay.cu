@@ -2926,7 +2926,9 @@ struct ChainArgs {
   // EP (k_chain<true>, the closed loop): epochs of epoch_us, per (scenario, epoch, device) {Bmax, L, T row offset}
   int E;
   int64_t epoch_us;
-  const int32_t *epP;             // [S][E][D][3]
+  const int32_t *epP;             // [S][E][D][4] {Bmax, L, T row offset, accuracy of the epoch's variant}
+  uint64_t *agg;                  // EP: [3][S] the counts, folded into the writers (the sink: k_ep_count)
+  int S;
   const int32_t *segBase, *cntED; // [E][D] segment of (epoch, device) in the device's array
 };
 
@@ -3012,7 +3014,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       const int w = tid >> 5, lane = tid & 31;
       const int64_t TB = EP ? 0 : sT[Bm - 1];
       // the rule's parameters for a decision at head h: Bmax, SLO, T(b) row, queue end
-      auto epp = [&](int h) -> const int32_t * { return a.epP + ((size_t)(s * a.E + sEp[h]) * a.D + d) * 3; };
+      auto epp = [&](int h) -> const int32_t * { return a.epP + ((size_t)(s * a.E + sEp[h]) * a.D + d) * 4; };
       auto HB = [&](int h) -> int { if constexpr (EP) return epp(h)[0]; else return Bm; };
       auto HL = [&](int h) -> int64_t { if constexpr (EP) return epp(h)[1]; else return p.L; };
       auto HT = [&](int h) -> const int32_t * { if constexpr (EP) return a.lat + epp(h)[2]; else return sT; };
@@ -3040,6 +3042,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       };
       // latencies of the batch [hh, hh + b) finishing at fin, positions < lim
       unsigned long long ont = 0;  // on-time latencies this thread wrote (R6: latency <= SLO)
+      unsigned long long nwr = 0, accs = 0;  // EP: latencies written, accuracy sum of the on-time ones (R9)
       auto put = [&](int hh, int b, int64_t fin, int lim) {
         const int e = hh + b < lim ? hh + b : lim;
         for (int j = hh + lane; j < e; j += 32) {
@@ -3335,10 +3338,23 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
           int64_t fin;
           if (FF <= ti) { b = sB[hh]; fin = ti + HT(hh)[b - 1]; }
           else { b = greedy(hh, FF); fin = FF + HT(hh)[b - 1]; }
-          for (int j = 0; j < b; j++) {
-            const uint32_t l = sat_lat(fin - (int64_t)sA[hh + j]);
-            out[hh + j] = l;
-            ont += (int64_t)l <= p.L;
+          if constexpr (EP) {  // the batch's epoch gives the SLO and the accuracy (F4)
+            const int64_t Lh = HL(hh);
+            unsigned on = 0;
+            for (int j = 0; j < b; j++) {
+              const uint32_t l = sat_lat(fin - (int64_t)sA[hh + j]);
+              out[hh + j] = l;
+              on += (int64_t)l <= Lh;
+            }
+            ont += on;
+            nwr += (unsigned)b;
+            accs += (unsigned long long)on * (unsigned)epp(hh)[3];
+          } else {
+            for (int j = 0; j < b; j++) {
+              const uint32_t l = sat_lat(fin - (int64_t)sA[hh + j]);
+              out[hh + j] = l;
+              ont += (int64_t)l <= p.L;
+            }
           }
           nbat++;
           hh += b;
@@ -3355,6 +3371,18 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
       if (a.lcnt) {  // the lane's on-time count (violations = positions - on time, R6; accuracy = on time x A, R9)
         for (int o = 16; o; o >>= 1) ont += __shfl_xor_sync(0xffffffffu, ont, o);
         if ((tid & 31) == 0 && ont) atomicAdd(a.lcnt + li, ont);
+      }
+      if (EP && a.agg) {  // the scenario's counts (violations R6, on time, accuracy R9)
+        for (int o = 16; o; o >>= 1) {
+          ont += __shfl_xor_sync(0xffffffffu, ont, o);
+          nwr += __shfl_xor_sync(0xffffffffu, nwr, o);
+          accs += __shfl_xor_sync(0xffffffffu, accs, o);
+        }
+        if ((tid & 31) == 0 && nwr) {
+          if (nwr > ont) atomicAdd((unsigned long long *)&a.agg[s], nwr - ont);
+          if (ont) atomicAdd((unsigned long long *)&a.agg[a.S + s], ont);
+          if (accs) atomicAdd((unsigned long long *)&a.agg[2 * a.S + s], accs);
+        }
       }
     }
     __syncthreads();  // shared tables and sTicket are rewritten by the next unit
@@ -4482,12 +4510,13 @@ __global__ void k_ep_chparams(const __grid_constant__ EpArgs a, int32_t *epP, un
   if (i >= (int64_t)a.S * a.E * a.D) return;
   const int d = (int)(i % a.D), e = (int)((i / a.D) % a.E), s = (int)(i / ((int64_t)a.D * a.E));
   const int o = a.option[(size_t)e * a.D + d];
-  int32_t *q = epP + i * 3;
-  if (o <= 0) { q[0] = 1; q[1] = 0; q[2] = 0; return; }
+  int32_t *q = epP + i * 4;
+  if (o <= 0) { q[0] = 1; q[1] = 0; q[2] = 0; q[3] = 0; return; }
   const EpLane p = ep_lane(a, s, e, d);
   q[0] = p.Bmax;
   q[1] = (int32_t)(p.L < (1ll << 30) ? p.L : 0);
   q[2] = (int32_t)(((size_t)a.dev_type[d] * a.M + (o - 1)) * a.bmax);
+  q[3] = a.acc[o - 1];
   if (a.cntED[(size_t)e * a.D + d] > 0) {
     bool ok = p.Bmax >= 1 && p.Bmax <= 255 && p.L < (1ll << 30);
     for (int b = 1; ok && b < p.Bmax; b++) ok = p.T[b] >= p.T[b - 1];
@@ -4608,7 +4637,7 @@ __global__ void __launch_bounds__(128) k_ep_stitch(const __grid_constant__ EpArg
 // per-scenario counts over the device-major rows (each position's epoch
 // variant gives its SLO and accuracy); the sink segment is written dropped
 __global__ void __launch_bounds__(256) k_ep_count(const __grid_constant__ EpArgs a, int64_t N, int64_t epoch_us,
-                                                  uint64_t *agg) {
+                                                  uint64_t *agg, int sink_only) {
   __shared__ int64_t sOff[PX_MAXD + 2];
   __shared__ unsigned long long red[3][8];
   for (int k = threadIdx.x; k <= a.D + 1; k += blockDim.x) sOff[k] = a.devOff[k];
@@ -4616,7 +4645,8 @@ __global__ void __launch_bounds__(256) k_ep_count(const __grid_constant__ EpArgs
   const int s = blockIdx.y;
   uint32_t *row = a.latd + (size_t)s * a.NS;
   unsigned long long v = 0, o = 0, ac = 0;
-  for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < N; p += (int64_t)gridDim.x * blockDim.x) {
+  const int64_t p0 = sink_only ? sOff[a.D] : 0;
+  for (int64_t p = p0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < N; p += (int64_t)gridDim.x * blockDim.x) {
     int d = 0;
     while (p >= sOff[d + 1]) d++;
     if (d == a.D) { row[p] = 0xFFFFFFFFu; v++; continue; }
@@ -4761,7 +4791,7 @@ int px_replay_epochs(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_f
       PX_CUDA(ctx, cudaDeviceGetAttribute(&smax, cudaDevAttrMaxSharedMemoryPerBlockOptin, ctx->device));
       while (C > 256 && chain_smem(C, ctx->bmax, SEG, true) + 1024 > (size_t)smax) C -= 256;
     }
-    int32_t *epP = (int32_t *)px_buf(ctx, B_E_CHAIN, (size_t)S * E * D * 12 + 64);
+    int32_t *epP = (int32_t *)px_buf(ctx, B_E_CHAIN, (size_t)S * E * D * 16 + 64);
     if (!epP) return px_fail(ctx, PROTEUS_ENOMEM, "closed-loop chain parameters");
     PX_CUDA(ctx, cudaMemsetAsync(d_flags, 0, 4, ctx->stream));
     const int64_t np = (int64_t)S * E * D;
@@ -4818,6 +4848,7 @@ int px_replay_epochs(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_f
         ca.ex = (unsigned long long *)(q + chain_exoff(nl));
         ca.lat = ctx->d_lat; ca.devOff = off; ca.devArr = darr; ca.latd = latd;
         ca.E = E; ca.epoch_us = epoch_us; ca.epP = epP; ca.segBase = d_segBase; ca.cntED = d_cntED;
+        ca.agg = d_agg; ca.S = S;
         const size_t smc = chain_smem(C, ctx->bmax, SEG, true);
         PX_CUDA(ctx, cudaFuncSetAttribute(k_chain<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smc));
         int nsm = 0, occ = 0;
@@ -4839,7 +4870,8 @@ int px_replay_epochs(proteus_ctx *ctx, const uint32_t *d_arr, const uint8_t *d_f
     PX_LAUNCH(ctx, "loop_spec", k_ep_spec, dim3((unsigned)((nseg + 127) / 128), (unsigned)S), 128, 0, ea);
     PX_LAUNCH(ctx, "loop_stitch", k_ep_stitch, (unsigned)((S * D + 3) / 4), 128, 0, ea);
   }
-  PX_LAUNCH(ctx, "loop_count", k_ep_count, dim3(296, (unsigned)S), 256, 0, ea, N, epoch_us, d_agg);
+  // counts: the chain writers folded every device's; k_ep_count takes the rest (the sink)
+  PX_LAUNCH(ctx, "loop_count", k_ep_count, dim3(296, (unsigned)S), 256, 0, ea, N, epoch_us, d_agg, chained ? 1 : 0);
   if (d_lat_out) {
     const int64_t nb = (N + 256 * UNP_PER - 1) / (256 * UNP_PER);
     PX_LAUNCH(ctx, "loop_unpermute", k_unpermute, (unsigned)nb, 256, 0, N, NS, S, d_sc, dinv, dinv, latd, d_lat_out);
