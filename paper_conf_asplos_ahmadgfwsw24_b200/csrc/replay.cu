@@ -3208,12 +3208,13 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
         __syncthreads();
       }
       CX_T(3);
-      if (w == 0) {
-        // the link: the true run through the chunk, one hop per run of
-        // idle-branch decisions (sJc), greedy batches between (full batches
-        // 32 per ballot); the chunk's exit is published at once.  Then the
-        // same run again, one hop per segment (sJ), recording the state at the
-        // first batch head of every segment for the writers.
+      if (w <= 1) {
+        // warp 0, the link: the true run through the chunk, one hop per run
+        // of idle-branch decisions (sJc), greedy batches between (full
+        // batches 32 per ballot); the chunk's exit is published at once.
+        // Warp 1, at the same time: the same run, one hop per segment (sJ),
+        // recording the state at the first batch head of every segment for
+        // the writers.
         int h;
         int64_t F;
 #ifdef PX_CHAIN_DEBUG
@@ -3227,6 +3228,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
         int hh = h;
         int64_t FF = F;
         long long hops = 0;
+        if (w == 0) {
         while (hh < Cn) {
           hops++;
           if (FF <= (int64_t)sA[hh] + sTi[hh]) {
@@ -3263,6 +3265,7 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
         }
 #endif
         CX_T(5);
+        } else {
         int nrec = 0;  // segments [0, nrec) recorded (warp-uniform)
         auto rec = [&](int hq, int64_t Fq) {  // free time first, then the head (the writers' flag)
           const int upto = hq / SEG + 1 < nseg ? hq / SEG + 1 : nseg;
@@ -3315,17 +3318,18 @@ __global__ void __launch_bounds__(CHAIN_THREADS, CHAIN_MINB) k_chain(const __gri
           rec(hh, FF);
         }
         CX_T(7);
+        }  // warp 1
 #ifdef PX_CHAIN_DEBUG
-        if (lane == 0) { atomicAdd(a.dbg + 8, 1ull); atomicAdd(a.dbg + 10, (unsigned long long)hops); }
+        if (lane == 0 && w == 0) { atomicAdd(a.dbg + 8, 1ull); atomicAdd(a.dbg + 10, (unsigned long long)hops); }
 #else
         (void)hops;
 #endif
       }
-      // the writers (warps 1..7, while warp 0 records): thread per segment,
+      // the writers (warps 2..7, while warp 1 records): thread per segment,
       // from the true state at its first batch head, as soon as it is
       // recorded; a batch is written whole by the segment it starts in
       long long nbat = 0;
-      for (int sg = tid - 32; sg < nseg; sg += CHAIN_THREADS - 32) {
+      for (int sg = tid - 64; sg < nseg; sg += CHAIN_THREADS - 64) {
         if (sg < 0) break;
         const int s1 = (sg + 1) * SEG < Cn ? (sg + 1) * SEG : Cn;
         int hh;
