@@ -182,6 +182,27 @@ def test_replay_c5_full_size(px, oracle_mod):
     assert np.array_equal(lat.cpu().numpy(), o["latency"])
 
 
+def test_replay_c5_full_size_routing1(px, oracle_mod):
+    """Config 5 at full size with routing 1 ("w/o QA": uniform
+    weights over the hosting devices that fit, no sink): the 64 §5 scenarios
+    on the default chain path, every latency against the oracle."""
+    import torch
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c5")
+    prof, cl = cfg["prof"], cfg["cluster"]
+    r = oracle_mod.solve(prof, cl.device_type, cl.slo_us, cfg["demand"][0], 2)
+    arr, fam = cfg["arrival_us"], cfg["family"]
+    sc = W.scenarios_64(1)
+    px.load_profiles(prof)
+    lat = torch.empty((len(sc), len(arr)), dtype=torch.uint32, device="cuda")
+    g = px.replay(torch.from_numpy(arr).cuda(), torch.from_numpy(fam).cuda(), r["option"], r["z"], cl.device_type,
+                  cfg["demand"][0], cl.slo_us, sc, latency=lat)
+    o = oracle_mod.replay(prof, cl.device_type, r["option"], r["z"], cfg["demand"][0], cl.slo_us, arr, fam, sc)
+    for k in ("violations", "on_time", "acc_sum"):
+        assert np.array_equal(g[k], o[k]), k
+    assert np.array_equal(lat.cpu().numpy(), o["latency"])
+
+
 @pytest.mark.parametrize("policy", [1, 2])
 def test_replay_baselines_c5_full_size(px, oracle_mod, policy):
     """§8(f2) at the bench's size and launch configuration: the c5 trace (10M
