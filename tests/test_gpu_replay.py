@@ -120,6 +120,53 @@ def test_replay_overload_with_sink(px, oracle_mod, path, monkeypatch):
     assert np.all(g["violations"] + g["on_time"] == len(arr))
 
 
+@pytest.mark.parametrize("epochs", [False, True], ids=["replay", "closed_loop"])
+def test_replay_nonmonotone_latency_mixed_paths(px, oracle_mod, epochs):
+    """A profile whose T(b) decreases at some batch sizes for half of the
+    variants: those lanes leave the chain path (the chain's idle decision is a
+    binary search that needs T non-decreasing) for the chunk runs + stitch
+    (the closed loop: every lane, its domain check fails), the others stay --
+    both paths in one call, against the oracle (whose rule does not assume
+    monotone T)."""
+    import dataclasses
+    from paper_conf_asplos_ahmadgfwsw24_b200 import workloads as W
+    cfg = W.config("c3")
+    prof = cfg["prof"]
+    lat = prof.lat_us.copy()
+    for m in range(0, prof.M, 2):  # every other variant: T(4) and T(9) below their predecessors
+        for t in range(prof.T):
+            for b in (3, 8):
+                if lat[t, m, b] > 0 and lat[t, m, b - 1] > 2:
+                    lat[t, m, b] = lat[t, m, b - 1] - 1
+    prof2 = dataclasses.replace(prof, lat_us=lat)
+    cl = cfg["cluster"]
+    r = oracle_mod.solve(prof2, cl.device_type, cl.slo_us, cfg["demand"][0], 2)
+    px.set_timing(True)
+    if not epochs:
+        arr, fam = W.query_trace(60_000, float(cfg["demand"][0].sum()), cfg["weights"], 21, "gamma")
+        _compare(px, oracle_mod, prof2, cl, r["option"], r["z"], cfg["demand"][0], arr, fam, W.scenarios_64(0))
+        names = {n for n, _ in px.kernel_times()}
+        px.set_timing(False)
+        assert {"replay_chain", "replay_stitch"} <= names, names  # both paths ran
+        return
+    f4 = W.config("f4", n_seconds=6, lam_mid=3000.0)
+    E, D = len(f4["demand"]), len(cl.device_type)
+    opts = np.stack([r["option"]] * E).astype(np.int32)
+    zs = np.stack([r["z"]] * E).astype(np.int32)
+    dem = np.stack([cfg["demand"][0]] * E).astype(np.int32)
+    sc = np.array([(m, c, 0, 0) for m in (1000, 3000) for c in (4, 32, 0)], np.int32)
+    px.load_profiles(prof2)
+    g = px.replay_epochs(f4["arrival_us"], f4["family"], f4["epoch_us"], opts, zs, cl.device_type, dem, cl.slo_us, sc)
+    names = {n for n, _ in px.kernel_times()}
+    px.set_timing(False)
+    assert "loop_stitch" in names and "loop_chain" in names, names  # domain check ran, the stitch replayed
+    o = oracle_mod.replay_epochs(prof2, cl.device_type, opts, zs, dem, cl.slo_us, f4["arrival_us"], f4["family"],
+                                 f4["epoch_us"], sc)
+    for k in ("violations", "on_time", "acc_sum"):
+        assert np.array_equal(g[k], o[k]), k
+    assert np.array_equal(g["latency"], o["latency"])
+
+
 def test_replay_edge_cases(px, oracle_mod):
     from paper_conf_asplos_ahmadgfwsw24_b200 import ProteusError, workloads as W
     cfg = W.config("c3")
